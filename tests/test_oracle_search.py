@@ -1,0 +1,114 @@
+"""Pins of the oracle's reference local-search step (no GPU).
+
+The search is the north star's method, not a paper method, so its pins are the properties
+its spec fixes: the counter-based draw, what each move type may change, the identity
+candidate, the min/commit rule, and that W simulated ranks give the single-rank result.
+"""
+
+import numpy as np
+
+from workloads import dag
+from workloads.rng import mix64
+
+MIX = (50, 20, 20, 10)
+
+
+def _setup(seed=5, n=60, D=2, allowed_frac=0.0, P=3):
+    g = dag.random_dag(seed, n, 1.4, D=D, p_max=2000, max_bytes=50_000, beta0=300,
+                       beta1_fs=20_000, allowed_frac=allowed_frac)
+    orders = np.stack([dag.random_topo_order(g, 10 + b) for b in range(P)]).astype(np.int32)
+    xs = dag.random_placements(g, 3, P)
+    return g, xs, orders
+
+
+def test_draw_matches_spec_text(O):
+    for (seed, step, P, b, j, k) in [(2021, 0, 4, 0, 0, 0), (1, 7, 3, 2, 12345, 15),
+                                     (2 ** 64 - 1, 2 ** 40, 4, 3, 2 ** 24 - 1, 9)]:
+        ctr = ((((step * P + b) * (1 << 24) + j) * 16 + k)) & ((1 << 64) - 1)
+        assert O.draw(seed, step, P, b, j, k) == mix64(seed ^ mix64(ctr))
+
+
+def test_identity_and_move_shapes(O):
+    g, xs, orders = _setup()
+    edges = set(zip(g.src.tolist(), g.dst.tolist()))
+    P, n = xs.shape
+    seen = {"flip": 0, "window": 0, "swap": 0}
+    for b in range(P):
+        ok, x, o = O.candidate(g, P, b, xs, orders, 0, 2021, 3, MIX)
+        assert ok and (x == xs[b]).all() and (o == orders[b]).all()
+        for j in range(1, 2048):
+            ok, x, o = O.candidate(g, P, b, xs, orders, j, 2021, 3, MIX)
+            assert ok
+            diff_pos = np.nonzero(o != orders[b])[0]
+            if len(diff_pos):
+                seen["swap"] += 1
+                k = int(diff_pos[0])
+                assert list(diff_pos) == [k, k + 1]
+                assert o[k] == orders[b][k + 1] and o[k + 1] == orders[b][k]
+                assert (int(orders[b][k]), int(orders[b][k + 1])) not in edges
+                assert O.makespan(g, x, o) >= 0           # still topological
+                if j % 32 == 0:
+                    assert (x == xs[b]).all()              # lane 0 of a swap group: pure swap
+            changed = np.nonzero(x != xs[b])[0]
+            if len(changed) == 0:
+                continue
+            dev = set(x[changed].tolist())
+            pos_changed = sorted(int(np.nonzero(orders[b] == v)[0][0]) for v in changed)
+            if len(changed) <= 4:
+                seen["flip"] += 1
+            if len(dev) == 1 and pos_changed[-1] - pos_changed[0] < 64:
+                seen["window"] += 1
+            assert len(changed) <= 4 or (len(dev) == 1 and pos_changed[-1] - pos_changed[0] < 64)
+    assert seen["flip"] > 0 and seen["window"] > 0 and seen["swap"] > 0
+
+
+def test_moves_respect_allowed(O):
+    g, xs, orders = _setup(seed=9, n=50, D=4, allowed_frac=0.6)
+    for v in range(g.n):                                  # make the bases feasible
+        if not (int(g.allowed[v]) >> int(xs[0][v])) & 1:
+            xs[:, v] = [d for d in range(4) if (int(g.allowed[v]) >> d) & 1][0]
+    P = xs.shape[0]
+    for b in range(P):
+        for j in range(1, 800):
+            ok, x, o = O.candidate(g, P, b, xs, orders, j, 77, 1, MIX)
+            if ok:
+                for v in range(g.n):
+                    assert (int(g.allowed[v]) >> int(x[v])) & 1
+
+
+def test_flip_without_movable_ops_is_invalid(O):
+    g, xs, orders = _setup(seed=4, n=20)
+    g.allowed = np.ones(g.n, np.uint8)                    # every op pinned to device 0
+    xs[:] = 0
+    keys = O.candidate_keys(g, 3, 0, xs, orders, 0, 256, 5, 0, (1, 0, 0, 0))
+    assert keys[0] != O.KEY_INVALID
+    assert all(k == O.KEY_INVALID for k in keys[1:])
+
+
+def test_step_min_commit_and_sharding(O):
+    g, xs, orders = _setup(seed=12, n=40)
+    P = xs.shape[0]
+    K = 300
+    mk = np.asarray([O.makespan(g, xs[b], orders[b]) for b in range(P)], np.int64)
+    for step in range(4):
+        keys_all = [O.candidate_keys(g, P, b, xs, orders, 0, K, 2021, step, MIX) for b in range(P)]
+        xs1, or1, mk1 = xs.copy(), orders.copy(), mk.copy()
+        keys1 = O.search_step(g, xs1, or1, mk1, K, 2021, step, MIX, world=1)
+        xs3, or3, mk3 = xs.copy(), orders.copy(), mk.copy()
+        keys3 = O.search_step(g, xs3, or3, mk3, K, 2021, step, MIX, world=3)
+        assert (keys1 == keys3).all() and (xs1 == xs3).all() and (or1 == or3).all()
+        for b in range(P):
+            assert int(keys1[b]) == int(keys_all[b].min())
+            assert int(keys_all[b][0]) == (int(mk[b]) << 24)      # j=0 is the base itself
+            assert mk1[b] <= mk[b]
+            assert O.makespan(g, xs1[b], or1[b]) == mk1[b]        # committed base re-evaluates
+        xs, orders, mk = xs1, or1, mk1
+
+
+def test_keys_equal_makespan_of_decoded_candidate(O):
+    g, xs, orders = _setup(seed=13, n=30)
+    keys = O.candidate_keys(g, 3, 1, xs, orders, 0, 200, 42, 9, MIX)
+    for j in range(200):
+        ok, x, o = O.candidate(g, 3, 1, xs, orders, j, 42, 9, MIX)
+        assert ok
+        assert int(keys[j]) == (O.makespan(g, x, o) << 24) | j
