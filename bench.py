@@ -1,0 +1,344 @@
+#!/usr/bin/env python
+"""Benchmark: placement candidates evaluated/sec (and op-relaxations/sec) of the Pesto search
+step on B200 (BASELINE.json metric).  One JSON line on rank 0.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--config NAME] [--impl pesto|reference]
+
+A step = one pass of the whole hot path over one batch: K2 neighbour decode + K1 makespan of
+every candidate + K3 argmin (one kernel) -> N1 allreduce-MIN over ranks -> K4 commit.  At N=1 the
+workload is BASELINE.json configs[1] (inception_v3_2dev: 65,536 candidates/step); per-GPU work
+is fixed as N grows (weak scaling).  `--impl reference` times the CPU oracle on the same
+workload (the reference arm of this tier).
+"""
+
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+from workloads import configs, dag  # noqa: E402
+
+METRIC = "placement candidates evaluated/sec (and op-relaxations/sec) at 1/2/4/8 B200"
+DEFAULT_CONFIG = "inception_v3_2dev"
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--config", default=DEFAULT_CONFIG, choices=sorted(configs.CONFIGS))
+    ap.add_argument("--impl", default="pesto", choices=["pesto", "reference"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--cpu-seconds", type=float, default=12.0)
+    return ap.parse_args()
+
+
+def dist_env():
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return rank, world, local
+
+
+def peaks():
+    try:
+        return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except Exception:
+        return {}
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.proc = None
+        self.path = None
+
+    def __enter__(self):
+        fd, self.path = tempfile.mkstemp(suffix=".csv")
+        os.close(fd)
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}",
+                 "--format=csv,noheader,nounits", "-lms", "100"],
+                stdout=open(self.path, "w"), stderr=subprocess.DEVNULL)
+        except Exception:
+            self.proc = None
+        return self
+
+    def __exit__(self, *a):
+        if self.proc is not None:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        out = {"sm_mhz": None, "sm_max_mhz": None, "reasons": [], "samples": 0}
+        try:
+            rows = [r.split(",") for r in open(self.path).read().strip().splitlines() if r.strip()]
+        except Exception:
+            return out
+        sm, smax, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for r in rows:
+            r = [x.strip() for x in r]
+            if len(r) < 9:
+                continue
+            try:
+                sm.append(float(r[1]))
+                smax.append(float(r[2]))
+            except ValueError:
+                continue
+            for nm, val in zip(names, r[5:9]):
+                if val.lower().startswith("active"):
+                    reasons.add(nm)
+        if sm:
+            out.update(sm_mhz=statistics.median(sm), sm_max_mhz=max(smax), samples=len(sm))
+        out["reasons"] = sorted(reasons)
+        return out
+
+
+def seeds_for(P, G, g, n_bases: int):
+    """Search incumbents (row a1): expert, topological split, single-device, random."""
+    o_cp = G.seed_order(P.ORDER_CRITICAL_PATH)
+    o_fifo = G.seed_order(P.ORDER_FIFO)
+    o_rand = G.seed_order(P.ORDER_RANDOM, 2021)
+    xs = [G.seed_placement(P.PLACE_EXPERT, layer=g.layer) if g.layer is not None
+          else G.seed_placement(P.PLACE_TOPO_SPLIT, order=o_cp),
+          G.seed_placement(P.PLACE_TOPO_SPLIT, order=o_cp),
+          G.seed_placement(P.PLACE_SINGLE),
+          G.seed_placement(P.PLACE_RANDOM, seed=2021)]
+    os_ = [o_cp, o_cp, o_fifo, o_rand]
+    return np.stack(xs[:n_bases]), np.stack(os_[:n_bases])
+
+
+def oracle_rate(g, xs, orders, k_per_base, seconds, threads):
+    """Oracle (as it stands) on a bounded sample of this workload's step-0 candidates."""
+    from oracle import oracle as O
+    P_ = xs.shape[0]
+    mix = configs.MOVE_MIX
+    # calibrate a sample size that takes about `seconds` on `threads` threads
+    t0 = time.perf_counter()
+    probe = max(threads, 8)
+    O.candidate_keys(g, P_, 0, xs, orders, 0, probe, configs.SEARCH_SEED, 0, mix, threads)
+    dt = time.perf_counter() - t0
+    per = dt / probe
+    sample = int(max(probe, min(k_per_base, seconds / max(per, 1e-9))))
+    t0 = time.perf_counter()
+    done = 0
+    for b in range(P_):
+        cnt = sample // P_
+        if cnt <= 0:
+            continue
+        O.candidate_keys(g, P_, b, xs, orders, 0, cnt, configs.SEARCH_SEED, 0, mix, threads)
+        done += cnt
+    dt = time.perf_counter() - t0
+    return done / dt, done, dt
+
+
+def run_reference(args, rank, world):
+    if rank != 0:
+        return
+    cfg = configs.CONFIGS[args.config]
+    g = configs.graph_for(cfg)
+    from oracle import oracle as O  # noqa: F401  (TEST INFRASTRUCTURE: the reference arm)
+    threads = len(os.sched_getaffinity(0))
+    # seeds via plain host code shared with nothing: CP order from the generator's Kahn
+    order = dag.random_topo_order(g, 0)
+    xs = np.stack([np.zeros(g.n, np.uint8), dag.random_placements(g, 1, 1)[0]])
+    orders = np.stack([order, order])
+    per_step_budget = max(1.0, args.cpu_seconds / max(1, args.steps + args.warmup))
+    rates, times = [], []
+    for i in range(args.warmup + args.steps):
+        rate, done, dt = oracle_rate(g, xs, orders, cfg.candidates_per_gpu // 2, per_step_budget,
+                                     threads)
+        if i >= args.warmup:
+            rates.append(rate)
+            times.append(dt)
+    value = statistics.median(rates)
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": "candidates/s",
+            "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": 1e3 * cfg.candidates_per_gpu / value, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "int64", "data": "synthetic",
+            "config": {"workload": args.config, "n_ops": g.n, "n_edges": g.m, "D": g.D,
+                       "candidates_per_step": cfg.candidates_per_gpu},
+            "op_relaxations_per_s": value * g.n,
+            "cpu_baseline": {"value": value, "unit": "candidates/s", "cores": threads,
+                             "kind": "oracle",
+                             "sample": f"{args.steps} steps x ~{per_step_budget:.1f}s of step-0 "
+                                       "neighbour candidates, event-driven simulator"},
+            "e2e": {"value": value, "unit": "candidates/s", "h2d_bytes_per_step": 0,
+                    "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def run_pesto(args, rank, world, local):
+    import torch
+    import torch.distributed as dist
+    from paper_conf_middleware_hafeezsg021_b200 import pesto as P
+
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    cfg = configs.CONFIGS[args.config]
+    g = configs.graph_for(cfg)
+    G = P.Graph.from_arrays(g, device=local)
+    n_bases = cfg.bases
+    xs, orders = seeds_for(P, G, g, n_bases)
+    k_gpu = cfg.candidates_per_gpu
+    k_per_base = (k_gpu * world) // n_bases          # global K per base; each rank gets 1/world
+    nid = None
+    if world > 1:
+        obj = [P.nccl_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(obj, src=0)
+        nid = obj[0]
+    S = P.Search(G, xs, orders, k_per_base, configs.MOVE_MIX, configs.SEARCH_SEED, rank, world,
+                 nid)
+    seed_mk = [S.get(b)[0] for b in range(n_bases)]
+    stream = torch.cuda.current_stream()
+    # L2 flush buffer (> 126 MB L2) written between timed steps
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
+
+    def one_step(ev=None):
+        if ev is not None:
+            ev[0].record(stream)
+        S.eval(stream)
+        if ev is not None:
+            ev[1].record(stream)
+        S.reduce(stream)
+        S.commit(stream)
+        if ev is not None:
+            ev[2].record(stream)
+
+    for _ in range(args.warmup):
+        one_step()
+    torch.cuda.synchronize()
+    evs = [[torch.cuda.Event(enable_timing=True) for _ in range(3)] for _ in range(args.steps)]
+    launches0 = P.launch_count()
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    with ClockSampler(local) as clk:
+        wall0 = time.perf_counter()
+        for i in range(args.steps):
+            flush.fill_(i & 0xFF)                    # evict L2 between timed steps (not timed)
+            one_step(evs[i])
+        torch.cuda.synchronize()
+        wall = time.perf_counter() - wall0
+    if world > 1:
+        dist.barrier()
+    launches = P.launch_count() - launches0
+    step_ms = [e[0].elapsed_time(e[2]) for e in evs]
+    eval_ms = [e[0].elapsed_time(e[1]) for e in evs]
+    tot_ms = sum(step_ms)
+    t = torch.tensor([tot_ms, sum(eval_ms)], dtype=torch.float64, device="cuda")
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    tot_ms, tot_eval_ms = float(t[0]), float(t[1])
+    total_cands = k_gpu * world * args.steps
+    value = total_cands / (tot_ms / 1e3)
+    best_mk = [S.get(b)[0] for b in range(n_bases)]
+
+    # ---- end to end through the public API with host buffers (eval_batch_host) ----
+    e2e = None
+    if not args.no_e2e:
+        rows = P.pack_rows(dag.random_placements(g, 11 + rank, k_gpu), g.D)
+        pinned = torch.from_numpy(rows).pin_memory()
+        rows_h = pinned.numpy()
+        out_h = torch.empty(k_gpu, dtype=torch.int64).pin_memory().numpy()
+        o = orders[0]
+        for _ in range(max(1, args.warmup)):
+            G.eval_host(o, rows_h, out_h)
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        e2e_steps = max(3, min(args.steps, 10))
+        for _ in range(e2e_steps):
+            G.eval_host(o, rows_h, out_h)
+        e2e_s = torch.tensor([time.perf_counter() - t0], dtype=torch.float64, device="cuda")
+        if world > 1:
+            dist.all_reduce(e2e_s, op=dist.ReduceOp.MAX)
+        e2e = {"value": k_gpu * world * e2e_steps / float(e2e_s[0]), "unit": "candidates/s",
+               "h2d_bytes_per_step": int(rows.nbytes), "d2h_bytes_per_step": int(8 * k_gpu),
+               "api": "pesto_eval_batch_host (explicit placement rows, pinned host memory)"}
+
+    if rank != 0:
+        if world > 1:
+            dist.destroy_process_group()
+        return
+
+    # ---- roofline of the dominant kernel (K1 eval) ----
+    pk = peaks()
+    hbm = pk.get("hbm_gbs")
+    peak_note = "measured (MEASURED_PEAKS.json hbm_gbs)"
+    if not hbm:
+        hbm, peak_note = 6650.0, "fallback (B200_PROFILING.md)"
+    # algorithmic bytes: the ready-time slot state moves 2 int64 accesses per edge per candidate
+    # (one push, one read-or-RMW): 16*m bytes per candidate
+    alg_bytes_launch = 16.0 * g.m * k_gpu
+    eval_avg_s = (tot_eval_ms / args.steps) / 1e3
+    achieved = alg_bytes_launch / eval_avg_s / 1e9
+    st = G.stats(orders[0])
+    line = {"metric": METRIC, "value": value, "unit": "candidates/s", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": tot_ms / args.steps,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int64",
+            "data": "synthetic",
+            "config": {"workload": args.config, "n_ops": g.n, "n_edges": g.m, "D": g.D,
+                       "candidates_per_step": k_gpu * world, "candidates_per_gpu": k_gpu,
+                       "bases": n_bases, "k_per_base": k_per_base, "move_mix": configs.MOVE_MIX,
+                       "live_slots": st["live_slots"], "l2": "flushed between timed steps",
+                       "parallelism": f"candidate-dp{world}"},
+            "op_relaxations_per_s": value * g.n, "edge_relaxations_per_s": value * g.m,
+            "eval_kernel_ms": tot_eval_ms / args.steps,
+            "roofline": {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",
+                         "frac": achieved / hbm, "traffic": None, "peak_source": peak_note,
+                         "note": "algorithmic slot-state bytes 16*m per candidate / K1 time"},
+            "gpu_launches": int(launches),
+            "wall_s_timed_region": wall,
+            "search": {"seed_makespans": seed_mk, "best_makespans": best_mk},
+            "e2e": e2e}
+    line["clocks"] = clk.summary()
+    if not args.no_cpu_baseline:
+        threads = len(os.sched_getaffinity(0))
+        rate, done, dt = oracle_rate(g, xs, orders, k_per_base, args.cpu_seconds, threads)
+        line["cpu_baseline"] = {"value": rate, "unit": "candidates/s", "cores": threads,
+                                "kind": "oracle",
+                                "sample": f"{done} step-0 neighbour candidates of the same "
+                                          f"{n_bases} bases ({dt:.1f}s)"}
+    print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def main():
+    args = parse()
+    rank, world, local = dist_env()
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+        return
+    run_pesto(args, rank, world, local)
+
+
+if __name__ == "__main__":
+    main()

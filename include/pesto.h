@@ -1,0 +1,202 @@
+/*
+ * pesto.h -- C ABI of libpesto.so: batched makespan evaluation and parallel local search over
+ * operation-level placements and schedules of a DNN op DAG, on B200 (sm_100a).
+ *
+ * The operation every entry point computes is Pesto's objective (Hafeez et al., Middleware'21,
+ * PAPER.md): the makespan C_max (L159-162 eq. (3); "time between the first task arrival and
+ * the last task completion", L111) of a DAG G=(V,E) whose ops have compute times p_i
+ * (L142 §3.2.1), under
+ *   - precedence: op j starts only after op i completed and its data transfer completed (L144);
+ *   - a transfer only when producer and consumer sit on different devices, taking
+ *     T = beta0 + beta1 * bytes (L138 §3.1) on the directed link between them (L144);
+ *   - no overlap on each device and on each link, no pre-emption (L146);
+ *   - one First-Come-First-Served queue per directed link (L144, L188-198 §3.2.2);
+ *   - a schedule given as a priority order pi: each device runs its ops in pi order (the
+ *     per-device order TF enforces with control dependencies, L279; the simulator's "adds
+ *     precedence constraints", L374).
+ * Readings of points PAPER.md leaves open are listed in DESIGN.md §2 (R1-R17).  All times are
+ * int64 nanoseconds, so results are exact and reproducible bit for bit.
+ *
+ * Conventions
+ *   - Host arrays passed to *_create / pesto_comm_model are COPIED; the caller may free them
+ *     on return.  Device pointers (placements, makespans, keys) are BORROWED and must stay
+ *     alive until the work enqueued on `cuda_stream` completes.  Streams are borrowed
+ *     (cudaStream_t passed as void*; NULL = the legacy default stream).
+ *   - Every call returns a pesto_status; no C++ exception crosses the ABI.  Validation
+ *     failures return before any GPU work.  Asynchronous CUDA/NCCL errors surface on the next
+ *     call that synchronises.  pesto_last_error() gives a thread-local description.
+ *   - Per-candidate infeasibility (a device code >= D, a device the op's mask forbids, an
+ *     invalid search move) is data, not an error: makespan INT64_MAX / key UINT64_MAX.
+ *   - Handles are not thread-safe.  Destroy a handle only after synchronising the streams
+ *     that used it.
+ */
+#ifndef PESTO_H
+#define PESTO_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct pesto_graph pesto_graph;     /* opaque: host copies + device buffers, one GPU */
+typedef struct pesto_search pesto_search;   /* opaque: population, keys, optional NCCL comm   */
+
+typedef enum {
+    PESTO_OK = 0,
+    PESTO_EINVAL = 1,      /* bad argument: index out of range, self loop, negative size ...  */
+    PESTO_ECYCLE = 2,      /* G is not a DAG (L142)                                            */
+    PESTO_ENOTTOPO = 3,    /* order is not a permutation / not a linear extension of G         */
+    PESTO_EOVERFLOW = 4,   /* sum p + sum_e max_L t_e >= 2^40 ns, or a t_e overflows int64     */
+    PESTO_ENOMEM = 5,      /* host or device allocation failed                                 */
+    PESTO_ECUDA = 6,       /* CUDA runtime error (see pesto_last_error)                        */
+    PESTO_ENCCL = 7,       /* NCCL unavailable or failed                                       */
+    PESTO_ESTATE = 8       /* call not valid in this state (comm model unset, host-only ...)   */
+} pesto_status;
+
+#define PESTO_INFEASIBLE INT64_MAX
+#define PESTO_KEY_INVALID UINT64_MAX
+#define PESTO_MAX_OPS (1 << 24)
+#define PESTO_MAX_DEVICES 8
+
+/* ------------------------------------------------------------------------------------------ */
+/* Graph ingest                                                              */
+/* ------------------------------------------------------------------------------------------ */
+typedef struct {
+    int32_t n_ops;              /* 1 .. 2^24                                                  */
+    const int64_t *compute_ns;  /* [n_ops] p_i >= 0 (L142)                                     */
+    int64_t n_edges;            /* >= 0; multi-edges allowed, each its own tensor (R4)         */
+    const int32_t *src;         /* [n_edges] producer op id                                    */
+    const int32_t *dst;         /* [n_edges] consumer op id; src != dst; G acyclic              */
+    const int64_t *bytes;       /* [n_edges] >= 0, tensor size for the comm model (L138)       */
+    int32_t n_devices;          /* D in 1..8; placement rows use b = 1 (D<=2), 2 (D<=4), 4 bits */
+    const uint8_t *allowed;     /* [n_ops] device bitmask (device affinity, L121/L175) or NULL  */
+    int32_t cuda_device;        /* ordinal for device buffers; -1 = host-only handle (ingest,    */
+                                /* layout, seeds; eval/search then return PESTO_ESTATE)         */
+} pesto_graph_desc;
+
+/* Validates (indices, self loops, Kahn cycle check) and copies G.  Errors: EINVAL, ECYCLE,
+ * ENOMEM, ECUDA. */
+pesto_status pesto_graph_create(const pesto_graph_desc *desc, pesto_graph **out);
+void pesto_graph_destroy(pesto_graph *g);                          /* NULL-safe */
+
+/* Linear comm model of the directed link src_dev -> dst_dev (L138 §3.1; per ordered pair,
+ * L188-198): t_e = beta0_ns + ceil(bytes_e * beta1_fs_per_byte / 10^6) (reading R6, exact via
+ * a 128-bit product).  src_dev/dst_dev = -1 is a wildcard (all pairs a != b).  Both
+ * coefficients >= 0.  Errors: EINVAL, EOVERFLOW (the 2^40 guard is checked here, over all
+ * links set so far). */
+pesto_status pesto_comm_model(pesto_graph *g, int32_t src_dev, int32_t dst_dev,
+                              int64_t beta0_ns, int64_t beta1_fs_per_byte);
+
+typedef struct {
+    int32_t n_ops, n_devices;
+    int64_t n_edges;
+    int32_t live_slots;         /* W: ready-time slots per candidate for this order           */
+    int32_t n_tiles;            /* DAG tiles streamed by TMA per candidate group               */
+    int64_t layout_bytes;       /* position-space record stream size                            */
+    int32_t max_in_degree, max_out_degree;
+    int32_t link_classes;       /* distinct (beta0, beta1) among the directed links              */
+    int32_t time32_exact;       /* 1 if every makespan fits int32 (worst-case guard < 2^31)      */
+} pesto_graph_stats;
+
+/* Builds (or fetches from the per-graph cache) the position-space layout for `order` and
+ * reports its statistics.  order: host [n_ops], a topological order.  Errors: ENOTTOPO. */
+pesto_status pesto_graph_stats_for(pesto_graph *g, const int32_t *order, pesto_graph_stats *st);
+
+/* ------------------------------------------------------------------------------------------ */
+/* Seeds (host, once)                                                         */
+/* ------------------------------------------------------------------------------------------ */
+enum { PESTO_ORDER_CRITICAL_PATH = 0,  /* Kahn, max-heap on bottom level (p only), ties by op id;
+                                          the naive critical-path list order of L98 */
+       PESTO_ORDER_FIFO = 1,           /* Kahn with a FIFO queue in op-id order                  */
+       PESTO_ORDER_RANDOM = 2 };       /* Kahn with a seeded random pick (TF ready queue, L90)    */
+pesto_status pesto_seed_order(pesto_graph *g, int32_t kind, uint64_t seed, int32_t *order_out);
+
+enum { PESTO_PLACE_SINGLE = 0,         /* every op on its lowest allowed device                  */
+       PESTO_PLACE_EXPERT = 1,         /* contiguous layers per device: floor(layer*D/n_layers)  */
+                                       /* (L308; the caller's layer tags carry the colocations)  */
+       PESTO_PLACE_TOPO_SPLIT = 2,     /* `order` cut into D contiguous segments of ~equal sum p  */
+                                       /* (an mTOPO-like split, L320)                             */
+       PESTO_PLACE_RANDOM = 3 };       /* seeded uniform over allowed devices                     */
+/* x_out: host [n_ops], one device code per op.  layer_tags needed only for EXPERT, order only
+ * for TOPO_SPLIT.  Ops whose mask forbids the chosen device take their lowest allowed one. */
+pesto_status pesto_seed_placement(pesto_graph *g, int32_t kind, const int32_t *order,
+                                  const int32_t *layer_tags, uint64_t seed, uint8_t *x_out);
+
+/* ------------------------------------------------------------------------------------------ */
+/* Batched evaluation of explicit candidates (SURVEY §8(a) a3 + a4, call stack C4)             */
+/* ------------------------------------------------------------------------------------------ */
+/* Makespan of n_cand candidates sharing one schedule order pi.
+ *   order:      HOST [n_ops] topological order (layout cached by content).
+ *   placements: DEVICE, n_cand rows; row c holds op i's device code in bits [b*i, b*i+b) of the
+ *               row (little-endian bytes), b = 1 (D<=2), 2 (D<=4), 4 (D<=8).
+ *   row_stride_bytes: >= ceil(n_ops*b/8), a multiple of 16.
+ *   makespans:  DEVICE [n_cand] int64 out; INT64_MAX for an infeasible row.
+ * Enqueued on cuda_stream; returns without synchronising.  Errors: EINVAL, ENOTTOPO, ESTATE
+ * (comm model missing for a link, or host-only handle), ENOMEM, ECUDA. */
+pesto_status pesto_eval_batch(pesto_graph *g, const int32_t *order, const void *placements,
+                              int64_t row_stride_bytes, int64_t n_cand, int64_t *makespans,
+                              void *cuda_stream);
+
+/* Same with HOST buffers (ideally pinned): copies the rows in, evaluates, copies makespans
+ * out, and synchronises the stream before returning (the end-to-end entry point). */
+pesto_status pesto_eval_batch_host(pesto_graph *g, const int32_t *order,
+                                   const void *placements_host, int64_t row_stride_bytes,
+                                   int64_t n_cand, int64_t *makespans_host, void *cuda_stream);
+
+/* ------------------------------------------------------------------------------------------ */
+/* Parallel local search (DESIGN.md §4 for the move spec)         */
+/* ------------------------------------------------------------------------------------------ */
+typedef struct {
+    int32_t n_bases;            /* P >= 1 independent incumbents                               */
+    const uint8_t *base_x;      /* HOST [P * n_ops] device code per op (must be feasible)      */
+    const int32_t *base_order;  /* HOST [P * n_ops] topological orders                          */
+    int64_t k_per_base;         /* K: global neighbours per base per step, 1 .. 2^24            */
+    int32_t mix[4];             /* FLIP1, FLIPk, WINDOW lane-move weights; SWAP % of groups      */
+    uint64_t seed;
+    int32_t rank, world;        /* candidate ids of base b split as [floor(rK/W), floor((r+1)K/W)) */
+    const uint8_t *nccl_unique_id;  /* 128 bytes (ncclUniqueId) when world > 1, else NULL; with  */
+                                    /* NULL and world > 1 the caller reduces keys itself          */
+} pesto_search_desc;
+
+pesto_status pesto_search_create(pesto_graph *g, const pesto_search_desc *desc,
+                                 pesto_search **out);
+
+/* One step: neighbour decode + makespan + CTA argmin (K1) -> ncclAllReduce MIN over ranks
+ * (N1, only with an NCCL comm) -> commit (K4) on every rank.  Enqueued on cuda_stream.  When
+ * SWAP moves are enabled it synchronises once to learn whether an order changed. */
+pesto_status pesto_search_step(pesto_search *s, void *cuda_stream);
+
+/* The three phases of a step, for callers that reduce keys themselves (tests, fake shards). */
+pesto_status pesto_search_eval(pesto_search *s, void *cuda_stream);   /* keys = local minima */
+pesto_status pesto_search_reduce(pesto_search *s, void *cuda_stream); /* NCCL MIN (no-op w/o) */
+pesto_status pesto_search_keys(pesto_search *s, uint64_t *keys_host, void *cuda_stream); /*syncs*/
+pesto_status pesto_search_set_keys(pesto_search *s, const uint64_t *keys_host, void *cuda_stream);
+pesto_status pesto_search_commit(pesto_search *s, void *cuda_stream); /* K4 + step += 1        */
+
+/* Keys (makespan << 24 | j, UINT64_MAX if invalid) of candidates j in [j0, j1) of `base` at
+ * the current step, into DEVICE keys_out[j1 - j0] (parity/debug; ignores rank/world). */
+pesto_status pesto_search_candidate_keys(pesto_search *s, int32_t base, int64_t j0, int64_t j1,
+                                         uint64_t *keys_out, void *cuda_stream);
+
+/* Current incumbent of `base` (synchronises): makespan, x (host [n_ops]) and order. */
+pesto_status pesto_search_get(pesto_search *s, int32_t base, int64_t *makespan,
+                              uint8_t *x_host, int32_t *order_host);
+int64_t pesto_search_step_count(const pesto_search *s);
+
+/* ncclGetUniqueId through the process's libnccl.so.2 (rank 0 calls it and broadcasts the 128
+ * bytes over its own process group).  Errors: ENCCL if NCCL cannot be loaded. */
+pesto_status pesto_nccl_unique_id(uint8_t *out128);
+void pesto_search_destroy(pesto_search *s);                        /* NULL-safe */
+
+/* ------------------------------------------------------------------------------------------ */
+const char *pesto_last_error(void);       /* thread-local detail of the last failure */
+const char *pesto_status_str(pesto_status s);
+int32_t pesto_version(void);              /* major*10000 + minor*100 + patch */
+/* Number of kernel launches this process has enqueued through libpesto (bench evidence). */
+int64_t pesto_launch_count(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif

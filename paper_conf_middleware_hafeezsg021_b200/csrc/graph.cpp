@@ -1,0 +1,683 @@
+// graph.cpp -- graph ingest, comm model, position-space layout, seeds and batched evaluation
+// (SURVEY §8(a) rows a0, a1, a3/a4 host side; C ABI in include/pesto.h).
+#include <algorithm>
+#include <cstring>
+#include <queue>
+#include <string>
+
+#include "host.h"
+#include "moves.cuh"
+
+using namespace pesto;
+
+namespace pesto {
+
+static thread_local std::string g_err;
+
+void set_error(const std::string &msg) { g_err = msg; }
+pesto_status fail(pesto_status s, const std::string &msg) {
+    g_err = msg;
+    return s;
+}
+pesto_status cuda_fail(cudaError_t e, const char *what) {
+    g_err = std::string(what) + ": " + cudaGetErrorString(e);
+    return e == cudaErrorMemoryAllocation ? PESTO_ENOMEM : PESTO_ECUDA;
+}
+
+static constexpr int64_t kGuard40 = int64_t(1) << 40;
+static constexpr int kMaxInlineBytes = 2048;
+
+// t = beta0 + ceil(bytes * beta1_fs / 10^6) (PAPER.md L138 linear model, reading R6); -1 overflow
+static int64_t transfer_ns(int64_t bytes, int64_t beta0, int64_t beta1) {
+    unsigned __int128 prod = (unsigned __int128)(uint64_t)bytes * (uint64_t)beta1;
+    unsigned __int128 q = (prod + 999999u) / 1000000u;
+    unsigned __int128 t = q + (uint64_t)beta0;
+    if (t > (unsigned __int128)INT64_MAX) return -1;
+    return (int64_t)t;
+}
+
+static int planes_for(int D) { return D <= 2 ? 1 : (D <= 4 ? 2 : 4); }
+
+// worst-case makespan bound over the links set so far: sum p + sum_e max_L t_e (a0 step 3)
+static int64_t worst_total(const pesto_graph *g, const std::vector<int64_t> &b0,
+                           const std::vector<int64_t> &b1, const std::vector<uint8_t> &set) {
+    int64_t total = 0;
+    for (int32_t v = 0; v < g->n; v++) {
+        total += g->p[v];
+        if (total >= kGuard40) return -1;
+    }
+    for (int64_t e = 0; e < g->m; e++) {
+        int64_t worst = 0;
+        for (int L = 0; L < g->D * g->D; L++) {
+            if (!set[L]) continue;
+            int64_t t = transfer_ns(g->bytes[e], b0[L], b1[L]);
+            if (t < 0) return -1;
+            worst = std::max(worst, t);
+        }
+        total += worst;
+        if (total >= kGuard40) return -1;
+    }
+    return total;
+}
+
+pesto_status ensure_comm_tables(pesto_graph *g) {
+    const int D = g->D;
+    for (int a = 0; a < D; a++)
+        for (int b = 0; b < D; b++)
+            if (a != b && !g->link_set[a * D + b])
+                return fail(PESTO_ESTATE, "comm model not set for link " + std::to_string(a) +
+                                              "->" + std::to_string(b));
+    if (g->t_gen == g->comm_gen) return PESTO_OK;
+    // link classes: distinct (beta0, beta1) in order of first appearance
+    std::vector<std::pair<int64_t, int64_t>> cls;
+    std::memset(g->link_class, 0, sizeof(g->link_class));
+    for (int a = 0; a < D; a++)
+        for (int b = 0; b < D; b++) {
+            if (a == b) continue;
+            const int L = a * D + b;
+            std::pair<int64_t, int64_t> k{g->beta0[L], g->beta1[L]};
+            int c = -1;
+            for (size_t i = 0; i < cls.size(); i++)
+                if (cls[i] == k) c = (int)i;
+            if (c < 0) { c = (int)cls.size(); cls.push_back(k); }
+            g->link_class[L] = (uint8_t)c;
+        }
+    if (cls.empty()) cls.push_back({0, 0});                 // D == 1: no links at all
+    g->n_classes = (int32_t)cls.size();
+    g->t_class.assign((size_t)g->m * g->n_classes, 0);
+    for (int64_t e = 0; e < g->m; e++)
+        for (int c = 0; c < g->n_classes; c++)
+            g->t_class[(size_t)e * g->n_classes + c] = transfer_ns(g->bytes[e], cls[c].first, cls[c].second);
+    g->t_gen = g->comm_gen;
+    g->cache.clear();                                        // layouts embed t
+    return PESTO_OK;
+}
+
+// ---------------------------------------------------------------------------------------------
+// position-space layout for one order (a0 steps 4-5)
+// ---------------------------------------------------------------------------------------------
+pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<Layout> &out,
+                          bool use_cache) {
+    pesto_status s = ensure_comm_tables(g);
+    if (s) return s;
+    const int32_t n = g->n;
+    if (!order) return fail(PESTO_EINVAL, "order is NULL");
+    if (use_cache) {
+        for (auto it = g->cache.begin(); it != g->cache.end(); ++it) {
+            if ((*it)->comm_gen == g->comm_gen &&
+                std::memcmp((*it)->order.data(), order, (size_t)n * 4) == 0) {
+                out = *it;
+                g->cache.splice(g->cache.begin(), g->cache, it);
+                return PESTO_OK;
+            }
+        }
+    }
+    auto L = std::make_shared<Layout>();
+    L->comm_gen = g->comm_gen;
+    L->order.assign(order, order + n);
+    L->pos.assign(n, -1);
+    for (int32_t k = 0; k < n; k++) {
+        const int32_t v = order[k];
+        if (v < 0 || v >= n || L->pos[v] != -1) return fail(PESTO_ENOTTOPO, "order is not a permutation");
+        L->pos[v] = k;
+    }
+    for (int64_t e = 0; e < g->m; e++)
+        if (L->pos[g->src[e]] >= L->pos[g->dst[e]])
+            return fail(PESTO_ENOTTOPO, "order violates edge " + std::to_string(e));
+    const std::vector<int32_t> &pos = L->pos;
+
+    // out-edges of every producer sorted by (successor position, edge index): FCFS tie order R3
+    std::vector<int64_t> sorted(g->out_edges);
+    for (int32_t u = 0; u < n; u++) {
+        auto b = sorted.begin() + g->out_off[u], e = sorted.begin() + g->out_off[u + 1];
+        std::sort(b, e, [&](int64_t a, int64_t c) {
+            const int32_t pa = pos[g->dst[a]], pc = pos[g->dst[c]];
+            return pa != pc ? pa < pc : a < c;
+        });
+    }
+    // ready-time slot intervals: consumer w lives from its first producer's position through
+    // pos(w) + 1 (one position of padding keeps an adjacent swap exact)
+    std::vector<int32_t> first(n, INT32_MAX);
+    for (int64_t e = 0; e < g->m; e++) first[g->dst[e]] = std::min(first[g->dst[e]], pos[g->src[e]]);
+    std::vector<std::vector<int32_t>> starts(n), frees(n);
+    for (int32_t w = 0; w < n; w++) {
+        if (first[w] == INT32_MAX) continue;
+        starts[first[w]].push_back(w);
+        if (pos[w] + 2 < n) frees[pos[w] + 2].push_back(w);
+    }
+    std::vector<int32_t> slot(n, kNoSlot), free_stack;
+    int32_t W = 0;
+    for (int32_t k = 0; k < n; k++) {
+        for (int32_t w : frees[k]) free_stack.push_back(slot[w]);
+        for (int32_t w : starts[k]) {
+            if (!free_stack.empty()) { slot[w] = free_stack.back(); free_stack.pop_back(); }
+            else slot[w] = W++;
+        }
+    }
+    L->W = std::max(W, 1);
+    // first push into each slot, in processing order
+    std::vector<uint8_t> seen(n, 0), first_flag(g->m, 0);
+    for (int32_t k = 0; k < n; k++) {
+        const int32_t u = order[k];
+        for (int64_t i = g->out_off[u]; i < g->out_off[u + 1]; i++) {
+            const int64_t e = sorted[i];
+            if (!seen[g->dst[e]]) { seen[g->dst[e]] = 1; first_flag[e] = 1; }
+        }
+    }
+    // records + tiles
+    const int C = g->n_classes;
+    const int es = edge_stride_for(C);
+    auto put_edge = [&](std::vector<uint8_t> &buf, int64_t e) {
+        size_t at = buf.size();
+        buf.resize(at + es, 0);
+        EdgeRec r;
+        r.t0 = g->t_class[(size_t)e * C];
+        r.succ_pos = pos[g->dst[e]];
+        r.slot = (uint32_t)slot[g->dst[e]] | (first_flag[e] ? kEdgeFirst : 0u);
+        std::memcpy(buf.data() + at, &r, sizeof r);
+        for (int c = 1; c < C; c++) {
+            int64_t t = g->t_class[(size_t)e * C + c];
+            std::memcpy(buf.data() + at + 16 + 8 * (c - 1), &t, 8);
+        }
+    };
+    L->blob.clear();
+    L->heavy.clear();
+    L->tiles.clear();
+    size_t tile_start = 0;
+    int32_t tile_pos = 0;
+    auto open_tile = [&](int32_t k) {
+        tile_start = L->blob.size();
+        tile_pos = k;
+        L->blob.resize(tile_start + kTileHeader, 0);
+    };
+    auto close_tile = [&](int32_t k_end) {
+        TileDesc td{};
+        td.byte_off = (int64_t)tile_start;
+        td.bytes = (int32_t)(L->blob.size() - tile_start);
+        td.pos_begin = tile_pos;
+        td.pos_end = k_end;
+        int32_t hdr[4] = {tile_pos, k_end, td.bytes, 0};
+        std::memcpy(L->blob.data() + tile_start, hdr, 16);
+        L->tiles.push_back(td);
+        L->stage_bytes = std::max(L->stage_bytes, td.bytes);
+    };
+    open_tile(0);
+    for (int32_t k = 0; k < n; k++) {
+        const int32_t u = order[k];
+        const int64_t nout = g->out_off[u + 1] - g->out_off[u];
+        const bool heavy = nout * es > kMaxInlineBytes;
+        const size_t rec_bytes = 16 + (heavy ? 16 : (size_t)nout * es);
+        if (k > tile_pos && L->blob.size() - tile_start + rec_bytes > (size_t)kTileTarget) {
+            close_tile(k);
+            open_tile(k);
+        }
+        OpRec op;
+        op.p = g->p[u];
+        op.in_slot = slot[u];
+        op.nout = heavy ? (kOpHeavy | 0u) : (uint32_t)nout;
+        size_t at = L->blob.size();
+        L->blob.resize(at + 16);
+        std::memcpy(L->blob.data() + at, &op, 16);
+        if (heavy) {
+            ExtRec ext{(int64_t)L->heavy.size(), nout};
+            at = L->blob.size();
+            L->blob.resize(at + 16);
+            std::memcpy(L->blob.data() + at, &ext, 16);
+            for (int64_t i = g->out_off[u]; i < g->out_off[u + 1]; i++) put_edge(L->heavy, sorted[i]);
+        } else {
+            for (int64_t i = g->out_off[u]; i < g->out_off[u + 1]; i++) put_edge(L->blob, sorted[i]);
+        }
+    }
+    close_tile(n);
+    // order-move helpers
+    L->adj_next.assign(n, 0);
+    for (int32_t k = 0; k + 1 < n; k++) {
+        const int32_t u = order[k], w = order[k + 1];
+        for (int64_t i = g->out_off[u]; i < g->out_off[u + 1]; i++)
+            if (g->dst[g->out_edges[i]] == w) L->adj_next[k] = 1;
+    }
+    L->allowed_pos.resize(n);
+    for (int32_t k = 0; k < n; k++) L->allowed_pos[k] = g->allowed[order[k]];
+    if (use_cache) {
+        g->cache.push_front(L);
+        while (g->cache.size() > 8) g->cache.pop_back();
+    }
+    out = L;
+    return PESTO_OK;
+}
+
+template <class T>
+static cudaError_t upload_vec(DevBuf &d, const std::vector<T> &v) {
+    cudaError_t e = d.ensure(std::max<size_t>(v.size() * sizeof(T), 16));
+    if (e != cudaSuccess) return e;
+    if (!v.empty()) e = cudaMemcpy(d.ptr, v.data(), v.size() * sizeof(T), cudaMemcpyHostToDevice);
+    return e;
+}
+
+pesto_status upload_layout(pesto_graph *g, Layout &L) {
+    if (L.on_device) return PESTO_OK;
+    DeviceGuard guard(g->device);
+    cudaError_t e;
+    if ((e = upload_vec(L.d_blob, L.blob)) != cudaSuccess) return cuda_fail(e, "upload layout");
+    if ((e = upload_vec(L.d_heavy, L.heavy)) != cudaSuccess) return cuda_fail(e, "upload layout");
+    if ((e = upload_vec(L.d_tiles, L.tiles)) != cudaSuccess) return cuda_fail(e, "upload layout");
+    if ((e = upload_vec(L.d_pos, L.pos)) != cudaSuccess) return cuda_fail(e, "upload layout");
+    if ((e = upload_vec(L.d_adj, L.adj_next)) != cudaSuccess) return cuda_fail(e, "upload layout");
+    if ((e = upload_vec(L.d_allowed_pos, L.allowed_pos)) != cudaSuccess)
+        return cuda_fail(e, "upload layout");
+    L.on_device = true;
+    std::vector<BaseLayoutDev> view{layout_view(L)};
+    if ((e = upload_vec(L.d_view, view)) != cudaSuccess) return cuda_fail(e, "upload layout");
+    return PESTO_OK;
+}
+
+BaseLayoutDev layout_view(const Layout &L) {
+    BaseLayoutDev v{};
+    v.blob = L.d_blob.as<uint8_t>();
+    v.tiles = L.d_tiles.as<TileDesc>();
+    v.heavy = L.d_heavy.as<uint8_t>();
+    v.pos_of = L.d_pos.as<int32_t>();
+    v.allowed_pos = L.d_allowed_pos.as<uint8_t>();
+    v.adj_next = L.d_adj.as<uint8_t>();
+    v.bits = nullptr;
+    v.n_tiles = (int32_t)L.tiles.size();
+    v.W = L.W;
+    return v;
+}
+
+void fill_eval_common(const pesto_graph *g, EvalParams &p) {
+    std::memset(&p, 0, sizeof p);
+    p.n = g->n;
+    p.D = g->D;
+    p.planes = g->planes;
+    p.words = g->words;
+    p.edge_stride = edge_stride_for(g->n_classes);
+    p.n_classes = g->n_classes;
+    std::memcpy(p.link_class, g->link_class, 64);
+    p.all_allowed = g->all_allowed ? 1 : 0;
+}
+
+pesto_status ensure_state(pesto_graph *g, const EvalParams &p, int search_mode, int64_t n_tasks,
+                          int *grid_out) {
+    int per_sm = eval_max_ctas_per_sm(p, search_mode);
+    if (per_sm <= 0)
+        return fail(PESTO_ECUDA, "eval kernel does not fit on an SM (smem " +
+                                     std::to_string(eval_smem_bytes(p, search_mode)) + " B)");
+    int64_t grid = std::min<int64_t>(n_tasks, (int64_t)g->sms * per_sm);
+    grid = std::max<int64_t>(grid, 1);
+    size_t bytes = (size_t)grid * kWarps * (size_t)std::max(p.max_W, 1) * 32 * sizeof(int64_t);
+    cudaError_t e = g->d_state.ensure(bytes);
+    if (e != cudaSuccess) return cuda_fail(e, "allocate slot state");
+    *grid_out = (int)grid;
+    return PESTO_OK;
+}
+
+static uint64_t splitmix_next(uint64_t &s) {
+    s += 0x9E3779B97F4A7C15ull;
+    return mix64(s);
+}
+
+}  // namespace pesto
+
+// =============================================================================================
+// C ABI
+// =============================================================================================
+extern "C" {
+
+const char *pesto_last_error(void) { return g_err.c_str(); }
+
+const char *pesto_status_str(pesto_status s) {
+    switch (s) {
+        case PESTO_OK: return "PESTO_OK";
+        case PESTO_EINVAL: return "PESTO_EINVAL";
+        case PESTO_ECYCLE: return "PESTO_ECYCLE";
+        case PESTO_ENOTTOPO: return "PESTO_ENOTTOPO";
+        case PESTO_EOVERFLOW: return "PESTO_EOVERFLOW";
+        case PESTO_ENOMEM: return "PESTO_ENOMEM";
+        case PESTO_ECUDA: return "PESTO_ECUDA";
+        case PESTO_ENCCL: return "PESTO_ENCCL";
+        case PESTO_ESTATE: return "PESTO_ESTATE";
+    }
+    return "PESTO_?";
+}
+
+int32_t pesto_version(void) { return 100; }
+int64_t pesto_launch_count(void) { return launch_count_value(); }
+
+pesto_status pesto_graph_create(const pesto_graph_desc *d, pesto_graph **out) {
+    if (!d || !out) return fail(PESTO_EINVAL, "NULL argument");
+    *out = nullptr;
+    if (d->n_ops < 1 || d->n_ops > PESTO_MAX_OPS) return fail(PESTO_EINVAL, "n_ops out of range");
+    if (d->n_edges < 0) return fail(PESTO_EINVAL, "n_edges < 0");
+    if (d->n_devices < 1 || d->n_devices > PESTO_MAX_DEVICES)
+        return fail(PESTO_EINVAL, "n_devices out of range");
+    if (!d->compute_ns) return fail(PESTO_EINVAL, "compute_ns is NULL");
+    if (d->n_edges > 0 && (!d->src || !d->dst || !d->bytes))
+        return fail(PESTO_EINVAL, "edge arrays are NULL");
+    std::unique_ptr<pesto_graph> g(new (std::nothrow) pesto_graph());
+    if (!g) return fail(PESTO_ENOMEM, "host allocation");
+    const int32_t n = d->n_ops;
+    const int64_t m = d->n_edges;
+    g->n = n;
+    g->m = m;
+    g->D = d->n_devices;
+    g->planes = planes_for(g->D);
+    g->words = (n + 31) / 32;
+    g->device = d->cuda_device;
+    try {
+        g->p.assign(d->compute_ns, d->compute_ns + n);
+        if (m) {
+            g->src.assign(d->src, d->src + m);
+            g->dst.assign(d->dst, d->dst + m);
+            g->bytes.assign(d->bytes, d->bytes + m);
+        }
+    } catch (...) {
+        return fail(PESTO_ENOMEM, "host allocation");
+    }
+    for (int32_t v = 0; v < n; v++)
+        if (g->p[v] < 0) return fail(PESTO_EINVAL, "compute_ns[" + std::to_string(v) + "] < 0");
+    for (int64_t e = 0; e < m; e++) {
+        if (g->src[e] < 0 || g->src[e] >= n || g->dst[e] < 0 || g->dst[e] >= n)
+            return fail(PESTO_EINVAL, "edge " + std::to_string(e) + " index out of range");
+        if (g->src[e] == g->dst[e]) return fail(PESTO_EINVAL, "self loop at edge " + std::to_string(e));
+        if (g->bytes[e] < 0) return fail(PESTO_EINVAL, "bytes[" + std::to_string(e) + "] < 0");
+    }
+    const unsigned full = (1u << g->D) - 1u;
+    g->allowed.assign(n, (uint8_t)full);
+    if (d->allowed) {
+        for (int32_t v = 0; v < n; v++) {
+            const unsigned msk = d->allowed[v] & full;
+            if (!msk) return fail(PESTO_EINVAL, "op " + std::to_string(v) + " allows no device");
+            g->allowed[v] = (uint8_t)msk;
+            if (msk != full) g->all_allowed = false;
+        }
+    }
+    // out-edge CSR + Kahn cycle check (L142: G is a DAG)
+    g->out_off.assign((size_t)n + 1, 0);
+    g->indeg.assign(n, 0);
+    for (int64_t e = 0; e < m; e++) { g->out_off[g->src[e] + 1]++; g->indeg[g->dst[e]]++; }
+    for (int32_t v = 0; v < n; v++) g->out_off[v + 1] += g->out_off[v];
+    g->out_edges.resize(m);
+    {
+        std::vector<int64_t> fill(g->out_off.begin(), g->out_off.end() - 1);
+        for (int64_t e = 0; e < m; e++) g->out_edges[fill[g->src[e]]++] = e;
+        std::vector<int32_t> deg(g->indeg), q;
+        q.reserve(n);
+        for (int32_t v = 0; v < n; v++) if (!deg[v]) q.push_back(v);
+        for (size_t h = 0; h < q.size(); h++)
+            for (int64_t i = g->out_off[q[h]]; i < g->out_off[q[h] + 1]; i++)
+                if (--deg[g->dst[g->out_edges[i]]] == 0) q.push_back(g->dst[g->out_edges[i]]);
+        if ((int32_t)q.size() != n) return fail(PESTO_ECYCLE, "graph has a cycle");
+    }
+    {
+        int64_t total = 0;
+        for (int32_t v = 0; v < n; v++) {
+            total += g->p[v];
+            if (total >= kGuard40) return fail(PESTO_EOVERFLOW, "sum of compute times >= 2^40 ns");
+        }
+        g->worst_total = total;
+    }
+    g->beta0.assign((size_t)g->D * g->D, 0);
+    g->beta1.assign((size_t)g->D * g->D, 0);
+    g->link_set.assign((size_t)g->D * g->D, 0);
+    for (int32_t v = 0; v < n; v++)
+        if (popc32(g->allowed[v]) >= 2) g->movable.push_back(v);
+    const int P = g->planes;
+    g->fmask.assign(n, 0);
+    for (int32_t v = 0; v < n; v++)
+        for (int c = 0; c < (1 << P); c++)
+            if (c >= g->D || !((g->allowed[v] >> c) & 1)) g->fmask[v] |= (uint16_t)(1u << c);
+    if (g->device >= 0) {
+        DeviceGuard guard(g->device);
+        cudaError_t e = cudaDeviceGetAttribute(&g->sms, cudaDevAttrMultiProcessorCount, g->device);
+        if (e != cudaSuccess) return cuda_fail(e, "query device");
+        if ((e = upload_vec(g->d_fmask, g->fmask)) != cudaSuccess) return cuda_fail(e, "upload");
+        if ((e = upload_vec(g->d_movable, g->movable)) != cudaSuccess) return cuda_fail(e, "upload");
+        if ((e = upload_vec(g->d_allowed, g->allowed)) != cudaSuccess) return cuda_fail(e, "upload");
+    }
+    *out = g.release();
+    return PESTO_OK;
+}
+
+void pesto_graph_destroy(pesto_graph *g) {
+    if (!g) return;
+    DeviceGuard guard(g->device);
+    delete g;
+}
+
+pesto_status pesto_comm_model(pesto_graph *g, int32_t a, int32_t b, int64_t beta0,
+                              int64_t beta1) {
+    if (!g) return fail(PESTO_EINVAL, "NULL graph");
+    if (beta0 < 0 || beta1 < 0) return fail(PESTO_EINVAL, "negative comm coefficient");
+    if (a < -1 || a >= g->D || b < -1 || b >= g->D) return fail(PESTO_EINVAL, "device out of range");
+    if (a >= 0 && a == b) return fail(PESTO_EINVAL, "a link joins two different devices");
+    std::vector<int64_t> b0 = g->beta0, b1 = g->beta1;
+    std::vector<uint8_t> set = g->link_set;
+    for (int x = 0; x < g->D; x++)
+        for (int y = 0; y < g->D; y++) {
+            if (x == y || (a >= 0 && x != a) || (b >= 0 && y != b)) continue;
+            b0[x * g->D + y] = beta0;
+            b1[x * g->D + y] = beta1;
+            set[x * g->D + y] = 1;
+        }
+    const int64_t tot = worst_total(g, b0, b1, set);
+    if (tot < 0) return fail(PESTO_EOVERFLOW, "sum p + sum_e max_L t_e >= 2^40 ns");
+    g->beta0 = b0;
+    g->beta1 = b1;
+    g->link_set = set;
+    g->worst_total = tot;
+    g->comm_gen++;
+    return PESTO_OK;
+}
+
+pesto_status pesto_graph_stats_for(pesto_graph *g, const int32_t *order, pesto_graph_stats *st) {
+    if (!g || !st) return fail(PESTO_EINVAL, "NULL argument");
+    std::shared_ptr<Layout> L;
+    pesto_status s = build_layout(g, order, L, true);
+    if (s) return s;
+    st->n_ops = g->n;
+    st->n_devices = g->D;
+    st->n_edges = g->m;
+    st->live_slots = L->W;
+    st->n_tiles = (int32_t)L->tiles.size();
+    st->layout_bytes = (int64_t)(L->blob.size() + L->heavy.size());
+    int32_t mi = 0, mo = 0;
+    for (int32_t v = 0; v < g->n; v++) {
+        mi = std::max(mi, g->indeg[v]);
+        mo = std::max<int32_t>(mo, (int32_t)(g->out_off[v + 1] - g->out_off[v]));
+    }
+    st->max_in_degree = mi;
+    st->max_out_degree = mo;
+    st->link_classes = g->n_classes;
+    st->time32_exact = g->worst_total < (int64_t(1) << 31) ? 1 : 0;
+    return PESTO_OK;
+}
+
+pesto_status pesto_seed_order(pesto_graph *g, int32_t kind, uint64_t seed, int32_t *order_out) {
+    if (!g || !order_out) return fail(PESTO_EINVAL, "NULL argument");
+    const int32_t n = g->n;
+    std::vector<int32_t> deg(g->indeg);
+    std::vector<int32_t> out;
+    out.reserve(n);
+    if (kind == PESTO_ORDER_CRITICAL_PATH) {
+        // bottom level (longest path to a sink counting p only), then Kahn by max bottom level,
+        // ties by smaller op id: the critical-path list order of PAPER.md L98 (Fig. 2b)
+        std::vector<int32_t> topo;
+        {
+            std::vector<int32_t> d2(g->indeg);
+            for (int32_t v = 0; v < n; v++) if (!d2[v]) topo.push_back(v);
+            for (size_t h = 0; h < topo.size(); h++)
+                for (int64_t i = g->out_off[topo[h]]; i < g->out_off[topo[h] + 1]; i++)
+                    if (--d2[g->dst[g->out_edges[i]]] == 0) topo.push_back(g->dst[g->out_edges[i]]);
+        }
+        std::vector<int64_t> bl(n, 0);
+        for (int32_t k = n - 1; k >= 0; k--) {
+            const int32_t v = topo[k];
+            int64_t best = 0;
+            for (int64_t i = g->out_off[v]; i < g->out_off[v + 1]; i++)
+                best = std::max(best, bl[g->dst[g->out_edges[i]]]);
+            bl[v] = g->p[v] + best;
+        }
+        auto cmp = [&](int32_t a, int32_t b) { return bl[a] != bl[b] ? bl[a] < bl[b] : a > b; };
+        std::priority_queue<int32_t, std::vector<int32_t>, decltype(cmp)> pq(cmp);
+        for (int32_t v = 0; v < n; v++) if (!deg[v]) pq.push(v);
+        while (!pq.empty()) {
+            const int32_t v = pq.top();
+            pq.pop();
+            out.push_back(v);
+            for (int64_t i = g->out_off[v]; i < g->out_off[v + 1]; i++)
+                if (--deg[g->dst[g->out_edges[i]]] == 0) pq.push(g->dst[g->out_edges[i]]);
+        }
+    } else if (kind == PESTO_ORDER_FIFO) {
+        for (int32_t v = 0; v < n; v++) if (!deg[v]) out.push_back(v);
+        for (size_t h = 0; h < out.size(); h++)
+            for (int64_t i = g->out_off[out[h]]; i < g->out_off[out[h] + 1]; i++)
+                if (--deg[g->dst[g->out_edges[i]]] == 0) out.push_back(g->dst[g->out_edges[i]]);
+    } else if (kind == PESTO_ORDER_RANDOM) {
+        // seeded random pick from the ready set: TF's default dispatch
+        uint64_t s = seed;
+        std::vector<int32_t> ready;
+        for (int32_t v = 0; v < n; v++) if (!deg[v]) ready.push_back(v);
+        while (!ready.empty()) {
+            const size_t i = (size_t)(splitmix_next(s) % ready.size());
+            const int32_t v = ready[i];
+            ready[i] = ready.back();
+            ready.pop_back();
+            out.push_back(v);
+            for (int64_t k = g->out_off[v]; k < g->out_off[v + 1]; k++)
+                if (--deg[g->dst[g->out_edges[k]]] == 0) ready.push_back(g->dst[g->out_edges[k]]);
+        }
+    } else {
+        return fail(PESTO_EINVAL, "unknown order kind");
+    }
+    std::copy(out.begin(), out.end(), order_out);
+    return PESTO_OK;
+}
+
+pesto_status pesto_seed_placement(pesto_graph *g, int32_t kind, const int32_t *order,
+                                  const int32_t *layer, uint64_t seed, uint8_t *x) {
+    if (!g || !x) return fail(PESTO_EINVAL, "NULL argument");
+    const int32_t n = g->n, D = g->D;
+    auto lowest = [&](int32_t v) {
+        for (int d = 0; d < D; d++) if ((g->allowed[v] >> d) & 1) return d;
+        return 0;
+    };
+    auto fix = [&](int32_t v, int d) { return ((g->allowed[v] >> d) & 1) ? d : lowest(v); };
+    if (kind == PESTO_PLACE_SINGLE) {
+        for (int32_t v = 0; v < n; v++) x[v] = (uint8_t)lowest(v);
+    } else if (kind == PESTO_PLACE_EXPERT) {
+        // contiguous layers per device ("Expert"): floor(layer * D / n_layers)
+        if (!layer) return fail(PESTO_EINVAL, "EXPERT needs layer tags");
+        int32_t nl = 0;
+        for (int32_t v = 0; v < n; v++) {
+            if (layer[v] < 0) return fail(PESTO_EINVAL, "negative layer tag");
+            nl = std::max(nl, layer[v] + 1);
+        }
+        for (int32_t v = 0; v < n; v++)
+            x[v] = (uint8_t)fix(v, (int)((int64_t)layer[v] * D / nl));
+    } else if (kind == PESTO_PLACE_TOPO_SPLIT) {
+        // pi cut into D contiguous segments of about equal sum p (mTOPO-like)
+        if (!order) return fail(PESTO_EINVAL, "TOPO_SPLIT needs an order");
+        int64_t total = 0;
+        for (int32_t v = 0; v < n; v++) total += g->p[v];
+        int64_t before = 0;
+        for (int32_t k = 0; k < n; k++) {
+            const int32_t v = order[k];
+            if (v < 0 || v >= n) return fail(PESTO_EINVAL, "order entry out of range");
+            int d;
+            if (total > 0) d = (int)(((__int128)(2 * before + g->p[v]) * D) / (2 * (__int128)total));
+            else d = (int)((int64_t)k * D / n);
+            x[v] = (uint8_t)fix(v, std::min(d, D - 1));
+            before += g->p[v];
+        }
+    } else if (kind == PESTO_PLACE_RANDOM) {
+        uint64_t s = seed;
+        for (int32_t v = 0; v < n; v++) {
+            const int na = popc32(g->allowed[v]);
+            int pick = (int)(splitmix_next(s) % (uint64_t)na);
+            for (int d = 0; d < D; d++)
+                if ((g->allowed[v] >> d) & 1) {
+                    if (pick == 0) { x[v] = (uint8_t)d; break; }
+                    pick--;
+                }
+        }
+    } else {
+        return fail(PESTO_EINVAL, "unknown placement kind");
+    }
+    return PESTO_OK;
+}
+
+pesto_status pesto_eval_batch(pesto_graph *g, const int32_t *order, const void *placements,
+                              int64_t stride, int64_t n_cand, int64_t *makespans, void *stream) {
+    if (!g) return fail(PESTO_EINVAL, "NULL graph");
+    if (g->device < 0) return fail(PESTO_ESTATE, "host-only graph handle");
+    if (n_cand < 0) return fail(PESTO_EINVAL, "n_cand < 0");
+    const int64_t row_bytes = ((int64_t)g->n * g->planes + 7) / 8;
+    if (stride < row_bytes || stride % 16) return fail(PESTO_EINVAL, "row_stride_bytes must be >= ceil(n*b/8) and a multiple of 16");
+    if (n_cand == 0) return PESTO_OK;
+    if (!placements || !makespans) return fail(PESTO_EINVAL, "NULL buffer");
+    if ((reinterpret_cast<uintptr_t>(placements) & 15) != 0) return fail(PESTO_EINVAL, "placements must be 16-byte aligned");
+    DeviceGuard guard(g->device);
+    std::shared_ptr<Layout> L;
+    pesto_status s = build_layout(g, order, L, true);
+    if (s) return s;
+    if ((s = upload_layout(g, *L))) return s;
+    cudaStream_t st = (cudaStream_t)stream;
+    const int64_t n_groups = (n_cand + 31) / 32;
+    cudaError_t e = g->d_planes.ensure((size_t)n_groups * g->n * g->planes * 4);
+    if (e != cudaSuccess) return cuda_fail(e, "allocate bit-sliced placements");
+    if ((e = g->d_invalid.ensure((size_t)n_groups * 4)) != cudaSuccess) return cuda_fail(e, "allocate");
+    TransposeParams tp{};
+    tp.rows = static_cast<const uint8_t *>(placements);
+    tp.stride = stride;
+    tp.n_cand = n_cand;
+    tp.n_groups = n_groups;
+    tp.n = g->n;
+    tp.planes = g->planes;
+    tp.pos_of = L->d_pos.as<int32_t>();
+    tp.fmask = g->d_fmask.as<uint16_t>();
+    tp.planes_out = g->d_planes.as<uint32_t>();
+    tp.invalid_out = g->d_invalid.as<uint32_t>();
+    if ((e = launch_transpose(tp, st)) != cudaSuccess) return cuda_fail(e, "launch transpose");
+    EvalParams p;
+    fill_eval_common(g, p);
+    p.stage_bytes = L->stage_bytes;
+    p.max_W = L->W;
+    p.planes_in = g->d_planes.as<uint32_t>();
+    p.invalid = g->d_invalid.as<uint32_t>();
+    p.n_cand = n_cand;
+    p.makespans = makespans;
+    p.bases = L->d_view.as<BaseLayoutDev>();
+    p.group_begin = 0;
+    p.groups_per_base = n_groups;
+    p.tasks_per_base = (n_groups + kWarps - 1) / kWarps;
+    p.n_tasks = p.tasks_per_base;
+    int grid = 0;
+    if ((s = ensure_state(g, p, 0, p.n_tasks, &grid))) return s;
+    p.state = g->d_state.as<int64_t>();
+    if ((e = launch_eval(p, 0, grid, st)) != cudaSuccess) return cuda_fail(e, "launch eval");
+    return PESTO_OK;
+}
+
+pesto_status pesto_eval_batch_host(pesto_graph *g, const int32_t *order, const void *rows,
+                                   int64_t stride, int64_t n_cand, int64_t *mk_host, void *stream) {
+    if (!g) return fail(PESTO_EINVAL, "NULL graph");
+    if (g->device < 0) return fail(PESTO_ESTATE, "host-only graph handle");
+    if (n_cand <= 0) return n_cand == 0 ? PESTO_OK : fail(PESTO_EINVAL, "n_cand < 0");
+    if (!rows || !mk_host) return fail(PESTO_EINVAL, "NULL buffer");
+    DeviceGuard guard(g->device);
+    cudaStream_t st = (cudaStream_t)stream;
+    cudaError_t e = g->d_rows.ensure((size_t)n_cand * stride);
+    if (e != cudaSuccess) return cuda_fail(e, "allocate rows");
+    if ((e = g->d_out.ensure((size_t)n_cand * 8)) != cudaSuccess) return cuda_fail(e, "allocate out");
+    if ((e = cudaMemcpyAsync(g->d_rows.ptr, rows, (size_t)n_cand * stride, cudaMemcpyHostToDevice, st)) != cudaSuccess)
+        return cuda_fail(e, "copy rows in");
+    pesto_status s = pesto_eval_batch(g, order, g->d_rows.ptr, stride, n_cand, g->d_out.as<int64_t>(), stream);
+    if (s) return s;
+    if ((e = cudaMemcpyAsync(mk_host, g->d_out.ptr, (size_t)n_cand * 8, cudaMemcpyDeviceToHost, st)) != cudaSuccess)
+        return cuda_fail(e, "copy makespans out");
+    if ((e = cudaStreamSynchronize(st)) != cudaSuccess) return cuda_fail(e, "eval_batch_host");
+    return PESTO_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,115 @@
+// host.h -- host-side structures of libpesto (product code).
+#pragma once
+#include <cuda_runtime.h>
+
+#include <cstdint>
+#include <list>
+#include <memory>
+#include <string>
+#include <vector>
+
+#include "internal.h"
+#include "pesto.h"
+
+namespace pesto {
+
+void set_error(const std::string &msg);
+pesto_status fail(pesto_status s, const std::string &msg);
+pesto_status cuda_fail(cudaError_t e, const char *what);
+int64_t launch_count_value();
+
+// RAII device buffer
+struct DevBuf {
+    void *ptr = nullptr;
+    size_t bytes = 0;
+    DevBuf() = default;
+    DevBuf(const DevBuf &) = delete;
+    DevBuf &operator=(const DevBuf &) = delete;
+    ~DevBuf() { release(); }
+    void release() {
+        if (ptr) cudaFree(ptr);
+        ptr = nullptr;
+        bytes = 0;
+    }
+    cudaError_t ensure(size_t want) {          // grow-only, contents not preserved
+        if (want <= bytes && ptr) return cudaSuccess;
+        release();
+        cudaError_t e = cudaMalloc(&ptr, want ? want : 16);
+        if (e == cudaSuccess) bytes = want ? want : 16;
+        else ptr = nullptr;
+        return e;
+    }
+    template <class T> T *as() const { return static_cast<T *>(ptr); }
+};
+
+// Position-space layout of one schedule order.
+struct Layout {
+    std::vector<int32_t> order, pos;
+    int32_t W = 0;                      // live ready-time slots (padded intervals)
+    int32_t stage_bytes = 0;            // largest tile (incl. header)
+    std::vector<uint8_t> blob, heavy;   // record stream (tiles) and out-of-line edges
+    std::vector<TileDesc> tiles;
+    std::vector<uint8_t> adj_next, allowed_pos;
+    int64_t comm_gen = -1;
+    // device copies
+    DevBuf d_blob, d_heavy, d_tiles, d_pos, d_adj, d_allowed_pos, d_view;
+    bool on_device = false;
+};
+
+}  // namespace pesto
+
+struct pesto_graph {
+    int32_t n = 0, D = 1, planes = 1, words = 0;
+    int64_t m = 0;
+    int32_t device = -1;
+    std::vector<int64_t> p, bytes;
+    std::vector<int32_t> src, dst;
+    std::vector<uint8_t> allowed;         // always filled (full mask when the caller gave NULL)
+    bool all_allowed = true;
+    std::vector<int64_t> out_off;         // CSR of out-edges by producer (edge ids)
+    std::vector<int64_t> out_edges;
+    std::vector<int32_t> indeg;
+    // comm model per directed link a*D+b
+    std::vector<int64_t> beta0, beta1;
+    std::vector<uint8_t> link_set;
+    int64_t comm_gen = 0;
+    // derived from the comm model
+    int32_t n_classes = 0;
+    uint8_t link_class[64] = {0};
+    std::vector<int64_t> t_class;         // [m][n_classes]
+    int64_t t_gen = -1;
+    int64_t worst_total = 0;              // sum p + sum_e max_L t_e
+    // movable ops (>= 2 allowed devices), ascending id; forbidden-code masks
+    std::vector<int32_t> movable;
+    std::vector<uint16_t> fmask;
+    // layout cache (most recent first)
+    std::list<std::shared_ptr<pesto::Layout>> cache;
+    // device buffers
+    pesto::DevBuf d_state, d_planes, d_invalid, d_fmask, d_movable, d_allowed, d_bases, d_rows,
+        d_out;
+    int32_t sms = 148;
+};
+
+namespace pesto {
+// graph.cpp helpers used by search.cpp
+pesto_status ensure_comm_tables(pesto_graph *g);
+pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<Layout> &out,
+                          bool use_cache);
+pesto_status upload_layout(pesto_graph *g, Layout &L);
+BaseLayoutDev layout_view(const Layout &L);
+void fill_eval_common(const pesto_graph *g, EvalParams &p);
+pesto_status ensure_state(pesto_graph *g, const EvalParams &p, int search_mode, int64_t n_tasks,
+                          int *grid_out);
+struct DeviceGuard {
+    int prev = -1;
+    explicit DeviceGuard(int dev) {
+        cudaGetDevice(&prev);
+        if (dev >= 0 && dev != prev) cudaSetDevice(dev);
+    }
+    ~DeviceGuard() {
+        int cur = -1;
+        cudaGetDevice(&cur);
+        if (prev >= 0 && cur != prev) cudaSetDevice(prev);
+    }
+};
+}  // namespace pesto

@@ -1,0 +1,89 @@
+// internal.h -- product-internal declarations shared by the host code and the CUDA kernels.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "layout_format.h"
+
+namespace pesto {
+
+constexpr int kWarps = 8;            // consumer warps per CTA (each = 32 candidates)
+constexpr int kStages = 4;           // TMA tile ring depth
+constexpr int kTileTarget = 8192;    // record bytes per tile (a single op may exceed it)
+constexpr int kTileHeader = 16;      // {pos_begin, pos_end, bytes, 0} at the head of each tile
+
+// One schedule order's layout on the device (the eval path uses one, the search one per base).
+struct BaseLayoutDev {
+    const uint8_t *blob;        // tiles, each = 16-byte header + records
+    const TileDesc *tiles;
+    const uint8_t *heavy;       // out-of-line edge records of high fan-out ops
+    const int32_t *pos_of;      // [n] op id -> position
+    const uint8_t *allowed_pos; // [n] device mask by position
+    const uint8_t *adj_next;    // [n] 1 if an edge joins order[k] -> order[k+1]
+    const uint32_t *bits;       // search: base placement, [planes][words] bit planes, by position
+    int32_t n_tiles;
+    int32_t W;                  // live ready-time slots
+};
+
+struct EvalParams {
+    int32_t n, D, planes, words;        // planes = bits per device code; words = ceil(n/32)
+    int32_t edge_stride, n_classes;
+    uint8_t link_class[64];             // class of directed link a*D+b
+    int32_t stage_bytes;                // per-stage smem bytes (>= largest tile)
+    int32_t all_allowed;
+    // ready-time slot state: [cta][warp][W_max][32] int64
+    int64_t *state;
+    int32_t max_W;
+    // explicit-placement mode
+    const uint32_t *planes_in;          // [group][pos][planes] bit-sliced codes
+    const uint32_t *invalid;            // [group] lanes with an infeasible row
+    int64_t n_cand;
+    int64_t *makespans;
+    // search mode
+    const BaseLayoutDev *bases;         // [P_local]
+    int32_t b_offset, P_total;          // real base id = b_offset + local
+    int64_t j_begin, j_end;             // candidate ids this launch covers (per base)
+    uint64_t seed, step;
+    int32_t mix[4];
+    const int32_t *movable;
+    int32_t n_movable;
+    const uint8_t *allowed_op;          // [n] by op id
+    uint64_t *keys;                     // [P_local] atomicMin targets
+    uint64_t *keys_dbg;                 // nullable: key of every candidate in [j_begin, j_end)
+    // work decomposition
+    int64_t group_begin, groups_per_base, tasks_per_base, n_tasks;
+};
+
+struct TransposeParams {
+    const uint8_t *rows;
+    int64_t stride, n_cand, n_groups;
+    int32_t n, planes;
+    const int32_t *pos_of;
+    const uint16_t *fmask;              // [n] forbidden device codes per op (bit c = code c)
+    uint32_t *planes_out;
+    uint32_t *invalid_out;
+};
+
+struct CommitParams {
+    const BaseLayoutDev *bases;         // [P]
+    uint32_t *bits;                     // [P][planes][words] (writable view of bases[b].bits)
+    int32_t n, D, planes, words, P;
+    uint64_t seed, step;
+    int32_t mix[4];
+    const int32_t *movable;
+    int32_t n_movable;
+    const uint8_t *allowed_op;
+    const uint64_t *keys;
+    int64_t *base_mk;
+    int32_t *swap_out;                  // [P] committed swap position or -1
+};
+
+// launchers (kernels.cu); they return the launch error, if any
+cudaError_t launch_eval(const EvalParams &p, int search_mode, int grid, cudaStream_t st);
+cudaError_t launch_transpose(const TransposeParams &p, cudaStream_t st);
+cudaError_t launch_commit(const CommitParams &p, cudaStream_t st);
+int eval_smem_bytes(const EvalParams &p, int search_mode);
+int eval_max_ctas_per_sm(const EvalParams &p, int search_mode);
+void note_launch();
+
+}  // namespace pesto

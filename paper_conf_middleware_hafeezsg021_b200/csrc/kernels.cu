@@ -1,0 +1,696 @@
+// kernels.cu -- sm_100a kernels of the Pesto hot path (product code).
+//
+//   K1 eval_kernel      makespan of 32 candidates per warp (one lane = one candidate), the DAG
+//                       record stream TMA-staged (cp.async.bulk + mbarrier ring) into shared
+//                       memory and shared by every warp of the CTA; neighbour moves (K2) decoded
+//                       in the prologue; warp argmin + atomicMin epilogue (K3).
+//   K5 transpose_kernel explicit placement rows -> bit-sliced [group][pos][plane] words.
+//   K4 commit_kernel    apply each base's winning move.
+//
+// What K1 computes per lane is PAPER.md's objective for one (placement, order) candidate:
+// ops run in pi order per device with no overlap (L146, L279, L374), an op starts after every
+// input arrived (L144), a cross-device input arrives after its transfer, which waits for the
+// directed link in FCFS order (L144, L188-198) and takes t_e = beta0 + beta1*bytes (L138);
+// makespan = max completion (L159-162 eq. (3)).  Recursion:
+//   S_v = max(max_in arrival, dev_free[x_v]);  C_v = S_v + p_v;  dev_free[x_v] = C_v
+//   cross e=(v,w): A_e = max(C_v, link_free[x_v->x_w]) + t_e;  link_free[..] = A_e
+//   arrival pushed (max) into w's ready-time slot, read when w is processed.
+#include <algorithm>
+#include <cstdio>
+#include <type_traits>
+
+#include "internal.h"
+#include "moves.cuh"
+
+namespace pesto {
+namespace {
+
+constexpr int64_t kInf64 = INT64_MAX;
+
+__device__ __forceinline__ uint32_t su32(const void *p) {
+    return (uint32_t)__cvta_generic_to_shared(p);
+}
+__device__ __forceinline__ void mbar_init(uint64_t *bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(su32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_fence_init() {
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t *bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(su32(bar)),
+                 "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(su32(bar)) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
+    uint32_t ok = 0;
+    while (!ok) {
+        asm volatile(
+            "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n"
+            " selp.u32 %0, 1, 0, p;\n}\n"
+            : "=r"(ok) : "r"(su32(bar)), "r"(parity) : "memory");
+    }
+}
+// one TMA bulk copy global -> shared, completion counted on `bar` (bytes % 16 == 0)
+__device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t bytes, uint64_t *bar) {
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+        ::"r"(su32(dst)), "l"(src), "r"(bytes), "r"(su32(bar)) : "memory");
+}
+
+// ---------------------------------------------------------------------------------------------
+// per-lane device / link state
+// ---------------------------------------------------------------------------------------------
+struct RegState {            // D <= 2: two devices, two directed links, in registers
+    int64_t d0, d1, l01, l10;
+    __device__ void init(int) { d0 = d1 = l01 = l10 = 0; }
+    __device__ int64_t dev(int x) const { return x ? d1 : d0; }
+    __device__ void set_dev(int x, int64_t v) { if (x) d1 = v; else d0 = v; }
+    __device__ int64_t link(int x, int) const { return x ? l10 : l01; }
+    __device__ void set_link(int x, int, int64_t v) { if (x) l10 = v; else l01 = v; }
+    __device__ int64_t makespan(int) const { return max(d0, d1); }
+};
+
+struct SmemState {           // D <= 8: [slot][lane] columns in shared memory
+    int64_t *d;              // [D][32] + lane
+    int64_t *l;              // [D*D][32] + lane
+    int D;
+    __device__ void init(int) {
+        for (int x = 0; x < D; x++) d[x * 32] = 0;
+        for (int x = 0; x < D * D; x++) l[x * 32] = 0;
+    }
+    __device__ int64_t dev(int x) const { return d[x * 32]; }
+    __device__ void set_dev(int x, int64_t v) { d[x * 32] = v; }
+    __device__ int64_t link(int x, int y) const { return l[(x * D + y) * 32]; }
+    __device__ void set_link(int x, int y, int64_t v) { l[(x * D + y) * 32] = v; }
+    __device__ int64_t makespan(int) const {
+        int64_t m = 0;
+        for (int x = 0; x < D; x++) m = max(m, d[x * 32]);
+        return m;
+    }
+};
+
+// ---------------------------------------------------------------------------------------------
+// placement sources: each lane's device code for any position q (q is warp-uniform)
+// ---------------------------------------------------------------------------------------------
+template <int PL>
+__device__ __forceinline__ int base_dev_at(const uint32_t *bits, int words, int32_t q) {
+    int x = 0;
+#pragma unroll
+    for (int k = 0; k < PL; k++) x |= (int)((__ldg(bits + k * words + (q >> 5)) >> (q & 31)) & 1u) << k;
+    return x;
+}
+
+template <int MODE, int PL>
+struct Placement {
+    // explicit rows (MODE 0): bit-sliced words of this warp's 32 candidates
+    const uint32_t *pl;
+    // search (MODE 1): base bits + warp-private "touched" bitmap + this lane's move
+    const uint32_t *bits;
+    const uint32_t *touched;
+    const uint8_t *allowed_pos;
+    int words;
+    int all_allowed;
+    LaneMove mv;
+    int lane;
+
+    __device__ __forceinline__ int operator()(int32_t q) const {
+        if (MODE == 0) {
+            if (PL == 1) return (int)((__ldg(pl + q) >> lane) & 1u);
+            if (PL == 2) {
+                uint2 w = __ldg(reinterpret_cast<const uint2 *>(pl) + q);
+                return (int)(((w.x >> lane) & 1u) | (((w.y >> lane) & 1u) << 1));
+            }
+            uint4 w = __ldg(reinterpret_cast<const uint4 *>(pl) + q);
+            return (int)(((w.x >> lane) & 1u) | (((w.y >> lane) & 1u) << 1) |
+                         (((w.z >> lane) & 1u) << 2) | (((w.w >> lane) & 1u) << 3));
+        } else {
+            int x = base_dev_at<PL>(bits, words, q);
+            if ((touched[q >> 5] >> (q & 31)) & 1u) {          // warp-uniform branch
+                unsigned aq = all_allowed ? 0xFFu : (unsigned)__ldg(allowed_pos + q);
+                x = apply_lane(mv, q, x, aq);
+            }
+            return x;
+        }
+    }
+};
+
+// ---------------------------------------------------------------------------------------------
+// the relaxation of one op and its pushes
+// ---------------------------------------------------------------------------------------------
+struct Ctx {
+    int64_t *R;                  // this lane's ready-time slots: R[slot * 32]
+    const uint8_t *lclass;       // shared-memory copy of the link-class table
+    int edge_stride;
+    int D;
+};
+
+template <bool GLOBAL>
+__device__ __forceinline__ uint4 load_rec(const uint8_t *p) {
+    if (GLOBAL) return __ldg(reinterpret_cast<const uint4 *>(p));
+    return *reinterpret_cast<const uint4 *>(p);
+}
+
+template <bool MULTI, bool GLOBAL, bool ALL_MAX, class PlaceT, class StateT>
+__device__ __forceinline__ void push_edge(const uint8_t *ep, const uint4 rec, int x, int64_t c,
+                                          const PlaceT &place, StateT &st, const Ctx &cx) {
+    const int64_t t0 = (int64_t)(((uint64_t)rec.y << 32) | rec.x);
+    const int32_t succ = (int32_t)rec.z;
+    const uint32_t sl = rec.w;
+    const int y = place(succ);
+    int64_t a = c;                                           // same device: C_v (L144)
+    if (y != x) {                                            // cross: FCFS link x -> y
+        int64_t t = t0;
+        if (MULTI) {
+            int cls = cx.lclass[x * cx.D + y];
+            if (cls) {
+                const int64_t *ext = reinterpret_cast<const int64_t *>(ep + 16) + (cls - 1);
+                t = GLOBAL ? (int64_t)__ldg(reinterpret_cast<const long long *>(ext)) : *ext;
+            }
+        }
+        a = max(c, st.link(x, y)) + t;
+        st.set_link(x, y, a);
+    }
+    int64_t *slot = cx.R + (int64_t)(sl & kEdgeSlotMask) * 32;
+    if (ALL_MAX || !(sl & kEdgeFirst)) a = max(a, *slot);
+    *slot = a;
+}
+
+// out-edges of one producer, in record order except that under an active swap (ks, ks+1) the
+// run of edges to ks+1 is pushed before the run to ks (the swapped order's consumer order).
+template <bool MULTI, bool GLOBAL, bool ALL_MAX, class PlaceT, class StateT>
+__device__ __forceinline__ void push_edges(const uint8_t *ep, uint32_t nout, int32_t ks, int x,
+                                           int64_t c, const PlaceT &place, StateT &st,
+                                           const Ctx &cx) {
+    const int es = cx.edge_stride;
+    for (uint32_t i = 0; i < nout;) {
+        const uint4 rec = load_rec<GLOBAL>(ep + (size_t)i * es);
+        if ((int32_t)rec.z != ks) {
+            push_edge<MULTI, GLOBAL, ALL_MAX>(ep + (size_t)i * es, rec, x, c, place, st, cx);
+            i++;
+            continue;
+        }
+        uint32_t a_end = i;
+        while (a_end < nout && (int32_t)load_rec<GLOBAL>(ep + (size_t)a_end * es).z == ks) a_end++;
+        uint32_t b_end = a_end;
+        while (b_end < nout && (int32_t)load_rec<GLOBAL>(ep + (size_t)b_end * es).z == ks + 1) b_end++;
+        for (uint32_t e = a_end; e < b_end; e++)
+            push_edge<MULTI, GLOBAL, ALL_MAX>(ep + (size_t)e * es, load_rec<GLOBAL>(ep + (size_t)e * es),
+                                              x, c, place, st, cx);
+        for (uint32_t e = i; e < a_end; e++)
+            push_edge<MULTI, GLOBAL, ALL_MAX>(ep + (size_t)e * es, load_rec<GLOBAL>(ep + (size_t)e * es),
+                                              x, c, place, st, cx);
+        i = b_end;
+    }
+}
+
+__device__ __forceinline__ const uint8_t *skip_op(const uint8_t *rp, int es) {
+    const OpRec op = *reinterpret_cast<const OpRec *>(rp);
+    if (op.nout & kOpHeavy) return rp + 32;
+    return rp + 16 + (size_t)(op.nout & kOpNoutMask) * es;
+}
+
+// relax the op whose record starts at rp (shared memory), at position v
+template <bool MULTI, bool ALL_MAX, class PlaceT, class StateT>
+__device__ __forceinline__ void relax_op(const uint8_t *rp, int32_t v, int32_t ks,
+                                         const uint8_t *heavy, const PlaceT &place, StateT &st,
+                                         const Ctx &cx) {
+    const OpRec op = *reinterpret_cast<const OpRec *>(rp);
+    const int x = place(v);
+    int64_t r = 0;
+    if (op.in_slot >= 0) r = cx.R[(int64_t)op.in_slot * 32];
+    const int64_t c = max(r, st.dev(x)) + op.p;              // S_v + p_v
+    st.set_dev(x, c);
+    if (!(op.nout & kOpHeavy)) {
+        push_edges<MULTI, false, ALL_MAX>(rp + 16, op.nout & kOpNoutMask, ks, x, c, place, st, cx);
+    } else {
+        const ExtRec ext = *reinterpret_cast<const ExtRec *>(rp + 16);
+        push_edges<MULTI, true, ALL_MAX>(heavy + ext.edge_off, (uint32_t)ext.nout, ks, x, c, place,
+                                         st, cx);
+    }
+}
+
+// zero the slots an op opens with a first push (swap pairs only; times are >= 0)
+__device__ __forceinline__ void clear_first_targets(const uint8_t *rp, const uint8_t *heavy,
+                                                    const Ctx &cx) {
+    const OpRec op = *reinterpret_cast<const OpRec *>(rp);
+    const uint8_t *ep;
+    uint32_t nout;
+    bool global = (op.nout & kOpHeavy) != 0;
+    if (global) {
+        const ExtRec ext = *reinterpret_cast<const ExtRec *>(rp + 16);
+        ep = heavy + ext.edge_off;
+        nout = (uint32_t)ext.nout;
+    } else {
+        ep = rp + 16;
+        nout = op.nout & kOpNoutMask;
+    }
+    for (uint32_t i = 0; i < nout; i++) {
+        uint4 rec = global ? load_rec<true>(ep + (size_t)i * cx.edge_stride)
+                           : load_rec<false>(ep + (size_t)i * cx.edge_stride);
+        if (rec.w & kEdgeFirst) cx.R[(int64_t)(rec.w & kEdgeSlotMask) * 32] = 0;
+    }
+}
+
+__device__ __forceinline__ uint64_t warp_min_u64(uint64_t v) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        uint64_t w = __shfl_xor_sync(0xffffffffu, v, o);
+        v = w < v ? w : v;
+    }
+    return v;
+}
+
+__device__ __forceinline__ uint8_t *align16(uint8_t *p) {
+    return reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(p) + 15) & ~uintptr_t(15));
+}
+
+// ---------------------------------------------------------------------------------------------
+// K1
+// ---------------------------------------------------------------------------------------------
+template <int MODE, int PL, bool MULTI>
+__global__ void __launch_bounds__((kWarps + 1) * 32)
+eval_kernel(const EvalParams P) {
+    extern __shared__ __align__(128) uint8_t smem[];
+    uint8_t *stage_buf = smem;
+    uint64_t *full = reinterpret_cast<uint64_t *>(smem + (size_t)kStages * P.stage_bytes);
+    uint64_t *empty = full + kStages;
+    uint8_t *cur = align16(reinterpret_cast<uint8_t *>(empty + kStages));
+    uint8_t *lclass = cur;
+    cur = align16(cur + 64);
+    uint32_t *touched_all = reinterpret_cast<uint32_t *>(cur);
+    if (MODE == 1) cur = align16(cur + (size_t)kWarps * P.words * 4);
+    int64_t *dstate = reinterpret_cast<int64_t *>(cur);
+
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < kStages; s++) {
+            mbar_init(&full[s], 1);
+            mbar_init(&empty[s], kWarps);
+        }
+        mbar_fence_init();
+    }
+    if (threadIdx.x < 64) lclass[threadIdx.x] = P.link_class[threadIdx.x];
+    __syncthreads();
+
+    if (warp == kWarps) {
+        // ---- producer: stream every task's tiles through the ring ----
+        if (lane == 0) {
+            uint32_t it = 0;
+            for (int64_t task = blockIdx.x; task < P.n_tasks; task += gridDim.x) {
+                const int bl = MODE ? (int)(task / P.tasks_per_base) : 0;
+                const BaseLayoutDev *B = &P.bases[bl];
+                const int nt = B->n_tiles;
+                for (int t = 0; t < nt; t++, it++) {
+                    const int s = it % kStages;
+                    if (it >= (uint32_t)kStages) mbar_wait(&empty[s], ((it / kStages) - 1) & 1);
+                    const TileDesc td = B->tiles[t];
+                    mbar_expect_tx(&full[s], (uint32_t)td.bytes);
+                    bulk_g2s(stage_buf + (size_t)s * P.stage_bytes, B->blob + td.byte_off,
+                             (uint32_t)td.bytes, &full[s]);
+                }
+            }
+        }
+        return;
+    }
+
+    // ---- consumers ----
+    Ctx cx;
+    cx.lclass = lclass;
+    cx.edge_stride = P.edge_stride;
+    cx.D = P.D;
+    cx.R = P.state + ((int64_t)(blockIdx.x * kWarps + warp) * P.max_W) * 32 + lane;
+    uint32_t *touched = touched_all + (size_t)warp * P.words;
+
+    using StateT = typename std::conditional<PL == 1, RegState, SmemState>::type;
+    StateT st;
+    if constexpr (PL != 1) {
+        st.D = P.D;
+        st.d = dstate + (size_t)warp * (P.D + P.D * P.D) * 32 + lane;
+        st.l = st.d + (size_t)P.D * 32;
+    }
+
+    uint32_t it = 0;
+    for (int64_t task = blockIdx.x; task < P.n_tasks; task += gridDim.x) {
+        const int bl = MODE ? (int)(task / P.tasks_per_base) : 0;
+        const int64_t local = MODE ? task % P.tasks_per_base : task;
+        const BaseLayoutDev *B = &P.bases[bl];
+        const int nt = B->n_tiles;
+        const uint8_t *heavy = B->heavy;
+        const int64_t g = P.group_begin + local * kWarps + warp;
+
+        Placement<MODE, PL> place;
+        place.lane = lane;
+        place.words = P.words;
+        place.all_allowed = P.all_allowed;
+        bool active, valid = true;
+        int64_t j = g * 32 + lane;
+        int32_t ks = -1;
+        if (MODE == 0) {
+            active = g * 32 < P.n_cand;
+            place.pl = P.planes_in + (size_t)g * P.n * PL;
+            if (active) valid = !((__ldg(P.invalid + g) >> lane) & 1u);
+        } else {
+            active = g < P.group_begin + P.groups_per_base;
+            const int breal = P.b_offset + bl;
+            const uint64_t cb = ctr_base_of(P.step, P.P_total, breal);
+            place.bits = B->bits;
+            place.touched = touched;
+            place.allowed_pos = B->allowed_pos;
+            const uint8_t *adj = B->adj_next;
+            ks = active ? decode_swap(P.seed, cb, g, P.n, P.mix[3],
+                                      [&](int32_t k) { return __ldg(adj + k) != 0; })
+                        : -1;
+            const bool in_range = active && j >= P.j_begin && j < P.j_end;
+            const int32_t *movable = P.movable;
+            const int32_t *pos_of = B->pos_of;
+            const uint32_t *bits = B->bits;
+            const uint8_t *aop = P.allowed_op;
+            const int words = P.words;
+            if (in_range) {
+                place.mv = decode_lane(
+                    P.seed, cb, j, ks >= 0 && lane == 0, P.n, P.D, P.mix, P.n_movable,
+                    [&](int32_t i) { return __ldg(movable + i); },
+                    [&](int32_t op) { return __ldg(pos_of + op); },
+                    [&](int32_t q) { return base_dev_at<PL>(bits, words, q); },
+                    [&](int32_t op) { return (unsigned)__ldg(aop + op); });
+            } else {
+                place.mv.kind = kMoveNone;
+                place.mv.nflip = 0;
+                place.mv.ws = place.mv.wl = place.mv.wd = 0;
+                for (int q = 0; q < 4; q++) { place.mv.fpos[q] = -1; place.mv.fdev[q] = 0; }
+            }
+            valid = in_range && place.mv.kind != kMoveInvalid;
+            if (place.mv.kind == kMoveInvalid) place.mv.kind = kMoveNone;
+            // warp-private bitmap of positions where any lane deviates from the base
+            for (int w = lane; w < P.words; w += 32) touched[w] = 0u;
+            __syncwarp();
+            if (place.mv.kind == kMoveFlip) {
+                for (int f = 0; f < place.mv.nflip; f++) {
+                    const int32_t q = place.mv.fpos[f];
+                    atomicOr(&touched[q >> 5], 1u << (q & 31));
+                }
+            } else if (place.mv.kind == kMoveWindow && place.mv.wl > 0) {
+                const int32_t a = place.mv.ws, e = place.mv.ws + place.mv.wl;   // [a, e)
+                for (int32_t w = a >> 5; w <= (e - 1) >> 5; w++) {
+                    const int32_t lo = max(a, w * 32) - w * 32, hi = min(e, w * 32 + 32) - w * 32;
+                    const uint32_t msk = (hi - lo == 32) ? 0xffffffffu : (((1u << (hi - lo)) - 1u) << lo);
+                    atomicOr(&touched[w], msk);
+                }
+            }
+            __syncwarp();
+        }
+        st.init(P.D);
+
+        bool skip_first = false;
+        for (int t = 0; t < nt; t++, it++) {
+            const int s = it % kStages;
+            mbar_wait(&full[s], (it / kStages) & 1);
+            if (active) {
+                const uint8_t *tile = stage_buf + (size_t)s * P.stage_bytes;
+                const int32_t pos_begin = reinterpret_cast<const int32_t *>(tile)[0];
+                const int32_t pos_end = reinterpret_cast<const int32_t *>(tile)[1];
+                const uint8_t *rp = tile + kTileHeader;
+                int32_t v = pos_begin;
+                if (skip_first) {
+                    rp = skip_op(rp, P.edge_stride);
+                    v++;
+                    skip_first = false;
+                }
+                while (v < pos_end) {
+                    if (v != ks) {
+                        relax_op<MULTI, false>(rp, v, ks, heavy, place, st, cx);
+                        rp = skip_op(rp, P.edge_stride);
+                        v++;
+                        continue;
+                    }
+                    // swapped pair: ops at ks+1 then ks
+                    const uint8_t *rk = rp;
+                    const uint8_t *rk1;
+                    const bool straddle = (v + 1 == pos_end);
+                    if (straddle) {
+                        const int s2 = (it + 1) % kStages;
+                        mbar_wait(&full[s2], ((it + 1) / kStages) & 1);
+                        rk1 = stage_buf + (size_t)s2 * P.stage_bytes + kTileHeader;
+                    } else {
+                        rk1 = skip_op(rk, P.edge_stride);
+                    }
+                    clear_first_targets(rk, heavy, cx);
+                    relax_op<MULTI, false>(rk1, v + 1, ks, heavy, place, st, cx);
+                    relax_op<MULTI, true>(rk, v, ks, heavy, place, st, cx);
+                    if (straddle) {
+                        skip_first = true;
+                        v = pos_end;
+                    } else {
+                        rp = skip_op(rk1, P.edge_stride);
+                        v += 2;
+                    }
+                }
+            }
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&empty[s]);
+        }
+
+        if (!active) continue;
+        const int64_t mk = st.makespan(P.D);                 // C_max = max_d dev_free[d]
+        if (MODE == 0) {
+            if (j < P.n_cand) P.makespans[j] = valid ? mk : kInf64;
+        } else {
+            uint64_t key = valid ? (((uint64_t)mk << 24) | (uint64_t)j) : ~0ull;
+            if (P.keys_dbg && j >= P.j_begin && j < P.j_end) P.keys_dbg[j - P.j_begin] = key;
+            key = warp_min_u64(key);
+            if (lane == 0 && key != ~0ull)
+                atomicMin(reinterpret_cast<unsigned long long *>(P.keys + bl),
+                          (unsigned long long)key);
+        }
+    }
+}
+
+// ---------------------------------------------------------------------------------------------
+// K5: rows of b-bit codes (op-id order) -> per group of 32 rows, [pos][plane] words whose bit l
+// is candidate l's bit; plus the mask of rows holding an infeasible code.
+// ---------------------------------------------------------------------------------------------
+__device__ __forceinline__ uint32_t compress2(uint32_t w) {  // even bits -> low 16
+    w &= 0x55555555u;
+    w = (w | (w >> 1)) & 0x33333333u;
+    w = (w | (w >> 2)) & 0x0F0F0F0Fu;
+    w = (w | (w >> 4)) & 0x00FF00FFu;
+    w = (w | (w >> 8)) & 0x0000FFFFu;
+    return w;
+}
+__device__ __forceinline__ uint32_t compress4(uint32_t w) {  // every 4th bit -> low 8
+    w &= 0x11111111u;
+    w = (w | (w >> 3)) & 0x03030303u;
+    w = (w | (w >> 6)) & 0x000F000Fu;
+    w = (w | (w >> 12)) & 0x000000FFu;
+    return w;
+}
+__device__ __forceinline__ uint32_t transpose32(uint32_t w, int lane) {
+    const uint32_t masks[5] = {0x0000FFFFu, 0x00FF00FFu, 0x0F0F0F0Fu, 0x33333333u, 0x55555555u};
+#pragma unroll
+    for (int s = 0; s < 5; s++) {
+        const int j = 16 >> s;
+        const uint32_t m = masks[s];
+        const uint32_t o = __shfl_xor_sync(0xffffffffu, w, j);
+        w = (lane & j) ? ((w & ~m) | ((o & ~m) >> j)) : ((w & m) | ((o & m) << j));
+    }
+    return w;
+}
+
+template <int PL>
+__global__ void __launch_bounds__(256) transpose_kernel(const TransposeParams P) {
+    const int lane = threadIdx.x & 31;
+    const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
+    for (int64_t g = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); g < P.n_groups;
+         g += warps) {
+        const int64_t row = g * 32 + lane;
+        const uint8_t *rp = P.rows + row * P.stride;
+        const bool have = row < P.n_cand;
+        uint32_t bad = 0;
+        const int chunks = (P.n + 31) >> 5;
+        for (int c = 0; c < chunks; c++) {
+            uint32_t pw[PL];
+            if (PL == 1) {
+                pw[0] = have ? __ldg(reinterpret_cast<const uint32_t *>(rp) + c) : 0u;
+            } else if (PL == 2) {
+                uint2 w = have ? __ldg(reinterpret_cast<const uint2 *>(rp) + c) : make_uint2(0, 0);
+                pw[0] = compress2(w.x) | (compress2(w.y) << 16);
+                pw[1] = compress2(w.x >> 1) | (compress2(w.y >> 1) << 16);
+            } else {
+                uint4 w = have ? __ldg(reinterpret_cast<const uint4 *>(rp) + c) : make_uint4(0, 0, 0, 0);
+#pragma unroll
+                for (int k = 0; k < PL; k++)
+                    pw[k] = compress4(w.x >> k) | (compress4(w.y >> k) << 8) |
+                            (compress4(w.z >> k) << 16) | (compress4(w.w >> k) << 24);
+            }
+#pragma unroll
+            for (int k = 0; k < PL; k++) pw[k] = transpose32(pw[k], lane);
+            const int op = c * 32 + lane;                     // lane now holds op's 32 codes
+            if (op < P.n) {
+                const unsigned fm = __ldg(P.fmask + op);
+                if (fm) {
+                    for (int code = 0; code < (1 << PL); code++) {
+                        if (!((fm >> code) & 1u)) continue;
+                        uint32_t match = 0xffffffffu;
+#pragma unroll
+                        for (int k = 0; k < PL; k++) match &= ((code >> k) & 1) ? pw[k] : ~pw[k];
+                        bad |= match;
+                    }
+                }
+                uint32_t *out = P.planes_out + ((size_t)g * P.n + __ldg(P.pos_of + op)) * PL;
+                if (PL == 1) out[0] = pw[0];
+                else if (PL == 2) *reinterpret_cast<uint2 *>(out) = make_uint2(pw[0], pw[1]);
+                else *reinterpret_cast<uint4 *>(out) = make_uint4(pw[0], pw[1], pw[2], pw[3]);
+            }
+        }
+        bad = __reduce_or_sync(0xffffffffu, bad);
+        if (lane == 0) P.invalid_out[g] = bad;
+    }
+}
+
+// ---------------------------------------------------------------------------------------------
+// K4: commit the winner of every base (one thread per base)
+// ---------------------------------------------------------------------------------------------
+template <int PL>
+__device__ void set_dev_at(uint32_t *bits, int words, int32_t q, int x) {
+#pragma unroll
+    for (int k = 0; k < PL; k++) {
+        uint32_t *w = bits + k * words + (q >> 5);
+        const uint32_t m = 1u << (q & 31);
+        *w = ((x >> k) & 1) ? (*w | m) : (*w & ~m);
+    }
+}
+template <int PL>
+__device__ int get_dev_at(const uint32_t *bits, int words, int32_t q) {
+    int x = 0;
+#pragma unroll
+    for (int k = 0; k < PL; k++) x |= (int)((bits[k * words + (q >> 5)] >> (q & 31)) & 1u) << k;
+    return x;
+}
+
+template <int PL>
+__global__ void commit_kernel(const CommitParams P) {
+    const int b = threadIdx.x;
+    if (b >= P.P) return;
+    const uint64_t key = P.keys[b];
+    P.swap_out[b] = -1;
+    if (key == ~0ull) return;
+    P.base_mk[b] = (int64_t)(key >> 24);
+    const int64_t j = (int64_t)(key & ((1ull << 24) - 1));
+    if (j == 0) return;
+    const BaseLayoutDev &B = P.bases[b];
+    uint32_t *bits = P.bits + (size_t)b * PL * P.words;
+    const uint64_t cb = ctr_base_of(P.step, P.P, b);
+    const uint8_t *adj = B.adj_next;
+    const int32_t ks = decode_swap(P.seed, cb, j >> 5, P.n, P.mix[3],
+                                   [&](int32_t k) { return adj[k] != 0; });
+    const int words = P.words;
+    const LaneMove mv = decode_lane(
+        P.seed, cb, j, ks >= 0 && (j & 31) == 0, P.n, P.D, P.mix, P.n_movable,
+        [&](int32_t i) { return P.movable[i]; }, [&](int32_t op) { return B.pos_of[op]; },
+        [&](int32_t q) { return get_dev_at<PL>(bits, words, q); },
+        [&](int32_t op) { return (unsigned)P.allowed_op[op]; });
+    if (mv.kind == kMoveFlip) {
+        for (int f = 0; f < mv.nflip; f++) set_dev_at<PL>(bits, words, mv.fpos[f], mv.fdev[f]);
+    } else if (mv.kind == kMoveWindow) {
+        for (int32_t q = mv.ws; q < mv.ws + mv.wl; q++)
+            if ((B.allowed_pos[q] >> mv.wd) & 1u) set_dev_at<PL>(bits, words, q, mv.wd);
+    }
+    if (ks >= 0) {                       // ops at ks and ks+1 exchange positions
+        const int a = get_dev_at<PL>(bits, words, ks), c = get_dev_at<PL>(bits, words, ks + 1);
+        set_dev_at<PL>(bits, words, ks, c);
+        set_dev_at<PL>(bits, words, ks + 1, a);
+        P.swap_out[b] = ks;
+    }
+}
+
+template <int MODE, int PL, bool MULTI>
+cudaError_t launch_one(const EvalParams &p, int grid, cudaStream_t st) {
+    const int smem = eval_smem_bytes(p, MODE);
+    auto kern = eval_kernel<MODE, PL, MULTI>;
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    if (e != cudaSuccess) return e;
+    kern<<<grid, (kWarps + 1) * 32, smem, st>>>(p);
+    return cudaGetLastError();
+}
+
+template <int MODE, int PL, bool MULTI>
+int occupancy_one(const EvalParams &p) {
+    const int smem = eval_smem_bytes(p, MODE);
+    auto kern = eval_kernel<MODE, PL, MULTI>;
+    if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) != cudaSuccess)
+        return 0;
+    int n = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kern, (kWarps + 1) * 32, smem) != cudaSuccess)
+        return 0;
+    return n;
+}
+
+int planes_of(int D) { return D <= 2 ? 1 : (D <= 4 ? 2 : 4); }
+
+}  // namespace
+
+static int64_t g_launches = 0;
+void note_launch() { __atomic_add_fetch(&g_launches, 1, __ATOMIC_RELAXED); }
+int64_t launch_count_value() { return __atomic_load_n(&g_launches, __ATOMIC_RELAXED); }
+
+int eval_smem_bytes(const EvalParams &p, int search_mode) {
+    size_t b = (size_t)kStages * p.stage_bytes + 2 * kStages * 8;
+    b = (b + 15) & ~size_t(15);
+    b += 64;
+    b = (b + 15) & ~size_t(15);
+    if (search_mode) b += (size_t)kWarps * p.words * 4;
+    b = (b + 15) & ~size_t(15);
+    if (planes_of(p.D) != 1) b += (size_t)kWarps * (p.D + p.D * p.D) * 32 * 8;
+    return (int)b + 128;
+}
+
+#define PESTO_DISPATCH(FN, ...)                                                            \
+    do {                                                                                   \
+        const int pl = planes_of(p.D);                                                     \
+        const bool multi = p.n_classes > 1;                                                \
+        if (search_mode) {                                                                 \
+            if (pl == 1) return multi ? FN<1, 1, true>(__VA_ARGS__) : FN<1, 1, false>(__VA_ARGS__); \
+            if (pl == 2) return multi ? FN<1, 2, true>(__VA_ARGS__) : FN<1, 2, false>(__VA_ARGS__); \
+            return multi ? FN<1, 4, true>(__VA_ARGS__) : FN<1, 4, false>(__VA_ARGS__);     \
+        } else {                                                                           \
+            if (pl == 1) return multi ? FN<0, 1, true>(__VA_ARGS__) : FN<0, 1, false>(__VA_ARGS__); \
+            if (pl == 2) return multi ? FN<0, 2, true>(__VA_ARGS__) : FN<0, 2, false>(__VA_ARGS__); \
+            return multi ? FN<0, 4, true>(__VA_ARGS__) : FN<0, 4, false>(__VA_ARGS__);     \
+        }                                                                                  \
+    } while (0)
+
+cudaError_t launch_eval(const EvalParams &p, int search_mode, int grid, cudaStream_t st) {
+    note_launch();
+    PESTO_DISPATCH(launch_one, p, grid, st);
+}
+
+int eval_max_ctas_per_sm(const EvalParams &p, int search_mode) {
+    PESTO_DISPATCH(occupancy_one, p);
+}
+
+cudaError_t launch_transpose(const TransposeParams &p, cudaStream_t st) {
+    note_launch();
+    int dev = 0, sms = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    const int64_t blocks_needed = (p.n_groups + 7) / 8;
+    const int grid = (int)std::min<int64_t>(blocks_needed, (int64_t)sms * 8);
+    if (grid <= 0) return cudaSuccess;
+    if (p.planes == 1) transpose_kernel<1><<<grid, 256, 0, st>>>(p);
+    else if (p.planes == 2) transpose_kernel<2><<<grid, 256, 0, st>>>(p);
+    else transpose_kernel<4><<<grid, 256, 0, st>>>(p);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_commit(const CommitParams &p, cudaStream_t st) {
+    note_launch();
+    const int threads = ((p.P + 31) / 32) * 32;
+    if (p.planes == 1) commit_kernel<1><<<1, threads, 0, st>>>(p);
+    else if (p.planes == 2) commit_kernel<2><<<1, threads, 0, st>>>(p);
+    else commit_kernel<4><<<1, threads, 0, st>>>(p);
+    return cudaGetLastError();
+}
+
+}  // namespace pesto

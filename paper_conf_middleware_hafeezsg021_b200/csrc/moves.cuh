@@ -1,0 +1,126 @@
+// moves.cuh -- counter-based neighbour moves of the local search (rows a2/a7).
+//
+// The search is the north star's method (not a PAPER.md method); it explores the two decision
+// variables of the Pesto problem: the placement x_i (L175, L208 for >2 devices) and the
+// schedule order (L171, L279).  Everything is integer and derived from the counter
+// (seed, step, base, candidate j, draw k), so any rank can regenerate any candidate.
+#pragma once
+#include <stdint.h>
+
+#ifdef __CUDACC__
+#define PESTO_HD __host__ __device__ __forceinline__
+#else
+#define PESTO_HD inline
+#endif
+
+namespace pesto {
+
+PESTO_HD uint64_t mix64(uint64_t z) {            // SplitMix64 finaliser
+    z ^= z >> 30; z *= 0xBF58476D1CE4E5B9ull;
+    z ^= z >> 27; z *= 0x94D049BB133111EBull;
+    z ^= z >> 31;
+    return z;
+}
+
+// draw_k(j) = mix64(seed ^ mix64(((step*P + b) * 2^24 + j) * 16 + k))
+PESTO_HD uint64_t draw(uint64_t seed, uint64_t ctr_base, int64_t j, int k) {
+    return mix64(seed ^ mix64((ctr_base + (uint64_t)j) * 16ull + (uint64_t)k));
+}
+PESTO_HD uint64_t ctr_base_of(uint64_t step, int P, int b) {
+    return (step * (uint64_t)P + (uint64_t)b) << 24;
+}
+
+PESTO_HD int popc32(unsigned v) {
+#ifdef __CUDA_ARCH__
+    return __popc(v);
+#else
+    return __builtin_popcount(v);
+#endif
+}
+
+enum MoveKind : int { kMoveNone = 0, kMoveFlip = 1, kMoveWindow = 2, kMoveInvalid = 3 };
+
+struct LaneMove {
+    int kind;
+    int nflip;
+    int32_t fpos[4];     // flipped positions (in the base order), applied in sequence
+    int32_t fdev[4];
+    int32_t ws, wl, wd;  // window: positions [ws, ws + wl) move to wd where allowed
+};
+
+// Group (warp) order move: adjacent swap of positions (k, k+1) of the base order, or -1.
+// adj_next(k) must say whether an edge joins order[k] -> order[k+1].
+template <class AdjNext>
+PESTO_HD int32_t decode_swap(uint64_t seed, uint64_t cb, int64_t group, int n, int swap_pct,
+                             AdjNext adj_next) {
+    if (group == 0 || swap_pct <= 0 || n < 2) return -1;
+    int64_t j0 = group * 32;
+    if ((int)(draw(seed, cb, j0, 15) % 100u) >= swap_pct) return -1;
+    int32_t k = (int32_t)(draw(seed, cb, j0, 14) % (uint64_t)(n - 1));
+    return adj_next(k) ? -1 : k;
+}
+
+// Lane placement move of candidate j.  Callbacks:
+//   movable(i) -> op id of the i-th movable op;  pos_of(op) -> position in the base order;
+//   base_dev(pos) -> base device at a position;  allowed(op) -> device mask.
+template <class Movable, class PosOf, class BaseDev, class Allowed>
+PESTO_HD LaneMove decode_lane(uint64_t seed, uint64_t cb, int64_t j, bool pure_swap, int n, int D,
+                              const int32_t mix[4], int n_movable, Movable movable, PosOf pos_of,
+                              BaseDev base_dev, Allowed allowed) {
+    LaneMove mv;
+    mv.kind = kMoveNone;
+    mv.nflip = 0;
+    mv.ws = 0; mv.wl = 0; mv.wd = 0;
+    for (int q = 0; q < 4; q++) { mv.fpos[q] = -1; mv.fdev[q] = 0; }
+    if (j == 0 || pure_swap) return mv;
+    int wsum = mix[0] + mix[1] + mix[2];
+    if (wsum <= 0) return mv;
+    int r = (int)(draw(seed, cb, j, 0) % (uint64_t)wsum);
+    if (r < mix[0] + mix[1]) {
+        if (n_movable == 0) { mv.kind = kMoveInvalid; return mv; }
+        int flips = 1;
+        if (r >= mix[0]) flips = 2 + (int)(draw(seed, cb, j, 1) % 3u);
+        mv.kind = kMoveFlip;
+        mv.nflip = flips;
+        for (int q = 0; q < flips; q++) {
+            int32_t op = movable((int32_t)(draw(seed, cb, j, 2 + 2 * q) % (uint64_t)n_movable));
+            int32_t pos = pos_of(op);
+            int cur = base_dev(pos);
+            for (int e = 0; e < q; e++)
+                if (mv.fpos[e] == pos) cur = mv.fdev[e];      // device after earlier flips
+            unsigned msk = allowed(op) & ((1u << D) - 1u) & ~(1u << cur);
+            int na = popc32(msk);
+            int pick = (int)(draw(seed, cb, j, 3 + 2 * q) % (uint64_t)na);
+            int dev = 0;
+            for (int d = 0; d < D; d++) {                      // pick-th set bit, ascending
+                if ((msk >> d) & 1u) {
+                    if (pick == 0) { dev = d; break; }
+                    pick--;
+                }
+            }
+            mv.fpos[q] = pos;
+            mv.fdev[q] = dev;
+        }
+    } else {
+        mv.kind = kMoveWindow;
+        int32_t s = (int32_t)(draw(seed, cb, j, 2) % (uint64_t)n);
+        int32_t len = 1 + (int32_t)(draw(seed, cb, j, 3) % 64u);
+        if (s + len > n) len = n - s;
+        mv.ws = s;
+        mv.wl = len;
+        mv.wd = (int32_t)(draw(seed, cb, j, 4) % (uint64_t)D);
+    }
+    return mv;
+}
+
+// device of position q under move mv (base device xb, op mask at q for the window check)
+PESTO_HD int apply_lane(const LaneMove &mv, int32_t q, int xb, unsigned allowed_q) {
+    int x = xb;
+    if ((uint32_t)(q - mv.ws) < (uint32_t)mv.wl && ((allowed_q >> mv.wd) & 1u)) x = mv.wd;
+#pragma unroll
+    for (int f = 0; f < 4; f++)
+        if (q == mv.fpos[f]) x = mv.fdev[f];
+    return x;
+}
+
+}  // namespace pesto

@@ -1,0 +1,198 @@
+"""CUDA path (through the C ABI) vs the CPU oracle, element by element, bit-exact (int64 ns).
+
+North star tolerance: "GPU makespans must match the oracle bit-exactly (all times are integer
+nanoseconds)" -- every comparison below is exact equality.
+"""
+
+import json
+import os
+
+import numpy as np
+import pytest
+
+from workloads import configs, dag
+
+pytestmark = pytest.mark.gpu
+
+GOLD = os.path.join(os.path.dirname(__file__), "golden")
+MIX = (50, 20, 20, 10)
+
+
+@pytest.fixture(scope="module")
+def P():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_middleware_hafeezsg021_b200 import pesto
+    return pesto
+
+
+def _gpu_eval(P, G, g, order, x):
+    import torch
+    rows = torch.from_numpy(dag.pack_placements(x, g.D)).cuda()
+    out = G.eval(order, rows)
+    torch.cuda.synchronize()
+    return out.cpu().numpy()
+
+
+def test_tiny12_exhaustive(P, O):
+    """all 4096 placements x 186 orders = 761,856 schedules, each bit-exact; min = optimum."""
+    g = dag.tiny12()
+    G = P.Graph.from_arrays(g)
+    xs = np.asarray([[(c >> i) & 1 for i in range(12)] for c in range(4096)], np.uint8)
+    best = None
+    for order in dag.all_linear_extensions(g):
+        gpu = _gpu_eval(P, G, g, order, xs)
+        ref, _ = O.makespan_batch(g, xs, np.asarray(order, np.int32))
+        assert (gpu == ref).all(), order
+        best = gpu.min() if best is None else min(best, gpu.min())
+    assert best == json.load(open(os.path.join(GOLD, "tiny12_optimum.json")))["optimum"]
+
+
+CASES = [
+    # (seed, n, avg_out, D, extra kwargs)
+    (1, 1, 0.0, 2, {}),
+    (2, 2, 1.0, 2, {}),
+    (3, 37, 1.5, 2, {}),
+    (4, 300, 1.6, 2, {"multi_frac": 0.2, "zero_frac": 0.3}),
+    (5, 2500, 1.5, 2, {"fan_in_hub": 1500}),                     # fan-in > 1024, many tiles
+    (6, 2000, 1.4, 2, {"fan_out_hub": 700}),                     # out-of-line edge records
+    (7, 400, 1.5, 3, {"allowed_frac": 0.4}),                      # D=3: invalid codes exist
+    (8, 800, 1.5, 4, {"hetero_links": True}),                     # several link classes
+    (9, 500, 1.5, 4, {"allowed_frac": 0.5, "hetero_links": True}),
+    (10, 300, 1.5, 8, {"hetero_links": True}),
+    (11, 3000, 1.7, 2, {"locality": 40}),
+    (12, 600, 1.5, 1, {}),
+]
+
+
+@pytest.mark.parametrize("case", CASES, ids=lambda c: f"seed{c[0]}_n{c[1]}_D{c[3]}")
+def test_random_dags(P, O, case):
+    seed, n, avg, D, kw = case
+    g = dag.random_dag(seed, n, avg, D=D, p_max=5000, max_bytes=400_000, beta0=700,
+                       beta1_fs=30_000, **kw)
+    G = P.Graph.from_arrays(g)
+    for s, n_cand in [(0, 1), (1, 33), (2, 517)]:          # ragged candidate counts
+        order = dag.random_topo_order(g, 100 + s)
+        x = dag.random_placements(g, 200 + s, n_cand)
+        if D == 3 or kw.get("allowed_frac"):
+            # include infeasible rows: codes >= D or disallowed devices
+            rng = np.random.default_rng(s)
+            bad = rng.random(n_cand) < 0.1
+            x[bad, 0] = (1 << (1 if D <= 2 else (2 if D <= 4 else 3))) - 1
+        gpu = _gpu_eval(P, G, g, order, x)
+        ref, _ = O.makespan_batch(g, x, order)
+        assert (gpu == ref).all(), (s, np.nonzero(gpu != ref)[0][:5], gpu[:3], ref[:3])
+
+
+@pytest.mark.parametrize("name", ["inception_v3_2dev", "nmt4_2dev_commheavy",
+                                  "transformer_2dev", "transformer_4dev_8gpu"])
+def test_full_size_sampled(P, O, name):
+    """full BASELINE-size graphs: 4096 candidates on the GPU, a sample checked one by one."""
+    cfg = configs.CONFIGS[name]
+    g = configs.graph_for(cfg)
+    G = P.Graph.from_arrays(g)
+    order = G.seed_order(P.ORDER_CRITICAL_PATH)
+    seeds = [G.seed_placement(P.PLACE_EXPERT, layer=g.layer),
+             G.seed_placement(P.PLACE_TOPO_SPLIT, order=order),
+             G.seed_placement(P.PLACE_SINGLE)]
+    x = np.concatenate([np.stack(seeds), dag.random_placements(g, 5, 4093)])
+    gpu = _gpu_eval(P, G, g, order, x)
+    idx = np.concatenate([np.arange(3), np.random.default_rng(1).choice(np.arange(3, 4096), 45,
+                                                                         replace=False)])
+    ref, _ = O.makespan_batch(g, x[idx], order)
+    assert (gpu[idx] == ref).all()
+    assert gpu[2] == int(g.p.sum())                           # single device = sum p
+
+
+def _search_graph(seed=21, n=150, D=2, allowed_frac=0.0):
+    g = dag.random_dag(seed, n, 1.5, D=D, p_max=3000, max_bytes=200_000, beta0=500,
+                       beta1_fs=25_000, allowed_frac=allowed_frac)
+    return g
+
+
+def _bases(g, P_, seed=0):
+    orders = np.stack([dag.random_topo_order(g, seed + b) for b in range(P_)]).astype(np.int32)
+    xs = dag.random_placements(g, seed + 50, P_)
+    return xs, orders
+
+
+@pytest.mark.parametrize("D,allowed_frac", [(2, 0.0), (4, 0.5)])
+def test_search_candidate_keys(P, O, D, allowed_frac):
+    g = _search_graph(D=D, allowed_frac=allowed_frac)
+    G = P.Graph.from_arrays(g)
+    xs, orders = _bases(g, 3)
+    K = 1500
+    S = P.Search(G, xs, orders, K, MIX, seed=99)
+    for b in range(3):
+        gk = S.candidate_keys(b, 0, K)
+        ok = O.candidate_keys(g, 3, b, xs, orders, 0, K, 99, 0, MIX)
+        assert (gk == ok).all(), (b, np.nonzero(gk != ok)[0][:5])
+    gk = S.candidate_keys(1, 77, 1013)                       # unaligned range
+    ok = O.candidate_keys(g, 3, 1, xs, orders, 77, 1013, 99, 0, MIX)
+    assert (gk == ok).all()
+
+
+def test_search_steps_match_reference(P, O):
+    g = _search_graph(seed=31, n=120)
+    G = P.Graph.from_arrays(g)
+    xs, orders = _bases(g, 4, seed=7)
+    K = 2048
+    mix = (40, 20, 20, 30)                                   # many swaps: exercise rebuilds
+    S = P.Search(G, xs, orders, K, mix, seed=5)
+    rx, ro = xs.copy(), orders.copy()
+    rmk = np.asarray([O.makespan(g, rx[b], ro[b]) for b in range(4)], np.int64)
+    for b in range(4):
+        assert S.get(b)[0] == rmk[b]
+    for step in range(6):
+        S.step()
+        keys = O.search_step(g, rx, ro, rmk, K, 5, step, mix)
+        for b in range(4):
+            mk, x, o = S.get(b)
+            assert mk == rmk[b] and (x == rx[b]).all() and (o == ro[b]).all(), (step, b)
+        assert S.step_count == step + 1
+        del keys
+
+
+def test_fake_sharding_equals_single_rank(P, O):
+    """W rank ranges evaluated one after another on one GPU, minima reduced on the host."""
+    g = _search_graph(seed=41, n=90)
+    G = P.Graph.from_arrays(g)
+    xs, orders = _bases(g, 2, seed=3)
+    K, W = 3000, 3
+    single = P.Search(G, xs, orders, K, MIX, seed=8)
+    shards = [P.Search(G, xs, orders, K, MIX, seed=8, rank=r, world=W) for r in range(W)]
+    for step in range(3):
+        single.eval()
+        k1 = single.keys()
+        per = []
+        for s in shards:
+            s.eval()
+            per.append(s.keys())
+        kmin = np.minimum.reduce(per)
+        assert (kmin == k1).all()
+        single.commit()
+        for s in shards:
+            s.set_keys(kmin)
+            s.commit()
+        for b in range(2):
+            a, s0 = single.get(b), shards[0].get(b)
+            assert a[0] == s0[0] and (a[1] == s0[1]).all() and (a[2] == s0[2]).all()
+
+
+def test_search_full_size_sampled(P, O):
+    """transformer_2dev at full size: a sample of search candidates checked one by one."""
+    cfg = configs.CONFIGS["transformer_2dev"]
+    g = configs.graph_for(cfg)
+    G = P.Graph.from_arrays(g)
+    order = G.seed_order(P.ORDER_CRITICAL_PATH)
+    xs = np.stack([G.seed_placement(P.PLACE_EXPERT, layer=g.layer),
+                   G.seed_placement(P.PLACE_TOPO_SPLIT, order=order)])
+    orders = np.stack([order, order])
+    S = P.Search(G, xs, orders, 1 << 20, MIX, seed=2021)
+    for b in range(2):
+        sample = [0, 1, 31, 32, 33, 4097, 65535, 524287, (1 << 20) - 1]
+        for j in sample:
+            gk = S.candidate_keys(b, j, j + 1)
+            ok = O.candidate_keys(g, 2, b, xs, orders, j, j + 1, 2021, 0, MIX)
+            assert (gk == ok).all(), (b, j)

@@ -121,7 +121,8 @@ def all_linear_extensions(g: Graph) -> List[List[int]]:
 # ---------------------------------------------------------------------------------------
 def random_dag(seed: int, n: int, avg_out: float = 1.5, D: int = 2, *, max_bytes: int = 1 << 20,
                p_max: int = 10_000, zero_frac: float = 0.1, multi_frac: float = 0.05,
-               fan_in_hub: int = 0, locality: int = 0, allowed_frac: float = 0.0,
+               fan_in_hub: int = 0, fan_out_hub: int = 0, locality: int = 0,
+               allowed_frac: float = 0.0,
                beta0: Optional[int] = None, beta1_fs: Optional[int] = None,
                hetero_links: bool = False) -> Graph:
     """Random DAG on n ops: a hidden random rank order; edges go from lower to higher rank.
@@ -129,6 +130,7 @@ def random_dag(seed: int, n: int, avg_out: float = 1.5, D: int = 2, *, max_bytes
     zero_frac: fraction of zero-duration ops and zero-byte edges.
     multi_frac: fraction of edges duplicated as multi-edges (Q4).
     fan_in_hub: if > 0, one op receives that many extra in-edges (fan-in > 32 / > 1024 cases).
+    fan_out_hub: if > 0, one op gets that many extra out-edges (out-of-line edge records).
     locality: if > 0, edge endpoints are at most `locality` ranks apart (long-lived slots rarer).
     allowed_frac: fraction of ops given a random non-full allowed-device mask.
     """
@@ -169,6 +171,13 @@ def random_dag(seed: int, n: int, avg_out: float = 1.5, D: int = 2, *, max_bytes
         for _ in range(fan_in_hub):
             a = r.below(n - 1)
             edges.append((rank[a], hub))
+            nb.append(r.log_uniform_int(1, max_bytes + 1))
+    if fan_out_hub > 0 and n > 2:
+        # the first op of the hidden order feeds fan_out_hub random later ops
+        hub = rank[0]
+        for _ in range(fan_out_hub):
+            b = 1 + r.below(n - 1)
+            edges.append((hub, rank[b]))
             nb.append(r.log_uniform_int(1, max_bytes + 1))
     allowed = None
     if allowed_frac > 0:
