@@ -114,17 +114,20 @@ struct Placement {
     int all_allowed;
     LaneMove mv;
     int lane;
+    int dmax;
 
     __device__ __forceinline__ int operator()(int32_t q) const {
         if (MODE == 0) {
             if (PL == 1) return (int)((__ldg(pl + q) >> lane) & 1u);
+            // codes >= D belong to rows K5 flagged infeasible; clamp so the discarded lane
+            // still indexes inside its state columns
             if (PL == 2) {
                 uint2 w = __ldg(reinterpret_cast<const uint2 *>(pl) + q);
-                return (int)(((w.x >> lane) & 1u) | (((w.y >> lane) & 1u) << 1));
+                return min((int)(((w.x >> lane) & 1u) | (((w.y >> lane) & 1u) << 1)), dmax);
             }
             uint4 w = __ldg(reinterpret_cast<const uint4 *>(pl) + q);
-            return (int)(((w.x >> lane) & 1u) | (((w.y >> lane) & 1u) << 1) |
-                         (((w.z >> lane) & 1u) << 2) | (((w.w >> lane) & 1u) << 3));
+            return min((int)(((w.x >> lane) & 1u) | (((w.y >> lane) & 1u) << 1) |
+                             (((w.z >> lane) & 1u) << 2) | (((w.w >> lane) & 1u) << 3)), dmax);
         } else {
             int x = base_dev_at<PL>(bits, words, q);
             if ((touched[q >> 5] >> (q & 31)) & 1u) {          // warp-uniform branch
@@ -342,6 +345,7 @@ eval_kernel(const EvalParams P) {
 
         Placement<MODE, PL> place;
         place.lane = lane;
+        place.dmax = P.D - 1;
         place.words = P.words;
         place.all_allowed = P.all_allowed;
         bool active, valid = true;
