@@ -15,9 +15,9 @@ CUDA = os.environ.get("CUDA_HOME", "/usr/local/cuda")
 NVCC = os.path.join(CUDA, "bin", "nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 
-CU_SOURCES = ["kernels.cu"]
+CU_SOURCES = ["kernels.cu", "eval32.cu"]
 CPP_SOURCES = ["graph.cpp", "search.cpp"]
-HEADERS = ["internal.h", "host.h", "layout_format.h", "moves.cuh"]
+HEADERS = ["internal.h", "host.h", "layout_format.h", "moves.cuh", "device_common.cuh"]
 
 
 def _stale() -> bool:

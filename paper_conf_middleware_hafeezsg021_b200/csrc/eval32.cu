@@ -1,0 +1,462 @@
+// eval32.cu -- K1 fast path: the makespan recursion in 32-bit saturating time (product code).
+//
+// Same recursion as eval64 (kernels.cu; PAPER.md L142-146, L188-198, L374 -- DESIGN.md §3):
+//   S_v = max(max_in arrival, dev_free[x_v]);  C_v = S_v + p_v;  dev_free[x_v] = C_v
+//   cross e=(v,w): A_e = max(C_v, link_free[x_v->x_w]) + t_e;  link_free = A_e
+// with the ready-time state split by producer distance:
+//   near (consumer within kNearDelta positions): the warp's shared-memory ring, slot = pos & 15
+//   far:  a global cold slot written with fire-and-forget STG (first push) / RED.MAX, and
+//         prefetched into L1 kPrefetchDist positions before the consumer reads it.
+// One lane = one candidate, 32 candidates per warp share every DAG tile, which the producer
+// warp streams into shared memory with cp.async.bulk (TMA) through an mbarrier ring.
+#include <algorithm>
+#include <type_traits>
+
+#include "device_common.cuh"
+#include "internal.h"
+
+namespace pesto {
+namespace {
+
+using namespace dev;
+
+__device__ __forceinline__ uint32_t add_sat(uint32_t a, uint32_t b) {
+    return min(a + b, kSat32);                 // a <= kSat32, b < kMaxDur32: never wraps
+}
+
+struct RegState32 {          // D <= 2
+    uint32_t d0, d1, l01, l10;
+    __device__ void init() { d0 = d1 = l01 = l10 = 0u; }
+    __device__ uint32_t dev(int x) const { return x ? d1 : d0; }
+    __device__ void set_dev(int x, uint32_t v) { if (x) d1 = v; else d0 = v; }
+    __device__ uint32_t link(int x, int) const { return x ? l10 : l01; }
+    __device__ void set_link(int x, int, uint32_t v) { if (x) l10 = v; else l01 = v; }
+    __device__ uint32_t makespan() const { return max(d0, d1); }
+};
+
+struct SmemState32 {         // D <= 8: [column][lane] in shared memory
+    uint32_t *d, *l;
+    int D;
+    __device__ void init() {
+        for (int x = 0; x < D; x++) d[x * 32] = 0u;
+        for (int x = 0; x < D * D; x++) l[x * 32] = 0u;
+    }
+    __device__ uint32_t dev(int x) const { return d[x * 32]; }
+    __device__ void set_dev(int x, uint32_t v) { d[x * 32] = v; }
+    __device__ uint32_t link(int x, int y) const { return l[(x * D + y) * 32]; }
+    __device__ void set_link(int x, int y, uint32_t v) { l[(x * D + y) * 32] = v; }
+    __device__ uint32_t makespan() const {
+        uint32_t m = 0;
+        for (int x = 0; x < D; x++) m = max(m, d[x * 32]);
+        return m;
+    }
+};
+
+template <int MODE, int PL>
+struct Place32 {
+    const uint32_t *pl;          // MODE 0: this group's bit-sliced words
+    const uint32_t *bits;        // MODE 1: base placement bits (shared memory)
+    const uint32_t *touched;     // MODE 1: warp-private deviation bitmap (shared memory)
+    const uint8_t *allowed_pos;
+    int words, all_allowed, lane, dmax;
+    LaneMove mv;
+    __device__ __forceinline__ int operator()(int32_t q) const {
+        if (MODE == 0) return planes_dev_at<PL>(pl, q, lane, dmax);
+        int x = bits_dev_at<PL>(bits, words, q);
+        if ((touched[q >> 5] >> (q & 31)) & 1u) {           // warp-uniform branch
+            const unsigned aq = all_allowed ? 0xFFu : (unsigned)__ldg(allowed_pos + q);
+            x = apply_lane(mv, q, x, aq);
+        }
+        return x;
+    }
+};
+
+struct Ctx32 {
+    uint32_t *ring;              // shared: ring[(pos & 15) * 32 + lane]
+    uint32_t *cold;              // global: cold[slot * 32 + lane]
+    const uint8_t *lclass;
+    int edge_stride, D;
+};
+
+__device__ __forceinline__ void prefetch_l1(const void *p) {
+    asm volatile("prefetch.global.L1 [%0];" ::"l"(p));
+}
+
+template <bool GLOBAL>
+__device__ __forceinline__ uint4 load_rec32(const uint8_t *p) {
+    if (GLOBAL) return __ldg(reinterpret_cast<const uint4 *>(p));
+    return *reinterpret_cast<const uint4 *>(p);
+}
+
+template <bool MULTI, bool GLOBAL, bool ALL_MAX, class PlaceT, class StateT>
+__device__ __forceinline__ void push32(const uint8_t *ep, const uint4 rec, int x, uint32_t c,
+                                       const PlaceT &place, StateT &st, const Ctx32 &cx) {
+    const int32_t succ = (int32_t)rec.y;
+    const uint32_t tgt = rec.z;
+    const int y = place(succ);
+    uint32_t a = c;                                          // same device: C_v (L144)
+    if (y != x) {                                            // cross: FCFS link x -> y
+        uint32_t t = rec.x;
+        if (MULTI) {
+            const int cls = cx.lclass[x * cx.D + y];
+            if (cls == 1) t = rec.w;
+            else if (cls > 1) {
+                const uint32_t *ext = reinterpret_cast<const uint32_t *>(ep + 16) + (cls - 2);
+                t = GLOBAL ? __ldg(ext) : *ext;
+            }
+        }
+        a = add_sat(max(c, st.link(x, y)), t);
+        st.set_link(x, y, a);
+    }
+    if (tgt & kT32Near) {
+        uint32_t *slot = cx.ring + (succ & (kRing - 1)) * 32;
+        if (ALL_MAX || !(tgt & kT32First)) a = max(a, *slot);
+        *slot = a;
+    } else {
+        uint32_t *slot = cx.cold + (size_t)(tgt & kT32SlotMask) * 32;
+        if (!ALL_MAX && (tgt & kT32First)) *slot = a;        // first far push: plain store
+        else atomicMax(slot, a);                             // RED.MAX, no wait for a reply
+    }
+}
+
+template <bool MULTI, bool GLOBAL, bool ALL_MAX, class PlaceT, class StateT>
+__device__ __forceinline__ void push_all32(const uint8_t *ep, uint32_t nout, int32_t ks, int x,
+                                           uint32_t c, const PlaceT &place, StateT &st,
+                                           const Ctx32 &cx) {
+    const int es = cx.edge_stride;
+    for (uint32_t i = 0; i < nout;) {
+        const uint4 rec = load_rec32<GLOBAL>(ep + (size_t)i * es);
+        if ((int32_t)rec.y != ks) {
+            push32<MULTI, GLOBAL, ALL_MAX>(ep + (size_t)i * es, rec, x, c, place, st, cx);
+            i++;
+            continue;
+        }
+        // swapped pair (ks, ks+1): the consumer now first in pi receives its transfers first
+        uint32_t a_end = i;
+        while (a_end < nout && (int32_t)load_rec32<GLOBAL>(ep + (size_t)a_end * es).y == ks) a_end++;
+        uint32_t b_end = a_end;
+        while (b_end < nout && (int32_t)load_rec32<GLOBAL>(ep + (size_t)b_end * es).y == ks + 1) b_end++;
+        for (uint32_t e = a_end; e < b_end; e++)
+            push32<MULTI, GLOBAL, ALL_MAX>(ep + (size_t)e * es, load_rec32<GLOBAL>(ep + (size_t)e * es),
+                                           x, c, place, st, cx);
+        for (uint32_t e = i; e < a_end; e++)
+            push32<MULTI, GLOBAL, ALL_MAX>(ep + (size_t)e * es, load_rec32<GLOBAL>(ep + (size_t)e * es),
+                                           x, c, place, st, cx);
+        i = b_end;
+    }
+}
+
+// relax the op at position v whose records start at rp (shared memory); returns the next op
+template <bool MULTI, bool ALL_MAX, class PlaceT, class StateT>
+__device__ __forceinline__ const uint8_t *relax32(const uint8_t *rp, int32_t v, int32_t ks,
+                                                  const uint8_t *heavy, const PlaceT &place,
+                                                  StateT &st, const Ctx32 &cx) {
+    const uint4 o = *reinterpret_cast<const uint4 *>(rp);   // {p, cold_slot, pf_slot, nout}
+    if ((int32_t)o.z >= 0) prefetch_l1(cx.cold + (size_t)o.z * 32);
+    const int x = place(v);
+    uint32_t r = 0;
+    if (o.w & kOp32HasNear) r = cx.ring[(v & (kRing - 1)) * 32];
+    if ((int32_t)o.y >= 0) r = max(r, cx.cold[(size_t)o.y * 32]);   // L1 hit after prefetch
+    const uint32_t c = add_sat(max(r, st.dev(x)), o.x);    // C_v = S_v + p_v
+    st.set_dev(x, c);
+    if (!(o.w & kOpHeavy)) {
+        const uint32_t nout = o.w & kOpNoutMask;
+        push_all32<MULTI, false, ALL_MAX>(rp + 16, nout, ks, x, c, place, st, cx);
+        return rp + 16 + (size_t)nout * cx.edge_stride;
+    }
+    const ExtRec ext = *reinterpret_cast<const ExtRec *>(rp + 16);
+    push_all32<MULTI, true, ALL_MAX>(heavy + ext.edge_off, (uint32_t)ext.nout, ks, x, c, place, st, cx);
+    return rp + 32;
+}
+
+__device__ __forceinline__ const uint8_t *skip32(const uint8_t *rp, int es) {
+    const uint32_t nout = reinterpret_cast<const uint32_t *>(rp)[3];
+    if (nout & kOpHeavy) return rp + 32;
+    return rp + 16 + (size_t)(nout & kOpNoutMask) * es;
+}
+
+// zero the slots an op opens with a first push (swap pairs only; times are >= 0)
+__device__ __forceinline__ void clear_first32(const uint8_t *rp, const uint8_t *heavy,
+                                              const Ctx32 &cx) {
+    const uint4 o = *reinterpret_cast<const uint4 *>(rp);
+    const bool global = (o.w & kOpHeavy) != 0;
+    const uint8_t *ep = rp + 16;
+    uint32_t nout = o.w & kOpNoutMask;
+    if (global) {
+        const ExtRec ext = *reinterpret_cast<const ExtRec *>(rp + 16);
+        ep = heavy + ext.edge_off;
+        nout = (uint32_t)ext.nout;
+    }
+    for (uint32_t i = 0; i < nout; i++) {
+        const uint4 rec = global ? load_rec32<true>(ep + (size_t)i * cx.edge_stride)
+                                 : load_rec32<false>(ep + (size_t)i * cx.edge_stride);
+        if (!(rec.z & kT32First)) continue;
+        if (rec.z & kT32Near) cx.ring[(((int32_t)rec.y) & (kRing - 1)) * 32] = 0u;
+        else cx.cold[(size_t)(rec.z & kT32SlotMask) * 32] = 0u;
+    }
+}
+
+template <int MODE, int PL, bool MULTI>
+__global__ void __launch_bounds__((kWarps + 1) * 32, 2)
+eval32_kernel(const EvalParams P) {
+    extern __shared__ __align__(128) uint8_t smem[];
+    const int sb = P.stage_bytes32;
+    uint8_t *stage_buf = smem;
+    uint64_t *full = reinterpret_cast<uint64_t *>(smem + (size_t)kStages * sb);
+    uint64_t *empty = full + kStages;
+    uint8_t *cur = align16(reinterpret_cast<uint8_t *>(empty + kStages));
+    uint8_t *lclass = cur;
+    cur = align16(cur + 64);
+    uint32_t *ring_all = reinterpret_cast<uint32_t *>(cur);
+    cur = align16(cur + (size_t)kWarps * kRing * 32 * 4);
+    uint32_t *bits_s = reinterpret_cast<uint32_t *>(cur);
+    uint32_t *touched_all = bits_s + (MODE == 1 ? PL * P.words : 0);
+    if (MODE == 1) cur = align16(cur + ((size_t)PL * P.words + (size_t)kWarps * P.words) * 4);
+    uint32_t *dstate = reinterpret_cast<uint32_t *>(cur);
+
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < kStages; s++) {
+            mbar_init(&full[s], 1);
+            mbar_init(&empty[s], kWarps);
+        }
+        mbar_fence_init();
+    }
+    if (threadIdx.x < 64) lclass[threadIdx.x] = P.link_class[threadIdx.x];
+    __syncthreads();
+
+    auto runs_here = [&](int bl) {           // search: this kernel owns bases below saturation
+        return MODE != 1 || P.gate == 0 || P.base_mk[bl] < (int64_t)kSat32;
+    };
+
+    if (warp == kWarps) {
+        if (lane == 0) {
+            uint32_t it = 0;
+            for (int64_t task = blockIdx.x; task < P.n_tasks; task += gridDim.x) {
+                const int bl = MODE ? (int)(task / P.tasks_per_base) : 0;
+                if (!runs_here(bl)) continue;
+                const BaseLayoutDev *B = &P.bases[bl];
+                const int nt = B->n_tiles32;
+                for (int t = 0; t < nt; t++, it++) {
+                    const int s = it % kStages;
+                    if (it >= (uint32_t)kStages) mbar_wait(&empty[s], ((it / kStages) - 1) & 1);
+                    const TileDesc td = B->tiles32[t];
+                    mbar_expect_tx(&full[s], (uint32_t)td.bytes);
+                    bulk_g2s(stage_buf + (size_t)s * sb, B->blob32 + td.byte_off, (uint32_t)td.bytes,
+                             &full[s]);
+                }
+            }
+        }
+        return;
+    }
+
+    Ctx32 cx;
+    cx.ring = ring_all + (size_t)warp * kRing * 32 + lane;
+    cx.cold = P.state32 + ((size_t)(blockIdx.x * kWarps + warp) * P.max_W32) * 32 + lane;
+    cx.lclass = lclass;
+    cx.edge_stride = P.edge_stride;
+    cx.D = P.D;
+    uint32_t *touched = touched_all + (size_t)warp * P.words;
+
+    using StateT = typename std::conditional<PL == 1, RegState32, SmemState32>::type;
+    StateT st;
+    if constexpr (PL != 1) {
+        st.D = P.D;
+        st.d = dstate + (size_t)warp * (P.D + P.D * P.D) * 32 + lane;
+        st.l = st.d + (size_t)P.D * 32;
+    }
+
+    uint32_t it = 0;
+    int loaded_base = -1;
+    for (int64_t task = blockIdx.x; task < P.n_tasks; task += gridDim.x) {
+        const int bl = MODE ? (int)(task / P.tasks_per_base) : 0;
+        if (!runs_here(bl)) continue;
+        const int64_t local = MODE ? task % P.tasks_per_base : task;
+        const BaseLayoutDev *B = &P.bases[bl];
+        const int nt = B->n_tiles32;
+        const uint8_t *heavy = B->heavy32;
+        const int64_t g = P.group_begin + local * kWarps + warp;
+
+        Place32<MODE, PL> place;
+        place.lane = lane;
+        place.dmax = P.D - 1;
+        place.words = P.words;
+        place.all_allowed = P.all_allowed;
+        bool active, valid = true;
+        const int64_t j = g * 32 + lane;
+        int32_t ks = -1;
+        if (MODE == 0) {
+            active = g * 32 < P.n_cand;
+            place.pl = P.planes_in + (size_t)g * P.n * PL;
+            if (active) valid = !((__ldg(P.invalid + g) >> lane) & 1u);
+        } else {
+            if (bl != loaded_base) {             // base placement bits -> shared memory
+                asm volatile("bar.sync 1, %0;" ::"r"(kWarps * 32));
+                for (int w = threadIdx.x; w < PL * P.words; w += kWarps * 32) bits_s[w] = __ldg(B->bits + w);
+                asm volatile("bar.sync 1, %0;" ::"r"(kWarps * 32));
+                loaded_base = bl;
+            }
+            active = g < P.group_begin + P.groups_per_base;
+            const int breal = P.b_offset + bl;
+            const uint64_t cb = ctr_base_of(P.step, P.P_total, breal);
+            place.bits = bits_s;
+            place.touched = touched;
+            place.allowed_pos = B->allowed_pos;
+            const uint8_t *adj = B->adj_next;
+            ks = active ? decode_swap(P.seed, cb, g, P.n, P.mix[3],
+                                      [&](int32_t k) { return __ldg(adj + k) != 0; })
+                        : -1;
+            const bool in_range = active && j >= P.j_begin && j < P.j_end;
+            const int32_t *movable = P.movable;
+            const int32_t *pos_of = B->pos_of;
+            const uint8_t *aop = P.allowed_op;
+            const int words = P.words;
+            place.mv = in_range
+                ? decode_lane(P.seed, cb, j, ks >= 0 && lane == 0, P.n, P.D, P.mix, P.n_movable,
+                              [&](int32_t i) { return __ldg(movable + i); },
+                              [&](int32_t op) { return __ldg(pos_of + op); },
+                              [&](int32_t q) { return bits_dev_at<PL>(bits_s, words, q); },
+                              [&](int32_t op) { return (unsigned)__ldg(aop + op); })
+                : no_move();
+            valid = in_range && place.mv.kind != kMoveInvalid;
+            if (place.mv.kind == kMoveInvalid) place.mv.kind = kMoveNone;
+            build_touched(touched, P.words, place.mv, lane);
+        }
+        st.init();
+
+        bool skip_first = false;
+        for (int t = 0; t < nt; t++, it++) {
+            const int s = it % kStages;
+            mbar_wait(&full[s], (it / kStages) & 1);
+            if (active) {
+                const uint8_t *tile = stage_buf + (size_t)s * sb;
+                const int32_t pos_end = reinterpret_cast<const int32_t *>(tile)[1];
+                int32_t v = reinterpret_cast<const int32_t *>(tile)[0];
+                const uint8_t *rp = tile + kTileHeader;
+                if (skip_first) {
+                    rp = skip32(rp, P.edge_stride);
+                    v++;
+                    skip_first = false;
+                }
+                while (v < pos_end) {
+                    if (v != ks) {
+                        rp = relax32<MULTI, false>(rp, v, ks, heavy, place, st, cx);
+                        v++;
+                        continue;
+                    }
+                    // swapped pair: ops at ks+1 then ks
+                    const uint8_t *rk = rp;
+                    const uint8_t *rk1;
+                    const bool straddle = (v + 1 == pos_end);
+                    if (straddle) {
+                        const int s2 = (it + 1) % kStages;
+                        mbar_wait(&full[s2], ((it + 1) / kStages) & 1);
+                        rk1 = stage_buf + (size_t)s2 * sb + kTileHeader;
+                    } else {
+                        rk1 = skip32(rk, P.edge_stride);
+                    }
+                    clear_first32(rk, heavy, cx);
+                    const uint8_t *after = relax32<MULTI, false>(rk1, v + 1, ks, heavy, place, st, cx);
+                    relax32<MULTI, true>(rk, v, ks, heavy, place, st, cx);
+                    if (straddle) {
+                        skip_first = true;
+                        v = pos_end;
+                    } else {
+                        rp = after;
+                        v += 2;
+                    }
+                }
+            }
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&empty[s]);
+        }
+
+        if (!active) continue;
+        const uint32_t mk = st.makespan();
+        if (MODE == 0) {
+            if (j < P.n_cand) {
+                if (!valid) {
+                    P.makespans[j] = INT64_MAX;
+                } else if (mk < kSat32) {
+                    P.makespans[j] = (int64_t)mk;
+                } else {                             // saturated: exact value from eval64
+                    P.makespans[j] = INT64_MAX;
+                    P.flag_list[atomicAdd(P.flag_count, 1)] = (int32_t)j;
+                }
+            }
+        } else {
+            // a saturated candidate's true makespan is >= kSat32 > this base's makespan, so it
+            // never wins the argmin; its clamped key still sorts after the base's (exact) key
+            uint64_t key = valid ? (((uint64_t)mk << 24) | (uint64_t)j) : ~0ull;
+            key = warp_min_u64(key);
+            if (lane == 0 && key != ~0ull)
+                atomicMin(reinterpret_cast<unsigned long long *>(P.keys + bl), (unsigned long long)key);
+        }
+    }
+}
+
+template <int MODE, int PL, bool MULTI>
+cudaError_t launch_one32(const EvalParams &p, int grid, cudaStream_t st) {
+    const int smem = eval32_smem_bytes(p, MODE);
+    auto kern = eval32_kernel<MODE, PL, MULTI>;
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    if (e != cudaSuccess) return e;
+    kern<<<grid, (kWarps + 1) * 32, smem, st>>>(p);
+    return cudaGetLastError();
+}
+
+template <int MODE, int PL, bool MULTI>
+int occupancy_one32(const EvalParams &p) {
+    const int smem = eval32_smem_bytes(p, MODE);
+    auto kern = eval32_kernel<MODE, PL, MULTI>;
+    if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) != cudaSuccess)
+        return 0;
+    int n = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kern, (kWarps + 1) * 32, smem) != cudaSuccess)
+        return 0;
+    return n;
+}
+
+int planes_of32(int D) { return D <= 2 ? 1 : (D <= 4 ? 2 : 4); }
+
+}  // namespace
+
+int eval32_smem_bytes(const EvalParams &p, int search_mode) {
+    const int pl = planes_of32(p.D);
+    size_t b = (size_t)kStages * p.stage_bytes32 + 2 * kStages * 8;
+    b = (b + 15) & ~size_t(15);
+    b += 64;
+    b = (b + 15) & ~size_t(15);
+    b += (size_t)kWarps * kRing * 32 * 4;
+    b = (b + 15) & ~size_t(15);
+    if (search_mode) b += ((size_t)pl * p.words + (size_t)kWarps * p.words) * 4;
+    b = (b + 15) & ~size_t(15);
+    if (pl != 1) b += (size_t)kWarps * (p.D + p.D * p.D) * 32 * 4;
+    return (int)b + 128;
+}
+
+#define PESTO_DISPATCH32(FN, ...)                                                          \
+    do {                                                                                   \
+        const int pl = planes_of32(p.D);                                                   \
+        const bool multi = p.n_classes > 1;                                                \
+        if (search_mode) {                                                                 \
+            if (pl == 1) return multi ? FN<1, 1, true>(__VA_ARGS__) : FN<1, 1, false>(__VA_ARGS__); \
+            if (pl == 2) return multi ? FN<1, 2, true>(__VA_ARGS__) : FN<1, 2, false>(__VA_ARGS__); \
+            return multi ? FN<1, 4, true>(__VA_ARGS__) : FN<1, 4, false>(__VA_ARGS__);     \
+        } else {                                                                           \
+            if (pl == 1) return multi ? FN<0, 1, true>(__VA_ARGS__) : FN<0, 1, false>(__VA_ARGS__); \
+            if (pl == 2) return multi ? FN<0, 2, true>(__VA_ARGS__) : FN<0, 2, false>(__VA_ARGS__); \
+            return multi ? FN<0, 4, true>(__VA_ARGS__) : FN<0, 4, false>(__VA_ARGS__);     \
+        }                                                                                  \
+    } while (0)
+
+cudaError_t launch_eval32(const EvalParams &p, int search_mode, int grid, cudaStream_t st) {
+    note_launch();
+    PESTO_DISPATCH32(launch_one32, p, grid, st);
+}
+
+int eval32_max_ctas_per_sm(const EvalParams &p, int search_mode) {
+    PESTO_DISPATCH32(occupancy_one32, p);
+}
+
+}  // namespace pesto

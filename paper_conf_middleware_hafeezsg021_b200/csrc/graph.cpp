@@ -89,6 +89,11 @@ pesto_status ensure_comm_tables(pesto_graph *g) {
         for (int c = 0; c < g->n_classes; c++)
             g->t_class[(size_t)e * g->n_classes + c] = transfer_ns(g->bytes[e], cls[c].first, cls[c].second);
     g->t_gen = g->comm_gen;
+    g->eligible32 = true;                                    // eval32: all durations < 2^28 ns
+    for (int32_t v = 0; v < g->n; v++)
+        if (g->p[v] >= (int64_t)kMaxDur32) g->eligible32 = false;
+    for (int64_t t : g->t_class)
+        if (t >= (int64_t)kMaxDur32) g->eligible32 = false;
     g->cache.clear();                                        // layouts embed t
     return PESTO_OK;
 }
@@ -229,6 +234,116 @@ pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<
         }
     }
     close_tile(n);
+
+    // ---- 32-bit saturating stream (eval32): near ring vs cold global slots ----
+    {
+        auto near_edge = [&](int64_t e) { return pos[g->dst[e]] - pos[g->src[e]] <= kNearDelta; };
+        std::vector<int32_t> first_far(n, INT32_MAX);
+        std::vector<uint8_t> has_near(n, 0);
+        for (int64_t e = 0; e < g->m; e++) {
+            const int32_t w = g->dst[e];
+            if (near_edge(e)) has_near[w] = 1;
+            else first_far[w] = std::min(first_far[w], pos[g->src[e]]);
+        }
+        // cold slot intervals [first far producer, pos(w) + 1], LIFO colouring as above
+        std::vector<std::vector<int32_t>> cs(n), cf(n);
+        for (int32_t w = 0; w < n; w++) {
+            if (first_far[w] == INT32_MAX) continue;
+            cs[first_far[w]].push_back(w);
+            if (pos[w] + 2 < n) cf[pos[w] + 2].push_back(w);
+        }
+        std::vector<int32_t> cslot(n, -1), fstack;
+        int32_t Wc = 0;
+        for (int32_t k = 0; k < n; k++) {
+            for (int32_t w : cf[k]) fstack.push_back(cslot[w]);
+            for (int32_t w : cs[k]) {
+                if (!fstack.empty()) { cslot[w] = fstack.back(); fstack.pop_back(); }
+                else cslot[w] = Wc++;
+            }
+        }
+        L->W32 = std::max(Wc, 1);
+        std::vector<uint8_t> seen_near(n, 0), seen_far(n, 0), first32(g->m, 0);
+        for (int32_t k = 0; k < n; k++) {
+            const int32_t u = order[k];
+            for (int64_t i = g->out_off[u]; i < g->out_off[u + 1]; i++) {
+                const int64_t e = sorted[i];
+                const int32_t w = g->dst[e];
+                uint8_t &seen = near_edge(e) ? seen_near[w] : seen_far[w];
+                if (!seen) { seen = 1; first32[e] = 1; }
+            }
+        }
+        const int es32 = edge_stride32_for(C);
+        auto tclamp = [&](int64_t e, int c) {
+            return (uint32_t)std::min<int64_t>(g->t_class[(size_t)e * C + c], kSat32);
+        };
+        auto put_edge32 = [&](std::vector<uint8_t> &buf, int64_t e) {
+            size_t at = buf.size();
+            buf.resize(at + es32, 0);
+            EdgeRec32 r;
+            r.t0 = tclamp(e, 0);
+            r.t1 = C > 1 ? tclamp(e, 1) : 0u;
+            r.succ_pos = pos[g->dst[e]];
+            r.target = (near_edge(e) ? kT32Near : (uint32_t)cslot[g->dst[e]]) |
+                       (first32[e] ? kT32First : 0u);
+            std::memcpy(buf.data() + at, &r, sizeof r);
+            for (int c = 2; c < C; c++) {
+                const uint32_t t = tclamp(e, c);
+                std::memcpy(buf.data() + at + 16 + 4 * (c - 2), &t, 4);
+            }
+        };
+        L->blob32.clear();
+        L->heavy32.clear();
+        L->tiles32.clear();
+        L->stage_bytes32 = 0;
+        size_t t_start = 0;
+        int32_t t_pos = 0;
+        auto open32 = [&](int32_t k) {
+            t_start = L->blob32.size();
+            t_pos = k;
+            L->blob32.resize(t_start + kTileHeader, 0);
+        };
+        auto close32 = [&](int32_t k_end) {
+            TileDesc td{};
+            td.byte_off = (int64_t)t_start;
+            td.bytes = (int32_t)(L->blob32.size() - t_start);
+            td.pos_begin = t_pos;
+            td.pos_end = k_end;
+            int32_t hdr[4] = {t_pos, k_end, td.bytes, 0};
+            std::memcpy(L->blob32.data() + t_start, hdr, 16);
+            L->tiles32.push_back(td);
+            L->stage_bytes32 = std::max(L->stage_bytes32, td.bytes);
+        };
+        open32(0);
+        for (int32_t k = 0; k < n; k++) {
+            const int32_t u = order[k];
+            const int64_t nout = g->out_off[u + 1] - g->out_off[u];
+            const bool heavy = nout * es32 > kMaxInlineBytes;
+            const size_t rec_bytes = 16 + (heavy ? 16 : (size_t)nout * es32);
+            if (k > t_pos && L->blob32.size() - t_start + rec_bytes > (size_t)kTileTarget) {
+                close32(k);
+                open32(k);
+            }
+            OpRec32 op;
+            op.p = (uint32_t)std::min<int64_t>(g->p[u], kSat32);
+            op.cold_slot = cslot[u];
+            const int32_t ahead = k + kPrefetchDist;
+            op.pf_slot = ahead < n ? cslot[order[ahead]] : -1;
+            op.nout = (heavy ? kOpHeavy : (uint32_t)nout) | (has_near[u] ? kOp32HasNear : 0u);
+            size_t at = L->blob32.size();
+            L->blob32.resize(at + 16);
+            std::memcpy(L->blob32.data() + at, &op, 16);
+            if (heavy) {
+                ExtRec ext{(int64_t)L->heavy32.size(), nout};
+                at = L->blob32.size();
+                L->blob32.resize(at + 16);
+                std::memcpy(L->blob32.data() + at, &ext, 16);
+                for (int64_t i = g->out_off[u]; i < g->out_off[u + 1]; i++) put_edge32(L->heavy32, sorted[i]);
+            } else {
+                for (int64_t i = g->out_off[u]; i < g->out_off[u + 1]; i++) put_edge32(L->blob32, sorted[i]);
+            }
+        }
+        close32(n);
+    }
     // order-move helpers
     L->adj_next.assign(n, 0);
     for (int32_t k = 0; k + 1 < n; k++) {
@@ -265,6 +380,9 @@ pesto_status upload_layout(pesto_graph *g, Layout &L) {
     if ((e = upload_vec(L.d_adj, L.adj_next)) != cudaSuccess) return cuda_fail(e, "upload layout");
     if ((e = upload_vec(L.d_allowed_pos, L.allowed_pos)) != cudaSuccess)
         return cuda_fail(e, "upload layout");
+    if ((e = upload_vec(L.d_blob32, L.blob32)) != cudaSuccess) return cuda_fail(e, "upload layout");
+    if ((e = upload_vec(L.d_heavy32, L.heavy32)) != cudaSuccess) return cuda_fail(e, "upload layout");
+    if ((e = upload_vec(L.d_tiles32, L.tiles32)) != cudaSuccess) return cuda_fail(e, "upload layout");
     L.on_device = true;
     std::vector<BaseLayoutDev> view{layout_view(L)};
     if ((e = upload_vec(L.d_view, view)) != cudaSuccess) return cuda_fail(e, "upload layout");
@@ -282,6 +400,11 @@ BaseLayoutDev layout_view(const Layout &L) {
     v.bits = nullptr;
     v.n_tiles = (int32_t)L.tiles.size();
     v.W = L.W;
+    v.blob32 = L.d_blob32.as<uint8_t>();
+    v.tiles32 = L.d_tiles32.as<TileDesc>();
+    v.heavy32 = L.d_heavy32.as<uint8_t>();
+    v.n_tiles32 = (int32_t)L.tiles32.size();
+    v.W32 = L.W32;
     return v;
 }
 
@@ -308,6 +431,21 @@ pesto_status ensure_state(pesto_graph *g, const EvalParams &p, int search_mode, 
     size_t bytes = (size_t)grid * kWarps * (size_t)std::max(p.max_W, 1) * 32 * sizeof(int64_t);
     cudaError_t e = g->d_state.ensure(bytes);
     if (e != cudaSuccess) return cuda_fail(e, "allocate slot state");
+    *grid_out = (int)grid;
+    return PESTO_OK;
+}
+
+pesto_status ensure_state32(pesto_graph *g, const EvalParams &p, int search_mode, int64_t n_tasks,
+                            int *grid_out) {
+    int per_sm = eval32_max_ctas_per_sm(p, search_mode);
+    if (per_sm <= 0)
+        return fail(PESTO_ECUDA, "eval32 kernel does not fit on an SM (smem " +
+                                     std::to_string(eval32_smem_bytes(p, search_mode)) + " B)");
+    int64_t grid = std::min<int64_t>(n_tasks, (int64_t)g->sms * per_sm);
+    grid = std::max<int64_t>(grid, 1);
+    size_t bytes = (size_t)grid * kWarps * (size_t)std::max(p.max_W32, 1) * 32 * sizeof(uint32_t);
+    cudaError_t e = g->d_state32.ensure(bytes);
+    if (e != cudaSuccess) return cuda_fail(e, "allocate cold slot state");
     *grid_out = (int)grid;
     return PESTO_OK;
 }
@@ -643,6 +781,8 @@ pesto_status pesto_eval_batch(pesto_graph *g, const int32_t *order, const void *
     fill_eval_common(g, p);
     p.stage_bytes = L->stage_bytes;
     p.max_W = L->W;
+    p.stage_bytes32 = L->stage_bytes32;
+    p.max_W32 = L->W32;
     p.planes_in = g->d_planes.as<uint32_t>();
     p.invalid = g->d_invalid.as<uint32_t>();
     p.n_cand = n_cand;
@@ -653,9 +793,26 @@ pesto_status pesto_eval_batch(pesto_graph *g, const int32_t *order, const void *
     p.tasks_per_base = (n_groups + kWarps - 1) / kWarps;
     p.n_tasks = p.tasks_per_base;
     int grid = 0;
-    if ((s = ensure_state(g, p, 0, p.n_tasks, &grid))) return s;
+    if (!g->eligible32) {                                     // 64-bit path for every row
+        if ((s = ensure_state(g, p, 0, p.n_tasks, &grid))) return s;
+        p.state = g->d_state.as<int64_t>();
+        if ((e = launch_eval(p, 0, grid, st)) != cudaSuccess) return cuda_fail(e, "launch eval");
+        return PESTO_OK;
+    }
+    // fast path: 32-bit saturating K1; rows that saturate are listed and re-run in 64-bit
+    if ((e = g->d_flags.ensure((size_t)(n_cand + 4) * 4)) != cudaSuccess) return cuda_fail(e, "allocate");
+    if ((e = cudaMemsetAsync(g->d_flags.ptr, 0, 4, st)) != cudaSuccess) return cuda_fail(e, "reset flags");
+    p.flag_count = g->d_flags.as<int32_t>();
+    p.flag_list = g->d_flags.as<int32_t>() + 4;
+    if ((s = ensure_state32(g, p, 0, p.n_tasks, &grid))) return s;
+    p.state32 = g->d_state32.as<uint32_t>();
+    if ((e = launch_eval32(p, 0, grid, st)) != cudaSuccess) return cuda_fail(e, "launch eval32");
+    p.list = p.flag_list;
+    p.list_count = p.flag_count;
+    const int64_t fix_tasks = std::min<int64_t>(p.n_tasks, g->sms);
+    if ((s = ensure_state(g, p, 2, fix_tasks, &grid))) return s;
     p.state = g->d_state.as<int64_t>();
-    if ((e = launch_eval(p, 0, grid, st)) != cudaSuccess) return cuda_fail(e, "launch eval");
+    if ((e = launch_eval(p, 2, grid, st)) != cudaSuccess) return cuda_fail(e, "launch eval fixup");
     return PESTO_OK;
 }
 

@@ -50,9 +50,14 @@ struct Layout {
     std::vector<uint8_t> blob, heavy;   // record stream (tiles) and out-of-line edges
     std::vector<TileDesc> tiles;
     std::vector<uint8_t> adj_next, allowed_pos;
+    // 32-bit saturating stream (eval32)
+    int32_t W32 = 0, stage_bytes32 = 0;
+    std::vector<uint8_t> blob32, heavy32;
+    std::vector<TileDesc> tiles32;
     int64_t comm_gen = -1;
     // device copies
     DevBuf d_blob, d_heavy, d_tiles, d_pos, d_adj, d_allowed_pos, d_view;
+    DevBuf d_blob32, d_heavy32, d_tiles32;
     bool on_device = false;
 };
 
@@ -78,6 +83,7 @@ struct pesto_graph {
     uint8_t link_class[64] = {0};
     std::vector<int64_t> t_class;         // [m][n_classes]
     int64_t t_gen = -1;
+    bool eligible32 = false;              // every p and t < kMaxDur32: eval32 may run
     int64_t worst_total = 0;              // sum p + sum_e max_L t_e
     // movable ops (>= 2 allowed devices), ascending id; forbidden-code masks
     std::vector<int32_t> movable;
@@ -86,7 +92,7 @@ struct pesto_graph {
     std::list<std::shared_ptr<pesto::Layout>> cache;
     // device buffers
     pesto::DevBuf d_state, d_planes, d_invalid, d_fmask, d_movable, d_allowed, d_bases, d_rows,
-        d_out;
+        d_out, d_state32, d_flags;        // d_flags: [count | list of saturated candidates]
     int32_t sms = 148;
 };
 
@@ -100,6 +106,8 @@ BaseLayoutDev layout_view(const Layout &L);
 void fill_eval_common(const pesto_graph *g, EvalParams &p);
 pesto_status ensure_state(pesto_graph *g, const EvalParams &p, int search_mode, int64_t n_tasks,
                           int *grid_out);
+pesto_status ensure_state32(pesto_graph *g, const EvalParams &p, int search_mode, int64_t n_tasks,
+                            int *grid_out);
 struct DeviceGuard {
     int prev = -1;
     explicit DeviceGuard(int dev) {

@@ -23,6 +23,12 @@ struct BaseLayoutDev {
     const uint32_t *bits;       // search: base placement, [planes][words] bit planes, by position
     int32_t n_tiles;
     int32_t W;                  // live ready-time slots
+    // eval32 stream
+    const uint8_t *blob32;
+    const TileDesc *tiles32;
+    const uint8_t *heavy32;
+    int32_t n_tiles32;
+    int32_t W32;                // cold slots
 };
 
 struct EvalParams {
@@ -52,6 +58,16 @@ struct EvalParams {
     uint64_t *keys_dbg;                 // nullable: key of every candidate in [j_begin, j_end)
     // work decomposition
     int64_t group_begin, groups_per_base, tasks_per_base, n_tasks;
+    // eval32 (32-bit saturating) state and its explicit-mode fixup list
+    uint32_t *state32;                  // [cta][warp][W32_max][32] cold slots
+    int32_t max_W32, stage_bytes32;
+    int32_t *flag_list, *flag_count;    // saturated candidates, re-evaluated by eval64
+    // search: base b runs on eval32 iff base_mk[b] < kSat32 (gate 1), on eval64 iff not (gate 2)
+    const int64_t *base_mk;
+    int32_t gate;
+    // eval64 list mode (MODE 2): candidates list[0 .. *list_count)
+    const int32_t *list;
+    const int32_t *list_count;
 };
 
 struct TransposeParams {
@@ -78,8 +94,12 @@ struct CommitParams {
     int32_t *swap_out;                  // [P] committed swap position or -1
 };
 
-// launchers (kernels.cu); they return the launch error, if any
+// launchers (kernels.cu / eval32.cu); they return the launch error, if any.
+// mode: 0 explicit rows, 1 search, 2 explicit list (eval64 only)
 cudaError_t launch_eval(const EvalParams &p, int search_mode, int grid, cudaStream_t st);
+cudaError_t launch_eval32(const EvalParams &p, int search_mode, int grid, cudaStream_t st);
+int eval32_smem_bytes(const EvalParams &p, int search_mode);
+int eval32_max_ctas_per_sm(const EvalParams &p, int search_mode);
 cudaError_t launch_transpose(const TransposeParams &p, cudaStream_t st);
 cudaError_t launch_commit(const CommitParams &p, cudaStream_t st);
 int eval_smem_bytes(const EvalParams &p, int search_mode);

@@ -19,45 +19,14 @@
 #include <cstdio>
 #include <type_traits>
 
+#include "device_common.cuh"
 #include "internal.h"
-#include "moves.cuh"
 
 namespace pesto {
 namespace {
 
 constexpr int64_t kInf64 = INT64_MAX;
-
-__device__ __forceinline__ uint32_t su32(const void *p) {
-    return (uint32_t)__cvta_generic_to_shared(p);
-}
-__device__ __forceinline__ void mbar_init(uint64_t *bar, uint32_t count) {
-    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(su32(bar)), "r"(count) : "memory");
-}
-__device__ __forceinline__ void mbar_fence_init() {
-    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-}
-__device__ __forceinline__ void mbar_expect_tx(uint64_t *bar, uint32_t bytes) {
-    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(su32(bar)),
-                 "r"(bytes) : "memory");
-}
-__device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
-    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(su32(bar)) : "memory");
-}
-__device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
-    uint32_t ok = 0;
-    while (!ok) {
-        asm volatile(
-            "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n"
-            " selp.u32 %0, 1, 0, p;\n}\n"
-            : "=r"(ok) : "r"(su32(bar)), "r"(parity) : "memory");
-    }
-}
-// one TMA bulk copy global -> shared, completion counted on `bar` (bytes % 16 == 0)
-__device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t bytes, uint64_t *bar) {
-    asm volatile(
-        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
-        ::"r"(su32(dst)), "l"(src), "r"(bytes), "r"(su32(bar)) : "memory");
-}
+using namespace dev;
 
 // ---------------------------------------------------------------------------------------------
 // per-lane device / link state
@@ -94,14 +63,6 @@ struct SmemState {           // D <= 8: [slot][lane] columns in shared memory
 // ---------------------------------------------------------------------------------------------
 // placement sources: each lane's device code for any position q (q is warp-uniform)
 // ---------------------------------------------------------------------------------------------
-template <int PL>
-__device__ __forceinline__ int base_dev_at(const uint32_t *bits, int words, int32_t q) {
-    int x = 0;
-#pragma unroll
-    for (int k = 0; k < PL; k++) x |= (int)((__ldg(bits + k * words + (q >> 5)) >> (q & 31)) & 1u) << k;
-    return x;
-}
-
 template <int MODE, int PL>
 struct Placement {
     // explicit rows (MODE 0): bit-sliced words of this warp's 32 candidates
@@ -117,19 +78,11 @@ struct Placement {
     int dmax;
 
     __device__ __forceinline__ int operator()(int32_t q) const {
-        if (MODE == 0) {
-            if (PL == 1) return (int)((__ldg(pl + q) >> lane) & 1u);
-            // codes >= D belong to rows K5 flagged infeasible; clamp so the discarded lane
-            // still indexes inside its state columns
-            if (PL == 2) {
-                uint2 w = __ldg(reinterpret_cast<const uint2 *>(pl) + q);
-                return min((int)(((w.x >> lane) & 1u) | (((w.y >> lane) & 1u) << 1)), dmax);
-            }
-            uint4 w = __ldg(reinterpret_cast<const uint4 *>(pl) + q);
-            return min((int)(((w.x >> lane) & 1u) | (((w.y >> lane) & 1u) << 1) |
-                             (((w.z >> lane) & 1u) << 2) | (((w.w >> lane) & 1u) << 3)), dmax);
-        } else {
-            int x = base_dev_at<PL>(bits, words, q);
+        // MODE 0: this warp's group words, bit `lane`; MODE 2 (fixup list): each lane's own
+        // candidate, i.e. its group's words (per-lane pointer) and bit (lane field = bit index)
+        if (MODE != 1) return planes_dev_at<PL>(pl, q, lane, dmax);
+        {
+            int x = ldg_bits_dev_at<PL>(bits, words, q);
             if ((touched[q >> 5] >> (q & 31)) & 1u) {          // warp-uniform branch
                 unsigned aq = all_allowed ? 0xFFu : (unsigned)__ldg(allowed_pos + q);
                 x = apply_lane(mv, q, x, aq);
@@ -256,24 +209,11 @@ __device__ __forceinline__ void clear_first_targets(const uint8_t *rp, const uin
     }
 }
 
-__device__ __forceinline__ uint64_t warp_min_u64(uint64_t v) {
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) {
-        uint64_t w = __shfl_xor_sync(0xffffffffu, v, o);
-        v = w < v ? w : v;
-    }
-    return v;
-}
-
-__device__ __forceinline__ uint8_t *align16(uint8_t *p) {
-    return reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(p) + 15) & ~uintptr_t(15));
-}
-
 // ---------------------------------------------------------------------------------------------
 // K1
 // ---------------------------------------------------------------------------------------------
 template <int MODE, int PL, bool MULTI>
-__global__ void __launch_bounds__((kWarps + 1) * 32)
+__global__ void __launch_bounds__((kWarps + 1) * 32, 2)
 eval_kernel(const EvalParams P) {
     extern __shared__ __align__(128) uint8_t smem[];
     uint8_t *stage_buf = smem;
@@ -297,12 +237,22 @@ eval_kernel(const EvalParams P) {
     if (threadIdx.x < 64) lclass[threadIdx.x] = P.link_class[threadIdx.x];
     __syncthreads();
 
+    // MODE 2 (fixup list) sizes its work from the device-side count; search bases may be
+    // gated to eval32 (gate 1 there) and only the saturated ones run here (gate 2)
+    const int64_t n_tasks = (MODE == 2) ? ((int64_t)*(volatile const int32_t *)P.list_count +
+                                           kWarps * 32 - 1) / (kWarps * 32)
+                                        : P.n_tasks;
+    auto runs_here = [&](int bl) {
+        return MODE != 1 || P.gate != 2 || P.base_mk[bl] >= (int64_t)kSat32;
+    };
+
     if (warp == kWarps) {
         // ---- producer: stream every task's tiles through the ring ----
         if (lane == 0) {
             uint32_t it = 0;
-            for (int64_t task = blockIdx.x; task < P.n_tasks; task += gridDim.x) {
-                const int bl = MODE ? (int)(task / P.tasks_per_base) : 0;
+            for (int64_t task = blockIdx.x; task < n_tasks; task += gridDim.x) {
+                const int bl = MODE == 1 ? (int)(task / P.tasks_per_base) : 0;
+                if (!runs_here(bl)) continue;
                 const BaseLayoutDev *B = &P.bases[bl];
                 const int nt = B->n_tiles;
                 for (int t = 0; t < nt; t++, it++) {
@@ -335,9 +285,10 @@ eval_kernel(const EvalParams P) {
     }
 
     uint32_t it = 0;
-    for (int64_t task = blockIdx.x; task < P.n_tasks; task += gridDim.x) {
-        const int bl = MODE ? (int)(task / P.tasks_per_base) : 0;
-        const int64_t local = MODE ? task % P.tasks_per_base : task;
+    for (int64_t task = blockIdx.x; task < n_tasks; task += gridDim.x) {
+        const int bl = MODE == 1 ? (int)(task / P.tasks_per_base) : 0;
+        if (!runs_here(bl)) continue;
+        const int64_t local = MODE == 1 ? task % P.tasks_per_base : task;
         const BaseLayoutDev *B = &P.bases[bl];
         const int nt = B->n_tiles;
         const uint8_t *heavy = B->heavy;
@@ -355,6 +306,14 @@ eval_kernel(const EvalParams P) {
             active = g * 32 < P.n_cand;
             place.pl = P.planes_in + (size_t)g * P.n * PL;
             if (active) valid = !((__ldg(P.invalid + g) >> lane) & 1u);
+        } else if (MODE == 2) {
+            const int32_t count = *(volatile const int32_t *)P.list_count;
+            active = g * 32 < count;
+            valid = j < count;
+            const int32_t c = valid ? P.list[j] : 0;      // this lane's candidate
+            place.pl = P.planes_in + (size_t)(c >> 5) * P.n * PL;
+            place.lane = c & 31;
+            j = c;
         } else {
             active = g < P.group_begin + P.groups_per_base;
             const int breal = P.b_offset + bl;
@@ -372,38 +331,16 @@ eval_kernel(const EvalParams P) {
             const uint32_t *bits = B->bits;
             const uint8_t *aop = P.allowed_op;
             const int words = P.words;
-            if (in_range) {
-                place.mv = decode_lane(
-                    P.seed, cb, j, ks >= 0 && lane == 0, P.n, P.D, P.mix, P.n_movable,
-                    [&](int32_t i) { return __ldg(movable + i); },
-                    [&](int32_t op) { return __ldg(pos_of + op); },
-                    [&](int32_t q) { return base_dev_at<PL>(bits, words, q); },
-                    [&](int32_t op) { return (unsigned)__ldg(aop + op); });
-            } else {
-                place.mv.kind = kMoveNone;
-                place.mv.nflip = 0;
-                place.mv.ws = place.mv.wl = place.mv.wd = 0;
-                for (int q = 0; q < 4; q++) { place.mv.fpos[q] = -1; place.mv.fdev[q] = 0; }
-            }
+            place.mv = in_range
+                ? decode_lane(P.seed, cb, j, ks >= 0 && lane == 0, P.n, P.D, P.mix, P.n_movable,
+                              [&](int32_t i) { return __ldg(movable + i); },
+                              [&](int32_t op) { return __ldg(pos_of + op); },
+                              [&](int32_t q) { return ldg_bits_dev_at<PL>(bits, words, q); },
+                              [&](int32_t op) { return (unsigned)__ldg(aop + op); })
+                : no_move();
             valid = in_range && place.mv.kind != kMoveInvalid;
             if (place.mv.kind == kMoveInvalid) place.mv.kind = kMoveNone;
-            // warp-private bitmap of positions where any lane deviates from the base
-            for (int w = lane; w < P.words; w += 32) touched[w] = 0u;
-            __syncwarp();
-            if (place.mv.kind == kMoveFlip) {
-                for (int f = 0; f < place.mv.nflip; f++) {
-                    const int32_t q = place.mv.fpos[f];
-                    atomicOr(&touched[q >> 5], 1u << (q & 31));
-                }
-            } else if (place.mv.kind == kMoveWindow && place.mv.wl > 0) {
-                const int32_t a = place.mv.ws, e = place.mv.ws + place.mv.wl;   // [a, e)
-                for (int32_t w = a >> 5; w <= (e - 1) >> 5; w++) {
-                    const int32_t lo = max(a, w * 32) - w * 32, hi = min(e, w * 32 + 32) - w * 32;
-                    const uint32_t msk = (hi - lo == 32) ? 0xffffffffu : (((1u << (hi - lo)) - 1u) << lo);
-                    atomicOr(&touched[w], msk);
-                }
-            }
-            __syncwarp();
+            build_touched(touched, P.words, place.mv, lane);
         }
         st.init(P.D);
 
@@ -460,6 +397,8 @@ eval_kernel(const EvalParams P) {
         const int64_t mk = st.makespan(P.D);                 // C_max = max_d dev_free[d]
         if (MODE == 0) {
             if (j < P.n_cand) P.makespans[j] = valid ? mk : kInf64;
+        } else if (MODE == 2) {
+            if (valid) P.makespans[j] = mk;                  // listed rows are feasible
         } else {
             uint64_t key = valid ? (((uint64_t)mk << 24) | (uint64_t)j) : ~0ull;
             if (P.keys_dbg && j >= P.j_begin && j < P.j_end) P.keys_dbg[j - P.j_begin] = key;
@@ -654,7 +593,11 @@ int eval_smem_bytes(const EvalParams &p, int search_mode) {
     do {                                                                                   \
         const int pl = planes_of(p.D);                                                     \
         const bool multi = p.n_classes > 1;                                                \
-        if (search_mode) {                                                                 \
+        if (search_mode == 2) {                                                            \
+            if (pl == 1) return multi ? FN<2, 1, true>(__VA_ARGS__) : FN<2, 1, false>(__VA_ARGS__); \
+            if (pl == 2) return multi ? FN<2, 2, true>(__VA_ARGS__) : FN<2, 2, false>(__VA_ARGS__); \
+            return multi ? FN<2, 4, true>(__VA_ARGS__) : FN<2, 4, false>(__VA_ARGS__);     \
+        } else if (search_mode) {                                                          \
             if (pl == 1) return multi ? FN<1, 1, true>(__VA_ARGS__) : FN<1, 1, false>(__VA_ARGS__); \
             if (pl == 2) return multi ? FN<1, 2, true>(__VA_ARGS__) : FN<1, 2, false>(__VA_ARGS__); \
             return multi ? FN<1, 4, true>(__VA_ARGS__) : FN<1, 4, false>(__VA_ARGS__);     \

@@ -48,4 +48,44 @@ struct alignas(16) TileDesc {
 // edge record stride for C link classes: 16 bytes + 8 bytes per extra class, 16-aligned
 inline int edge_stride_for(int classes) { return 16 * ((classes + 2) / 2); }
 
+// ---------------------------------------------------------------------------------------------
+// 32-bit saturating layout (eval32).  Times are uint32 ns saturating at kSat32:
+// every duration is < kMaxDur32 (else the graph is not eval32-eligible), so a + b never wraps
+// (kSat32 + kMaxDur32 < 2^32) and min(a + b, kSat32) is exact while the true value is below
+// kSat32.  Every start, finish and arrival time is <= the makespan, so a candidate whose
+// makespan comes out < kSat32 is exact; the others are re-evaluated by the 64-bit path.
+//
+// A producer within kNearDelta positions of its consumer pushes into the warp's shared-memory
+// ring (slot = consumer position mod kRing); farther producers push to a global "cold" slot
+// with fire-and-forget stores / atomic max, and the cold value is prefetched to L1
+// kPrefetchDist positions before the consumer reads it.
+// ---------------------------------------------------------------------------------------------
+constexpr uint32_t kSat32 = 0xF0000000u;        // 4,026,531,840 ns
+constexpr uint32_t kMaxDur32 = 0x10000000u;     // durations must be < 2^28 ns
+constexpr int kNearDelta = 12;
+constexpr int kRing = 16;                       // >= kNearDelta + 3 (swap margins)
+constexpr int kPrefetchDist = kNearDelta - 1;
+constexpr uint32_t kOp32HasNear = 1u << 24;     // OpRec32.nout: read the near ring
+constexpr uint32_t kT32First = 1u << 31;        // EdgeRec32.target: first push into its slot
+constexpr uint32_t kT32Near = 1u << 30;         // push into the near ring (slot = succ & 15)
+constexpr uint32_t kT32SlotMask = (1u << 30) - 1;
+
+struct alignas(16) OpRec32 {
+    uint32_t p;          // p_v (< kMaxDur32)
+    int32_t cold_slot;   // global slot holding far pushes into this op; -1 = none
+    int32_t pf_slot;     // cold slot of the op kPrefetchDist positions ahead; -1 = none
+    uint32_t nout;       // out-degree | kOp32HasNear | kOpHeavy
+};
+
+struct alignas(16) EdgeRec32 {
+    uint32_t t0;         // transfer time, link class 0 (< kMaxDur32)
+    int32_t succ_pos;
+    uint32_t target;     // cold slot | kT32Near | kT32First
+    uint32_t t1;         // link class 1; classes >= 2 follow in 4-byte words
+};
+
+inline int edge_stride32_for(int classes) {
+    return classes <= 2 ? 16 : 16 * (1 + (classes - 2 + 3) / 4);
+}
+
 }  // namespace pesto

@@ -69,7 +69,11 @@ struct pesto_search {
     uint64_t *h_keys = nullptr;
     ncclComm_t comm = nullptr;
     cudaStream_t last_stream = nullptr;
-    int32_t max_W = 1, stage_bytes = 16;
+    int32_t max_W = 1, stage_bytes = 16, max_W32 = 1, stage_bytes32 = 16;
+    // upper bounds of the base makespans known on the host (they never increase): once all are
+    // below kSat32 every base runs on eval32 and the 64-bit kernel is not launched at all
+    std::vector<int64_t> h_mk;
+    bool all_below = false;
 };
 
 namespace {
@@ -77,22 +81,38 @@ namespace {
 void refresh_views(pesto_search *s) {
     s->max_W = 1;
     s->stage_bytes = 16;
+    s->max_W32 = 1;
+    s->stage_bytes32 = 16;
     for (int b = 0; b < s->P; b++) {
         s->views[b] = layout_view(*s->layouts[b]);
         s->views[b].bits = s->d_bits.as<uint32_t>() + (size_t)b * s->g->planes * s->g->words;
         s->max_W = std::max(s->max_W, s->layouts[b]->W);
         s->stage_bytes = std::max(s->stage_bytes, s->layouts[b]->stage_bytes);
+        s->max_W32 = std::max(s->max_W32, s->layouts[b]->W32);
+        s->stage_bytes32 = std::max(s->stage_bytes32, s->layouts[b]->stage_bytes32);
     }
 }
 
+void update_all_below(pesto_search *s) {
+    s->all_below = s->g->eligible32;
+    for (int64_t mk : s->h_mk)
+        if (mk >= (int64_t)kSat32) s->all_below = false;
+}
+
+// fast: eval32 for the bases below saturation (+ eval64 for the others while any may exist);
+// otherwise (debug keys, initial makespans, ineligible graphs) eval64 for all candidates
 pesto_status launch_search_eval(pesto_search *s, int b_first, int n_bases, int64_t j0, int64_t j1,
-                                uint64_t *keys, uint64_t *keys_dbg, cudaStream_t st) {
+                                uint64_t *keys, uint64_t *keys_dbg, cudaStream_t st,
+                                bool fast = false) {
     pesto_graph *g = s->g;
     if (j1 <= j0) return PESTO_OK;
     EvalParams p;
     fill_eval_common(g, p);
     p.stage_bytes = s->stage_bytes;
     p.max_W = s->max_W;
+    p.stage_bytes32 = s->stage_bytes32;
+    p.max_W32 = s->max_W32;
+    p.base_mk = s->d_mk.as<int64_t>() + b_first;
     p.bases = s->d_views.as<BaseLayoutDev>() + b_first;
     p.b_offset = b_first;
     p.P_total = s->P;
@@ -111,11 +131,20 @@ pesto_status launch_search_eval(pesto_search *s, int b_first, int n_bases, int64
     p.tasks_per_base = (p.groups_per_base + kWarps - 1) / kWarps;
     p.n_tasks = p.tasks_per_base * n_bases;
     int grid = 0;
-    pesto_status rc = ensure_state(g, p, 1, p.n_tasks, &grid);
-    if (rc) return rc;
+    pesto_status rc;
+    cudaError_t e;
+    const bool use32 = fast && g->eligible32 && keys_dbg == nullptr;
+    if (use32) {
+        p.gate = 1;
+        if ((rc = ensure_state32(g, p, 1, p.n_tasks, &grid))) return rc;
+        p.state32 = g->d_state32.as<uint32_t>();
+        if ((e = launch_eval32(p, 1, grid, st)) != cudaSuccess) return cuda_fail(e, "launch eval32");
+        if (s->all_below) return PESTO_OK;
+        p.gate = 2;
+    }
+    if ((rc = ensure_state(g, p, 1, p.n_tasks, &grid))) return rc;
     p.state = g->d_state.as<int64_t>();
-    cudaError_t e = launch_eval(p, 1, grid, st);
-    if (e != cudaSuccess) return cuda_fail(e, "launch search eval");
+    if ((e = launch_eval(p, 1, grid, st)) != cudaSuccess) return cuda_fail(e, "launch search eval");
     return PESTO_OK;
 }
 
@@ -212,6 +241,8 @@ pesto_status pesto_search_create(pesto_graph *g, const pesto_search_desc *d, pes
     std::vector<int64_t> mk0(s->P);
     for (int b = 0; b < s->P; b++) mk0[b] = (int64_t)(k0[b] >> 24);
     cudaMemcpy(s->d_mk.ptr, mk0.data(), 8 * s->P, cudaMemcpyHostToDevice);
+    s->h_mk = mk0;
+    update_all_below(s.get());
     if (s->world > 1 && d->nccl_unique_id) {
         if (!nccl().ok) return fail(PESTO_ENCCL, "libnccl.so.2 not loadable");
         ncclUniqueId id;
@@ -230,7 +261,8 @@ pesto_status pesto_search_eval(pesto_search *s, void *stream) {
     s->last_stream = st;
     cudaError_t e = cudaMemsetAsync(s->d_keys.ptr, 0xFF, 8 * s->P, st);
     if (e != cudaSuccess) return cuda_fail(e, "reset keys");
-    return launch_search_eval(s, 0, s->P, s->j_begin, s->j_end, s->d_keys.as<uint64_t>(), nullptr, st);
+    return launch_search_eval(s, 0, s->P, s->j_begin, s->j_end, s->d_keys.as<uint64_t>(), nullptr, st,
+                              true);
 }
 
 pesto_status pesto_search_keys(pesto_search *s, uint64_t *keys_host, void *stream) {
@@ -283,8 +315,11 @@ pesto_status pesto_search_commit(pesto_search *s, void *stream) {
     if (s->mix[3] > 0) {
         // a committed adjacent swap changes a base's order: rebuild its position-space layout
         if ((e = cudaMemcpyAsync(s->h_swap, s->d_swap.ptr, 4 * s->P, cudaMemcpyDeviceToHost, st)) != cudaSuccess ||
+            (e = cudaMemcpyAsync(s->h_keys, s->d_mk.ptr, 8 * s->P, cudaMemcpyDeviceToHost, st)) != cudaSuccess ||
             (e = cudaStreamSynchronize(st)) != cudaSuccess)
             return cuda_fail(e, "read committed swaps");
+        std::memcpy(s->h_mk.data(), s->h_keys, 8 * s->P);   // h_keys doubles as a staging buffer
+        update_all_below(s);
         bool changed = false;
         for (int b = 0; b < s->P; b++) {
             const int32_t k = s->h_swap[b];

@@ -85,6 +85,54 @@ def test_random_dags(P, O, case):
         assert (gpu == ref).all(), (s, np.nonzero(gpu != ref)[0][:5], gpu[:3], ref[:3])
 
 
+def test_saturated_rows_take_the_64bit_path(P, O):
+    """makespans above the 32-bit kernel's saturation (4.03 s) are re-evaluated in int64."""
+    g = dag.random_dag(51, 60, 1.5, D=2, p_max=250_000_000, zero_frac=0.0, max_bytes=1 << 20,
+                       beta0=1000, beta1_fs=40_000)
+    g.p[:] = np.maximum(g.p, 60_000_000)                     # every op 60-250 ms: sum p >> 4 s
+    G = P.Graph.from_arrays(g)
+    order = dag.random_topo_order(g, 1)
+    x = dag.random_placements(g, 2, 300)
+    x[0] = 0                                                 # single device: sum p (saturated)
+    gpu = _gpu_eval(P, G, g, order, x)
+    ref, _ = O.makespan_batch(g, x, order)
+    assert (gpu == ref).all()
+    assert (ref > 0xF0000000).mean() > 0.5
+
+
+def test_ineligible_durations_use_64bit_path(P, O):
+    """a transfer >= 2^28 ns makes the graph ineligible for the 32-bit kernel."""
+    g = dag.random_dag(52, 200, 1.5, D=2, p_max=5000, max_bytes=1 << 20, beta0=10,
+                       beta1_fs=300_000_000)                 # 1 MB -> 300 ms transfers
+    G = P.Graph.from_arrays(g)
+    order = dag.random_topo_order(g, 3)
+    x = dag.random_placements(g, 4, 100)
+    gpu = _gpu_eval(P, G, g, order, x)
+    ref, _ = O.makespan_batch(g, x, order)
+    assert (gpu == ref).all()
+
+
+def test_search_with_bases_above_saturation(P, O):
+    """bases whose makespan exceeds 4.03 s run on the 64-bit kernel until they drop below."""
+    g = dag.random_dag(53, 50, 1.4, D=2, p_max=200_000_000, zero_frac=0.0, max_bytes=1 << 20,
+                       beta0=1000, beta1_fs=40_000)
+    g.p[:] = np.maximum(g.p, 40_000_000)
+    G = P.Graph.from_arrays(g)
+    xs, orders = _bases(g, 2, seed=11)
+    xs[0] = 0                                                # base 0: sum p > 4.03 s
+    mix = (50, 20, 20, 10)
+    S = P.Search(G, xs, orders, 512, mix, seed=4)
+    rx, ro = xs.copy(), orders.copy()
+    rmk = np.asarray([O.makespan(g, rx[b], ro[b]) for b in range(2)], np.int64)
+    assert rmk[0] > 0xF0000000
+    for step in range(4):
+        S.step()
+        O.search_step(g, rx, ro, rmk, 512, 4, step, mix)
+        for b in range(2):
+            mk, x, o = S.get(b)
+            assert mk == rmk[b] and (x == rx[b]).all() and (o == ro[b]).all(), (step, b)
+
+
 @pytest.mark.parametrize("name", ["inception_v3_2dev", "nmt4_2dev_commheavy",
                                   "transformer_2dev", "transformer_4dev_8gpu"])
 def test_full_size_sampled(P, O, name):
