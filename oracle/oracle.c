@@ -613,11 +613,15 @@ int oracle_candidate(int32_t n, int64_t m, const int32_t *src, const int32_t *ds
     memcpy(order_out, bo, (size_t)n * sizeof(int32_t));
     int64_t g = j >> 5, lane = j & 31;
     int swap = 0;
+    /* the group's region: positions [c, c + len) of the base order (DESIGN §4 S2) */
+    int64_t c0 = (int64_t)(oracle_draw(seed, step, P, b, 32 * g, 13) % (uint64_t)n);
+    int64_t rlen = n - c0 < 64 ? n - c0 : 64;
     /* order move: one adjacent swap per group of 32 candidates (DESIGN §4 S3) */
     if (g != 0 && mix[3] > 0 && n >= 2) {
         uint64_t u = oracle_draw(seed, step, P, b, 32 * g, 15);
         if ((int64_t)(u % 100u) < mix[3]) {
-            int64_t k = (int64_t)(oracle_draw(seed, step, P, b, 32 * g, 14) % (uint64_t)(n - 1));
+            int64_t k = c0 + (int64_t)(oracle_draw(seed, step, P, b, 32 * g, 14) % (uint64_t)rlen);
+            if (k > n - 2) k = n - 2;
             int32_t a = bo[k], c = bo[k + 1];
             int joined = 0;
             for (int64_t e = 0; e < m; e++)
@@ -632,35 +636,29 @@ int oracle_candidate(int32_t n, int64_t m, const int32_t *src, const int32_t *ds
     if (j == 0 || (swap && lane == 0)) return 1;
     int32_t wsum = mix[0] + mix[1] + mix[2];
     if (wsum <= 0) return 1;
-    /* movable ops: >= 2 allowed devices, ascending op id */
-    int32_t *mov = malloc((size_t)n * sizeof(int32_t));
-    int32_t nmov = 0, alts[8];
-    for (int32_t v = 0; v < n; v++) {
-        unsigned msk = allowed ? (unsigned)allowed[v] : 0xFFu;
-        if (popcount8(msk & ((1u << D) - 1u)) >= 2) mov[nmov++] = v;
-    }
-    int valid = 1;
+    int32_t alts[8];
     int64_t r = (int64_t)(oracle_draw(seed, step, P, b, j, 0) % (uint64_t)wsum);
-    if (r < mix[0] + mix[1]) {                               /* FLIP1 or FLIPk */
+    if (r < mix[0] + mix[1]) {                               /* FLIP1 or FLIPk (S4) */
         int32_t flips = 1;
         if (r >= mix[0]) flips = 2 + (int32_t)(oracle_draw(seed, step, P, b, j, 1) % 3u);
-        if (nmov == 0) valid = 0;
-        for (int32_t q = 0; valid && q < flips; q++) {
-            int32_t v = mov[oracle_draw(seed, step, P, b, j, 2 + 2 * q) % (uint64_t)nmov];
+        for (int32_t q = 0; q < flips; q++) {
+            int64_t pos = c0 + (int64_t)(oracle_draw(seed, step, P, b, j, 2 + 2 * q) % (uint64_t)rlen);
+            int32_t v = bo[pos];
+            unsigned msk = allowed ? (unsigned)allowed[v] : 0xFFu;
+            if (popcount8(msk & ((1u << D) - 1u)) < 2) return 0;   /* op cannot move: invalid */
             int32_t na = alt_devices(allowed, D, v, x_out[v], alts);
             x_out[v] = (uint8_t)alts[oracle_draw(seed, step, P, b, j, 3 + 2 * q) % (uint64_t)na];
         }
-    } else {                                                 /* WINDOW */
-        int64_t s = (int64_t)(oracle_draw(seed, step, P, b, j, 2) % (uint64_t)n);
+    } else {                                                 /* WINDOW (S4) */
+        int64_t s = c0 + (int64_t)(oracle_draw(seed, step, P, b, j, 2) % (uint64_t)rlen);
         int64_t len = 1 + (int64_t)(oracle_draw(seed, step, P, b, j, 3) % 64u);
         int32_t d = (int32_t)(oracle_draw(seed, step, P, b, j, 4) % (uint64_t)D);
-        for (int64_t q = s; q < s + len && q < n; q++) {
+        for (int64_t q = s; q < s + len && q < c0 + rlen; q++) {
             int32_t v = bo[q];
             if (allowed_dev(allowed, v, d)) x_out[v] = (uint8_t)d;
         }
     }
-    free(mov);
-    return valid;
+    return 1;
 }
 
 typedef struct {

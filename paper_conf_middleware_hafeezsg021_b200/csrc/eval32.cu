@@ -5,10 +5,12 @@
 //   cross e=(v,w): A_e = max(C_v, link_free[x_v->x_w]) + t_e;  link_free = A_e
 // with the ready-time state split by producer distance:
 //   near (consumer within kNearDelta positions): the warp's shared-memory ring, slot = pos & 15
-//   far:  a global cold slot written with fire-and-forget STG (first push) / RED.MAX, and
-//         prefetched into L1 kPrefetchDist positions before the consumer reads it.
+//   far:  a global cold slot written with fire-and-forget STG (first push) / RED.MAX, prefetched
+//         into L1 kPrefetchDist positions ahead and loaded one op before the consumer runs.
 // One lane = one candidate, 32 candidates per warp share every DAG tile, which the producer
 // warp streams into shared memory with cp.async.bulk (TMA) through an mbarrier ring.
+// Search candidates differ from their base only inside their group's 64-position region
+// (DESIGN.md §4), so outside it a lane's device is the base code embedded in the record.
 #include <algorithm>
 #include <type_traits>
 
@@ -52,22 +54,21 @@ struct SmemState32 {         // D <= 8: [column][lane] in shared memory
     }
 };
 
+// lane's device at position q; xb = the base code carried by the record that names q
 template <int MODE, int PL>
 struct Place32 {
     const uint32_t *pl;          // MODE 0: this group's bit-sliced words
-    const uint32_t *bits;        // MODE 1: base placement bits (shared memory)
-    const uint32_t *touched;     // MODE 1: warp-private deviation bitmap (shared memory)
-    const uint8_t *allowed_pos;
-    int words, all_allowed, lane, dmax;
+    const uint8_t *allowed_pos;  // MODE 1: masks by position (window moves)
+    int32_t rc, rlen;            // MODE 1: the group's region [rc, rc + rlen)
+    int all_allowed, lane, dmax;
     LaneMove mv;
-    __device__ __forceinline__ int operator()(int32_t q) const {
+    __device__ __forceinline__ int operator()(int32_t q, int xb) const {
         if (MODE == 0) return planes_dev_at<PL>(pl, q, lane, dmax);
-        int x = bits_dev_at<PL>(bits, words, q);
-        if ((touched[q >> 5] >> (q & 31)) & 1u) {           // warp-uniform branch
+        if ((uint32_t)(q - rc) < (uint32_t)rlen) {           // warp-uniform branch
             const unsigned aq = all_allowed ? 0xFFu : (unsigned)__ldg(allowed_pos + q);
-            x = apply_lane(mv, q, x, aq);
+            return apply_lane(mv, q, xb, aq);
         }
-        return x;
+        return xb;
     }
 };
 
@@ -91,9 +92,9 @@ __device__ __forceinline__ uint4 load_rec32(const uint8_t *p) {
 template <bool MULTI, bool GLOBAL, bool ALL_MAX, class PlaceT, class StateT>
 __device__ __forceinline__ void push32(const uint8_t *ep, const uint4 rec, int x, uint32_t c,
                                        const PlaceT &place, StateT &st, const Ctx32 &cx) {
-    const int32_t succ = (int32_t)rec.y;
+    const int32_t succ = (int32_t)(rec.y & kSuccPosMask);
     const uint32_t tgt = rec.z;
-    const int y = place(succ);
+    const int y = place(succ, (int)((rec.y >> kSuccXShift) & 7u));
     uint32_t a = c;                                          // same device: C_v (L144)
     if (y != x) {                                            // cross: FCFS link x -> y
         uint32_t t = rec.x;
@@ -119,23 +120,32 @@ __device__ __forceinline__ void push32(const uint8_t *ep, const uint4 rec, int x
     }
 }
 
+// out-edges of one producer in record order.  Only a producer feeding two adjacent positions
+// (kOpAdj) can see its order change under a swap (ks, ks+1): then the run of edges to ks+1 is
+// pushed before the run to ks (the swapped order's consumer order).
 template <bool MULTI, bool GLOBAL, bool ALL_MAX, class PlaceT, class StateT>
-__device__ __forceinline__ void push_all32(const uint8_t *ep, uint32_t nout, int32_t ks, int x,
-                                           uint32_t c, const PlaceT &place, StateT &st,
+__device__ __forceinline__ void push_all32(const uint8_t *ep, uint32_t nout, bool adj, int32_t ks,
+                                           int x, uint32_t c, const PlaceT &place, StateT &st,
                                            const Ctx32 &cx) {
     const int es = cx.edge_stride;
+    if (!adj || ks < 0) {
+        for (uint32_t i = 0; i < nout; i++)
+            push32<MULTI, GLOBAL, ALL_MAX>(ep + (size_t)i * es, load_rec32<GLOBAL>(ep + (size_t)i * es),
+                                           x, c, place, st, cx);
+        return;
+    }
+    auto spos = [&](uint32_t i) { return (int32_t)(load_rec32<GLOBAL>(ep + (size_t)i * es).y & kSuccPosMask); };
     for (uint32_t i = 0; i < nout;) {
-        const uint4 rec = load_rec32<GLOBAL>(ep + (size_t)i * es);
-        if ((int32_t)rec.y != ks) {
-            push32<MULTI, GLOBAL, ALL_MAX>(ep + (size_t)i * es, rec, x, c, place, st, cx);
+        if (spos(i) != ks) {
+            push32<MULTI, GLOBAL, ALL_MAX>(ep + (size_t)i * es, load_rec32<GLOBAL>(ep + (size_t)i * es),
+                                           x, c, place, st, cx);
             i++;
             continue;
         }
-        // swapped pair (ks, ks+1): the consumer now first in pi receives its transfers first
         uint32_t a_end = i;
-        while (a_end < nout && (int32_t)load_rec32<GLOBAL>(ep + (size_t)a_end * es).y == ks) a_end++;
+        while (a_end < nout && spos(a_end) == ks) a_end++;
         uint32_t b_end = a_end;
-        while (b_end < nout && (int32_t)load_rec32<GLOBAL>(ep + (size_t)b_end * es).y == ks + 1) b_end++;
+        while (b_end < nout && spos(b_end) == ks + 1) b_end++;
         for (uint32_t e = a_end; e < b_end; e++)
             push32<MULTI, GLOBAL, ALL_MAX>(ep + (size_t)e * es, load_rec32<GLOBAL>(ep + (size_t)e * es),
                                            x, c, place, st, cx);
@@ -146,26 +156,30 @@ __device__ __forceinline__ void push_all32(const uint8_t *ep, uint32_t nout, int
     }
 }
 
-// relax the op at position v whose records start at rp (shared memory); returns the next op
+// Relax the op at position v (records at rp, shared memory).  `cold_in` is its far arrivals
+// (loaded one op earlier); the far arrivals of the next position are loaded into `cold_out`.
 template <bool MULTI, bool ALL_MAX, class PlaceT, class StateT>
 __device__ __forceinline__ const uint8_t *relax32(const uint8_t *rp, int32_t v, int32_t ks,
                                                   const uint8_t *heavy, const PlaceT &place,
-                                                  StateT &st, const Ctx32 &cx) {
-    const uint4 o = *reinterpret_cast<const uint4 *>(rp);   // {p, cold_slot, pf_slot, nout}
+                                                  StateT &st, const Ctx32 &cx, uint32_t cold_in,
+                                                  uint32_t &cold_out) {
+    const uint4 o = *reinterpret_cast<const uint4 *>(rp);   // {p, cold_next, pf_slot, nout}
     if ((int32_t)o.z >= 0) prefetch_l1(cx.cold + (size_t)o.z * 32);
-    const int x = place(v);
-    uint32_t r = 0;
-    if (o.w & kOp32HasNear) r = cx.ring[(v & (kRing - 1)) * 32];
-    if ((int32_t)o.y >= 0) r = max(r, cx.cold[(size_t)o.y * 32]);   // L1 hit after prefetch
+    cold_out = (int32_t)o.y >= 0 ? cx.cold[(size_t)o.y * 32] : 0u;
+    const int x = place(v, (int)((o.w >> kOpXShift) & 7u));
+    uint32_t r = cold_in;
+    if (o.w & kOp32HasNear) r = max(r, cx.ring[(v & (kRing - 1)) * 32]);
     const uint32_t c = add_sat(max(r, st.dev(x)), o.x);    // C_v = S_v + p_v
     st.set_dev(x, c);
+    const bool adj = (o.w & kOpAdj) != 0;
     if (!(o.w & kOpHeavy)) {
         const uint32_t nout = o.w & kOpNoutMask;
-        push_all32<MULTI, false, ALL_MAX>(rp + 16, nout, ks, x, c, place, st, cx);
+        push_all32<MULTI, false, ALL_MAX>(rp + 16, nout, adj, ks, x, c, place, st, cx);
         return rp + 16 + (size_t)nout * cx.edge_stride;
     }
     const ExtRec ext = *reinterpret_cast<const ExtRec *>(rp + 16);
-    push_all32<MULTI, true, ALL_MAX>(heavy + ext.edge_off, (uint32_t)ext.nout, ks, x, c, place, st, cx);
+    push_all32<MULTI, true, ALL_MAX>(heavy + ext.edge_off, (uint32_t)ext.nout, adj, ks, x, c, place,
+                                     st, cx);
     return rp + 32;
 }
 
@@ -191,7 +205,7 @@ __device__ __forceinline__ void clear_first32(const uint8_t *rp, const uint8_t *
         const uint4 rec = global ? load_rec32<true>(ep + (size_t)i * cx.edge_stride)
                                  : load_rec32<false>(ep + (size_t)i * cx.edge_stride);
         if (!(rec.z & kT32First)) continue;
-        if (rec.z & kT32Near) cx.ring[(((int32_t)rec.y) & (kRing - 1)) * 32] = 0u;
+        if (rec.z & kT32Near) cx.ring[(((int32_t)(rec.y & kSuccPosMask)) & (kRing - 1)) * 32] = 0u;
         else cx.cold[(size_t)(rec.z & kT32SlotMask) * 32] = 0u;
     }
 }
@@ -209,9 +223,6 @@ eval32_kernel(const EvalParams P) {
     cur = align16(cur + 64);
     uint32_t *ring_all = reinterpret_cast<uint32_t *>(cur);
     cur = align16(cur + (size_t)kWarps * kRing * 32 * 4);
-    uint32_t *bits_s = reinterpret_cast<uint32_t *>(cur);
-    uint32_t *touched_all = bits_s + (MODE == 1 ? PL * P.words : 0);
-    if (MODE == 1) cur = align16(cur + ((size_t)PL * P.words + (size_t)kWarps * P.words) * 4);
     uint32_t *dstate = reinterpret_cast<uint32_t *>(cur);
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -254,9 +265,8 @@ eval32_kernel(const EvalParams P) {
     cx.ring = ring_all + (size_t)warp * kRing * 32 + lane;
     cx.cold = P.state32 + ((size_t)(blockIdx.x * kWarps + warp) * P.max_W32) * 32 + lane;
     cx.lclass = lclass;
-    cx.edge_stride = P.edge_stride;
+    cx.edge_stride = P.edge_stride32;
     cx.D = P.D;
-    uint32_t *touched = touched_all + (size_t)warp * P.words;
 
     using StateT = typename std::conditional<PL == 1, RegState32, SmemState32>::type;
     StateT st;
@@ -267,7 +277,6 @@ eval32_kernel(const EvalParams P) {
     }
 
     uint32_t it = 0;
-    int loaded_base = -1;
     for (int64_t task = blockIdx.x; task < P.n_tasks; task += gridDim.x) {
         const int bl = MODE ? (int)(task / P.tasks_per_base) : 0;
         if (!runs_here(bl)) continue;
@@ -280,8 +289,9 @@ eval32_kernel(const EvalParams P) {
         Place32<MODE, PL> place;
         place.lane = lane;
         place.dmax = P.D - 1;
-        place.words = P.words;
         place.all_allowed = P.all_allowed;
+        place.rc = 0;
+        place.rlen = 0;
         bool active, valid = true;
         const int64_t j = g * 32 + lane;
         int32_t ks = -1;
@@ -290,41 +300,35 @@ eval32_kernel(const EvalParams P) {
             place.pl = P.planes_in + (size_t)g * P.n * PL;
             if (active) valid = !((__ldg(P.invalid + g) >> lane) & 1u);
         } else {
-            if (bl != loaded_base) {             // base placement bits -> shared memory
-                asm volatile("bar.sync 1, %0;" ::"r"(kWarps * 32));
-                for (int w = threadIdx.x; w < PL * P.words; w += kWarps * 32) bits_s[w] = __ldg(B->bits + w);
-                asm volatile("bar.sync 1, %0;" ::"r"(kWarps * 32));
-                loaded_base = bl;
-            }
             active = g < P.group_begin + P.groups_per_base;
             const int breal = P.b_offset + bl;
             const uint64_t cb = ctr_base_of(P.step, P.P_total, breal);
-            place.bits = bits_s;
-            place.touched = touched;
+            const Region rg = decode_region(P.seed, cb, g, P.n);
+            place.rc = rg.c;
+            place.rlen = rg.len;
             place.allowed_pos = B->allowed_pos;
             const uint8_t *adj = B->adj_next;
-            ks = active ? decode_swap(P.seed, cb, g, P.n, P.mix[3],
+            ks = active ? decode_swap(P.seed, cb, g, P.n, P.mix[3], rg,
                                       [&](int32_t k) { return __ldg(adj + k) != 0; })
                         : -1;
             const bool in_range = active && j >= P.j_begin && j < P.j_end;
-            const int32_t *movable = P.movable;
-            const int32_t *pos_of = B->pos_of;
+            const int32_t *ord = B->order;
+            const uint32_t *bits = B->bits;
             const uint8_t *aop = P.allowed_op;
             const int words = P.words;
             place.mv = in_range
-                ? decode_lane(P.seed, cb, j, ks >= 0 && lane == 0, P.n, P.D, P.mix, P.n_movable,
-                              [&](int32_t i) { return __ldg(movable + i); },
-                              [&](int32_t op) { return __ldg(pos_of + op); },
-                              [&](int32_t q) { return bits_dev_at<PL>(bits_s, words, q); },
+                ? decode_lane(P.seed, cb, j, ks >= 0 && lane == 0, P.D, P.mix, rg,
+                              [&](int32_t q) { return __ldg(ord + q); },
+                              [&](int32_t q) { return ldg_bits_dev_at<PL>(bits, words, q); },
                               [&](int32_t op) { return (unsigned)__ldg(aop + op); })
                 : no_move();
             valid = in_range && place.mv.kind != kMoveInvalid;
-            if (place.mv.kind == kMoveInvalid) place.mv.kind = kMoveNone;
-            build_touched(touched, P.words, place.mv, lane);
+            if (place.mv.kind == kMoveInvalid) place.mv = no_move();
         }
         st.init();
 
         bool skip_first = false;
+        uint32_t cold_v = 0;                         // far arrivals of the next op to relax
         for (int t = 0; t < nt; t++, it++) {
             const int s = it % kStages;
             mbar_wait(&full[s], (it / kStages) & 1);
@@ -334,13 +338,13 @@ eval32_kernel(const EvalParams P) {
                 int32_t v = reinterpret_cast<const int32_t *>(tile)[0];
                 const uint8_t *rp = tile + kTileHeader;
                 if (skip_first) {
-                    rp = skip32(rp, P.edge_stride);
+                    rp = skip32(rp, cx.edge_stride);
                     v++;
                     skip_first = false;
                 }
                 while (v < pos_end) {
                     if (v != ks) {
-                        rp = relax32<MULTI, false>(rp, v, ks, heavy, place, st, cx);
+                        rp = relax32<MULTI, false>(rp, v, ks, heavy, place, st, cx, cold_v, cold_v);
                         v++;
                         continue;
                     }
@@ -353,11 +357,16 @@ eval32_kernel(const EvalParams P) {
                         mbar_wait(&full[s2], ((it + 1) / kStages) & 1);
                         rk1 = stage_buf + (size_t)s2 * sb + kTileHeader;
                     } else {
-                        rk1 = skip32(rk, P.edge_stride);
+                        rk1 = skip32(rk, cx.edge_stride);
                     }
+                    const int32_t cold_k1 = reinterpret_cast<const int32_t *>(rk)[1];
+                    const uint32_t cold_first = cold_k1 >= 0 ? cx.cold[(size_t)cold_k1 * 32] : 0u;
+                    uint32_t dummy, next_v;
                     clear_first32(rk, heavy, cx);
-                    const uint8_t *after = relax32<MULTI, false>(rk1, v + 1, ks, heavy, place, st, cx);
-                    relax32<MULTI, true>(rk, v, ks, heavy, place, st, cx);
+                    const uint8_t *after =
+                        relax32<MULTI, false>(rk1, v + 1, ks, heavy, place, st, cx, cold_first, next_v);
+                    relax32<MULTI, true>(rk, v, ks, heavy, place, st, cx, cold_v, dummy);
+                    cold_v = next_v;                 // ks+1's record names the op at ks+2
                     if (straddle) {
                         skip_first = true;
                         v = pos_end;
@@ -422,14 +431,13 @@ int planes_of32(int D) { return D <= 2 ? 1 : (D <= 4 ? 2 : 4); }
 }  // namespace
 
 int eval32_smem_bytes(const EvalParams &p, int search_mode) {
+    (void)search_mode;
     const int pl = planes_of32(p.D);
     size_t b = (size_t)kStages * p.stage_bytes32 + 2 * kStages * 8;
     b = (b + 15) & ~size_t(15);
     b += 64;
     b = (b + 15) & ~size_t(15);
     b += (size_t)kWarps * kRing * 32 * 4;
-    b = (b + 15) & ~size_t(15);
-    if (search_mode) b += ((size_t)pl * p.words + (size_t)kWarps * p.words) * 4;
     b = (b + 15) & ~size_t(15);
     if (pl != 1) b += (size_t)kWarps * (p.D + p.D * p.D) * 32 * 4;
     return (int)b + 128;

@@ -25,7 +25,6 @@ pesto_status cuda_fail(cudaError_t e, const char *what) {
 }
 
 static constexpr int64_t kGuard40 = int64_t(1) << 40;
-static constexpr int kMaxInlineBytes = 2048;
 
 // t = beta0 + ceil(bytes * beta1_fs / 10^6) (PAPER.md L138 linear model, reading R6); -1 overflow
 static int64_t transfer_ns(int64_t bytes, int64_t beta0, int64_t beta1) {
@@ -98,269 +97,6 @@ pesto_status ensure_comm_tables(pesto_graph *g) {
     return PESTO_OK;
 }
 
-// ---------------------------------------------------------------------------------------------
-// position-space layout for one order (a0 steps 4-5)
-// ---------------------------------------------------------------------------------------------
-pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<Layout> &out,
-                          bool use_cache) {
-    pesto_status s = ensure_comm_tables(g);
-    if (s) return s;
-    const int32_t n = g->n;
-    if (!order) return fail(PESTO_EINVAL, "order is NULL");
-    if (use_cache) {
-        for (auto it = g->cache.begin(); it != g->cache.end(); ++it) {
-            if ((*it)->comm_gen == g->comm_gen &&
-                std::memcmp((*it)->order.data(), order, (size_t)n * 4) == 0) {
-                out = *it;
-                g->cache.splice(g->cache.begin(), g->cache, it);
-                return PESTO_OK;
-            }
-        }
-    }
-    auto L = std::make_shared<Layout>();
-    L->comm_gen = g->comm_gen;
-    L->order.assign(order, order + n);
-    L->pos.assign(n, -1);
-    for (int32_t k = 0; k < n; k++) {
-        const int32_t v = order[k];
-        if (v < 0 || v >= n || L->pos[v] != -1) return fail(PESTO_ENOTTOPO, "order is not a permutation");
-        L->pos[v] = k;
-    }
-    for (int64_t e = 0; e < g->m; e++)
-        if (L->pos[g->src[e]] >= L->pos[g->dst[e]])
-            return fail(PESTO_ENOTTOPO, "order violates edge " + std::to_string(e));
-    const std::vector<int32_t> &pos = L->pos;
-
-    // out-edges of every producer sorted by (successor position, edge index): FCFS tie order R3
-    std::vector<int64_t> sorted(g->out_edges);
-    for (int32_t u = 0; u < n; u++) {
-        auto b = sorted.begin() + g->out_off[u], e = sorted.begin() + g->out_off[u + 1];
-        std::sort(b, e, [&](int64_t a, int64_t c) {
-            const int32_t pa = pos[g->dst[a]], pc = pos[g->dst[c]];
-            return pa != pc ? pa < pc : a < c;
-        });
-    }
-    // ready-time slot intervals: consumer w lives from its first producer's position through
-    // pos(w) + 1 (one position of padding keeps an adjacent swap exact)
-    std::vector<int32_t> first(n, INT32_MAX);
-    for (int64_t e = 0; e < g->m; e++) first[g->dst[e]] = std::min(first[g->dst[e]], pos[g->src[e]]);
-    std::vector<std::vector<int32_t>> starts(n), frees(n);
-    for (int32_t w = 0; w < n; w++) {
-        if (first[w] == INT32_MAX) continue;
-        starts[first[w]].push_back(w);
-        if (pos[w] + 2 < n) frees[pos[w] + 2].push_back(w);
-    }
-    std::vector<int32_t> slot(n, kNoSlot), free_stack;
-    int32_t W = 0;
-    for (int32_t k = 0; k < n; k++) {
-        for (int32_t w : frees[k]) free_stack.push_back(slot[w]);
-        for (int32_t w : starts[k]) {
-            if (!free_stack.empty()) { slot[w] = free_stack.back(); free_stack.pop_back(); }
-            else slot[w] = W++;
-        }
-    }
-    L->W = std::max(W, 1);
-    // first push into each slot, in processing order
-    std::vector<uint8_t> seen(n, 0), first_flag(g->m, 0);
-    for (int32_t k = 0; k < n; k++) {
-        const int32_t u = order[k];
-        for (int64_t i = g->out_off[u]; i < g->out_off[u + 1]; i++) {
-            const int64_t e = sorted[i];
-            if (!seen[g->dst[e]]) { seen[g->dst[e]] = 1; first_flag[e] = 1; }
-        }
-    }
-    // records + tiles
-    const int C = g->n_classes;
-    const int es = edge_stride_for(C);
-    auto put_edge = [&](std::vector<uint8_t> &buf, int64_t e) {
-        size_t at = buf.size();
-        buf.resize(at + es, 0);
-        EdgeRec r;
-        r.t0 = g->t_class[(size_t)e * C];
-        r.succ_pos = pos[g->dst[e]];
-        r.slot = (uint32_t)slot[g->dst[e]] | (first_flag[e] ? kEdgeFirst : 0u);
-        std::memcpy(buf.data() + at, &r, sizeof r);
-        for (int c = 1; c < C; c++) {
-            int64_t t = g->t_class[(size_t)e * C + c];
-            std::memcpy(buf.data() + at + 16 + 8 * (c - 1), &t, 8);
-        }
-    };
-    L->blob.clear();
-    L->heavy.clear();
-    L->tiles.clear();
-    size_t tile_start = 0;
-    int32_t tile_pos = 0;
-    auto open_tile = [&](int32_t k) {
-        tile_start = L->blob.size();
-        tile_pos = k;
-        L->blob.resize(tile_start + kTileHeader, 0);
-    };
-    auto close_tile = [&](int32_t k_end) {
-        TileDesc td{};
-        td.byte_off = (int64_t)tile_start;
-        td.bytes = (int32_t)(L->blob.size() - tile_start);
-        td.pos_begin = tile_pos;
-        td.pos_end = k_end;
-        int32_t hdr[4] = {tile_pos, k_end, td.bytes, 0};
-        std::memcpy(L->blob.data() + tile_start, hdr, 16);
-        L->tiles.push_back(td);
-        L->stage_bytes = std::max(L->stage_bytes, td.bytes);
-    };
-    open_tile(0);
-    for (int32_t k = 0; k < n; k++) {
-        const int32_t u = order[k];
-        const int64_t nout = g->out_off[u + 1] - g->out_off[u];
-        const bool heavy = nout * es > kMaxInlineBytes;
-        const size_t rec_bytes = 16 + (heavy ? 16 : (size_t)nout * es);
-        if (k > tile_pos && L->blob.size() - tile_start + rec_bytes > (size_t)kTileTarget) {
-            close_tile(k);
-            open_tile(k);
-        }
-        OpRec op;
-        op.p = g->p[u];
-        op.in_slot = slot[u];
-        op.nout = heavy ? (kOpHeavy | 0u) : (uint32_t)nout;
-        size_t at = L->blob.size();
-        L->blob.resize(at + 16);
-        std::memcpy(L->blob.data() + at, &op, 16);
-        if (heavy) {
-            ExtRec ext{(int64_t)L->heavy.size(), nout};
-            at = L->blob.size();
-            L->blob.resize(at + 16);
-            std::memcpy(L->blob.data() + at, &ext, 16);
-            for (int64_t i = g->out_off[u]; i < g->out_off[u + 1]; i++) put_edge(L->heavy, sorted[i]);
-        } else {
-            for (int64_t i = g->out_off[u]; i < g->out_off[u + 1]; i++) put_edge(L->blob, sorted[i]);
-        }
-    }
-    close_tile(n);
-
-    // ---- 32-bit saturating stream (eval32): near ring vs cold global slots ----
-    {
-        auto near_edge = [&](int64_t e) { return pos[g->dst[e]] - pos[g->src[e]] <= kNearDelta; };
-        std::vector<int32_t> first_far(n, INT32_MAX);
-        std::vector<uint8_t> has_near(n, 0);
-        for (int64_t e = 0; e < g->m; e++) {
-            const int32_t w = g->dst[e];
-            if (near_edge(e)) has_near[w] = 1;
-            else first_far[w] = std::min(first_far[w], pos[g->src[e]]);
-        }
-        // cold slot intervals [first far producer, pos(w) + 1], LIFO colouring as above
-        std::vector<std::vector<int32_t>> cs(n), cf(n);
-        for (int32_t w = 0; w < n; w++) {
-            if (first_far[w] == INT32_MAX) continue;
-            cs[first_far[w]].push_back(w);
-            if (pos[w] + 2 < n) cf[pos[w] + 2].push_back(w);
-        }
-        std::vector<int32_t> cslot(n, -1), fstack;
-        int32_t Wc = 0;
-        for (int32_t k = 0; k < n; k++) {
-            for (int32_t w : cf[k]) fstack.push_back(cslot[w]);
-            for (int32_t w : cs[k]) {
-                if (!fstack.empty()) { cslot[w] = fstack.back(); fstack.pop_back(); }
-                else cslot[w] = Wc++;
-            }
-        }
-        L->W32 = std::max(Wc, 1);
-        std::vector<uint8_t> seen_near(n, 0), seen_far(n, 0), first32(g->m, 0);
-        for (int32_t k = 0; k < n; k++) {
-            const int32_t u = order[k];
-            for (int64_t i = g->out_off[u]; i < g->out_off[u + 1]; i++) {
-                const int64_t e = sorted[i];
-                const int32_t w = g->dst[e];
-                uint8_t &seen = near_edge(e) ? seen_near[w] : seen_far[w];
-                if (!seen) { seen = 1; first32[e] = 1; }
-            }
-        }
-        const int es32 = edge_stride32_for(C);
-        auto tclamp = [&](int64_t e, int c) {
-            return (uint32_t)std::min<int64_t>(g->t_class[(size_t)e * C + c], kSat32);
-        };
-        auto put_edge32 = [&](std::vector<uint8_t> &buf, int64_t e) {
-            size_t at = buf.size();
-            buf.resize(at + es32, 0);
-            EdgeRec32 r;
-            r.t0 = tclamp(e, 0);
-            r.t1 = C > 1 ? tclamp(e, 1) : 0u;
-            r.succ_pos = pos[g->dst[e]];
-            r.target = (near_edge(e) ? kT32Near : (uint32_t)cslot[g->dst[e]]) |
-                       (first32[e] ? kT32First : 0u);
-            std::memcpy(buf.data() + at, &r, sizeof r);
-            for (int c = 2; c < C; c++) {
-                const uint32_t t = tclamp(e, c);
-                std::memcpy(buf.data() + at + 16 + 4 * (c - 2), &t, 4);
-            }
-        };
-        L->blob32.clear();
-        L->heavy32.clear();
-        L->tiles32.clear();
-        L->stage_bytes32 = 0;
-        size_t t_start = 0;
-        int32_t t_pos = 0;
-        auto open32 = [&](int32_t k) {
-            t_start = L->blob32.size();
-            t_pos = k;
-            L->blob32.resize(t_start + kTileHeader, 0);
-        };
-        auto close32 = [&](int32_t k_end) {
-            TileDesc td{};
-            td.byte_off = (int64_t)t_start;
-            td.bytes = (int32_t)(L->blob32.size() - t_start);
-            td.pos_begin = t_pos;
-            td.pos_end = k_end;
-            int32_t hdr[4] = {t_pos, k_end, td.bytes, 0};
-            std::memcpy(L->blob32.data() + t_start, hdr, 16);
-            L->tiles32.push_back(td);
-            L->stage_bytes32 = std::max(L->stage_bytes32, td.bytes);
-        };
-        open32(0);
-        for (int32_t k = 0; k < n; k++) {
-            const int32_t u = order[k];
-            const int64_t nout = g->out_off[u + 1] - g->out_off[u];
-            const bool heavy = nout * es32 > kMaxInlineBytes;
-            const size_t rec_bytes = 16 + (heavy ? 16 : (size_t)nout * es32);
-            if (k > t_pos && L->blob32.size() - t_start + rec_bytes > (size_t)kTileTarget) {
-                close32(k);
-                open32(k);
-            }
-            OpRec32 op;
-            op.p = (uint32_t)std::min<int64_t>(g->p[u], kSat32);
-            op.cold_slot = cslot[u];
-            const int32_t ahead = k + kPrefetchDist;
-            op.pf_slot = ahead < n ? cslot[order[ahead]] : -1;
-            op.nout = (heavy ? kOpHeavy : (uint32_t)nout) | (has_near[u] ? kOp32HasNear : 0u);
-            size_t at = L->blob32.size();
-            L->blob32.resize(at + 16);
-            std::memcpy(L->blob32.data() + at, &op, 16);
-            if (heavy) {
-                ExtRec ext{(int64_t)L->heavy32.size(), nout};
-                at = L->blob32.size();
-                L->blob32.resize(at + 16);
-                std::memcpy(L->blob32.data() + at, &ext, 16);
-                for (int64_t i = g->out_off[u]; i < g->out_off[u + 1]; i++) put_edge32(L->heavy32, sorted[i]);
-            } else {
-                for (int64_t i = g->out_off[u]; i < g->out_off[u + 1]; i++) put_edge32(L->blob32, sorted[i]);
-            }
-        }
-        close32(n);
-    }
-    // order-move helpers
-    L->adj_next.assign(n, 0);
-    for (int32_t k = 0; k + 1 < n; k++) {
-        const int32_t u = order[k], w = order[k + 1];
-        for (int64_t i = g->out_off[u]; i < g->out_off[u + 1]; i++)
-            if (g->dst[g->out_edges[i]] == w) L->adj_next[k] = 1;
-    }
-    L->allowed_pos.resize(n);
-    for (int32_t k = 0; k < n; k++) L->allowed_pos[k] = g->allowed[order[k]];
-    if (use_cache) {
-        g->cache.push_front(L);
-        while (g->cache.size() > 8) g->cache.pop_back();
-    }
-    out = L;
-    return PESTO_OK;
-}
-
 template <class T>
 static cudaError_t upload_vec(DevBuf &d, const std::vector<T> &v) {
     cudaError_t e = d.ensure(std::max<size_t>(v.size() * sizeof(T), 16));
@@ -383,6 +119,10 @@ pesto_status upload_layout(pesto_graph *g, Layout &L) {
     if ((e = upload_vec(L.d_blob32, L.blob32)) != cudaSuccess) return cuda_fail(e, "upload layout");
     if ((e = upload_vec(L.d_heavy32, L.heavy32)) != cudaSuccess) return cuda_fail(e, "upload layout");
     if ((e = upload_vec(L.d_tiles32, L.tiles32)) != cudaSuccess) return cuda_fail(e, "upload layout");
+    if ((e = upload_vec(L.d_order, L.order)) != cudaSuccess) return cuda_fail(e, "upload layout");
+    if ((e = upload_vec(L.d_op_off32, L.op_off32)) != cudaSuccess) return cuda_fail(e, "upload layout");
+    if ((e = upload_vec(L.d_pin_off, L.pin_off)) != cudaSuccess) return cuda_fail(e, "upload layout");
+    if ((e = upload_vec(L.d_pin_ref, L.pin_ref)) != cudaSuccess) return cuda_fail(e, "upload layout");
     L.on_device = true;
     std::vector<BaseLayoutDev> view{layout_view(L)};
     if ((e = upload_vec(L.d_view, view)) != cudaSuccess) return cuda_fail(e, "upload layout");
@@ -405,6 +145,10 @@ BaseLayoutDev layout_view(const Layout &L) {
     v.heavy32 = L.d_heavy32.as<uint8_t>();
     v.n_tiles32 = (int32_t)L.tiles32.size();
     v.W32 = L.W32;
+    v.order = L.d_order.as<int32_t>();
+    v.op_off32 = L.d_op_off32.as<uint32_t>();
+    v.pin_off = L.d_pin_off.as<uint32_t>();
+    v.pin_ref = L.d_pin_ref.as<uint32_t>();
     return v;
 }
 
@@ -415,6 +159,7 @@ void fill_eval_common(const pesto_graph *g, EvalParams &p) {
     p.planes = g->planes;
     p.words = g->words;
     p.edge_stride = edge_stride_for(g->n_classes);
+    p.edge_stride32 = edge_stride32_for(g->n_classes);
     p.n_classes = g->n_classes;
     std::memcpy(p.link_class, g->link_class, 64);
     p.all_allowed = g->all_allowed ? 1 : 0;
@@ -546,6 +291,14 @@ pesto_status pesto_graph_create(const pesto_graph_desc *d, pesto_graph **out) {
             for (int64_t i = g->out_off[q[h]]; i < g->out_off[q[h] + 1]; i++)
                 if (--deg[g->dst[g->out_edges[i]]] == 0) q.push_back(g->dst[g->out_edges[i]]);
         if ((int32_t)q.size() != n) return fail(PESTO_ECYCLE, "graph has a cycle");
+    }
+    g->in_off.assign((size_t)n + 1, 0);
+    for (int64_t e = 0; e < m; e++) g->in_off[g->dst[e] + 1]++;
+    for (int32_t v = 0; v < n; v++) g->in_off[v + 1] += g->in_off[v];
+    g->in_edges.resize(m);
+    {
+        std::vector<int64_t> fill(g->in_off.begin(), g->in_off.end() - 1);
+        for (int64_t e = 0; e < m; e++) g->in_edges[fill[g->dst[e]]++] = e;
     }
     {
         int64_t total = 0;

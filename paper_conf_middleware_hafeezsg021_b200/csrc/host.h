@@ -54,10 +54,11 @@ struct Layout {
     int32_t W32 = 0, stage_bytes32 = 0;
     std::vector<uint8_t> blob32, heavy32;
     std::vector<TileDesc> tiles32;
+    std::vector<uint32_t> op_off32, pin_off, pin_ref;   // K4 patch index into blob32/heavy32
     int64_t comm_gen = -1;
     // device copies
-    DevBuf d_blob, d_heavy, d_tiles, d_pos, d_adj, d_allowed_pos, d_view;
-    DevBuf d_blob32, d_heavy32, d_tiles32;
+    DevBuf d_blob, d_heavy, d_tiles, d_pos, d_adj, d_allowed_pos, d_view, d_order;
+    DevBuf d_blob32, d_heavy32, d_tiles32, d_op_off32, d_pin_off, d_pin_ref;
     bool on_device = false;
 };
 
@@ -73,6 +74,8 @@ struct pesto_graph {
     bool all_allowed = true;
     std::vector<int64_t> out_off;         // CSR of out-edges by producer (edge ids)
     std::vector<int64_t> out_edges;
+    std::vector<int64_t> in_off;          // CSR of in-edges by consumer, ascending edge id
+    std::vector<int64_t> in_edges;
     std::vector<int32_t> indeg;
     // comm model per directed link a*D+b
     std::vector<int64_t> beta0, beta1;
@@ -99,8 +102,9 @@ struct pesto_graph {
 namespace pesto {
 // graph.cpp helpers used by search.cpp
 pesto_status ensure_comm_tables(pesto_graph *g);
+// x_op (device code per op id, nullable) is embedded in the eval32 records (search bases)
 pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<Layout> &out,
-                          bool use_cache);
+                          bool use_cache, const uint8_t *x_op = nullptr);
 pesto_status upload_layout(pesto_graph *g, Layout &L);
 BaseLayoutDev layout_view(const Layout &L);
 void fill_eval_common(const pesto_graph *g, EvalParams &p);

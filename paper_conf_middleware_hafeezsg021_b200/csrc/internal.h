@@ -29,6 +29,10 @@ struct BaseLayoutDev {
     const uint8_t *heavy32;
     int32_t n_tiles32;
     int32_t W32;                // cold slots
+    const int32_t *order;       // [n] op id at each position
+    const uint32_t *op_off32;   // [n] byte offset of the op record at each position (blob32)
+    const uint32_t *pin_off;    // [n+1] CSR: edge records whose successor is at each position
+    const uint32_t *pin_ref;    // byte offsets (| kPinHeavy for the out-of-line array)
 };
 
 struct EvalParams {
@@ -60,7 +64,7 @@ struct EvalParams {
     int64_t group_begin, groups_per_base, tasks_per_base, n_tasks;
     // eval32 (32-bit saturating) state and its explicit-mode fixup list
     uint32_t *state32;                  // [cta][warp][W32_max][32] cold slots
-    int32_t max_W32, stage_bytes32;
+    int32_t max_W32, stage_bytes32, edge_stride32;
     int32_t *flag_list, *flag_count;    // saturated candidates, re-evaluated by eval64
     // search: base b runs on eval32 iff base_mk[b] < kSat32 (gate 1), on eval64 iff not (gate 2)
     const int64_t *base_mk;
@@ -92,6 +96,7 @@ struct CommitParams {
     const uint64_t *keys;
     int64_t *base_mk;
     int32_t *swap_out;                  // [P] committed swap position or -1
+    int32_t patch32;                    // eval32 records carry base codes: patch them too
 };
 
 // launchers (kernels.cu / eval32.cu); they return the launch error, if any.

@@ -67,10 +67,10 @@ template <int MODE, int PL>
 struct Placement {
     // explicit rows (MODE 0): bit-sliced words of this warp's 32 candidates
     const uint32_t *pl;
-    // search (MODE 1): base bits + warp-private "touched" bitmap + this lane's move
+    // search (MODE 1): base bits + the group's region + this lane's move
     const uint32_t *bits;
-    const uint32_t *touched;
     const uint8_t *allowed_pos;
+    int32_t rc, rlen;
     int words;
     int all_allowed;
     LaneMove mv;
@@ -81,14 +81,12 @@ struct Placement {
         // MODE 0: this warp's group words, bit `lane`; MODE 2 (fixup list): each lane's own
         // candidate, i.e. its group's words (per-lane pointer) and bit (lane field = bit index)
         if (MODE != 1) return planes_dev_at<PL>(pl, q, lane, dmax);
-        {
-            int x = ldg_bits_dev_at<PL>(bits, words, q);
-            if ((touched[q >> 5] >> (q & 31)) & 1u) {          // warp-uniform branch
-                unsigned aq = all_allowed ? 0xFFu : (unsigned)__ldg(allowed_pos + q);
-                x = apply_lane(mv, q, x, aq);
-            }
-            return x;
+        int x = ldg_bits_dev_at<PL>(bits, words, q);
+        if ((uint32_t)(q - rc) < (uint32_t)rlen) {            // warp-uniform branch
+            unsigned aq = all_allowed ? 0xFFu : (unsigned)__ldg(allowed_pos + q);
+            x = apply_lane(mv, q, x, aq);
         }
+        return x;
     }
 };
 
@@ -222,8 +220,6 @@ eval_kernel(const EvalParams P) {
     uint8_t *cur = align16(reinterpret_cast<uint8_t *>(empty + kStages));
     uint8_t *lclass = cur;
     cur = align16(cur + 64);
-    uint32_t *touched_all = reinterpret_cast<uint32_t *>(cur);
-    if (MODE == 1) cur = align16(cur + (size_t)kWarps * P.words * 4);
     int64_t *dstate = reinterpret_cast<int64_t *>(cur);
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -274,7 +270,6 @@ eval_kernel(const EvalParams P) {
     cx.edge_stride = P.edge_stride;
     cx.D = P.D;
     cx.R = P.state + ((int64_t)(blockIdx.x * kWarps + warp) * P.max_W) * 32 + lane;
-    uint32_t *touched = touched_all + (size_t)warp * P.words;
 
     using StateT = typename std::conditional<PL == 1, RegState, SmemState>::type;
     StateT st;
@@ -318,29 +313,28 @@ eval_kernel(const EvalParams P) {
             active = g < P.group_begin + P.groups_per_base;
             const int breal = P.b_offset + bl;
             const uint64_t cb = ctr_base_of(P.step, P.P_total, breal);
+            const Region rg = decode_region(P.seed, cb, g, P.n);
+            place.rc = rg.c;
+            place.rlen = rg.len;
             place.bits = B->bits;
-            place.touched = touched;
             place.allowed_pos = B->allowed_pos;
             const uint8_t *adj = B->adj_next;
-            ks = active ? decode_swap(P.seed, cb, g, P.n, P.mix[3],
+            ks = active ? decode_swap(P.seed, cb, g, P.n, P.mix[3], rg,
                                       [&](int32_t k) { return __ldg(adj + k) != 0; })
                         : -1;
             const bool in_range = active && j >= P.j_begin && j < P.j_end;
-            const int32_t *movable = P.movable;
-            const int32_t *pos_of = B->pos_of;
+            const int32_t *ord = B->order;
             const uint32_t *bits = B->bits;
             const uint8_t *aop = P.allowed_op;
             const int words = P.words;
             place.mv = in_range
-                ? decode_lane(P.seed, cb, j, ks >= 0 && lane == 0, P.n, P.D, P.mix, P.n_movable,
-                              [&](int32_t i) { return __ldg(movable + i); },
-                              [&](int32_t op) { return __ldg(pos_of + op); },
+                ? decode_lane(P.seed, cb, j, ks >= 0 && lane == 0, P.D, P.mix, rg,
+                              [&](int32_t q) { return __ldg(ord + q); },
                               [&](int32_t q) { return ldg_bits_dev_at<PL>(bits, words, q); },
                               [&](int32_t op) { return (unsigned)__ldg(aop + op); })
                 : no_move();
             valid = in_range && place.mv.kind != kMoveInvalid;
-            if (place.mv.kind == kMoveInvalid) place.mv.kind = kMoveNone;
-            build_touched(touched, P.words, place.mv, lane);
+            if (place.mv.kind == kMoveInvalid) place.mv = no_move();
         }
         st.init(P.D);
 
@@ -526,19 +520,36 @@ __global__ void commit_kernel(const CommitParams P) {
     uint32_t *bits = P.bits + (size_t)b * PL * P.words;
     const uint64_t cb = ctr_base_of(P.step, P.P, b);
     const uint8_t *adj = B.adj_next;
-    const int32_t ks = decode_swap(P.seed, cb, j >> 5, P.n, P.mix[3],
+    const Region rg = decode_region(P.seed, cb, j >> 5, P.n);
+    const int32_t ks = decode_swap(P.seed, cb, j >> 5, P.n, P.mix[3], rg,
                                    [&](int32_t k) { return adj[k] != 0; });
     const int words = P.words;
     const LaneMove mv = decode_lane(
-        P.seed, cb, j, ks >= 0 && (j & 31) == 0, P.n, P.D, P.mix, P.n_movable,
-        [&](int32_t i) { return P.movable[i]; }, [&](int32_t op) { return B.pos_of[op]; },
+        P.seed, cb, j, ks >= 0 && (j & 31) == 0, P.D, P.mix, rg,
+        [&](int32_t q) { return B.order[q]; },
         [&](int32_t q) { return get_dev_at<PL>(bits, words, q); },
         [&](int32_t op) { return (unsigned)P.allowed_op[op]; });
+    // the base code is also embedded in the eval32 records that name position q: the op's
+    // own record and every edge record whose successor sits at q
+    uint8_t *blob32 = const_cast<uint8_t *>(B.blob32);
+    uint8_t *heavy32 = const_cast<uint8_t *>(B.heavy32);
+    auto set_dev = [&](int32_t q, int x) {
+        set_dev_at<PL>(bits, words, q, x);
+        if (!P.patch32) return;
+        uint32_t *nout = reinterpret_cast<uint32_t *>(blob32 + B.op_off32[q]) + 3;
+        *nout = (*nout & ~(7u << kOpXShift)) | ((uint32_t)x << kOpXShift);
+        for (uint32_t i = B.pin_off[q]; i < B.pin_off[q + 1]; i++) {
+            const uint32_t ref = B.pin_ref[i];
+            uint8_t *base = (ref & kPinHeavy) ? heavy32 : blob32;
+            uint32_t *succ = reinterpret_cast<uint32_t *>(base + (ref & ~kPinHeavy)) + 1;
+            *succ = (*succ & ~(7u << kSuccXShift)) | ((uint32_t)x << kSuccXShift);
+        }
+    };
     if (mv.kind == kMoveFlip) {
-        for (int f = 0; f < mv.nflip; f++) set_dev_at<PL>(bits, words, mv.fpos[f], mv.fdev[f]);
+        for (int f = 0; f < mv.nflip; f++) set_dev(mv.fpos[f], mv.fdev[f]);
     } else if (mv.kind == kMoveWindow) {
         for (int32_t q = mv.ws; q < mv.ws + mv.wl; q++)
-            if ((B.allowed_pos[q] >> mv.wd) & 1u) set_dev_at<PL>(bits, words, q, mv.wd);
+            if ((B.allowed_pos[q] >> mv.wd) & 1u) set_dev(q, mv.wd);
     }
     if (ks >= 0) {                       // ops at ks and ks+1 exchange positions
         const int a = get_dev_at<PL>(bits, words, ks), c = get_dev_at<PL>(bits, words, ks + 1);

@@ -1,0 +1,303 @@
+// layout.cpp -- position-space layouts of one schedule order.
+//
+// For an order pi (the per-device op order) every op is relabelled by its
+// position.  Two record streams are emitted, one per kernel:
+//   eval64: ready-time slots in global memory, interval-coloured (one slot per consumer, live
+//           from its first producer to one position past itself -- DESIGN.md §3.3);
+//   eval32: near/far split with the base placement embedded in the records
+//           (search bases only; patched in place by K4 when a placement move is committed).
+// Everything is O(n + m): counting sorts by position, flat CSR arrays, one pass per field.
+#include <algorithm>
+#include <cstring>
+#include <string>
+
+#include "host.h"
+
+namespace pesto {
+
+static constexpr int kMaxInlineBytes = 2048;
+
+namespace {
+
+// LIFO interval colouring: interval of consumer w is [start[w], end[w]] (end = pos(w) + 1),
+// w without interval has start < 0.  Returns the slot count.
+int32_t colour_intervals(int32_t n, const std::vector<int32_t> &start, const std::vector<int32_t> &pos,
+                         std::vector<int32_t> &slot) {
+    std::vector<int32_t> s_off(n + 1, 0), f_off(n + 1, 0);
+    for (int32_t w = 0; w < n; w++) {
+        if (start[w] < 0) continue;
+        s_off[start[w] + 1]++;
+        if (pos[w] + 2 < n) f_off[pos[w] + 2 + 1]++;
+    }
+    for (int32_t k = 0; k < n; k++) { s_off[k + 1] += s_off[k]; f_off[k + 1] += f_off[k]; }
+    std::vector<int32_t> s_list(s_off[n]), f_list(f_off[n]);
+    {
+        std::vector<int32_t> sf(s_off.begin(), s_off.end() - 1), ff(f_off.begin(), f_off.end() - 1);
+        // consumers in position order so the colouring is deterministic
+        for (int32_t w = 0; w < n; w++) {
+            if (start[w] < 0) continue;
+            s_list[sf[start[w]]++] = w;
+            if (pos[w] + 2 < n) f_list[ff[pos[w] + 2]++] = w;
+        }
+    }
+    slot.assign(n, -1);
+    std::vector<int32_t> stack;
+    stack.reserve(1024);
+    int32_t W = 0;
+    for (int32_t k = 0; k < n; k++) {
+        for (int32_t i = f_off[k]; i < f_off[k + 1]; i++) stack.push_back(slot[f_list[i]]);
+        for (int32_t i = s_off[k]; i < s_off[k + 1]; i++) {
+            const int32_t w = s_list[i];
+            if (!stack.empty()) { slot[w] = stack.back(); stack.pop_back(); }
+            else slot[w] = W++;
+        }
+    }
+    return W;
+}
+
+struct TileWriter {
+    std::vector<uint8_t> &blob;
+    std::vector<TileDesc> &tiles;
+    int32_t &stage_bytes;
+    size_t start = 0;
+    int32_t pos0 = 0;
+    TileWriter(std::vector<uint8_t> &b, std::vector<TileDesc> &t, int32_t &sb) : blob(b), tiles(t), stage_bytes(sb) {}
+    void open(int32_t k) {
+        start = blob.size();
+        pos0 = k;
+        blob.resize(start + kTileHeader, 0);
+    }
+    void close(int32_t k_end) {
+        TileDesc td{};
+        td.byte_off = (int64_t)start;
+        td.bytes = (int32_t)(blob.size() - start);
+        td.pos_begin = pos0;
+        td.pos_end = k_end;
+        const int32_t hdr[4] = {pos0, k_end, td.bytes, 0};
+        std::memcpy(blob.data() + start, hdr, 16);
+        tiles.push_back(td);
+        stage_bytes = std::max(stage_bytes, td.bytes);
+    }
+    // start a new tile before an op whose records take `rec_bytes` if the current one is full
+    void maybe_cut(int32_t k, size_t rec_bytes) {
+        if (k > pos0 && blob.size() - start + rec_bytes > (size_t)kTileTarget) {
+            close(k);
+            open(k);
+        }
+    }
+};
+
+template <class T>
+void append(std::vector<uint8_t> &buf, const T &v) {
+    const size_t at = buf.size();
+    buf.resize(at + sizeof(T));
+    std::memcpy(buf.data() + at, &v, sizeof(T));
+}
+
+}  // namespace
+
+pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<Layout> &out,
+                          bool use_cache, const uint8_t *x_op) {
+    pesto_status s = ensure_comm_tables(g);
+    if (s) return s;
+    const int32_t n = g->n;
+    const int64_t m = g->m;
+    if (!order) return fail(PESTO_EINVAL, "order is NULL");
+    if (use_cache && !x_op) {
+        for (auto it = g->cache.begin(); it != g->cache.end(); ++it) {
+            if ((*it)->comm_gen == g->comm_gen &&
+                std::memcmp((*it)->order.data(), order, (size_t)n * 4) == 0) {
+                out = *it;
+                g->cache.splice(g->cache.begin(), g->cache, it);
+                return PESTO_OK;
+            }
+        }
+    }
+    auto L = std::make_shared<Layout>();
+    L->comm_gen = g->comm_gen;
+    L->order.assign(order, order + n);
+    L->pos.assign(n, -1);
+    std::vector<int32_t> &pos = L->pos;
+    for (int32_t k = 0; k < n; k++) {
+        const int32_t v = order[k];
+        if (v < 0 || v >= n || pos[v] != -1) return fail(PESTO_ENOTTOPO, "order is not a permutation");
+        pos[v] = k;
+    }
+    for (int64_t e = 0; e < m; e++)
+        if (pos[g->src[e]] >= pos[g->dst[e]])
+            return fail(PESTO_ENOTTOPO, "order violates edge " + std::to_string(e));
+
+    // out-edges of every producer sorted by (successor position, edge index) -- the FCFS tie
+    // order of reading R3 -- by one pass over consumers in position order (in-edges of a
+    // consumer are listed by edge index)
+    std::vector<int64_t> sorted(m);
+    {
+        std::vector<int64_t> fill(g->out_off.begin(), g->out_off.end() - 1);
+        for (int32_t q = 0; q < n; q++) {
+            const int32_t w = order[q];
+            for (int64_t i = g->in_off[w]; i < g->in_off[w + 1]; i++) {
+                const int64_t e = g->in_edges[i];
+                sorted[fill[g->src[e]]++] = e;
+            }
+        }
+    }
+    auto succ_pos = [&](int64_t e) { return pos[g->dst[e]]; };
+    const int C = g->n_classes;
+
+    // ---------------- eval64 stream ----------------
+    {
+        std::vector<int32_t> first(n, -1);
+        for (int64_t e = 0; e < m; e++) {
+            const int32_t w = g->dst[e], ps = pos[g->src[e]];
+            if (first[w] < 0 || ps < first[w]) first[w] = ps;
+        }
+        std::vector<int32_t> slot;
+        L->W = std::max(colour_intervals(n, first, pos, slot), 1);
+        std::vector<uint8_t> seen(n, 0), first_flag(m, 0);
+        for (int32_t k = 0; k < n; k++) {
+            const int32_t u = order[k];
+            for (int64_t i = g->out_off[u]; i < g->out_off[u + 1]; i++) {
+                const int64_t e = sorted[i];
+                if (!seen[g->dst[e]]) { seen[g->dst[e]] = 1; first_flag[e] = 1; }
+            }
+        }
+        const int es = edge_stride_for(C);
+        L->blob.clear();
+        L->heavy.clear();
+        L->tiles.clear();
+        L->blob.reserve((size_t)n * 16 + (size_t)m * es + 64 * kTileHeader);
+        auto put_edge = [&](std::vector<uint8_t> &buf, int64_t e) {
+            const size_t at = buf.size();
+            buf.resize(at + es, 0);
+            EdgeRec r;
+            r.t0 = g->t_class[(size_t)e * C];
+            r.succ_pos = succ_pos(e);
+            r.slot = (uint32_t)slot[g->dst[e]] | (first_flag[e] ? kEdgeFirst : 0u);
+            std::memcpy(buf.data() + at, &r, sizeof r);
+            for (int c = 1; c < C; c++)
+                std::memcpy(buf.data() + at + 16 + 8 * (c - 1), &g->t_class[(size_t)e * C + c], 8);
+        };
+        TileWriter tw(L->blob, L->tiles, L->stage_bytes);
+        tw.open(0);
+        for (int32_t k = 0; k < n; k++) {
+            const int32_t u = order[k];
+            const int64_t nout = g->out_off[u + 1] - g->out_off[u];
+            const bool heavy = nout * es > kMaxInlineBytes;
+            tw.maybe_cut(k, 16 + (heavy ? 16 : (size_t)nout * es));
+            OpRec op;
+            op.p = g->p[u];
+            op.in_slot = slot[u];
+            op.nout = heavy ? kOpHeavy : (uint32_t)nout;
+            append(L->blob, op);
+            if (heavy) {
+                append(L->blob, ExtRec{(int64_t)L->heavy.size(), nout});
+                for (int64_t i = g->out_off[u]; i < g->out_off[u + 1]; i++) put_edge(L->heavy, sorted[i]);
+            } else {
+                for (int64_t i = g->out_off[u]; i < g->out_off[u + 1]; i++) put_edge(L->blob, sorted[i]);
+            }
+        }
+        tw.close(n);
+    }
+
+    // ---------------- eval32 stream ----------------
+    if (g->eligible32) {
+        auto near_edge = [&](int64_t e) { return pos[g->dst[e]] - pos[g->src[e]] <= kNearDelta; };
+        std::vector<int32_t> first_far(n, -1);
+        std::vector<uint8_t> has_near(n, 0);
+        for (int64_t e = 0; e < m; e++) {
+            const int32_t w = g->dst[e];
+            if (near_edge(e)) { has_near[w] = 1; continue; }
+            const int32_t ps = pos[g->src[e]];
+            if (first_far[w] < 0 || ps < first_far[w]) first_far[w] = ps;
+        }
+        std::vector<int32_t> cslot;
+        L->W32 = std::max(colour_intervals(n, first_far, pos, cslot), 1);
+        std::vector<uint8_t> seen_near(n, 0), seen_far(n, 0), first32(m, 0);
+        for (int32_t k = 0; k < n; k++) {
+            const int32_t u = order[k];
+            for (int64_t i = g->out_off[u]; i < g->out_off[u + 1]; i++) {
+                const int64_t e = sorted[i];
+                const int32_t w = g->dst[e];
+                uint8_t &seen = near_edge(e) ? seen_near[w] : seen_far[w];
+                if (!seen) { seen = 1; first32[e] = 1; }
+            }
+        }
+        const int es32 = edge_stride32_for(C);
+        auto t32 = [&](int64_t e, int c) { return (uint32_t)g->t_class[(size_t)e * C + c]; };
+        auto xcode = [&](int32_t op) { return x_op ? (uint32_t)(x_op[op] & 7u) : 0u; };
+        L->blob32.clear();
+        L->heavy32.clear();
+        L->tiles32.clear();
+        L->stage_bytes32 = 0;
+        L->blob32.reserve((size_t)n * 16 + (size_t)m * es32 + 64 * kTileHeader);
+        L->op_off32.assign(n, 0);
+        // patch index: locations of every edge record by successor position
+        L->pin_off.assign((size_t)n + 1, 0);
+        L->pin_ref.assign(m, 0);
+        for (int64_t e = 0; e < m; e++) L->pin_off[pos[g->dst[e]] + 1]++;
+        for (int32_t q = 0; q < n; q++) L->pin_off[q + 1] += L->pin_off[q];
+        std::vector<uint32_t> pfill(L->pin_off.begin(), L->pin_off.end() - 1);
+        auto put_edge32 = [&](std::vector<uint8_t> &buf, int64_t e, bool heavy) {
+            const size_t at = buf.size();
+            buf.resize(at + es32, 0);
+            EdgeRec32 r;
+            r.t0 = t32(e, 0);
+            r.t1 = C > 1 ? t32(e, 1) : 0u;
+            const int32_t w = g->dst[e];
+            r.succ_pos = (int32_t)((uint32_t)pos[w] | (xcode(w) << kSuccXShift));
+            r.target = (near_edge(e) ? kT32Near : (uint32_t)cslot[w]) | (first32[e] ? kT32First : 0u);
+            std::memcpy(buf.data() + at, &r, sizeof r);
+            for (int c = 2; c < C; c++) {
+                const uint32_t t = t32(e, c);
+                std::memcpy(buf.data() + at + 16 + 4 * (c - 2), &t, 4);
+            }
+            L->pin_ref[pfill[pos[w]]++] = (uint32_t)at | (heavy ? kPinHeavy : 0u);
+        };
+        TileWriter tw(L->blob32, L->tiles32, L->stage_bytes32);
+        tw.open(0);
+        for (int32_t k = 0; k < n; k++) {
+            const int32_t u = order[k];
+            const int64_t b0 = g->out_off[u], b1 = g->out_off[u + 1];
+            const int64_t nout = b1 - b0;
+            const bool heavy = nout * es32 > kMaxInlineBytes;
+            tw.maybe_cut(k, 16 + (heavy ? 16 : (size_t)nout * es32));
+            bool adj = false;                   // feeds two adjacent positions (swap reorder)
+            for (int64_t i = b0 + 1; i < b1; i++)
+                if (succ_pos(sorted[i]) == succ_pos(sorted[i - 1]) + 1) adj = true;
+            OpRec32 op;
+            op.p = (uint32_t)g->p[u];
+            op.cold_next = k + 1 < n ? cslot[order[k + 1]] : -1;
+            const int32_t ahead = k + kPrefetchDist;
+            op.pf_slot = ahead < n ? cslot[order[ahead]] : -1;
+            op.nout = (heavy ? kOpHeavy : (uint32_t)nout) | (has_near[u] ? kOp32HasNear : 0u) |
+                      (adj ? kOpAdj : 0u) | (xcode(u) << kOpXShift);
+            L->op_off32[k] = (uint32_t)L->blob32.size();
+            append(L->blob32, op);
+            if (heavy) {
+                append(L->blob32, ExtRec{(int64_t)L->heavy32.size(), nout});
+                for (int64_t i = b0; i < b1; i++) put_edge32(L->heavy32, sorted[i], true);
+            } else {
+                for (int64_t i = b0; i < b1; i++) put_edge32(L->blob32, sorted[i], false);
+            }
+        }
+        tw.close(n);
+    }
+
+    // order-move helpers
+    L->adj_next.assign(n, 0);
+    for (int32_t k = 0; k + 1 < n; k++) {
+        const int32_t u = order[k], w = order[k + 1];
+        for (int64_t i = g->out_off[u]; i < g->out_off[u + 1]; i++)
+            if (g->dst[g->out_edges[i]] == w) { L->adj_next[k] = 1; break; }
+    }
+    L->allowed_pos.resize(n);
+    for (int32_t k = 0; k < n; k++) L->allowed_pos[k] = g->allowed[order[k]];
+    if (use_cache && !x_op) {
+        g->cache.push_front(L);
+        while (g->cache.size() > 8) g->cache.pop_back();
+    }
+    out = L;
+    return PESTO_OK;
+}
+
+}  // namespace pesto

@@ -66,20 +66,25 @@ constexpr int kNearDelta = 12;
 constexpr int kRing = 16;                       // >= kNearDelta + 3 (swap margins)
 constexpr int kPrefetchDist = kNearDelta - 1;
 constexpr uint32_t kOp32HasNear = 1u << 24;     // OpRec32.nout: read the near ring
+constexpr int kOpXShift = 25;                   // OpRec32.nout bits 25-27: base device code
+constexpr uint32_t kOpAdj = 1u << 28;           // producer feeds two adjacent positions
+constexpr int kSuccXShift = 24;                 // EdgeRec32.succ_pos bits 24-26: base device
+constexpr uint32_t kSuccPosMask = (1u << 24) - 1;
+constexpr uint32_t kPinHeavy = 1u << 31;        // patch reference into the out-of-line array
 constexpr uint32_t kT32First = 1u << 31;        // EdgeRec32.target: first push into its slot
 constexpr uint32_t kT32Near = 1u << 30;         // push into the near ring (slot = succ & 15)
 constexpr uint32_t kT32SlotMask = (1u << 30) - 1;
 
 struct alignas(16) OpRec32 {
     uint32_t p;          // p_v (< kMaxDur32)
-    int32_t cold_slot;   // global slot holding far pushes into this op; -1 = none
+    int32_t cold_next;   // cold slot of the op at the next position (loaded one op ahead); -1
     int32_t pf_slot;     // cold slot of the op kPrefetchDist positions ahead; -1 = none
-    uint32_t nout;       // out-degree | kOp32HasNear | kOpHeavy
+    uint32_t nout;       // out-degree | kOp32HasNear | kOpAdj | base code << 25 | kOpHeavy
 };
 
 struct alignas(16) EdgeRec32 {
     uint32_t t0;         // transfer time, link class 0 (< kMaxDur32)
-    int32_t succ_pos;
+    int32_t succ_pos;    // successor position | its base code << 24
     uint32_t target;     // cold slot | kT32Near | kT32First
     uint32_t t1;         // link class 1; classes >= 2 follow in 4-byte words
 };

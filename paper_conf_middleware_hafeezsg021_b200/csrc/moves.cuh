@@ -48,25 +48,39 @@ struct LaneMove {
     int32_t ws, wl, wd;  // window: positions [ws, ws + wl) move to wd where allowed
 };
 
+constexpr int kRegion = 64;     // positions a group of 32 candidates may change (DESIGN §4 S2)
+
+// The group's region [c, c + len) of the base order.
+struct Region {
+    int32_t c, len;
+};
+PESTO_HD Region decode_region(uint64_t seed, uint64_t cb, int64_t group, int n) {
+    Region r;
+    r.c = (int32_t)(draw(seed, cb, group * 32, 13) % (uint64_t)n);
+    r.len = n - r.c < kRegion ? n - r.c : kRegion;
+    return r;
+}
+
 // Group (warp) order move: adjacent swap of positions (k, k+1) of the base order, or -1.
 // adj_next(k) must say whether an edge joins order[k] -> order[k+1].
 template <class AdjNext>
 PESTO_HD int32_t decode_swap(uint64_t seed, uint64_t cb, int64_t group, int n, int swap_pct,
-                             AdjNext adj_next) {
+                             Region rg, AdjNext adj_next) {
     if (group == 0 || swap_pct <= 0 || n < 2) return -1;
     int64_t j0 = group * 32;
     if ((int)(draw(seed, cb, j0, 15) % 100u) >= swap_pct) return -1;
-    int32_t k = (int32_t)(draw(seed, cb, j0, 14) % (uint64_t)(n - 1));
+    int32_t k = rg.c + (int32_t)(draw(seed, cb, j0, 14) % (uint64_t)rg.len);
+    if (k > n - 2) k = n - 2;
     return adj_next(k) ? -1 : k;
 }
 
-// Lane placement move of candidate j.  Callbacks:
-//   movable(i) -> op id of the i-th movable op;  pos_of(op) -> position in the base order;
-//   base_dev(pos) -> base device at a position;  allowed(op) -> device mask.
-template <class Movable, class PosOf, class BaseDev, class Allowed>
-PESTO_HD LaneMove decode_lane(uint64_t seed, uint64_t cb, int64_t j, bool pure_swap, int n, int D,
-                              const int32_t mix[4], int n_movable, Movable movable, PosOf pos_of,
-                              BaseDev base_dev, Allowed allowed) {
+// Lane placement move of candidate j inside region rg.  Callbacks:
+//   op_at(pos) -> op id at a position of the base order;  base_dev(pos) -> base device there;
+//   allowed(op) -> device mask.
+template <class OpAt, class BaseDev, class Allowed>
+PESTO_HD LaneMove decode_lane(uint64_t seed, uint64_t cb, int64_t j, bool pure_swap, int D,
+                              const int32_t mix[4], Region rg, OpAt op_at, BaseDev base_dev,
+                              Allowed allowed) {
     LaneMove mv;
     mv.kind = kMoveNone;
     mv.nflip = 0;
@@ -77,18 +91,19 @@ PESTO_HD LaneMove decode_lane(uint64_t seed, uint64_t cb, int64_t j, bool pure_s
     if (wsum <= 0) return mv;
     int r = (int)(draw(seed, cb, j, 0) % (uint64_t)wsum);
     if (r < mix[0] + mix[1]) {
-        if (n_movable == 0) { mv.kind = kMoveInvalid; return mv; }
         int flips = 1;
         if (r >= mix[0]) flips = 2 + (int)(draw(seed, cb, j, 1) % 3u);
         mv.kind = kMoveFlip;
         mv.nflip = flips;
         for (int q = 0; q < flips; q++) {
-            int32_t op = movable((int32_t)(draw(seed, cb, j, 2 + 2 * q) % (uint64_t)n_movable));
-            int32_t pos = pos_of(op);
+            int32_t pos = rg.c + (int32_t)(draw(seed, cb, j, 2 + 2 * q) % (uint64_t)rg.len);
+            int32_t op = op_at(pos);
+            const unsigned am = allowed(op) & ((1u << D) - 1u);
+            if (popc32(am) < 2) { mv.kind = kMoveInvalid; return mv; }   // op cannot move
             int cur = base_dev(pos);
             for (int e = 0; e < q; e++)
                 if (mv.fpos[e] == pos) cur = mv.fdev[e];      // device after earlier flips
-            unsigned msk = allowed(op) & ((1u << D) - 1u) & ~(1u << cur);
+            unsigned msk = am & ~(1u << cur);
             int na = popc32(msk);
             int pick = (int)(draw(seed, cb, j, 3 + 2 * q) % (uint64_t)na);
             int dev = 0;
@@ -103,9 +118,9 @@ PESTO_HD LaneMove decode_lane(uint64_t seed, uint64_t cb, int64_t j, bool pure_s
         }
     } else {
         mv.kind = kMoveWindow;
-        int32_t s = (int32_t)(draw(seed, cb, j, 2) % (uint64_t)n);
+        int32_t s = rg.c + (int32_t)(draw(seed, cb, j, 2) % (uint64_t)rg.len);
         int32_t len = 1 + (int32_t)(draw(seed, cb, j, 3) % 64u);
-        if (s + len > n) len = n - s;
+        if (s + len > rg.c + rg.len) len = rg.c + rg.len - s;
         mv.ws = s;
         mv.wl = len;
         mv.wd = (int32_t)(draw(seed, cb, j, 4) % (uint64_t)D);

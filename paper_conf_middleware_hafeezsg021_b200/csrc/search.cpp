@@ -162,6 +162,22 @@ pesto_status upload_bits(pesto_search *s, int b, const uint8_t *x_op) {
     return e == cudaSuccess ? PESTO_OK : cuda_fail(e, "upload base placement");
 }
 
+// the base placement by op id, from the device bit planes (position space of order[b])
+pesto_status download_x(pesto_search *s, int b, uint8_t *x_op) {
+    pesto_graph *g = s->g;
+    std::vector<uint32_t> bits((size_t)g->planes * g->words);
+    cudaError_t e = cudaMemcpy(bits.data(), s->d_bits.as<uint32_t>() + (size_t)b * bits.size(),
+                               bits.size() * 4, cudaMemcpyDeviceToHost);
+    if (e != cudaSuccess) return cuda_fail(e, "read placement");
+    for (int32_t q = 0; q < g->n; q++) {
+        int x = 0;
+        for (int k = 0; k < g->planes; k++)
+            x |= (int)((bits[(size_t)k * g->words + (q >> 5)] >> (q & 31)) & 1u) << k;
+        x_op[s->order[b][q]] = (uint8_t)x;
+    }
+    return PESTO_OK;
+}
+
 }  // namespace
 
 extern "C" {
@@ -213,7 +229,8 @@ pesto_status pesto_search_create(pesto_graph *g, const pesto_search_desc *d, pes
         return cuda_fail(e, "allocate");
     for (int b = 0; b < s->P; b++) {
         s->order[b].assign(d->base_order + (size_t)b * n, d->base_order + (size_t)(b + 1) * n);
-        pesto_status rc = build_layout(g, s->order[b].data(), s->layouts[b], false);
+        pesto_status rc = build_layout(g, s->order[b].data(), s->layouts[b], false,
+                                       d->base_x + (size_t)b * n);
         if (rc) return rc;
         if ((rc = upload_layout(g, *s->layouts[b]))) return rc;
         if ((rc = upload_bits(s.get(), b, d->base_x + (size_t)b * n))) return rc;
@@ -309,6 +326,7 @@ pesto_status pesto_search_commit(pesto_search *s, void *stream) {
     cp.keys = s->d_keys.as<uint64_t>();
     cp.base_mk = s->d_mk.as<int64_t>();
     cp.swap_out = s->d_swap.as<int32_t>();
+    cp.patch32 = g->eligible32 ? 1 : 0;
     cudaError_t e = launch_commit(cp, st);
     if (e != cudaSuccess) return cuda_fail(e, "launch commit");
     s->step++;
@@ -325,8 +343,10 @@ pesto_status pesto_search_commit(pesto_search *s, void *stream) {
             const int32_t k = s->h_swap[b];
             if (k < 0) continue;
             std::swap(s->order[b][k], s->order[b][k + 1]);
-            pesto_status rc = build_layout(g, s->order[b].data(), s->layouts[b], false);
+            std::vector<uint8_t> x_op(g->n);
+            pesto_status rc = download_x(s, b, x_op.data());      // K4 already swapped the bits
             if (rc) return rc;
+            if ((rc = build_layout(g, s->order[b].data(), s->layouts[b], false, x_op.data()))) return rc;
             if ((rc = upload_layout(g, *s->layouts[b]))) return rc;
             changed = true;
         }
@@ -383,16 +403,8 @@ pesto_status pesto_search_get(pesto_search *s, int32_t base, int64_t *mk, uint8_
     if (mk && (e = cudaMemcpy(mk, s->d_mk.as<int64_t>() + base, 8, cudaMemcpyDeviceToHost)) != cudaSuccess)
         return cuda_fail(e, "read makespan");
     if (x_host) {
-        std::vector<uint32_t> bits((size_t)g->planes * g->words);
-        e = cudaMemcpy(bits.data(), s->d_bits.as<uint32_t>() + (size_t)base * bits.size(),
-                       bits.size() * 4, cudaMemcpyDeviceToHost);
-        if (e != cudaSuccess) return cuda_fail(e, "read placement");
-        for (int32_t q = 0; q < g->n; q++) {
-            int x = 0;
-            for (int k = 0; k < g->planes; k++)
-                x |= (int)((bits[(size_t)k * g->words + (q >> 5)] >> (q & 31)) & 1u) << k;
-            x_host[s->order[base][q]] = (uint8_t)x;
-        }
+        pesto_status rc = download_x(s, base, x_host);
+        if (rc) return rc;
     }
     if (order_host) std::copy(s->order[base].begin(), s->order[base].end(), order_host);
     return PESTO_OK;

@@ -89,7 +89,7 @@ def test_saturated_rows_take_the_64bit_path(P, O):
     """makespans above the 32-bit kernel's saturation (4.03 s) are re-evaluated in int64."""
     g = dag.random_dag(51, 60, 1.5, D=2, p_max=250_000_000, zero_frac=0.0, max_bytes=1 << 20,
                        beta0=1000, beta1_fs=40_000)
-    g.p[:] = np.maximum(g.p, 60_000_000)                     # every op 60-250 ms: sum p >> 4 s
+    g.p[:] = np.maximum(g.p, 170_000_000)                    # every op 170-250 ms: sum p >> 4 s
     G = P.Graph.from_arrays(g)
     order = dag.random_topo_order(g, 1)
     x = dag.random_placements(g, 2, 300)
@@ -116,7 +116,7 @@ def test_search_with_bases_above_saturation(P, O):
     """bases whose makespan exceeds 4.03 s run on the 64-bit kernel until they drop below."""
     g = dag.random_dag(53, 50, 1.4, D=2, p_max=200_000_000, zero_frac=0.0, max_bytes=1 << 20,
                        beta0=1000, beta1_fs=40_000)
-    g.p[:] = np.maximum(g.p, 40_000_000)
+    g.p[:] = np.maximum(g.p, 150_000_000)
     G = P.Graph.from_arrays(g)
     xs, orders = _bases(g, 2, seed=11)
     xs[0] = 0                                                # base 0: sum p > 4.03 s

@@ -62,6 +62,25 @@ def test_identity_and_move_shapes(O):
     assert seen["flip"] > 0 and seen["window"] > 0 and seen["swap"] > 0
 
 
+def test_group_changes_stay_in_its_region(O):
+    """every change a group of 32 candidates makes lies in [c_g, c_g + 64) (DESIGN §4 S2)."""
+    g, xs, orders = _setup(seed=6, n=300)
+    P = xs.shape[0]
+    for b in range(P):
+        for grp in range(1, 40):
+            c = O.draw(2021, 2, P, b, 32 * grp, 13) % g.n
+            hi = min(g.n, c + 64)
+            for lane in range(32):
+                j = 32 * grp + lane
+                ok, x, o = O.candidate(g, P, b, xs, orders, j, 2021, 2, MIX)
+                changed = np.nonzero(x != xs[b])[0]
+                pos = [int(np.nonzero(orders[b] == v)[0][0]) for v in changed]
+                assert all(c <= q < hi for q in pos), (grp, lane, c, pos)
+                diff = np.nonzero(o != orders[b])[0]
+                if len(diff):
+                    assert c <= diff[0] < hi or diff[0] == g.n - 2
+
+
 def test_moves_respect_allowed(O):
     g, xs, orders = _setup(seed=9, n=50, D=4, allowed_frac=0.6)
     for v in range(g.n):                                  # make the bases feasible
