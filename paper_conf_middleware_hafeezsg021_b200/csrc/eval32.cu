@@ -36,20 +36,20 @@ struct RegState32 {          // D <= 2
     __device__ uint32_t makespan() const { return max(d0, d1); }
 };
 
-struct SmemState32 {         // D <= 8: [column][lane] in shared memory
-    uint32_t *d, *l;
+struct SmemState32 {         // D <= 8: [column][lane] in shared memory (shared addresses)
+    uint32_t d, l;
     int D;
     __device__ void init() {
-        for (int x = 0; x < D; x++) d[x * 32] = 0u;
-        for (int x = 0; x < D * D; x++) l[x * 32] = 0u;
+        for (int x = 0; x < D; x++) sts_u32(d + x * 128, 0u);
+        for (int x = 0; x < D * D; x++) sts_u32(l + x * 128, 0u);
     }
-    __device__ uint32_t dev(int x) const { return d[x * 32]; }
-    __device__ void set_dev(int x, uint32_t v) { d[x * 32] = v; }
-    __device__ uint32_t link(int x, int y) const { return l[(x * D + y) * 32]; }
-    __device__ void set_link(int x, int y, uint32_t v) { l[(x * D + y) * 32] = v; }
+    __device__ uint32_t dev(int x) const { return lds_u32(d + x * 128); }
+    __device__ void set_dev(int x, uint32_t v) { sts_u32(d + x * 128, v); }
+    __device__ uint32_t link(int x, int y) const { return lds_u32(l + (x * D + y) * 128); }
+    __device__ void set_link(int x, int y, uint32_t v) { sts_u32(l + (x * D + y) * 128, v); }
     __device__ uint32_t makespan() const {
         uint32_t m = 0;
-        for (int x = 0; x < D; x++) m = max(m, d[x * 32]);
+        for (int x = 0; x < D; x++) m = max(m, lds_u32(d + x * 128));
         return m;
     }
 };
@@ -73,7 +73,7 @@ struct Place32 {
 };
 
 struct Ctx32 {
-    uint32_t *ring;              // shared: ring[(pos & 15) * 32 + lane]
+    uint32_t ring;               // shared address of ring[0][lane]; slot s at ring + s * 128
     uint32_t *cold;              // global: cold[slot * 32 + lane]
     const uint8_t *lclass;
     int edge_stride, D;
@@ -110,9 +110,9 @@ __device__ __forceinline__ void push32(const uint8_t *ep, const uint4 rec, int x
         st.set_link(x, y, a);
     }
     if (tgt & kT32Near) {
-        uint32_t *slot = cx.ring + (succ & (kRing - 1)) * 32;
-        if (ALL_MAX || !(tgt & kT32First)) a = max(a, *slot);
-        *slot = a;
+        const uint32_t slot = cx.ring + (uint32_t)(succ & (kRing - 1)) * 128;
+        if (ALL_MAX || !(tgt & kT32First)) a = max(a, lds_u32(slot));
+        sts_u32(slot, a);
     } else {
         uint32_t *slot = cx.cold + (size_t)(tgt & kT32SlotMask) * 32;
         if (!ALL_MAX && (tgt & kT32First)) *slot = a;        // first far push: plain store
@@ -168,7 +168,7 @@ __device__ __forceinline__ const uint8_t *relax32(const uint8_t *rp, int32_t v, 
     cold_out = (int32_t)o.y >= 0 ? cx.cold[(size_t)o.y * 32] : 0u;
     const int x = place(v, (int)((o.w >> kOpXShift) & 7u));
     uint32_t r = cold_in;
-    if (o.w & kOp32HasNear) r = max(r, cx.ring[(v & (kRing - 1)) * 32]);
+    if (o.w & kOp32HasNear) r = max(r, lds_u32(cx.ring + (uint32_t)(v & (kRing - 1)) * 128));
     const uint32_t c = add_sat(max(r, st.dev(x)), o.x);    // C_v = S_v + p_v
     st.set_dev(x, c);
     const bool adj = (o.w & kOpAdj) != 0;
@@ -205,7 +205,7 @@ __device__ __forceinline__ void clear_first32(const uint8_t *rp, const uint8_t *
         const uint4 rec = global ? load_rec32<true>(ep + (size_t)i * cx.edge_stride)
                                  : load_rec32<false>(ep + (size_t)i * cx.edge_stride);
         if (!(rec.z & kT32First)) continue;
-        if (rec.z & kT32Near) cx.ring[(((int32_t)(rec.y & kSuccPosMask)) & (kRing - 1)) * 32] = 0u;
+        if (rec.z & kT32Near) sts_u32(cx.ring + (rec.y & (kRing - 1)) * 128, 0u);
         else cx.cold[(size_t)(rec.z & kT32SlotMask) * 32] = 0u;
     }
 }
@@ -262,7 +262,7 @@ eval32_kernel(const EvalParams P) {
     }
 
     Ctx32 cx;
-    cx.ring = ring_all + (size_t)warp * kRing * 32 + lane;
+    cx.ring = su32(ring_all + (size_t)warp * kRing * 32 + lane);
     cx.cold = P.state32 + ((size_t)(blockIdx.x * kWarps + warp) * P.max_W32) * 32 + lane;
     cx.lclass = lclass;
     cx.edge_stride = P.edge_stride32;
@@ -272,8 +272,8 @@ eval32_kernel(const EvalParams P) {
     StateT st;
     if constexpr (PL != 1) {
         st.D = P.D;
-        st.d = dstate + (size_t)warp * (P.D + P.D * P.D) * 32 + lane;
-        st.l = st.d + (size_t)P.D * 32;
+        st.d = su32(dstate + (size_t)warp * (P.D + P.D * P.D) * 32 + lane);
+        st.l = st.d + (uint32_t)P.D * 128;
     }
 
     uint32_t it = 0;

@@ -41,21 +41,21 @@ struct RegState {            // D <= 2: two devices, two directed links, in regi
     __device__ int64_t makespan(int) const { return max(d0, d1); }
 };
 
-struct SmemState {           // D <= 8: [slot][lane] columns in shared memory
-    int64_t *d;              // [D][32] + lane
-    int64_t *l;              // [D*D][32] + lane
+struct SmemState {           // D <= 8: [slot][lane] columns in shared memory (shared addresses)
+    uint32_t d;              // [D][32] + lane
+    uint32_t l;              // [D*D][32] + lane
     int D;
     __device__ void init(int) {
-        for (int x = 0; x < D; x++) d[x * 32] = 0;
-        for (int x = 0; x < D * D; x++) l[x * 32] = 0;
+        for (int x = 0; x < D; x++) sts_u64(d + x * 256, 0);
+        for (int x = 0; x < D * D; x++) sts_u64(l + x * 256, 0);
     }
-    __device__ int64_t dev(int x) const { return d[x * 32]; }
-    __device__ void set_dev(int x, int64_t v) { d[x * 32] = v; }
-    __device__ int64_t link(int x, int y) const { return l[(x * D + y) * 32]; }
-    __device__ void set_link(int x, int y, int64_t v) { l[(x * D + y) * 32] = v; }
+    __device__ int64_t dev(int x) const { return (int64_t)lds_u64(d + x * 256); }
+    __device__ void set_dev(int x, int64_t v) { sts_u64(d + x * 256, (uint64_t)v); }
+    __device__ int64_t link(int x, int y) const { return (int64_t)lds_u64(l + (x * D + y) * 256); }
+    __device__ void set_link(int x, int y, int64_t v) { sts_u64(l + (x * D + y) * 256, (uint64_t)v); }
     __device__ int64_t makespan(int) const {
         int64_t m = 0;
-        for (int x = 0; x < D; x++) m = max(m, d[x * 32]);
+        for (int x = 0; x < D; x++) m = max(m, (int64_t)lds_u64(d + x * 256));
         return m;
     }
 };
@@ -275,8 +275,8 @@ eval_kernel(const EvalParams P) {
     StateT st;
     if constexpr (PL != 1) {
         st.D = P.D;
-        st.d = dstate + (size_t)warp * (P.D + P.D * P.D) * 32 + lane;
-        st.l = st.d + (size_t)P.D * 32;
+        st.d = su32(dstate + (size_t)warp * (P.D + P.D * P.D) * 32 + lane);
+        st.l = st.d + (uint32_t)P.D * 256;
     }
 
     uint32_t it = 0;
