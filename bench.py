@@ -288,17 +288,29 @@ def run_pesto(args, rank, world, local):
             dist.destroy_process_group()
         return
 
-    # ---- roofline of the dominant kernel (K1 eval) ----
+    # ---- roofline of the dominant kernel (K1 eval), DESIGN.md §5 ----
+    # K1 is bound by integer issue and latency, not by HBM (the ncu capture in profiles/ shows
+    # DRAM at ~12% of peak).  Algorithmic work per candidate: per op one max + one add (C_v), per
+    # edge one max (the arrival push), per crossing edge one more max + add (the link queue):
+    # 2n + m + 2*cross integer ops; cross is counted at the base placements.
     pk = peaks()
-    hbm = pk.get("hbm_gbs")
-    peak_note = "measured (MEASURED_PEAKS.json hbm_gbs)"
-    if not hbm:
-        hbm, peak_note = 6650.0, "fallback (B200_PROFILING.md)"
-    # algorithmic bytes: the ready-time slot state moves 2 int64 accesses per edge per candidate
-    # (one push, one read-or-RMW): 16*m bytes per candidate
-    alg_bytes_launch = 16.0 * g.m * k_gpu
+    sm_mhz = pk.get("sm_max_mhz") or 1965.0
+    peak_note = ("148 SMs x 128 int32 lanes/clk (4 SMSPs x 32 lanes, one integer warp-instr per "
+                 f"clk per SMSP) x {sm_mhz:.0f} MHz (MEASURED_PEAKS.json sm_max_mhz)")
+    peak_tops = 148 * 128 * sm_mhz * 1e6 / 1e12
+    cross = float(np.mean([int((xs[b][g.src] != xs[b][g.dst]).sum()) for b in range(n_bases)]))
+    alg_ops_launch = (2.0 * g.n + g.m + 2.0 * cross) * k_gpu
     eval_avg_s = (tot_eval_ms / args.steps) / 1e3
-    achieved = alg_bytes_launch / eval_avg_s / 1e9
+    achieved = alg_ops_launch / eval_avg_s / 1e12
+    traffic = None
+    prof = os.path.join(ROOT, "profiles", f"r1_eval32_{args.config.split('_')[0]}_ncu.json")
+    if os.path.exists(prof) and world == 1:
+        try:
+            pj = json.load(open(prof))
+            if pj.get("config") == args.config:
+                traffic = pj["dram_bytes_per_launch"]
+        except Exception:
+            traffic = None
     st = G.stats(orders[0])
     line = {"metric": METRIC, "value": value, "unit": "candidates/s", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": tot_ms / args.steps,
@@ -311,9 +323,12 @@ def run_pesto(args, rank, world, local):
                        "parallelism": f"candidate-dp{world}"},
             "op_relaxations_per_s": value * g.n, "edge_relaxations_per_s": value * g.m,
             "eval_kernel_ms": tot_eval_ms / args.steps,
-            "roofline": {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",
-                         "frac": achieved / hbm, "traffic": None, "peak_source": peak_note,
-                         "note": "algorithmic slot-state bytes 16*m per candidate / K1 time"},
+            "roofline": {"bound": "alu", "achieved": achieved, "peak": peak_tops,
+                         "unit": "TOP/s (int32)", "frac": achieved / peak_tops,
+                         "traffic": traffic, "peak_source": peak_note,
+                         "ops_per_candidate": 2.0 * g.n + g.m + 2.0 * cross,
+                         "note": "algorithmic int ops (2n+m+2*cross per candidate) / K1 time; "
+                                 "traffic = ncu DRAM bytes per K1 launch (profiles/)"},
             "gpu_launches": int(launches),
             "wall_s_timed_region": wall,
             "search": {"seed_makespans": seed_mk, "best_makespans": best_mk},

@@ -246,10 +246,12 @@ pesto_status pesto_search_create(pesto_graph *g, const pesto_search_desc *d, pes
     if ((e = s->d_dbg_key.ensure(8)) != cudaSuccess) return cuda_fail(e, "allocate");
     if ((e = cudaMallocHost((void **)&s->h_swap, 4 * s->P)) != cudaSuccess) return cuda_fail(e, "pinned");
     if ((e = cudaMallocHost((void **)&s->h_keys, 8 * s->P)) != cudaSuccess) return cuda_fail(e, "pinned");
-    // initial base makespans: candidate j = 0 of every base is the base itself
-    for (int b = 0; b < s->P; b++) {
-        pesto_status rc = launch_search_eval(s.get(), b, 1, 0, 1, s->d_dbg_key.as<uint64_t>(),
-                                             s->d_keys.as<uint64_t>() + b, nullptr);
+    // initial base makespans: candidate j = 0 of every base is the base itself (exact, eval64,
+    // one launch for all bases)
+    if ((e = cudaMemset(s->d_keys.ptr, 0xFF, 8 * s->P)) != cudaSuccess) return cuda_fail(e, "reset keys");
+    {
+        pesto_status rc = launch_search_eval(s.get(), 0, s->P, 0, 1, s->d_keys.as<uint64_t>(),
+                                             nullptr, nullptr);
         if (rc) return rc;
     }
     if ((e = cudaDeviceSynchronize()) != cudaSuccess) return cuda_fail(e, "initial evaluation");
