@@ -10,7 +10,8 @@
 // One lane = one candidate, 32 candidates per warp share every DAG tile, which the producer
 // warp streams into shared memory with cp.async.bulk (TMA) through an mbarrier ring.
 // Search candidates differ from their base only inside their group's 64-position region
-// (DESIGN.md §4), so outside it a lane's device is the base code embedded in the record.
+// (DESIGN.md §4), so outside it a lane's device is the base code embedded in the record, and
+// once the walk is past the region no lookup needs the check at all (successors come later).
 #include <algorithm>
 #include <type_traits>
 
@@ -54,7 +55,8 @@ struct SmemState32 {         // D <= 8: [column][lane] in shared memory (shared 
     }
 };
 
-// lane's device at position q; xb = the base code carried by the record that names q
+// lane's device at position q; xb = the base code carried by the record that names q.
+// CHECK = false once the walk is past the group's region (no lookup can fall inside it).
 template <int MODE, int PL>
 struct Place32 {
     const uint32_t *pl;          // MODE 0: this group's bit-sliced words
@@ -62,9 +64,10 @@ struct Place32 {
     int32_t rc, rlen;            // MODE 1: the group's region [rc, rc + rlen)
     int all_allowed, lane, dmax;
     LaneMove mv;
-    __device__ __forceinline__ int operator()(int32_t q, int xb) const {
+    template <bool CHECK>
+    __device__ __forceinline__ int at(int32_t q, int xb) const {
         if (MODE == 0) return planes_dev_at<PL>(pl, q, lane, dmax);
-        if ((uint32_t)(q - rc) < (uint32_t)rlen) {           // warp-uniform branch
+        if (CHECK && (uint32_t)(q - rc) < (uint32_t)rlen) {  // warp-uniform branch
             const unsigned aq = all_allowed ? 0xFFu : (unsigned)__ldg(allowed_pos + q);
             return apply_lane(mv, q, xb, aq);
         }
@@ -73,48 +76,57 @@ struct Place32 {
 };
 
 struct Ctx32 {
-    uint32_t ring;               // shared address of ring[0][lane]; slot s at ring + s * 128
+    const uint8_t *smem;         // the CTA's dynamic shared memory (records addressed from here)
+    uint32_t ring;               // shared address of ring[0][lane]; slot bytes from the record
     uint32_t *cold;              // global: cold[slot * 32 + lane]
-    const uint8_t *lclass;
+    uint32_t lclass;             // shared address of the link-class table
     int edge_stride, D;
+    bool two_classes;            // a second link class exists (its t is EdgeRec32.t1)
 };
 
 __device__ __forceinline__ void prefetch_l1(const void *p) {
     asm volatile("prefetch.global.L1 [%0];" ::"l"(p));
 }
 
+// record at byte offset `off` of shared memory (GLOBAL: of the out-of-line array)
 template <bool GLOBAL>
-__device__ __forceinline__ uint4 load_rec32(const uint8_t *p) {
-    if (GLOBAL) return __ldg(reinterpret_cast<const uint4 *>(p));
-    return *reinterpret_cast<const uint4 *>(p);
+__device__ __forceinline__ uint4 rec_at(const Ctx32 &cx, const uint8_t *heavy, uint32_t off) {
+    if (GLOBAL) return __ldg(reinterpret_cast<const uint4 *>(heavy + off));
+    return *reinterpret_cast<const uint4 *>(cx.smem + off);
 }
 
-template <bool MULTI, bool GLOBAL, bool ALL_MAX, class PlaceT, class StateT>
-__device__ __forceinline__ void push32(const uint8_t *ep, const uint4 rec, int x, uint32_t c,
-                                       const PlaceT &place, StateT &st, const Ctx32 &cx) {
+template <bool MULTI>
+__device__ __forceinline__ int stride32(const Ctx32 &cx) { return MULTI ? cx.edge_stride : 16; }
+
+template <bool MULTI, bool GLOBAL, bool ALL_MAX, bool CHECK, class PlaceT, class StateT>
+__device__ __forceinline__ void push32(const Ctx32 &cx, const uint8_t *heavy, uint32_t off,
+                                       const uint4 rec, int x, uint32_t c, const PlaceT &place,
+                                       StateT &st) {
     const int32_t succ = (int32_t)(rec.y & kSuccPosMask);
     const uint32_t tgt = rec.z;
-    const int y = place(succ, (int)((rec.y >> kSuccXShift) & 7u));
+    const int y = place.template at<CHECK>(succ, (int)((rec.y >> kSuccXShift) & 7u));
     uint32_t a = c;                                          // same device: C_v (L144)
     if (y != x) {                                            // cross: FCFS link x -> y
         uint32_t t = rec.x;
-        if (MULTI) {
-            const int cls = cx.lclass[x * cx.D + y];
+        if (MULTI || cx.two_classes) {
+            const int cls = (int)lds_u8(cx.lclass + (uint32_t)(x * cx.D + y));
             if (cls == 1) t = rec.w;
-            else if (cls > 1) {
-                const uint32_t *ext = reinterpret_cast<const uint32_t *>(ep + 16) + (cls - 2);
-                t = GLOBAL ? __ldg(ext) : *ext;
+            else if (MULTI && cls > 1) {
+                const uint32_t eo = off + 16 + 4 * (cls - 2);
+                t = GLOBAL ? __ldg(reinterpret_cast<const uint32_t *>(heavy + eo))
+                           : *reinterpret_cast<const uint32_t *>(cx.smem + eo);
             }
         }
         a = add_sat(max(c, st.link(x, y)), t);
         st.set_link(x, y, a);
     }
+    const uint32_t bytes = tgt & kT32SlotMask;
     if (tgt & kT32Near) {
-        const uint32_t slot = cx.ring + (uint32_t)(succ & (kRing - 1)) * 128;
+        const uint32_t slot = cx.ring + bytes;
         if (ALL_MAX || !(tgt & kT32First)) a = max(a, lds_u32(slot));
         sts_u32(slot, a);
     } else {
-        uint32_t *slot = cx.cold + (size_t)(tgt & kT32SlotMask) * 32;
+        uint32_t *slot = reinterpret_cast<uint32_t *>(reinterpret_cast<uint8_t *>(cx.cold) + bytes);
         if (!ALL_MAX && (tgt & kT32First)) *slot = a;        // first far push: plain store
         else atomicMax(slot, a);                             // RED.MAX, no wait for a reply
     }
@@ -123,22 +135,30 @@ __device__ __forceinline__ void push32(const uint8_t *ep, const uint4 rec, int x
 // out-edges of one producer in record order.  Only a producer feeding two adjacent positions
 // (kOpAdj) can see its order change under a swap (ks, ks+1): then the run of edges to ks+1 is
 // pushed before the run to ks (the swapped order's consumer order).
-template <bool MULTI, bool GLOBAL, bool ALL_MAX, class PlaceT, class StateT>
-__device__ __forceinline__ void push_all32(const uint8_t *ep, uint32_t nout, bool adj, int32_t ks,
-                                           int x, uint32_t c, const PlaceT &place, StateT &st,
-                                           const Ctx32 &cx) {
-    const int es = cx.edge_stride;
+template <bool MULTI, bool GLOBAL, bool ALL_MAX, bool CHECK, class PlaceT, class StateT>
+__device__ __forceinline__ void push_all32(const Ctx32 &cx, const uint8_t *heavy, uint32_t ep,
+                                           uint32_t nout, bool adj, int32_t ks, int x, uint32_t c,
+                                           const PlaceT &place, StateT &st) {
+    const int es = stride32<MULTI>(cx);
     if (!adj || ks < 0) {
-        for (uint32_t i = 0; i < nout; i++)
-            push32<MULTI, GLOBAL, ALL_MAX>(ep + (size_t)i * es, load_rec32<GLOBAL>(ep + (size_t)i * es),
-                                           x, c, place, st, cx);
+        for (uint32_t i = 0; i < nout; i++) {
+            const uint32_t off = ep + i * es;
+            push32<MULTI, GLOBAL, ALL_MAX, CHECK>(cx, heavy, off, rec_at<GLOBAL>(cx, heavy, off), x, c,
+                                                  place, st);
+        }
         return;
     }
-    auto spos = [&](uint32_t i) { return (int32_t)(load_rec32<GLOBAL>(ep + (size_t)i * es).y & kSuccPosMask); };
+    auto spos = [&](uint32_t i) {
+        return (int32_t)(rec_at<GLOBAL>(cx, heavy, ep + i * es).y & kSuccPosMask);
+    };
+    auto push_i = [&](uint32_t i) {
+        const uint32_t off = ep + i * es;
+        push32<MULTI, GLOBAL, ALL_MAX, CHECK>(cx, heavy, off, rec_at<GLOBAL>(cx, heavy, off), x, c,
+                                              place, st);
+    };
     for (uint32_t i = 0; i < nout;) {
         if (spos(i) != ks) {
-            push32<MULTI, GLOBAL, ALL_MAX>(ep + (size_t)i * es, load_rec32<GLOBAL>(ep + (size_t)i * es),
-                                           x, c, place, st, cx);
+            push_i(i);
             i++;
             continue;
         }
@@ -146,27 +166,22 @@ __device__ __forceinline__ void push_all32(const uint8_t *ep, uint32_t nout, boo
         while (a_end < nout && spos(a_end) == ks) a_end++;
         uint32_t b_end = a_end;
         while (b_end < nout && spos(b_end) == ks + 1) b_end++;
-        for (uint32_t e = a_end; e < b_end; e++)
-            push32<MULTI, GLOBAL, ALL_MAX>(ep + (size_t)e * es, load_rec32<GLOBAL>(ep + (size_t)e * es),
-                                           x, c, place, st, cx);
-        for (uint32_t e = i; e < a_end; e++)
-            push32<MULTI, GLOBAL, ALL_MAX>(ep + (size_t)e * es, load_rec32<GLOBAL>(ep + (size_t)e * es),
-                                           x, c, place, st, cx);
+        for (uint32_t e = a_end; e < b_end; e++) push_i(e);
+        for (uint32_t e = i; e < a_end; e++) push_i(e);
         i = b_end;
     }
 }
 
-// Relax the op at position v (records at rp, shared memory).  `cold_in` is its far arrivals
-// (loaded one op earlier); the far arrivals of the next position are loaded into `cold_out`.
-template <bool MULTI, bool ALL_MAX, class PlaceT, class StateT>
-__device__ __forceinline__ const uint8_t *relax32(const uint8_t *rp, int32_t v, int32_t ks,
-                                                  const uint8_t *heavy, const PlaceT &place,
-                                                  StateT &st, const Ctx32 &cx, uint32_t cold_in,
-                                                  uint32_t &cold_out) {
-    const uint4 o = *reinterpret_cast<const uint4 *>(rp);   // {p, cold_next, pf_slot, nout}
+// Relax the op at position v whose records start at shared byte offset rp.  `cold_in` is its
+// far arrivals (loaded one op earlier); the next position's are loaded into `cold_out`.
+template <bool MULTI, bool ALL_MAX, bool CHECK, class PlaceT, class StateT>
+__device__ __forceinline__ uint32_t relax32(const Ctx32 &cx, uint32_t rp, int32_t v, int32_t ks,
+                                            const uint8_t *heavy, const PlaceT &place,
+                                            StateT &st, uint32_t cold_in, uint32_t &cold_out) {
+    const uint4 o = *reinterpret_cast<const uint4 *>(cx.smem + rp);  // {p, cold_next, pf, nout}
     if ((int32_t)o.z >= 0) prefetch_l1(cx.cold + (size_t)o.z * 32);
     cold_out = (int32_t)o.y >= 0 ? cx.cold[(size_t)o.y * 32] : 0u;
-    const int x = place(v, (int)((o.w >> kOpXShift) & 7u));
+    const int x = place.template at<CHECK>(v, (int)((o.w >> kOpXShift) & 7u));
     uint32_t r = cold_in;
     if (o.w & kOp32HasNear) r = max(r, lds_u32(cx.ring + (uint32_t)(v & (kRing - 1)) * 128));
     const uint32_t c = add_sat(max(r, st.dev(x)), o.x);    // C_v = S_v + p_v
@@ -174,39 +189,40 @@ __device__ __forceinline__ const uint8_t *relax32(const uint8_t *rp, int32_t v, 
     const bool adj = (o.w & kOpAdj) != 0;
     if (!(o.w & kOpHeavy)) {
         const uint32_t nout = o.w & kOpNoutMask;
-        push_all32<MULTI, false, ALL_MAX>(rp + 16, nout, adj, ks, x, c, place, st, cx);
-        return rp + 16 + (size_t)nout * cx.edge_stride;
+        push_all32<MULTI, false, ALL_MAX, CHECK>(cx, heavy, rp + 16, nout, adj, ks, x, c, place, st);
+        return rp + 16 + nout * stride32<MULTI>(cx);
     }
-    const ExtRec ext = *reinterpret_cast<const ExtRec *>(rp + 16);
-    push_all32<MULTI, true, ALL_MAX>(heavy + ext.edge_off, (uint32_t)ext.nout, adj, ks, x, c, place,
-                                     st, cx);
+    const uint4 ext = *reinterpret_cast<const uint4 *>(cx.smem + rp + 16);   // ExtRec
+    push_all32<MULTI, true, ALL_MAX, CHECK>(cx, heavy, ext.x, ext.z, adj, ks, x, c, place, st);
     return rp + 32;
 }
 
-__device__ __forceinline__ const uint8_t *skip32(const uint8_t *rp, int es) {
-    const uint32_t nout = reinterpret_cast<const uint32_t *>(rp)[3];
+template <bool MULTI>
+__device__ __forceinline__ uint32_t skip32(const Ctx32 &cx, uint32_t rp) {
+    const uint32_t nout = reinterpret_cast<const uint32_t *>(cx.smem + rp)[3];
     if (nout & kOpHeavy) return rp + 32;
-    return rp + 16 + (size_t)(nout & kOpNoutMask) * es;
+    return rp + 16 + (nout & kOpNoutMask) * stride32<MULTI>(cx);
 }
 
 // zero the slots an op opens with a first push (swap pairs only; times are >= 0)
-__device__ __forceinline__ void clear_first32(const uint8_t *rp, const uint8_t *heavy,
-                                              const Ctx32 &cx) {
-    const uint4 o = *reinterpret_cast<const uint4 *>(rp);
+template <bool MULTI>
+__device__ __forceinline__ void clear_first32(const Ctx32 &cx, uint32_t rp, const uint8_t *heavy) {
+    const uint4 o = *reinterpret_cast<const uint4 *>(cx.smem + rp);
     const bool global = (o.w & kOpHeavy) != 0;
-    const uint8_t *ep = rp + 16;
-    uint32_t nout = o.w & kOpNoutMask;
+    uint32_t ep = rp + 16, nout = o.w & kOpNoutMask;
     if (global) {
-        const ExtRec ext = *reinterpret_cast<const ExtRec *>(rp + 16);
-        ep = heavy + ext.edge_off;
-        nout = (uint32_t)ext.nout;
+        const uint4 ext = *reinterpret_cast<const uint4 *>(cx.smem + rp + 16);
+        ep = ext.x;
+        nout = ext.z;
     }
+    const int es = stride32<MULTI>(cx);
     for (uint32_t i = 0; i < nout; i++) {
-        const uint4 rec = global ? load_rec32<true>(ep + (size_t)i * cx.edge_stride)
-                                 : load_rec32<false>(ep + (size_t)i * cx.edge_stride);
+        const uint4 rec = global ? rec_at<true>(cx, heavy, ep + i * es)
+                                 : rec_at<false>(cx, heavy, ep + i * es);
         if (!(rec.z & kT32First)) continue;
-        if (rec.z & kT32Near) sts_u32(cx.ring + (rec.y & (kRing - 1)) * 128, 0u);
-        else cx.cold[(size_t)(rec.z & kT32SlotMask) * 32] = 0u;
+        const uint32_t bytes = rec.z & kT32SlotMask;
+        if (rec.z & kT32Near) sts_u32(cx.ring + bytes, 0u);
+        else *reinterpret_cast<uint32_t *>(reinterpret_cast<uint8_t *>(cx.cold) + bytes) = 0u;
     }
 }
 
@@ -215,7 +231,6 @@ __global__ void __launch_bounds__((kWarps + 1) * 32, 2)
 eval32_kernel(const EvalParams P) {
     extern __shared__ __align__(128) uint8_t smem[];
     const int sb = P.stage_bytes32;
-    uint8_t *stage_buf = smem;
     uint64_t *full = reinterpret_cast<uint64_t *>(smem + (size_t)kStages * sb);
     uint64_t *empty = full + kStages;
     uint8_t *cur = align16(reinterpret_cast<uint8_t *>(empty + kStages));
@@ -253,7 +268,7 @@ eval32_kernel(const EvalParams P) {
                     if (it >= (uint32_t)kStages) mbar_wait(&empty[s], ((it / kStages) - 1) & 1);
                     const TileDesc td = B->tiles32[t];
                     mbar_expect_tx(&full[s], (uint32_t)td.bytes);
-                    bulk_g2s(stage_buf + (size_t)s * sb, B->blob32 + td.byte_off, (uint32_t)td.bytes,
+                    bulk_g2s(smem + (size_t)s * sb, B->blob32 + td.byte_off, (uint32_t)td.bytes,
                              &full[s]);
                 }
             }
@@ -262,11 +277,13 @@ eval32_kernel(const EvalParams P) {
     }
 
     Ctx32 cx;
+    cx.smem = smem;
     cx.ring = su32(ring_all + (size_t)warp * kRing * 32 + lane);
     cx.cold = P.state32 + ((size_t)(blockIdx.x * kWarps + warp) * P.max_W32) * 32 + lane;
-    cx.lclass = lclass;
+    cx.lclass = su32(lclass);
     cx.edge_stride = P.edge_stride32;
     cx.D = P.D;
+    cx.two_classes = P.n_classes > 1;
 
     using StateT = typename std::conditional<PL == 1, RegState32, SmemState32>::type;
     StateT st;
@@ -295,6 +312,7 @@ eval32_kernel(const EvalParams P) {
         bool active, valid = true;
         const int64_t j = g * 32 + lane;
         int32_t ks = -1;
+        int32_t check_end = P.n;                     // positions from here on need no check
         if (MODE == 0) {
             active = g * 32 < P.n_cand;
             place.pl = P.planes_in + (size_t)g * P.n * PL;
@@ -306,6 +324,7 @@ eval32_kernel(const EvalParams P) {
             const Region rg = decode_region(P.seed, cb, g, P.n);
             place.rc = rg.c;
             place.rlen = rg.len;
+            check_end = rg.c + rg.len;
             place.allowed_pos = B->allowed_pos;
             const uint8_t *adj = B->adj_next;
             ks = active ? decode_swap(P.seed, cb, g, P.n, P.mix[3], rg,
@@ -333,39 +352,44 @@ eval32_kernel(const EvalParams P) {
             const int s = it % kStages;
             mbar_wait(&full[s], (it / kStages) & 1);
             if (active) {
-                const uint8_t *tile = stage_buf + (size_t)s * sb;
-                const int32_t pos_end = reinterpret_cast<const int32_t *>(tile)[1];
-                int32_t v = reinterpret_cast<const int32_t *>(tile)[0];
-                const uint8_t *rp = tile + kTileHeader;
+                const uint32_t tile = (uint32_t)s * sb;
+                const int32_t pos_end = reinterpret_cast<const int32_t *>(smem + tile)[1];
+                int32_t v = reinterpret_cast<const int32_t *>(smem + tile)[0];
+                uint32_t rp = tile + kTileHeader;
                 if (skip_first) {
-                    rp = skip32(rp, cx.edge_stride);
+                    rp = skip32<MULTI>(cx, rp);
                     v++;
                     skip_first = false;
                 }
+                // past the region (and past any swap, which lies in it) every op is base-coded
+                if (MODE == 0 || (v >= check_end && ks < v)) {
+                    for (; v < pos_end; v++)
+                        rp = relax32<MULTI, false, false>(cx, rp, v, -1, heavy, place, st, cold_v, cold_v);
+                }
                 while (v < pos_end) {
                     if (v != ks) {
-                        rp = relax32<MULTI, false>(rp, v, ks, heavy, place, st, cx, cold_v, cold_v);
+                        rp = relax32<MULTI, false, true>(cx, rp, v, ks, heavy, place, st, cold_v, cold_v);
                         v++;
                         continue;
                     }
                     // swapped pair: ops at ks+1 then ks
-                    const uint8_t *rk = rp;
-                    const uint8_t *rk1;
+                    const uint32_t rk = rp;
+                    uint32_t rk1;
                     const bool straddle = (v + 1 == pos_end);
                     if (straddle) {
                         const int s2 = (it + 1) % kStages;
                         mbar_wait(&full[s2], ((it + 1) / kStages) & 1);
-                        rk1 = stage_buf + (size_t)s2 * sb + kTileHeader;
+                        rk1 = (uint32_t)s2 * sb + kTileHeader;
                     } else {
-                        rk1 = skip32(rk, cx.edge_stride);
+                        rk1 = skip32<MULTI>(cx, rk);
                     }
-                    const int32_t cold_k1 = reinterpret_cast<const int32_t *>(rk)[1];
+                    const int32_t cold_k1 = reinterpret_cast<const int32_t *>(smem + rk)[1];
                     const uint32_t cold_first = cold_k1 >= 0 ? cx.cold[(size_t)cold_k1 * 32] : 0u;
                     uint32_t dummy, next_v;
-                    clear_first32(rk, heavy, cx);
-                    const uint8_t *after =
-                        relax32<MULTI, false>(rk1, v + 1, ks, heavy, place, st, cx, cold_first, next_v);
-                    relax32<MULTI, true>(rk, v, ks, heavy, place, st, cx, cold_v, dummy);
+                    clear_first32<MULTI>(cx, rk, heavy);
+                    const uint32_t after = relax32<MULTI, false, true>(cx, rk1, v + 1, ks, heavy, place,
+                                                                       st, cold_first, next_v);
+                    relax32<MULTI, true, true>(cx, rk, v, ks, heavy, place, st, cold_v, dummy);
                     cold_v = next_v;                 // ks+1's record names the op at ks+2
                     if (straddle) {
                         skip_first = true;
@@ -443,10 +467,11 @@ int eval32_smem_bytes(const EvalParams &p, int search_mode) {
     return (int)b + 128;
 }
 
+// the edge stride is a compile-time 16 bytes unless some link class beyond the second exists
 #define PESTO_DISPATCH32(FN, ...)                                                          \
     do {                                                                                   \
         const int pl = planes_of32(p.D);                                                   \
-        const bool multi = p.n_classes > 1;                                                \
+        const bool multi = p.n_classes > 2;                                                \
         if (search_mode) {                                                                 \
             if (pl == 1) return multi ? FN<1, 1, true>(__VA_ARGS__) : FN<1, 1, false>(__VA_ARGS__); \
             if (pl == 2) return multi ? FN<1, 2, true>(__VA_ARGS__) : FN<1, 2, false>(__VA_ARGS__); \

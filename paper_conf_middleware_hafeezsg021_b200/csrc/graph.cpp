@@ -546,7 +546,7 @@ pesto_status pesto_eval_batch(pesto_graph *g, const int32_t *order, const void *
     p.tasks_per_base = (n_groups + kWarps - 1) / kWarps;
     p.n_tasks = p.tasks_per_base;
     int grid = 0;
-    if (!g->eligible32) {                                     // 64-bit path for every row
+    if (!g->eligible32 || L->W32 == 0) {                      // 64-bit path for every row
         if ((s = ensure_state(g, p, 0, p.n_tasks, &grid))) return s;
         p.state = g->d_state.as<int64_t>();
         if ((e = launch_eval(p, 0, grid, st)) != cudaSuccess) return cuda_fail(e, "launch eval");

@@ -200,18 +200,23 @@ pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<
     }
 
     // ---------------- eval32 stream ----------------
+    auto near_edge = [&](int64_t e) { return pos[g->dst[e]] - pos[g->src[e]] <= kNearDelta; };
+    std::vector<int32_t> first_far, cslot;
+    std::vector<uint8_t> has_near;
+    L->W32 = 0;
     if (g->eligible32) {
-        auto near_edge = [&](int64_t e) { return pos[g->dst[e]] - pos[g->src[e]] <= kNearDelta; };
-        std::vector<int32_t> first_far(n, -1);
-        std::vector<uint8_t> has_near(n, 0);
+        first_far.assign(n, -1);
+        has_near.assign(n, 0);
         for (int64_t e = 0; e < m; e++) {
             const int32_t w = g->dst[e];
             if (near_edge(e)) { has_near[w] = 1; continue; }
             const int32_t ps = pos[g->src[e]];
             if (first_far[w] < 0 || ps < first_far[w]) first_far[w] = ps;
         }
-        std::vector<int32_t> cslot;
         L->W32 = std::max(colour_intervals(n, first_far, pos, cslot), 1);
+        if (L->W32 >= (1 << 23)) L->W32 = 0;  // slot byte offsets must fit 30 bits: 64-bit path
+    }
+    if (L->W32 > 0) {
         std::vector<uint8_t> seen_near(n, 0), seen_far(n, 0), first32(m, 0);
         for (int32_t k = 0; k < n; k++) {
             const int32_t u = order[k];
@@ -245,7 +250,10 @@ pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<
             r.t1 = C > 1 ? t32(e, 1) : 0u;
             const int32_t w = g->dst[e];
             r.succ_pos = (int32_t)((uint32_t)pos[w] | (xcode(w) << kSuccXShift));
-            r.target = (near_edge(e) ? kT32Near : (uint32_t)cslot[w]) | (first32[e] ? kT32First : 0u);
+            // byte offset of the lane's slot column: ring slot (pos & 15) or cold slot, x 128
+            r.target = (near_edge(e) ? (kT32Near | (uint32_t)(pos[w] & (kRing - 1)) * 128u)
+                                     : (uint32_t)cslot[w] * 128u) |
+                       (first32[e] ? kT32First : 0u);
             std::memcpy(buf.data() + at, &r, sizeof r);
             for (int c = 2; c < C; c++) {
                 const uint32_t t = t32(e, c);

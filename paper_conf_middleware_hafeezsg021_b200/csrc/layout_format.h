@@ -73,7 +73,7 @@ constexpr uint32_t kSuccPosMask = (1u << 24) - 1;
 constexpr uint32_t kPinHeavy = 1u << 31;        // patch reference into the out-of-line array
 constexpr uint32_t kT32First = 1u << 31;        // EdgeRec32.target: first push into its slot
 constexpr uint32_t kT32Near = 1u << 30;         // push into the near ring (slot = succ & 15)
-constexpr uint32_t kT32SlotMask = (1u << 30) - 1;
+constexpr uint32_t kT32SlotMask = (1u << 30) - 1;   // byte offset (slot x 128) of the target
 
 struct alignas(16) OpRec32 {
     uint32_t p;          // p_v (< kMaxDur32)
@@ -85,7 +85,7 @@ struct alignas(16) OpRec32 {
 struct alignas(16) EdgeRec32 {
     uint32_t t0;         // transfer time, link class 0 (< kMaxDur32)
     int32_t succ_pos;    // successor position | its base code << 24
-    uint32_t target;     // cold slot | kT32Near | kT32First
+    uint32_t target;     // slot byte offset (ring: (pos & 15) * 128, cold: slot * 128) | kT32Near | kT32First
     uint32_t t1;         // link class 1; classes >= 2 follow in 4-byte words
 };
 

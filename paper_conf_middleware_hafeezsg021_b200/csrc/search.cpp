@@ -74,6 +74,7 @@ struct pesto_search {
     // below kSat32 every base runs on eval32 and the 64-bit kernel is not launched at all
     std::vector<int64_t> h_mk;
     bool all_below = false;
+    bool use32 = false;            // eval32 records exist for every base
 };
 
 namespace {
@@ -83,7 +84,9 @@ void refresh_views(pesto_search *s) {
     s->stage_bytes = 16;
     s->max_W32 = 1;
     s->stage_bytes32 = 16;
+    s->use32 = s->g->eligible32;
     for (int b = 0; b < s->P; b++) {
+        if (s->layouts[b]->W32 == 0) s->use32 = false;
         s->views[b] = layout_view(*s->layouts[b]);
         s->views[b].bits = s->d_bits.as<uint32_t>() + (size_t)b * s->g->planes * s->g->words;
         s->max_W = std::max(s->max_W, s->layouts[b]->W);
@@ -94,7 +97,7 @@ void refresh_views(pesto_search *s) {
 }
 
 void update_all_below(pesto_search *s) {
-    s->all_below = s->g->eligible32;
+    s->all_below = s->use32;
     for (int64_t mk : s->h_mk)
         if (mk >= (int64_t)kSat32) s->all_below = false;
 }
@@ -133,7 +136,7 @@ pesto_status launch_search_eval(pesto_search *s, int b_first, int n_bases, int64
     int grid = 0;
     pesto_status rc;
     cudaError_t e;
-    const bool use32 = fast && g->eligible32 && keys_dbg == nullptr;
+    const bool use32 = fast && s->use32 && keys_dbg == nullptr;
     if (use32) {
         p.gate = 1;
         if ((rc = ensure_state32(g, p, 1, p.n_tasks, &grid))) return rc;
@@ -328,7 +331,7 @@ pesto_status pesto_search_commit(pesto_search *s, void *stream) {
     cp.keys = s->d_keys.as<uint64_t>();
     cp.base_mk = s->d_mk.as<int64_t>();
     cp.swap_out = s->d_swap.as<int32_t>();
-    cp.patch32 = g->eligible32 ? 1 : 0;
+    cp.patch32 = s->use32 ? 1 : 0;
     cudaError_t e = launch_commit(cp, st);
     if (e != cudaSuccess) return cuda_fail(e, "launch commit");
     s->step++;
