@@ -101,7 +101,7 @@ __device__ __forceinline__ int stride32(const Ctx32 &cx) { return MULTI ? cx.edg
 template <bool MULTI, bool GLOBAL, bool ALL_MAX, bool CHECK, class PlaceT, class StateT>
 __device__ __forceinline__ void push32(const Ctx32 &cx, const uint8_t *heavy, uint32_t off,
                                        const uint4 rec, int x, uint32_t c, const PlaceT &place,
-                                       StateT &st) {
+                                       StateT &st, uint32_t &fwd) {
     const int32_t succ = (int32_t)(rec.y & kSuccPosMask);
     const uint32_t tgt = rec.z;
     const int y = place.template at<CHECK>(succ, (int)((rec.y >> kSuccXShift) & 7u));
@@ -120,6 +120,10 @@ __device__ __forceinline__ void push32(const Ctx32 &cx, const uint8_t *heavy, ui
         a = add_sat(max(c, st.link(x, y)), t);
         st.set_link(x, y, a);
     }
+    if (tgt & kT32Next) {                                    // consumer is the next position
+        fwd = max(fwd, a);
+        return;
+    }
     const uint32_t bytes = tgt & kT32SlotMask;
     if (tgt & kT32Near) {
         const uint32_t slot = cx.ring + bytes;
@@ -136,17 +140,18 @@ __device__ __forceinline__ void push32(const Ctx32 &cx, const uint8_t *heavy, ui
 // (kOpAdj) can see its order change under a swap (ks, ks+1): then the run of edges to ks+1 is
 // pushed before the run to ks (the swapped order's consumer order).
 template <bool MULTI, bool GLOBAL, bool ALL_MAX, bool CHECK, class PlaceT, class StateT>
-__device__ __forceinline__ void push_all32(const Ctx32 &cx, const uint8_t *heavy, uint32_t ep,
-                                           uint32_t nout, bool adj, int32_t ks, int x, uint32_t c,
-                                           const PlaceT &place, StateT &st) {
+__device__ __forceinline__ uint32_t push_all32(const Ctx32 &cx, const uint8_t *heavy, uint32_t ep,
+                                               uint32_t nout, bool adj, int32_t ks, int x,
+                                               uint32_t c, const PlaceT &place, StateT &st) {
     const int es = stride32<MULTI>(cx);
+    uint32_t fwd = 0;
     if (!adj || ks < 0) {
         for (uint32_t i = 0; i < nout; i++) {
             const uint32_t off = ep + i * es;
             push32<MULTI, GLOBAL, ALL_MAX, CHECK>(cx, heavy, off, rec_at<GLOBAL>(cx, heavy, off), x, c,
-                                                  place, st);
+                                                  place, st, fwd);
         }
-        return;
+        return fwd;
     }
     auto spos = [&](uint32_t i) {
         return (int32_t)(rec_at<GLOBAL>(cx, heavy, ep + i * es).y & kSuccPosMask);
@@ -154,7 +159,7 @@ __device__ __forceinline__ void push_all32(const Ctx32 &cx, const uint8_t *heavy
     auto push_i = [&](uint32_t i) {
         const uint32_t off = ep + i * es;
         push32<MULTI, GLOBAL, ALL_MAX, CHECK>(cx, heavy, off, rec_at<GLOBAL>(cx, heavy, off), x, c,
-                                              place, st);
+                                              place, st, fwd);
     };
     for (uint32_t i = 0; i < nout;) {
         if (spos(i) != ks) {
@@ -170,44 +175,50 @@ __device__ __forceinline__ void push_all32(const Ctx32 &cx, const uint8_t *heavy
         for (uint32_t e = i; e < a_end; e++) push_i(e);
         i = b_end;
     }
+    return fwd;
 }
 
-// Relax the op at position v whose records start at shared byte offset rp.  `cold_in` is its
-// far arrivals (loaded one op earlier); the next position's are loaded into `cold_out`.
+// Relax the op at position v (record o at shared offset rp) whose arrivals are r (the max of
+// its far, ring and forwarded arrivals).  Returns the forwarded arrival for position v + 1.
 template <bool MULTI, bool ALL_MAX, bool CHECK, class PlaceT, class StateT>
-__device__ __forceinline__ uint32_t relax32(const Ctx32 &cx, uint32_t rp, int32_t v, int32_t ks,
-                                            const uint8_t *heavy, const PlaceT &place,
-                                            StateT &st, uint32_t cold_in, uint32_t &cold_out) {
-    const uint4 o = *reinterpret_cast<const uint4 *>(cx.smem + rp);  // {p, cold_next, pf, nout}
-    if ((int32_t)o.z >= 0) prefetch_l1(cx.cold + (size_t)o.z * 32);
-    cold_out = (int32_t)o.y >= 0 ? cx.cold[(size_t)o.y * 32] : 0u;
+__device__ __forceinline__ uint32_t relax32(const Ctx32 &cx, uint32_t rp, const uint4 o, int32_t v,
+                                            int32_t ks, const uint8_t *heavy, const PlaceT &place,
+                                            StateT &st, uint32_t r) {
     const int x = place.template at<CHECK>(v, (int)((o.w >> kOpXShift) & 7u));
-    uint32_t r = cold_in;
-    if (o.w & kOp32HasNear) r = max(r, lds_u32(cx.ring + (uint32_t)(v & (kRing - 1)) * 128));
     const uint32_t c = add_sat(max(r, st.dev(x)), o.x);    // C_v = S_v + p_v
     st.set_dev(x, c);
     const bool adj = (o.w & kOpAdj) != 0;
-    if (!(o.w & kOpHeavy)) {
-        const uint32_t nout = o.w & kOpNoutMask;
-        push_all32<MULTI, false, ALL_MAX, CHECK>(cx, heavy, rp + 16, nout, adj, ks, x, c, place, st);
-        return rp + 16 + nout * stride32<MULTI>(cx);
-    }
+    if (!(o.w & kOpHeavy))
+        return push_all32<MULTI, false, ALL_MAX, CHECK>(cx, heavy, rp + 16, o.w & kOpNoutMask, adj,
+                                                        ks, x, c, place, st);
     const uint4 ext = *reinterpret_cast<const uint4 *>(cx.smem + rp + 16);   // ExtRec
-    push_all32<MULTI, true, ALL_MAX, CHECK>(cx, heavy, ext.x, ext.z, adj, ks, x, c, place, st);
-    return rp + 32;
+    return push_all32<MULTI, true, ALL_MAX, CHECK>(cx, heavy, ext.x, ext.z, adj, ks, x, c, place, st);
 }
 
 template <bool MULTI>
-__device__ __forceinline__ uint32_t skip32(const Ctx32 &cx, uint32_t rp) {
-    const uint32_t nout = reinterpret_cast<const uint32_t *>(cx.smem + rp)[3];
+__device__ __forceinline__ uint32_t next_rp(const Ctx32 &cx, uint32_t rp, uint32_t nout) {
     if (nout & kOpHeavy) return rp + 32;
     return rp + 16 + (nout & kOpNoutMask) * stride32<MULTI>(cx);
+}
+
+__device__ __forceinline__ uint4 op_at(const Ctx32 &cx, uint32_t rp) {
+    return *reinterpret_cast<const uint4 *>(cx.smem + rp);
+}
+__device__ __forceinline__ uint32_t ring_at(const Ctx32 &cx, int32_t v) {
+    return lds_u32(cx.ring + (uint32_t)(v & (kRing - 1)) * 128);
+}
+__device__ __forceinline__ uint32_t cold_at(const Ctx32 &cx, int32_t slot) {
+    return slot >= 0 ? cx.cold[(size_t)slot * 32] : 0u;
+}
+__device__ __forceinline__ uint32_t arrivals(const uint4 o, uint32_t ring, uint32_t cold, uint32_t fwd) {
+    uint32_t r = max(cold, fwd);
+    return (o.w & kOp32HasNear) ? max(r, ring) : r;
 }
 
 // zero the slots an op opens with a first push (swap pairs only; times are >= 0)
 template <bool MULTI>
 __device__ __forceinline__ void clear_first32(const Ctx32 &cx, uint32_t rp, const uint8_t *heavy) {
-    const uint4 o = *reinterpret_cast<const uint4 *>(cx.smem + rp);
+    const uint4 o = op_at(cx, rp);
     const bool global = (o.w & kOpHeavy) != 0;
     uint32_t ep = rp + 16, nout = o.w & kOpNoutMask;
     if (global) {
@@ -219,7 +230,7 @@ __device__ __forceinline__ void clear_first32(const Ctx32 &cx, uint32_t rp, cons
     for (uint32_t i = 0; i < nout; i++) {
         const uint4 rec = global ? rec_at<true>(cx, heavy, ep + i * es)
                                  : rec_at<false>(cx, heavy, ep + i * es);
-        if (!(rec.z & kT32First)) continue;
+        if (!(rec.z & kT32First) || (rec.z & kT32Next)) continue;
         const uint32_t bytes = rec.z & kT32SlotMask;
         if (rec.z & kT32Near) sts_u32(cx.ring + bytes, 0u);
         else *reinterpret_cast<uint32_t *>(reinterpret_cast<uint8_t *>(cx.cold) + bytes) = 0u;
@@ -346,8 +357,10 @@ eval32_kernel(const EvalParams P) {
         }
         st.init();
 
+        // Software-pipelined walk: while op v is relaxed, op v+1's record, its ring value and
+        // its far arrivals are already in flight; its distance-1 arrival is forwarded in `fwd`.
         bool skip_first = false;
-        uint32_t cold_v = 0;                         // far arrivals of the next op to relax
+        uint32_t cold_v = 0, fwd = 0;
         for (int t = 0; t < nt; t++, it++) {
             const int s = it % kStages;
             mbar_wait(&full[s], (it / kStages) & 1);
@@ -357,23 +370,42 @@ eval32_kernel(const EvalParams P) {
                 int32_t v = reinterpret_cast<const int32_t *>(smem + tile)[0];
                 uint32_t rp = tile + kTileHeader;
                 if (skip_first) {
-                    rp = skip32<MULTI>(cx, rp);
+                    rp = next_rp<MULTI>(cx, rp, op_at(cx, rp).w);
                     v++;
                     skip_first = false;
                 }
+                uint4 o = op_at(cx, rp);
+                uint32_t ringv = ring_at(cx, v);
                 // past the region (and past any swap, which lies in it) every op is base-coded
-                if (MODE == 0 || (v >= check_end && ks < v)) {
-                    for (; v < pos_end; v++)
-                        rp = relax32<MULTI, false, false>(cx, rp, v, -1, heavy, place, st, cold_v, cold_v);
-                }
+                const bool plain = MODE == 0 || (v >= check_end && ks < v);
                 while (v < pos_end) {
+                    if (plain || (v != ks && v >= check_end)) {
+                        const uint32_t rp_n = next_rp<MULTI>(cx, rp, o.w);
+                        uint4 o_n = o;
+                        uint32_t ring_n = 0;
+                        if (v + 1 < pos_end) { o_n = op_at(cx, rp_n); ring_n = ring_at(cx, v + 1); }
+                        const uint32_t cold_n = cold_at(cx, (int32_t)o.y);
+                        if ((int32_t)o.z >= 0) prefetch_l1(cx.cold + (size_t)o.z * 32);
+                        fwd = relax32<MULTI, false, false>(cx, rp, o, v, -1, heavy, place, st,
+                                                           arrivals(o, ringv, cold_v, fwd));
+                        rp = rp_n; o = o_n; ringv = ring_n; cold_v = cold_n; v++;
+                        continue;
+                    }
                     if (v != ks) {
-                        rp = relax32<MULTI, false, true>(cx, rp, v, ks, heavy, place, st, cold_v, cold_v);
-                        v++;
+                        const uint32_t rp_n = next_rp<MULTI>(cx, rp, o.w);
+                        uint4 o_n = o;
+                        uint32_t ring_n = 0;
+                        if (v + 1 < pos_end) { o_n = op_at(cx, rp_n); ring_n = ring_at(cx, v + 1); }
+                        const uint32_t cold_n = cold_at(cx, (int32_t)o.y);
+                        if ((int32_t)o.z >= 0) prefetch_l1(cx.cold + (size_t)o.z * 32);
+                        fwd = relax32<MULTI, false, true>(cx, rp, o, v, ks, heavy, place, st,
+                                                          arrivals(o, ringv, cold_v, fwd));
+                        rp = rp_n; o = o_n; ringv = ring_n; cold_v = cold_n; v++;
                         continue;
                     }
                     // swapped pair: ops at ks+1 then ks
                     const uint32_t rk = rp;
+                    const uint4 o_k = o;
                     uint32_t rk1;
                     const bool straddle = (v + 1 == pos_end);
                     if (straddle) {
@@ -381,22 +413,27 @@ eval32_kernel(const EvalParams P) {
                         mbar_wait(&full[s2], ((it + 1) / kStages) & 1);
                         rk1 = (uint32_t)s2 * sb + kTileHeader;
                     } else {
-                        rk1 = skip32<MULTI>(cx, rk);
+                        rk1 = next_rp<MULTI>(cx, rk, o_k.w);
                     }
-                    const int32_t cold_k1 = reinterpret_cast<const int32_t *>(smem + rk)[1];
-                    const uint32_t cold_first = cold_k1 >= 0 ? cx.cold[(size_t)cold_k1 * 32] : 0u;
-                    uint32_t dummy, next_v;
+                    const uint4 o_k1 = op_at(cx, rk1);
+                    const uint32_t ring_k1 = ring_at(cx, v + 1);
+                    const uint32_t cold_k1 = cold_at(cx, (int32_t)o_k.y);   // k's record names k+1
+                    const uint32_t cold_k2 = cold_at(cx, (int32_t)o_k1.y);
                     clear_first32<MULTI>(cx, rk, heavy);
-                    const uint32_t after = relax32<MULTI, false, true>(cx, rk1, v + 1, ks, heavy, place,
-                                                                       st, cold_first, next_v);
-                    relax32<MULTI, true, true>(cx, rk, v, ks, heavy, place, st, cold_v, dummy);
-                    cold_v = next_v;                 // ks+1's record names the op at ks+2
+                    // k+1 first: its only distance-1 producer would be k, which it does not use
+                    const uint32_t fwd_k2 = relax32<MULTI, false, true>(
+                        cx, rk1, o_k1, v + 1, ks, heavy, place, st, arrivals(o_k1, ring_k1, cold_k1, 0u));
+                    relax32<MULTI, true, true>(cx, rk, o_k, v, ks, heavy, place, st,
+                                               arrivals(o_k, ringv, cold_v, fwd));
+                    fwd = fwd_k2;
+                    cold_v = cold_k2;
                     if (straddle) {
                         skip_first = true;
                         v = pos_end;
                     } else {
-                        rp = after;
+                        rp = next_rp<MULTI>(cx, rk1, o_k1.w);
                         v += 2;
+                        if (v < pos_end) { o = op_at(cx, rp); ringv = ring_at(cx, v); }
                     }
                 }
             }

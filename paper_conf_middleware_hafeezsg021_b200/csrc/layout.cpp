@@ -200,6 +200,8 @@ pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<
     }
 
     // ---------------- eval32 stream ----------------
+    // distance 1: the next op's forwarding register; 2..kNearDelta: the ring; farther: cold slot
+    auto next_edge = [&](int64_t e) { return pos[g->dst[e]] - pos[g->src[e]] == 1; };
     auto near_edge = [&](int64_t e) { return pos[g->dst[e]] - pos[g->src[e]] <= kNearDelta; };
     std::vector<int32_t> first_far, cslot;
     std::vector<uint8_t> has_near;
@@ -209,12 +211,13 @@ pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<
         has_near.assign(n, 0);
         for (int64_t e = 0; e < m; e++) {
             const int32_t w = g->dst[e];
-            if (near_edge(e)) { has_near[w] = 1; continue; }
+            if (next_edge(e)) continue;                       // register-forwarded
+            if (near_edge(e)) { has_near[w] = 1; continue; }  // shared-memory ring
             const int32_t ps = pos[g->src[e]];
             if (first_far[w] < 0 || ps < first_far[w]) first_far[w] = ps;
         }
         L->W32 = std::max(colour_intervals(n, first_far, pos, cslot), 1);
-        if (L->W32 >= (1 << 23)) L->W32 = 0;  // slot byte offsets must fit 30 bits: 64-bit path
+        if (L->W32 >= (1 << 22)) L->W32 = 0;  // slot byte offsets must fit 29 bits: 64-bit path
     }
     if (L->W32 > 0) {
         std::vector<uint8_t> seen_near(n, 0), seen_far(n, 0), first32(m, 0);
@@ -223,6 +226,7 @@ pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<
             for (int64_t i = g->out_off[u]; i < g->out_off[u + 1]; i++) {
                 const int64_t e = sorted[i];
                 const int32_t w = g->dst[e];
+                if (next_edge(e)) continue;
                 uint8_t &seen = near_edge(e) ? seen_near[w] : seen_far[w];
                 if (!seen) { seen = 1; first32[e] = 1; }
             }
@@ -251,7 +255,8 @@ pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<
             const int32_t w = g->dst[e];
             r.succ_pos = (int32_t)((uint32_t)pos[w] | (xcode(w) << kSuccXShift));
             // byte offset of the lane's slot column: ring slot (pos & 15) or cold slot, x 128
-            r.target = (near_edge(e) ? (kT32Near | (uint32_t)(pos[w] & (kRing - 1)) * 128u)
+            r.target = next_edge(e) ? kT32Next
+                     : (near_edge(e) ? (kT32Near | (uint32_t)(pos[w] & (kRing - 1)) * 128u)
                                      : (uint32_t)cslot[w] * 128u) |
                        (first32[e] ? kT32First : 0u);
             std::memcpy(buf.data() + at, &r, sizeof r);

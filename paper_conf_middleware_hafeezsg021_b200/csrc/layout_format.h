@@ -73,7 +73,8 @@ constexpr uint32_t kSuccPosMask = (1u << 24) - 1;
 constexpr uint32_t kPinHeavy = 1u << 31;        // patch reference into the out-of-line array
 constexpr uint32_t kT32First = 1u << 31;        // EdgeRec32.target: first push into its slot
 constexpr uint32_t kT32Near = 1u << 30;         // push into the near ring (slot = succ & 15)
-constexpr uint32_t kT32SlotMask = (1u << 30) - 1;   // byte offset (slot x 128) of the target
+constexpr uint32_t kT32Next = 1u << 29;         // consumer is the next position: register
+constexpr uint32_t kT32SlotMask = (1u << 29) - 1;   // byte offset (slot x 128) of the target
 
 struct alignas(16) OpRec32 {
     uint32_t p;          // p_v (< kMaxDur32)
