@@ -67,6 +67,21 @@ __device__ __forceinline__ void sts_u64(uint32_t addr, uint64_t v) {
     asm volatile("st.shared.u64 [%0], %1;" ::"r"(addr), "l"(v) : "memory");
 }
 
+// per-thread async copy of 4 bytes global -> shared (LDGSTS), in commit groups
+__device__ __forceinline__ void cp_async4(uint32_t smem_addr, const void *gptr, bool pred) {
+    asm volatile(
+        "{\n .reg .pred p;\n setp.ne.b32 p, %2, 0;\n"
+        " @p cp.async.ca.shared.global [%0], [%1], 4;\n}\n"
+        ::"r"(smem_addr), "l"(gptr), "r"((int)pred) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() {
+    asm volatile("cp.async.commit_group;" ::: "memory");
+}
+template <int N>
+__device__ __forceinline__ void cp_async_wait() {
+    asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
+}
+
 template <int PL>
 __device__ __forceinline__ int bits_dev_at(const uint32_t *bits, int words, int32_t q) {
     int x = 0;

@@ -5,8 +5,8 @@
 //   cross e=(v,w): A_e = max(C_v, link_free[x_v->x_w]) + t_e;  link_free = A_e
 // with the ready-time state split by producer distance:
 //   near (consumer within kNearDelta positions): the warp's shared-memory ring, slot = pos & 15
-//   far:  a global cold slot written with fire-and-forget STG (first push) / RED.MAX, prefetched
-//         into L1 kPrefetchDist positions ahead and loaded one op before the consumer runs.
+//   far:  a global cold slot written with fire-and-forget STG (first push) / RED.MAX, and
+//         copied into a shared staging ring with cp.async kPrefetchDist positions ahead.
 // One lane = one candidate, 32 candidates per warp share every DAG tile, which the producer
 // warp streams into shared memory with cp.async.bulk (TMA) through an mbarrier ring.
 // Search candidates differ from their base only inside their group's 64-position region
@@ -249,6 +249,8 @@ eval32_kernel(const EvalParams P) {
     cur = align16(cur + 64);
     uint32_t *ring_all = reinterpret_cast<uint32_t *>(cur);
     cur = align16(cur + (size_t)kWarps * kRing * 32 * 4);
+    uint32_t *stage_all = reinterpret_cast<uint32_t *>(cur);          // far-arrival staging
+    cur = align16(cur + (size_t)kWarps * kRing * 32 * 4);
     uint32_t *dstate = reinterpret_cast<uint32_t *>(cur);
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -295,6 +297,7 @@ eval32_kernel(const EvalParams P) {
     cx.edge_stride = P.edge_stride32;
     cx.D = P.D;
     cx.two_classes = P.n_classes > 1;
+    const uint32_t stage = su32(stage_all + (size_t)warp * kRing * 32 + lane);
 
     using StateT = typename std::conditional<PL == 1, RegState32, SmemState32>::type;
     StateT st;
@@ -303,6 +306,21 @@ eval32_kernel(const EvalParams P) {
         st.d = su32(dstate + (size_t)warp * (P.D + P.D * P.D) * 32 + lane);
         st.l = st.d + (uint32_t)P.D * 128;
     }
+
+    // Far arrivals of position q arrive by cp.async into stage[q & 15], issued while position
+    // q - kPrefetchDist is relaxed (its record names the slot); one commit group per position,
+    // so waiting for all but kPrefetchDist groups makes position q's value visible.  The first
+    // kPrefetchDist positions of a task load it directly.
+    auto issue_far = [&](const uint4 o, int32_t v) {
+        cp_async4(stage + (uint32_t)((v + kPrefetchDist) & (kRing - 1)) * 128,
+                  cx.cold + (size_t)(int32_t)o.z * 32, (int32_t)o.z >= 0);
+        cp_async_commit();
+    };
+    auto far_of = [&](const uint4 o, int32_t v) -> uint32_t {
+        if ((int32_t)o.y < 0) return 0u;
+        if (v < kPrefetchDist) return cx.cold[(size_t)(int32_t)o.y * 32];
+        return lds_u32(stage + (uint32_t)(v & (kRing - 1)) * 128);
+    };
 
     uint32_t it = 0;
     for (int64_t task = blockIdx.x; task < P.n_tasks; task += gridDim.x) {
@@ -357,10 +375,10 @@ eval32_kernel(const EvalParams P) {
         }
         st.init();
 
-        // Software-pipelined walk: while op v is relaxed, op v+1's record, its ring value and
-        // its far arrivals are already in flight; its distance-1 arrival is forwarded in `fwd`.
+        // While op v is relaxed, op v+1's record and ring value are already loaded; its
+        // distance-1 arrival is forwarded in `fwd`; far arrivals come through the staging ring.
         bool skip_first = false;
-        uint32_t cold_v = 0, fwd = 0;
+        uint32_t fwd = 0;
         for (int t = 0; t < nt; t++, it++) {
             const int s = it % kStages;
             mbar_wait(&full[s], (it / kStages) & 1);
@@ -376,31 +394,21 @@ eval32_kernel(const EvalParams P) {
                 }
                 uint4 o = op_at(cx, rp);
                 uint32_t ringv = ring_at(cx, v);
-                // past the region (and past any swap, which lies in it) every op is base-coded
-                const bool plain = MODE == 0 || (v >= check_end && ks < v);
                 while (v < pos_end) {
-                    if (plain || (v != ks && v >= check_end)) {
+                    const bool plain = MODE == 0 || (v >= check_end && ks < v);
+                    if (plain || v != ks) {
                         const uint32_t rp_n = next_rp<MULTI>(cx, rp, o.w);
                         uint4 o_n = o;
                         uint32_t ring_n = 0;
                         if (v + 1 < pos_end) { o_n = op_at(cx, rp_n); ring_n = ring_at(cx, v + 1); }
-                        const uint32_t cold_n = cold_at(cx, (int32_t)o.y);
-                        if ((int32_t)o.z >= 0) prefetch_l1(cx.cold + (size_t)o.z * 32);
-                        fwd = relax32<MULTI, false, false>(cx, rp, o, v, -1, heavy, place, st,
-                                                           arrivals(o, ringv, cold_v, fwd));
-                        rp = rp_n; o = o_n; ringv = ring_n; cold_v = cold_n; v++;
-                        continue;
-                    }
-                    if (v != ks) {
-                        const uint32_t rp_n = next_rp<MULTI>(cx, rp, o.w);
-                        uint4 o_n = o;
-                        uint32_t ring_n = 0;
-                        if (v + 1 < pos_end) { o_n = op_at(cx, rp_n); ring_n = ring_at(cx, v + 1); }
-                        const uint32_t cold_n = cold_at(cx, (int32_t)o.y);
-                        if ((int32_t)o.z >= 0) prefetch_l1(cx.cold + (size_t)o.z * 32);
-                        fwd = relax32<MULTI, false, true>(cx, rp, o, v, ks, heavy, place, st,
-                                                          arrivals(o, ringv, cold_v, fwd));
-                        rp = rp_n; o = o_n; ringv = ring_n; cold_v = cold_n; v++;
+                        issue_far(o, v);
+                        cp_async_wait<kPrefetchDist>();
+                        const uint32_t r = arrivals(o, ringv, far_of(o, v), fwd);
+                        if (plain)
+                            fwd = relax32<MULTI, false, false>(cx, rp, o, v, -1, heavy, place, st, r);
+                        else
+                            fwd = relax32<MULTI, false, true>(cx, rp, o, v, ks, heavy, place, st, r);
+                        rp = rp_n; o = o_n; ringv = ring_n; v++;
                         continue;
                     }
                     // swapped pair: ops at ks+1 then ks
@@ -417,16 +425,17 @@ eval32_kernel(const EvalParams P) {
                     }
                     const uint4 o_k1 = op_at(cx, rk1);
                     const uint32_t ring_k1 = ring_at(cx, v + 1);
-                    const uint32_t cold_k1 = cold_at(cx, (int32_t)o_k.y);   // k's record names k+1
-                    const uint32_t cold_k2 = cold_at(cx, (int32_t)o_k1.y);
+                    issue_far(o_k, v);
+                    issue_far(o_k1, v + 1);
+                    cp_async_wait<kPrefetchDist>();
+                    const uint32_t far_k = far_of(o_k, v), far_k1 = far_of(o_k1, v + 1);
                     clear_first32<MULTI>(cx, rk, heavy);
                     // k+1 first: its only distance-1 producer would be k, which it does not use
                     const uint32_t fwd_k2 = relax32<MULTI, false, true>(
-                        cx, rk1, o_k1, v + 1, ks, heavy, place, st, arrivals(o_k1, ring_k1, cold_k1, 0u));
+                        cx, rk1, o_k1, v + 1, ks, heavy, place, st, arrivals(o_k1, ring_k1, far_k1, 0u));
                     relax32<MULTI, true, true>(cx, rk, o_k, v, ks, heavy, place, st,
-                                               arrivals(o_k, ringv, cold_v, fwd));
+                                               arrivals(o_k, ringv, far_k, fwd));
                     fwd = fwd_k2;
-                    cold_v = cold_k2;
                     if (straddle) {
                         skip_first = true;
                         v = pos_end;
@@ -440,6 +449,7 @@ eval32_kernel(const EvalParams P) {
             __syncwarp();
             if (lane == 0) mbar_arrive(&empty[s]);
         }
+        cp_async_wait<0>();
 
         if (!active) continue;
         const uint32_t mk = st.makespan();
@@ -498,7 +508,9 @@ int eval32_smem_bytes(const EvalParams &p, int search_mode) {
     b = (b + 15) & ~size_t(15);
     b += 64;
     b = (b + 15) & ~size_t(15);
-    b += (size_t)kWarps * kRing * 32 * 4;
+    b += (size_t)kWarps * kRing * 32 * 4;          // near ring
+    b = (b + 15) & ~size_t(15);
+    b += (size_t)kWarps * kRing * 32 * 4;          // far-arrival staging
     b = (b + 15) & ~size_t(15);
     if (pl != 1) b += (size_t)kWarps * (p.D + p.D * p.D) * 32 * 4;
     return (int)b + 128;

@@ -279,7 +279,7 @@ pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<
                 if (succ_pos(sorted[i]) == succ_pos(sorted[i - 1]) + 1) adj = true;
             OpRec32 op;
             op.p = (uint32_t)g->p[u];
-            op.cold_next = k + 1 < n ? cslot[order[k + 1]] : -1;
+            op.cold_slot = cslot[u];
             const int32_t ahead = k + kPrefetchDist;
             op.pf_slot = ahead < n ? cslot[order[ahead]] : -1;
             op.nout = (heavy ? kOpHeavy : (uint32_t)nout) | (has_near[u] ? kOp32HasNear : 0u) |

@@ -78,8 +78,8 @@ constexpr uint32_t kT32SlotMask = (1u << 29) - 1;   // byte offset (slot x 128) 
 
 struct alignas(16) OpRec32 {
     uint32_t p;          // p_v (< kMaxDur32)
-    int32_t cold_next;   // cold slot of the op at the next position (loaded one op ahead); -1
-    int32_t pf_slot;     // cold slot of the op kPrefetchDist positions ahead; -1 = none
+    int32_t cold_slot;   // this op's cold slot (far arrivals); -1 = none
+    int32_t pf_slot;     // cold slot of the op kPrefetchDist positions ahead (async-copied); -1
     uint32_t nout;       // out-degree | kOp32HasNear | kOpAdj | base code << 25 | kOpHeavy
 };
 
