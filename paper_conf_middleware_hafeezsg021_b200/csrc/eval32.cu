@@ -76,7 +76,7 @@ struct Place32 {
 };
 
 struct Ctx32 {
-    const uint8_t *smem;         // the CTA's dynamic shared memory (records addressed from here)
+    uint32_t smem;               // shared address of the CTA's dynamic shared memory (records)
     uint32_t ring;               // shared address of ring[0][lane]; slot bytes from the record
     uint32_t *cold;              // global: cold[slot * 32 + lane]
     uint32_t lclass;             // shared address of the link-class table
@@ -92,7 +92,7 @@ __device__ __forceinline__ void prefetch_l1(const void *p) {
 template <bool GLOBAL>
 __device__ __forceinline__ uint4 rec_at(const Ctx32 &cx, const uint8_t *heavy, uint32_t off) {
     if (GLOBAL) return __ldg(reinterpret_cast<const uint4 *>(heavy + off));
-    return *reinterpret_cast<const uint4 *>(cx.smem + off);
+    return lds_v4(cx.smem + off);
 }
 
 template <bool MULTI>
@@ -114,7 +114,7 @@ __device__ __forceinline__ void push32(const Ctx32 &cx, const uint8_t *heavy, ui
             else if (MULTI && cls > 1) {
                 const uint32_t eo = off + 16 + 4 * (cls - 2);
                 t = GLOBAL ? __ldg(reinterpret_cast<const uint32_t *>(heavy + eo))
-                           : *reinterpret_cast<const uint32_t *>(cx.smem + eo);
+                           : lds_u32(cx.smem + eo);
             }
         }
         a = add_sat(max(c, st.link(x, y)), t);
@@ -191,7 +191,7 @@ __device__ __forceinline__ uint32_t relax32(const Ctx32 &cx, uint32_t rp, const 
     if (!(o.w & kOpHeavy))
         return push_all32<MULTI, false, ALL_MAX, CHECK>(cx, heavy, rp + 16, o.w & kOpNoutMask, adj,
                                                         ks, x, c, place, st);
-    const uint4 ext = *reinterpret_cast<const uint4 *>(cx.smem + rp + 16);   // ExtRec
+    const uint4 ext = lds_v4(cx.smem + rp + 16);   // ExtRec
     return push_all32<MULTI, true, ALL_MAX, CHECK>(cx, heavy, ext.x, ext.z, adj, ks, x, c, place, st);
 }
 
@@ -202,7 +202,7 @@ __device__ __forceinline__ uint32_t next_rp(const Ctx32 &cx, uint32_t rp, uint32
 }
 
 __device__ __forceinline__ uint4 op_at(const Ctx32 &cx, uint32_t rp) {
-    return *reinterpret_cast<const uint4 *>(cx.smem + rp);
+    return lds_v4(cx.smem + rp);
 }
 __device__ __forceinline__ uint32_t ring_at(const Ctx32 &cx, int32_t v) {
     return lds_u32(cx.ring + (uint32_t)(v & (kRing - 1)) * 128);
@@ -222,7 +222,7 @@ __device__ __forceinline__ void clear_first32(const Ctx32 &cx, uint32_t rp, cons
     const bool global = (o.w & kOpHeavy) != 0;
     uint32_t ep = rp + 16, nout = o.w & kOpNoutMask;
     if (global) {
-        const uint4 ext = *reinterpret_cast<const uint4 *>(cx.smem + rp + 16);
+        const uint4 ext = lds_v4(cx.smem + rp + 16);
         ep = ext.x;
         nout = ext.z;
     }
@@ -290,7 +290,7 @@ eval32_kernel(const EvalParams P) {
     }
 
     Ctx32 cx;
-    cx.smem = smem;
+    cx.smem = su32(smem);
     cx.ring = su32(ring_all + (size_t)warp * kRing * 32 + lane);
     cx.cold = P.state32 + ((size_t)(blockIdx.x * kWarps + warp) * P.max_W32) * 32 + lane;
     cx.lclass = su32(lclass);
@@ -384,8 +384,9 @@ eval32_kernel(const EvalParams P) {
             mbar_wait(&full[s], (it / kStages) & 1);
             if (active) {
                 const uint32_t tile = (uint32_t)s * sb;
-                const int32_t pos_end = reinterpret_cast<const int32_t *>(smem + tile)[1];
-                int32_t v = reinterpret_cast<const int32_t *>(smem + tile)[0];
+                const uint4 hdr = lds_v4(cx.smem + tile);
+                const int32_t pos_end = (int32_t)hdr.y;
+                int32_t v = (int32_t)hdr.x;
                 uint32_t rp = tile + kTileHeader;
                 if (skip_first) {
                     rp = next_rp<MULTI>(cx, rp, op_at(cx, rp).w);
