@@ -611,16 +611,16 @@ int oracle_candidate(int32_t n, int64_t m, const int32_t *src, const int32_t *ds
     const int32_t *bo = base_order + (int64_t)b * n;
     memcpy(x_out, bx, (size_t)n);
     memcpy(order_out, bo, (size_t)n * sizeof(int32_t));
-    int64_t g = j >> 5, lane = j & 31;
+    int64_t g = j >> 7, lane = j & 127;      /* groups of 128 candidate ids (DESIGN §4 S2) */
     int swap = 0;
     /* the group's region: positions [c, c + len) of the base order (DESIGN §4 S2) */
-    int64_t c0 = (int64_t)(oracle_draw(seed, step, P, b, 32 * g, 13) % (uint64_t)n);
+    int64_t c0 = (int64_t)(oracle_draw(seed, step, P, b, 128 * g, 13) % (uint64_t)n);
     int64_t rlen = n - c0 < 64 ? n - c0 : 64;
-    /* order move: one adjacent swap per group of 32 candidates (DESIGN §4 S3) */
+    /* order move: one adjacent swap per group (DESIGN §4 S3) */
     if (g != 0 && mix[3] > 0 && n >= 2) {
-        uint64_t u = oracle_draw(seed, step, P, b, 32 * g, 15);
+        uint64_t u = oracle_draw(seed, step, P, b, 128 * g, 15);
         if ((int64_t)(u % 100u) < mix[3]) {
-            int64_t k = c0 + (int64_t)(oracle_draw(seed, step, P, b, 32 * g, 14) % (uint64_t)rlen);
+            int64_t k = c0 + (int64_t)(oracle_draw(seed, step, P, b, 128 * g, 14) % (uint64_t)rlen);
             if (k > n - 2) k = n - 2;
             int32_t a = bo[k], c = bo[k + 1];
             int joined = 0;

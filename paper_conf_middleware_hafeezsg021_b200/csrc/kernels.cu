@@ -313,13 +313,14 @@ eval_kernel(const EvalParams P) {
             active = g < P.group_begin + P.groups_per_base;
             const int breal = P.b_offset + bl;
             const uint64_t cb = ctr_base_of(P.step, P.P_total, breal);
-            const Region rg = decode_region(P.seed, cb, g, P.n);
+            const int64_t grp = (g * 32) >> kGroupShift;          // spec group of this warp
+            const Region rg = decode_region(P.seed, cb, grp, P.n);
             place.rc = rg.c;
             place.rlen = rg.len;
             place.bits = B->bits;
             place.allowed_pos = B->allowed_pos;
             const uint8_t *adj = B->adj_next;
-            ks = active ? decode_swap(P.seed, cb, g, P.n, P.mix[3], rg,
+            ks = active ? decode_swap(P.seed, cb, grp, P.n, P.mix[3], rg,
                                       [&](int32_t k) { return __ldg(adj + k) != 0; })
                         : -1;
             const bool in_range = active && j >= P.j_begin && j < P.j_end;
@@ -328,7 +329,7 @@ eval_kernel(const EvalParams P) {
             const uint8_t *aop = P.allowed_op;
             const int words = P.words;
             place.mv = in_range
-                ? decode_lane(P.seed, cb, j, ks >= 0 && lane == 0, P.D, P.mix, rg,
+                ? decode_lane(P.seed, cb, j, ks >= 0 && (j & (kGroup - 1)) == 0, P.D, P.mix, rg,
                               [&](int32_t q) { return __ldg(ord + q); },
                               [&](int32_t q) { return ldg_bits_dev_at<PL>(bits, words, q); },
                               [&](int32_t op) { return (unsigned)__ldg(aop + op); })
@@ -520,12 +521,12 @@ __global__ void commit_kernel(const CommitParams P) {
     uint32_t *bits = P.bits + (size_t)b * PL * P.words;
     const uint64_t cb = ctr_base_of(P.step, P.P, b);
     const uint8_t *adj = B.adj_next;
-    const Region rg = decode_region(P.seed, cb, j >> 5, P.n);
-    const int32_t ks = decode_swap(P.seed, cb, j >> 5, P.n, P.mix[3], rg,
+    const Region rg = decode_region(P.seed, cb, j >> kGroupShift, P.n);
+    const int32_t ks = decode_swap(P.seed, cb, j >> kGroupShift, P.n, P.mix[3], rg,
                                    [&](int32_t k) { return adj[k] != 0; });
     const int words = P.words;
     const LaneMove mv = decode_lane(
-        P.seed, cb, j, ks >= 0 && (j & 31) == 0, P.D, P.mix, rg,
+        P.seed, cb, j, ks >= 0 && (j & (kGroup - 1)) == 0, P.D, P.mix, rg,
         [&](int32_t q) { return B.order[q]; },
         [&](int32_t q) { return get_dev_at<PL>(bits, words, q); },
         [&](int32_t op) { return (unsigned)P.allowed_op[op]; });

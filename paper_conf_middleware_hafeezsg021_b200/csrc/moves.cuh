@@ -48,7 +48,9 @@ struct LaneMove {
     int32_t ws, wl, wd;  // window: positions [ws, ws + wl) move to wd where allowed
 };
 
-constexpr int kRegion = 64;     // positions a group of 32 candidates may change (DESIGN §4 S2)
+constexpr int kRegion = 64;     // positions a group of candidates may change (DESIGN §4 S2)
+constexpr int kGroupShift = 7;  // a group = 128 consecutive candidate ids
+constexpr int kGroup = 1 << kGroupShift;
 
 // The group's region [c, c + len) of the base order.
 struct Region {
@@ -56,18 +58,18 @@ struct Region {
 };
 PESTO_HD Region decode_region(uint64_t seed, uint64_t cb, int64_t group, int n) {
     Region r;
-    r.c = (int32_t)(draw(seed, cb, group * 32, 13) % (uint64_t)n);
+    r.c = (int32_t)(draw(seed, cb, group * kGroup, 13) % (uint64_t)n);
     r.len = n - r.c < kRegion ? n - r.c : kRegion;
     return r;
 }
 
-// Group (warp) order move: adjacent swap of positions (k, k+1) of the base order, or -1.
+// Group order move: adjacent swap of positions (k, k+1) of the base order, or -1.
 // adj_next(k) must say whether an edge joins order[k] -> order[k+1].
 template <class AdjNext>
 PESTO_HD int32_t decode_swap(uint64_t seed, uint64_t cb, int64_t group, int n, int swap_pct,
                              Region rg, AdjNext adj_next) {
     if (group == 0 || swap_pct <= 0 || n < 2) return -1;
-    int64_t j0 = group * 32;
+    int64_t j0 = group * kGroup;
     if ((int)(draw(seed, cb, j0, 15) % 100u) >= swap_pct) return -1;
     int32_t k = rg.c + (int32_t)(draw(seed, cb, j0, 14) % (uint64_t)rg.len);
     if (k > n - 2) k = n - 2;

@@ -47,7 +47,7 @@ def test_identity_and_move_shapes(O):
                 assert o[k] == orders[b][k + 1] and o[k + 1] == orders[b][k]
                 assert (int(orders[b][k]), int(orders[b][k + 1])) not in edges
                 assert O.makespan(g, x, o) >= 0           # still topological
-                if j % 32 == 0:
+                if j % 128 == 0:
                     assert (x == xs[b]).all()              # lane 0 of a swap group: pure swap
             changed = np.nonzero(x != xs[b])[0]
             if len(changed) == 0:
@@ -67,11 +67,11 @@ def test_group_changes_stay_in_its_region(O):
     g, xs, orders = _setup(seed=6, n=300)
     P = xs.shape[0]
     for b in range(P):
-        for grp in range(1, 40):
-            c = O.draw(2021, 2, P, b, 32 * grp, 13) % g.n
+        for grp in range(1, 12):
+            c = O.draw(2021, 2, P, b, 128 * grp, 13) % g.n
             hi = min(g.n, c + 64)
-            for lane in range(32):
-                j = 32 * grp + lane
+            for lane in range(128):
+                j = 128 * grp + lane
                 ok, x, o = O.candidate(g, P, b, xs, orders, j, 2021, 2, MIX)
                 changed = np.nonzero(x != xs[b])[0]
                 pos = [int(np.nonzero(orders[b] == v)[0][0]) for v in changed]
