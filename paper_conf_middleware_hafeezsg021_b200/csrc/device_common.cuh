@@ -11,6 +11,13 @@ namespace dev {
 __device__ __forceinline__ uint32_t su32(const void *p) {
     return (uint32_t)__cvta_generic_to_shared(p);
 }
+// a shared address the compiler keeps in a register instead of rematerialising it from
+// SR_CgaCtaId before every access
+__device__ __forceinline__ uint32_t su32_reg(const void *p) {
+    uint32_t a;
+    asm volatile("mov.b32 %0, %1;" : "=r"(a) : "r"(su32(p)));
+    return a;
+}
 __device__ __forceinline__ void mbar_init(uint64_t *bar, uint32_t count) {
     asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(su32(bar)), "r"(count) : "memory");
 }

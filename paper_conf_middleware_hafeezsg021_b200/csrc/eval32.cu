@@ -45,8 +45,9 @@ struct RegState32 {          // D <= 2
         if (x) d1[c] = v; else d0[c] = v;
     }
     __device__ __forceinline__ uint32_t link(int c, int x, int) const { return x ? l10[c] : l01[c]; }
-    __device__ __forceinline__ void set_link(int c, int x, int, uint32_t v) {
-        if (x) l10[c] = v; else l01[c] = v;
+    __device__ __forceinline__ void set_link_if(int c, int x, int, bool cond, uint32_t v) {
+        l10[c] = (cond && x) ? v : l10[c];
+        l01[c] = (cond && !x) ? v : l01[c];
     }
     __device__ __forceinline__ uint32_t makespan(int c) const { return max(d0[c], d1[c]); }
 };
@@ -69,8 +70,8 @@ struct SmemState32 {         // D <= 8: [column][CPL][32] in shared memory (shar
     __device__ __forceinline__ uint32_t link(int c, int x, int y) const {
         return lds_u32(at(l, x * D + y, c));
     }
-    __device__ __forceinline__ void set_link(int c, int x, int y, uint32_t v) {
-        sts_u32(at(l, x * D + y, c), v);
+    __device__ __forceinline__ void set_link_if(int c, int x, int y, bool cond, uint32_t v) {
+        if (cond) sts_u32(at(l, x * D + y, c), v);
     }
     __device__ __forceinline__ uint32_t makespan(int c) const {
         uint32_t m = 0;
@@ -135,21 +136,21 @@ __device__ __forceinline__ void push32(const Ctx32 &cx, const uint8_t *heavy, ui
     uint32_t a[CPL];
 #pragma unroll
     for (int c = 0; c < CPL; c++) {
-        a[c] = cc[c];                                        // same device: C_v (L144)
-        if (y[c] != x[c]) {                                  // cross: FCFS link x -> y
-            uint32_t t = rec.x;
-            if (MULTI || cx.two_classes) {
-                const int cls = (int)lds_u8(cx.lclass + (uint32_t)(x[c] * cx.D + y[c]));
-                if (cls == 1) t = rec.w;
-                else if (MULTI && cls > 1) {
-                    const uint32_t eo = off + 16 + 4 * (cls - 2);
-                    t = GLOBAL ? __ldg(reinterpret_cast<const uint32_t *>(heavy + eo))
-                               : lds_u32(cx.smem + eo);
-                }
+        const bool cross = y[c] != x[c];                     // cross: FCFS link x -> y
+        uint32_t t = rec.x;
+        if ((MULTI || cx.two_classes) && cross) {
+            const int cls = (int)lds_u8(cx.lclass + (uint32_t)(x[c] * cx.D + y[c]));
+            if (cls == 1) t = rec.w;
+            else if (MULTI && cls > 1) {
+                const uint32_t eo = off + 16 + 4 * (cls - 2);
+                t = GLOBAL ? __ldg(reinterpret_cast<const uint32_t *>(heavy + eo))
+                           : lds_u32(cx.smem + eo);
             }
-            a[c] = add_sat(max(cc[c], st.link(c, x[c], y[c])), t);
-            st.set_link(c, x[c], y[c], a[c]);
         }
+        // branch-free: the transfer's arrival when crossing, C_v (L144) when not
+        const uint32_t ac = add_sat(max(cc[c], st.link(c, x[c], y[c])), t);
+        a[c] = cross ? ac : cc[c];
+        st.set_link_if(c, x[c], y[c], cross, ac);
     }
     if (tgt & kT32Next) {                                    // consumer is the next position
 #pragma unroll
@@ -323,20 +324,20 @@ eval32_kernel(const EvalParams P) {
     }
 
     Ctx32 cx;
-    cx.smem = su32(smem);
-    cx.ring = su32(ring_all + (size_t)warp * kRing * CW + lane);
+    cx.smem = su32_reg(smem);
+    cx.ring = su32_reg(ring_all + (size_t)warp * kRing * CW + lane);
     cx.cold = reinterpret_cast<uint8_t *>(P.state32 + ((size_t)(blockIdx.x * NW + warp) * P.max_W32) * CW + lane);
-    cx.lclass = su32(lclass);
+    cx.lclass = su32_reg(lclass);
     cx.edge_stride = P.edge_stride32;
     cx.D = P.D;
     cx.two_classes = P.n_classes > 1;
-    const uint32_t stage = su32(stage_all + (size_t)warp * kRing * CW + lane);
+    const uint32_t stage = su32_reg(stage_all + (size_t)warp * kRing * CW + lane);
 
     using StateT = typename std::conditional<PL == 1, RegState32<CPL>, SmemState32<CPL>>::type;
     StateT st;
     if constexpr (PL != 1) {
         st.D = P.D;
-        st.d = su32(dstate + (size_t)warp * (P.D + P.D * P.D) * CW + lane);
+        st.d = su32_reg(dstate + (size_t)warp * (P.D + P.D * P.D) * CW + lane);
         st.l = st.d + (uint32_t)(P.D * CPL) * 128;
     }
 
@@ -457,6 +458,7 @@ eval32_kernel(const EvalParams P) {
                 while (v < pos_end) {
                     if (v != ks) {
                         const uint32_t rp_n = next_rp<MULTI>(cx, rp, o.w);
+                        const uint4 o_n = (v + 1 < pos_end) ? lds_v4(cx.smem + rp_n) : o;
                         issue_far(o, v);
                         cp_async_wait<kPrefetchDist>();
                         uint32_t r[CPL], f[CPL], rg[CPL];
@@ -467,7 +469,7 @@ eval32_kernel(const EvalParams P) {
                         relax32<CPL, MULTI, false>(cx, rp, o, v, ks, heavy, place, st, r, fwd);
                         rp = rp_n;
                         v++;
-                        if (v < pos_end) o = lds_v4(cx.smem + rp);
+                        o = o_n;
                         continue;
                     }
                     // swapped pair: ops at ks+1 then ks
