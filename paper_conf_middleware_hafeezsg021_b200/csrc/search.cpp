@@ -269,7 +269,7 @@ pesto_status pesto_search_create(pesto_graph *g, const pesto_search_desc *d, pes
     cudaMemcpy(s->d_mk.ptr, mk0.data(), 8 * s->P, cudaMemcpyHostToDevice);
     s->h_mk = mk0;
     update_all_below(s.get());
-    if (s->world > 1 && d->nccl_unique_id) {
+    if (d->nccl_unique_id) {                 // (a 1-rank comm is allowed: exercises the path)
         if (!nccl().ok) return fail(PESTO_ENCCL, "libnccl.so.2 not loadable");
         ncclUniqueId id;
         std::memcpy(&id, d->nccl_unique_id, sizeof id);
@@ -372,7 +372,7 @@ pesto_status pesto_search_commit(pesto_search *s, void *stream) {
 
 pesto_status pesto_search_reduce(pesto_search *s, void *stream) {
     if (!s) return fail(PESTO_EINVAL, "NULL search");
-    if (s->world > 1 && s->comm) {
+    if (s->comm) {
         DeviceGuard guard(s->g->device);
         // the step's only cross-GPU exchange: global best (makespan, candidate id) per base
         ncclResult_t r = nccl().all_reduce(s->d_keys.ptr, s->d_keys.ptr, (size_t)s->P, ncclUint64,

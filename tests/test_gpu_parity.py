@@ -228,6 +228,22 @@ def test_fake_sharding_equals_single_rank(P, O):
             assert a[0] == s0[0] and (a[1] == s0[1]).all() and (a[2] == s0[2]).all()
 
 
+def test_nccl_allreduce_path_single_rank(P, O):
+    """the NCCL comm + allreduce-MIN path (1-rank comm) commits the same bases as no comm."""
+    g = _search_graph(seed=71, n=100)
+    G = P.Graph.from_arrays(g)
+    xs, orders = _bases(g, 3, seed=5)
+    plain = P.Search(G, xs, orders, 1024, MIX, seed=3)
+    nccl = P.Search(G, xs, orders, 1024, MIX, seed=3, rank=0, world=1,
+                    nccl_id=P.nccl_unique_id())
+    for _ in range(3):
+        plain.step()
+        nccl.step()
+        for b in range(3):
+            a, c = plain.get(b), nccl.get(b)
+            assert a[0] == c[0] and (a[1] == c[1]).all() and (a[2] == c[2]).all()
+
+
 def test_search_full_size_sampled(P, O):
     """transformer_2dev at full size: a sample of search candidates checked one by one."""
     cfg = configs.CONFIGS["transformer_2dev"]
