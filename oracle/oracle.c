@@ -623,9 +623,26 @@ int oracle_candidate(int32_t n, int64_t m, const int32_t *src, const int32_t *ds
             int64_t k = c0 + (int64_t)(oracle_draw(seed, step, P, b, 128 * g, 14) % (uint64_t)rlen);
             if (k > n - 2) k = n - 2;
             int32_t a = bo[k], c = bo[k + 1];
+            /* blocked (S3): an edge joins them, they share a producer or a consumer, or
+               either has more than 64 successors */
             int joined = 0;
-            for (int64_t e = 0; e < m; e++)
+            int64_t out_a = 0, out_c = 0;
+            for (int64_t e = 0; e < m; e++) {
                 if ((src[e] == a && dst[e] == c) || (src[e] == c && dst[e] == a)) joined = 1;
+                if (src[e] == a) out_a++;
+                if (src[e] == c) out_c++;
+            }
+            uint8_t *mark = calloc((size_t)n, 2);   /* [n] preds of a, [n] succs of a */
+            for (int64_t e = 0; e < m; e++) {
+                if (dst[e] == a) mark[src[e]] = 1;
+                if (src[e] == a) mark[n + dst[e]] = 1;
+            }
+            for (int64_t e = 0; e < m; e++) {
+                if (dst[e] == c && mark[src[e]]) joined = 1;       /* common producer */
+                if (src[e] == c && mark[n + dst[e]]) joined = 1;   /* common consumer */
+            }
+            free(mark);
+            if (out_a > 64 || out_c > 64) joined = 1;
             if (!joined) {
                 order_out[k] = c;
                 order_out[k + 1] = a;

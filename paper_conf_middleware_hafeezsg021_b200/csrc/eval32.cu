@@ -7,8 +7,10 @@
 //   * one warp walks the DAG record stream once for 32 x CPL candidates: every lane carries
 //     CPL candidates, so the warp-uniform work (records, flags, loop control, region checks)
 //     is paid once per CPL candidates;
-//   * the stream is TMA-staged (cp.async.bulk + mbarrier ring) by a producer warp and shared by
-//     all consumer warps of the CTA;
+//   * the stream is a run of fixed 48-byte steps (a head + two out-edge records; an op with
+//     more out-edges continues in CONT steps), so the walk is one straight-line loop; it is
+//     TMA-staged (cp.async.bulk + mbarrier ring) by a producer warp and shared by all consumer
+//     warps of the CTA;
 //   * ready-time state by producer distance: distance 1 -> a register (`fwd`), 2..kNearDelta ->
 //     the warp's shared-memory ring (slot = pos & 15), farther -> a global cold slot written
 //     with fire-and-forget STG / RED.MAX and staged back by cp.async kPrefetchDist positions
@@ -109,24 +111,13 @@ struct Ctx32 {
     uint32_t smem;               // shared address of the CTA's dynamic shared memory (records)
     uint32_t ring;               // shared address of ring[0][0][lane]; slot s, cand c: + (s*CPL+c)*128
     uint8_t *cold;               // global byte address of cold[0][0][lane]; same layout
-    uint32_t lclass;             // shared address of the link-class table
-    int edge_stride, D;
-    bool two_classes;            // a second link class exists (its t is EdgeRec32.t1)
+    uint64_t cls1;               // bit a*D+b: directed link a -> b is in link class 1 (t = t1)
+    int D;
 };
 
-template <bool GLOBAL>
-__device__ __forceinline__ uint4 rec_at(const Ctx32 &cx, const uint8_t *heavy, uint32_t off) {
-    if (GLOBAL) return __ldg(reinterpret_cast<const uint4 *>(heavy + off));
-    return lds_v4(cx.smem + off);
-}
-
-template <bool MULTI>
-__device__ __forceinline__ int stride32(const Ctx32 &cx) { return MULTI ? cx.edge_stride : 16; }
-
-// one out-edge, for the lane's CPL candidates
-template <int CPL, bool MULTI, bool GLOBAL, bool ALL_MAX, class PlaceT, class StateT>
-__device__ __forceinline__ void push32(const Ctx32 &cx, const uint8_t *heavy, uint32_t off,
-                                       const uint4 rec, const int (&x)[CPL],
+// one out-edge record, for the lane's CPL candidates (FCFS link of L144 / L188-198)
+template <int CPL, class PlaceT, class StateT>
+__device__ __forceinline__ void push32(const Ctx32 &cx, const uint4 rec, const int (&x)[CPL],
                                        const uint32_t (&cc)[CPL], const PlaceT &place,
                                        StateT &st, uint32_t (&fwd)[CPL]) {
     const int32_t succ = (int32_t)(rec.y & kSuccPosMask);
@@ -137,16 +128,7 @@ __device__ __forceinline__ void push32(const Ctx32 &cx, const uint8_t *heavy, ui
 #pragma unroll
     for (int c = 0; c < CPL; c++) {
         const bool cross = y[c] != x[c];                     // cross: FCFS link x -> y
-        uint32_t t = rec.x;
-        if ((MULTI || cx.two_classes) && cross) {
-            const int cls = (int)lds_u8(cx.lclass + (uint32_t)(x[c] * cx.D + y[c]));
-            if (cls == 1) t = rec.w;
-            else if (MULTI && cls > 1) {
-                const uint32_t eo = off + 16 + 4 * (cls - 2);
-                t = GLOBAL ? __ldg(reinterpret_cast<const uint32_t *>(heavy + eo))
-                           : lds_u32(cx.smem + eo);
-            }
-        }
+        const uint32_t t = ((cx.cls1 >> (x[c] * cx.D + y[c])) & 1u) ? rec.w : rec.x;
         // branch-free: the transfer's arrival when crossing, C_v (L144) when not
         const uint32_t ac = add_sat(max(cc[c], st.link(c, x[c], y[c])), t);
         a[c] = cross ? ac : cc[c];
@@ -163,113 +145,44 @@ __device__ __forceinline__ void push32(const Ctx32 &cx, const uint8_t *heavy, ui
         for (int c = 0; c < CPL; c++) {
             const uint32_t slot = cx.ring + bytes + c * 128;
             uint32_t v = a[c];
-            if (ALL_MAX || !(tgt & kT32First)) v = max(v, lds_u32(slot));
+            if (!(tgt & kT32First)) v = max(v, lds_u32(slot));
             sts_u32(slot, v);
         }
     } else {
 #pragma unroll
         for (int c = 0; c < CPL; c++) {
             uint32_t *slot = reinterpret_cast<uint32_t *>(cx.cold + bytes + c * 128);
-            if (!ALL_MAX && (tgt & kT32First)) *slot = a[c];     // first far push: plain store
+            if (tgt & kT32First) *slot = a[c];                   // first far push: plain store
             else atomicMax(slot, a[c]);                          // RED.MAX, no reply awaited
         }
     }
 }
 
-// out-edges of one producer in record order.  Only a producer feeding two adjacent positions
-// (kOpAdj) can see its order change under a swap (ks, ks+1): then the run of edges to ks+1 is
-// pushed before the run to ks (the swapped order's consumer order).
-template <int CPL, bool MULTI, bool GLOBAL, bool ALL_MAX, class PlaceT, class StateT>
-__device__ __forceinline__ void push_all32(const Ctx32 &cx, const uint8_t *heavy, uint32_t ep,
-                                           uint32_t nout, bool adj, int32_t ks,
-                                           const int (&x)[CPL], const uint32_t (&cc)[CPL],
-                                           const PlaceT &place, StateT &st, uint32_t (&fwd)[CPL]) {
-    const int es = stride32<MULTI>(cx);
-    auto push_i = [&](uint32_t i) {
-        const uint32_t off = ep + i * es;
-        push32<CPL, MULTI, GLOBAL, ALL_MAX>(cx, heavy, off, rec_at<GLOBAL>(cx, heavy, off), x, cc,
-                                            place, st, fwd);
-    };
-    if (!adj || ks < 0) {
-        for (uint32_t i = 0; i < nout; i++) push_i(i);
-        return;
-    }
-    auto spos = [&](uint32_t i) {
-        return (int32_t)(rec_at<GLOBAL>(cx, heavy, ep + i * es).y & kSuccPosMask);
-    };
-    for (uint32_t i = 0; i < nout;) {
-        if (spos(i) != ks) {
-            push_i(i);
-            i++;
-            continue;
-        }
-        uint32_t a_end = i;
-        while (a_end < nout && spos(a_end) == ks) a_end++;
-        uint32_t b_end = a_end;
-        while (b_end < nout && spos(b_end) == ks + 1) b_end++;
-        for (uint32_t e = a_end; e < b_end; e++) push_i(e);
-        for (uint32_t e = i; e < a_end; e++) push_i(e);
-        i = b_end;
-    }
+// the (up to two) out-edges of one step at shared offset sp
+template <int CPL, class PlaceT, class StateT>
+__device__ __forceinline__ void edges32(const Ctx32 &cx, uint32_t sp, uint32_t flags,
+                                        const int (&x)[CPL], const uint32_t (&cc)[CPL],
+                                        const PlaceT &place, StateT &st, uint32_t (&fwd)[CPL]) {
+    const uint32_t ne = (flags >> kStEdgeShift) & 3u;
+    const uint4 e0 = lds_v4(cx.smem + sp + 16);
+    const uint4 e1 = lds_v4(cx.smem + sp + 32);
+    if (ne >= 1) push32<CPL>(cx, e0, x, cc, place, st, fwd);
+    if (ne >= 2) push32<CPL>(cx, e1, x, cc, place, st, fwd);
 }
 
-// Relax the op at position v (record o at shared offset rp) whose arrivals are r[c].
-// Returns, in fwd[c], the forwarded arrivals for position v + 1.
-template <int CPL, bool MULTI, bool ALL_MAX, class PlaceT, class StateT>
-__device__ __forceinline__ void relax32(const Ctx32 &cx, uint32_t rp, const uint4 o, int32_t v,
-                                        int32_t ks, const uint8_t *heavy, const PlaceT &place,
-                                        StateT &st, const uint32_t (&r)[CPL], uint32_t (&fwd)[CPL]) {
-    int x[CPL];
-    place.at(v, (int)((o.w >> kOpXShift) & 7u), x);
-    uint32_t cc[CPL];
+// start the op at position v (head h) whose arrivals are r[c]: S_v, C_v (L142-146)
+template <int CPL, class PlaceT, class StateT>
+__device__ __forceinline__ void begin32(const uint4 h, int32_t v, const PlaceT &place, StateT &st,
+                                        const uint32_t (&r)[CPL], int (&x)[CPL], uint32_t (&cc)[CPL]) {
+    place.at(v, (int)(h.w & kStXMask), x);
 #pragma unroll
     for (int c = 0; c < CPL; c++) {
-        cc[c] = add_sat(max(r[c], st.dev(c, x[c])), o.x);    // C_v = S_v + p_v
+        cc[c] = add_sat(max(r[c], st.dev(c, x[c])), h.x);    // C_v = S_v + p_v
         st.set_dev(c, x[c], cc[c]);
-        fwd[c] = 0u;
-    }
-    const bool adj = (o.w & kOpAdj) != 0;
-    if (!(o.w & kOpHeavy)) {
-        push_all32<CPL, MULTI, false, ALL_MAX>(cx, heavy, rp + 16, o.w & kOpNoutMask, adj, ks, x, cc,
-                                               place, st, fwd);
-        return;
-    }
-    const uint4 ext = lds_v4(cx.smem + rp + 16);             // ExtRec
-    push_all32<CPL, MULTI, true, ALL_MAX>(cx, heavy, ext.x, ext.z, adj, ks, x, cc, place, st, fwd);
-}
-
-template <bool MULTI>
-__device__ __forceinline__ uint32_t next_rp(const Ctx32 &cx, uint32_t rp, uint32_t nout) {
-    if (nout & kOpHeavy) return rp + 32;
-    return rp + 16 + (nout & kOpNoutMask) * stride32<MULTI>(cx);
-}
-
-// zero the slots an op opens with a first push (swap pairs only; times are >= 0)
-template <int CPL, bool MULTI>
-__device__ __forceinline__ void clear_first32(const Ctx32 &cx, uint32_t rp, const uint8_t *heavy) {
-    const uint4 o = lds_v4(cx.smem + rp);
-    const bool global = (o.w & kOpHeavy) != 0;
-    uint32_t ep = rp + 16, nout = o.w & kOpNoutMask;
-    if (global) {
-        const uint4 ext = lds_v4(cx.smem + rp + 16);
-        ep = ext.x;
-        nout = ext.z;
-    }
-    const int es = stride32<MULTI>(cx);
-    for (uint32_t i = 0; i < nout; i++) {
-        const uint4 rec = global ? rec_at<true>(cx, heavy, ep + i * es)
-                                 : rec_at<false>(cx, heavy, ep + i * es);
-        if (!(rec.z & kT32First) || (rec.z & kT32Next)) continue;
-        const uint32_t bytes = (rec.z & kT32SlotMask) * CPL;
-#pragma unroll
-        for (int c = 0; c < CPL; c++) {
-            if (rec.z & kT32Near) sts_u32(cx.ring + bytes + c * 128, 0u);
-            else *reinterpret_cast<uint32_t *>(cx.cold + bytes + c * 128) = 0u;
-        }
     }
 }
 
-template <int MODE, int PL, bool MULTI, int CPL>
+template <int MODE, int PL, int CPL>
 __global__ void __launch_bounds__((warps_for(CPL) + 1) * 32, 2)
 eval32_kernel(const EvalParams P) {
     constexpr int NW = warps_for(CPL);          // consumer warps per CTA (256 candidates)
@@ -279,8 +192,6 @@ eval32_kernel(const EvalParams P) {
     uint64_t *full = reinterpret_cast<uint64_t *>(smem + (size_t)kStages * sb);
     uint64_t *empty = full + kStages;
     uint8_t *cur = align16(reinterpret_cast<uint8_t *>(empty + kStages));
-    uint8_t *lclass = cur;
-    cur = align16(cur + 64);
     uint32_t *ring_all = reinterpret_cast<uint32_t *>(cur);
     cur = align16(cur + (size_t)NW * kRing * CW * 4);
     uint32_t *stage_all = reinterpret_cast<uint32_t *>(cur);          // far-arrival staging
@@ -295,7 +206,6 @@ eval32_kernel(const EvalParams P) {
         }
         mbar_fence_init();
     }
-    if (threadIdx.x < 64) lclass[threadIdx.x] = P.link_class[threadIdx.x];
     __syncthreads();
 
     auto runs_here = [&](int bl) {           // search: this kernel owns bases below saturation
@@ -327,10 +237,10 @@ eval32_kernel(const EvalParams P) {
     cx.smem = su32_reg(smem);
     cx.ring = su32_reg(ring_all + (size_t)warp * kRing * CW + lane);
     cx.cold = reinterpret_cast<uint8_t *>(P.state32 + ((size_t)(blockIdx.x * NW + warp) * P.max_W32) * CW + lane);
-    cx.lclass = su32_reg(lclass);
-    cx.edge_stride = P.edge_stride32;
     cx.D = P.D;
-    cx.two_classes = P.n_classes > 1;
+    cx.cls1 = 0;
+    for (int i = 0; i < P.D * P.D; i++)
+        if (P.link_class[i] == 1) cx.cls1 |= 1ull << i;
     const uint32_t stage = su32_reg(stage_all + (size_t)warp * kRing * CW + lane);
 
     using StateT = typename std::conditional<PL == 1, RegState32<CPL>, SmemState32<CPL>>::type;
@@ -342,35 +252,37 @@ eval32_kernel(const EvalParams P) {
     }
 
     // Far arrivals of position q arrive by cp.async into stage[q & 15], issued while position
-    // q - kPrefetchDist is relaxed (its record names the slot); one commit group per position,
-    // so waiting for all but kPrefetchDist groups makes position q's values visible.  The first
+    // q - kPrefetchDist starts (its head names the slot); one commit group per position, so
+    // waiting for all but kPrefetchDist groups makes position q's values visible.  The first
     // kPrefetchDist positions of a task load them directly.
-    auto issue_far = [&](const uint4 o, int32_t v) {
+    auto issue_far = [&](const uint4 h, int32_t v) {
         const uint32_t dst = stage + (uint32_t)(((v + kPrefetchDist) & (kRing - 1)) * CPL) * 128;
-        const bool have = (int32_t)o.z >= 0;
-        const uint8_t *src = cx.cold + (size_t)(have ? o.z : 0) * CW * 4;
+        const bool have = (int32_t)h.z >= 0;
+        const uint8_t *src = cx.cold + (size_t)(have ? h.z : 0) * CW * 4;
 #pragma unroll
         for (int c = 0; c < CPL; c++) cp_async4(dst + c * 128, src + c * 128, have);
         cp_async_commit();
     };
-    auto far_of = [&](const uint4 o, int32_t v, uint32_t (&f)[CPL]) {
+    // arrivals of the op at position v from far producers and the near ring
+    auto arrivals = [&](const uint4 h, int32_t v, uint32_t (&r)[CPL]) {
 #pragma unroll
-        for (int c = 0; c < CPL; c++) f[c] = 0u;
-        if ((int32_t)o.y < 0) return;
-        if (v < kPrefetchDist) {
+        for (int c = 0; c < CPL; c++) r[c] = 0u;
+        if ((int32_t)h.y >= 0) {
+            if (v < kPrefetchDist) {
 #pragma unroll
-            for (int c = 0; c < CPL; c++)
-                f[c] = *reinterpret_cast<const uint32_t *>(cx.cold + (size_t)o.y * CW * 4 + c * 128);
-            return;
+                for (int c = 0; c < CPL; c++)
+                    r[c] = *reinterpret_cast<const uint32_t *>(cx.cold + (size_t)h.y * CW * 4 + c * 128);
+            } else {
+                const uint32_t src = stage + (uint32_t)((v & (kRing - 1)) * CPL) * 128;
+#pragma unroll
+                for (int c = 0; c < CPL; c++) r[c] = lds_u32(src + c * 128);
+            }
         }
-        const uint32_t src = stage + (uint32_t)((v & (kRing - 1)) * CPL) * 128;
+        if (h.w & kStHasNear) {
+            const uint32_t src = cx.ring + (uint32_t)((v & (kRing - 1)) * CPL) * 128;
 #pragma unroll
-        for (int c = 0; c < CPL; c++) f[c] = lds_u32(src + c * 128);
-    };
-    auto ring_of = [&](const uint4 o, int32_t v, uint32_t (&f)[CPL]) {
-        const uint32_t src = cx.ring + (uint32_t)((v & (kRing - 1)) * CPL) * 128;
-#pragma unroll
-        for (int c = 0; c < CPL; c++) f[c] = (o.w & kOp32HasNear) ? lds_u32(src + c * 128) : 0u;
+            for (int c = 0; c < CPL; c++) r[c] = max(r[c], lds_u32(src + c * 128));
+        }
     };
 
     uint32_t it = 0;
@@ -380,7 +292,6 @@ eval32_kernel(const EvalParams P) {
         const int64_t local = MODE ? task % P.tasks_per_base : task;
         const BaseLayoutDev *B = &P.bases[bl];
         const int nt = B->n_tiles32;
-        const uint8_t *heavy = B->heavy32;
         // a task = 256 consecutive candidate ids starting at a multiple of 256; a warp = CW of them
         const int64_t j0 = (P.j_begin & ~(int64_t)255) + local * 256 + warp * CW;
         const int64_t gw = j0 >> 5;                                 // first 32-row group
@@ -412,9 +323,9 @@ eval32_kernel(const EvalParams P) {
             place.rc = rg.c;
             place.rlen = rg.len;
             place.allowed_pos = B->allowed_pos;
-            const uint8_t *adj = B->adj_next;
+            const uint8_t *blocked = B->swap_blocked;
             ks = active ? decode_swap(P.seed, cb, grp, P.n, P.mix[3], rg,
-                                      [&](int32_t k) { return __ldg(adj + k) != 0; })
+                                      [&](int32_t k) { return __ldg(blocked + k) != 0; })
                         : -1;
             const int32_t *ord = B->order;
             const uint32_t *bits = B->bits;
@@ -436,81 +347,81 @@ eval32_kernel(const EvalParams P) {
         }
         st.init();
 
-        bool skip_first = false;
-        uint32_t fwd[CPL];
+        // the op being walked (its devices and C_v) and the arrivals it forwards to v + 1
+        int x[CPL];
+        uint32_t cc[CPL], fwd[CPL];
 #pragma unroll
-        for (int c = 0; c < CPL; c++) fwd[c] = 0u;
+        for (int c = 0; c < CPL; c++) { x[c] = 0; cc[c] = 0u; fwd[c] = 0u; }
+        int32_t v = -1;
+        int32_t skip = 0;            // steps of the next tile already walked (swap pair)
         for (int t = 0; t < nt; t++, it++) {
             const int s = it % kStages;
             mbar_wait(&full[s], (it / kStages) & 1);
             if (active) {
                 const uint32_t tile = (uint32_t)s * sb;
-                const uint4 hdr = lds_v4(cx.smem + tile);
-                const int32_t pos_end = (int32_t)hdr.y;
-                int32_t v = (int32_t)hdr.x;
-                uint32_t rp = tile + kTileHeader;
-                if (skip_first) {
-                    rp = next_rp<MULTI>(cx, rp, lds_v4(cx.smem + rp).w);
-                    v++;
-                    skip_first = false;
-                }
-                uint4 o = lds_v4(cx.smem + rp);
-                while (v < pos_end) {
-                    if (v != ks) {
-                        const uint32_t rp_n = next_rp<MULTI>(cx, rp, o.w);
-                        const uint4 o_n = (v + 1 < pos_end) ? lds_v4(cx.smem + rp_n) : o;
-                        issue_far(o, v);
-                        cp_async_wait<kPrefetchDist>();
-                        uint32_t r[CPL], f[CPL], rg[CPL];
-                        far_of(o, v, f);
-                        ring_of(o, v, rg);
-#pragma unroll
-                        for (int c = 0; c < CPL; c++) r[c] = max(max(f[c], rg[c]), fwd[c]);
-                        relax32<CPL, MULTI, false>(cx, rp, o, v, ks, heavy, place, st, r, fwd);
-                        rp = rp_n;
+                const int32_t nsteps = (int32_t)lds_u32(cx.smem + tile);
+                uint32_t sp = tile + kTileHeader + (uint32_t)skip * kStepBytes;
+                int32_t i = skip;
+                skip = 0;
+                while (i < nsteps) {
+                    const uint4 h = lds_v4(cx.smem + sp);
+                    if (!(h.w & kStCont)) {
                         v++;
-                        o = o_n;
-                        continue;
-                    }
-                    // swapped pair: ops at ks+1 then ks
-                    const uint32_t rk = rp;
-                    const uint4 o_k = o;
-                    uint32_t rk1;
-                    const bool straddle = (v + 1 == pos_end);
-                    if (straddle) {
-                        const int s2 = (it + 1) % kStages;
-                        mbar_wait(&full[s2], ((it + 1) / kStages) & 1);
-                        rk1 = (uint32_t)s2 * sb + kTileHeader;
-                    } else {
-                        rk1 = next_rp<MULTI>(cx, rk, o_k.w);
-                    }
-                    const uint4 o_k1 = lds_v4(cx.smem + rk1);
-                    issue_far(o_k, v);
-                    issue_far(o_k1, v + 1);
-                    cp_async_wait<kPrefetchDist>();
-                    uint32_t f0[CPL], g0[CPL], f1[CPL], g1[CPL], r0[CPL], r1[CPL], fwd_k2[CPL], dummy[CPL];
-                    far_of(o_k, v, f0);
-                    ring_of(o_k, v, g0);
-                    far_of(o_k1, v + 1, f1);
-                    ring_of(o_k1, v + 1, g1);
+                        if (v == ks) {
+                            // swapped pair: the op at ks+1 runs first, then the op at ks.  They
+                            // share no producer, no consumer and no edge (DESIGN.md §4 S3), so
+                            // every slot's first push is unchanged; only device and link queues
+                            // see the new order.
+                            const int32_t nk = (int32_t)(h.w >> kStStepsShift);
+                            const bool straddle = i + nk >= nsteps;
+                            uint32_t sp1;
+                            if (straddle) {
+                                const int s2 = (it + 1) % kStages;
+                                mbar_wait(&full[s2], ((it + 1) / kStages) & 1);
+                                sp1 = (uint32_t)s2 * sb + kTileHeader;
+                            } else {
+                                sp1 = sp + (uint32_t)nk * kStepBytes;
+                            }
+                            const uint4 h1 = lds_v4(cx.smem + sp1);
+                            const int32_t n1 = (int32_t)(h1.w >> kStStepsShift);
+                            issue_far(h, v);
+                            issue_far(h1, v + 1);
+                            cp_async_wait<kPrefetchDist>();
+                            uint32_t r0[CPL], r1[CPL];
+                            arrivals(h, v, r0);
+                            arrivals(h1, v + 1, r1);   // ks+1's distance-1 producer is ks: none
 #pragma unroll
-                    for (int c = 0; c < CPL; c++) {
-                        r0[c] = max(max(f0[c], g0[c]), fwd[c]);
-                        r1[c] = max(f1[c], g1[c]);     // k+1's only distance-1 producer is k: none
-                    }
-                    clear_first32<CPL, MULTI>(cx, rk, heavy);
-                    relax32<CPL, MULTI, false>(cx, rk1, o_k1, v + 1, ks, heavy, place, st, r1, fwd_k2);
-                    relax32<CPL, MULTI, true>(cx, rk, o_k, v, ks, heavy, place, st, r0, dummy);
+                            for (int c = 0; c < CPL; c++) { r0[c] = max(r0[c], fwd[c]); fwd[c] = 0u; }
+                            begin32<CPL>(h1, v + 1, place, st, r1, x, cc);
+                            for (int32_t q = 0; q < n1; q++) {
+                                const uint32_t f = q ? lds_u32(cx.smem + sp1 + q * kStepBytes + 12) : h1.w;
+                                edges32<CPL>(cx, sp1 + q * kStepBytes, f, x, cc, place, st, fwd);
+                            }
+                            begin32<CPL>(h, v, place, st, r0, x, cc);
+                            for (int32_t q = 0; q < nk; q++) {
+                                const uint32_t f = q ? lds_u32(cx.smem + sp + q * kStepBytes + 12) : h.w;
+                                edges32<CPL>(cx, sp + q * kStepBytes, f, x, cc, place, st, fwd);
+                            }
+                            v++;
+                            if (straddle) {
+                                skip = n1;
+                                break;
+                            }
+                            sp = sp1 + (uint32_t)n1 * kStepBytes;
+                            i += nk + n1;
+                            continue;
+                        }
+                        issue_far(h, v);
+                        cp_async_wait<kPrefetchDist>();
+                        uint32_t r[CPL];
+                        arrivals(h, v, r);
 #pragma unroll
-                    for (int c = 0; c < CPL; c++) fwd[c] = fwd_k2[c];
-                    if (straddle) {
-                        skip_first = true;
-                        v = pos_end;
-                    } else {
-                        rp = next_rp<MULTI>(cx, rk1, o_k1.w);
-                        v += 2;
-                        if (v < pos_end) o = lds_v4(cx.smem + rp);
+                        for (int c = 0; c < CPL; c++) { r[c] = max(r[c], fwd[c]); fwd[c] = 0u; }
+                        begin32<CPL>(h, v, place, st, r, x, cc);
                     }
+                    edges32<CPL>(cx, sp, h.w, x, cc, place, st, fwd);
+                    sp += kStepBytes;
+                    i++;
                 }
             }
             __syncwarp();
@@ -551,20 +462,20 @@ eval32_kernel(const EvalParams P) {
     }
 }
 
-template <int MODE, int PL, bool MULTI, int CPL>
+template <int MODE, int PL, int CPL>
 cudaError_t launch_one32(const EvalParams &p, int grid, cudaStream_t st) {
     const int smem = eval32_smem_bytes(p, MODE);
-    auto kern = eval32_kernel<MODE, PL, MULTI, CPL>;
+    auto kern = eval32_kernel<MODE, PL, CPL>;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     if (e != cudaSuccess) return e;
     kern<<<grid, (warps_for(CPL) + 1) * 32, smem, st>>>(p);
     return cudaGetLastError();
 }
 
-template <int MODE, int PL, bool MULTI, int CPL>
+template <int MODE, int PL, int CPL>
 int occupancy_one32(const EvalParams &p) {
     const int smem = eval32_smem_bytes(p, MODE);
-    auto kern = eval32_kernel<MODE, PL, MULTI, CPL>;
+    auto kern = eval32_kernel<MODE, PL, CPL>;
     if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) != cudaSuccess)
         return 0;
     int n = 0;
@@ -587,8 +498,6 @@ int eval32_smem_bytes(const EvalParams &p, int search_mode) {
     const int pl = planes_of32(p.D);
     size_t b = (size_t)kStages * p.stage_bytes32 + 2 * kStages * 8;
     b = (b + 15) & ~size_t(15);
-    b += 64;
-    b = (b + 15) & ~size_t(15);
     b += (size_t)nw * kRing * 32 * cpl * 4;        // near ring
     b = (b + 15) & ~size_t(15);
     b += (size_t)nw * kRing * 32 * cpl * 4;        // far-arrival staging
@@ -597,20 +506,19 @@ int eval32_smem_bytes(const EvalParams &p, int search_mode) {
     return (int)b + 128;
 }
 
-// the edge stride is a compile-time 16 bytes unless some link class beyond the second exists
+// eval32 runs graphs with at most two link classes (layout.cpp emits no stream otherwise)
 #define PESTO_DISPATCH32(FN, ...)                                                          \
     do {                                                                                   \
         constexpr int C = kEval32Cpl;                                                      \
         const int pl = planes_of32(p.D);                                                   \
-        const bool multi = p.n_classes > 2;                                                \
         if (search_mode) {                                                                 \
-            if (pl == 1) return multi ? FN<1, 1, true, C>(__VA_ARGS__) : FN<1, 1, false, C>(__VA_ARGS__); \
-            if (pl == 2) return multi ? FN<1, 2, true, C>(__VA_ARGS__) : FN<1, 2, false, C>(__VA_ARGS__); \
-            return multi ? FN<1, 4, true, C>(__VA_ARGS__) : FN<1, 4, false, C>(__VA_ARGS__); \
+            if (pl == 1) return FN<1, 1, C>(__VA_ARGS__);                                  \
+            if (pl == 2) return FN<1, 2, C>(__VA_ARGS__);                                  \
+            return FN<1, 4, C>(__VA_ARGS__);                                               \
         } else {                                                                           \
-            if (pl == 1) return multi ? FN<0, 1, true, C>(__VA_ARGS__) : FN<0, 1, false, C>(__VA_ARGS__); \
-            if (pl == 2) return multi ? FN<0, 2, true, C>(__VA_ARGS__) : FN<0, 2, false, C>(__VA_ARGS__); \
-            return multi ? FN<0, 4, true, C>(__VA_ARGS__) : FN<0, 4, false, C>(__VA_ARGS__); \
+            if (pl == 1) return FN<0, 1, C>(__VA_ARGS__);                                  \
+            if (pl == 2) return FN<0, 2, C>(__VA_ARGS__);                                  \
+            return FN<0, 4, C>(__VA_ARGS__);                                               \
         }                                                                                  \
     } while (0)
 

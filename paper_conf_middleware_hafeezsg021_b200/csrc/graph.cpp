@@ -113,7 +113,7 @@ pesto_status upload_layout(pesto_graph *g, Layout &L) {
     if ((e = upload_vec(L.d_heavy, L.heavy)) != cudaSuccess) return cuda_fail(e, "upload layout");
     if ((e = upload_vec(L.d_tiles, L.tiles)) != cudaSuccess) return cuda_fail(e, "upload layout");
     if ((e = upload_vec(L.d_pos, L.pos)) != cudaSuccess) return cuda_fail(e, "upload layout");
-    if ((e = upload_vec(L.d_adj, L.adj_next)) != cudaSuccess) return cuda_fail(e, "upload layout");
+    if ((e = upload_vec(L.d_adj, L.swap_blocked)) != cudaSuccess) return cuda_fail(e, "upload layout");
     if ((e = upload_vec(L.d_allowed_pos, L.allowed_pos)) != cudaSuccess)
         return cuda_fail(e, "upload layout");
     if ((e = upload_vec(L.d_blob32, L.blob32)) != cudaSuccess) return cuda_fail(e, "upload layout");
@@ -136,7 +136,7 @@ BaseLayoutDev layout_view(const Layout &L) {
     v.heavy = L.d_heavy.as<uint8_t>();
     v.pos_of = L.d_pos.as<int32_t>();
     v.allowed_pos = L.d_allowed_pos.as<uint8_t>();
-    v.adj_next = L.d_adj.as<uint8_t>();
+    v.swap_blocked = L.d_adj.as<uint8_t>();
     v.bits = nullptr;
     v.n_tiles = (int32_t)L.tiles.size();
     v.W = L.W;

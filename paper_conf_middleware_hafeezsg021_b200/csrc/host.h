@@ -49,7 +49,7 @@ struct Layout {
     int32_t stage_bytes = 0;            // largest tile (incl. header)
     std::vector<uint8_t> blob, heavy;   // record stream (tiles) and out-of-line edges
     std::vector<TileDesc> tiles;
-    std::vector<uint8_t> adj_next, allowed_pos;
+    std::vector<uint8_t> swap_blocked, allowed_pos;   // swap_blocked[k]: (k, k+1) not swappable
     // 32-bit saturating stream (eval32)
     int32_t W32 = 0, stage_bytes32 = 0;
     std::vector<uint8_t> blob32, heavy32;

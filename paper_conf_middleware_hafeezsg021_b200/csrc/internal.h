@@ -23,7 +23,7 @@ struct BaseLayoutDev {
     const uint8_t *heavy;       // out-of-line edge records of high fan-out ops
     const int32_t *pos_of;      // [n] op id -> position
     const uint8_t *allowed_pos; // [n] device mask by position
-    const uint8_t *adj_next;    // [n] 1 if an edge joins order[k] -> order[k+1]
+    const uint8_t *swap_blocked; // [n] 1 if positions (k, k+1) may not be swapped (DESIGN §4 S3)
     const uint32_t *bits;       // search: base placement, [planes][words] bit planes, by position
     int32_t n_tiles;
     int32_t W;                  // live ready-time slots

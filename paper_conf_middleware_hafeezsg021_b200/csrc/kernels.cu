@@ -319,7 +319,7 @@ eval_kernel(const EvalParams P) {
             place.rlen = rg.len;
             place.bits = B->bits;
             place.allowed_pos = B->allowed_pos;
-            const uint8_t *adj = B->adj_next;
+            const uint8_t *adj = B->swap_blocked;
             ks = active ? decode_swap(P.seed, cb, grp, P.n, P.mix[3], rg,
                                       [&](int32_t k) { return __ldg(adj + k) != 0; })
                         : -1;
@@ -520,7 +520,7 @@ __global__ void commit_kernel(const CommitParams P) {
     const BaseLayoutDev &B = P.bases[b];
     uint32_t *bits = P.bits + (size_t)b * PL * P.words;
     const uint64_t cb = ctr_base_of(P.step, P.P, b);
-    const uint8_t *adj = B.adj_next;
+    const uint8_t *adj = B.swap_blocked;
     const Region rg = decode_region(P.seed, cb, j >> kGroupShift, P.n);
     const int32_t ks = decode_swap(P.seed, cb, j >> kGroupShift, P.n, P.mix[3], rg,
                                    [&](int32_t k) { return adj[k] != 0; });
@@ -537,8 +537,8 @@ __global__ void commit_kernel(const CommitParams P) {
     auto set_dev = [&](int32_t q, int x) {
         set_dev_at<PL>(bits, words, q, x);
         if (!P.patch32) return;
-        uint32_t *nout = reinterpret_cast<uint32_t *>(blob32 + B.op_off32[q]) + 3;
-        *nout = (*nout & ~(7u << kOpXShift)) | ((uint32_t)x << kOpXShift);
+        uint32_t *flags = reinterpret_cast<uint32_t *>(blob32 + B.op_off32[q]) + 3;   // StepHead
+        *flags = (*flags & ~kStXMask) | (uint32_t)x;
         for (uint32_t i = B.pin_off[q]; i < B.pin_off[q + 1]; i++) {
             const uint32_t ref = B.pin_ref[i];
             uint8_t *base = (ref & kPinHeavy) ? heavy32 : blob32;

@@ -12,6 +12,7 @@
 #include <string>
 
 #include "host.h"
+#include "moves.cuh"
 
 namespace pesto {
 
@@ -219,6 +220,7 @@ pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<
         L->W32 = std::max(colour_intervals(n, first_far, pos, cslot), 1);
         if (L->W32 >= (1 << 22)) L->W32 = 0;  // slot byte offsets must fit 29 bits: 64-bit path
     }
+    if (L->W32 > 0 && C > 2) L->W32 = 0;     // the step format carries two link classes
     if (L->W32 > 0) {
         std::vector<uint8_t> seen_near(n, 0), seen_far(n, 0), first32(m, 0);
         for (int32_t k = 0; k < n; k++) {
@@ -231,14 +233,13 @@ pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<
                 if (!seen) { seen = 1; first32[e] = 1; }
             }
         }
-        const int es32 = edge_stride32_for(C);
         auto t32 = [&](int64_t e, int c) { return (uint32_t)g->t_class[(size_t)e * C + c]; };
         auto xcode = [&](int32_t op) { return x_op ? (uint32_t)(x_op[op] & 7u) : 0u; };
         L->blob32.clear();
         L->heavy32.clear();
         L->tiles32.clear();
         L->stage_bytes32 = 0;
-        L->blob32.reserve((size_t)n * 16 + (size_t)m * es32 + 64 * kTileHeader);
+        L->blob32.reserve((size_t)(n + m / 2 + 64) * kStepBytes + 64 * kTileHeader);
         L->op_off32.assign(n, 0);
         // patch index: locations of every edge record by successor position
         L->pin_off.assign((size_t)n + 1, 0);
@@ -246,9 +247,7 @@ pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<
         for (int64_t e = 0; e < m; e++) L->pin_off[pos[g->dst[e]] + 1]++;
         for (int32_t q = 0; q < n; q++) L->pin_off[q + 1] += L->pin_off[q];
         std::vector<uint32_t> pfill(L->pin_off.begin(), L->pin_off.end() - 1);
-        auto put_edge32 = [&](std::vector<uint8_t> &buf, int64_t e, bool heavy) {
-            const size_t at = buf.size();
-            buf.resize(at + es32, 0);
+        auto edge_rec = [&](int64_t e, size_t at) {
             EdgeRec32 r;
             r.t0 = t32(e, 0);
             r.t1 = C > 1 ? t32(e, 1) : 0u;
@@ -259,49 +258,88 @@ pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<
                      : (near_edge(e) ? (kT32Near | (uint32_t)(pos[w] & (kRing - 1)) * 128u)
                                      : (uint32_t)cslot[w] * 128u) |
                        (first32[e] ? kT32First : 0u);
-            std::memcpy(buf.data() + at, &r, sizeof r);
-            for (int c = 2; c < C; c++) {
-                const uint32_t t = t32(e, c);
-                std::memcpy(buf.data() + at + 16 + 4 * (c - 2), &t, 4);
-            }
-            L->pin_ref[pfill[pos[w]]++] = (uint32_t)at | (heavy ? kPinHeavy : 0u);
+            L->pin_ref[pfill[pos[w]]++] = (uint32_t)at;
+            return r;
         };
-        TileWriter tw(L->blob32, L->tiles32, L->stage_bytes32);
-        tw.open(0);
+        // tiles hold whole ops, except an op larger than a tile, which continues in the next
+        std::vector<uint8_t> &blob = L->blob32;
+        size_t t_start = 0;
+        int32_t t_steps = 0;
+        auto open = [&]() { t_start = blob.size(); t_steps = 0; blob.resize(t_start + kTileHeader, 0); };
+        auto close = [&]() {
+            TileDesc td{};
+            td.byte_off = (int64_t)t_start;
+            td.bytes = (int32_t)(blob.size() - t_start);
+            td.pos_begin = t_steps;                  // (steps in the tile)
+            const int32_t hdr[4] = {t_steps, 0, td.bytes, 0};
+            std::memcpy(blob.data() + t_start, hdr, 16);
+            L->tiles32.push_back(td);
+            L->stage_bytes32 = std::max(L->stage_bytes32, td.bytes);
+        };
+        const size_t budget = (size_t)kTileTarget;
+        open();
         for (int32_t k = 0; k < n; k++) {
             const int32_t u = order[k];
             const int64_t b0 = g->out_off[u], b1 = g->out_off[u + 1];
             const int64_t nout = b1 - b0;
-            const bool heavy = nout * es32 > kMaxInlineBytes;
-            tw.maybe_cut(k, 16 + (heavy ? 16 : (size_t)nout * es32));
-            bool adj = false;                   // feeds two adjacent positions (swap reorder)
-            for (int64_t i = b0 + 1; i < b1; i++)
-                if (succ_pos(sorted[i]) == succ_pos(sorted[i - 1]) + 1) adj = true;
-            OpRec32 op;
-            op.p = (uint32_t)g->p[u];
-            op.cold_slot = cslot[u];
-            const int32_t ahead = k + kPrefetchDist;
-            op.pf_slot = ahead < n ? cslot[order[ahead]] : -1;
-            op.nout = (heavy ? kOpHeavy : (uint32_t)nout) | (has_near[u] ? kOp32HasNear : 0u) |
-                      (adj ? kOpAdj : 0u) | (xcode(u) << kOpXShift);
-            L->op_off32[k] = (uint32_t)L->blob32.size();
-            append(L->blob32, op);
-            if (heavy) {
-                append(L->blob32, ExtRec{(int64_t)L->heavy32.size(), nout});
-                for (int64_t i = b0; i < b1; i++) put_edge32(L->heavy32, sorted[i], true);
-            } else {
-                for (int64_t i = b0; i < b1; i++) put_edge32(L->blob32, sorted[i], false);
+            const int64_t nsteps = std::max<int64_t>(1, (nout + 1) / 2);
+            const size_t op_bytes = (size_t)nsteps * kStepBytes;
+            if (t_steps > 0 && blob.size() - t_start + op_bytes > budget) { close(); open(); }
+            L->op_off32[k] = (uint32_t)blob.size();
+            for (int64_t s = 0; s < nsteps; s++) {
+                if (t_steps > 0 && blob.size() - t_start + kStepBytes > budget) { close(); open(); }
+                const size_t at = blob.size();
+                blob.resize(at + kStepBytes, 0);
+                StepHead h;
+                const int64_t ne = std::min<int64_t>(2, nout - 2 * s);
+                if (s == 0) {
+                    h.p = (uint32_t)g->p[u];
+                    h.cold_slot = cslot[u];
+                    const int32_t ahead = k + kPrefetchDist;
+                    h.pf_slot = ahead < n ? cslot[order[ahead]] : -1;
+                    h.flags = xcode(u) | (has_near[u] ? kStHasNear : 0u) |
+                              ((uint32_t)std::max<int64_t>(ne, 0) << kStEdgeShift) |
+                              ((uint32_t)nsteps << kStStepsShift);
+                } else {
+                    h.p = 0;
+                    h.cold_slot = -1;
+                    h.pf_slot = -1;
+                    h.flags = kStCont | ((uint32_t)ne << kStEdgeShift);
+                }
+                std::memcpy(blob.data() + at, &h, 16);
+                for (int64_t q = 0; q < ne; q++) {
+                    const size_t eo = at + 16 + 16 * q;
+                    const EdgeRec32 r = edge_rec(sorted[b0 + 2 * s + q], eo);
+                    std::memcpy(blob.data() + eo, &r, 16);
+                }
+                t_steps++;
             }
         }
-        tw.close(n);
+        close();
+        if ((int64_t)blob.size() >= ((int64_t)1 << 31)) return fail(PESTO_ENOMEM, "layout too large");
     }
 
-    // order-move helpers
-    L->adj_next.assign(n, 0);
-    for (int32_t k = 0; k + 1 < n; k++) {
-        const int32_t u = order[k], w = order[k + 1];
-        for (int64_t i = g->out_off[u]; i < g->out_off[u + 1]; i++)
-            if (g->dst[g->out_edges[i]] == w) { L->adj_next[k] = 1; break; }
+    // order moves: positions (k, k+1) may be swapped unless an edge joins them, they share a
+    // producer or a consumer, or either has more than kSwapMaxOut successors (DESIGN §4 S3)
+    L->swap_blocked.assign(n, 1);
+    {
+        std::vector<int32_t> mark_pred(n, -1), mark_succ(n, -1);
+        for (int32_t k = 0; k + 1 < n; k++) {
+            const int32_t a = order[k], c = order[k + 1];
+            bool blocked = g->out_off[a + 1] - g->out_off[a] > kSwapMaxOut ||
+                           g->out_off[c + 1] - g->out_off[c] > kSwapMaxOut;
+            for (int64_t i = g->in_off[a]; i < g->in_off[a + 1]; i++) mark_pred[g->src[g->in_edges[i]]] = k;
+            for (int64_t i = g->out_off[a]; i < g->out_off[a + 1]; i++) {
+                const int32_t w = g->dst[g->out_edges[i]];
+                if (w == c) blocked = true;
+                mark_succ[w] = k;
+            }
+            for (int64_t i = g->in_off[c]; i < g->in_off[c + 1] && !blocked; i++)
+                if (mark_pred[g->src[g->in_edges[i]]] == k) blocked = true;
+            for (int64_t i = g->out_off[c]; i < g->out_off[c + 1] && !blocked; i++)
+                if (mark_succ[g->dst[g->out_edges[i]]] == k) blocked = true;
+            L->swap_blocked[k] = blocked ? 1 : 0;
+        }
     }
     L->allowed_pos.resize(n);
     for (int32_t k = 0; k < n; k++) L->allowed_pos[k] = g->allowed[order[k]];

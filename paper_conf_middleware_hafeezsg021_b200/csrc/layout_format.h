@@ -94,4 +94,21 @@ inline int edge_stride32_for(int classes) {
     return classes <= 2 ? 16 : 16 * (1 + (classes - 2 + 3) / 4);
 }
 
+// eval32 step stream: the π-ordered ops as fixed 48-byte steps -- a head and
+// two EdgeRec32 slots -- so the walk is a straight-line loop with no per-op edge loop.  An op
+// with more than two out-edges continues in CONT steps (head p/cold/pf unused).  Graphs with
+// more than two distinct link classes use eval64.
+struct alignas(16) StepHead {
+    uint32_t p;          // p_v (< kMaxDur32)
+    int32_t cold_slot;   // this op's cold slot (far arrivals); -1 = none
+    int32_t pf_slot;     // cold slot of the op kPrefetchDist positions ahead; -1 = none
+    uint32_t flags;      // base code | kStHasNear | kStCont | edges << 5 | op steps << 8
+};
+constexpr int kStepBytes = 48;
+constexpr uint32_t kStXMask = 7u;               // bits 0-2: base device code of the op
+constexpr uint32_t kStHasNear = 1u << 3;        // read the near ring
+constexpr uint32_t kStCont = 1u << 4;           // continuation step of the previous op
+constexpr int kStEdgeShift = 5;                 // bits 5-6: edges in this step (0..2)
+constexpr int kStStepsShift = 8;                // bits 8-31 (first step): steps of this op
+
 }  // namespace pesto

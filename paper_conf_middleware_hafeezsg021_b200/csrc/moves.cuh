@@ -64,16 +64,18 @@ PESTO_HD Region decode_region(uint64_t seed, uint64_t cb, int64_t group, int n) 
 }
 
 // Group order move: adjacent swap of positions (k, k+1) of the base order, or -1.
-// adj_next(k) must say whether an edge joins order[k] -> order[k+1].
-template <class AdjNext>
+// blocked(k) says whether (k, k+1) may not be swapped: an edge joins them, they share a
+// producer or a consumer, or either has more than kSwapMaxOut successors (DESIGN §4 S3).
+constexpr int kSwapMaxOut = 64;
+template <class Blocked>
 PESTO_HD int32_t decode_swap(uint64_t seed, uint64_t cb, int64_t group, int n, int swap_pct,
-                             Region rg, AdjNext adj_next) {
+                             Region rg, Blocked blocked) {
     if (group == 0 || swap_pct <= 0 || n < 2) return -1;
     int64_t j0 = group * kGroup;
     if ((int)(draw(seed, cb, j0, 15) % 100u) >= swap_pct) return -1;
     int32_t k = rg.c + (int32_t)(draw(seed, cb, j0, 14) % (uint64_t)rg.len);
     if (k > n - 2) k = n - 2;
-    return adj_next(k) ? -1 : k;
+    return blocked(k) ? -1 : k;
 }
 
 // Lane placement move of candidate j inside region rg.  Callbacks:

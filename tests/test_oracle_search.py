@@ -45,7 +45,13 @@ def test_identity_and_move_shapes(O):
                 k = int(diff_pos[0])
                 assert list(diff_pos) == [k, k + 1]
                 assert o[k] == orders[b][k + 1] and o[k + 1] == orders[b][k]
-                assert (int(orders[b][k]), int(orders[b][k + 1])) not in edges
+                a, c = int(orders[b][k]), int(orders[b][k + 1])
+                assert (a, c) not in edges
+                # S3: swapped ops share no producer and no consumer, fan-out <= 64
+                preds = lambda v: {s for s, d in edges if d == v}
+                succs = lambda v: {d for s, d in edges if s == v}
+                assert not (preds(a) & preds(c)) and not (succs(a) & succs(c))
+                assert len(succs(a)) <= 64 and len(succs(c)) <= 64
                 assert O.makespan(g, x, o) >= 0           # still topological
                 if j % 128 == 0:
                     assert (x == xs[b]).all()              # lane 0 of a swap group: pure swap
