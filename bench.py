@@ -258,6 +258,7 @@ def run_pesto(args, rank, world, local):
     total_cands = k_gpu * world * args.steps
     value = total_cands / (tot_ms / 1e3)
     best_mk = [S.get(b)[0] for b in range(n_bases)]
+    swap_stats = S.swap_stats()
 
     # ---- end to end through the public API with host buffers (eval_batch_host) ----
     e2e = None
@@ -331,7 +332,8 @@ def run_pesto(args, rank, world, local):
                                  "traffic = ncu DRAM bytes per K1 launch (profiles/)"},
             "gpu_launches": int(launches),
             "wall_s_timed_region": wall,
-            "search": {"seed_makespans": seed_mk, "best_makespans": best_mk},
+            "search": {"seed_makespans": seed_mk, "best_makespans": best_mk,
+                       "swaps_patched_in_place": swap_stats[0], "swaps_rebuilt": swap_stats[1]},
             "e2e": e2e}
     line["clocks"] = clk.summary()
     if not args.no_cpu_baseline:

@@ -184,6 +184,11 @@ pesto_status pesto_search_get(pesto_search *s, int32_t base, int64_t *makespan,
                               uint8_t *x_host, int32_t *order_host);
 int64_t pesto_search_step_count(const pesto_search *s);
 
+/* Committed adjacent swaps so far: patched in place on the device (in_place)
+ * or handled by a host rebuild of that base's layout (rebuilt).  Either pointer may be NULL.
+ * Errors: EINVAL if s is NULL. */
+pesto_status pesto_search_swap_stats(const pesto_search *s, int64_t *in_place, int64_t *rebuilt);
+
 /* ncclGetUniqueId through the process's libnccl.so.2 (rank 0 calls it and broadcasts the 128
  * bytes over its own process group).  Errors: ENCCL if NCCL cannot be loaded. */
 pesto_status pesto_nccl_unique_id(uint8_t *out128);

@@ -88,6 +88,11 @@ __device__ __forceinline__ void cp_async4(uint32_t smem_addr, const void *gptr, 
         " @p cp.async.ca.shared.global [%0], [%1], 4;\n}\n"
         ::"r"(smem_addr), "l"(gptr), "r"((int)pred) : "memory");
 }
+// 4-byte async copy that writes zero when `have` is false (src-size 0: nothing is read)
+__device__ __forceinline__ void cp_async4_zfill(uint32_t smem_addr, const void *gptr, bool have) {
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4, %2;\n"
+                 ::"r"(smem_addr), "l"(gptr), "r"(have ? 4 : 0) : "memory");
+}
 __device__ __forceinline__ void cp_async_commit() {
     asm volatile("cp.async.commit_group;" ::: "memory");
 }

@@ -116,7 +116,7 @@ struct Ctx32 {
 };
 
 // one out-edge record, for the lane's CPL candidates (FCFS link of L144 / L188-198)
-template <int CPL, class PlaceT, class StateT>
+template <int PL, int CPL, class PlaceT, class StateT>
 __device__ __forceinline__ void push32(const Ctx32 &cx, const uint4 rec, const int (&x)[CPL],
                                        const uint32_t (&cc)[CPL], const PlaceT &place,
                                        StateT &st, uint32_t (&fwd)[CPL]) {
@@ -128,7 +128,9 @@ __device__ __forceinline__ void push32(const Ctx32 &cx, const uint4 rec, const i
 #pragma unroll
     for (int c = 0; c < CPL; c++) {
         const bool cross = y[c] != x[c];                     // cross: FCFS link x -> y
-        const uint32_t t = ((cx.cls1 >> (x[c] * cx.D + y[c])) & 1u) ? rec.w : rec.x;
+        uint32_t t;
+        if constexpr (PL == 1) t = x[c] ? rec.w : rec.x;     // D = 2: t by direction
+        else t = ((cx.cls1 >> (x[c] * cx.D + y[c])) & 1u) ? rec.w : rec.x;
         // branch-free: the transfer's arrival when crossing, C_v (L144) when not
         const uint32_t ac = add_sat(max(cc[c], st.link(c, x[c], y[c])), t);
         a[c] = cross ? ac : cc[c];
@@ -158,16 +160,15 @@ __device__ __forceinline__ void push32(const Ctx32 &cx, const uint4 rec, const i
     }
 }
 
-// the (up to two) out-edges of one step at shared offset sp
-template <int CPL, class PlaceT, class StateT>
-__device__ __forceinline__ void edges32(const Ctx32 &cx, uint32_t sp, uint32_t flags,
-                                        const int (&x)[CPL], const uint32_t (&cc)[CPL],
-                                        const PlaceT &place, StateT &st, uint32_t (&fwd)[CPL]) {
+// the (up to two) out-edges of one step, records already in registers
+template <int PL, int CPL, class PlaceT, class StateT>
+__device__ __forceinline__ void edges32(const Ctx32 &cx, uint32_t flags, const uint4 e0,
+                                        const uint4 e1, const int (&x)[CPL],
+                                        const uint32_t (&cc)[CPL], const PlaceT &place,
+                                        StateT &st, uint32_t (&fwd)[CPL]) {
     const uint32_t ne = (flags >> kStEdgeShift) & 3u;
-    const uint4 e0 = lds_v4(cx.smem + sp + 16);
-    const uint4 e1 = lds_v4(cx.smem + sp + 32);
-    if (ne >= 1) push32<CPL>(cx, e0, x, cc, place, st, fwd);
-    if (ne >= 2) push32<CPL>(cx, e1, x, cc, place, st, fwd);
+    if (ne >= 1) push32<PL, CPL>(cx, e0, x, cc, place, st, fwd);
+    if (ne >= 2) push32<PL, CPL>(cx, e1, x, cc, place, st, fwd);
 }
 
 // start the op at position v (head h) whose arrivals are r[c]: S_v, C_v (L142-146)
@@ -188,7 +189,9 @@ eval32_kernel(const EvalParams P) {
     constexpr int NW = warps_for(CPL);          // consumer warps per CTA (256 candidates)
     constexpr int CW = 32 * CPL;                // candidates per warp
     extern __shared__ __align__(128) uint8_t smem[];
-    const int sb = P.stage_bytes32;
+    // stage stride: the largest tile + one step of padding, so the walk may read the records of
+    // the step after a tile's last one without leaving its own stage
+    const int sb = P.stage_bytes32 + kStepBytes;
     uint64_t *full = reinterpret_cast<uint64_t *>(smem + (size_t)kStages * sb);
     uint64_t *empty = full + kStages;
     uint8_t *cur = align16(reinterpret_cast<uint8_t *>(empty + kStages));
@@ -251,38 +254,34 @@ eval32_kernel(const EvalParams P) {
         st.l = st.d + (uint32_t)(P.D * CPL) * 128;
     }
 
-    // Far arrivals of position q arrive by cp.async into stage[q & 15], issued while position
-    // q - kPrefetchDist starts (its head names the slot); one commit group per position, so
-    // waiting for all but kPrefetchDist groups makes position q's values visible.  The first
-    // kPrefetchDist positions of a task load them directly.
+    // Far arrivals of position q arrive by cp.async into stage[q & 15] (zero when q has no far
+    // producer), issued while position q - kPrefetchDist starts (its head names the slot); one
+    // commit group per position.  Only positions > kNearDelta have far producers, so the first
+    // positions of a task need no prefetch.
     auto issue_far = [&](const uint4 h, int32_t v) {
         const uint32_t dst = stage + (uint32_t)(((v + kPrefetchDist) & (kRing - 1)) * CPL) * 128;
         const bool have = (int32_t)h.z >= 0;
         const uint8_t *src = cx.cold + (size_t)(have ? h.z : 0) * CW * 4;
 #pragma unroll
-        for (int c = 0; c < CPL; c++) cp_async4(dst + c * 128, src + c * 128, have);
+        for (int c = 0; c < CPL; c++) cp_async4_zfill(dst + c * 128, src + c * 128, have);
         cp_async_commit();
     };
-    // arrivals of the op at position v from far producers and the near ring
-    auto arrivals = [&](const uint4 h, int32_t v, uint32_t (&r)[CPL]) {
+    // The arrivals of position q from far producers (stage) and near producers (ring) are final
+    // once the op at q - 1 starts (a distance-1 producer forwards in `fwd`), so they are read one
+    // op ahead, off the critical path: nfar/nnear hold them for the next position.
+    auto load_next = [&](int32_t q, uint32_t (&nfar)[CPL], uint32_t (&nnear)[CPL]) {
+        const uint32_t o = (uint32_t)((q & (kRing - 1)) * CPL) * 128;
 #pragma unroll
-        for (int c = 0; c < CPL; c++) r[c] = 0u;
-        if ((int32_t)h.y >= 0) {
-            if (v < kPrefetchDist) {
-#pragma unroll
-                for (int c = 0; c < CPL; c++)
-                    r[c] = *reinterpret_cast<const uint32_t *>(cx.cold + (size_t)h.y * CW * 4 + c * 128);
-            } else {
-                const uint32_t src = stage + (uint32_t)((v & (kRing - 1)) * CPL) * 128;
-#pragma unroll
-                for (int c = 0; c < CPL; c++) r[c] = lds_u32(src + c * 128);
-            }
+        for (int c = 0; c < CPL; c++) {
+            nfar[c] = lds_u32(stage + o + c * 128);
+            nnear[c] = lds_u32(cx.ring + o + c * 128);
         }
-        if (h.w & kStHasNear) {
-            const uint32_t src = cx.ring + (uint32_t)((v & (kRing - 1)) * CPL) * 128;
+    };
+    auto arrivals = [&](uint32_t flags, const uint32_t (&nfar)[CPL], const uint32_t (&nnear)[CPL],
+                        const uint32_t (&fwd)[CPL], uint32_t (&r)[CPL]) {
+        const bool near = (flags & kStHasNear) != 0;          // else the ring slot is stale
 #pragma unroll
-            for (int c = 0; c < CPL; c++) r[c] = max(r[c], lds_u32(src + c * 128));
-        }
+        for (int c = 0; c < CPL; c++) r[c] = max(max(nfar[c], fwd[c]), near ? nnear[c] : 0u);
     };
 
     uint32_t it = 0;
@@ -346,12 +345,16 @@ eval32_kernel(const EvalParams P) {
             }
         }
         st.init();
-
-        // the op being walked (its devices and C_v) and the arrivals it forwards to v + 1
-        int x[CPL];
-        uint32_t cc[CPL], fwd[CPL];
+        // positions 0 .. kPrefetchDist - 1 are never prefetched (they have no far producer)
 #pragma unroll
-        for (int c = 0; c < CPL; c++) { x[c] = 0; cc[c] = 0u; fwd[c] = 0u; }
+        for (int q = 0; q < kRing * CPL; q++) sts_u32(stage + q * 128, 0u);
+
+        // the op being walked (its devices and C_v), the arrivals it forwards to v + 1, and the
+        // far / near arrivals of v + 1 read ahead
+        int x[CPL];
+        uint32_t cc[CPL], fwd[CPL], nfar[CPL], nnear[CPL];
+#pragma unroll
+        for (int c = 0; c < CPL; c++) { x[c] = 0; cc[c] = 0u; fwd[c] = 0u; nfar[c] = 0u; nnear[c] = 0u; }
         int32_t v = -1;
         int32_t skip = 0;            // steps of the next tile already walked (swap pair)
         for (int t = 0; t < nt; t++, it++) {
@@ -360,11 +363,13 @@ eval32_kernel(const EvalParams P) {
             if (active) {
                 const uint32_t tile = (uint32_t)s * sb;
                 const int32_t nsteps = (int32_t)lds_u32(cx.smem + tile);
-                uint32_t sp = tile + kTileHeader + (uint32_t)skip * kStepBytes;
+                uint32_t sp = cx.smem + tile + kTileHeader + (uint32_t)skip * kStepBytes;
                 int32_t i = skip;
                 skip = 0;
+                uint4 h = lds_v4(sp), e0 = lds_v4(sp + 16), e1 = lds_v4(sp + 32);
                 while (i < nsteps) {
-                    const uint4 h = lds_v4(cx.smem + sp);
+                    // the next step's records (past the tile's end: padding, never used)
+                    const uint4 hn = lds_v4(sp + 48), e0n = lds_v4(sp + 64), e1n = lds_v4(sp + 80);
                     if (!(h.w & kStCont)) {
                         v++;
                         if (v == ks) {
@@ -378,50 +383,64 @@ eval32_kernel(const EvalParams P) {
                             if (straddle) {
                                 const int s2 = (it + 1) % kStages;
                                 mbar_wait(&full[s2], ((it + 1) / kStages) & 1);
-                                sp1 = (uint32_t)s2 * sb + kTileHeader;
+                                sp1 = cx.smem + (uint32_t)s2 * sb + kTileHeader;
                             } else {
                                 sp1 = sp + (uint32_t)nk * kStepBytes;
                             }
-                            const uint4 h1 = lds_v4(cx.smem + sp1);
+                            const uint4 h1 = lds_v4(sp1);
                             const int32_t n1 = (int32_t)(h1.w >> kStStepsShift);
                             issue_far(h, v);
                             issue_far(h1, v + 1);
-                            cp_async_wait<kPrefetchDist>();
-                            uint32_t r0[CPL], r1[CPL];
-                            arrivals(h, v, r0);
-                            arrivals(h1, v + 1, r1);   // ks+1's distance-1 producer is ks: none
+                            cp_async_wait<kPrefetchDist - 1>();  // v+1 and v+2 have landed
+                            uint32_t r0[CPL], r1[CPL], f1[CPL], g1[CPL], zero[CPL];
 #pragma unroll
-                            for (int c = 0; c < CPL; c++) { r0[c] = max(r0[c], fwd[c]); fwd[c] = 0u; }
+                            for (int c = 0; c < CPL; c++) zero[c] = 0u;
+                            arrivals(h.w, nfar, nnear, fwd, r0);
+                            load_next(v + 1, f1, g1);
+                            arrivals(h1.w, f1, g1, zero, r1);   // ks+1's distance-1 producer is ks: none
+#pragma unroll
+                            for (int c = 0; c < CPL; c++) fwd[c] = 0u;
                             begin32<CPL>(h1, v + 1, place, st, r1, x, cc);
                             for (int32_t q = 0; q < n1; q++) {
-                                const uint32_t f = q ? lds_u32(cx.smem + sp1 + q * kStepBytes + 12) : h1.w;
-                                edges32<CPL>(cx, sp1 + q * kStepBytes, f, x, cc, place, st, fwd);
+                                const uint32_t a = sp1 + q * kStepBytes;
+                                edges32<PL, CPL>(cx, lds_u32(a + 12), lds_v4(a + 16), lds_v4(a + 32), x,
+                                                 cc, place, st, fwd);
                             }
                             begin32<CPL>(h, v, place, st, r0, x, cc);
-                            for (int32_t q = 0; q < nk; q++) {
-                                const uint32_t f = q ? lds_u32(cx.smem + sp + q * kStepBytes + 12) : h.w;
-                                edges32<CPL>(cx, sp + q * kStepBytes, f, x, cc, place, st, fwd);
+                            edges32<PL, CPL>(cx, h.w, e0, e1, x, cc, place, st, fwd);
+                            for (int32_t q = 1; q < nk; q++) {
+                                const uint32_t a = sp + q * kStepBytes;
+                                edges32<PL, CPL>(cx, lds_u32(a + 12), lds_v4(a + 16), lds_v4(a + 32), x,
+                                                 cc, place, st, fwd);
                             }
                             v++;
+                            load_next(v + 1, nfar, nnear);
                             if (straddle) {
                                 skip = n1;
                                 break;
                             }
                             sp = sp1 + (uint32_t)n1 * kStepBytes;
                             i += nk + n1;
+                            h = lds_v4(sp);
+                            e0 = lds_v4(sp + 16);
+                            e1 = lds_v4(sp + 32);
                             continue;
                         }
                         issue_far(h, v);
-                        cp_async_wait<kPrefetchDist>();
+                        cp_async_wait<kPrefetchDist - 1>();      // v+1 has landed
                         uint32_t r[CPL];
-                        arrivals(h, v, r);
+                        arrivals(h.w, nfar, nnear, fwd, r);
+                        load_next(v + 1, nfar, nnear);
 #pragma unroll
-                        for (int c = 0; c < CPL; c++) { r[c] = max(r[c], fwd[c]); fwd[c] = 0u; }
+                        for (int c = 0; c < CPL; c++) fwd[c] = 0u;
                         begin32<CPL>(h, v, place, st, r, x, cc);
                     }
-                    edges32<CPL>(cx, sp, h.w, x, cc, place, st, fwd);
+                    edges32<PL, CPL>(cx, h.w, e0, e1, x, cc, place, st, fwd);
                     sp += kStepBytes;
                     i++;
+                    h = hn;
+                    e0 = e0n;
+                    e1 = e1n;
                 }
             }
             __syncwarp();
@@ -496,7 +515,7 @@ int eval32_smem_bytes(const EvalParams &p, int search_mode) {
     const int cpl = kEval32Cpl;
     const int nw = warps_for(cpl);
     const int pl = planes_of32(p.D);
-    size_t b = (size_t)kStages * p.stage_bytes32 + 2 * kStages * 8;
+    size_t b = (size_t)kStages * (p.stage_bytes32 + kStepBytes) + 2 * kStages * 8;
     b = (b + 15) & ~size_t(15);
     b += (size_t)nw * kRing * 32 * cpl * 4;        // near ring
     b = (b + 15) & ~size_t(15);

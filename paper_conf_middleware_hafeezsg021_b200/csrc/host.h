@@ -13,6 +13,8 @@
 
 namespace pesto {
 
+constexpr int kMaxInlineBytes = 2048;   // eval64: an op's edges beyond this go out of line
+
 void set_error(const std::string &msg);
 pesto_status fail(pesto_status s, const std::string &msg);
 pesto_status cuda_fail(cudaError_t e, const char *what);
@@ -55,6 +57,12 @@ struct Layout {
     std::vector<uint8_t> blob32, heavy32;
     std::vector<TileDesc> tiles32;
     std::vector<uint32_t> op_off32, pin_off, pin_ref;   // K4 patch index into blob32/heavy32
+    // in-place swap patching (search.cpp): slot colourings and record locations
+    std::vector<int32_t> slot64, first64;           // [op] eval64 slot, first producer position
+    std::vector<int32_t> cslot, first_far;          // [op] eval32 cold slot (-1), first far producer
+    std::vector<uint32_t> op_off64;                 // [pos] byte offset of the op record in blob
+    std::vector<int32_t> tile64_of, tile32_of;      // [pos] tile holding the op's records
+    std::vector<uint32_t> eloc64, eloc32;           // [edge] record offset (| kPinHeavy: heavy)
     int64_t comm_gen = -1;
     // device copies
     DevBuf d_blob, d_heavy, d_tiles, d_pos, d_adj, d_allowed_pos, d_view, d_order;
@@ -106,6 +114,8 @@ pesto_status ensure_comm_tables(pesto_graph *g);
 pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<Layout> &out,
                           bool use_cache, const uint8_t *x_op = nullptr);
 pesto_status upload_layout(pesto_graph *g, Layout &L);
+// v4 swap rule (DESIGN.md §4 S3) for the ops a (first) and c (second) of an adjacent pair
+bool pair_blocked(const pesto_graph *g, int32_t a, int32_t c);
 BaseLayoutDev layout_view(const Layout &L);
 void fill_eval_common(const pesto_graph *g, EvalParams &p);
 pesto_status ensure_state(pesto_graph *g, const EvalParams &p, int search_mode, int64_t n_tasks,

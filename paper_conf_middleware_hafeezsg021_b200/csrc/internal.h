@@ -103,7 +103,20 @@ struct CommitParams {
     int32_t patch32;                    // eval32 records carry base codes: patch them too
 };
 
+// In-place layout patch (a committed adjacent swap, search.cpp): block rotations first, in list
+// order, then masked word / byte stores in list order.
+enum PatchKind : uint32_t { kPatchSet32 = 0, kPatchRotate = 1, kPatchSet8 = 2 };
+struct PatchOp {
+    uint64_t ptr;        // device address (16-aligned for rotations, 4-aligned for Set32)
+    uint32_t kind;
+    uint32_t a, b;       // rotate: [ptr, ptr+a) and [ptr+a, ptr+a+b) exchange places (16-multiples)
+    uint32_t mask, val;  // set: *ptr = (*ptr & ~mask) | (val & mask)
+    uint32_t pad;
+};
+constexpr int kPatchMaxBlock = 48 * 1024;      // rotation bytes a + b (shared-memory staging)
+
 // launchers (kernels.cu / eval32.cu); they return the launch error, if any.
+cudaError_t launch_patch(const PatchOp *ops_dev, int n_ops, int max_block, cudaStream_t st);
 // mode: 0 explicit rows, 1 search, 2 explicit list (eval64 only)
 cudaError_t launch_eval(const EvalParams &p, int search_mode, int grid, cudaStream_t st);
 cudaError_t launch_eval32(const EvalParams &p, int search_mode, int grid, cudaStream_t st);

@@ -643,6 +643,39 @@ cudaError_t launch_transpose(const TransposeParams &p, cudaStream_t st) {
     return cudaGetLastError();
 }
 
+// ---------------------------------------------------------------------------------------------
+// Layout patch for committed swaps (search.cpp swap_in_place): one CTA applies the host's list.
+// ---------------------------------------------------------------------------------------------
+static __global__ void patch_kernel(const PatchOp *ops, int n_ops) {
+    extern __shared__ uint4 pbuf[];
+    for (int i = 0; i < n_ops; i++) {
+        const PatchOp op = ops[i];
+        if (op.kind != kPatchRotate) continue;
+        uint4 *p = reinterpret_cast<uint4 *>(op.ptr);
+        const int na = (int)(op.a / 16), nb = (int)(op.b / 16);
+        for (int t = threadIdx.x; t < na + nb; t += blockDim.x) pbuf[t] = p[t];
+        __syncthreads();
+        for (int t = threadIdx.x; t < na + nb; t += blockDim.x) p[t] = t < nb ? pbuf[na + t] : pbuf[t - nb];
+        __syncthreads();
+    }
+    if (threadIdx.x != 0) return;
+    for (int i = 0; i < n_ops; i++) {            // in order: later stores win
+        const PatchOp op = ops[i];
+        if (op.kind == kPatchSet32) {
+            uint32_t *w = reinterpret_cast<uint32_t *>(op.ptr);
+            *w = (*w & ~op.mask) | (op.val & op.mask);
+        } else if (op.kind == kPatchSet8) {
+            *reinterpret_cast<uint8_t *>(op.ptr) = (uint8_t)op.val;
+        }
+    }
+}
+
+cudaError_t launch_patch(const PatchOp *ops_dev, int n_ops, int max_block, cudaStream_t st) {
+    note_launch();
+    patch_kernel<<<1, 256, (size_t)std::max(max_block, 16), st>>>(ops_dev, n_ops);
+    return cudaGetLastError();
+}
+
 cudaError_t launch_commit(const CommitParams &p, cudaStream_t st) {
     note_launch();
     const int threads = ((p.P + 31) / 32) * 32;

@@ -16,8 +16,6 @@
 
 namespace pesto {
 
-static constexpr int kMaxInlineBytes = 2048;
-
 namespace {
 
 // LIFO interval colouring: interval of consumer w is [start[w], end[w]] (end = pos(w) + 1),
@@ -114,7 +112,11 @@ pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<
             }
         }
     }
-    auto L = std::make_shared<Layout>();
+    // a search base rebuilt after a committed swap reuses its layout object, so the device
+    // buffers are recycled instead of freed (cudaFree synchronises the device) and reallocated
+    std::shared_ptr<Layout> L = (x_op && out && out.use_count() == 1) ? out : std::make_shared<Layout>();
+    L->on_device = false;
+    L->stage_bytes = 0;
     L->comm_gen = g->comm_gen;
     L->order.assign(order, order + n);
     L->pos.assign(n, -1);
@@ -147,12 +149,13 @@ pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<
 
     // ---------------- eval64 stream ----------------
     {
-        std::vector<int32_t> first(n, -1);
+        std::vector<int32_t> &first = L->first64;
+        first.assign(n, -1);
         for (int64_t e = 0; e < m; e++) {
             const int32_t w = g->dst[e], ps = pos[g->src[e]];
             if (first[w] < 0 || ps < first[w]) first[w] = ps;
         }
-        std::vector<int32_t> slot;
+        std::vector<int32_t> &slot = L->slot64;
         L->W = std::max(colour_intervals(n, first, pos, slot), 1);
         std::vector<uint8_t> seen(n, 0), first_flag(m, 0);
         for (int32_t k = 0; k < n; k++) {
@@ -167,8 +170,12 @@ pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<
         L->heavy.clear();
         L->tiles.clear();
         L->blob.reserve((size_t)n * 16 + (size_t)m * es + 64 * kTileHeader);
+        L->op_off64.assign(n, 0);
+        L->tile64_of.assign(n, 0);
+        L->eloc64.assign(m, 0);
         auto put_edge = [&](std::vector<uint8_t> &buf, int64_t e) {
             const size_t at = buf.size();
+            L->eloc64[e] = (uint32_t)at | (&buf == &L->heavy ? kPinHeavy : 0u);
             buf.resize(at + es, 0);
             EdgeRec r;
             r.t0 = g->t_class[(size_t)e * C];
@@ -185,6 +192,8 @@ pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<
             const int64_t nout = g->out_off[u + 1] - g->out_off[u];
             const bool heavy = nout * es > kMaxInlineBytes;
             tw.maybe_cut(k, 16 + (heavy ? 16 : (size_t)nout * es));
+            L->op_off64[k] = (uint32_t)L->blob.size();
+            L->tile64_of[k] = (int32_t)L->tiles.size();
             OpRec op;
             op.p = g->p[u];
             op.in_slot = slot[u];
@@ -204,7 +213,9 @@ pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<
     // distance 1: the next op's forwarding register; 2..kNearDelta: the ring; farther: cold slot
     auto next_edge = [&](int64_t e) { return pos[g->dst[e]] - pos[g->src[e]] == 1; };
     auto near_edge = [&](int64_t e) { return pos[g->dst[e]] - pos[g->src[e]] <= kNearDelta; };
-    std::vector<int32_t> first_far, cslot;
+    std::vector<int32_t> &first_far = L->first_far, &cslot = L->cslot;
+    first_far.clear();
+    cslot.clear();
     std::vector<uint8_t> has_near;
     L->W32 = 0;
     if (g->eligible32) {
@@ -241,6 +252,8 @@ pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<
         L->stage_bytes32 = 0;
         L->blob32.reserve((size_t)(n + m / 2 + 64) * kStepBytes + 64 * kTileHeader);
         L->op_off32.assign(n, 0);
+        L->tile32_of.assign(n, 0);
+        L->eloc32.assign(m, 0);
         // patch index: locations of every edge record by successor position
         L->pin_off.assign((size_t)n + 1, 0);
         L->pin_ref.assign(m, 0);
@@ -249,8 +262,13 @@ pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<
         std::vector<uint32_t> pfill(L->pin_off.begin(), L->pin_off.end() - 1);
         auto edge_rec = [&](int64_t e, size_t at) {
             EdgeRec32 r;
-            r.t0 = t32(e, 0);
-            r.t1 = C > 1 ? t32(e, 1) : 0u;
+            if (g->D == 2) {             // by direction: t0 on link 0 -> 1, t1 on link 1 -> 0
+                r.t0 = t32(e, g->link_class[1]);
+                r.t1 = t32(e, g->link_class[2]);
+            } else {                     // by link class (D > 2: at most two classes here)
+                r.t0 = t32(e, 0);
+                r.t1 = C > 1 ? t32(e, 1) : 0u;
+            }
             const int32_t w = g->dst[e];
             r.succ_pos = (int32_t)((uint32_t)pos[w] | (xcode(w) << kSuccXShift));
             // byte offset of the lane's slot column: ring slot (pos & 15) or cold slot, x 128
@@ -259,6 +277,7 @@ pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<
                                      : (uint32_t)cslot[w] * 128u) |
                        (first32[e] ? kT32First : 0u);
             L->pin_ref[pfill[pos[w]]++] = (uint32_t)at;
+            L->eloc32[e] = (uint32_t)at;
             return r;
         };
         // tiles hold whole ops, except an op larger than a tile, which continues in the next
@@ -286,6 +305,7 @@ pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<
             const size_t op_bytes = (size_t)nsteps * kStepBytes;
             if (t_steps > 0 && blob.size() - t_start + op_bytes > budget) { close(); open(); }
             L->op_off32[k] = (uint32_t)blob.size();
+            L->tile32_of[k] = (int32_t)L->tiles32.size();
             for (int64_t s = 0; s < nsteps; s++) {
                 if (t_steps > 0 && blob.size() - t_start + kStepBytes > budget) { close(); open(); }
                 const size_t at = blob.size();
@@ -349,6 +369,23 @@ pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<
     }
     out = L;
     return PESTO_OK;
+}
+
+bool pair_blocked(const pesto_graph *g, int32_t a, int32_t c) {
+    if (g->out_off[a + 1] - g->out_off[a] > kSwapMaxOut || g->out_off[c + 1] - g->out_off[c] > kSwapMaxOut)
+        return true;
+    for (int64_t i = g->out_off[a]; i < g->out_off[a + 1]; i++) {
+        const int32_t w = g->dst[g->out_edges[i]];
+        if (w == c) return true;
+        for (int64_t j = g->out_off[c]; j < g->out_off[c + 1]; j++)
+            if (g->dst[g->out_edges[j]] == w) return true;        // common consumer
+    }
+    for (int64_t i = g->in_off[a]; i < g->in_off[a + 1]; i++) {
+        const int32_t u = g->src[g->in_edges[i]];
+        for (int64_t j = g->in_off[c]; j < g->in_off[c + 1]; j++)
+            if (g->src[g->in_edges[j]] == u) return true;         // common producer
+    }
+    return false;
 }
 
 }  // namespace pesto

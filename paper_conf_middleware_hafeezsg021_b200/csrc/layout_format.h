@@ -84,10 +84,10 @@ struct alignas(16) OpRec32 {
 };
 
 struct alignas(16) EdgeRec32 {
-    uint32_t t0;         // transfer time, link class 0 (< kMaxDur32)
+    uint32_t t0;         // transfer time (< kMaxDur32): D = 2 link 0 -> 1, else link class 0
     int32_t succ_pos;    // successor position | its base code << 24
     uint32_t target;     // slot byte offset (ring: (pos & 15) * 128, cold: slot * 128) | kT32Near | kT32First
-    uint32_t t1;         // link class 1; classes >= 2 follow in 4-byte words
+    uint32_t t1;         // D = 2: link 1 -> 0, else link class 1
 };
 
 inline int edge_stride32_for(int classes) {

@@ -75,6 +75,9 @@ struct pesto_search {
     std::vector<int64_t> h_mk;
     bool all_below = false;
     bool use32 = false;            // eval32 records exist for every base
+    // committed swaps: patched in place on the device vs. layout rebuilt on the host
+    DevBuf d_patch;
+    int64_t n_swap_inplace = 0, n_swap_rebuilt = 0;
 };
 
 namespace {
@@ -183,6 +186,223 @@ pesto_status download_x(pesto_search *s, int b, uint8_t *x_op) {
         x_op[s->order[b][q]] = (uint8_t)x;
     }
     return PESTO_OK;
+}
+
+// ---------------------------------------------------------------------------------------------
+// In-place patch of a committed adjacent swap (k, k+1) of base b.
+// Under the v4 rule (§4 S3) the two ops share no edge, producer or consumer, so only local
+// records change: the two ops' record blocks exchange places inside their tile, their in-edge
+// records get the new successor positions (and, in eval32, targets), the eval32 heads that name
+// their cold slots for prefetch are re-pointed, and the position-indexed arrays are updated.
+// The slot colourings are kept; the swap is refused (-> full rebuild) when that would break the
+// padded-interval invariant of §3.3, when an edge would change between near and far, or when
+// the pair spans two tiles.  The host copies are patched the same way; the device copies are
+// patched by one kernel (their embedded base codes are newer than the host's and are kept).
+// ---------------------------------------------------------------------------------------------
+struct Patcher {
+    std::vector<PatchOp> ops;
+    int max_block = 0;
+    void set32(const DevBuf &d, uint8_t *host, size_t off, uint32_t mask, uint32_t val) {
+        uint32_t w;
+        std::memcpy(&w, host + off, 4);
+        w = (w & ~mask) | (val & mask);
+        std::memcpy(host + off, &w, 4);
+        ops.push_back(PatchOp{(uint64_t)(uintptr_t)(d.as<uint8_t>() + off), kPatchSet32, 0, 0, mask, val, 0});
+    }
+    template <class T>
+    void set_elem(const DevBuf &d, std::vector<T> &host, size_t i, T val) {
+        static_assert(sizeof(T) == 4 || sizeof(T) == 1, "4- or 1-byte elements");
+        host[i] = val;
+        uint32_t v = 0;
+        std::memcpy(&v, &val, sizeof(T));
+        ops.push_back(PatchOp{(uint64_t)(uintptr_t)(d.as<uint8_t>() + i * sizeof(T)),
+                              sizeof(T) == 4 ? (uint32_t)kPatchSet32 : (uint32_t)kPatchSet8, 0, 0,
+                              ~0u, v, 0});
+    }
+    void rotate(const DevBuf &d, std::vector<uint8_t> &host, size_t off, uint32_t a, uint32_t b) {
+        std::rotate(host.begin() + off, host.begin() + off + a, host.begin() + off + a + b);
+        ops.push_back(PatchOp{(uint64_t)(uintptr_t)(d.as<uint8_t>() + off), kPatchRotate, a, b, 0, 0, 0});
+        max_block = std::max(max_block, (int)(a + b));
+    }
+};
+
+bool swap_in_place(pesto_search *s, int b, int32_t k, Patcher &pt) {
+    pesto_graph *g = s->g;
+    Layout &L = *s->layouts[b];
+    const int32_t n = g->n;
+    if (k < 0 || k + 1 >= n || L.slot64.empty()) return false;
+    const int32_t a = L.order[k], c = L.order[k + 1];
+    const bool has32 = L.W32 > 0;
+    const int C = g->n_classes;
+    const int es = edge_stride_for(C);
+    auto nout = [&](int32_t op) { return g->out_off[op + 1] - g->out_off[op]; };
+    auto heavy64 = [&](int32_t op) { return nout(op) * es > kMaxInlineBytes; };
+    auto size64 = [&](int32_t op) { return (uint32_t)(heavy64(op) ? 32 : 16 + nout(op) * es); };
+    auto nst = [&](int32_t op) { return (uint32_t)std::max<int64_t>(1, (nout(op) + 1) / 2); };
+    auto npos = [&](int32_t op) { return op == a ? k + 1 : (op == c ? k : L.pos[op]); };
+    auto cls = [](int32_t d) { return d == 1 ? 0 : (d <= kNearDelta ? 1 : 2); };
+    const int32_t prev = k >= 1 ? L.order[k - 1] : -1;
+    const int32_t p2 = k + 2 < n ? L.order[k + 2] : -1;
+
+    // ---- checks (nothing is modified before all pass) ----
+    if (L.tile64_of[k] != L.tile64_of[k + 1]) return false;
+    if (size64(a) + size64(c) > (uint32_t)kPatchMaxBlock) return false;
+    if (has32) {
+        if (L.tile32_of[k] != L.tile32_of[k + 1]) return false;
+        if ((nst(a) + nst(c)) * kStepBytes > (uint32_t)kPatchMaxBlock) return false;
+        for (int32_t op : {a, c}) {
+            for (int64_t i = g->in_off[op]; i < g->in_off[op + 1]; i++) {
+                const int64_t e = g->in_edges[i];
+                const int32_t u = g->src[e];
+                if ((cls(L.pos[op] - L.pos[u]) == 2) != (cls(npos(op) - npos(u)) == 2)) return false;
+            }
+            for (int64_t i = g->out_off[op]; i < g->out_off[op + 1]; i++) {
+                const int32_t w = g->dst[g->out_edges[i]];
+                if ((cls(L.pos[w] - L.pos[op]) == 2) != (cls(npos(w) - npos(op)) == 2)) return false;
+            }
+        }
+    }
+    // padded intervals (§3.3): a's interval now ends at k+2; consumers first fed by c now start at k
+    auto intervals_ok = [&](const std::vector<int32_t> &first, const std::vector<int32_t> &slot,
+                            bool far_only) {
+        auto counts = [&](int32_t u, int32_t w) {       // does edge u -> w open w's interval?
+            return !far_only || cls(npos(w) - npos(u)) == 2;
+        };
+        if (slot[a] >= 0 && first[a] >= 0 && p2 >= 0) {
+            for (int64_t i = g->out_off[p2]; i < g->out_off[p2 + 1]; i++) {
+                const int32_t u = g->dst[g->out_edges[i]];
+                if (counts(p2, u) && first[u] == k + 2 && slot[u] == slot[a]) return false;
+            }
+        }
+        if (prev >= 0 && first[prev] >= 0 && slot[prev] >= 0) {
+            for (int64_t i = g->out_off[c]; i < g->out_off[c + 1]; i++) {
+                const int32_t u = g->dst[g->out_edges[i]];
+                if (counts(c, u) && first[u] == k + 1 && slot[u] == slot[prev]) return false;
+            }
+        }
+        return true;
+    };
+    if (!intervals_ok(L.first64, L.slot64, false)) return false;
+    if (has32 && !intervals_ok(L.first_far, L.cslot, true)) return false;
+
+    // ---- order, positions, per-position arrays ----
+    std::swap(L.order[k], L.order[k + 1]);
+    L.pos[a] = k + 1;
+    L.pos[c] = k;
+    pt.set_elem(L.d_order, L.order, k, c);
+    pt.set_elem(L.d_order, L.order, k + 1, a);
+    pt.set_elem(L.d_pos, L.pos, a, k + 1);
+    pt.set_elem(L.d_pos, L.pos, c, k);
+    pt.set_elem(L.d_allowed_pos, L.allowed_pos, k, g->allowed[c]);
+    pt.set_elem(L.d_allowed_pos, L.allowed_pos, k + 1, g->allowed[a]);
+    for (int32_t q = std::max(0, k - 1); q <= k + 1 && q + 1 < n; q++)
+        pt.set_elem(L.d_adj, L.swap_blocked, q, (uint8_t)(pair_blocked(g, L.order[q], L.order[q + 1]) ? 1 : 0));
+    // first producer positions of the consumers of a and c
+    auto refirst = [&](int32_t u, std::vector<int32_t> &first, bool far_only) {
+        int32_t f = -1;
+        for (int64_t i = g->in_off[u]; i < g->in_off[u + 1]; i++) {
+            const int32_t p = L.pos[g->src[g->in_edges[i]]];
+            if (far_only && cls(L.pos[u] - p) != 2) continue;
+            if (f < 0 || p < f) f = p;
+        }
+        first[u] = f;
+    };
+
+    // ---- eval64 stream ----
+    {
+        const uint32_t off = L.op_off64[k], A = size64(a), B = size64(c);
+        pt.rotate(L.d_blob, L.blob, off, A, B);
+        L.op_off64[k] = off;
+        L.op_off64[k + 1] = off + B;
+        if (!heavy64(a))
+            for (int64_t i = g->out_off[a]; i < g->out_off[a + 1]; i++) L.eloc64[g->out_edges[i]] += B;
+        if (!heavy64(c))
+            for (int64_t i = g->out_off[c]; i < g->out_off[c + 1]; i++) L.eloc64[g->out_edges[i]] -= A;
+        for (int32_t op : {a, c}) {
+            for (int64_t i = g->in_off[op]; i < g->in_off[op + 1]; i++) {
+                const uint32_t loc = L.eloc64[g->in_edges[i]];
+                const bool hv = (loc & kPinHeavy) != 0;
+                pt.set32(hv ? L.d_heavy : L.d_blob, hv ? L.heavy.data() : L.blob.data(),
+                         (loc & ~kPinHeavy) + 8, ~0u, (uint32_t)L.pos[op]);
+            }
+            for (int64_t i = g->out_off[op]; i < g->out_off[op + 1]; i++)
+                refirst(g->dst[g->out_edges[i]], L.first64, false);
+        }
+    }
+
+    // ---- eval32 stream ----
+    if (has32) {
+        const uint32_t off = L.op_off32[k], A = nst(a) * kStepBytes, B = nst(c) * kStepBytes;
+        pt.rotate(L.d_blob32, L.blob32, off, A, B);
+        pt.set_elem(L.d_op_off32, L.op_off32, k, off);
+        pt.set_elem(L.d_op_off32, L.op_off32, k + 1, off + B);
+        // records of the out-edges of a and c moved: their locations and patch-index entries
+        // (one pass per successor over its entries, old -> new, so parallel edges stay exact)
+        for (int32_t op : {a, c}) {
+            const uint32_t base = op == a ? off : off + A, len = op == a ? A : B;   // old block
+            const uint32_t shift = op == a ? B : (uint32_t)(0u - A);       // mod 2^32
+            std::vector<int32_t> succ_q;
+            for (int64_t i = g->out_off[op]; i < g->out_off[op + 1]; i++)
+                succ_q.push_back(L.pos[g->dst[g->out_edges[i]]]);
+            std::sort(succ_q.begin(), succ_q.end());
+            succ_q.erase(std::unique(succ_q.begin(), succ_q.end()), succ_q.end());
+            for (int32_t q : succ_q)                  // entries into op's old block move with it
+                for (uint32_t r = L.pin_off[q]; r < L.pin_off[q + 1]; r++)
+                    if (L.pin_ref[r] >= base && L.pin_ref[r] < base + len)
+                        pt.set_elem(L.d_pin_ref, L.pin_ref, r, L.pin_ref[r] + shift);
+            for (int64_t i = g->out_off[op]; i < g->out_off[op + 1]; i++)
+                L.eloc32[g->out_edges[i]] += shift;
+        }
+        // patch index of positions k (now c) and k+1 (now a)
+        {
+            uint32_t r = L.pin_off[k];
+            for (int64_t i = g->in_off[c]; i < g->in_off[c + 1]; i++)
+                pt.set_elem(L.d_pin_ref, L.pin_ref, r++, L.eloc32[g->in_edges[i]]);
+            pt.set_elem(L.d_pin_off, L.pin_off, k + 1, r);
+            for (int64_t i = g->in_off[a]; i < g->in_off[a + 1]; i++)
+                pt.set_elem(L.d_pin_ref, L.pin_ref, r++, L.eloc32[g->in_edges[i]]);
+        }
+        for (int32_t op : {a, c})
+            for (int64_t i = g->out_off[op]; i < g->out_off[op + 1]; i++)
+                refirst(g->dst[g->out_edges[i]], L.first_far, true);
+        // targets of every in-edge of a, c and the op after them (NEXT <-> NEAR may change there)
+        auto retarget = [&](int32_t w) {
+            const int32_t q = L.pos[w];
+            int64_t near_first = -1, far_first = -1;
+            int32_t near_p = 0, far_p = 0;
+            for (int64_t i = g->in_off[w]; i < g->in_off[w + 1]; i++) {   // ascending edge id
+                const int64_t e = g->in_edges[i];
+                const int32_t p = L.pos[g->src[e]];
+                const int cl = cls(q - p);
+                if (cl == 1 && (near_first < 0 || p < near_p)) { near_first = e; near_p = p; }
+                if (cl == 2 && (far_first < 0 || p < far_p)) { far_first = e; far_p = p; }
+            }
+            for (int64_t i = g->in_off[w]; i < g->in_off[w + 1]; i++) {
+                const int64_t e = g->in_edges[i];
+                const int cl = cls(q - L.pos[g->src[e]]);
+                const uint32_t tgt = cl == 0 ? kT32Next
+                                   : cl == 1 ? (kT32Near | (uint32_t)(q & (kRing - 1)) * 128u |
+                                                (e == near_first ? kT32First : 0u))
+                                             : ((uint32_t)L.cslot[w] * 128u | (e == far_first ? kT32First : 0u));
+                const uint32_t loc = L.eloc32[e];
+                pt.set32(L.d_blob32, L.blob32.data(), loc + 4, kSuccPosMask, (uint32_t)q);
+                pt.set32(L.d_blob32, L.blob32.data(), loc + 8, ~0u, tgt);
+            }
+            pt.set32(L.d_blob32, L.blob32.data(), L.op_off32[q] + 12, kStHasNear,
+                     near_first >= 0 ? kStHasNear : 0u);
+        };
+        retarget(a);
+        retarget(c);
+        if (p2 >= 0) retarget(p2);
+        // heads that name a cold slot for prefetch: q names the op at q + kPrefetchDist
+        for (int32_t q : {k - kPrefetchDist, k + 1 - kPrefetchDist, k, k + 1}) {
+            if (q < 0 || q >= n) continue;
+            const int32_t ahead = q + kPrefetchDist;
+            const int32_t pf = ahead < n ? L.cslot[L.order[ahead]] : -1;
+            pt.set32(L.d_blob32, L.blob32.data(), L.op_off32[q] + 8, ~0u, (uint32_t)pf);
+        }
+    }
+    return true;
 }
 
 }  // namespace
@@ -348,16 +568,30 @@ pesto_status pesto_search_commit(pesto_search *s, void *stream) {
         std::memcpy(s->h_mk.data(), s->h_keys, 8 * s->P);   // h_keys doubles as a staging buffer
         update_all_below(s);
         bool changed = false;
+        Patcher pt;
         for (int b = 0; b < s->P; b++) {
             const int32_t k = s->h_swap[b];
             if (k < 0) continue;
             std::swap(s->order[b][k], s->order[b][k + 1]);
+            if (swap_in_place(s, b, k, pt)) {
+                s->n_swap_inplace++;
+                continue;
+            }
+            s->n_swap_rebuilt++;
             std::vector<uint8_t> x_op(g->n);
             pesto_status rc = download_x(s, b, x_op.data());      // K4 already swapped the bits
             if (rc) return rc;
             if ((rc = build_layout(g, s->order[b].data(), s->layouts[b], false, x_op.data()))) return rc;
             if ((rc = upload_layout(g, *s->layouts[b]))) return rc;
             changed = true;
+        }
+        if (!pt.ops.empty()) {
+            const size_t bytes = pt.ops.size() * sizeof(PatchOp);
+            if ((e = s->d_patch.ensure(bytes)) != cudaSuccess ||
+                (e = cudaMemcpyAsync(s->d_patch.ptr, pt.ops.data(), bytes, cudaMemcpyHostToDevice, st)) != cudaSuccess ||
+                (e = launch_patch(s->d_patch.as<PatchOp>(), (int)pt.ops.size(), pt.max_block, st)) != cudaSuccess ||
+                (e = cudaStreamSynchronize(st)) != cudaSuccess)
+                return cuda_fail(e, "patch swapped layouts");
         }
         if (changed) {
             refresh_views(s);
@@ -420,6 +654,13 @@ pesto_status pesto_search_get(pesto_search *s, int32_t base, int64_t *mk, uint8_
 }
 
 int64_t pesto_search_step_count(const pesto_search *s) { return s ? s->step : -1; }
+
+pesto_status pesto_search_swap_stats(const pesto_search *s, int64_t *in_place, int64_t *rebuilt) {
+    if (!s) return fail(PESTO_EINVAL, "NULL search");
+    if (in_place) *in_place = s->n_swap_inplace;
+    if (rebuilt) *rebuilt = s->n_swap_rebuilt;
+    return PESTO_OK;
+}
 
 void pesto_search_destroy(pesto_search *s) {
     if (!s) return;

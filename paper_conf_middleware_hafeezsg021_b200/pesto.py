@@ -73,6 +73,7 @@ SIGNATURES = {
     "pesto_search_candidate_keys": (_I32, [_VP, _I32, _I64, _I64, _VP, _VP]),
     "pesto_search_get": (_I32, [_VP, _I32, _VP, _VP, _VP]),
     "pesto_search_step_count": (_I64, [_VP]),
+    "pesto_search_swap_stats": (_I32, [_VP, _VP, _VP]),
     "pesto_search_destroy": (None, [_VP]),
     "pesto_nccl_unique_id": (_I32, [_VP]),
     "pesto_last_error": (C.c_char_p, []),
@@ -289,3 +290,9 @@ class Search:
     @property
     def step_count(self) -> int:
         return int(_L.pesto_search_step_count(self._h))
+
+    def swap_stats(self) -> tuple:
+        """(committed swaps patched in place on the device, swaps that rebuilt a layout)."""
+        a, b = C.c_int64(), C.c_int64()
+        _check(_L.pesto_search_swap_stats(self._h, C.byref(a), C.byref(b)))
+        return int(a.value), int(b.value)

@@ -202,6 +202,38 @@ def test_search_steps_match_reference(P, O):
         del keys
 
 
+@pytest.mark.parametrize("D,mix,steps", [(2, (0, 0, 0, 100), 24), (2, (30, 10, 10, 50), 12),
+                                         (4, (20, 10, 10, 60), 10)])
+def test_committed_swaps_patch_layouts(P, O, D, mix, steps):
+    """swap-heavy search on a multi-tile graph: committed swaps are patched into the device
+    layouts in place or rebuilt; either way every step matches the oracle, and
+    afterwards every candidate key of the patched bases matches too (eval64 layouts)."""
+    g = dag.random_dag(61 + D, 1400, 1.6, D=D, p_max=4000, max_bytes=300_000, beta0=700,
+                       beta1_fs=30_000)
+    G = P.Graph.from_arrays(g)
+    xs, orders = _bases(g, 2, seed=13)
+    K = 4096
+    S = P.Search(G, xs, orders, K, mix, seed=17)
+    rx, ro = xs.copy(), orders.copy()
+    rmk = np.asarray([O.makespan(g, rx[b], ro[b]) for b in range(2)], np.int64)
+    swaps = 0
+    for step in range(steps):
+        before = ro.copy()
+        S.step()
+        O.search_step(g, rx, ro, rmk, K, 17, step, mix)
+        swaps += int(sum((before[b] != ro[b]).any() for b in range(2)))
+        for b in range(2):
+            mk, x, o = S.get(b)
+            assert mk == rmk[b] and (x == rx[b]).all() and (o == ro[b]).all(), (step, b)
+    in_place, rebuilt = S.swap_stats()
+    assert in_place + rebuilt == swaps and swaps > 0
+    assert in_place > 0
+    for b in range(2):
+        gk = S.candidate_keys(b, 0, K)
+        ok = O.candidate_keys(g, 2, b, rx, ro, 0, K, 17, steps, mix)
+        assert (gk == ok).all(), (b, np.nonzero(gk != ok)[0][:5])
+
+
 def test_fake_sharding_equals_single_rank(P, O):
     """W rank ranges evaluated one after another on one GPU, minima reduced on the host."""
     g = _search_graph(seed=41, n=90)
