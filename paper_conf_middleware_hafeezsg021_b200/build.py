@@ -44,8 +44,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
     objs = []
     for f in CU_SOURCES:
         o = os.path.join(BUILD, f + ".o")
-        cpl = os.environ.get("PESTO_EVAL32_CPL")
-        extra = [f"-DPESTO_EVAL32_CPL={int(cpl)}"] if cpl else []
+        extra = []
         cmd = [NVCC, *ARCH, "-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC", *extra,
                "-Xptxas", "-v" if verbose else "-O3", "-I", INC, "-I", CSRC, "-c",
                os.path.join(CSRC, f), "-o", o]

@@ -88,6 +88,26 @@ __device__ __forceinline__ void cp_async4(uint32_t smem_addr, const void *gptr, 
         " @p cp.async.ca.shared.global [%0], [%1], 4;\n}\n"
         ::"r"(smem_addr), "l"(gptr), "r"((int)pred) : "memory");
 }
+// predicated forms (a guard predicate, not a branch): the walk's per-edge pushes stay in one
+// basic block so the scheduler can interleave the lane's independent candidate chains
+__device__ __forceinline__ uint32_t lds_u32_if(uint32_t addr, bool p) {
+    uint32_t v = 0;
+    asm volatile("{\n .reg .pred q;\n setp.ne.b32 q, %2, 0;\n @q ld.shared.u32 %0, [%1];\n}\n"
+                 : "+r"(v) : "r"(addr), "r"((int)p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void sts_u32_if(uint32_t addr, uint32_t v, bool p) {
+    asm volatile("{\n .reg .pred q;\n setp.ne.b32 q, %2, 0;\n @q st.shared.u32 [%0], %1;\n}\n"
+                 ::"r"(addr), "r"(v), "r"((int)p) : "memory");
+}
+__device__ __forceinline__ void stg_u32_if(void *ptr, uint32_t v, bool p) {
+    asm volatile("{\n .reg .pred q;\n setp.ne.b32 q, %2, 0;\n @q st.global.u32 [%0], %1;\n}\n"
+                 ::"l"(ptr), "r"(v), "r"((int)p) : "memory");
+}
+__device__ __forceinline__ void redmax_u32_if(void *ptr, uint32_t v, bool p) {
+    asm volatile("{\n .reg .pred q;\n setp.ne.b32 q, %2, 0;\n @q red.relaxed.gpu.global.max.u32 [%0], %1;\n}\n"
+                 ::"l"(ptr), "r"(v), "r"((int)p) : "memory");
+}
 // 4-byte async copy that writes zero when `have` is false (src-size 0: nothing is read)
 __device__ __forceinline__ void cp_async4_zfill(uint32_t smem_addr, const void *gptr, bool have) {
     asm volatile("cp.async.ca.shared.global [%0], [%1], 4, %2;\n"

@@ -508,11 +508,9 @@ int planes_of32(int D) { return D <= 2 ? 1 : (D <= 4 ? 2 : 4); }
 
 }  // namespace
 
-int eval32_cpl() { return kEval32Cpl; }
-
 int eval32_smem_bytes(const EvalParams &p, int search_mode) {
     (void)search_mode;
-    const int cpl = kEval32Cpl;
+    const int cpl = p.cpl32 == 1 ? 1 : 2;
     const int nw = warps_for(cpl);
     const int pl = planes_of32(p.D);
     size_t b = (size_t)kStages * (p.stage_bytes32 + kStepBytes) + 2 * kStages * 8;
@@ -525,10 +523,10 @@ int eval32_smem_bytes(const EvalParams &p, int search_mode) {
     return (int)b + 128;
 }
 
-// eval32 runs graphs with at most two link classes (layout.cpp emits no stream otherwise)
-#define PESTO_DISPATCH32(FN, ...)                                                          \
+// eval32 runs graphs with at most two link classes (layout.cpp emits no stream otherwise);
+// candidates per lane: p.cpl32 (1 or 2, chosen by the host: choose_cpl32)
+#define PESTO_DISPATCH32_C(FN, C, ...)                                                     \
     do {                                                                                   \
-        constexpr int C = kEval32Cpl;                                                      \
         const int pl = planes_of32(p.D);                                                   \
         if (search_mode) {                                                                 \
             if (pl == 1) return FN<1, 1, C>(__VA_ARGS__);                                  \
@@ -539,6 +537,11 @@ int eval32_smem_bytes(const EvalParams &p, int search_mode) {
             if (pl == 2) return FN<0, 2, C>(__VA_ARGS__);                                  \
             return FN<0, 4, C>(__VA_ARGS__);                                               \
         }                                                                                  \
+    } while (0)
+#define PESTO_DISPATCH32(FN, ...)                                                          \
+    do {                                                                                   \
+        if (p.cpl32 == 1) PESTO_DISPATCH32_C(FN, 1, __VA_ARGS__);                          \
+        PESTO_DISPATCH32_C(FN, 2, __VA_ARGS__);                                            \
     } while (0)
 
 cudaError_t launch_eval32(const EvalParams &p, int search_mode, int grid, cudaStream_t st) {

@@ -1,6 +1,7 @@
 // graph.cpp -- graph ingest, comm model, position-space layout, seeds and batched evaluation
 // (SURVEY §8(a) rows a0, a1, a3/a4 host side; C ABI in include/pesto.h).
 #include <algorithm>
+#include <cstdlib>
 #include <cstring>
 #include <queue>
 #include <string>
@@ -178,6 +179,15 @@ pesto_status ensure_state(pesto_graph *g, const EvalParams &p, int search_mode, 
     if (e != cudaSuccess) return cuda_fail(e, "allocate slot state");
     *grid_out = (int)grid;
     return PESTO_OK;
+}
+
+int choose_cpl32(const pesto_graph *g, int64_t n_tasks) {
+    static const int forced = [] {
+        const char *e = std::getenv("PESTO_EVAL32_CPL");
+        return e ? std::atoi(e) : 0;
+    }();
+    if (forced == 1 || forced == 2) return forced;
+    return n_tasks <= 2 * (int64_t)g->sms ? 1 : 2;
 }
 
 pesto_status ensure_state32(pesto_graph *g, const EvalParams &p, int search_mode, int64_t n_tasks,
@@ -557,6 +567,7 @@ pesto_status pesto_eval_batch(pesto_graph *g, const int32_t *order, const void *
     if ((e = cudaMemsetAsync(g->d_flags.ptr, 0, 4, st)) != cudaSuccess) return cuda_fail(e, "reset flags");
     p.flag_count = g->d_flags.as<int32_t>();
     p.flag_list = g->d_flags.as<int32_t>() + 4;
+    p.cpl32 = choose_cpl32(g, p.n_tasks);
     if ((s = ensure_state32(g, p, 0, p.n_tasks, &grid))) return s;
     p.state32 = g->d_state32.as<uint32_t>();
     if ((e = launch_eval32(p, 0, grid, st)) != cudaSuccess) return cuda_fail(e, "launch eval32");

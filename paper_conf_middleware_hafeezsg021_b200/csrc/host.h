@@ -120,6 +120,9 @@ BaseLayoutDev layout_view(const Layout &L);
 void fill_eval_common(const pesto_graph *g, EvalParams &p);
 pesto_status ensure_state(pesto_graph *g, const EvalParams &p, int search_mode, int64_t n_tasks,
                           int *grid_out);
+// eval32 candidates per lane for a launch of n_tasks 256-candidate tasks:
+// 1 when every task is resident at once (latency-bound: more warps), else 2
+int choose_cpl32(const pesto_graph *g, int64_t n_tasks);
 pesto_status ensure_state32(pesto_graph *g, const EvalParams &p, int search_mode, int64_t n_tasks,
                             int *grid_out);
 struct DeviceGuard {

@@ -8,10 +8,6 @@
 namespace pesto {
 
 constexpr int kWarps = 8;            // consumer warps per CTA (each = 32 candidates)
-#ifndef PESTO_EVAL32_CPL
-#define PESTO_EVAL32_CPL 2
-#endif
-constexpr int kEval32Cpl = PESTO_EVAL32_CPL;   // eval32: candidates per lane (1, 2 or 4)
 constexpr int kStages = 4;           // TMA tile ring depth
 constexpr int kTileTarget = 8192;    // record bytes per tile (a single op may exceed it)
 constexpr int kTileHeader = 16;      // {pos_begin, pos_end, bytes, 0} at the head of each tile
@@ -73,6 +69,8 @@ struct EvalParams {
     // search: base b runs on eval32 iff base_mk[b] < kSat32 (gate 1), on eval64 iff not (gate 2)
     const int64_t *base_mk;
     int32_t gate;
+    // eval32 candidates per lane (1 or 2): more warps vs. more work per warp instruction
+    int32_t cpl32;
     // eval64 list mode (MODE 2): candidates list[0 .. *list_count)
     const int32_t *list;
     const int32_t *list_count;
@@ -121,7 +119,6 @@ cudaError_t launch_patch(const PatchOp *ops_dev, int n_ops, int max_block, cudaS
 cudaError_t launch_eval(const EvalParams &p, int search_mode, int grid, cudaStream_t st);
 cudaError_t launch_eval32(const EvalParams &p, int search_mode, int grid, cudaStream_t st);
 int eval32_smem_bytes(const EvalParams &p, int search_mode);
-int eval32_cpl();
 int eval32_max_ctas_per_sm(const EvalParams &p, int search_mode);
 cudaError_t launch_transpose(const TransposeParams &p, cudaStream_t st);
 cudaError_t launch_commit(const CommitParams &p, cudaStream_t st);

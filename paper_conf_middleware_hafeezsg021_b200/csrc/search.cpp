@@ -146,6 +146,7 @@ pesto_status launch_search_eval(pesto_search *s, int b_first, int n_bases, int64
         p32.gate = 1;
         p32.tasks_per_base = (j1 - (j0 & ~(int64_t)255) + 255) / 256;
         p32.n_tasks = p32.tasks_per_base * n_bases;
+        p32.cpl32 = choose_cpl32(g, p32.n_tasks);
         if ((rc = ensure_state32(g, p32, 1, p32.n_tasks, &grid))) return rc;
         p32.state32 = g->d_state32.as<uint32_t>();
         if ((e = launch_eval32(p32, 1, grid, st)) != cudaSuccess) return cuda_fail(e, "launch eval32");
