@@ -107,6 +107,38 @@ struct Place32 {
     }
 };
 
+// explicit rows: one 32-row group's bit-sliced plane words at a position (K5 layout)
+template <int PL>
+struct PlaneWords {
+    uint32_t w[PL];
+};
+template <int PL>
+__device__ __forceinline__ PlaneWords<PL> ldg_planes(const uint32_t *pl, int32_t q) {
+    PlaneWords<PL> r;
+    if constexpr (PL == 1) {
+        r.w[0] = __ldg(pl + q);
+    } else if constexpr (PL == 2) {
+        const uint2 t = __ldg(reinterpret_cast<const uint2 *>(pl) + q);
+        r.w[0] = t.x;
+        r.w[1] = t.y;
+    } else {
+        const uint4 t = __ldg(reinterpret_cast<const uint4 *>(pl) + q);
+        r.w[0] = t.x;
+        r.w[1] = t.y;
+        r.w[2] = t.z;
+        r.w[3] = t.w;
+    }
+    return r;
+}
+// codes >= D belong to rows K5 flagged infeasible: clamped so the lane stays in its columns
+template <int PL>
+__device__ __forceinline__ int plane_dev(const PlaneWords<PL> &p, int lane, int dmax) {
+    int x = 0;
+#pragma unroll
+    for (int k = 0; k < PL; k++) x |= (int)((p.w[k] >> lane) & 1u) << k;
+    return PL == 1 ? x : min(x, dmax);
+}
+
 struct Ctx32 {
     uint32_t smem;               // shared address of the CTA's dynamic shared memory (records)
     uint32_t ring;               // shared address of ring[0][0][lane]; slot s, cand c: + (s*CPL+c)*128
@@ -116,14 +148,11 @@ struct Ctx32 {
 };
 
 // one out-edge record, for the lane's CPL candidates (FCFS link of L144 / L188-198)
-template <int PL, int CPL, class PlaceT, class StateT>
+template <int PL, int CPL, class StateT>
 __device__ __forceinline__ void push32(const Ctx32 &cx, const uint4 rec, const int (&x)[CPL],
-                                       const uint32_t (&cc)[CPL], const PlaceT &place,
+                                       const int (&y)[CPL], const uint32_t (&cc)[CPL],
                                        StateT &st, uint32_t (&fwd)[CPL]) {
-    const int32_t succ = (int32_t)(rec.y & kSuccPosMask);
     const uint32_t tgt = rec.z;
-    int y[CPL];
-    place.at(succ, (int)((rec.y >> kSuccXShift) & 7u), y);
     uint32_t a[CPL];
 #pragma unroll
     for (int c = 0; c < CPL; c++) {
@@ -160,22 +189,30 @@ __device__ __forceinline__ void push32(const Ctx32 &cx, const uint4 rec, const i
     }
 }
 
-// the (up to two) out-edges of one step, records already in registers
-template <int PL, int CPL, class PlaceT, class StateT>
+// the (up to two) out-edges of one step, records already in registers; yfn(k, rec, y) gives
+// the successor's devices of edge k
+template <int PL, int CPL, class YFn, class StateT>
 __device__ __forceinline__ void edges32(const Ctx32 &cx, uint32_t flags, const uint4 e0,
                                         const uint4 e1, const int (&x)[CPL],
-                                        const uint32_t (&cc)[CPL], const PlaceT &place,
+                                        const uint32_t (&cc)[CPL], const YFn &yfn,
                                         StateT &st, uint32_t (&fwd)[CPL]) {
     const uint32_t ne = (flags >> kStEdgeShift) & 3u;
-    if (ne >= 1) push32<PL, CPL>(cx, e0, x, cc, place, st, fwd);
-    if (ne >= 2) push32<PL, CPL>(cx, e1, x, cc, place, st, fwd);
+    if (ne >= 1) {
+        int y[CPL];
+        yfn(0, e0, y);
+        push32<PL, CPL>(cx, e0, x, y, cc, st, fwd);
+    }
+    if (ne >= 2) {
+        int y[CPL];
+        yfn(1, e1, y);
+        push32<PL, CPL>(cx, e1, x, y, cc, st, fwd);
+    }
 }
 
-// start the op at position v (head h) whose arrivals are r[c]: S_v, C_v (L142-146)
-template <int CPL, class PlaceT, class StateT>
-__device__ __forceinline__ void begin32(const uint4 h, int32_t v, const PlaceT &place, StateT &st,
-                                        const uint32_t (&r)[CPL], int (&x)[CPL], uint32_t (&cc)[CPL]) {
-    place.at(v, (int)(h.w & kStXMask), x);
+// start the op at position v (head h, devices x) whose arrivals are r[c]: S_v, C_v (L142-146)
+template <int CPL, class StateT>
+__device__ __forceinline__ void begin32(const uint4 h, StateT &st, const uint32_t (&r)[CPL],
+                                        const int (&x)[CPL], uint32_t (&cc)[CPL]) {
 #pragma unroll
     for (int c = 0; c < CPL; c++) {
         cc[c] = add_sat(max(r[c], st.dev(c, x[c])), h.x);    // C_v = S_v + p_v
@@ -355,6 +392,23 @@ eval32_kernel(const EvalParams P) {
         uint32_t cc[CPL], fwd[CPL], nfar[CPL], nnear[CPL];
 #pragma unroll
         for (int c = 0; c < CPL; c++) { x[c] = 0; cc[c] = 0u; fwd[c] = 0u; nfar[c] = 0u; nnear[c] = 0u; }
+        // devices by direct lookup (search: base code + region moves; rows: plane words)
+        auto place_y = [&](int, const uint4 rec, int (&y)[CPL]) {
+            place.at((int32_t)(rec.y & kSuccPosMask), (int)((rec.y >> kSuccXShift) & 7u), y);
+        };
+        // explicit rows: the plane words of the next op and of the next step's successors are
+        // loaded one step ahead (a successor's word is usually an L2 access)
+        PlaneWords<PL> pwx[CPL], pwy[2][CPL];
+        auto pw_load = [&](int32_t q, PlaneWords<PL> (&w)[CPL]) {
+            q = min(q, P.n - 1);                       // padding records name no real position
+#pragma unroll
+            for (int c = 0; c < CPL; c++) w[c] = ldg_planes<PL>(place.pl + c * place.pl_stride, q);
+        };
+        auto pw_y = [&](int k, const uint4, int (&y)[CPL]) {
+#pragma unroll
+            for (int c = 0; c < CPL; c++) y[c] = plane_dev<PL>(pwy[k][c], lane, place.dmax);
+        };
+        if constexpr (MODE == 0) pw_load(0, pwx);
         int32_t v = -1;
         int32_t skip = 0;            // steps of the next tile already walked (swap pair)
         for (int t = 0; t < nt; t++, it++) {
@@ -367,12 +421,16 @@ eval32_kernel(const EvalParams P) {
                 int32_t i = skip;
                 skip = 0;
                 uint4 h = lds_v4(sp), e0 = lds_v4(sp + 16), e1 = lds_v4(sp + 32);
+                if constexpr (MODE == 0) {
+                    pw_load((int32_t)(e0.y & kSuccPosMask), pwy[0]);
+                    pw_load((int32_t)(e1.y & kSuccPosMask), pwy[1]);
+                }
                 while (i < nsteps) {
                     // the next step's records (past the tile's end: padding, never used)
                     const uint4 hn = lds_v4(sp + 48), e0n = lds_v4(sp + 64), e1n = lds_v4(sp + 80);
                     if (!(h.w & kStCont)) {
                         v++;
-                        if (v == ks) {
+                        if (MODE == 1 && v == ks) {
                             // swapped pair: the op at ks+1 runs first, then the op at ks.  They
                             // share no producer, no consumer and no edge (DESIGN.md §4 S3), so
                             // every slot's first push is unchanged; only device and link queues
@@ -400,18 +458,20 @@ eval32_kernel(const EvalParams P) {
                             arrivals(h1.w, f1, g1, zero, r1);   // ks+1's distance-1 producer is ks: none
 #pragma unroll
                             for (int c = 0; c < CPL; c++) fwd[c] = 0u;
-                            begin32<CPL>(h1, v + 1, place, st, r1, x, cc);
+                            place.at(v + 1, (int)(h1.w & kStXMask), x);
+                            begin32<CPL>(h1, st, r1, x, cc);
                             for (int32_t q = 0; q < n1; q++) {
                                 const uint32_t a = sp1 + q * kStepBytes;
                                 edges32<PL, CPL>(cx, lds_u32(a + 12), lds_v4(a + 16), lds_v4(a + 32), x,
-                                                 cc, place, st, fwd);
+                                                 cc, place_y, st, fwd);
                             }
-                            begin32<CPL>(h, v, place, st, r0, x, cc);
-                            edges32<PL, CPL>(cx, h.w, e0, e1, x, cc, place, st, fwd);
+                            place.at(v, (int)(h.w & kStXMask), x);
+                            begin32<CPL>(h, st, r0, x, cc);
+                            edges32<PL, CPL>(cx, h.w, e0, e1, x, cc, place_y, st, fwd);
                             for (int32_t q = 1; q < nk; q++) {
                                 const uint32_t a = sp + q * kStepBytes;
                                 edges32<PL, CPL>(cx, lds_u32(a + 12), lds_v4(a + 16), lds_v4(a + 32), x,
-                                                 cc, place, st, fwd);
+                                                 cc, place_y, st, fwd);
                             }
                             v++;
                             load_next(v + 1, nfar, nnear);
@@ -433,9 +493,22 @@ eval32_kernel(const EvalParams P) {
                         load_next(v + 1, nfar, nnear);
 #pragma unroll
                         for (int c = 0; c < CPL; c++) fwd[c] = 0u;
-                        begin32<CPL>(h, v, place, st, r, x, cc);
+                        if constexpr (MODE == 0) {
+#pragma unroll
+                            for (int c = 0; c < CPL; c++) x[c] = plane_dev<PL>(pwx[c], lane, place.dmax);
+                            pw_load(v + 1, pwx);
+                        } else {
+                            place.at(v, (int)(h.w & kStXMask), x);
+                        }
+                        begin32<CPL>(h, st, r, x, cc);
                     }
-                    edges32<PL, CPL>(cx, h.w, e0, e1, x, cc, place, st, fwd);
+                    if constexpr (MODE == 0) {
+                        edges32<PL, CPL>(cx, h.w, e0, e1, x, cc, pw_y, st, fwd);
+                        pw_load((int32_t)(e0n.y & kSuccPosMask), pwy[0]);
+                        pw_load((int32_t)(e1n.y & kSuccPosMask), pwy[1]);
+                    } else {
+                        edges32<PL, CPL>(cx, h.w, e0, e1, x, cc, place_y, st, fwd);
+                    }
                     sp += kStepBytes;
                     i++;
                     h = hn;

@@ -172,7 +172,7 @@ class Graph:
 
     def __del__(self):
         h = getattr(self, "_h", None)
-        if h:
+        if h and _L is not None:                      # module globals are gone at exit
             _L.pesto_graph_destroy(h)
             self._h = None
 
@@ -247,7 +247,7 @@ class Search:
 
     def __del__(self):
         h = getattr(self, "_h", None)
-        if h:
+        if h and _L is not None:
             _L.pesto_search_destroy(h)
             self._h = None
 

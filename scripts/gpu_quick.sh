@@ -2,4 +2,7 @@ cd $GRAFT_REPO_ROOT
 mkdir -p gpurun_out
 timeout 900 python -m pytest tests -m gpu -x -q > gpurun_out/pytest_gpu.log 2>&1; echo "pytest rc=$?" >> gpurun_out/pytest_gpu.log
 timeout 300 python bench.py --steps 20 --warmup 5 --no-cpu-baseline > gpurun_out/bench.log 2>&1
-timeout 300 python bench.py --config transformer_2dev --steps 5 --warmup 3 --no-cpu-baseline --no-e2e > gpurun_out/bench_transformer_2dev.log 2>&1
+timeout 300 python scripts/time_explicit.py inception_v3_2dev > gpurun_out/texp.log 2>&1
+for c in ${CONFIGS:-transformer_2dev}; do
+timeout 300 python bench.py --config $c --steps 5 --warmup 3 --no-cpu-baseline --no-e2e > gpurun_out/bench_$c.log 2>&1
+done
