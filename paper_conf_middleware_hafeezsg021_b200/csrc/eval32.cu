@@ -426,8 +426,18 @@ eval32_kernel(const EvalParams P) {
                     pw_load((int32_t)(e1.y & kSuccPosMask), pwy[1]);
                 }
                 while (i < nsteps) {
-                    // the next step's records (past the tile's end: padding, never used)
-                    const uint4 hn = lds_v4(sp + 48), e0n = lds_v4(sp + 64), e1n = lds_v4(sp + 80);
+                    // the next step's head (past the tile's end: padding, never used); the edge
+                    // records are read here for this step (search: their first use is after the
+                    // head's work) or one step ahead (rows: they address the plane words)
+                    const uint4 hn = lds_v4(sp + 48);
+                    uint4 e0n = e0, e1n = e1;
+                    if constexpr (MODE == 0) {
+                        e0n = lds_v4(sp + 64);
+                        e1n = lds_v4(sp + 80);
+                    } else {
+                        e0 = lds_v4(sp + 16);
+                        e1 = lds_v4(sp + 32);
+                    }
                     if (!(h.w & kStCont)) {
                         v++;
                         if (MODE == 1 && v == ks) {
@@ -512,8 +522,10 @@ eval32_kernel(const EvalParams P) {
                     sp += kStepBytes;
                     i++;
                     h = hn;
-                    e0 = e0n;
-                    e1 = e1n;
+                    if constexpr (MODE == 0) {
+                        e0 = e0n;
+                        e1 = e1n;
+                    }
                 }
             }
             __syncwarp();

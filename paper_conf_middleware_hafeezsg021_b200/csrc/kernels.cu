@@ -488,15 +488,16 @@ __global__ void __launch_bounds__(256) transpose_kernel(const TransposeParams P)
 }
 
 // ---------------------------------------------------------------------------------------------
-// K4: commit the winner of every base (one thread per base)
+// K4: commit the winner of every base (one warp per base: the lanes share the move's positions)
 // ---------------------------------------------------------------------------------------------
 template <int PL>
-__device__ void set_dev_at(uint32_t *bits, int words, int32_t q, int x) {
+__device__ void set_dev_at(uint32_t *bits, int words, int32_t q, int x) {   // lanes may share words
 #pragma unroll
     for (int k = 0; k < PL; k++) {
         uint32_t *w = bits + k * words + (q >> 5);
         const uint32_t m = 1u << (q & 31);
-        *w = ((x >> k) & 1) ? (*w | m) : (*w & ~m);
+        if ((x >> k) & 1) atomicOr(w, m);
+        else atomicAnd(w, ~m);
     }
 }
 template <int PL>
@@ -509,27 +510,33 @@ __device__ int get_dev_at(const uint32_t *bits, int words, int32_t q) {
 
 template <int PL>
 __global__ void commit_kernel(const CommitParams P) {
-    const int b = threadIdx.x;
-    if (b >= P.P) return;
+    const int b = blockIdx.x, lane = threadIdx.x;
     const uint64_t key = P.keys[b];
-    P.swap_out[b] = -1;
-    if (key == ~0ull) return;
-    P.base_mk[b] = (int64_t)(key >> 24);
+    if (key == ~0ull) {
+        if (lane == 0) P.swap_out[b] = -1;
+        return;
+    }
     const int64_t j = (int64_t)(key & ((1ull << 24) - 1));
-    if (j == 0) return;
     const BaseLayoutDev &B = P.bases[b];
     uint32_t *bits = P.bits + (size_t)b * PL * P.words;
     const uint64_t cb = ctr_base_of(P.step, P.P, b);
     const uint8_t *adj = B.swap_blocked;
     const Region rg = decode_region(P.seed, cb, j >> kGroupShift, P.n);
-    const int32_t ks = decode_swap(P.seed, cb, j >> kGroupShift, P.n, P.mix[3], rg,
-                                   [&](int32_t k) { return adj[k] != 0; });
+    const int32_t ks = j == 0 ? -1
+                              : decode_swap(P.seed, cb, j >> kGroupShift, P.n, P.mix[3], rg,
+                                            [&](int32_t k) { return adj[k] != 0; });
     const int words = P.words;
-    const LaneMove mv = decode_lane(
-        P.seed, cb, j, ks >= 0 && (j & (kGroup - 1)) == 0, P.D, P.mix, rg,
-        [&](int32_t q) { return B.order[q]; },
-        [&](int32_t q) { return get_dev_at<PL>(bits, words, q); },
-        [&](int32_t op) { return (unsigned)P.allowed_op[op]; });
+    const LaneMove mv = j == 0 ? no_move()
+        : decode_lane(P.seed, cb, j, ks >= 0 && (j & (kGroup - 1)) == 0, P.D, P.mix, rg,
+                      [&](int32_t q) { return B.order[q]; },
+                      [&](int32_t q) { return get_dev_at<PL>(bits, words, q); },
+                      [&](int32_t op) { return (unsigned)P.allowed_op[op]; });
+    __syncwarp();                       // every lane decoded from the unmodified base
+    if (lane == 0) {
+        P.base_mk[b] = (int64_t)(key >> 24);
+        P.swap_out[b] = ks;
+    }
+    if (j == 0) return;
     // the base code is also embedded in the eval32 records that name position q: the op's
     // own record and every edge record whose successor sits at q
     uint8_t *blob32 = const_cast<uint8_t *>(B.blob32);
@@ -547,16 +554,22 @@ __global__ void commit_kernel(const CommitParams P) {
         }
     };
     if (mv.kind == kMoveFlip) {
-        for (int f = 0; f < mv.nflip; f++) set_dev(mv.fpos[f], mv.fdev[f]);
+        // flips apply in sequence; a position flipped twice keeps its last device
+        if (lane < mv.nflip) {
+            bool last = true;
+            for (int f = lane + 1; f < mv.nflip; f++) last = last && mv.fpos[f] != mv.fpos[lane];
+            if (last) set_dev(mv.fpos[lane], mv.fdev[lane]);
+        }
     } else if (mv.kind == kMoveWindow) {
-        for (int32_t q = mv.ws; q < mv.ws + mv.wl; q++)
+        for (int32_t q = mv.ws + lane; q < mv.ws + mv.wl; q += 32)
             if ((B.allowed_pos[q] >> mv.wd) & 1u) set_dev(q, mv.wd);
     }
-    if (ks >= 0) {                       // ops at ks and ks+1 exchange positions
+    __threadfence();                     // every lane's bit updates are performed ...
+    __syncwarp();                        // ... before lane 0 reads the planes for the swap
+    if (ks >= 0 && lane == 0) {          // ops at ks and ks+1 exchange positions
         const int a = get_dev_at<PL>(bits, words, ks), c = get_dev_at<PL>(bits, words, ks + 1);
         set_dev_at<PL>(bits, words, ks, c);
         set_dev_at<PL>(bits, words, ks + 1, a);
-        P.swap_out[b] = ks;
     }
 }
 
@@ -678,10 +691,9 @@ cudaError_t launch_patch(const PatchOp *ops_dev, int n_ops, int max_block, cudaS
 
 cudaError_t launch_commit(const CommitParams &p, cudaStream_t st) {
     note_launch();
-    const int threads = ((p.P + 31) / 32) * 32;
-    if (p.planes == 1) commit_kernel<1><<<1, threads, 0, st>>>(p);
-    else if (p.planes == 2) commit_kernel<2><<<1, threads, 0, st>>>(p);
-    else commit_kernel<4><<<1, threads, 0, st>>>(p);
+    if (p.planes == 1) commit_kernel<1><<<p.P, 32, 0, st>>>(p);
+    else if (p.planes == 2) commit_kernel<2><<<p.P, 32, 0, st>>>(p);
+    else commit_kernel<4><<<p.P, 32, 0, st>>>(p);
     return cudaGetLastError();
 }
 
