@@ -128,8 +128,8 @@ pesto_status pesto_seed_placement(pesto_graph *g, int32_t kind, const int32_t *o
 /* ------------------------------------------------------------------------------------------ */
 /* Makespan of n_cand candidates sharing one schedule order pi.
  *   order:      HOST [n_ops] topological order (layout cached by content).
- *   placements: DEVICE, n_cand rows; row c holds op i's device code in bits [b*i, b*i+b) of the
- *               row (little-endian bytes), b = 1 (D<=2), 2 (D<=4), 4 (D<=8).
+ *   placements: DEVICE, 16-byte aligned, n_cand rows; row c holds op i's device code in bits
+ *               [b*i, b*i+b) of the row (little-endian bytes), b = 1 (D<=2), 2 (D<=4), 4 (D<=8).
  *   row_stride_bytes: >= ceil(n_ops*b/8), a multiple of 16.
  *   makespans:  DEVICE [n_cand] int64 out; INT64_MAX for an infeasible row.
  * Enqueued on cuda_stream; returns without synchronising.  Errors: EINVAL, ENOTTOPO, ESTATE

@@ -112,6 +112,7 @@ struct PatchOp {
     uint32_t pad;
 };
 constexpr int kPatchMaxBlock = 48 * 1024;      // rotation bytes a + b (shared-memory staging)
+constexpr int kTransposeSmemMax = 200 * 1024;  // K5 smem variant: a group's n*planes words
 
 // launchers (kernels.cu / eval32.cu); they return the launch error, if any.
 cudaError_t launch_patch(const PatchOp *ops_dev, int n_ops, int max_block, cudaStream_t st);

@@ -487,6 +487,82 @@ __global__ void __launch_bounds__(256) transpose_kernel(const TransposeParams P)
     }
 }
 
+// K5, shared-memory variant: one CTA per 32-row group.  The rows are read once with 16-byte
+// loads (a row's sectors are reused from L1 by the following loads), the permutation to
+// position order is applied in shared memory, and the group's n*PL words leave with coalesced
+// stores -- the global-scatter variant above wrote 4 bytes per 32-byte sector.
+template <int PL>
+__global__ void __launch_bounds__(256) transpose_smem_kernel(const TransposeParams P) {
+    extern __shared__ uint4 tsm[];
+    uint32_t *out_s = reinterpret_cast<uint32_t *>(tsm);
+    __shared__ uint32_t bad_s;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const int n16 = (P.n * PL + 127) / 128;             // 16-byte chunks of a row
+    const int nw = P.n * PL;                            // output words of a group
+    for (int64_t g = blockIdx.x; g < P.n_groups; g += gridDim.x) {
+        if (threadIdx.x == 0) bad_s = 0;
+        const int64_t row = g * 32 + lane;
+        const bool have = row < P.n_cand;
+        const uint4 *rp = reinterpret_cast<const uint4 *>(P.rows + row * P.stride);
+        uint32_t bad = 0;
+        auto emit = [&](int c, uint32_t (&pw)[PL]) {   // chunk c = ops [32c, 32c + 32)
+#pragma unroll
+            for (int k = 0; k < PL; k++) pw[k] = transpose32(pw[k], lane);
+            const int op = c * 32 + lane;
+            if (op >= P.n) return;
+            const unsigned fm = __ldg(P.fmask + op);
+            if (fm) {
+                for (int code = 0; code < (1 << PL); code++) {
+                    if (!((fm >> code) & 1u)) continue;
+                    uint32_t match = 0xffffffffu;
+#pragma unroll
+                    for (int k = 0; k < PL; k++) match &= ((code >> k) & 1) ? pw[k] : ~pw[k];
+                    bad |= match;
+                }
+            }
+            const int q = __ldg(P.pos_of + op);
+#pragma unroll
+            for (int k = 0; k < PL; k++) out_s[q * PL + k] = pw[k];
+        };
+        __syncthreads();
+        for (int k16 = warp; k16 < n16; k16 += 8) {
+            const uint4 w = have ? __ldg(rp + k16) : make_uint4(0, 0, 0, 0);
+            if (PL == 1) {
+                const uint32_t ws[4] = {w.x, w.y, w.z, w.w};
+#pragma unroll
+                for (int j = 0; j < 4; j++) {
+                    uint32_t pw[PL];
+                    pw[0] = ws[j];
+                    emit(4 * k16 + j, pw);
+                }
+            } else if (PL == 2) {
+                const uint32_t ws[4] = {w.x, w.y, w.z, w.w};
+#pragma unroll
+                for (int j = 0; j < 2; j++) {
+                    uint32_t pw[PL];
+                    const uint32_t lo = ws[2 * j], hi = ws[2 * j + 1];
+                    pw[0] = compress2(lo) | (compress2(hi) << 16);
+                    pw[1] = compress2(lo >> 1) | (compress2(hi >> 1) << 16);
+                    emit(2 * k16 + j, pw);
+                }
+            } else {
+                uint32_t pw[PL];
+#pragma unroll
+                for (int k = 0; k < PL; k++)
+                    pw[k] = compress4(w.x >> k) | (compress4(w.y >> k) << 8) |
+                            (compress4(w.z >> k) << 16) | (compress4(w.w >> k) << 24);
+                emit(k16, pw);
+            }
+        }
+        bad = __reduce_or_sync(0xffffffffu, bad);
+        if (lane == 0 && bad) atomicOr(&bad_s, bad);
+        __syncthreads();
+        uint32_t *dst = P.planes_out + (size_t)g * nw;
+        for (int i = threadIdx.x; i < nw; i += blockDim.x) dst[i] = out_s[i];
+        if (threadIdx.x == 0) P.invalid_out[g] = bad_s;
+    }
+}
+
 // ---------------------------------------------------------------------------------------------
 // K4: commit the winner of every base (one warp per base: the lanes share the move's positions)
 // ---------------------------------------------------------------------------------------------
@@ -647,9 +723,25 @@ cudaError_t launch_transpose(const TransposeParams &p, cudaStream_t st) {
     int dev = 0, sms = 148;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    if (p.n_groups <= 0) return cudaSuccess;
+    const size_t smem = (size_t)p.n * p.planes * 4;
+    if (smem <= (size_t)kTransposeSmemMax) {          // one CTA per group, output staged in smem
+        auto set = [&](const void *f) {
+            return cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        };
+        cudaError_t e = p.planes == 1 ? set((const void *)transpose_smem_kernel<1>)
+                      : p.planes == 2 ? set((const void *)transpose_smem_kernel<2>)
+                                      : set((const void *)transpose_smem_kernel<4>);
+        if (e != cudaSuccess) return e;
+        const int per_sm = std::max(1, (int)(200 * 1024 / std::max<size_t>(smem, 1)));
+        const int grid = (int)std::min<int64_t>(p.n_groups, (int64_t)sms * std::min(per_sm, 8));
+        if (p.planes == 1) transpose_smem_kernel<1><<<grid, 256, smem, st>>>(p);
+        else if (p.planes == 2) transpose_smem_kernel<2><<<grid, 256, smem, st>>>(p);
+        else transpose_smem_kernel<4><<<grid, 256, smem, st>>>(p);
+        return cudaGetLastError();
+    }
     const int64_t blocks_needed = (p.n_groups + 7) / 8;
     const int grid = (int)std::min<int64_t>(blocks_needed, (int64_t)sms * 8);
-    if (grid <= 0) return cudaSuccess;
     if (p.planes == 1) transpose_kernel<1><<<grid, 256, 0, st>>>(p);
     else if (p.planes == 2) transpose_kernel<2><<<grid, 256, 0, st>>>(p);
     else transpose_kernel<4><<<grid, 256, 0, st>>>(p);
