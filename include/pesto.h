@@ -88,6 +88,16 @@ void pesto_graph_destroy(pesto_graph *g);                          /* NULL-safe 
 pesto_status pesto_comm_model(pesto_graph *g, int32_t src_dev, int32_t dst_dev,
                               int64_t beta0_ns, int64_t beta1_fs_per_byte);
 
+/* Link model.  PESTO_LINKS_FCFS (the default, Pesto's model): each
+ * directed link is one serial FCFS queue, a transfer starts at
+ * max(producer completion, link free).  PESTO_LINKS_UNLIMITED: transfers never queue and start
+ * at the producer's completion -- the "unlimited bandwidth" assumption of prior work that
+ * PAPER.md L113 / L200 (Fig. 5) contrasts with.  Applies to every later pesto_eval_batch* and
+ * search step on g; evaluations under PESTO_LINKS_UNLIMITED run on the exact 64-bit kernel
+ * (a modelling variant, not the throughput path).  Errors: EINVAL. */
+typedef enum { PESTO_LINKS_FCFS = 0, PESTO_LINKS_UNLIMITED = 1 } pesto_link_model;
+pesto_status pesto_graph_set_link_model(pesto_graph *g, int32_t model);
+
 typedef struct {
     int32_t n_ops, n_devices;
     int64_t n_edges;

@@ -162,6 +162,7 @@ void fill_eval_common(const pesto_graph *g, EvalParams &p) {
     p.edge_stride = edge_stride_for(g->n_classes);
     p.edge_stride32 = edge_stride32_for(g->n_classes);
     p.n_classes = g->n_classes;
+    p.link_queue = g->link_model == PESTO_LINKS_FCFS ? 1 : 0;
     std::memcpy(p.link_class, g->link_class, 64);
     p.all_allowed = g->all_allowed ? 1 : 0;
 }
@@ -344,6 +345,13 @@ void pesto_graph_destroy(pesto_graph *g) {
     if (!g) return;
     DeviceGuard guard(g->device);
     delete g;
+}
+
+pesto_status pesto_graph_set_link_model(pesto_graph *g, int32_t model) {
+    if (!g) return fail(PESTO_EINVAL, "NULL graph");
+    if (model != PESTO_LINKS_FCFS && model != PESTO_LINKS_UNLIMITED) return fail(PESTO_EINVAL, "unknown link model");
+    g->link_model = model;
+    return PESTO_OK;
 }
 
 pesto_status pesto_comm_model(pesto_graph *g, int32_t a, int32_t b, int64_t beta0,
@@ -556,7 +564,9 @@ pesto_status pesto_eval_batch(pesto_graph *g, const int32_t *order, const void *
     p.tasks_per_base = (n_groups + kWarps - 1) / kWarps;
     p.n_tasks = p.tasks_per_base;
     int grid = 0;
-    if (!g->eligible32 || L->W32 == 0) {                      // 64-bit path for every row
+    // 64-bit path for every row: ineligible durations, no eval32 stream, or congestion-free
+    // links (row f4(ii) is a modelling variant; eval32 carries only the FCFS link queues)
+    if (!g->eligible32 || L->W32 == 0 || g->link_model != PESTO_LINKS_FCFS) {
         if ((s = ensure_state(g, p, 0, p.n_tasks, &grid))) return s;
         p.state = g->d_state.as<int64_t>();
         if ((e = launch_eval(p, 0, grid, st)) != cudaSuccess) return cuda_fail(e, "launch eval");

@@ -105,6 +105,7 @@ struct pesto_graph {
     pesto::DevBuf d_state, d_planes, d_invalid, d_fmask, d_movable, d_allowed, d_bases, d_rows,
         d_out, d_state32, d_flags;        // d_flags: [count | list of saturated candidates]
     int32_t sms = 148;
+    int32_t link_model = 0;               // PESTO_LINKS_FCFS / PESTO_LINKS_UNLIMITED
 };
 
 namespace pesto {

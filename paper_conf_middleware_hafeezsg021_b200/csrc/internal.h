@@ -71,6 +71,8 @@ struct EvalParams {
     int32_t gate;
     // eval32 candidates per lane (1 or 2): more warps vs. more work per warp instruction
     int32_t cpl32;
+    // 1: FCFS link queues; 0: congestion-free links (row f4(ii))
+    int32_t link_queue;
     // eval64 list mode (MODE 2): candidates list[0 .. *list_count)
     const int32_t *list;
     const int32_t *list_count;

@@ -98,6 +98,7 @@ struct Ctx {
     const uint8_t *lclass;       // shared-memory copy of the link-class table
     int edge_stride;
     int D;
+    bool queue;                  // FCFS link queues; false: congestion-free links (f4)
 };
 
 template <bool GLOBAL>
@@ -123,8 +124,8 @@ __device__ __forceinline__ void push_edge(const uint8_t *ep, const uint4 rec, in
                 t = GLOBAL ? (int64_t)__ldg(reinterpret_cast<const long long *>(ext)) : *ext;
             }
         }
-        a = max(c, st.link(x, y)) + t;
-        st.set_link(x, y, a);
+        a = max(c, st.link(x, y)) + t;                       // link state stays 0 if free
+        if (cx.queue) st.set_link(x, y, a);
     }
     int64_t *slot = cx.R + (int64_t)(sl & kEdgeSlotMask) * 32;
     if (ALL_MAX || !(sl & kEdgeFirst)) a = max(a, *slot);
@@ -269,6 +270,7 @@ eval_kernel(const EvalParams P) {
     cx.lclass = lclass;
     cx.edge_stride = P.edge_stride;
     cx.D = P.D;
+    cx.queue = P.link_queue != 0;
     cx.R = P.state + ((int64_t)(blockIdx.x * kWarps + warp) * P.max_W) * 32 + lane;
 
     using StateT = typename std::conditional<PL == 1, RegState, SmemState>::type;

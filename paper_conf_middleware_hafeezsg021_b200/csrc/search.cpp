@@ -139,7 +139,8 @@ pesto_status launch_search_eval(pesto_search *s, int b_first, int n_bases, int64
     int grid = 0;
     pesto_status rc;
     cudaError_t e;
-    const bool use32 = fast && s->use32 && keys_dbg == nullptr;
+    const bool use32 = fast && s->use32 && keys_dbg == nullptr &&
+                       g->link_model == PESTO_LINKS_FCFS;   // f4(ii) runs on eval64
     if (use32) {
         // eval32 tasks: 256 consecutive ids starting at a multiple of 256
         EvalParams p32 = p;

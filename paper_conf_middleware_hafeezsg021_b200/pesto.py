@@ -19,6 +19,7 @@ OK, EINVAL, ECYCLE, ENOTTOPO, EOVERFLOW, ENOMEM, ECUDA, ENCCL, ESTATE = range(9)
 INFEASIBLE = (1 << 63) - 1
 KEY_INVALID = (1 << 64) - 1
 ORDER_CRITICAL_PATH, ORDER_FIFO, ORDER_RANDOM = 0, 1, 2
+LINKS_FCFS, LINKS_UNLIMITED = 0, 1
 PLACE_SINGLE, PLACE_EXPERT, PLACE_TOPO_SPLIT, PLACE_RANDOM = 0, 1, 2, 3
 
 
@@ -58,6 +59,7 @@ SIGNATURES = {
     "pesto_graph_create": (_I32, [C.POINTER(GraphDesc), C.POINTER(_VP)]),
     "pesto_graph_destroy": (None, [_VP]),
     "pesto_comm_model": (_I32, [_VP, _I32, _I32, _I64, _I64]),
+    "pesto_graph_set_link_model": (_I32, [_VP, _I32]),
     "pesto_graph_stats_for": (_I32, [_VP, _VP, C.POINTER(GraphStats)]),
     "pesto_seed_order": (_I32, [_VP, _I32, _U64, _VP]),
     "pesto_seed_placement": (_I32, [_VP, _I32, _VP, _VP, _U64, _VP]),
@@ -182,6 +184,10 @@ class Graph:
 
     def comm_model(self, src_dev: int, dst_dev: int, beta0_ns: int, beta1_fs_per_byte: int):
         _check(_L.pesto_comm_model(self._h, src_dev, dst_dev, beta0_ns, beta1_fs_per_byte))
+
+    def set_link_model(self, model: int):
+        """LINKS_FCFS (default; serial FCFS queue per directed link) or LINKS_UNLIMITED."""
+        _check(_L.pesto_graph_set_link_model(self._h, model))
 
     def stats(self, order) -> dict:
         o = np.ascontiguousarray(order, dtype=np.int32)

@@ -234,6 +234,44 @@ def test_committed_swaps_patch_layouts(P, O, D, mix, steps):
         assert (gk == ok).all(), (b, np.nonzero(gk != ok)[0][:5])
 
 
+@pytest.mark.parametrize("seed,n,D,kw", [(91, 700, 2, {}), (92, 500, 4, {"hetero_links": True}),
+                                          (93, 2500, 2, {"fan_out_hub": 300})])
+def test_congestion_free_links_match_oracle(P, O, seed, n, D, kw):
+    """row f4(ii): PESTO_LINKS_UNLIMITED vs the oracle's congestion-free simulator (W2 pin)."""
+    g = dag.random_dag(seed, n, 1.5, D=D, p_max=5000, max_bytes=400_000, beta0=700,
+                       beta1_fs=30_000, **kw)
+    G = P.Graph.from_arrays(g)
+    G.set_link_model(P.LINKS_UNLIMITED)
+    order = dag.random_topo_order(g, seed)
+    x = dag.random_placements(g, seed + 1, 300)
+    gpu = _gpu_eval(P, G, g, order, x)
+    ref = np.asarray([O.makespan_nocongest(g, x[i], order) for i in range(len(x))], np.int64)
+    assert (gpu == ref).all(), np.nonzero(gpu != ref)[0][:5]
+    fcfs, _ = O.makespan_batch(g, x, order)
+    assert (ref <= fcfs).all() and (ref < fcfs).any()        # queues only ever delay
+    G.set_link_model(P.LINKS_FCFS)
+    assert (_gpu_eval(P, G, g, order, x) == fcfs).all()
+
+
+def test_congestion_free_search_keys(P, O):
+    """the search kernels under PESTO_LINKS_UNLIMITED: every key of a step (eval32 argmin and
+    the eval64 per-candidate keys) equals the oracle's decode + congestion-free makespan."""
+    g = _search_graph(seed=95, n=160)
+    G = P.Graph.from_arrays(g)
+    G.set_link_model(P.LINKS_UNLIMITED)
+    xs, orders = _bases(g, 2, seed=9)
+    K = 700
+    S = P.Search(G, xs, orders, K, MIX, seed=12)
+    keys = np.empty((2, K), np.uint64)
+    for b in range(2):
+        for j in range(K):
+            ok, x, o = O.candidate(g, 2, b, xs, orders, j, 12, 0, MIX)
+            keys[b, j] = ((O.makespan_nocongest(g, x, o) << 24) | j) if ok else (1 << 64) - 1
+        assert (S.candidate_keys(b, 0, K) == keys[b]).all(), b
+    S.eval()
+    assert (S.keys() == keys.min(axis=1)).all()
+
+
 def test_fake_sharding_equals_single_rank(P, O):
     """W rank ranges evaluated one after another on one GPU, minima reduced on the host."""
     g = _search_graph(seed=41, n=90)
