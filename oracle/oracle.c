@@ -119,12 +119,89 @@ static int64_t check_order(int32_t n, int64_t m, const int32_t *src, const int32
 }
 
 /* a placement is feasible iff every op sits on an existing device its mask allows (Q16) */
+/* ------------------------------------------------------------------------------------- */
+/* row f3: memory footprint per device (L202) and colocation groups (L175)                 */
+/* ------------------------------------------------------------------------------------- */
+static struct {
+    int active;
+    int32_t n, D;
+    int64_t *mem;        /* [n] footprint of each op */
+    int64_t *cap;        /* [D] or NULL */
+    int32_t *coloc;      /* [n] or NULL */
+} g_cons;
+
+void oracle_clear_constraints(void) {
+    free(g_cons.mem);
+    free(g_cons.cap);
+    free(g_cons.coloc);
+    memset(&g_cons, 0, sizeof g_cons);
+}
+
+int oracle_set_constraints(int32_t n, int64_t m, const int32_t *src, const int32_t *dst,
+                           const int64_t *bytes, int32_t D, const int64_t *mem,
+                           const int64_t *cap, const int32_t *coloc) {
+    oracle_clear_constraints();
+    if (n < 1 || m < 0 || D < 1 || D > 8) return ORACLE_EINVAL;
+    g_cons.mem = calloc((size_t)n, sizeof(int64_t));
+    if (!g_cons.mem) return ORACLE_ENOMEM;
+    if (mem) {
+        for (int32_t v = 0; v < n; v++) {
+            if (mem[v] < 0) { oracle_clear_constraints(); return ORACLE_EINVAL; }
+            g_cons.mem[v] = mem[v];
+        }
+    } else {                                 /* L202: input + output tensor sizes of the op */
+        for (int64_t e = 0; e < m; e++) {
+            g_cons.mem[src[e]] += bytes[e];
+            g_cons.mem[dst[e]] += bytes[e];
+        }
+    }
+    if (cap) {
+        g_cons.cap = malloc((size_t)D * sizeof(int64_t));
+        for (int32_t d = 0; d < D; d++) g_cons.cap[d] = cap[d];
+    }
+    if (coloc) {
+        g_cons.coloc = malloc((size_t)n * sizeof(int32_t));
+        for (int32_t v = 0; v < n; v++) {
+            if (coloc[v] < -1 || coloc[v] >= n) { oracle_clear_constraints(); return ORACLE_EINVAL; }
+            g_cons.coloc[v] = coloc[v];
+        }
+    }
+    g_cons.n = n;
+    g_cons.D = D;
+    g_cons.active = 1;
+    return 0;
+}
+
+int oracle_constraints_ok(int32_t n, const uint8_t *x) {
+    if (!g_cons.active || n != g_cons.n) return 1;
+    if (g_cons.cap) {                        /* footprint of the ops on each device <= cap */
+        int64_t F[8] = {0};
+        for (int32_t v = 0; v < n; v++) F[x[v]] += g_cons.mem[v];
+        for (int32_t d = 0; d < g_cons.D; d++)
+            if (F[d] > g_cons.cap[d]) return 0;
+    }
+    if (g_cons.coloc) {                      /* every op of a group on one device */
+        int32_t *dev = malloc((size_t)n * sizeof(int32_t));
+        int ok = 1;
+        for (int32_t v = 0; v < n; v++) dev[v] = -1;
+        for (int32_t v = 0; v < n && ok; v++) {
+            const int32_t grp = g_cons.coloc[v];
+            if (grp < 0) continue;
+            if (dev[grp] < 0) dev[grp] = x[v];
+            else if (dev[grp] != x[v]) ok = 0;
+        }
+        free(dev);
+        if (!ok) return 0;
+    }
+    return 1;
+}
+
 static int feasible(int32_t n, int32_t D, const uint8_t *allowed, const uint8_t *x) {
     for (int32_t v = 0; v < n; v++) {
         if (x[v] >= D) return 0;
         if (!allowed_dev(allowed, v, x[v])) return 0;
     }
-    return 1;
+    return oracle_constraints_ok(n, x);
 }
 
 /* ------------------------------------------------------------------------------------- */

@@ -66,6 +66,23 @@ int64_t oracle_makespan_nocongest(int32_t n, const int64_t *p, int64_t m, const 
                                   const uint8_t *allowed, const uint8_t *x,
                                   const int32_t *order);
 
+/* Feasibility constraints, row f3 (PAPER.md L202 memory, L175 colocation).  While set, every
+ * makespan / key function of this library treats a placement that violates them as infeasible
+ * (INT64_MAX, key UINT64_MAX).  For the graph (n, m, src, dst, bytes, D):
+ *   mem  [n] footprint of each op in bytes; NULL: the sum of its input and output tensor sizes
+ *        (L202), i.e. the bytes of every edge into or out of the op;
+ *   cap  [D] per-device cap on the summed footprint of the ops placed there; NULL: none;
+ *   coloc[n] colocation group of each op in [0, n), -1 = none (L175: x equal within a group);
+ *        NULL: none.
+ * Global state (test infrastructure, not thread-safe against concurrent set/clear); applies
+ * only to calls with the same n.  Returns 0 or ORACLE_EINVAL. */
+int oracle_set_constraints(int32_t n, int64_t m, const int32_t *src, const int32_t *dst,
+                           const int64_t *bytes, int32_t D, const int64_t *mem,
+                           const int64_t *cap, const int32_t *coloc);
+void oracle_clear_constraints(void);
+/* 1 if x satisfies the constraints set (or none are set), else 0. */
+int oracle_constraints_ok(int32_t n, const uint8_t *x);
+
 /* Batch: out[c] = oracle_makespan(x + c*n, order) for c < count, `threads` pthreads
  * (threads <= 0: 1).  Returns wall seconds, or a negative error code. */
 double oracle_makespan_batch(int32_t n, const int64_t *p, int64_t m, const int32_t *src,

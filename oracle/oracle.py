@@ -76,6 +76,13 @@ def lib():
                                              C.c_uint64, C.c_uint64, _i32p, C.c_int32,
                                              C.c_int32, _u64p]
         L.oracle_search_step.restype = C.c_int
+        L.oracle_set_constraints.argtypes = [C.c_int32, C.c_int64, _i32p, _i32p, _i64p,
+                                             C.c_int32, C.c_void_p, C.c_void_p, C.c_void_p]
+        L.oracle_set_constraints.restype = C.c_int
+        L.oracle_clear_constraints.argtypes = []
+        L.oracle_clear_constraints.restype = None
+        L.oracle_constraints_ok.argtypes = [C.c_int32, _u8p]
+        L.oracle_constraints_ok.restype = C.c_int
         _LIB = L
     return _LIB
 
@@ -117,6 +124,35 @@ def longest_path(g, x, order) -> int:
     a, keep = _g(g)
     return int(lib().oracle_longest_path(*a, np.ascontiguousarray(x, dtype=np.uint8),
                                          np.ascontiguousarray(order, dtype=np.int32)))
+
+
+class constraints:
+    """Row f3 feasibility constraints (L202 memory, L175 colocation), active inside `with`.
+
+    mem: [n] op footprints or None (= input + output tensor bytes); cap: [D] or None;
+    coloc: [n] group ids (-1 none) or None."""
+
+    def __init__(self, g, mem=None, cap=None, coloc=None):
+        self.g = g
+        self.arrs = [None if a is None else np.ascontiguousarray(a, dt)
+                     for a, dt in ((mem, np.int64), (cap, np.int64), (coloc, np.int32))]
+
+    def __enter__(self):
+        g = self.g
+        rc = lib().oracle_set_constraints(int(g.n), int(len(g.src)),
+                                          np.ascontiguousarray(g.src, np.int32),
+                                          np.ascontiguousarray(g.dst, np.int32),
+                                          np.ascontiguousarray(g.nbytes, np.int64), int(g.D),
+                                          *[None if a is None else a.ctypes.data for a in self.arrs])
+        if rc != 0:
+            raise ValueError(f"oracle_set_constraints: {rc}")
+        return self
+
+    def __exit__(self, *a):
+        lib().oracle_clear_constraints()
+
+    def ok(self, x) -> bool:
+        return bool(lib().oracle_constraints_ok(int(self.g.n), np.ascontiguousarray(x, np.uint8)))
 
 
 def makespan_nocongest(g, x, order) -> int:

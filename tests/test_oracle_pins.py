@@ -392,3 +392,74 @@ def test_error_codes(O):
     allowed = dag.make_graph("aff", [1, 1], [(0, 1)], [1], D=2, beta0=1, allowed=[1, 2])
     assert O.makespan(allowed, [1, 1], [0, 1]) == O.INFEASIBLE
     assert O.makespan(allowed, [0, 1], [0, 1]) == 3
+
+
+# ---------------------------------------------------------------------------------------
+# Row f3: memory footprint and colocation (L175) constraints
+# ---------------------------------------------------------------------------------------
+def _f3_graph():
+    # a -> b carries 100 B, a -> c 50 B; footprints (input + output tensors, L202):
+    # a = 150, b = 100, c = 50 (hand-computed)
+    return dag.make_graph("f3", [1, 1, 1], [(0, 1), (0, 2)], [100, 50], D=2, beta0=3,
+                          beta1_fs=0)
+
+
+def test_f3_memory_caps_worked_example(O):
+    """cap 200 B per device: feasible placements (x_a x_b x_c) are exactly 010, 011, 100, 101
+    (hand-computed: e.g. 000 puts 300 B on device 0, 110 puts 250 B on device 1)."""
+    g = _f3_graph()
+    order = np.asarray([0, 1, 2], np.int32)
+    feasible = {"010", "011", "100", "101"}
+    with O.constraints(g, cap=[200, 200]) as c:
+        for bits in itertools.product([0, 1], repeat=3):
+            x = np.asarray(bits, np.uint8)
+            key = "".join(map(str, bits))
+            assert c.ok(x) == (key in feasible), key
+            mk = O.makespan(g, x, order)
+            assert (mk == INF) == (key not in feasible), key
+    # the constraint is off again outside the block
+    assert O.makespan(g, np.zeros(3, np.uint8), order) == 3
+
+
+def test_f3_explicit_footprints_and_colocation(O):
+    g = _f3_graph()
+    order = np.asarray([0, 1, 2], np.int32)
+    # explicit footprints: a = 10, b = 10, c = 100; cap [100, 1000]: c may not join a or b on 0
+    with O.constraints(g, mem=[10, 10, 100], cap=[100, 1000]) as c:
+        assert c.ok(np.asarray([0, 0, 1], np.uint8)) and not c.ok(np.asarray([1, 0, 0], np.uint8))
+    # colocation {a, c}: x_a == x_c (L175)
+    with O.constraints(g, coloc=[2, -1, 2]) as c:
+        for bits in itertools.product([0, 1], repeat=3):
+            x = np.asarray(bits, np.uint8)
+            assert c.ok(x) == (bits[0] == bits[2])
+            assert (O.makespan(g, x, order) == INF) == (bits[0] != bits[2])
+
+
+def test_f3_search_respects_constraints(O):
+    """the reference search never commits an infeasible candidate and its keys mark them."""
+    g = dag.random_dag(77, 60, 1.5, D=2, p_max=3000, max_bytes=200_000, beta0=500,
+                       beta1_fs=25_000)
+    mem = np.zeros(g.n, np.int64)
+    np.add.at(mem, g.src, g.nbytes)
+    np.add.at(mem, g.dst, g.nbytes)
+    cap = [int(mem.sum() * 0.6)] * 2
+    coloc = np.full(g.n, -1, np.int32)
+    coloc[[3, 9, 17]] = 4
+    x0 = (np.arange(g.n) % 2).astype(np.uint8)
+    x0[[3, 9, 17]] = 1
+    orders = np.stack([dag.random_topo_order(g, 1)]).astype(np.int32)
+    with O.constraints(g, cap=cap, coloc=coloc) as c:
+        assert c.ok(x0)
+        xs = x0[None].copy()
+        mk = np.asarray([O.makespan(g, xs[0], orders[0])], np.int64)
+        keys = O.candidate_keys(g, 1, 0, xs, orders, 0, 600, 5, 0, (50, 20, 20, 10))
+        n_bad = 0
+        for j in range(600):
+            ok, x, o = O.candidate(g, 1, 0, xs, orders, j, 5, 0, (50, 20, 20, 10))
+            if ok and not c.ok(x):
+                assert keys[j] == (1 << 64) - 1
+                n_bad += 1
+        assert n_bad > 0
+        for step in range(3):
+            O.search_step(g, xs, orders, mk, 600, 5, step, (50, 20, 20, 10))
+            assert c.ok(xs[0])
