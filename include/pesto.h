@@ -98,6 +98,21 @@ pesto_status pesto_comm_model(pesto_graph *g, int32_t src_dev, int32_t dst_dev,
 typedef enum { PESTO_LINKS_FCFS = 0, PESTO_LINKS_UNLIMITED = 1 } pesto_link_model;
 pesto_status pesto_graph_set_link_model(pesto_graph *g, int32_t model);
 
+/* Feasibility constraints: per-device memory footprint and
+ * colocation groups (L175).  A candidate violating one is infeasible: makespan INT64_MAX,
+ * search key UINT64_MAX.  All arrays HOST, copied:
+ *   mem_bytes:  [n_ops] footprint of each op, >= 0; NULL = the sum of its input and output
+ *               tensor bytes (every edge into or out of the op, L202);
+ *   cap_bytes:  [n_devices] cap on the summed footprint of the ops on each device, >= 0;
+ *               NULL = no memory constraint;
+ *   coloc:      [n_ops] colocation group of each op in [0, n_ops), -1 = none; ops of one
+ *               group must share a device; NULL = no colocation.
+ * Both NULL (cap_bytes and coloc) clears the constraints.  Search bases must satisfy them
+ * (pesto_search_create fails with EINVAL otherwise; a later change is checked at the next
+ * step: ESTATE).  Errors: EINVAL. */
+pesto_status pesto_graph_set_constraints(pesto_graph *g, const int64_t *mem_bytes,
+                                         const int64_t *cap_bytes, const int32_t *coloc);
+
 typedef struct {
     int32_t n_ops, n_devices;
     int64_t n_edges;

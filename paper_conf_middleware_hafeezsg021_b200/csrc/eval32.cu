@@ -21,6 +21,7 @@
 #include <type_traits>
 
 #include "device_common.cuh"
+#include "feasibility.cuh"
 #include "internal.h"
 
 namespace pesto {
@@ -379,6 +380,10 @@ eval32_kernel(const EvalParams P) {
                     : no_move();
                 valid[c] = in_range && place.mv[c].kind != kMoveInvalid;
                 if (place.mv[c].kind == kMoveInvalid) place.mv[c] = no_move();
+                if (valid[c] && (P.feas.has_cap || P.feas.has_coloc))   // row f3
+                    valid[c] = move_feasible<PL>(place.mv[c], rg, P.D, bits, words, ord,
+                                                 B->allowed_pos, P.all_allowed, P.feas,
+                                                 P.feas.fbase + (size_t)bl * 8);
             }
         }
         st.init();

@@ -163,6 +163,7 @@ void fill_eval_common(const pesto_graph *g, EvalParams &p) {
     p.edge_stride32 = edge_stride32_for(g->n_classes);
     p.n_classes = g->n_classes;
     p.link_queue = g->link_model == PESTO_LINKS_FCFS ? 1 : 0;
+    p.feas = feasibility_view(g);
     std::memcpy(p.link_class, g->link_class, 64);
     p.all_allowed = g->all_allowed ? 1 : 0;
 }
@@ -204,6 +205,40 @@ pesto_status ensure_state32(pesto_graph *g, const EvalParams &p, int search_mode
     if (e != cudaSuccess) return cuda_fail(e, "allocate cold slot state");
     *grid_out = (int)grid;
     return PESTO_OK;
+}
+
+Feasibility feasibility_view(const pesto_graph *g) {
+    Feasibility f{};
+    f.has_cap = g->has_cap ? 1 : 0;
+    f.has_coloc = g->has_coloc ? 1 : 0;
+    if (!f.has_cap && !f.has_coloc) return f;
+    f.mem = g->d_mem.as<int64_t>();
+    f.cap = g->d_cap.as<int64_t>();
+    f.coloc = g->d_coloc.as<int32_t>();
+    f.coloc_size = g->d_coloc_size.as<int32_t>();
+    f.coloc_pairs = g->d_coloc_pairs.as<int2>();
+    f.n_pairs = (int32_t)g->coloc_pairs.size();
+    return f;
+}
+
+bool placement_feasible(const pesto_graph *g, const uint8_t *x, int64_t *footprint8) {
+    int64_t F[8] = {0};
+    for (int32_t v = 0; v < g->n; v++)
+        if (!g->mem.empty()) F[x[v] & 7] += g->mem[v];
+    if (footprint8) std::copy(F, F + 8, footprint8);
+    if (g->has_cap)
+        for (int d = 0; d < g->D; d++)
+            if (F[d] > g->cap[d]) return false;
+    if (g->has_coloc) {
+        std::vector<int32_t> dev(g->n, -1);
+        for (int32_t v = 0; v < g->n; v++) {
+            const int32_t c = g->coloc[v];
+            if (c < 0) continue;
+            if (dev[c] < 0) dev[c] = x[v];
+            else if (dev[c] != x[v]) return false;
+        }
+    }
+    return true;
 }
 
 static uint64_t splitmix_next(uint64_t &s) {
@@ -345,6 +380,58 @@ void pesto_graph_destroy(pesto_graph *g) {
     if (!g) return;
     DeviceGuard guard(g->device);
     delete g;
+}
+
+pesto_status pesto_graph_set_constraints(pesto_graph *g, const int64_t *mem, const int64_t *cap,
+                                         const int32_t *coloc) {
+    if (!g) return fail(PESTO_EINVAL, "NULL graph");
+    const int32_t n = g->n;
+    if (mem)
+        for (int32_t v = 0; v < n; v++)
+            if (mem[v] < 0) return fail(PESTO_EINVAL, "negative footprint");
+    if (cap)
+        for (int d = 0; d < g->D; d++)
+            if (cap[d] < 0) return fail(PESTO_EINVAL, "negative cap");
+    if (coloc)
+        for (int32_t v = 0; v < n; v++)
+            if (coloc[v] < -1 || coloc[v] >= n) return fail(PESTO_EINVAL, "colocation group out of [-1, n)");
+    DeviceGuard guard(g->device);
+    g->has_cap = cap != nullptr;
+    g->has_coloc = coloc != nullptr;
+    g->mem.assign(n, 0);
+    if (mem) {
+        std::copy(mem, mem + n, g->mem.begin());
+    } else {                                      // L202: input + output tensor sizes
+        for (int64_t e = 0; e < g->m; e++) {
+            g->mem[g->src[e]] += g->bytes[e];
+            g->mem[g->dst[e]] += g->bytes[e];
+        }
+    }
+    g->cap.assign(8, 0);
+    if (cap) std::copy(cap, cap + g->D, g->cap.begin());
+    g->coloc.assign(n, -1);
+    g->coloc_size.assign(n, 0);
+    g->coloc_pairs.clear();
+    if (coloc) {
+        std::vector<int32_t> rep(n, -1);
+        for (int32_t v = 0; v < n; v++) {
+            const int32_t c = coloc[v];
+            g->coloc[v] = c;
+            if (c < 0) continue;
+            g->coloc_size[c]++;
+            if (rep[c] < 0) rep[c] = v;
+            else g->coloc_pairs.push_back(make_int2(v, rep[c]));
+        }
+    }
+    g->cons_gen++;
+    if (g->device < 0) return PESTO_OK;
+    cudaError_t e;
+    if ((e = upload_vec(g->d_mem, g->mem)) != cudaSuccess || (e = upload_vec(g->d_cap, g->cap)) != cudaSuccess ||
+        (e = upload_vec(g->d_coloc, g->coloc)) != cudaSuccess ||
+        (e = upload_vec(g->d_coloc_size, g->coloc_size)) != cudaSuccess ||
+        (e = upload_vec(g->d_coloc_pairs, g->coloc_pairs)) != cudaSuccess)
+        return cuda_fail(e, "upload constraints");
+    return PESTO_OK;
 }
 
 pesto_status pesto_graph_set_link_model(pesto_graph *g, int32_t model) {
@@ -548,6 +635,19 @@ pesto_status pesto_eval_batch(pesto_graph *g, const int32_t *order, const void *
     tp.planes_out = g->d_planes.as<uint32_t>();
     tp.invalid_out = g->d_invalid.as<uint32_t>();
     if ((e = launch_transpose(tp, st)) != cudaSuccess) return cuda_fail(e, "launch transpose");
+    if (g->has_cap || g->has_coloc) {                 // row f3: mark infeasible rows
+        FeasParams fp{};
+        fp.planes = g->d_planes.as<uint32_t>();
+        fp.invalid = g->d_invalid.as<uint32_t>();
+        fp.n_groups = n_groups;
+        fp.n = g->n;
+        fp.D = g->D;
+        fp.planes_n = g->planes;
+        fp.order = L->d_order.as<int32_t>();
+        fp.pos_of = L->d_pos.as<int32_t>();
+        fp.feas = feasibility_view(g);
+        if ((e = launch_feasibility(fp, st)) != cudaSuccess) return cuda_fail(e, "launch feasibility");
+    }
     EvalParams p;
     fill_eval_common(g, p);
     p.stage_bytes = L->stage_bytes;

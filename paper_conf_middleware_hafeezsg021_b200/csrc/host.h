@@ -106,6 +106,13 @@ struct pesto_graph {
         d_out, d_state32, d_flags;        // d_flags: [count | list of saturated candidates]
     int32_t sms = 148;
     int32_t link_model = 0;               // PESTO_LINKS_FCFS / PESTO_LINKS_UNLIMITED
+    // row f3 constraints (host copies + device arrays); cons_gen counts changes
+    bool has_cap = false, has_coloc = false;
+    std::vector<int64_t> mem, cap;
+    std::vector<int32_t> coloc, coloc_size;
+    std::vector<int2> coloc_pairs;
+    int64_t cons_gen = 0;
+    pesto::DevBuf d_mem, d_cap, d_coloc, d_coloc_size, d_coloc_pairs;
 };
 
 namespace pesto {
@@ -117,6 +124,9 @@ pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<
 pesto_status upload_layout(pesto_graph *g, Layout &L);
 // v4 swap rule (DESIGN.md §4 S3) for the ops a (first) and c (second) of an adjacent pair
 bool pair_blocked(const pesto_graph *g, int32_t a, int32_t c);
+// row f3: the kernels' view of the constraints; a placement (by op id) satisfies them?
+Feasibility feasibility_view(const pesto_graph *g);
+bool placement_feasible(const pesto_graph *g, const uint8_t *x, int64_t *footprint8);
 BaseLayoutDev layout_view(const Layout &L);
 void fill_eval_common(const pesto_graph *g, EvalParams &p);
 pesto_status ensure_state(pesto_graph *g, const EvalParams &p, int search_mode, int64_t n_tasks,

@@ -35,6 +35,18 @@ struct BaseLayoutDev {
     const uint32_t *pin_ref;    // byte offsets (| kPinHeavy for the out-of-line array)
 };
 
+// Row f3 constraints as the kernels see them (PAPER.md L202 memory, L175 colocation).
+struct Feasibility {
+    int32_t has_cap, has_coloc;
+    const int64_t *mem;                 // [n] footprint by op id
+    const int64_t *cap;                 // [D]
+    const int32_t *coloc;               // [n] group by op id (-1 none)
+    const int32_t *coloc_size;          // [n] members per group id
+    const int2 *coloc_pairs;            // {op, representative op} for every non-first member
+    int32_t n_pairs;
+    int64_t *fbase;                     // search: [P][8] footprint of each base per device
+};
+
 struct EvalParams {
     int32_t n, D, planes, words;        // planes = bits per device code; words = ceil(n/32)
     int32_t edge_stride, n_classes;
@@ -73,6 +85,8 @@ struct EvalParams {
     int32_t cpl32;
     // 1: FCFS link queues; 0: congestion-free links (row f4(ii))
     int32_t link_queue;
+    // row f3 feasibility (search mode prologue): memory caps and colocation
+    Feasibility feas;
     // eval64 list mode (MODE 2): candidates list[0 .. *list_count)
     const int32_t *list;
     const int32_t *list_count;
@@ -101,6 +115,18 @@ struct CommitParams {
     int64_t *base_mk;
     int32_t *swap_out;                  // [P] committed swap position or -1
     int32_t patch32;                    // eval32 records carry base codes: patch them too
+    Feasibility feas;                   // f3: the committed move updates fbase
+};
+
+// explicit rows: OR the candidates violating the f3 constraints into the per-group masks
+struct FeasParams {
+    const uint32_t *planes;             // [group][pos][planes] (K5 output)
+    uint32_t *invalid;                  // [group]
+    int64_t n_groups;
+    int32_t n, D, planes_n;
+    const int32_t *order;               // [n] op at each position
+    const int32_t *pos_of;              // [n] position of each op
+    Feasibility feas;
 };
 
 // In-place layout patch (a committed adjacent swap, search.cpp): block rotations first, in list
@@ -124,6 +150,7 @@ cudaError_t launch_eval32(const EvalParams &p, int search_mode, int grid, cudaSt
 int eval32_smem_bytes(const EvalParams &p, int search_mode);
 int eval32_max_ctas_per_sm(const EvalParams &p, int search_mode);
 cudaError_t launch_transpose(const TransposeParams &p, cudaStream_t st);
+cudaError_t launch_feasibility(const FeasParams &p, cudaStream_t st);
 cudaError_t launch_commit(const CommitParams &p, cudaStream_t st);
 int eval_smem_bytes(const EvalParams &p, int search_mode);
 int eval_max_ctas_per_sm(const EvalParams &p, int search_mode);

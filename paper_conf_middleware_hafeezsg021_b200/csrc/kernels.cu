@@ -20,6 +20,7 @@
 #include <type_traits>
 
 #include "device_common.cuh"
+#include "feasibility.cuh"
 #include "internal.h"
 
 namespace pesto {
@@ -338,6 +339,9 @@ eval_kernel(const EvalParams P) {
                 : no_move();
             valid = in_range && place.mv.kind != kMoveInvalid;
             if (place.mv.kind == kMoveInvalid) place.mv = no_move();
+            if (valid && (P.feas.has_cap || P.feas.has_coloc))    // row f3
+                valid = move_feasible<PL>(place.mv, rg, P.D, bits, words, ord, B->allowed_pos,
+                                          P.all_allowed, P.feas, P.feas.fbase + (size_t)bl * 8);
         }
         st.init(P.D);
 
@@ -620,6 +624,14 @@ __global__ void commit_kernel(const CommitParams P) {
     uint8_t *blob32 = const_cast<uint8_t *>(B.blob32);
     uint8_t *heavy32 = const_cast<uint8_t *>(B.heavy32);
     auto set_dev = [&](int32_t q, int x) {
+        if (P.feas.has_cap) {                 // row f3: the base's footprint per device
+            const int old = get_dev_at<PL>(bits, words, q);
+            const long long m = (long long)P.feas.mem[B.order[q]];
+            atomicAdd(reinterpret_cast<unsigned long long *>(P.feas.fbase + (size_t)b * 8 + old),
+                      (unsigned long long)(-m));
+            atomicAdd(reinterpret_cast<unsigned long long *>(P.feas.fbase + (size_t)b * 8 + x),
+                      (unsigned long long)m);
+        }
         set_dev_at<PL>(bits, words, q, x);
         if (!P.patch32) return;
         uint32_t *flags = reinterpret_cast<uint32_t *>(blob32 + B.op_off32[q]) + 3;   // StepHead
@@ -780,6 +792,74 @@ static __global__ void patch_kernel(const PatchOp *ops, int n_ops) {
 cudaError_t launch_patch(const PatchOp *ops_dev, int n_ops, int max_block, cudaStream_t st) {
     note_launch();
     patch_kernel<<<1, 256, (size_t)std::max(max_block, 16), st>>>(ops_dev, n_ops);
+    return cudaGetLastError();
+}
+
+// ---------------------------------------------------------------------------------------------
+// Row f3 for explicit rows: one CTA per 32-row group marks the rows whose per-device footprint
+// exceeds its cap (L202) or whose colocation groups are split (L175).  Lane = row; the 8 warps
+// share the positions, then warp 0 adds their partial footprints.
+// ---------------------------------------------------------------------------------------------
+template <int PL>
+__global__ void __launch_bounds__(256) feasibility_kernel(const FeasParams P) {
+    __shared__ long long part[8][8][32];             // [warp][device][lane]
+    __shared__ uint32_t bad_s;
+    const int lane = threadIdx.x & 31, wq = threadIdx.x >> 5;
+    const Feasibility &F = P.feas;
+    for (int64_t g = blockIdx.x; g < P.n_groups; g += gridDim.x) {
+        if (threadIdx.x == 0) bad_s = 0;
+        const uint32_t *pl = P.planes + (size_t)g * P.n * PL;
+        __syncthreads();
+        if (F.has_cap) {
+            long long f[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+            for (int32_t q = wq; q < P.n; q += 8) {
+                int code = 0;
+#pragma unroll
+                for (int k = 0; k < PL; k++) code |= (int)((__ldg(pl + (size_t)q * PL + k) >> lane) & 1u) << k;
+                const long long m = __ldg(reinterpret_cast<const long long *>(F.mem) + __ldg(P.order + q));
+#pragma unroll
+                for (int d = 0; d < 8; d++) f[d] += d == code ? m : 0;
+            }
+#pragma unroll
+            for (int d = 0; d < 8; d++) part[wq][d][lane] = f[d];
+        }
+        uint32_t bad = 0;
+        if (F.has_coloc) {
+            for (int i = threadIdx.x; i < F.n_pairs; i += blockDim.x) {
+                const int2 pr = F.coloc_pairs[i];
+                const int32_t qa = __ldg(P.pos_of + pr.x), qb = __ldg(P.pos_of + pr.y);
+#pragma unroll
+                for (int k = 0; k < PL; k++) bad |= __ldg(pl + (size_t)qa * PL + k) ^ __ldg(pl + (size_t)qb * PL + k);
+            }
+        }
+        __syncthreads();
+        if (F.has_cap && wq == 0) {
+            bool over = false;
+            for (int d = 0; d < P.D; d++) {
+                long long tot = 0;
+#pragma unroll
+                for (int w = 0; w < 8; w++) tot += part[w][d][lane];
+                over = over || tot > __ldg(reinterpret_cast<const long long *>(F.cap) + d);
+            }
+            bad |= __ballot_sync(0xffffffffu, over);
+        }
+        if (bad) atomicOr(&bad_s, bad);
+        __syncthreads();
+        if (threadIdx.x == 0 && bad_s) P.invalid[g] |= bad_s;
+        __syncthreads();
+    }
+}
+
+cudaError_t launch_feasibility(const FeasParams &p, cudaStream_t st) {
+    note_launch();
+    if (p.n_groups <= 0) return cudaSuccess;
+    int dev = 0, sms = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    const int grid = (int)std::min<int64_t>(p.n_groups, (int64_t)sms * 4);
+    if (p.planes_n == 1) feasibility_kernel<1><<<grid, 256, 0, st>>>(p);
+    else if (p.planes_n == 2) feasibility_kernel<2><<<grid, 256, 0, st>>>(p);
+    else feasibility_kernel<4><<<grid, 256, 0, st>>>(p);
     return cudaGetLastError();
 }
 

@@ -75,6 +75,9 @@ struct pesto_search {
     std::vector<int64_t> h_mk;
     bool all_below = false;
     bool use32 = false;            // eval32 records exist for every base
+    // row f3: footprint of each base per device ([P][8]), for the constraints of cons_gen
+    DevBuf d_fbase;
+    int64_t cons_gen = -1;
     // committed swaps: patched in place on the device vs. layout rebuilt on the host
     DevBuf d_patch;
     int64_t n_swap_inplace = 0, n_swap_rebuilt = 0;
@@ -105,6 +108,29 @@ void update_all_below(pesto_search *s) {
         if (mk >= (int64_t)kSat32) s->all_below = false;
 }
 
+pesto_status download_x(pesto_search *s, int b, uint8_t *x_op);
+
+// row f3: (re)compute the bases' footprints when the graph's constraints changed; the bases
+// must satisfy the new constraints
+pesto_status sync_constraints(pesto_search *s) {
+    pesto_graph *g = s->g;
+    if (s->cons_gen == g->cons_gen) return PESTO_OK;
+    std::vector<int64_t> fb((size_t)s->P * 8, 0);
+    std::vector<uint8_t> x(g->n);
+    for (int b = 0; b < s->P; b++) {
+        pesto_status rc = download_x(s, b, x.data());
+        if (rc) return rc;
+        if (!placement_feasible(g, x.data(), fb.data() + (size_t)b * 8))
+            return fail(PESTO_ESTATE, "search base " + std::to_string(b) + " violates the constraints");
+    }
+    cudaError_t e;
+    if ((e = s->d_fbase.ensure(fb.size() * 8)) != cudaSuccess ||
+        (e = cudaMemcpy(s->d_fbase.ptr, fb.data(), fb.size() * 8, cudaMemcpyHostToDevice)) != cudaSuccess)
+        return cuda_fail(e, "upload base footprints");
+    s->cons_gen = g->cons_gen;
+    return PESTO_OK;
+}
+
 // fast: eval32 for the bases below saturation (+ eval64 for the others while any may exist);
 // otherwise (debug keys, initial makespans, ineligible graphs) eval64 for all candidates
 pesto_status launch_search_eval(pesto_search *s, int b_first, int n_bases, int64_t j0, int64_t j1,
@@ -112,8 +138,11 @@ pesto_status launch_search_eval(pesto_search *s, int b_first, int n_bases, int64
                                 bool fast = false) {
     pesto_graph *g = s->g;
     if (j1 <= j0) return PESTO_OK;
+    pesto_status rc0 = sync_constraints(s);
+    if (rc0) return rc0;
     EvalParams p;
     fill_eval_common(g, p);
+    p.feas.fbase = s->d_fbase.as<int64_t>() + (size_t)b_first * 8;
     p.stage_bytes = s->stage_bytes;
     p.max_W = s->max_W;
     p.stage_bytes32 = s->stage_bytes32;
@@ -439,6 +468,9 @@ pesto_status pesto_search_create(pesto_graph *g, const pesto_search_desc *d, pes
         if (d->base_x[i] >= g->D || !((g->allowed[v] >> d->base_x[i]) & 1))
             return fail(PESTO_EINVAL, "infeasible base placement at op " + std::to_string(v));
     }
+    for (int b = 0; b < d->n_bases; b++)                  // row f3 constraints
+        if (!placement_feasible(g, d->base_x + (size_t)b * n, nullptr))
+            return fail(PESTO_EINVAL, "base " + std::to_string(b) + " violates the graph's constraints");
     DeviceGuard guard(g->device);
     std::unique_ptr<pesto_search> s(new pesto_search());
     s->g = g;
@@ -558,6 +590,8 @@ pesto_status pesto_search_commit(pesto_search *s, void *stream) {
     cp.base_mk = s->d_mk.as<int64_t>();
     cp.swap_out = s->d_swap.as<int32_t>();
     cp.patch32 = s->use32 ? 1 : 0;
+    cp.feas = feasibility_view(g);
+    cp.feas.fbase = s->d_fbase.as<int64_t>();
     cudaError_t e = launch_commit(cp, st);
     if (e != cudaSuccess) return cuda_fail(e, "launch commit");
     s->step++;

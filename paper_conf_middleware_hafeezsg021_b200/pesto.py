@@ -60,6 +60,7 @@ SIGNATURES = {
     "pesto_graph_destroy": (None, [_VP]),
     "pesto_comm_model": (_I32, [_VP, _I32, _I32, _I64, _I64]),
     "pesto_graph_set_link_model": (_I32, [_VP, _I32]),
+    "pesto_graph_set_constraints": (_I32, [_VP, _VP, _VP, _VP]),
     "pesto_graph_stats_for": (_I32, [_VP, _VP, C.POINTER(GraphStats)]),
     "pesto_seed_order": (_I32, [_VP, _I32, _U64, _VP]),
     "pesto_seed_placement": (_I32, [_VP, _I32, _VP, _VP, _U64, _VP]),
@@ -188,6 +189,14 @@ class Graph:
     def set_link_model(self, model: int):
         """LINKS_FCFS (default; serial FCFS queue per directed link) or LINKS_UNLIMITED."""
         _check(_L.pesto_graph_set_link_model(self._h, model))
+
+    def set_constraints(self, mem=None, cap=None, coloc=None):
+        """Row f3: per-op footprint (None: input + output tensor bytes), per-device caps
+        (None: no memory constraint), colocation group per op (-1 none; None: no colocation)."""
+        arrs = [None if a is None else np.ascontiguousarray(a, dt)
+                for a, dt in ((mem, np.int64), (cap, np.int64), (coloc, np.int32))]
+        _check(_L.pesto_graph_set_constraints(self._h, *[None if a is None else _ptr(a)
+                                                          for a in arrs]))
 
     def stats(self, order) -> dict:
         o = np.ascontiguousarray(order, dtype=np.int32)

@@ -330,3 +330,81 @@ def test_search_full_size_sampled(P, O):
             gk = S.candidate_keys(b, j, j + 1)
             ok = O.candidate_keys(g, 2, b, xs, orders, j, j + 1, 2021, 0, MIX)
             assert (gk == ok).all(), (b, j)
+
+
+# ---------------------------------------------------------------------------------------------
+# Row f3: memory caps (L202) and colocation (L175)
+# ---------------------------------------------------------------------------------------------
+def _f3_constraints(g, frac=0.58, n_groups=6, size=3, seed=0):
+    rng = np.random.default_rng(seed)
+    mem = np.zeros(g.n, np.int64)
+    np.add.at(mem, g.src, g.nbytes)
+    np.add.at(mem, g.dst, g.nbytes)
+    cap = np.full(g.D, int(mem.sum() * frac), np.int64)
+    coloc = np.full(g.n, -1, np.int32)
+    ops = rng.choice(g.n, n_groups * size, replace=False)
+    for k in range(n_groups):
+        coloc[ops[k * size:(k + 1) * size]] = k
+    return mem, cap, coloc
+
+
+@pytest.mark.parametrize("D", [2, 4])
+def test_constraints_explicit_rows(P, O, D):
+    """explicit rows under memory caps and colocation: infeasible rows -> INT64_MAX, others
+    bit-exact, both equal to the oracle under the same constraints."""
+    g = dag.random_dag(101 + D, 900, 1.5, D=D, p_max=5000, max_bytes=400_000, beta0=700,
+                       beta1_fs=30_000)
+    mem, cap, coloc = _f3_constraints(g, frac=0.55 if D == 2 else 0.3)
+    G = P.Graph.from_arrays(g)
+    G.set_constraints(cap=cap, coloc=coloc)
+    order = dag.random_topo_order(g, 5)
+    x = dag.random_placements(g, 6, 700)
+    # make a third of the rows colocation-feasible so both outcomes occur
+    for i in range(0, len(x), 3):
+        for k in range(6):
+            x[i, coloc == k] = x[i, np.nonzero(coloc == k)[0][0]]
+    gpu = _gpu_eval(P, G, g, order, x)
+    with O.constraints(g, cap=cap, coloc=coloc) as c:
+        ok = np.asarray([c.ok(r) for r in x])
+        ref, _ = O.makespan_batch(g, x, order)
+    assert (gpu == ref).all(), np.nonzero(gpu != ref)[0][:5]
+    assert ok.any() and (~ok).any()
+    assert (gpu[~ok] == (1 << 63) - 1).all()
+    G.set_constraints()                                      # cleared: plain makespans
+    plain, _ = O.makespan_batch(g, x, order)
+    assert (_gpu_eval(P, G, g, order, x) == plain).all()
+
+
+@pytest.mark.parametrize("D", [2, 4])
+def test_constraints_search(P, O, D):
+    """search under caps + colocation: every candidate key (eval64) and each step's commits
+    (eval32 argmin, K4 footprint update) match the oracle's constrained search."""
+    g = dag.random_dag(111 + D, 400, 1.5, D=D, p_max=4000, max_bytes=300_000, beta0=600,
+                       beta1_fs=30_000)
+    mem, cap, coloc = _f3_constraints(g, frac=0.56 if D == 2 else 0.32, n_groups=5, seed=1)
+    xs, orders = _bases(g, 2, seed=21)
+    for b in range(2):                                       # feasible bases: groups together,
+        for k in range(5):                                   # then balance the footprint
+            xs[b, coloc == k] = 0
+        xs[b] = np.where(coloc >= 0, 0, np.arange(g.n) % D).astype(np.uint8)
+    G = P.Graph.from_arrays(g)
+    G.set_constraints(cap=cap, coloc=coloc)
+    mix = (40, 20, 20, 20)
+    K = 1024
+    S = P.Search(G, xs, orders, K, mix, seed=44)
+    rx, ro = xs.copy(), orders.copy()
+    with O.constraints(g, cap=cap, coloc=coloc) as c:
+        assert all(c.ok(rx[b]) for b in range(2))
+        rmk = np.asarray([O.makespan(g, rx[b], ro[b]) for b in range(2)], np.int64)
+        for b in range(2):
+            gk = S.candidate_keys(b, 0, K)
+            ok = O.candidate_keys(g, 2, b, rx, ro, 0, K, 44, 0, mix)
+            assert (gk == ok).all(), (b, np.nonzero(gk != ok)[0][:5])
+            assert (ok == (1 << 64) - 1).sum() > 0
+        for step in range(5):
+            S.step()
+            O.search_step(g, rx, ro, rmk, K, 44, step, mix)
+            for b in range(2):
+                mk, x, o = S.get(b)
+                assert mk == rmk[b] and (x == rx[b]).all() and (o == ro[b]).all(), (step, b)
+                assert c.ok(x)
