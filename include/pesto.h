@@ -113,6 +113,27 @@ pesto_status pesto_graph_set_link_model(pesto_graph *g, int32_t model);
 pesto_status pesto_graph_set_constraints(pesto_graph *g, const int64_t *mem_bytes,
                                          const int64_t *cap_bytes, const int32_t *coloc);
 
+/* Row f2: Pesto's graph coarsening (§3.3): heights (Def. 3.4), batch merges
+ * under Theorem 3.5 (reading R21 of (iii)), prioritised by the bytes between the merged
+ * vertices, repeated until at most `target` vertices remain or nothing can be merged.
+ *   coarse_of: HOST [n_ops] out, merged vertex of each op in [0, *n_coarse), numbered by each
+ *              vertex's smallest op id.   Host-only (works on a host-only handle).
+ * Errors: EINVAL (target < 1), ECYCLE (internal). */
+pesto_status pesto_coarsen(pesto_graph *g, int32_t target, int32_t *coarse_of, int32_t *n_coarse);
+
+/* Row f2: every placement of the merged vertices, each op on its vertex's device (L269),
+ * evaluated under order pi on the GPU: D^n_coarse candidates, candidate j giving vertex k the
+ * device (j >> (b*k)) & (D-1), b = log2 D.  Requires D in {1, 2, 4, 8}, b*n_coarse <= 24, the
+ * FCFS link model, no row-f3 constraints, an eval32-eligible graph and a best makespan below
+ * 4.03 s (else ESTATE).  Candidates with a vertex on a device some member may not use are
+ * skipped.  Outputs (HOST): the best makespan (INT64_MAX if none is feasible), the smallest
+ * best index, and its placement by op id [n_ops].  Synchronises.  Errors: EINVAL, ESTATE,
+ * ECUDA. */
+pesto_status pesto_eval_coarse_exhaustive(pesto_graph *g, const int32_t *order,
+                                          const int32_t *coarse_of, int32_t n_coarse,
+                                          int64_t *best_makespan, int64_t *best_index,
+                                          uint8_t *best_x, void *cuda_stream);
+
 typedef struct {
     int32_t n_ops, n_devices;
     int64_t n_edges;

@@ -68,9 +68,12 @@ def coarsen(n, src, dst, nbytes, target):
     rep = list(range(n))                       # op -> current vertex id (an op id)
 
     def find(a):
-        while rep[a] != a:
-            a = rep[a]
-        return a
+        r = a
+        while rep[r] != r:
+            r = rep[r]
+        while rep[a] != r:                     # path compression (roots are unchanged)
+            rep[a], a = r, rep[a]
+        return r
 
     while True:
         ids = sorted({find(a) for a in range(n)})

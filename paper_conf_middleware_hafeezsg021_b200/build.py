@@ -16,8 +16,9 @@ NVCC = os.path.join(CUDA, "bin", "nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 
 CU_SOURCES = ["kernels.cu", "eval32.cu"]
-CPP_SOURCES = ["graph.cpp", "layout.cpp", "search.cpp"]
-HEADERS = ["internal.h", "host.h", "layout_format.h", "moves.cuh", "device_common.cuh"]
+CPP_SOURCES = ["graph.cpp", "layout.cpp", "search.cpp", "coarsen.cpp"]
+HEADERS = ["internal.h", "host.h", "layout_format.h", "moves.cuh", "device_common.cuh",
+           "feasibility.cuh"]
 
 
 def _stale() -> bool:

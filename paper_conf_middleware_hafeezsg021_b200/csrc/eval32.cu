@@ -92,10 +92,19 @@ struct Place32 {
     int32_t rc, rlen;            // MODE 1: the group's region [rc, rc + rlen)
     int all_allowed, lane, dmax;
     LaneMove mv[CPL];
+    const uint8_t *cpos;         // MODE 4: merged vertex of the op at each position
+    int cbits;                   // MODE 4: bits per merged vertex in the candidate index
+    uint32_t jc[CPL];            // MODE 4: the lane's candidate indices
     __device__ __forceinline__ void at(int32_t q, int xb, int (&x)[CPL]) const {
         if (MODE == 0) {
 #pragma unroll
             for (int c = 0; c < CPL; c++) x[c] = planes_dev_at<PL>(pl + c * pl_stride, q, lane, dmax);
+            return;
+        }
+        if (MODE == 4) {                                       // digit of the merged vertex
+            const int sh = cbits * (int)__ldg(cpos + q);
+#pragma unroll
+            for (int c = 0; c < CPL; c++) x[c] = (int)((jc[c] >> sh) & (uint32_t)dmax);
             return;
         }
 #pragma unroll
@@ -257,7 +266,7 @@ eval32_kernel(const EvalParams P) {
         if (lane == 0) {
             uint32_t it = 0;
             for (int64_t task = blockIdx.x; task < P.n_tasks; task += gridDim.x) {
-                const int bl = MODE ? (int)(task / P.tasks_per_base) : 0;
+                const int bl = MODE == 1 ? (int)(task / P.tasks_per_base) : 0;
                 if (!runs_here(bl)) continue;
                 const BaseLayoutDev *B = &P.bases[bl];
                 const int nt = B->n_tiles32;
@@ -324,13 +333,13 @@ eval32_kernel(const EvalParams P) {
 
     uint32_t it = 0;
     for (int64_t task = blockIdx.x; task < P.n_tasks; task += gridDim.x) {
-        const int bl = MODE ? (int)(task / P.tasks_per_base) : 0;
+        const int bl = MODE == 1 ? (int)(task / P.tasks_per_base) : 0;
         if (!runs_here(bl)) continue;
-        const int64_t local = MODE ? task % P.tasks_per_base : task;
+        const int64_t local = MODE == 1 ? task % P.tasks_per_base : task;
         const BaseLayoutDev *B = &P.bases[bl];
         const int nt = B->n_tiles32;
         // a task = 256 consecutive candidate ids starting at a multiple of 256; a warp = CW of them
-        const int64_t j0 = (P.j_begin & ~(int64_t)255) + local * 256 + warp * CW;
+        const int64_t j0 = (MODE == 1 ? (P.j_begin & ~(int64_t)255) : 0) + local * 256 + warp * CW;
         const int64_t gw = j0 >> 5;                                 // first 32-row group
 
         Place32<MODE, PL, CPL> place;
@@ -342,7 +351,22 @@ eval32_kernel(const EvalParams P) {
         bool active;
         bool valid[CPL];
         int32_t ks = -1;
-        if (MODE == 0) {
+        if (MODE == 4) {
+            // exhaustive coarse placements (row f2): candidate j is its own placement code
+            active = j0 < P.n_cand;
+            place.cpos = P.coarse_pos;
+            place.cbits = P.coarse_bits;
+#pragma unroll
+            for (int c = 0; c < CPL; c++) {
+                const int64_t j = j0 + c * 32 + lane;
+                place.jc[c] = (uint32_t)j;
+                bool ok = j < P.n_cand;
+                if (!P.all_allowed)
+                    for (int k = 0; k < P.n_coarse; k++)
+                        ok = ok && ((P.coarse_allowed[k] >> ((j >> (P.coarse_bits * k)) & (P.D - 1))) & 1u);
+                valid[c] = ok;
+            }
+        } else if (MODE == 0) {
             active = j0 < P.n_cand;
             place.pl = P.planes_in + (size_t)gw * P.n * PL;
             place.pl_stride = (int64_t)P.n * PL;
@@ -618,7 +642,11 @@ int eval32_smem_bytes(const EvalParams &p, int search_mode) {
 #define PESTO_DISPATCH32_C(FN, C, ...)                                                     \
     do {                                                                                   \
         const int pl = planes_of32(p.D);                                                   \
-        if (search_mode) {                                                                 \
+        if (search_mode == 4) {                                                            \
+            if (pl == 1) return FN<4, 1, C>(__VA_ARGS__);                                  \
+            if (pl == 2) return FN<4, 2, C>(__VA_ARGS__);                                  \
+            return FN<4, 4, C>(__VA_ARGS__);                                               \
+        } else if (search_mode) {                                                          \
             if (pl == 1) return FN<1, 1, C>(__VA_ARGS__);                                  \
             if (pl == 2) return FN<1, 2, C>(__VA_ARGS__);                                  \
             return FN<1, 4, C>(__VA_ARGS__);                                               \

@@ -113,6 +113,7 @@ struct pesto_graph {
     std::vector<int2> coloc_pairs;
     int64_t cons_gen = 0;
     pesto::DevBuf d_mem, d_cap, d_coloc, d_coloc_size, d_coloc_pairs;
+    pesto::DevBuf d_cpos, d_ckey;         // row f2 exhaustive coarse search
 };
 
 namespace pesto {
@@ -124,6 +125,9 @@ pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<
 pesto_status upload_layout(pesto_graph *g, Layout &L);
 // v4 swap rule (DESIGN.md §4 S3) for the ops a (first) and c (second) of an adjacent pair
 bool pair_blocked(const pesto_graph *g, int32_t a, int32_t c);
+// row f2: PAPER.md §3.3 coarsening to at most `target` merged vertices (coarsen.cpp)
+pesto_status coarsen_graph(const pesto_graph *g, int32_t target, std::vector<int32_t> &coarse_of,
+                           int32_t &n_coarse);
 // row f3: the kernels' view of the constraints; a placement (by op id) satisfies them?
 Feasibility feasibility_view(const pesto_graph *g);
 bool placement_feasible(const pesto_graph *g, const uint8_t *x, int64_t *footprint8);

@@ -87,6 +87,11 @@ struct EvalParams {
     int32_t link_queue;
     // row f3 feasibility (search mode prologue): memory caps and colocation
     Feasibility feas;
+    // row f2 exhaustive coarse search (eval32 mode 4): candidate j gives coarse vertex k the
+    // device (j >> (coarse_bits * k)) & (D - 1); every op takes its merged vertex's device
+    const uint8_t *coarse_pos;          // [n] merged vertex of the op at each position
+    int32_t coarse_bits, n_coarse;
+    uint8_t coarse_allowed[32];         // device mask of each merged vertex (AND of members)
     // eval64 list mode (MODE 2): candidates list[0 .. *list_count)
     const int32_t *list;
     const int32_t *list_count;
@@ -144,7 +149,7 @@ constexpr int kTransposeSmemMax = 200 * 1024;  // K5 smem variant: a group's n*p
 
 // launchers (kernels.cu / eval32.cu); they return the launch error, if any.
 cudaError_t launch_patch(const PatchOp *ops_dev, int n_ops, int max_block, cudaStream_t st);
-// mode: 0 explicit rows, 1 search, 2 explicit list (eval64 only)
+// mode: 0 explicit rows, 1 search, 2 explicit list (eval64 only), 4 exhaustive coarse (eval32)
 cudaError_t launch_eval(const EvalParams &p, int search_mode, int grid, cudaStream_t st);
 cudaError_t launch_eval32(const EvalParams &p, int search_mode, int grid, cudaStream_t st);
 int eval32_smem_bytes(const EvalParams &p, int search_mode);

@@ -61,6 +61,8 @@ SIGNATURES = {
     "pesto_comm_model": (_I32, [_VP, _I32, _I32, _I64, _I64]),
     "pesto_graph_set_link_model": (_I32, [_VP, _I32]),
     "pesto_graph_set_constraints": (_I32, [_VP, _VP, _VP, _VP]),
+    "pesto_coarsen": (_I32, [_VP, _I32, _VP, _VP]),
+    "pesto_eval_coarse_exhaustive": (_I32, [_VP, _VP, _VP, _I32, _VP, _VP, _VP, _VP]),
     "pesto_graph_stats_for": (_I32, [_VP, _VP, C.POINTER(GraphStats)]),
     "pesto_seed_order": (_I32, [_VP, _I32, _U64, _VP]),
     "pesto_seed_placement": (_I32, [_VP, _I32, _VP, _VP, _U64, _VP]),
@@ -197,6 +199,24 @@ class Graph:
                 for a, dt in ((mem, np.int64), (cap, np.int64), (coloc, np.int32))]
         _check(_L.pesto_graph_set_constraints(self._h, *[None if a is None else _ptr(a)
                                                           for a in arrs]))
+
+    def coarsen(self, target: int):
+        """Row f2: PAPER.md §3.3 coarsening -> (coarse_of [n] int32, n_coarse)."""
+        out = np.empty(self.n, dtype=np.int32)
+        nc = C.c_int32()
+        _check(_L.pesto_coarsen(self._h, target, _ptr(out), C.byref(nc)))
+        return out, int(nc.value)
+
+    def eval_coarse_exhaustive(self, order, coarse_of, n_coarse: int, stream=None):
+        """Row f2: every placement of the merged vertices -> (best makespan, index, x)."""
+        o = np.ascontiguousarray(order, dtype=np.int32)
+        co = np.ascontiguousarray(coarse_of, dtype=np.int32)
+        mk, idx = C.c_int64(), C.c_int64()
+        x = np.empty(self.n, dtype=np.uint8)
+        _check(_L.pesto_eval_coarse_exhaustive(self._h, _ptr(o), _ptr(co), n_coarse,
+                                               C.byref(mk), C.byref(idx), _ptr(x),
+                                               _stream(stream)))
+        return int(mk.value), int(idx.value), x
 
     def stats(self, order) -> dict:
         o = np.ascontiguousarray(order, dtype=np.int32)

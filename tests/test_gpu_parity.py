@@ -408,3 +408,41 @@ def test_constraints_search(P, O, D):
                 mk, x, o = S.get(b)
                 assert mk == rmk[b] and (x == rx[b]).all() and (o == ro[b]).all(), (step, b)
                 assert c.ok(x)
+
+
+# ---------------------------------------------------------------------------------------------
+# Row f2: coarsening + exhaustive evaluation of the coarse placements
+# ---------------------------------------------------------------------------------------------
+@pytest.mark.parametrize("n,target,D", [(120, 10, 2), (300, 16, 2), (150, 6, 4)])
+def test_exhaustive_coarse_search(P, O, n, target, D):
+    """every coarse placement on the GPU (eval32 mode 4) vs the oracle's brute force over the
+    same D^n_coarse expanded placements: best makespan and smallest best index, bit-exact."""
+    from oracle import coarsen as OC
+    g = dag.random_dag(120 + n, n, 1.5, D=D, p_max=4000, max_bytes=200_000, beta0=500,
+                       beta1_fs=25_000)
+    G = P.Graph.from_arrays(g)
+    co, nc = G.coarsen(target)
+    assert nc == target
+    order = dag.random_topo_order(g, 3)
+    mk, idx, x = G.eval_coarse_exhaustive(order, co, nc)
+    best, bidx, allmk = OC.exhaustive(O, g, order, co, nc)
+    assert (mk, idx) == (best, bidx)
+    assert (x == OC.expand(co, D, idx)).all()
+
+
+def test_exhaustive_coarse_search_inception(P, O):
+    """PAPER.md §3.3 on the inception-shaped graph: coarsened to 20 vertices, all 2^20 coarse
+    placements evaluated on the GPU; the winner's makespan is re-checked by the oracle and no
+    sampled coarse placement beats it."""
+    from oracle import coarsen as OC
+    g = configs.graph_for(configs.CONFIGS["inception_v3_2dev"])
+    G = P.Graph.from_arrays(g)
+    co, nc = G.coarsen(20)
+    order = G.seed_order(P.ORDER_CRITICAL_PATH)
+    mk, idx, x = G.eval_coarse_exhaustive(order, co, nc)
+    assert O.makespan(g, x, order) == mk
+    rng = np.random.default_rng(0)
+    sample = rng.choice(1 << nc, 24, replace=False)
+    xs = np.stack([OC.expand(co, 2, int(c)) for c in sample])
+    ref, _ = O.makespan_batch(g, xs, order)
+    assert (ref >= mk).all()

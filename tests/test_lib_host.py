@@ -152,3 +152,25 @@ def test_layout_live_slots_bounds(P):
         assert 1 <= st["live_slots"] <= g.n
         assert st["n_tiles"] >= 1 and st["layout_bytes"] >= 16 * (g.n + g.m)
         assert st["max_in_degree"] == int(np.bincount(g.dst).max())
+
+
+def test_coarsen_matches_oracle(P):
+    """row f2 host code (§3.3 coarsening) equals the oracle's plain-Python coarsening
+    exactly, on random DAGs and on a shaped training-step graph."""
+    from oracle import coarsen as OC
+    cases = [dag.random_dag(800 + s, 50 + 23 * s, 1.5, D=2, max_bytes=50_000) for s in range(12)]
+    cases.append(dag.random_dag(900, 400, 1.6, D=2, max_bytes=50_000, fan_out_hub=60))
+    for g in cases:
+        G = _host_graph(P, g)
+        for target in (1, 5, 20, 64):
+            co, nc = G.coarsen(target)
+            ro, rn = OC.coarsen(g.n, g.src, g.dst, g.nbytes, target)
+            assert nc == rn and (co == ro).all(), (g.n, target)
+    # the shaped inception graph through its first, largest batches (the plain-Python oracle
+    # takes minutes to go all the way down; the random DAGs above reach the small targets)
+    g = configs.graph_for(configs.CONFIGS["inception_v3_2dev"])
+    co, nc = _host_graph(P, g).coarsen(8000)
+    ro, rn = OC.coarsen(g.n, g.src, g.dst, g.nbytes, 8000)
+    assert nc == rn == 8000 and (co == ro).all()
+    with pytest.raises(P.PestoError):
+        _host_graph(P, g).coarsen(0)
