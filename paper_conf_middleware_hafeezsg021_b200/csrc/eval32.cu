@@ -425,19 +425,44 @@ eval32_kernel(const EvalParams P) {
         auto place_y = [&](int, const uint4 rec, int (&y)[CPL]) {
             place.at((int32_t)(rec.y & kSuccPosMask), (int)((rec.y >> kSuccXShift) & 7u), y);
         };
-        // explicit rows: the plane words of the next op and of the next step's successors are
-        // loaded one step ahead (a successor's word is usually an L2 access)
-        PlaneWords<PL> pwx[CPL], pwy[2][CPL];
+        // explicit rows: the plane words of the next op are loaded one step ahead (consecutive
+        // positions share cache lines); the successors' words come from K5's edge-slot stream
+        // (DESIGN.md §3.4), read sequentially 32 words per lane-coalesced load, one window
+        // ahead, and handed out by shuffles -- no random lookups into the 139 MB of plane words
+        PlaneWords<PL> pwx[CPL];
         auto pw_load = [&](int32_t q, PlaneWords<PL> (&w)[CPL]) {
-            q = min(q, P.n - 1);                       // padding records name no real position
+            q = min(q, P.n - 1);
 #pragma unroll
             for (int c = 0; c < CPL; c++) w[c] = ldg_planes<PL>(place.pl + c * place.pl_stride, q);
         };
-        auto pw_y = [&](int k, const uint4, int (&y)[CPL]) {
+        constexpr int SW = 32 / PL;                    // edge slots per 32-word window
+        const int64_t ywords = P.n_slots * PL;         // words of one group's slot stream
+        uint32_t yw[CPL], yn[CPL];                     // this window / the next, per candidate
+        int64_t ywb = 0;                               // first slot of this window
+        int64_t slot0 = 0;                             // first slot of the current step
+        auto y_load = [&](int64_t slot, uint32_t (&w)[CPL]) {
+            const int64_t wi = slot * PL + lane;
 #pragma unroll
-            for (int c = 0; c < CPL; c++) y[c] = plane_dev<PL>(pwy[k][c], lane, place.dmax);
+            for (int c = 0; c < CPL; c++)
+                w[c] = wi < ywords ? __ldg(P.yplanes + (size_t)(gw + c) * ywords + wi) : 0u;
         };
-        if constexpr (MODE == 0) pw_load(0, pwx);
+        auto pw_y = [&](int k, const uint4, int (&y)[CPL]) {
+            const int base = (int)((slot0 + k - ywb) * PL);
+#pragma unroll
+            for (int c = 0; c < CPL; c++) {
+                PlaneWords<PL> w;
+#pragma unroll
+                for (int p = 0; p < PL; p++) w.w[p] = __shfl_sync(0xffffffffu, yw[c], base + p);
+                y[c] = plane_dev<PL>(w, lane, place.dmax);
+            }
+        };
+        if constexpr (MODE == 0) {
+            pw_load(0, pwx);
+            if (active) {
+                y_load(0, yw);
+                y_load(SW, yn);
+            }
+        }
         int32_t v = -1;
         int32_t skip = 0;            // steps of the next tile already walked (swap pair)
         for (int t = 0; t < nt; t++, it++) {
@@ -450,22 +475,19 @@ eval32_kernel(const EvalParams P) {
                 int32_t i = skip;
                 skip = 0;
                 uint4 h = lds_v4(sp), e0 = lds_v4(sp + 16), e1 = lds_v4(sp + 32);
-                if constexpr (MODE == 0) {
-                    pw_load((int32_t)(e0.y & kSuccPosMask), pwy[0]);
-                    pw_load((int32_t)(e1.y & kSuccPosMask), pwy[1]);
-                }
                 while (i < nsteps) {
-                    // the next step's head (past the tile's end: padding, never used); the edge
-                    // records are read here for this step (search: their first use is after the
-                    // head's work) or one step ahead (rows: they address the plane words)
+                    // the next step's head (past the tile's end: padding, never used); this
+                    // step's edge records (their first use is after the head's work)
                     const uint4 hn = lds_v4(sp + 48);
-                    uint4 e0n = e0, e1n = e1;
+                    e0 = lds_v4(sp + 16);
+                    e1 = lds_v4(sp + 32);
                     if constexpr (MODE == 0) {
-                        e0n = lds_v4(sp + 64);
-                        e1n = lds_v4(sp + 80);
-                    } else {
-                        e0 = lds_v4(sp + 16);
-                        e1 = lds_v4(sp + 32);
+                        if (slot0 >= ywb + SW) {               // next window; prefetch the one after
+#pragma unroll
+                            for (int c = 0; c < CPL; c++) yw[c] = yn[c];
+                            ywb += SW;
+                            y_load(ywb + SW, yn);
+                        }
                     }
                     if (!(h.w & kStCont)) {
                         v++;
@@ -543,18 +565,13 @@ eval32_kernel(const EvalParams P) {
                     }
                     if constexpr (MODE == 0) {
                         edges32<PL, CPL>(cx, h.w, e0, e1, x, cc, pw_y, st, fwd);
-                        pw_load((int32_t)(e0n.y & kSuccPosMask), pwy[0]);
-                        pw_load((int32_t)(e1n.y & kSuccPosMask), pwy[1]);
+                        slot0 += 2;
                     } else {
                         edges32<PL, CPL>(cx, h.w, e0, e1, x, cc, place_y, st, fwd);
                     }
                     sp += kStepBytes;
                     i++;
                     h = hn;
-                    if constexpr (MODE == 0) {
-                        e0 = e0n;
-                        e1 = e1n;
-                    }
                 }
             }
             __syncwarp();

@@ -124,6 +124,7 @@ pesto_status upload_layout(pesto_graph *g, Layout &L) {
     if ((e = upload_vec(L.d_op_off32, L.op_off32)) != cudaSuccess) return cuda_fail(e, "upload layout");
     if ((e = upload_vec(L.d_pin_off, L.pin_off)) != cudaSuccess) return cuda_fail(e, "upload layout");
     if ((e = upload_vec(L.d_pin_ref, L.pin_ref)) != cudaSuccess) return cuda_fail(e, "upload layout");
+    if ((e = upload_vec(L.d_slot_succ, L.slot_succ)) != cudaSuccess) return cuda_fail(e, "upload layout");
     L.on_device = true;
     std::vector<BaseLayoutDev> view{layout_view(L)};
     if ((e = upload_vec(L.d_view, view)) != cudaSuccess) return cuda_fail(e, "upload layout");
@@ -634,6 +635,15 @@ pesto_status pesto_eval_batch(pesto_graph *g, const int32_t *order, const void *
     tp.fmask = g->d_fmask.as<uint16_t>();
     tp.planes_out = g->d_planes.as<uint32_t>();
     tp.invalid_out = g->d_invalid.as<uint32_t>();
+    // the successors' codes in eval32 walk order (edge slots), for the explicit-row walk
+    const bool ystream = g->eligible32 && L->W32 > 0 && g->link_model == PESTO_LINKS_FCFS;
+    if (ystream) {
+        tp.slot_succ = L->d_slot_succ.as<int32_t>();
+        tp.n_slots = (int64_t)L->slot_succ.size();
+        if ((e = g->d_yplanes.ensure((size_t)n_groups * tp.n_slots * g->planes * 4)) != cudaSuccess)
+            return cuda_fail(e, "allocate edge-slot stream");
+        tp.yplanes_out = g->d_yplanes.as<uint32_t>();
+    }
     if ((e = launch_transpose(tp, st)) != cudaSuccess) return cuda_fail(e, "launch transpose");
     if (g->has_cap || g->has_coloc) {                 // row f3: mark infeasible rows
         FeasParams fp{};
@@ -655,6 +665,8 @@ pesto_status pesto_eval_batch(pesto_graph *g, const int32_t *order, const void *
     p.stage_bytes32 = L->stage_bytes32;
     p.max_W32 = L->W32;
     p.planes_in = g->d_planes.as<uint32_t>();
+    p.yplanes = g->d_yplanes.as<uint32_t>();
+    p.n_slots = (int64_t)L->slot_succ.size();
     p.invalid = g->d_invalid.as<uint32_t>();
     p.n_cand = n_cand;
     p.makespans = makespans;

@@ -63,10 +63,12 @@ struct Layout {
     std::vector<uint32_t> op_off64;                 // [pos] byte offset of the op record in blob
     std::vector<int32_t> tile64_of, tile32_of;      // [pos] tile holding the op's records
     std::vector<uint32_t> eloc64, eloc32;           // [edge] record offset (| kPinHeavy: heavy)
+    std::vector<int32_t> slot_succ;                 // [2 * steps] successor position of each
+                                                    // eval32 edge slot, -1 = empty (K5 y stream)
     int64_t comm_gen = -1;
     // device copies
     DevBuf d_blob, d_heavy, d_tiles, d_pos, d_adj, d_allowed_pos, d_view, d_order;
-    DevBuf d_blob32, d_heavy32, d_tiles32, d_op_off32, d_pin_off, d_pin_ref;
+    DevBuf d_blob32, d_heavy32, d_tiles32, d_op_off32, d_pin_off, d_pin_ref, d_slot_succ;
     bool on_device = false;
 };
 
@@ -114,6 +116,7 @@ struct pesto_graph {
     int64_t cons_gen = 0;
     pesto::DevBuf d_mem, d_cap, d_coloc, d_coloc_size, d_coloc_pairs;
     pesto::DevBuf d_cpos, d_ckey;         // row f2 exhaustive coarse search
+    pesto::DevBuf d_yplanes;              // explicit rows: codes per eval32 edge slot
 };
 
 namespace pesto {

@@ -58,6 +58,8 @@ struct EvalParams {
     int32_t max_W;
     // explicit-placement mode
     const uint32_t *planes_in;          // [group][pos][planes] bit-sliced codes
+    const uint32_t *yplanes;            // [group][slot][planes] codes of each edge slot's successor
+    int64_t n_slots;                    // edge slots of the eval32 stream (2 per step)
     const uint32_t *invalid;            // [group] lanes with an infeasible row
     int64_t n_cand;
     int64_t *makespans;
@@ -105,6 +107,9 @@ struct TransposeParams {
     const uint16_t *fmask;              // [n] forbidden device codes per op (bit c = code c)
     uint32_t *planes_out;
     uint32_t *invalid_out;
+    const int32_t *slot_succ;           // [n_slots] successor position of each edge slot, -1 none
+    int64_t n_slots;
+    uint32_t *yplanes_out;              // [group][n_slots][planes]
 };
 
 struct CommitParams {

@@ -565,7 +565,29 @@ __global__ void __launch_bounds__(256) transpose_smem_kernel(const TransposePara
         __syncthreads();
         uint32_t *dst = P.planes_out + (size_t)g * nw;
         for (int i = threadIdx.x; i < nw; i += blockDim.x) dst[i] = out_s[i];
+        if (P.yplanes_out) {                   // the edge-slot stream of the eval32 walk
+            uint32_t *ydst = P.yplanes_out + (size_t)g * P.n_slots * PL;
+            for (int64_t i = threadIdx.x; i < P.n_slots; i += blockDim.x) {
+                const int32_t q = __ldg(P.slot_succ + i);
+#pragma unroll
+                for (int k = 0; k < PL; k++) ydst[i * PL + k] = q >= 0 ? out_s[q * PL + k] : 0u;
+            }
+        }
         if (threadIdx.x == 0) P.invalid_out[g] = bad_s;
+    }
+}
+
+// the edge-slot stream from plane words in global memory (used after the global-scatter K5)
+template <int PL>
+__global__ void __launch_bounds__(256) ystream_kernel(const TransposeParams P) {
+    const int64_t total = P.n_groups * P.n_slots;
+    for (int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; t < total;
+         t += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t g = t / P.n_slots, i = t % P.n_slots;
+        const int32_t q = __ldg(P.slot_succ + i);
+        const uint32_t *src = P.planes_out + ((size_t)g * P.n + (q >= 0 ? q : 0)) * PL;
+#pragma unroll
+        for (int k = 0; k < PL; k++) P.yplanes_out[t * PL + k] = q >= 0 ? src[k] : 0u;
     }
 }
 
@@ -759,6 +781,14 @@ cudaError_t launch_transpose(const TransposeParams &p, cudaStream_t st) {
     if (p.planes == 1) transpose_kernel<1><<<grid, 256, 0, st>>>(p);
     else if (p.planes == 2) transpose_kernel<2><<<grid, 256, 0, st>>>(p);
     else transpose_kernel<4><<<grid, 256, 0, st>>>(p);
+    if (p.yplanes_out) {
+        cudaError_t e = cudaGetLastError();
+        if (e != cudaSuccess) return e;
+        const int yg = sms * 8;
+        if (p.planes == 1) ystream_kernel<1><<<yg, 256, 0, st>>>(p);
+        else if (p.planes == 2) ystream_kernel<2><<<yg, 256, 0, st>>>(p);
+        else ystream_kernel<4><<<yg, 256, 0, st>>>(p);
+    }
     return cudaGetLastError();
 }
 

@@ -253,6 +253,7 @@ pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<
         L->blob32.reserve((size_t)(n + m / 2 + 64) * kStepBytes + 64 * kTileHeader);
         L->op_off32.assign(n, 0);
         L->tile32_of.assign(n, 0);
+        L->slot_succ.clear();
         L->eloc32.assign(m, 0);
         // patch index: locations of every edge record by successor position
         L->pin_off.assign((size_t)n + 1, 0);
@@ -332,6 +333,8 @@ pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<
                     const EdgeRec32 r = edge_rec(sorted[b0 + 2 * s + q], eo);
                     std::memcpy(blob.data() + eo, &r, 16);
                 }
+                for (int64_t q = 0; q < 2; q++)       // explicit rows: successor of each slot
+                    L->slot_succ.push_back(q < ne ? pos[g->dst[sorted[b0 + 2 * s + q]]] : -1);
                 t_steps++;
             }
         }
