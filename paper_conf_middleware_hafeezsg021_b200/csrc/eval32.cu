@@ -429,11 +429,14 @@ eval32_kernel(const EvalParams P) {
         // positions share cache lines); the successors' words come from K5's edge-slot stream
         // (DESIGN.md §3.4), read sequentially 32 words per lane-coalesced load, one window
         // ahead, and handed out by shuffles -- no random lookups into the 139 MB of plane words
-        PlaneWords<PL> pwx[CPL];
-        auto pw_load = [&](int32_t q, PlaneWords<PL> (&w)[CPL]) {
-            q = min(q, P.n - 1);
+        // the op's own word likewise: position windows of 32 / PL positions
+        const int64_t xwords = (int64_t)P.n * PL;
+        uint32_t xw[CPL], xn[CPL];
+        int32_t xwb = 0;
+        auto x_load = [&](int32_t q, uint32_t (&w)[CPL]) {
+            const int64_t wi = (int64_t)q * PL + lane;
 #pragma unroll
-            for (int c = 0; c < CPL; c++) w[c] = ldg_planes<PL>(place.pl + c * place.pl_stride, q);
+            for (int c = 0; c < CPL; c++) w[c] = wi < xwords ? __ldg(place.pl + c * place.pl_stride + wi) : 0u;
         };
         constexpr int SW = 32 / PL;                    // edge slots per 32-word window
         const int64_t ywords = P.n_slots * PL;         // words of one group's slot stream
@@ -457,8 +460,9 @@ eval32_kernel(const EvalParams P) {
             }
         };
         if constexpr (MODE == 0) {
-            pw_load(0, pwx);
             if (active) {
+                x_load(0, xw);
+                x_load(SW, xn);
                 y_load(0, yw);
                 y_load(SW, yn);
             }
@@ -555,9 +559,20 @@ eval32_kernel(const EvalParams P) {
 #pragma unroll
                         for (int c = 0; c < CPL; c++) fwd[c] = 0u;
                         if constexpr (MODE == 0) {
+                            if (v >= xwb + SW) {               // next window; prefetch the one after
 #pragma unroll
-                            for (int c = 0; c < CPL; c++) x[c] = plane_dev<PL>(pwx[c], lane, place.dmax);
-                            pw_load(v + 1, pwx);
+                                for (int c = 0; c < CPL; c++) xw[c] = xn[c];
+                                xwb += SW;
+                                x_load(xwb + SW, xn);
+                            }
+#pragma unroll
+                            for (int c = 0; c < CPL; c++) {
+                                PlaneWords<PL> w;
+#pragma unroll
+                                for (int p = 0; p < PL; p++)
+                                    w.w[p] = __shfl_sync(0xffffffffu, xw[c], (v - xwb) * PL + p);
+                                x[c] = plane_dev<PL>(w, lane, place.dmax);
+                            }
                         } else {
                             place.at(v, (int)(h.w & kStXMask), x);
                         }
