@@ -304,12 +304,18 @@ def run_pesto(args, rank, world, local):
     eval_avg_s = (tot_eval_ms / args.steps) / 1e3
     achieved = alg_ops_launch / eval_avg_s / 1e12
     traffic = None
+    issue = None
     prof = os.path.join(ROOT, "profiles", f"r1_eval32_{args.config.split('_')[0]}_ncu.json")
     if os.path.exists(prof) and world == 1:
         try:
             pj = json.load(open(prof))
             if pj.get("config") == args.config:
                 traffic = pj["dram_bytes_per_launch"]
+                m = pj["metrics"]
+                issue = {"issue_slots_busy_pct": m["smsp__issue_active.avg.pct_of_peak_sustained_active"]["value"],
+                         "warps_per_smsp": m["smsp__warps_active.avg.per_cycle_active"]["value"],
+                         "dram_GBps": pj.get("dram_GBps"),
+                         "source": os.path.relpath(prof, ROOT)}
         except Exception:
             traffic = None
     st = G.stats(orders[0])
@@ -328,6 +334,7 @@ def run_pesto(args, rank, world, local):
                          "unit": "TOP/s (int32)", "frac": achieved / peak_tops,
                          "traffic": traffic, "peak_source": peak_note,
                          "ops_per_candidate": 2.0 * g.n + g.m + 2.0 * cross,
+                         "ncu": issue,
                          "note": "algorithmic int ops (2n+m+2*cross per candidate) / K1 time; "
                                  "traffic = ncu DRAM bytes per K1 launch (profiles/)"},
             "gpu_launches": int(launches),
