@@ -259,7 +259,7 @@ static int64_t simulate(int32_t n, const int64_t *p, int64_t m, const int32_t *s
                         const int32_t *dst, const int64_t *bytes, int32_t D,
                         const int64_t *beta0, const int64_t *beta1, const uint8_t *x,
                         const int32_t *order, const int32_t *pos, int congestion,
-                        oracle_trace *trace) {
+                        int nondelay, oracle_trace *trace) {
     int64_t ret = 0;
     int32_t L = D * D;
     /* out-edge lists (by producer) */
@@ -324,14 +324,27 @@ static int64_t simulate(int32_t n, const int64_t *p, int64_t m, const int32_t *s
                 if (hpush(&ev, evk)) { ret = ORACLE_ENOMEM; goto out; }
                 progress = 1;
             }
-            /* devices: no pre-emption, one op at a time (L146), next op of sigma_d only */
+            /* devices: no pre-emption, one op at a time (L146).  Fixed sequences (reading
+               Q1): the next op of sigma_d only, once its inputs are in.  Non-delay dispatch
+               (row f4(i), L90 "for each device, TensorFlow ... picks an operation from the
+               ready queue", with pi as the pick priority): the first op of sigma_d, in pi
+               order, that has not started and whose inputs are all in. */
             for (int32_t d = 0; d < D; d++) {
                 if (dbusy[d] || head[d] >= seq_off[d + 1]) continue;
-                int32_t v = seq[head[d]];
-                if (pending[v] != 0) continue;
+                int32_t v = -1;
+                if (!nondelay) {
+                    if (pending[seq[head[d]]] == 0) v = seq[head[d]];
+                } else {
+                    while (head[d] < seq_off[d + 1] && S[seq[head[d]]] >= 0) head[d]++;
+                    for (int32_t i = head[d]; i < seq_off[d + 1]; i++) {
+                        int32_t u = seq[i];
+                        if (S[u] < 0 && pending[u] == 0) { v = u; break; }
+                    }
+                }
+                if (v < 0) continue;
                 S[v] = now;
                 C[v] = now + p[v];
-                head[d]++;
+                if (!nondelay) head[d]++;
                 dbusy[d] = 1;
                 hkey evk = {{C[v], EV_OP_DONE, v, 0}};
                 if (hpush(&ev, evk)) { ret = ORACLE_ENOMEM; goto out; }
@@ -389,7 +402,7 @@ static int64_t makespan_common(int32_t n, const int64_t *p, int64_t m, const int
                                const int32_t *dst, const int64_t *bytes, int32_t D,
                                const int64_t *beta0, const int64_t *beta1,
                                const uint8_t *allowed, const uint8_t *x, const int32_t *order,
-                               int congestion, oracle_trace *trace) {
+                               int congestion, int nondelay, oracle_trace *trace) {
     int64_t rc = check_graph(n, p, m, src, dst, bytes, D, beta0, beta1);
     if (rc) return rc;
     int32_t *pos = malloc((size_t)n * sizeof(int32_t));
@@ -398,7 +411,7 @@ static int64_t makespan_common(int32_t n, const int64_t *p, int64_t m, const int
     if (rc == 0) {
         if (!feasible(n, D, allowed, x)) rc = INT64_MAX;
         else rc = simulate(n, p, m, src, dst, bytes, D, beta0, beta1, x, order, pos,
-                           congestion, trace);
+                           congestion, nondelay, trace);
     }
     free(pos);
     return rc;
@@ -408,7 +421,7 @@ int64_t oracle_makespan(int32_t n, const int64_t *p, int64_t m, const int32_t *s
                         const int32_t *dst, const int64_t *bytes, int32_t D,
                         const int64_t *beta0, const int64_t *beta1, const uint8_t *allowed,
                         const uint8_t *x, const int32_t *order, oracle_trace *trace) {
-    return makespan_common(n, p, m, src, dst, bytes, D, beta0, beta1, allowed, x, order, 1,
+    return makespan_common(n, p, m, src, dst, bytes, D, beta0, beta1, allowed, x, order, 1, 0,
                            trace);
 }
 
@@ -417,8 +430,17 @@ int64_t oracle_makespan_nocongest(int32_t n, const int64_t *p, int64_t m, const 
                                   const int64_t *beta0, const int64_t *beta1,
                                   const uint8_t *allowed, const uint8_t *x,
                                   const int32_t *order) {
-    return makespan_common(n, p, m, src, dst, bytes, D, beta0, beta1, allowed, x, order, 0,
+    return makespan_common(n, p, m, src, dst, bytes, D, beta0, beta1, allowed, x, order, 0, 0,
                            NULL);
+}
+
+int64_t oracle_makespan_model(int32_t n, const int64_t *p, int64_t m, const int32_t *src,
+                              const int32_t *dst, const int64_t *bytes, int32_t D,
+                              const int64_t *beta0, const int64_t *beta1, const uint8_t *allowed,
+                              const uint8_t *x, const int32_t *order, int32_t congestion,
+                              int32_t nondelay, oracle_trace *trace) {
+    return makespan_common(n, p, m, src, dst, bytes, D, beta0, beta1, allowed, x, order,
+                           congestion != 0, nondelay != 0, trace);
 }
 
 /* ------------------------------------------------------------------------------------- */
@@ -601,7 +623,7 @@ static void bf_all_placements(bf_ctx *c) {
     }
     for (;;) {
         int64_t mk = simulate(n, c->p, c->m, c->src, c->dst, c->bytes, c->D, c->beta0,
-                              c->beta1, c->x, c->order, c->pos, 1, NULL);
+                              c->beta1, c->x, c->order, c->pos, 1, 0, NULL);
         c->count++;
         if (mk < c->best) {
             c->best = mk;
@@ -761,6 +783,7 @@ typedef struct {
     int32_t P, b; const uint8_t *base_x; const int32_t *base_order;
     uint64_t seed, step; const int32_t *mix;
     int64_t j0, j1, base_j; uint64_t *out;
+    int32_t congestion, nondelay;
 } key_job;
 
 static void *key_worker(void *arg) {
@@ -771,8 +794,9 @@ static void *key_worker(void *arg) {
         uint64_t key = UINT64_MAX;
         if (oracle_candidate(k->n, k->m, k->src, k->dst, k->D, k->allowed, k->P, k->b, k->base_x,
                              k->base_order, j, k->seed, k->step, k->mix, x, ord)) {
-            int64_t mk = oracle_makespan(k->n, k->p, k->m, k->src, k->dst, k->bytes, k->D,
-                                         k->beta0, k->beta1, k->allowed, x, ord, NULL);
+            int64_t mk = oracle_makespan_model(k->n, k->p, k->m, k->src, k->dst, k->bytes, k->D,
+                                               k->beta0, k->beta1, k->allowed, x, ord,
+                                               k->congestion, k->nondelay, NULL);
             if (mk >= 0 && mk != INT64_MAX) key = ((uint64_t)mk << 24) | (uint64_t)j;
         }
         k->out[j - k->base_j] = key;
@@ -787,6 +811,19 @@ int oracle_candidate_keys(int32_t n, const int64_t *p, int64_t m, const int32_t 
                           int32_t P, int32_t b, const uint8_t *base_x, const int32_t *base_order,
                           int64_t j0, int64_t j1, uint64_t seed, uint64_t step,
                           const int32_t mix[4], int32_t threads, uint64_t *keys_out) {
+    return oracle_candidate_keys_model(n, p, m, src, dst, bytes, D, beta0, beta1, allowed, P, b,
+                                       base_x, base_order, j0, j1, seed, step, mix, 1, 0,
+                                       threads, keys_out);
+}
+
+int oracle_candidate_keys_model(int32_t n, const int64_t *p, int64_t m, const int32_t *src,
+                                const int32_t *dst, const int64_t *bytes, int32_t D,
+                                const int64_t *beta0, const int64_t *beta1,
+                                const uint8_t *allowed, int32_t P, int32_t b,
+                                const uint8_t *base_x, const int32_t *base_order, int64_t j0,
+                                int64_t j1, uint64_t seed, uint64_t step, const int32_t mix[4],
+                                int32_t congestion, int32_t nondelay, int32_t threads,
+                                uint64_t *keys_out) {
     int64_t rc = check_graph(n, p, m, src, dst, bytes, D, beta0, beta1);
     if (rc) return (int)rc;
     if (j0 < 0 || j1 < j0 || j1 > (1ll << 24)) return ORACLE_EINVAL;
@@ -798,7 +835,7 @@ int oracle_candidate_keys(int32_t n, const int64_t *p, int64_t m, const int32_t 
     for (int32_t t = 0; t < threads; t++) {
         key_job kj = {n, p, m, src, dst, bytes, D, beta0, beta1, allowed, P, b, base_x,
                       base_order, seed, step, mix, j0 + cnt * t / threads,
-                      j0 + cnt * (t + 1) / threads, j0, keys_out};
+                      j0 + cnt * (t + 1) / threads, j0, keys_out, congestion, nondelay};
         jobs[t] = kj;
         pthread_create(&th[t], NULL, key_worker, &jobs[t]);
     }

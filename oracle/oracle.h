@@ -66,6 +66,19 @@ int64_t oracle_makespan_nocongest(int32_t n, const int64_t *p, int64_t m, const 
                                   const uint8_t *allowed, const uint8_t *x,
                                   const int32_t *order);
 
+/* Row f4 evaluator variants in one entry point (event simulator, oracle #1):
+ *   congestion = 1: FCFS link queues (L144, L188-198); 0: congestion-free links (L113, L200);
+ *   nondelay   = 0: fixed per-device sequences sigma_d in pi order (reading Q1, L279, L374);
+ *                1: non-delay dispatch (row f4(i)): whenever a device is idle it starts, among
+ *                   its ops whose inputs have all arrived, the one earliest in pi -- TF's
+ *                   per-device ready queue (L90) with pi as the pick priority.
+ * oracle_makespan(...) == oracle_makespan_model(..., 1, 0, trace). */
+int64_t oracle_makespan_model(int32_t n, const int64_t *p, int64_t m, const int32_t *src,
+                              const int32_t *dst, const int64_t *bytes, int32_t D,
+                              const int64_t *beta0, const int64_t *beta1, const uint8_t *allowed,
+                              const uint8_t *x, const int32_t *order, int32_t congestion,
+                              int32_t nondelay, oracle_trace *trace);
+
 /* Feasibility constraints, row f3 (PAPER.md L202 memory, L175 colocation).  While set, every
  * makespan / key function of this library treats a placement that violates them as infeasible
  * (INT64_MAX, key UINT64_MAX).  For the graph (n, m, src, dst, bytes, D):
@@ -117,6 +130,16 @@ int oracle_candidate_keys(int32_t n, const int64_t *p, int64_t m, const int32_t 
                           int32_t P, int32_t b, const uint8_t *base_x, const int32_t *base_order,
                           int64_t j0, int64_t j1, uint64_t seed, uint64_t step,
                           const int32_t mix[4], int32_t threads, uint64_t *keys_out);
+
+/* The same under an evaluator variant (see oracle_makespan_model). */
+int oracle_candidate_keys_model(int32_t n, const int64_t *p, int64_t m, const int32_t *src,
+                                const int32_t *dst, const int64_t *bytes, int32_t D,
+                                const int64_t *beta0, const int64_t *beta1,
+                                const uint8_t *allowed, int32_t P, int32_t b,
+                                const uint8_t *base_x, const int32_t *base_order, int64_t j0,
+                                int64_t j1, uint64_t seed, uint64_t step, const int32_t mix[4],
+                                int32_t congestion, int32_t nondelay, int32_t threads,
+                                uint64_t *keys_out);
 
 /* One full step over P bases (in/out), K neighbours per base, W simulated ranks:
  * per-rank minima over [floor(rK/W), floor((r+1)K/W)) then the min of minima; commit. */

@@ -54,6 +54,13 @@ def lib():
         L.oracle_longest_path.restype = C.c_int64
         L.oracle_makespan_nocongest.argtypes = G + [_u8p, _i32p]
         L.oracle_makespan_nocongest.restype = C.c_int64
+        L.oracle_makespan_model.argtypes = G + [_u8p, _i32p, C.c_int32, C.c_int32, C.c_void_p]
+        L.oracle_makespan_model.restype = C.c_int64
+        L.oracle_candidate_keys_model.argtypes = G + [C.c_int32, C.c_int32, _u8p, _i32p,
+                                                      C.c_int64, C.c_int64, C.c_uint64,
+                                                      C.c_uint64, _i32p, C.c_int32, C.c_int32,
+                                                      C.c_int32, _u64p]
+        L.oracle_candidate_keys_model.restype = C.c_int
         L.oracle_makespan_batch.argtypes = G + [C.c_int64, _u8p, _i32p, C.c_int32, C.c_int32,
                                                 _i64p]
         L.oracle_makespan_batch.restype = C.c_double
@@ -114,6 +121,26 @@ def makespan(g, x, order, trace: bool = False):
          "XS": np.zeros(max(1, len(g.src)), np.int64), "XA": np.zeros(max(1, len(g.src)), np.int64)}
     tr = _Trace(t["S"].ctypes.data, t["C"].ctypes.data, t["XS"].ctypes.data, t["XA"].ctypes.data)
     mk = int(lib().oracle_makespan(*a, x, order, C.byref(tr)))
+    t["XS"] = t["XS"][:len(g.src)]
+    t["XA"] = t["XA"][:len(g.src)]
+    del keep
+    return mk, t
+
+
+def makespan_model(g, x, order, congestion: bool = True, nondelay: bool = False,
+                   trace: bool = False):
+    """Event simulator under a row-f4 variant: FCFS or congestion-free links, fixed per-device
+    sequences or non-delay dispatch by pi priority.  trace=True returns (makespan, trace)."""
+    a, keep = _g(g)
+    x = np.ascontiguousarray(x, dtype=np.uint8)
+    order = np.ascontiguousarray(order, dtype=np.int32)
+    if not trace:
+        return int(lib().oracle_makespan_model(*a, x, order, int(congestion), int(nondelay), None))
+    t = {"S": np.zeros(g.n, np.int64), "C": np.zeros(g.n, np.int64),
+         "XS": np.zeros(max(1, len(g.src)), np.int64), "XA": np.zeros(max(1, len(g.src)), np.int64)}
+    tr = _Trace(t["S"].ctypes.data, t["C"].ctypes.data, t["XS"].ctypes.data, t["XA"].ctypes.data)
+    mk = int(lib().oracle_makespan_model(*a, x, order, int(congestion), int(nondelay),
+                                         C.byref(tr)))
     t["XS"] = t["XS"][:len(g.src)]
     t["XA"] = t["XA"][:len(g.src)]
     del keep
@@ -217,6 +244,21 @@ def candidate_keys(g, P, b, base_x, base_order, j0, j1, seed, step, mix, threads
                                      step, np.asarray(mix, np.int32), threads, out)
     if rc != 0:
         raise ValueError(f"oracle_candidate_keys: {rc}")
+    return out[:j1 - j0]
+
+
+def candidate_keys_model(g, P, b, base_x, base_order, j0, j1, seed, step, mix,
+                         congestion: bool = True, nondelay: bool = False, threads: int = 0):
+    a, keep = _g(g)
+    out = np.zeros(max(1, j1 - j0), np.uint64)
+    if threads <= 0:
+        threads = len(os.sched_getaffinity(0))
+    rc = lib().oracle_candidate_keys_model(*a, P, b, np.ascontiguousarray(base_x, np.uint8),
+                                           np.ascontiguousarray(base_order, np.int32), j0, j1,
+                                           seed, step, np.asarray(mix, np.int32),
+                                           int(congestion), int(nondelay), threads, out)
+    if rc != 0:
+        raise ValueError(f"oracle_candidate_keys_model: {rc}")
     return out[:j1 - j0]
 
 

@@ -91,6 +91,9 @@ def test_worked_examples(O, ex):
         assert O.longest_path(g, case["x"], case["order"]) == case["makespan"]
         if "nocongest" in case:
             assert O.makespan_nocongest(g, case["x"], case["order"]) == case["nocongest"]
+        if "nondelay" in case:                                    # row f4(i), reading R24
+            assert O.makespan_model(g, case["x"], case["order"], nondelay=True) == case["nondelay"]
+        assert O.makespan_model(g, case["x"], case["order"]) == case["makespan"]
     if "optimum" in ex:
         assert O.bruteforce(g)[0] == ex["optimum"]
 
