@@ -43,6 +43,8 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
+    ap.add_argument("--dispatch", default="fixed", choices=["fixed", "nondelay"],
+                    help="row f4(i): nondelay = TF-style ready-queue dispatch by pi priority")
     return ap.parse_args()
 
 
@@ -132,15 +134,22 @@ def seeds_for(P, G, g, n_bases: int):
     return np.stack(xs[:n_bases]), np.stack(os_[:n_bases])
 
 
-def oracle_rate(g, xs, orders, k_per_base, seconds, threads):
+def oracle_rate(g, xs, orders, k_per_base, seconds, threads, nondelay=False):
     """Oracle (as it stands) on a bounded sample of this workload's step-0 candidates."""
     from oracle import oracle as O
     P_ = xs.shape[0]
     mix = configs.MOVE_MIX
+
+    def keys(b, j1):
+        if nondelay:
+            return O.candidate_keys_model(g, P_, b, xs, orders, 0, j1, configs.SEARCH_SEED, 0,
+                                          mix, nondelay=True, threads=threads)
+        return O.candidate_keys(g, P_, b, xs, orders, 0, j1, configs.SEARCH_SEED, 0, mix,
+                                threads)
     # calibrate a sample size that takes about `seconds` on `threads` threads
     t0 = time.perf_counter()
     probe = max(threads, 8)
-    O.candidate_keys(g, P_, 0, xs, orders, 0, probe, configs.SEARCH_SEED, 0, mix, threads)
+    keys(0, probe)
     dt = time.perf_counter() - t0
     per = dt / probe
     sample = int(max(probe, min(k_per_base, seconds / max(per, 1e-9))))
@@ -150,7 +159,7 @@ def oracle_rate(g, xs, orders, k_per_base, seconds, threads):
         cnt = sample // P_
         if cnt <= 0:
             continue
-        O.candidate_keys(g, P_, b, xs, orders, 0, cnt, configs.SEARCH_SEED, 0, mix, threads)
+        keys(b, cnt)
         done += cnt
     dt = time.perf_counter() - t0
     return done / dt, done, dt
@@ -169,9 +178,10 @@ def run_reference(args, rank, world):
     orders = np.stack([order, order])
     per_step_budget = max(1.0, args.cpu_seconds / max(1, args.steps + args.warmup))
     rates, times = [], []
+    nd = args.dispatch == "nondelay"
     for i in range(args.warmup + args.steps):
         rate, done, dt = oracle_rate(g, xs, orders, cfg.candidates_per_gpu // 2, per_step_budget,
-                                     threads)
+                                     threads, nondelay=nd)
         if i >= args.warmup:
             rates.append(rate)
             times.append(dt)
@@ -181,7 +191,7 @@ def run_reference(args, rank, world):
             "ms_per_step": 1e3 * cfg.candidates_per_gpu / value, "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "int64", "data": "synthetic",
             "config": {"workload": args.config, "n_ops": g.n, "n_edges": g.m, "D": g.D,
-                       "candidates_per_step": cfg.candidates_per_gpu},
+                       "candidates_per_step": cfg.candidates_per_gpu, "dispatch": args.dispatch},
             "op_relaxations_per_s": value * g.n,
             "cpu_baseline": {"value": value, "unit": "candidates/s", "cores": threads,
                              "kind": "oracle",
@@ -203,6 +213,9 @@ def run_pesto(args, rank, world, local):
     cfg = configs.CONFIGS[args.config]
     g = configs.graph_for(cfg)
     G = P.Graph.from_arrays(g, device=local)
+    nd = args.dispatch == "nondelay"
+    if nd:
+        G.set_dispatch(P.DISPATCH_NONDELAY)                 # row f4(i)
     n_bases = cfg.bases
     xs, orders = seeds_for(P, G, g, n_bases)
     k_gpu = cfg.candidates_per_gpu
@@ -306,7 +319,7 @@ def run_pesto(args, rank, world, local):
     traffic = None
     issue = None
     prof = os.path.join(ROOT, "profiles", f"r1_eval32_{args.config.split('_')[0]}_ncu.json")
-    if os.path.exists(prof) and world == 1:
+    if os.path.exists(prof) and world == 1 and not nd:
         try:
             pj = json.load(open(prof))
             if pj.get("config") == args.config:
@@ -327,7 +340,7 @@ def run_pesto(args, rank, world, local):
                        "candidates_per_step": k_gpu * world, "candidates_per_gpu": k_gpu,
                        "bases": n_bases, "k_per_base": k_per_base, "move_mix": configs.MOVE_MIX,
                        "live_slots": st["live_slots"], "l2": "flushed between timed steps",
-                       "parallelism": f"candidate-dp{world}"},
+                       "parallelism": f"candidate-dp{world}", "dispatch": args.dispatch},
             "op_relaxations_per_s": value * g.n, "edge_relaxations_per_s": value * g.m,
             "eval_kernel_ms": tot_eval_ms / args.steps,
             "roofline": {"bound": "alu", "achieved": achieved, "peak": peak_tops,
@@ -335,6 +348,7 @@ def run_pesto(args, rank, world, local):
                          "traffic": traffic, "peak_source": peak_note,
                          "ops_per_candidate": 2.0 * g.n + g.m + 2.0 * cross,
                          "ncu": issue,
+                         "kernel": "nondelay_kernel (row f4(i))" if nd else "eval32_kernel (K1)",
                          "note": "algorithmic int ops (2n+m+2*cross per candidate) / K1 time; "
                                  "traffic = ncu DRAM bytes per K1 launch (profiles/)"},
             "gpu_launches": int(launches),
@@ -345,7 +359,8 @@ def run_pesto(args, rank, world, local):
     line["clocks"] = clk.summary()
     if not args.no_cpu_baseline:
         threads = len(os.sched_getaffinity(0))
-        rate, done, dt = oracle_rate(g, xs, orders, k_per_base, args.cpu_seconds, threads)
+        rate, done, dt = oracle_rate(g, xs, orders, k_per_base, args.cpu_seconds, threads,
+                                     nondelay=nd)
         line["cpu_baseline"] = {"value": rate, "unit": "candidates/s", "cores": threads,
                                 "kind": "oracle",
                                 "sample": f"{done} step-0 neighbour candidates of the same "

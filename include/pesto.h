@@ -98,6 +98,19 @@ pesto_status pesto_comm_model(pesto_graph *g, int32_t src_dev, int32_t dst_dev,
 typedef enum { PESTO_LINKS_FCFS = 0, PESTO_LINKS_UNLIMITED = 1 } pesto_link_model;
 pesto_status pesto_graph_set_link_model(pesto_graph *g, int32_t model);
 
+/* Dispatch.  PESTO_DISPATCH_FIXED (the default, Pesto's schedule): each
+ * device runs its ops in pi order (L279 control dependencies, L374).  PESTO_DISPATCH_NONDELAY:
+ * TensorFlow's per-device ready queue ("picks an operation from the ready queue")
+ * with pi as the pick priority -- whenever a device is idle it starts, among its ops whose
+ * inputs have all arrived, the one earliest in pi (reading R24).  Links keep
+ * the link model.  Applies to every later pesto_eval_batch* and search step on g; runs on the
+ * exact 64-bit non-delay kernel (one warp per candidate; a modelling variant, not the
+ * throughput path).  Those calls return PESTO_ESTATE unless every p_i >= 1 ns, every transfer
+ * on every link >= 1 ns (R24: simultaneous zero-length events have no TF-defined order) and
+ * n_ops <= 2^20.  pesto_eval_coarse_exhaustive requires PESTO_DISPATCH_FIXED.  Errors: EINVAL. */
+typedef enum { PESTO_DISPATCH_FIXED = 0, PESTO_DISPATCH_NONDELAY = 1 } pesto_dispatch;
+pesto_status pesto_graph_set_dispatch(pesto_graph *g, int32_t mode);
+
 /* Feasibility constraints: per-device memory footprint and
  * colocation groups (L175).  A candidate violating one is infeasible: makespan INT64_MAX,
  * search key UINT64_MAX.  All arrays HOST, copied:
@@ -124,7 +137,7 @@ pesto_status pesto_coarsen(pesto_graph *g, int32_t target, int32_t *coarse_of, i
 /* Row f2: every placement of the merged vertices, each op on its vertex's device (L269),
  * evaluated under order pi on the GPU: D^n_coarse candidates, candidate j giving vertex k the
  * device (j >> (b*k)) & (D-1), b = log2 D.  Requires D in {1, 2, 4, 8}, b*n_coarse <= 24, the
- * FCFS link model, no row-f3 constraints, an eval32-eligible graph and a best makespan below
+ * FCFS link model, fixed dispatch, no row-f3 constraints, an eval32-eligible graph and a best makespan below
  * 4.03 s (else ESTATE).  Candidates with a vertex on a device some member may not use are
  * skipped.  Outputs (HOST): the best makespan (INT64_MAX if none is feasible), the smallest
  * best index, and its placement by op id [n_ops].  Synchronises.  Errors: EINVAL, ESTATE,

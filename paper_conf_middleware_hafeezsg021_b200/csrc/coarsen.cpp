@@ -220,8 +220,8 @@ pesto_status pesto_eval_coarse_exhaustive(pesto_graph *g, const int32_t *order,
     const int b = D == 1 ? 0 : D == 2 ? 1 : D == 4 ? 2 : D == 8 ? 3 : -1;
     if (b < 0) return fail(PESTO_EINVAL, "exhaustive coarse search needs D in {1, 2, 4, 8}");
     if (b * n_coarse > 24) return fail(PESTO_EINVAL, "D^n_coarse exceeds 2^24 candidates");
-    if (g->link_model != PESTO_LINKS_FCFS || g->has_cap || g->has_coloc)
-        return fail(PESTO_ESTATE, "exhaustive coarse search supports the FCFS model without constraints");
+    if (g->link_model != PESTO_LINKS_FCFS || g->dispatch != PESTO_DISPATCH_FIXED || g->has_cap || g->has_coloc)
+        return fail(PESTO_ESTATE, "exhaustive coarse search supports the FCFS fixed-sequence model without constraints");
     DeviceGuard guard(g->device);
     cudaStream_t st = (cudaStream_t)stream;
     std::shared_ptr<Layout> L;

@@ -151,7 +151,96 @@ BaseLayoutDev layout_view(const Layout &L) {
     v.op_off32 = L.d_op_off32.as<uint32_t>();
     v.pin_off = L.d_pin_off.as<uint32_t>();
     v.pin_ref = L.d_pin_ref.as<uint32_t>();
+    v.nd_dst = L.d_nd_dst.as<int32_t>();
+    v.nd_t = L.d_nd_t.as<int64_t>();
     return v;
+}
+
+// ---------------------------------------------------------------------------------------------
+// row f4(i): non-delay dispatch (reading R24)
+// ---------------------------------------------------------------------------------------------
+pesto_status nd_check(pesto_graph *g) {
+    pesto_status s = ensure_comm_tables(g);
+    if (s) return s;
+    if (g->n > (1 << 20)) return fail(PESTO_ESTATE, "non-delay dispatch supports n_ops <= 2^20");
+    for (int32_t v = 0; v < g->n; v++)
+        if (g->p[v] < 1)
+            return fail(PESTO_ESTATE, "non-delay dispatch needs every p_i >= 1 ns (reading R24); op " +
+                                          std::to_string(v) + " has p = 0");
+    if (g->D > 1)
+        for (int64_t t : g->t_class)
+            if (t < 1) return fail(PESTO_ESTATE, "non-delay dispatch needs every transfer >= 1 ns (reading R24)");
+    if (!g->nd_graph_ready) {
+        cudaError_t e;
+        if ((e = upload_vec(g->d_nd_p, g->p)) != cudaSuccess || (e = upload_vec(g->d_nd_indeg, g->indeg)) != cudaSuccess ||
+            (e = upload_vec(g->d_nd_off, g->out_off)) != cudaSuccess)
+            return cuda_fail(e, "upload non-delay graph arrays");
+        g->nd_graph_ready = true;
+    }
+    return PESTO_OK;
+}
+
+pesto_status nd_ensure_layout(pesto_graph *g, Layout &L) {
+    if (L.nd_gen == g->t_gen && L.d_nd_dst.ptr) return PESTO_OK;
+    const int NC = g->n_classes;
+    std::vector<int32_t> dst((size_t)g->m);
+    std::vector<int64_t> t((size_t)g->m * NC);
+    std::vector<int64_t> es;
+    for (int32_t v = 0; v < g->n; v++) {
+        es.assign(g->out_edges.begin() + g->out_off[v], g->out_edges.begin() + g->out_off[v + 1]);
+        std::sort(es.begin(), es.end(), [&](int64_t a, int64_t b) {   // FCFS ties: (pos w, e), R3
+            const int32_t pa = L.pos[g->dst[a]], pb = L.pos[g->dst[b]];
+            return pa != pb ? pa < pb : a < b;
+        });
+        for (size_t k = 0; k < es.size(); k++) {
+            const int64_t i = g->out_off[v] + (int64_t)k;
+            dst[i] = g->dst[es[k]];
+            for (int c = 0; c < NC; c++) t[(size_t)i * NC + c] = g->t_class[(size_t)es[k] * NC + c];
+        }
+    }
+    cudaError_t e;
+    if ((e = upload_vec(L.d_nd_dst, dst)) != cudaSuccess || (e = upload_vec(L.d_nd_t, t)) != cudaSuccess)
+        return cuda_fail(e, "upload non-delay edge order");
+    L.nd_gen = g->t_gen;
+    return PESTO_OK;
+}
+
+pesto_status nd_fill(pesto_graph *g, NdParams &p, int64_t n_tasks, int *grid_out) {
+    std::memset(&p, 0, sizeof p);
+    p.n = g->n;
+    p.D = g->D;
+    p.planes = g->planes;
+    p.words = g->words;
+    p.nw1 = (p.words + 31) / 32;
+    p.nw2 = (p.nw1 + 31) / 32;
+    p.rb = p.words + p.nw1 + p.nw2;
+    p.n_classes = g->n_classes;
+    p.link_queue = g->link_model == PESTO_LINKS_FCFS ? 1 : 0;
+    p.all_allowed = g->all_allowed ? 1 : 0;
+    std::memcpy(p.link_class, g->link_class, 64);
+    p.p = g->d_nd_p.as<int64_t>();
+    p.indeg = g->d_nd_indeg.as<int32_t>();
+    p.out_off = g->d_nd_off.as<int64_t>();
+    p.feas = feasibility_view(g);
+    p.warps_per_cta = nondelay_warps_per_cta(p);
+    if (p.warps_per_cta == 0)
+        return fail(PESTO_ESTATE, "non-delay kernel: the graph's per-warp state exceeds shared memory");
+    const int per_sm = nondelay_max_ctas_per_sm(p);
+    if (per_sm <= 0) return fail(PESTO_ECUDA, "non-delay kernel does not fit on an SM");
+    int64_t grid = std::min<int64_t>((n_tasks + p.warps_per_cta - 1) / p.warps_per_cta,
+                                     (int64_t)g->sms * per_sm);
+    grid = std::max<int64_t>(grid, 1);
+    const size_t slots = (size_t)grid * p.warps_per_cta;
+    cudaError_t e;
+    if ((e = g->d_nd_rem.ensure(slots * g->n * 4)) != cudaSuccess ||
+        (e = g->d_nd_rdy.ensure(slots * g->n * 8)) != cudaSuccess ||
+        (e = g->d_nd_pend.ensure(slots * g->n * g->D * 8)) != cudaSuccess)
+        return cuda_fail(e, "allocate non-delay scratch");
+    p.rem = g->d_nd_rem.as<int32_t>();
+    p.rdy = g->d_nd_rdy.as<int64_t>();
+    p.pend = g->d_nd_pend.as<uint64_t>();
+    *grid_out = (int)grid;
+    return PESTO_OK;
 }
 
 void fill_eval_common(const pesto_graph *g, EvalParams &p) {
@@ -435,6 +524,13 @@ pesto_status pesto_graph_set_constraints(pesto_graph *g, const int64_t *mem, con
     return PESTO_OK;
 }
 
+pesto_status pesto_graph_set_dispatch(pesto_graph *g, int32_t mode) {
+    if (!g) return fail(PESTO_EINVAL, "NULL graph");
+    if (mode != PESTO_DISPATCH_FIXED && mode != PESTO_DISPATCH_NONDELAY) return fail(PESTO_EINVAL, "unknown dispatch mode");
+    g->dispatch = mode;
+    return PESTO_OK;
+}
+
 pesto_status pesto_graph_set_link_model(pesto_graph *g, int32_t model) {
     if (!g) return fail(PESTO_EINVAL, "NULL graph");
     if (model != PESTO_LINKS_FCFS && model != PESTO_LINKS_UNLIMITED) return fail(PESTO_EINVAL, "unknown link model");
@@ -636,7 +732,12 @@ pesto_status pesto_eval_batch(pesto_graph *g, const int32_t *order, const void *
     tp.planes_out = g->d_planes.as<uint32_t>();
     tp.invalid_out = g->d_invalid.as<uint32_t>();
     // the successors' codes in eval32 walk order (edge slots), for the explicit-row walk
-    const bool ystream = g->eligible32 && L->W32 > 0 && g->link_model == PESTO_LINKS_FCFS;
+    const bool nondelay = g->dispatch == PESTO_DISPATCH_NONDELAY;
+    if (nondelay) {
+        if ((s = nd_check(g))) return s;
+        if ((s = nd_ensure_layout(g, *L))) return s;
+    }
+    const bool ystream = !nondelay && g->eligible32 && L->W32 > 0 && g->link_model == PESTO_LINKS_FCFS;
     if (ystream) {
         tp.slot_succ = L->d_slot_succ.as<int32_t>();
         tp.n_slots = (int64_t)L->slot_succ.size();
@@ -657,6 +758,22 @@ pesto_status pesto_eval_batch(pesto_graph *g, const int32_t *order, const void *
         fp.pos_of = L->d_pos.as<int32_t>();
         fp.feas = feasibility_view(g);
         if ((e = launch_feasibility(fp, st)) != cudaSuccess) return cuda_fail(e, "launch feasibility");
+    }
+    if (nondelay) {                                   // row f4(i): one warp per row
+        NdParams np;
+        int grid = 0;
+        if ((s = nd_fill(g, np, n_cand, &grid))) return s;
+        np.rows = tp.rows;
+        np.stride = stride;
+        np.n_cand = n_cand;
+        np.invalid = g->d_invalid.as<uint32_t>();
+        np.makespans = makespans;
+        np.nd_dst = L->d_nd_dst.as<int32_t>();
+        np.nd_t = L->d_nd_t.as<int64_t>();
+        np.pos_of = L->d_pos.as<int32_t>();
+        np.order = L->d_order.as<int32_t>();
+        if ((e = launch_nondelay(np, 0, grid, st)) != cudaSuccess) return cuda_fail(e, "launch non-delay");
+        return PESTO_OK;
     }
     EvalParams p;
     fill_eval_common(g, p);

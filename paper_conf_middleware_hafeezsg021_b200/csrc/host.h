@@ -69,6 +69,9 @@ struct Layout {
     // device copies
     DevBuf d_blob, d_heavy, d_tiles, d_pos, d_adj, d_allowed_pos, d_view, d_order;
     DevBuf d_blob32, d_heavy32, d_tiles32, d_op_off32, d_pin_off, d_pin_ref, d_slot_succ;
+    // row f4(i): producer-grouped out-edges in this order's FCFS tie order (built on demand)
+    DevBuf d_nd_dst, d_nd_t;
+    int64_t nd_gen = -1;                // comm tables generation the nd arrays were built for
     bool on_device = false;
 };
 
@@ -108,6 +111,9 @@ struct pesto_graph {
         d_out, d_state32, d_flags;        // d_flags: [count | list of saturated candidates]
     int32_t sms = 148;
     int32_t link_model = 0;               // PESTO_LINKS_FCFS / PESTO_LINKS_UNLIMITED
+    int32_t dispatch = 0;                 // PESTO_DISPATCH_FIXED / PESTO_DISPATCH_NONDELAY
+    pesto::DevBuf d_nd_p, d_nd_indeg, d_nd_off, d_nd_rem, d_nd_rdy, d_nd_pend;
+    bool nd_graph_ready = false;
     // row f3 constraints (host copies + device arrays); cons_gen counts changes
     bool has_cap = false, has_coloc = false;
     std::vector<int64_t> mem, cap;
@@ -128,6 +134,11 @@ pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<
 pesto_status upload_layout(pesto_graph *g, Layout &L);
 // v4 swap rule (DESIGN.md §4 S3) for the ops a (first) and c (second) of an adjacent pair
 bool pair_blocked(const pesto_graph *g, int32_t a, int32_t c);
+// row f4(i): device arrays of the non-delay kernel (graph-level and per order), the domain
+// check (positive durations, n <= 2^20) and the scratch for `slots` resident warps
+pesto_status nd_check(pesto_graph *g);
+pesto_status nd_ensure_layout(pesto_graph *g, Layout &L);
+pesto_status nd_fill(pesto_graph *g, NdParams &p, int64_t n_tasks, int *grid_out);
 // row f2: PAPER.md §3.3 coarsening to at most `target` merged vertices (coarsen.cpp)
 pesto_status coarsen_graph(const pesto_graph *g, int32_t target, std::vector<int32_t> &coarse_of,
                            int32_t &n_coarse);

@@ -33,6 +33,10 @@ struct BaseLayoutDev {
     const uint32_t *op_off32;   // [n] byte offset of the op record at each position (blob32)
     const uint32_t *pin_off;    // [n+1] CSR: edge records whose successor is at each position
     const uint32_t *pin_ref;    // byte offsets (| kPinHeavy for the out-of-line array)
+    // row f4(i) non-delay kernel: out-edges by producer op id (graph CSR offsets), each
+    // producer's edges in (successor position, edge index) order -- the FCFS tie order R3
+    const int32_t *nd_dst;      // [m] consumer op id
+    const int64_t *nd_t;        // [m][n_classes] transfer time per link class
 };
 
 // Row f3 constraints as the kernels see them (PAPER.md L202 memory, L175 colocation).
@@ -99,6 +103,36 @@ struct EvalParams {
     const int32_t *list_count;
 };
 
+// Row f4(i): non-delay dispatch, one warp per candidate.
+struct NdParams {
+    int32_t n, D, planes, words;        // words = ceil(n/32)
+    int32_t nw1, nw2, rb;               // ready-set bitmap levels: words, nw1, nw2 words; rb = sum
+    int32_t n_classes, link_queue, all_allowed, warps_per_cta;
+    uint8_t link_class[64];
+    const int64_t *p;                   // [n] by op id
+    const int32_t *indeg;               // [n] by op id
+    const int64_t *out_off;             // [n+1] out-edge CSR offsets by producer op id
+    int32_t *rem;                       // scratch per resident warp: [slot][n] inputs missing
+    int64_t *rdy;                       // [slot][n] latest arrival so far
+    uint64_t *pend;                     // [slot][D][n] per-device heaps of ops whose inputs arrive later
+    // explicit rows (mode 0)
+    const uint8_t *rows;                // [n_cand][stride], op i's code in bits [b*i, b*i+b)
+    int64_t stride, n_cand;
+    const uint32_t *invalid;            // [group] K5 (+ f3) infeasible-row masks
+    int64_t *makespans;
+    const int32_t *nd_dst, *pos_of, *order;
+    const int64_t *nd_t;
+    // search (mode 1)
+    const BaseLayoutDev *bases;
+    int32_t n_bases, b_offset, P_total;
+    int64_t j_begin, j_end;
+    uint64_t seed, step;
+    int32_t mix[4];
+    const uint8_t *allowed_op;
+    uint64_t *keys, *keys_dbg;
+    Feasibility feas;
+};
+
 struct TransposeParams {
     const uint8_t *rows;
     int64_t stride, n_cand, n_groups;
@@ -163,6 +197,11 @@ cudaError_t launch_transpose(const TransposeParams &p, cudaStream_t st);
 cudaError_t launch_feasibility(const FeasParams &p, cudaStream_t st);
 cudaError_t launch_commit(const CommitParams &p, cudaStream_t st);
 int eval_smem_bytes(const EvalParams &p, int search_mode);
+// row f4(i): warps per CTA that fit the shared-memory budget (0: the graph does not fit), the
+// resident CTAs per SM, and the launch (mode 0 explicit rows, 1 search)
+int nondelay_warps_per_cta(const NdParams &p);
+int nondelay_max_ctas_per_sm(const NdParams &p);
+cudaError_t launch_nondelay(const NdParams &p, int mode, int grid, cudaStream_t st);
 int eval_max_ctas_per_sm(const EvalParams &p, int search_mode);
 void note_launch();
 

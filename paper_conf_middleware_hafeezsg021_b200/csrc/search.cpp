@@ -131,6 +131,50 @@ pesto_status sync_constraints(pesto_search *s) {
     return PESTO_OK;
 }
 
+// row f4(i): every candidate on the non-delay kernel (one warp each); the bases' producer-grouped
+// edge orders are built on demand (a committed swap never reorders a producer's consumers: the
+// S3 rule blocks pairs that share a producer)
+pesto_status launch_search_nondelay(pesto_search *s, int b_first, int n_bases, int64_t j0, int64_t j1,
+                                    uint64_t *keys, uint64_t *keys_dbg, cudaStream_t st) {
+    pesto_graph *g = s->g;
+    pesto_status rc = nd_check(g);
+    if (rc) return rc;
+    bool changed = false;
+    for (int b = 0; b < s->P; b++) {
+        void *before = s->layouts[b]->d_nd_dst.ptr;
+        const int64_t gen = s->layouts[b]->nd_gen;
+        if ((rc = nd_ensure_layout(g, *s->layouts[b]))) return rc;
+        changed |= before != s->layouts[b]->d_nd_dst.ptr || gen != s->layouts[b]->nd_gen;
+    }
+    cudaError_t e;
+    if (changed) {
+        refresh_views(s);
+        if ((e = cudaMemcpyAsync(s->d_views.ptr, s->views.data(), sizeof(BaseLayoutDev) * s->P,
+                                 cudaMemcpyHostToDevice, st)) != cudaSuccess)
+            return cuda_fail(e, "upload views");
+        if ((e = cudaStreamSynchronize(st)) != cudaSuccess) return cuda_fail(e, "upload views");
+    }
+    NdParams p;
+    int grid = 0;
+    const int64_t n_tasks = (int64_t)n_bases * (j1 - j0);
+    if ((rc = nd_fill(g, p, n_tasks, &grid))) return rc;
+    p.feas.fbase = s->d_fbase.as<int64_t>() + (size_t)b_first * 8;
+    p.bases = s->d_views.as<BaseLayoutDev>() + b_first;
+    p.n_bases = n_bases;
+    p.b_offset = b_first;
+    p.P_total = s->P;
+    p.j_begin = j0;
+    p.j_end = j1;
+    p.seed = s->seed;
+    p.step = (uint64_t)s->step;
+    std::memcpy(p.mix, s->mix, sizeof p.mix);
+    p.allowed_op = g->d_allowed.as<uint8_t>();
+    p.keys = keys;
+    p.keys_dbg = keys_dbg;
+    if ((e = launch_nondelay(p, 1, grid, st)) != cudaSuccess) return cuda_fail(e, "launch non-delay search");
+    return PESTO_OK;
+}
+
 // fast: eval32 for the bases below saturation (+ eval64 for the others while any may exist);
 // otherwise (debug keys, initial makespans, ineligible graphs) eval64 for all candidates
 pesto_status launch_search_eval(pesto_search *s, int b_first, int n_bases, int64_t j0, int64_t j1,
@@ -140,6 +184,8 @@ pesto_status launch_search_eval(pesto_search *s, int b_first, int n_bases, int64
     if (j1 <= j0) return PESTO_OK;
     pesto_status rc0 = sync_constraints(s);
     if (rc0) return rc0;
+    if (g->dispatch == PESTO_DISPATCH_NONDELAY)
+        return launch_search_nondelay(s, b_first, n_bases, j0, j1, keys, keys_dbg, st);
     EvalParams p;
     fill_eval_common(g, p);
     p.feas.fbase = s->d_fbase.as<int64_t>() + (size_t)b_first * 8;

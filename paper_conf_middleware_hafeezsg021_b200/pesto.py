@@ -20,6 +20,7 @@ INFEASIBLE = (1 << 63) - 1
 KEY_INVALID = (1 << 64) - 1
 ORDER_CRITICAL_PATH, ORDER_FIFO, ORDER_RANDOM = 0, 1, 2
 LINKS_FCFS, LINKS_UNLIMITED = 0, 1
+DISPATCH_FIXED, DISPATCH_NONDELAY = 0, 1
 PLACE_SINGLE, PLACE_EXPERT, PLACE_TOPO_SPLIT, PLACE_RANDOM = 0, 1, 2, 3
 
 
@@ -60,6 +61,7 @@ SIGNATURES = {
     "pesto_graph_destroy": (None, [_VP]),
     "pesto_comm_model": (_I32, [_VP, _I32, _I32, _I64, _I64]),
     "pesto_graph_set_link_model": (_I32, [_VP, _I32]),
+    "pesto_graph_set_dispatch": (_I32, [_VP, _I32]),
     "pesto_graph_set_constraints": (_I32, [_VP, _VP, _VP, _VP]),
     "pesto_coarsen": (_I32, [_VP, _I32, _VP, _VP]),
     "pesto_eval_coarse_exhaustive": (_I32, [_VP, _VP, _VP, _I32, _VP, _VP, _VP, _VP]),
@@ -191,6 +193,10 @@ class Graph:
     def set_link_model(self, model: int):
         """LINKS_FCFS (default; serial FCFS queue per directed link) or LINKS_UNLIMITED."""
         _check(_L.pesto_graph_set_link_model(self._h, model))
+
+    def set_dispatch(self, mode: int):
+        """DISPATCH_FIXED (default; pi order per device) or DISPATCH_NONDELAY (row f4(i))."""
+        _check(_L.pesto_graph_set_dispatch(self._h, mode))
 
     def set_constraints(self, mem=None, cap=None, coloc=None):
         """Row f3: per-op footprint (None: input + output tensor bytes), per-device caps
