@@ -84,7 +84,7 @@ __device__ __forceinline__ int dev_of(const uint32_t *X, int words, int32_t v) {
 }
 
 template <int MODE, int PL>
-__global__ void __launch_bounds__(kNdMaxWarps * 32) nondelay_kernel(const NdParams P) {
+__global__ void __launch_bounds__(kNdMaxWarps * 32, 3) nondelay_kernel(const NdParams P) {
     extern __shared__ __align__(16) uint32_t nsm[];
     uint8_t *lclass = reinterpret_cast<uint8_t *>(nsm);
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
