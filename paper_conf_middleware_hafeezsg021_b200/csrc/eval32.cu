@@ -35,6 +35,20 @@ __device__ __forceinline__ uint32_t add_sat(uint32_t a, uint32_t b) {
 
 __host__ __device__ constexpr int warps_for(int cpl) { return cpl == 1 ? 8 : (cpl == 2 ? 4 : 2); }
 
+// TMA ring depth and the occupancy target (resident CTAs per SM the register allocation aims
+// for), per candidates-per-lane
+#ifndef PESTO_E32_STAGES
+#define PESTO_E32_STAGES 2
+#endif
+#ifndef PESTO_E32_MINB1
+#define PESTO_E32_MINB1 2
+#endif
+#ifndef PESTO_E32_MINB2
+#define PESTO_E32_MINB2 4
+#endif
+constexpr int kStages32 = PESTO_E32_STAGES;
+__host__ __device__ constexpr int min_blocks_for(int cpl) { return cpl == 1 ? PESTO_E32_MINB1 : PESTO_E32_MINB2; }
+
 // per-candidate device / link free times
 template <int CPL>
 struct RegState32 {          // D <= 2
@@ -53,6 +67,28 @@ struct RegState32 {          // D <= 2
         l01[c] = (cond && !x) ? v : l01[c];
     }
     __device__ __forceinline__ uint32_t makespan(int c) const { return max(d0[c], d1[c]); }
+    // warp-uniform device codes (search positions outside the group's region): branches on a
+    // uniform value instead of per-lane selects
+    __device__ __forceinline__ void begin_u(int xu, uint32_t p, const uint32_t (&r)[CPL],
+                                            uint32_t (&cc)[CPL]) {
+        if (xu) {
+#pragma unroll
+            for (int c = 0; c < CPL; c++) { cc[c] = min(max(r[c], d1[c]) + p, kSat32); d1[c] = cc[c]; }
+        } else {
+#pragma unroll
+            for (int c = 0; c < CPL; c++) { cc[c] = min(max(r[c], d0[c]) + p, kSat32); d0[c] = cc[c]; }
+        }
+    }
+    __device__ __forceinline__ void link_u(int xu, int, uint32_t t, const uint32_t (&cc)[CPL],
+                                           uint32_t (&a)[CPL]) {
+        if (xu) {
+#pragma unroll
+            for (int c = 0; c < CPL; c++) { a[c] = min(max(cc[c], l10[c]) + t, kSat32); l10[c] = a[c]; }
+        } else {
+#pragma unroll
+            for (int c = 0; c < CPL; c++) { a[c] = min(max(cc[c], l01[c]) + t, kSat32); l01[c] = a[c]; }
+        }
+    }
 };
 
 template <int CPL>
@@ -81,7 +117,78 @@ struct SmemState32 {         // D <= 8: [column][CPL][32] in shared memory (shar
         for (int x = 0; x < D; x++) m = max(m, lds_u32(at(d, x, c)));
         return m;
     }
+    __device__ __forceinline__ void begin_u(int xu, uint32_t p, const uint32_t (&r)[CPL],
+                                            uint32_t (&cc)[CPL]) {
+#pragma unroll
+        for (int c = 0; c < CPL; c++) {
+            const uint32_t a = at(d, xu, c);
+            cc[c] = min(max(r[c], lds_u32(a)) + p, kSat32);
+            sts_u32(a, cc[c]);
+        }
+    }
+    __device__ __forceinline__ void link_u(int xu, int yu, uint32_t t, const uint32_t (&cc)[CPL],
+                                           uint32_t (&a)[CPL]) {
+#pragma unroll
+        for (int c = 0; c < CPL; c++) {
+            const uint32_t ad = at(l, xu * D + yu, c);
+            a[c] = min(max(cc[c], lds_u32(ad)) + t, kSat32);
+            sts_u32(ad, a[c]);
+        }
+    }
 };
+
+// A lane move packed into two registers (the walk reads it only inside the 64-position region,
+// so the 13 words of a LaneMove need not stay live; for CPL = 2 that is 22 registers fewer).
+// Positions are offsets from the region start (0..63):
+//   w0: flip offsets 4 x 6 bits | nflip << 24 | kind << 27
+//   w1: flip devices 4 x 3 bits | window offset << 12 | window length << 18 | window device << 25
+struct PackedMove {
+    uint32_t w0, w1;
+};
+__device__ __forceinline__ PackedMove pack_move(const LaneMove &mv, int32_t rc) {
+    PackedMove p;
+    p.w0 = ((uint32_t)mv.nflip << 24) | ((uint32_t)mv.kind << 27);
+    p.w1 = 0u;
+#pragma unroll
+    for (int f = 0; f < 4; f++) {
+        if (f < mv.nflip) {
+            p.w0 |= (uint32_t)(mv.fpos[f] - rc) << (6 * f);
+            p.w1 |= (uint32_t)mv.fdev[f] << (3 * f);
+        }
+    }
+    if (mv.kind == kMoveWindow)
+        p.w1 |= ((uint32_t)(mv.ws - rc) << 12) | ((uint32_t)mv.wl << 18) | ((uint32_t)mv.wd << 25);
+    return p;
+}
+// = apply_lane (moves.cuh) for offset o = q - rc of a position inside the region
+__device__ __forceinline__ int apply_packed(const PackedMove &p, uint32_t o, int xb, unsigned aq) {
+    int x = xb;
+    const uint32_t kind = p.w0 >> 27;
+    if (kind == kMoveWindow) {
+        const uint32_t ws = (p.w1 >> 12) & 63u, wl = (p.w1 >> 18) & 127u, wd = (p.w1 >> 25) & 7u;
+        if (o - ws < wl && ((aq >> wd) & 1u)) x = (int)wd;
+    } else if (kind == kMoveFlip) {
+        const uint32_t nf = (p.w0 >> 24) & 7u;
+#pragma unroll
+        for (uint32_t f = 0; f < 4; f++)
+            if (f < nf && o == ((p.w0 >> (6 * f)) & 63u)) x = (int)((p.w1 >> (3 * f)) & 7u);
+    }
+    return x;
+}
+
+// the move as the walk keeps it: unpacked with one candidate per lane (registers are not the
+// limit there and the unpacked form applies with fewer instructions), packed with two
+__device__ __forceinline__ int apply_kept(const LaneMove &mv, int32_t q, int32_t, int xb, unsigned aq) {
+    return apply_lane(mv, q, xb, aq);
+}
+__device__ __forceinline__ int apply_kept(const PackedMove &mv, int32_t q, int32_t rc, int xb,
+                                          unsigned aq) {
+    return apply_packed(mv, (uint32_t)(q - rc), xb, aq);
+}
+__device__ __forceinline__ void keep_move(LaneMove &dst, const LaneMove &mv, int32_t) { dst = mv; }
+__device__ __forceinline__ void keep_move(PackedMove &dst, const LaneMove &mv, int32_t rc) {
+    dst = pack_move(mv, rc);
+}
 
 // devices of the lane's CPL candidates at position q; xb = the base code of the record naming q
 template <int MODE, int PL, int CPL>
@@ -91,7 +198,7 @@ struct Place32 {
     const uint8_t *allowed_pos;  // MODE 1: masks by position (window moves)
     int32_t rc, rlen;            // MODE 1: the group's region [rc, rc + rlen)
     int all_allowed, lane, dmax;
-    LaneMove mv[CPL];
+    typename std::conditional<CPL == 1, LaneMove, PackedMove>::type mv[CPL];
     const uint8_t *cpos;         // MODE 4: merged vertex of the op at each position
     int cbits;                   // MODE 4: bits per merged vertex in the candidate index
     uint32_t jc[CPL];            // MODE 4: the lane's candidate indices
@@ -112,7 +219,7 @@ struct Place32 {
         if ((uint32_t)(q - rc) < (uint32_t)rlen) {             // warp-uniform branch
             const unsigned aq = all_allowed ? 0xFFu : (unsigned)__ldg(allowed_pos + q);
 #pragma unroll
-            for (int c = 0; c < CPL; c++) x[c] = apply_lane(mv[c], q, xb, aq);
+            for (int c = 0; c < CPL; c++) x[c] = apply_kept(mv[c], q, rc, xb, aq);
         }
     }
 };
@@ -157,6 +264,10 @@ struct Ctx32 {
     int D;
 };
 
+template <int CPL>
+__device__ __forceinline__ void push_tail(const Ctx32 &cx, const uint32_t tgt,
+                                          const uint32_t (&a)[CPL], uint32_t (&fwd)[CPL]);
+
 // one out-edge record, for the lane's CPL candidates (FCFS link of L144 / L188-198)
 template <int PL, int CPL, class StateT>
 __device__ __forceinline__ void push32(const Ctx32 &cx, const uint4 rec, const int (&x)[CPL],
@@ -175,6 +286,13 @@ __device__ __forceinline__ void push32(const Ctx32 &cx, const uint4 rec, const i
         a[c] = cross ? ac : cc[c];
         st.set_link_if(c, x[c], y[c], cross, ac);
     }
+    push_tail<CPL>(cx, tgt, a, fwd);
+}
+
+// deliver the arrivals a[] of one edge: register (next position), near ring or cold slot
+template <int CPL>
+__device__ __forceinline__ void push_tail(const Ctx32 &cx, const uint32_t tgt,
+                                          const uint32_t (&a)[CPL], uint32_t (&fwd)[CPL]) {
     if (tgt & kT32Next) {                                    // consumer is the next position
 #pragma unroll
         for (int c = 0; c < CPL; c++) fwd[c] = max(fwd[c], a[c]);
@@ -197,6 +315,25 @@ __device__ __forceinline__ void push32(const Ctx32 &cx, const uint4 rec, const i
             else atomicMax(slot, a[c]);                          // RED.MAX, no reply awaited
         }
     }
+}
+
+// one out-edge whose producer and consumer devices are warp-uniform (xu, yu): a same-device
+// edge skips the link entirely (uniform branch), a crossing edge updates the one link xu -> yu
+template <int PL, int CPL, class StateT>
+__device__ __forceinline__ void push32_u(const Ctx32 &cx, const uint4 rec, int xu, int yu,
+                                         const uint32_t (&cc)[CPL], StateT &st,
+                                         uint32_t (&fwd)[CPL]) {
+    uint32_t a[CPL];
+    if (xu != yu) {
+        uint32_t t;
+        if constexpr (PL == 1) t = xu ? rec.w : rec.x;
+        else t = ((cx.cls1 >> (xu * cx.D + yu)) & 1u) ? rec.w : rec.x;
+        st.link_u(xu, yu, t, cc, a);
+    } else {
+#pragma unroll
+        for (int c = 0; c < CPL; c++) a[c] = cc[c];
+    }
+    push_tail<CPL>(cx, rec.z, a, fwd);
 }
 
 // the (up to two) out-edges of one step, records already in registers; yfn(k, rec, y) gives
@@ -231,7 +368,7 @@ __device__ __forceinline__ void begin32(const uint4 h, StateT &st, const uint32_
 }
 
 template <int MODE, int PL, int CPL>
-__global__ void __launch_bounds__((warps_for(CPL) + 1) * 32, 2)
+__global__ void __launch_bounds__((warps_for(CPL) + 1) * 32, min_blocks_for(CPL))
 eval32_kernel(const EvalParams P) {
     constexpr int NW = warps_for(CPL);          // consumer warps per CTA (256 candidates)
     constexpr int CW = 32 * CPL;                // candidates per warp
@@ -239,9 +376,9 @@ eval32_kernel(const EvalParams P) {
     // stage stride: the largest tile + one step of padding, so the walk may read the records of
     // the step after a tile's last one without leaving its own stage
     const int sb = P.stage_bytes32 + kStepBytes;
-    uint64_t *full = reinterpret_cast<uint64_t *>(smem + (size_t)kStages * sb);
-    uint64_t *empty = full + kStages;
-    uint8_t *cur = align16(reinterpret_cast<uint8_t *>(empty + kStages));
+    uint64_t *full = reinterpret_cast<uint64_t *>(smem + (size_t)kStages32 * sb);
+    uint64_t *empty = full + kStages32;
+    uint8_t *cur = align16(reinterpret_cast<uint8_t *>(empty + kStages32));
     uint32_t *ring_all = reinterpret_cast<uint32_t *>(cur);
     cur = align16(cur + (size_t)NW * kRing * CW * 4);
     uint32_t *stage_all = reinterpret_cast<uint32_t *>(cur);          // far-arrival staging
@@ -250,7 +387,7 @@ eval32_kernel(const EvalParams P) {
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     if (threadIdx.x == 0) {
-        for (int s = 0; s < kStages; s++) {
+        for (int s = 0; s < kStages32; s++) {
             mbar_init(&full[s], 1);
             mbar_init(&empty[s], NW);
         }
@@ -271,8 +408,8 @@ eval32_kernel(const EvalParams P) {
                 const BaseLayoutDev *B = &P.bases[bl];
                 const int nt = B->n_tiles32;
                 for (int t = 0; t < nt; t++, it++) {
-                    const int s = it % kStages;
-                    if (it >= (uint32_t)kStages) mbar_wait(&empty[s], ((it / kStages) - 1) & 1);
+                    const int s = it % kStages32;
+                    if (it >= (uint32_t)kStages32) mbar_wait(&empty[s], ((it / kStages32) - 1) & 1);
                     const TileDesc td = B->tiles32[t];
                     mbar_expect_tx(&full[s], (uint32_t)td.bytes);
                     bulk_g2s(smem + (size_t)s * sb, B->blob32 + td.byte_off, (uint32_t)td.bytes,
@@ -396,18 +533,19 @@ eval32_kernel(const EvalParams P) {
             for (int c = 0; c < CPL; c++) {
                 const int64_t j = j0 + c * 32 + lane;
                 const bool in_range = active && j >= P.j_begin && j < P.j_end;
-                place.mv[c] = in_range
+                LaneMove mv = in_range
                     ? decode_lane(P.seed, cb, j, ks >= 0 && (j & (kGroup - 1)) == 0, P.D, P.mix, rg,
                                   [&](int32_t q) { return __ldg(ord + q); },
                                   [&](int32_t q) { return ldg_bits_dev_at<PL>(bits, words, q); },
                                   [&](int32_t op) { return (unsigned)__ldg(aop + op); })
                     : no_move();
-                valid[c] = in_range && place.mv[c].kind != kMoveInvalid;
-                if (place.mv[c].kind == kMoveInvalid) place.mv[c] = no_move();
+                valid[c] = in_range && mv.kind != kMoveInvalid;
+                if (mv.kind == kMoveInvalid) mv = no_move();
                 if (valid[c] && (P.feas.has_cap || P.feas.has_coloc))   // row f3
-                    valid[c] = move_feasible<PL>(place.mv[c], rg, P.D, bits, words, ord,
+                    valid[c] = move_feasible<PL>(mv, rg, P.D, bits, words, ord,
                                                  B->allowed_pos, P.all_allowed, P.feas,
                                                  P.feas.fbase + (size_t)bl * 8);
+                keep_move(place.mv[c], mv, rg.c);
             }
         }
         st.init();
@@ -468,10 +606,11 @@ eval32_kernel(const EvalParams P) {
             }
         }
         int32_t v = -1;
+        int xu = -1;                 // search: the walked op's device if warp-uniform, else -1
         int32_t skip = 0;            // steps of the next tile already walked (swap pair)
         for (int t = 0; t < nt; t++, it++) {
-            const int s = it % kStages;
-            mbar_wait(&full[s], (it / kStages) & 1);
+            const int s = it % kStages32;
+            mbar_wait(&full[s], (it / kStages32) & 1);
             if (active) {
                 const uint32_t tile = (uint32_t)s * sb;
                 const int32_t nsteps = (int32_t)lds_u32(cx.smem + tile);
@@ -504,8 +643,8 @@ eval32_kernel(const EvalParams P) {
                             const bool straddle = i + nk >= nsteps;
                             uint32_t sp1;
                             if (straddle) {
-                                const int s2 = (it + 1) % kStages;
-                                mbar_wait(&full[s2], ((it + 1) / kStages) & 1);
+                                const int s2 = (it + 1) % kStages32;
+                                mbar_wait(&full[s2], ((it + 1) / kStages32) & 1);
                                 sp1 = cx.smem + (uint32_t)s2 * sb + kTileHeader;
                             } else {
                                 sp1 = sp + (uint32_t)nk * kStepBytes;
@@ -539,6 +678,7 @@ eval32_kernel(const EvalParams P) {
                                                  cc, place_y, st, fwd);
                             }
                             v++;
+                            xu = -1;
                             load_next(v + 1, nfar, nnear);
                             if (straddle) {
                                 skip = n1;
@@ -574,15 +714,38 @@ eval32_kernel(const EvalParams P) {
                                 x[c] = plane_dev<PL>(w, lane, place.dmax);
                             }
                         } else {
+                            // outside the group's region every lane has the base device
+                            // (CPL = 2 only: with one candidate per lane the launch is
+                            // latency-bound and the branch-free selects schedule better)
+                            xu = (MODE == 1 && CPL == 2 &&
+                                  (uint32_t)(v - place.rc) >= (uint32_t)place.rlen)
+                                     ? (int)(h.w & kStXMask) : -1;
                             place.at(v, (int)(h.w & kStXMask), x);
                         }
-                        begin32<CPL>(h, st, r, x, cc);
+                        if (MODE != 0 && xu >= 0) st.begin_u(xu, h.x, r, cc);
+                        else begin32<CPL>(h, st, r, x, cc);
                     }
                     if constexpr (MODE == 0) {
                         edges32<PL, CPL>(cx, h.w, e0, e1, x, cc, pw_y, st, fwd);
                         slot0 += 2;
                     } else {
-                        edges32<PL, CPL>(cx, h.w, e0, e1, x, cc, place_y, st, fwd);
+                        const uint32_t ne = (h.w >> kStEdgeShift) & 3u;
+                        if (xu >= 0) {
+                            if (ne >= 1) {
+                                const int32_t q0 = (int32_t)(e0.y & kSuccPosMask);
+                                if ((uint32_t)(q0 - place.rc) >= (uint32_t)place.rlen)
+                                    push32_u<PL, CPL>(cx, e0, xu, (int)((e0.y >> kSuccXShift) & 7u), cc, st, fwd);
+                                else { int y[CPL]; place_y(0, e0, y); push32<PL, CPL>(cx, e0, x, y, cc, st, fwd); }
+                            }
+                            if (ne >= 2) {
+                                const int32_t q1 = (int32_t)(e1.y & kSuccPosMask);
+                                if ((uint32_t)(q1 - place.rc) >= (uint32_t)place.rlen)
+                                    push32_u<PL, CPL>(cx, e1, xu, (int)((e1.y >> kSuccXShift) & 7u), cc, st, fwd);
+                                else { int y[CPL]; place_y(1, e1, y); push32<PL, CPL>(cx, e1, x, y, cc, st, fwd); }
+                            }
+                        } else {
+                            edges32<PL, CPL>(cx, h.w, e0, e1, x, cc, place_y, st, fwd);
+                        }
                     }
                     sp += kStepBytes;
                     i++;
@@ -659,7 +822,7 @@ int eval32_smem_bytes(const EvalParams &p, int search_mode) {
     const int cpl = p.cpl32 == 1 ? 1 : 2;
     const int nw = warps_for(cpl);
     const int pl = planes_of32(p.D);
-    size_t b = (size_t)kStages * (p.stage_bytes32 + kStepBytes) + 2 * kStages * 8;
+    size_t b = (size_t)kStages32 * (p.stage_bytes32 + kStepBytes) + 2 * kStages32 * 8;
     b = (b + 15) & ~size_t(15);
     b += (size_t)nw * kRing * 32 * cpl * 4;        // near ring
     b = (b + 15) & ~size_t(15);

@@ -13,7 +13,8 @@ from typing import Optional, Sequence
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libpesto.so")
+# PESTO_LIB: an alternative in-tree build of the same library (tuning experiments, scripts/)
+LIB_PATH = os.environ.get("PESTO_LIB") or os.path.join(_HERE, "libpesto.so")
 
 OK, EINVAL, ECYCLE, ENOTTOPO, EOVERFLOW, ENOMEM, ECUDA, ENCCL, ESTATE = range(9)
 INFEASIBLE = (1 << 63) - 1
