@@ -250,14 +250,13 @@ pesto_status pesto_eval_coarse_exhaustive(pesto_graph *g, const int32_t *order,
     p.max_W32 = L->W32;
     p.bases = L->d_view.as<BaseLayoutDev>();
     p.n_cand = total;
-    p.tasks_per_base = (total + 255) / 256;
-    p.n_tasks = p.tasks_per_base;
+
     p.keys = g->d_ckey.as<uint64_t>();
     p.coarse_pos = g->d_cpos.as<uint8_t>();
     p.coarse_bits = b;
     p.n_coarse = n_coarse;
     std::copy(cmask.begin(), cmask.end(), p.coarse_allowed);
-    p.cpl32 = choose_cpl32(g, p.n_tasks);
+    plan_eval32(g, p, 0, total, 1);
     int grid = 0;
     if ((s = ensure_state32(g, p, 4, p.n_tasks, &grid))) return s;
     p.state32 = g->d_state32.as<uint32_t>();

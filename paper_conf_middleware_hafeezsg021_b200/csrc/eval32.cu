@@ -33,7 +33,13 @@ __device__ __forceinline__ uint32_t add_sat(uint32_t a, uint32_t b) {
     return min(a + b, kSat32);                 // a <= kSat32, b < kMaxDur32: never wraps
 }
 
-__host__ __device__ constexpr int warps_for(int cpl) { return cpl == 1 ? 8 : (cpl == 2 ? 4 : 2); }
+// consumer warps per CTA: 256 candidates either way.  (Measured: 2-warp CTAs for CPL = 1, to
+// spread inception's 2,048 warps evenly over the SMs, fit only 6 CTAs per SM by registers and
+// shared memory, so the launch needed two waves: 5.84 -> 10.14 ms.)
+#ifndef PESTO_E32_W1
+#define PESTO_E32_W1 8
+#endif
+__host__ __device__ constexpr int warps_for(int cpl) { return cpl == 1 ? PESTO_E32_W1 : 4; }
 
 // TMA ring depth and the occupancy target (resident CTAs per SM the register allocation aims
 // for), per candidates-per-lane
@@ -475,8 +481,9 @@ eval32_kernel(const EvalParams P) {
         const int64_t local = MODE == 1 ? task % P.tasks_per_base : task;
         const BaseLayoutDev *B = &P.bases[bl];
         const int nt = B->n_tiles32;
-        // a task = 256 consecutive candidate ids starting at a multiple of 256; a warp = CW of them
-        const int64_t j0 = (MODE == 1 ? (P.j_begin & ~(int64_t)255) : 0) + local * 256 + warp * CW;
+        // a task = TS consecutive candidate ids starting at a multiple of TS; a warp = CW of them
+        constexpr int64_t TS = (int64_t)NW * CW;
+        const int64_t j0 = (MODE == 1 ? (P.j_begin & ~(TS - 1)) : 0) + local * TS + warp * CW;
         const int64_t gw = j0 >> 5;                                 // first 32-row group
 
         Place32<MODE, PL, CPL> place;
@@ -816,6 +823,8 @@ int occupancy_one32(const EvalParams &p) {
 int planes_of32(int D) { return D <= 2 ? 1 : (D <= 4 ? 2 : 4); }
 
 }  // namespace
+
+int eval32_task_size(int cpl) { return warps_for(cpl) * 32 * cpl; }
 
 int eval32_smem_bytes(const EvalParams &p, int search_mode) {
     (void)search_mode;

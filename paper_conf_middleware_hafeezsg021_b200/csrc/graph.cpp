@@ -282,6 +282,14 @@ int choose_cpl32(const pesto_graph *g, int64_t n_tasks) {
     return n_tasks <= 2 * (int64_t)g->sms ? 1 : 2;
 }
 
+void plan_eval32(const pesto_graph *g, EvalParams &p, int64_t j0, int64_t j1, int n_bases) {
+    const int64_t t256 = (j1 - (j0 & ~(int64_t)255) + 255) / 256 * n_bases;
+    p.cpl32 = choose_cpl32(g, t256);
+    const int64_t ts = eval32_task_size(p.cpl32);
+    p.tasks_per_base = (j1 - (j0 & ~(ts - 1)) + ts - 1) / ts;
+    p.n_tasks = p.tasks_per_base * n_bases;
+}
+
 pesto_status ensure_state32(pesto_graph *g, const EvalParams &p, int search_mode, int64_t n_tasks,
                             int *grid_out) {
     int per_sm = eval32_max_ctas_per_sm(p, search_mode);
@@ -290,7 +298,7 @@ pesto_status ensure_state32(pesto_graph *g, const EvalParams &p, int search_mode
                                      std::to_string(eval32_smem_bytes(p, search_mode)) + " B)");
     int64_t grid = std::min<int64_t>(n_tasks, (int64_t)g->sms * per_sm);
     grid = std::max<int64_t>(grid, 1);
-    size_t bytes = (size_t)grid * kWarps * (size_t)std::max(p.max_W32, 1) * 32 * sizeof(uint32_t);
+    size_t bytes = (size_t)grid * eval32_task_size(p.cpl32) * (size_t)std::max(p.max_W32, 1) * sizeof(uint32_t);
     cudaError_t e = g->d_state32.ensure(bytes);
     if (e != cudaSuccess) return cuda_fail(e, "allocate cold slot state");
     *grid_out = (int)grid;
@@ -806,10 +814,13 @@ pesto_status pesto_eval_batch(pesto_graph *g, const int32_t *order, const void *
     if ((e = cudaMemsetAsync(g->d_flags.ptr, 0, 4, st)) != cudaSuccess) return cuda_fail(e, "reset flags");
     p.flag_count = g->d_flags.as<int32_t>();
     p.flag_list = g->d_flags.as<int32_t>() + 4;
-    p.cpl32 = choose_cpl32(g, p.n_tasks);
-    if ((s = ensure_state32(g, p, 0, p.n_tasks, &grid))) return s;
-    p.state32 = g->d_state32.as<uint32_t>();
-    if ((e = launch_eval32(p, 0, grid, st)) != cudaSuccess) return cuda_fail(e, "launch eval32");
+    {
+        EvalParams p32 = p;
+        plan_eval32(g, p32, 0, n_cand, 1);
+        if ((s = ensure_state32(g, p32, 0, p32.n_tasks, &grid))) return s;
+        p32.state32 = g->d_state32.as<uint32_t>();
+        if ((e = launch_eval32(p32, 0, grid, st)) != cudaSuccess) return cuda_fail(e, "launch eval32");
+    }
     p.list = p.flag_list;
     p.list_count = p.flag_count;
     const int64_t fix_tasks = std::min<int64_t>(p.n_tasks, g->sms);

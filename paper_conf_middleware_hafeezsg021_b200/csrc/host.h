@@ -152,6 +152,9 @@ pesto_status ensure_state(pesto_graph *g, const EvalParams &p, int search_mode, 
 // eval32 candidates per lane for a launch of n_tasks 256-candidate tasks:
 // 1 when every task is resident at once (latency-bound: more warps), else 2
 int choose_cpl32(const pesto_graph *g, int64_t n_tasks);
+// eval32 launch plan for candidate ids [j0, j1) of n_bases bases: p.cpl32 (from the launch size
+// in 256-candidate units), p.tasks_per_base and p.n_tasks in tasks of eval32_task_size(cpl)
+void plan_eval32(const pesto_graph *g, EvalParams &p, int64_t j0, int64_t j1, int n_bases);
 pesto_status ensure_state32(pesto_graph *g, const EvalParams &p, int search_mode, int64_t n_tasks,
                             int *grid_out);
 struct DeviceGuard {

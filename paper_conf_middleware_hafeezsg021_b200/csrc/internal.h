@@ -192,6 +192,8 @@ cudaError_t launch_patch(const PatchOp *ops_dev, int n_ops, int max_block, cudaS
 cudaError_t launch_eval(const EvalParams &p, int search_mode, int grid, cudaStream_t st);
 cudaError_t launch_eval32(const EvalParams &p, int search_mode, int grid, cudaStream_t st);
 int eval32_smem_bytes(const EvalParams &p, int search_mode);
+// candidate ids per eval32 task (one CTA's share) for CPL candidates per lane
+int eval32_task_size(int cpl);
 int eval32_max_ctas_per_sm(const EvalParams &p, int search_mode);
 cudaError_t launch_transpose(const TransposeParams &p, cudaStream_t st);
 cudaError_t launch_feasibility(const FeasParams &p, cudaStream_t st);

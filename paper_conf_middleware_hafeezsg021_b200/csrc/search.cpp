@@ -217,12 +217,10 @@ pesto_status launch_search_eval(pesto_search *s, int b_first, int n_bases, int64
     const bool use32 = fast && s->use32 && keys_dbg == nullptr &&
                        g->link_model == PESTO_LINKS_FCFS;   // f4(ii) runs on eval64
     if (use32) {
-        // eval32 tasks: 256 consecutive ids starting at a multiple of 256
+        // eval32 tasks: consecutive ids from a multiple of the task size
         EvalParams p32 = p;
         p32.gate = 1;
-        p32.tasks_per_base = (j1 - (j0 & ~(int64_t)255) + 255) / 256;
-        p32.n_tasks = p32.tasks_per_base * n_bases;
-        p32.cpl32 = choose_cpl32(g, p32.n_tasks);
+        plan_eval32(g, p32, j0, j1, n_bases);
         if ((rc = ensure_state32(g, p32, 1, p32.n_tasks, &grid))) return rc;
         p32.state32 = g->d_state32.as<uint32_t>();
         if ((e = launch_eval32(p32, 1, grid, st)) != cudaSuccess) return cuda_fail(e, "launch eval32");
