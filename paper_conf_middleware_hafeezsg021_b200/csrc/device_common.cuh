@@ -113,6 +113,10 @@ __device__ __forceinline__ void cp_async4_zfill(uint32_t smem_addr, const void *
     asm volatile("cp.async.ca.shared.global [%0], [%1], 4, %2;\n"
                  ::"r"(smem_addr), "l"(gptr), "r"(have ? 4 : 0) : "memory");
 }
+__device__ __forceinline__ void cp_async8_zfill(uint32_t smem_addr, const void *gptr, bool have) {
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;\n"
+                 ::"r"(smem_addr), "l"(gptr), "r"(have ? 8 : 0) : "memory");
+}
 __device__ __forceinline__ void cp_async_commit() {
     asm volatile("cp.async.commit_group;" ::: "memory");
 }

@@ -32,6 +32,18 @@ using namespace dev;
 __device__ __forceinline__ uint32_t add_sat(uint32_t a, uint32_t b) {
     return min(a + b, kSat32);                 // a <= kSat32, b < kMaxDur32: never wraps
 }
+// The walk's time type T: uint32 saturating at kSat32 (the fast path) or uint64 exact (the
+// "wide" instance, for search bases whose makespan is >= kSat32: same records, same kernel,
+// 8-byte state; exact because every time is < 2^40, the ingest guard).
+__device__ __forceinline__ uint64_t add_sat(uint64_t a, uint64_t b) { return a + b; }
+template <class T> __device__ __forceinline__ T lds_t(uint32_t addr);
+template <> __device__ __forceinline__ uint32_t lds_t<uint32_t>(uint32_t addr) { return lds_u32(addr); }
+template <> __device__ __forceinline__ uint64_t lds_t<uint64_t>(uint32_t addr) { return lds_u64(addr); }
+__device__ __forceinline__ void sts_t(uint32_t addr, uint32_t v) { sts_u32(addr, v); }
+__device__ __forceinline__ void sts_t(uint32_t addr, uint64_t v) { sts_u64(addr, v); }
+// bytes of one 32-lane column of T; record slot offsets are written for 4-byte columns
+template <class T> constexpr uint32_t kColB = 32u * sizeof(T);
+template <class T> constexpr uint32_t kSc = sizeof(T) / 4u;
 
 // consumer warps per CTA: 256 candidates either way.  (Measured: 2-warp CTAs for CPL = 1, to
 // spread inception's 2,048 warps evenly over the SMs, fit only 6 CTAs per SM by registers and
@@ -56,89 +68,85 @@ constexpr int kStages32 = PESTO_E32_STAGES;
 __host__ __device__ constexpr int min_blocks_for(int cpl) { return cpl == 1 ? PESTO_E32_MINB1 : PESTO_E32_MINB2; }
 
 // per-candidate device / link free times
-template <int CPL>
+template <int CPL, class T>
 struct RegState32 {          // D <= 2
-    uint32_t d0[CPL], d1[CPL], l01[CPL], l10[CPL];
+    T d0[CPL], d1[CPL], l01[CPL], l10[CPL];
     __device__ __forceinline__ void init() {
 #pragma unroll
         for (int c = 0; c < CPL; c++) d0[c] = d1[c] = l01[c] = l10[c] = 0u;
     }
-    __device__ __forceinline__ uint32_t dev(int c, int x) const { return x ? d1[c] : d0[c]; }
-    __device__ __forceinline__ void set_dev(int c, int x, uint32_t v) {
+    __device__ __forceinline__ T dev(int c, int x) const { return x ? d1[c] : d0[c]; }
+    __device__ __forceinline__ void set_dev(int c, int x, T v) {
         if (x) d1[c] = v; else d0[c] = v;
     }
-    __device__ __forceinline__ uint32_t link(int c, int x, int) const { return x ? l10[c] : l01[c]; }
-    __device__ __forceinline__ void set_link_if(int c, int x, int, bool cond, uint32_t v) {
+    __device__ __forceinline__ T link(int c, int x, int) const { return x ? l10[c] : l01[c]; }
+    __device__ __forceinline__ void set_link_if(int c, int x, int, bool cond, T v) {
         l10[c] = (cond && x) ? v : l10[c];
         l01[c] = (cond && !x) ? v : l01[c];
     }
-    __device__ __forceinline__ uint32_t makespan(int c) const { return max(d0[c], d1[c]); }
+    __device__ __forceinline__ T makespan(int c) const { return max(d0[c], d1[c]); }
     // warp-uniform device codes (search positions outside the group's region): branches on a
     // uniform value instead of per-lane selects
-    __device__ __forceinline__ void begin_u(int xu, uint32_t p, const uint32_t (&r)[CPL],
-                                            uint32_t (&cc)[CPL]) {
+    __device__ __forceinline__ void begin_u(int xu, uint32_t p, const T (&r)[CPL], T (&cc)[CPL]) {
         if (xu) {
 #pragma unroll
-            for (int c = 0; c < CPL; c++) { cc[c] = min(max(r[c], d1[c]) + p, kSat32); d1[c] = cc[c]; }
+            for (int c = 0; c < CPL; c++) { cc[c] = add_sat(max(r[c], d1[c]), (T)p); d1[c] = cc[c]; }
         } else {
 #pragma unroll
-            for (int c = 0; c < CPL; c++) { cc[c] = min(max(r[c], d0[c]) + p, kSat32); d0[c] = cc[c]; }
+            for (int c = 0; c < CPL; c++) { cc[c] = add_sat(max(r[c], d0[c]), (T)p); d0[c] = cc[c]; }
         }
     }
-    __device__ __forceinline__ void link_u(int xu, int, uint32_t t, const uint32_t (&cc)[CPL],
-                                           uint32_t (&a)[CPL]) {
+    __device__ __forceinline__ void link_u(int xu, int, uint32_t t, const T (&cc)[CPL], T (&a)[CPL]) {
         if (xu) {
 #pragma unroll
-            for (int c = 0; c < CPL; c++) { a[c] = min(max(cc[c], l10[c]) + t, kSat32); l10[c] = a[c]; }
+            for (int c = 0; c < CPL; c++) { a[c] = add_sat(max(cc[c], l10[c]), (T)t); l10[c] = a[c]; }
         } else {
 #pragma unroll
-            for (int c = 0; c < CPL; c++) { a[c] = min(max(cc[c], l01[c]) + t, kSat32); l01[c] = a[c]; }
+            for (int c = 0; c < CPL; c++) { a[c] = add_sat(max(cc[c], l01[c]), (T)t); l01[c] = a[c]; }
         }
     }
 };
 
-template <int CPL>
+template <int CPL, class T>
 struct SmemState32 {         // D <= 8: [column][CPL][32] in shared memory (shared addresses)
-    uint32_t d, l;           // + lane * 4
+    uint32_t d, l;           // + lane * sizeof(T)
     int D;
     __device__ __forceinline__ uint32_t at(uint32_t base, int col, int c) const {
-        return base + (uint32_t)(col * CPL + c) * 128;
+        return base + (uint32_t)(col * CPL + c) * kColB<T>;
     }
     __device__ __forceinline__ void init() {
         for (int x = 0; x < D; x++)
-            for (int c = 0; c < CPL; c++) sts_u32(at(d, x, c), 0u);
+            for (int c = 0; c < CPL; c++) sts_t(at(d, x, c), (T)0);
         for (int x = 0; x < D * D; x++)
-            for (int c = 0; c < CPL; c++) sts_u32(at(l, x, c), 0u);
+            for (int c = 0; c < CPL; c++) sts_t(at(l, x, c), (T)0);
     }
-    __device__ __forceinline__ uint32_t dev(int c, int x) const { return lds_u32(at(d, x, c)); }
-    __device__ __forceinline__ void set_dev(int c, int x, uint32_t v) { sts_u32(at(d, x, c), v); }
-    __device__ __forceinline__ uint32_t link(int c, int x, int y) const {
-        return lds_u32(at(l, x * D + y, c));
+    __device__ __forceinline__ T dev(int c, int x) const { return lds_t<T>(at(d, x, c)); }
+    __device__ __forceinline__ void set_dev(int c, int x, T v) { sts_t(at(d, x, c), v); }
+    __device__ __forceinline__ T link(int c, int x, int y) const {
+        return lds_t<T>(at(l, x * D + y, c));
     }
-    __device__ __forceinline__ void set_link_if(int c, int x, int y, bool cond, uint32_t v) {
-        if (cond) sts_u32(at(l, x * D + y, c), v);
+    __device__ __forceinline__ void set_link_if(int c, int x, int y, bool cond, T v) {
+        if (cond) sts_t(at(l, x * D + y, c), v);
     }
-    __device__ __forceinline__ uint32_t makespan(int c) const {
-        uint32_t m = 0;
-        for (int x = 0; x < D; x++) m = max(m, lds_u32(at(d, x, c)));
+    __device__ __forceinline__ T makespan(int c) const {
+        T m = 0;
+        for (int x = 0; x < D; x++) m = max(m, lds_t<T>(at(d, x, c)));
         return m;
     }
-    __device__ __forceinline__ void begin_u(int xu, uint32_t p, const uint32_t (&r)[CPL],
-                                            uint32_t (&cc)[CPL]) {
+    __device__ __forceinline__ void begin_u(int xu, uint32_t p, const T (&r)[CPL], T (&cc)[CPL]) {
 #pragma unroll
         for (int c = 0; c < CPL; c++) {
             const uint32_t a = at(d, xu, c);
-            cc[c] = min(max(r[c], lds_u32(a)) + p, kSat32);
-            sts_u32(a, cc[c]);
+            cc[c] = add_sat(max(r[c], lds_t<T>(a)), (T)p);
+            sts_t(a, cc[c]);
         }
     }
-    __device__ __forceinline__ void link_u(int xu, int yu, uint32_t t, const uint32_t (&cc)[CPL],
-                                           uint32_t (&a)[CPL]) {
+    __device__ __forceinline__ void link_u(int xu, int yu, uint32_t t, const T (&cc)[CPL], T (&a)[CPL]) {
 #pragma unroll
         for (int c = 0; c < CPL; c++) {
             const uint32_t ad = at(l, xu * D + yu, c);
-            a[c] = min(max(cc[c], lds_u32(ad)) + t, kSat32);
-            sts_u32(ad, a[c]);
+            a[c] = add_sat(max(cc[c], lds_t<T>(ad)), (T)t);
+            sts_t(ad, a[c]);
         }
     }
 };
@@ -270,17 +278,17 @@ struct Ctx32 {
     int D;
 };
 
-template <int CPL>
-__device__ __forceinline__ void push_tail(const Ctx32 &cx, const uint32_t tgt,
-                                          const uint32_t (&a)[CPL], uint32_t (&fwd)[CPL]);
+template <int CPL, class T>
+__device__ __forceinline__ void push_tail(const Ctx32 &cx, const uint32_t tgt, const T (&a)[CPL],
+                                          T (&fwd)[CPL]);
 
 // one out-edge record, for the lane's CPL candidates (FCFS link of L144 / L188-198)
-template <int PL, int CPL, class StateT>
+template <int PL, int CPL, class T, class StateT>
 __device__ __forceinline__ void push32(const Ctx32 &cx, const uint4 rec, const int (&x)[CPL],
-                                       const int (&y)[CPL], const uint32_t (&cc)[CPL],
-                                       StateT &st, uint32_t (&fwd)[CPL]) {
+                                       const int (&y)[CPL], const T (&cc)[CPL],
+                                       StateT &st, T (&fwd)[CPL]) {
     const uint32_t tgt = rec.z;
-    uint32_t a[CPL];
+    T a[CPL];
 #pragma unroll
     for (int c = 0; c < CPL; c++) {
         const bool cross = y[c] != x[c];                     // cross: FCFS link x -> y
@@ -288,48 +296,48 @@ __device__ __forceinline__ void push32(const Ctx32 &cx, const uint4 rec, const i
         if constexpr (PL == 1) t = x[c] ? rec.w : rec.x;     // D = 2: t by direction
         else t = ((cx.cls1 >> (x[c] * cx.D + y[c])) & 1u) ? rec.w : rec.x;
         // branch-free: the transfer's arrival when crossing, C_v (L144) when not
-        const uint32_t ac = add_sat(max(cc[c], st.link(c, x[c], y[c])), t);
+        const T ac = add_sat(max(cc[c], st.link(c, x[c], y[c])), (T)t);
         a[c] = cross ? ac : cc[c];
         st.set_link_if(c, x[c], y[c], cross, ac);
     }
-    push_tail<CPL>(cx, tgt, a, fwd);
+    push_tail<CPL, T>(cx, tgt, a, fwd);
 }
 
 // deliver the arrivals a[] of one edge: register (next position), near ring or cold slot
-template <int CPL>
-__device__ __forceinline__ void push_tail(const Ctx32 &cx, const uint32_t tgt,
-                                          const uint32_t (&a)[CPL], uint32_t (&fwd)[CPL]) {
+template <int CPL, class T>
+__device__ __forceinline__ void push_tail(const Ctx32 &cx, const uint32_t tgt, const T (&a)[CPL],
+                                          T (&fwd)[CPL]) {
     if (tgt & kT32Next) {                                    // consumer is the next position
 #pragma unroll
         for (int c = 0; c < CPL; c++) fwd[c] = max(fwd[c], a[c]);
         return;
     }
-    const uint32_t bytes = (tgt & kT32SlotMask) * CPL;
+    const uint32_t bytes = (tgt & kT32SlotMask) * CPL * kSc<T>;
     if (tgt & kT32Near) {
 #pragma unroll
         for (int c = 0; c < CPL; c++) {
-            const uint32_t slot = cx.ring + bytes + c * 128;
-            uint32_t v = a[c];
-            if (!(tgt & kT32First)) v = max(v, lds_u32(slot));
-            sts_u32(slot, v);
+            const uint32_t slot = cx.ring + bytes + c * kColB<T>;
+            T v = a[c];
+            if (!(tgt & kT32First)) v = max(v, lds_t<T>(slot));
+            sts_t(slot, v);
         }
     } else {
 #pragma unroll
         for (int c = 0; c < CPL; c++) {
-            uint32_t *slot = reinterpret_cast<uint32_t *>(cx.cold + bytes + c * 128);
+            T *slot = reinterpret_cast<T *>(cx.cold + bytes + c * kColB<T>);
             if (tgt & kT32First) *slot = a[c];                   // first far push: plain store
-            else atomicMax(slot, a[c]);                          // RED.MAX, no reply awaited
+            else if constexpr (sizeof(T) == 4) atomicMax(slot, a[c]);   // RED.MAX, no reply
+            else atomicMax(reinterpret_cast<unsigned long long *>(slot), (unsigned long long)a[c]);
         }
     }
 }
 
 // one out-edge whose producer and consumer devices are warp-uniform (xu, yu): a same-device
 // edge skips the link entirely (uniform branch), a crossing edge updates the one link xu -> yu
-template <int PL, int CPL, class StateT>
+template <int PL, int CPL, class T, class StateT>
 __device__ __forceinline__ void push32_u(const Ctx32 &cx, const uint4 rec, int xu, int yu,
-                                         const uint32_t (&cc)[CPL], StateT &st,
-                                         uint32_t (&fwd)[CPL]) {
-    uint32_t a[CPL];
+                                         const T (&cc)[CPL], StateT &st, T (&fwd)[CPL]) {
+    T a[CPL];
     if (xu != yu) {
         uint32_t t;
         if constexpr (PL == 1) t = xu ? rec.w : rec.x;
@@ -339,41 +347,41 @@ __device__ __forceinline__ void push32_u(const Ctx32 &cx, const uint4 rec, int x
 #pragma unroll
         for (int c = 0; c < CPL; c++) a[c] = cc[c];
     }
-    push_tail<CPL>(cx, rec.z, a, fwd);
+    push_tail<CPL, T>(cx, rec.z, a, fwd);
 }
 
 // the (up to two) out-edges of one step, records already in registers; yfn(k, rec, y) gives
 // the successor's devices of edge k
-template <int PL, int CPL, class YFn, class StateT>
+template <int PL, int CPL, class T, class YFn, class StateT>
 __device__ __forceinline__ void edges32(const Ctx32 &cx, uint32_t flags, const uint4 e0,
                                         const uint4 e1, const int (&x)[CPL],
-                                        const uint32_t (&cc)[CPL], const YFn &yfn,
-                                        StateT &st, uint32_t (&fwd)[CPL]) {
+                                        const T (&cc)[CPL], const YFn &yfn,
+                                        StateT &st, T (&fwd)[CPL]) {
     const uint32_t ne = (flags >> kStEdgeShift) & 3u;
     if (ne >= 1) {
         int y[CPL];
         yfn(0, e0, y);
-        push32<PL, CPL>(cx, e0, x, y, cc, st, fwd);
+        push32<PL, CPL, T>(cx, e0, x, y, cc, st, fwd);
     }
     if (ne >= 2) {
         int y[CPL];
         yfn(1, e1, y);
-        push32<PL, CPL>(cx, e1, x, y, cc, st, fwd);
+        push32<PL, CPL, T>(cx, e1, x, y, cc, st, fwd);
     }
 }
 
 // start the op at position v (head h, devices x) whose arrivals are r[c]: S_v, C_v (L142-146)
-template <int CPL, class StateT>
-__device__ __forceinline__ void begin32(const uint4 h, StateT &st, const uint32_t (&r)[CPL],
-                                        const int (&x)[CPL], uint32_t (&cc)[CPL]) {
+template <int CPL, class T, class StateT>
+__device__ __forceinline__ void begin32(const uint4 h, StateT &st, const T (&r)[CPL],
+                                        const int (&x)[CPL], T (&cc)[CPL]) {
 #pragma unroll
     for (int c = 0; c < CPL; c++) {
-        cc[c] = add_sat(max(r[c], st.dev(c, x[c])), h.x);    // C_v = S_v + p_v
+        cc[c] = add_sat(max(r[c], st.dev(c, x[c])), (T)h.x);  // C_v = S_v + p_v
         st.set_dev(c, x[c], cc[c]);
     }
 }
 
-template <int MODE, int PL, int CPL>
+template <int MODE, int PL, int CPL, class T>
 __global__ void __launch_bounds__((warps_for(CPL) + 1) * 32, min_blocks_for(CPL))
 eval32_kernel(const EvalParams P) {
     constexpr int NW = warps_for(CPL);          // consumer warps per CTA (256 candidates)
@@ -385,11 +393,11 @@ eval32_kernel(const EvalParams P) {
     uint64_t *full = reinterpret_cast<uint64_t *>(smem + (size_t)kStages32 * sb);
     uint64_t *empty = full + kStages32;
     uint8_t *cur = align16(reinterpret_cast<uint8_t *>(empty + kStages32));
-    uint32_t *ring_all = reinterpret_cast<uint32_t *>(cur);
-    cur = align16(cur + (size_t)NW * kRing * CW * 4);
-    uint32_t *stage_all = reinterpret_cast<uint32_t *>(cur);          // far-arrival staging
-    cur = align16(cur + (size_t)NW * kRing * CW * 4);
-    uint32_t *dstate = reinterpret_cast<uint32_t *>(cur);
+    T *ring_all = reinterpret_cast<T *>(cur);
+    cur = align16(cur + (size_t)NW * kRing * CW * sizeof(T));
+    T *stage_all = reinterpret_cast<T *>(cur);                        // far-arrival staging
+    cur = align16(cur + (size_t)NW * kRing * CW * sizeof(T));
+    T *dstate = reinterpret_cast<T *>(cur);
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     if (threadIdx.x == 0) {
@@ -402,7 +410,9 @@ eval32_kernel(const EvalParams P) {
     __syncthreads();
 
     auto runs_here = [&](int bl) {           // search: this kernel owns bases below saturation
-        return MODE != 1 || P.gate == 0 || P.base_mk[bl] < (int64_t)kSat32;
+        // (the wide instance, gate 2, owns the bases at or above saturation)
+        return MODE != 1 || P.gate == 0 ||
+               (P.gate == 1 ? P.base_mk[bl] < (int64_t)kSat32 : P.base_mk[bl] >= (int64_t)kSat32);
     };
 
     if (warp == NW) {
@@ -429,19 +439,20 @@ eval32_kernel(const EvalParams P) {
     Ctx32 cx;
     cx.smem = su32_reg(smem);
     cx.ring = su32_reg(ring_all + (size_t)warp * kRing * CW + lane);
-    cx.cold = reinterpret_cast<uint8_t *>(P.state32 + ((size_t)(blockIdx.x * NW + warp) * P.max_W32) * CW + lane);
+    cx.cold = reinterpret_cast<uint8_t *>(reinterpret_cast<T *>(P.state32) +
+                                          ((size_t)(blockIdx.x * NW + warp) * P.max_W32) * CW + lane);
     cx.D = P.D;
     cx.cls1 = 0;
     for (int i = 0; i < P.D * P.D; i++)
         if (P.link_class[i] == 1) cx.cls1 |= 1ull << i;
     const uint32_t stage = su32_reg(stage_all + (size_t)warp * kRing * CW + lane);
 
-    using StateT = typename std::conditional<PL == 1, RegState32<CPL>, SmemState32<CPL>>::type;
+    using StateT = typename std::conditional<PL == 1, RegState32<CPL, T>, SmemState32<CPL, T>>::type;
     StateT st;
     if constexpr (PL != 1) {
         st.D = P.D;
         st.d = su32_reg(dstate + (size_t)warp * (P.D + P.D * P.D) * CW + lane);
-        st.l = st.d + (uint32_t)(P.D * CPL) * 128;
+        st.l = st.d + (uint32_t)(P.D * CPL) * kColB<T>;
     }
 
     // Far arrivals of position q arrive by cp.async into stage[q & 15] (zero when q has no far
@@ -449,29 +460,32 @@ eval32_kernel(const EvalParams P) {
     // commit group per position.  Only positions > kNearDelta have far producers, so the first
     // positions of a task need no prefetch.
     auto issue_far = [&](const uint4 h, int32_t v) {
-        const uint32_t dst = stage + (uint32_t)(((v + kPrefetchDist) & (kRing - 1)) * CPL) * 128;
+        const uint32_t dst = stage + (uint32_t)(((v + kPrefetchDist) & (kRing - 1)) * CPL) * kColB<T>;
         const bool have = (int32_t)h.z >= 0;
-        const uint8_t *src = cx.cold + (size_t)(have ? h.z : 0) * CW * 4;
+        const uint8_t *src = cx.cold + (size_t)(have ? h.z : 0) * CW * sizeof(T);
 #pragma unroll
-        for (int c = 0; c < CPL; c++) cp_async4_zfill(dst + c * 128, src + c * 128, have);
+        for (int c = 0; c < CPL; c++) {
+            if constexpr (sizeof(T) == 4) cp_async4_zfill(dst + c * kColB<T>, src + c * kColB<T>, have);
+            else cp_async8_zfill(dst + c * kColB<T>, src + c * kColB<T>, have);
+        }
         cp_async_commit();
     };
     // The arrivals of position q from far producers (stage) and near producers (ring) are final
     // once the op at q - 1 starts (a distance-1 producer forwards in `fwd`), so they are read one
     // op ahead, off the critical path: nfar/nnear hold them for the next position.
-    auto load_next = [&](int32_t q, uint32_t (&nfar)[CPL], uint32_t (&nnear)[CPL]) {
-        const uint32_t o = (uint32_t)((q & (kRing - 1)) * CPL) * 128;
+    auto load_next = [&](int32_t q, T (&nfar)[CPL], T (&nnear)[CPL]) {
+        const uint32_t o = (uint32_t)((q & (kRing - 1)) * CPL) * kColB<T>;
 #pragma unroll
         for (int c = 0; c < CPL; c++) {
-            nfar[c] = lds_u32(stage + o + c * 128);
-            nnear[c] = lds_u32(cx.ring + o + c * 128);
+            nfar[c] = lds_t<T>(stage + o + c * kColB<T>);
+            nnear[c] = lds_t<T>(cx.ring + o + c * kColB<T>);
         }
     };
-    auto arrivals = [&](uint32_t flags, const uint32_t (&nfar)[CPL], const uint32_t (&nnear)[CPL],
-                        const uint32_t (&fwd)[CPL], uint32_t (&r)[CPL]) {
+    auto arrivals = [&](uint32_t flags, const T (&nfar)[CPL], const T (&nnear)[CPL],
+                        const T (&fwd)[CPL], T (&r)[CPL]) {
         const bool near = (flags & kStHasNear) != 0;          // else the ring slot is stale
 #pragma unroll
-        for (int c = 0; c < CPL; c++) r[c] = max(max(nfar[c], fwd[c]), near ? nnear[c] : 0u);
+        for (int c = 0; c < CPL; c++) r[c] = max(max(nfar[c], fwd[c]), near ? nnear[c] : (T)0);
     };
 
     uint32_t it = 0;
@@ -558,12 +572,12 @@ eval32_kernel(const EvalParams P) {
         st.init();
         // positions 0 .. kPrefetchDist - 1 are never prefetched (they have no far producer)
 #pragma unroll
-        for (int q = 0; q < kRing * CPL; q++) sts_u32(stage + q * 128, 0u);
+        for (int q = 0; q < kRing * CPL; q++) sts_t(stage + q * kColB<T>, (T)0);
 
         // the op being walked (its devices and C_v), the arrivals it forwards to v + 1, and the
         // far / near arrivals of v + 1 read ahead
         int x[CPL];
-        uint32_t cc[CPL], fwd[CPL], nfar[CPL], nnear[CPL];
+        T cc[CPL], fwd[CPL], nfar[CPL], nnear[CPL];
 #pragma unroll
         for (int c = 0; c < CPL; c++) { x[c] = 0; cc[c] = 0u; fwd[c] = 0u; nfar[c] = 0u; nnear[c] = 0u; }
         // devices by direct lookup (search: base code + region moves; rows: plane words)
@@ -661,7 +675,7 @@ eval32_kernel(const EvalParams P) {
                             issue_far(h, v);
                             issue_far(h1, v + 1);
                             cp_async_wait<kPrefetchDist - 1>();  // v+1 and v+2 have landed
-                            uint32_t r0[CPL], r1[CPL], f1[CPL], g1[CPL], zero[CPL];
+                            T r0[CPL], r1[CPL], f1[CPL], g1[CPL], zero[CPL];
 #pragma unroll
                             for (int c = 0; c < CPL; c++) zero[c] = 0u;
                             arrivals(h.w, nfar, nnear, fwd, r0);
@@ -670,18 +684,18 @@ eval32_kernel(const EvalParams P) {
 #pragma unroll
                             for (int c = 0; c < CPL; c++) fwd[c] = 0u;
                             place.at(v + 1, (int)(h1.w & kStXMask), x);
-                            begin32<CPL>(h1, st, r1, x, cc);
+                            begin32<CPL, T>(h1, st, r1, x, cc);
                             for (int32_t q = 0; q < n1; q++) {
                                 const uint32_t a = sp1 + q * kStepBytes;
-                                edges32<PL, CPL>(cx, lds_u32(a + 12), lds_v4(a + 16), lds_v4(a + 32), x,
+                                edges32<PL, CPL, T>(cx, lds_u32(a + 12), lds_v4(a + 16), lds_v4(a + 32), x,
                                                  cc, place_y, st, fwd);
                             }
                             place.at(v, (int)(h.w & kStXMask), x);
-                            begin32<CPL>(h, st, r0, x, cc);
-                            edges32<PL, CPL>(cx, h.w, e0, e1, x, cc, place_y, st, fwd);
+                            begin32<CPL, T>(h, st, r0, x, cc);
+                            edges32<PL, CPL, T>(cx, h.w, e0, e1, x, cc, place_y, st, fwd);
                             for (int32_t q = 1; q < nk; q++) {
                                 const uint32_t a = sp + q * kStepBytes;
-                                edges32<PL, CPL>(cx, lds_u32(a + 12), lds_v4(a + 16), lds_v4(a + 32), x,
+                                edges32<PL, CPL, T>(cx, lds_u32(a + 12), lds_v4(a + 16), lds_v4(a + 32), x,
                                                  cc, place_y, st, fwd);
                             }
                             v++;
@@ -700,7 +714,7 @@ eval32_kernel(const EvalParams P) {
                         }
                         issue_far(h, v);
                         cp_async_wait<kPrefetchDist - 1>();      // v+1 has landed
-                        uint32_t r[CPL];
+                        T r[CPL];
                         arrivals(h.w, nfar, nnear, fwd, r);
                         load_next(v + 1, nfar, nnear);
 #pragma unroll
@@ -730,10 +744,10 @@ eval32_kernel(const EvalParams P) {
                             place.at(v, (int)(h.w & kStXMask), x);
                         }
                         if (MODE != 0 && xu >= 0) st.begin_u(xu, h.x, r, cc);
-                        else begin32<CPL>(h, st, r, x, cc);
+                        else begin32<CPL, T>(h, st, r, x, cc);
                     }
                     if constexpr (MODE == 0) {
-                        edges32<PL, CPL>(cx, h.w, e0, e1, x, cc, pw_y, st, fwd);
+                        edges32<PL, CPL, T>(cx, h.w, e0, e1, x, cc, pw_y, st, fwd);
                         slot0 += 2;
                     } else {
                         const uint32_t ne = (h.w >> kStEdgeShift) & 3u;
@@ -741,17 +755,17 @@ eval32_kernel(const EvalParams P) {
                             if (ne >= 1) {
                                 const int32_t q0 = (int32_t)(e0.y & kSuccPosMask);
                                 if ((uint32_t)(q0 - place.rc) >= (uint32_t)place.rlen)
-                                    push32_u<PL, CPL>(cx, e0, xu, (int)((e0.y >> kSuccXShift) & 7u), cc, st, fwd);
-                                else { int y[CPL]; place_y(0, e0, y); push32<PL, CPL>(cx, e0, x, y, cc, st, fwd); }
+                                    push32_u<PL, CPL, T>(cx, e0, xu, (int)((e0.y >> kSuccXShift) & 7u), cc, st, fwd);
+                                else { int y[CPL]; place_y(0, e0, y); push32<PL, CPL, T>(cx, e0, x, y, cc, st, fwd); }
                             }
                             if (ne >= 2) {
                                 const int32_t q1 = (int32_t)(e1.y & kSuccPosMask);
                                 if ((uint32_t)(q1 - place.rc) >= (uint32_t)place.rlen)
-                                    push32_u<PL, CPL>(cx, e1, xu, (int)((e1.y >> kSuccXShift) & 7u), cc, st, fwd);
-                                else { int y[CPL]; place_y(1, e1, y); push32<PL, CPL>(cx, e1, x, y, cc, st, fwd); }
+                                    push32_u<PL, CPL, T>(cx, e1, xu, (int)((e1.y >> kSuccXShift) & 7u), cc, st, fwd);
+                                else { int y[CPL]; place_y(1, e1, y); push32<PL, CPL, T>(cx, e1, x, y, cc, st, fwd); }
                             }
                         } else {
-                            edges32<PL, CPL>(cx, h.w, e0, e1, x, cc, place_y, st, fwd);
+                            edges32<PL, CPL, T>(cx, h.w, e0, e1, x, cc, place_y, st, fwd);
                         }
                     }
                     sp += kStepBytes;
@@ -770,7 +784,7 @@ eval32_kernel(const EvalParams P) {
             for (int c = 0; c < CPL; c++) {
                 const int64_t j = j0 + c * 32 + lane;
                 if (j >= P.n_cand) continue;
-                const uint32_t mk = st.makespan(c);
+                const uint64_t mk = (uint64_t)st.makespan(c);
                 if (!valid[c]) {
                     P.makespans[j] = INT64_MAX;
                 } else if (mk < kSat32) {
@@ -798,9 +812,18 @@ eval32_kernel(const EvalParams P) {
 }
 
 template <int MODE, int PL, int CPL>
+auto kernel_for(const EvalParams &p) {
+    // the wide (exact 64-bit) instance serves search bases at or above saturation only
+    if constexpr (MODE == 1) {
+        if (p.wide32) return eval32_kernel<MODE, PL, CPL, uint64_t>;
+    }
+    return eval32_kernel<MODE, PL, CPL, uint32_t>;
+}
+
+template <int MODE, int PL, int CPL>
 cudaError_t launch_one32(const EvalParams &p, int grid, cudaStream_t st) {
     const int smem = eval32_smem_bytes(p, MODE);
-    auto kern = eval32_kernel<MODE, PL, CPL>;
+    auto kern = kernel_for<MODE, PL, CPL>(p);
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     if (e != cudaSuccess) return e;
     kern<<<grid, (warps_for(CPL) + 1) * 32, smem, st>>>(p);
@@ -810,7 +833,7 @@ cudaError_t launch_one32(const EvalParams &p, int grid, cudaStream_t st) {
 template <int MODE, int PL, int CPL>
 int occupancy_one32(const EvalParams &p) {
     const int smem = eval32_smem_bytes(p, MODE);
-    auto kern = eval32_kernel<MODE, PL, CPL>;
+    auto kern = kernel_for<MODE, PL, CPL>(p);
     if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) != cudaSuccess)
         return 0;
     int n = 0;
@@ -827,17 +850,17 @@ int planes_of32(int D) { return D <= 2 ? 1 : (D <= 4 ? 2 : 4); }
 int eval32_task_size(int cpl) { return warps_for(cpl) * 32 * cpl; }
 
 int eval32_smem_bytes(const EvalParams &p, int search_mode) {
-    (void)search_mode;
     const int cpl = p.cpl32 == 1 ? 1 : 2;
     const int nw = warps_for(cpl);
     const int pl = planes_of32(p.D);
+    const size_t tb = (search_mode == 1 && p.wide32) ? 8 : 4;   // bytes per time value
     size_t b = (size_t)kStages32 * (p.stage_bytes32 + kStepBytes) + 2 * kStages32 * 8;
     b = (b + 15) & ~size_t(15);
-    b += (size_t)nw * kRing * 32 * cpl * 4;        // near ring
+    b += (size_t)nw * kRing * 32 * cpl * tb;       // near ring
     b = (b + 15) & ~size_t(15);
-    b += (size_t)nw * kRing * 32 * cpl * 4;        // far-arrival staging
+    b += (size_t)nw * kRing * 32 * cpl * tb;       // far-arrival staging
     b = (b + 15) & ~size_t(15);
-    if (pl != 1) b += (size_t)nw * (p.D + p.D * p.D) * 32 * cpl * 4;
+    if (pl != 1) b += (size_t)nw * (p.D + p.D * p.D) * 32 * cpl * tb;
     return (int)b + 128;
 }
 

@@ -298,7 +298,8 @@ pesto_status ensure_state32(pesto_graph *g, const EvalParams &p, int search_mode
                                      std::to_string(eval32_smem_bytes(p, search_mode)) + " B)");
     int64_t grid = std::min<int64_t>(n_tasks, (int64_t)g->sms * per_sm);
     grid = std::max<int64_t>(grid, 1);
-    size_t bytes = (size_t)grid * eval32_task_size(p.cpl32) * (size_t)std::max(p.max_W32, 1) * sizeof(uint32_t);
+    size_t bytes = (size_t)grid * eval32_task_size(p.cpl32) * (size_t)std::max(p.max_W32, 1) *
+                   (p.wide32 ? sizeof(uint64_t) : sizeof(uint32_t));
     cudaError_t e = g->d_state32.ensure(bytes);
     if (e != cudaSuccess) return cuda_fail(e, "allocate cold slot state");
     *grid_out = (int)grid;

@@ -89,6 +89,9 @@ struct EvalParams {
     int32_t gate;
     // eval32 candidates per lane (1 or 2): more warps vs. more work per warp instruction
     int32_t cpl32;
+    // eval32 search (mode 1): 1 = the wide instance (exact 64-bit times, same records) for the
+    // bases at or above saturation (gate 2)
+    int32_t wide32;
     // 1: FCFS link queues; 0: congestion-free links (row f4(ii))
     int32_t link_queue;
     // row f3 feasibility (search mode prologue): memory caps and colocation

@@ -225,7 +225,14 @@ pesto_status launch_search_eval(pesto_search *s, int b_first, int n_bases, int64
         p32.state32 = g->d_state32.as<uint32_t>();
         if ((e = launch_eval32(p32, 1, grid, st)) != cudaSuccess) return cuda_fail(e, "launch eval32");
         if (s->all_below) return PESTO_OK;
-        p.gate = 2;
+        // bases at or above saturation: the wide eval32 instance (exact 64-bit times, the
+        // same step records) -- about 2x the throughput of eval64 there
+        p32.gate = 2;
+        p32.wide32 = 1;
+        if ((rc = ensure_state32(g, p32, 1, p32.n_tasks, &grid))) return rc;
+        p32.state32 = g->d_state32.as<uint32_t>();
+        if ((e = launch_eval32(p32, 1, grid, st)) != cudaSuccess) return cuda_fail(e, "launch wide eval32");
+        return PESTO_OK;
     }
     if ((rc = ensure_state(g, p, 1, p.n_tasks, &grid))) return rc;
     p.state = g->d_state.as<int64_t>();

@@ -133,6 +133,31 @@ def test_search_with_bases_above_saturation(P, O):
             assert mk == rmk[b] and (x == rx[b]).all() and (o == ro[b]).all(), (step, b)
 
 
+@pytest.mark.parametrize("D,mix", [(2, (50, 20, 20, 10)), (4, (30, 10, 10, 50))])
+def test_wide_eval32_bases_above_saturation(P, O, D, mix):
+    """bases above 4.03 s run on the wide (exact 64-bit) eval32 instance: each step's argmin key
+    equals the minimum of the oracle's keys over every candidate, over several steps."""
+    g = dag.random_dag(57 + D, 900, 1.5, D=D, p_max=30_000_000, zero_frac=0.0, max_bytes=1 << 22,
+                       beta0=20_000, beta1_fs=400_000)
+    g.p[:] = np.maximum(g.p, 5_000_000 * D)
+    G = P.Graph.from_arrays(g)
+    xs, orders = _bases(g, 2, seed=21)
+    K = 1024
+    S = P.Search(G, xs, orders, K, mix, seed=6)
+    rx, ro = xs.copy(), orders.copy()
+    rmk = np.asarray([O.makespan(g, rx[b], ro[b]) for b in range(2)], np.int64)
+    assert (rmk > 0xF0000000).all()
+    for step in range(3):
+        S.eval()
+        got = S.keys()
+        keys = O.search_step(g, rx, ro, rmk, K, 6, step, mix)
+        assert (got == keys).all(), (step, got, keys)
+        S.commit()
+        for b in range(2):
+            mk, x, o = S.get(b)
+            assert mk == rmk[b] and (x == rx[b]).all() and (o == ro[b]).all(), (step, b)
+
+
 @pytest.mark.parametrize("name", ["inception_v3_2dev", "nmt4_2dev_commheavy",
                                   "transformer_2dev", "transformer_4dev_8gpu"])
 def test_full_size_sampled(P, O, name):
