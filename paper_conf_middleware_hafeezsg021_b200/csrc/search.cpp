@@ -7,6 +7,7 @@
 #include <nccl.h>
 
 #include <algorithm>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 
@@ -229,6 +230,16 @@ pesto_status launch_search_eval(pesto_search *s, int b_first, int n_bases, int64
         // same step records) -- about 2x the throughput of eval64 there
         p32.gate = 2;
         p32.wide32 = 1;
+        // one candidate per lane: the 64-bit state of two would spill at 4 CTAs/SM (measured on
+        // nmt4: CPL 1 5.17 vs CPL 2 4.96 M cand/s); PESTO_WIDE_CPL overrides for experiments
+        {
+            const char *w = std::getenv("PESTO_WIDE_CPL");
+            const int c = (w && std::atoi(w) == 2) ? 2 : 1;
+            p32.cpl32 = c;
+            const int64_t ts = eval32_task_size(c);
+            p32.tasks_per_base = (j1 - (j0 & ~(ts - 1)) + ts - 1) / ts;
+            p32.n_tasks = p32.tasks_per_base * n_bases;
+        }
         if ((rc = ensure_state32(g, p32, 1, p32.n_tasks, &grid))) return rc;
         p32.state32 = g->d_state32.as<uint32_t>();
         if ((e = launch_eval32(p32, 1, grid, st)) != cudaSuccess) return cuda_fail(e, "launch wide eval32");
