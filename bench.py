@@ -331,6 +331,22 @@ def run_pesto(args, rank, world, local):
                          "source": os.path.relpath(prof, ROOT)}
         except Exception:
             traffic = None
+    # SURVEY §8(d) issue roof: 148 SMs x 4 warp-instr/clk at sm_max_mhz, at the survey's
+    # estimate of 2 warp instructions per op-relaxation; the measured instructions per
+    # op-relaxation come from the ncu capture of the same kernel (profiles/)
+    issue_peak = 148 * 4 * sm_mhz * 1e6
+    op_relax_k1 = k_gpu * g.n / eval_avg_s
+    issue_roof = {"unit": "op-relax/s", "achieved": op_relax_k1, "peak": issue_peak / 2.0,
+                  "frac": op_relax_k1 / (issue_peak / 2.0),
+                  "peak_source": "148 SMs x 4 warp-instr/clk x sm_max_mhz / 2 warp-instr per "
+                                 "op-relax (SURVEY 8(d) estimate)",
+                  "measured_warp_instr_per_op_relax": None}
+    if issue is not None:
+        try:
+            inst = json.load(open(prof))["metrics"]["smsp__inst_executed.sum"]["value"]
+            issue_roof["measured_warp_instr_per_op_relax"] = inst / (k_gpu * g.n)
+        except Exception:
+            pass
     st = G.stats(orders[0])
     line = {"metric": METRIC, "value": value, "unit": "candidates/s", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": tot_ms / args.steps,
@@ -351,6 +367,7 @@ def run_pesto(args, rank, world, local):
                          "kernel": "nondelay_kernel (row f4(i))" if nd else "eval32_kernel (K1)",
                          "note": "algorithmic int ops (2n+m+2*cross per candidate) / K1 time; "
                                  "traffic = ncu DRAM bytes per K1 launch (profiles/)"},
+            "issue_roof": issue_roof,
             "gpu_launches": int(launches),
             "wall_s_timed_region": wall,
             "search": {"seed_makespans": seed_mk, "best_makespans": best_mk,
