@@ -229,6 +229,10 @@ pesto_status nd_fill(pesto_graph *g, NdParams &p, int64_t n_tasks, int *grid_out
     if (per_sm <= 0) return fail(PESTO_ECUDA, "non-delay kernel does not fit on an SM");
     int64_t grid = std::min<int64_t>((n_tasks + p.warps_per_cta - 1) / p.warps_per_cta,
                                      (int64_t)g->sms * per_sm);
+    if (const char *e = std::getenv("PESTO_ND_MAX_WARPS")) {     // tuning experiments
+        const int64_t w = std::atoll(e);
+        if (w > 0) grid = std::min<int64_t>(grid, std::max<int64_t>(1, w / p.warps_per_cta));
+    }
     grid = std::max<int64_t>(grid, 1);
     const size_t slots = (size_t)grid * p.warps_per_cta;
     cudaError_t e;

@@ -1,11 +1,7 @@
 cd $GRAFT_REPO_ROOT
 mkdir -p gpurun_out
 : > gpurun_out/quick.log
-for v in base pp; do
-  if [ $v = base ]; then L=""; else L=paper_conf_middleware_hafeezsg021_b200/libpesto_$v.so; fi
-  for c in inception_v3_2dev transformer_2dev; do
-    r=$(PESTO_LIB=$L timeout 300 python bench.py --config $c --steps 10 --warmup 3 --no-cpu-baseline --no-e2e 2>&1 | grep '^{' | tail -1 | python -c "import json,sys; d=json.loads(sys.stdin.read()); print(round(d['value']/1e6,3), round(d['eval_kernel_ms'],2))" 2>&1)
-    echo "$v $c $r" >> gpurun_out/quick.log
-  done
+for w in 0 600 1200 2400; do
+    r=$(PESTO_ND_MAX_WARPS=$w timeout 300 python scripts/time_nondelay.py inception_v3_2dev 8192 2>&1 | tail -1)
+    echo "maxwarps=$w $r" >> gpurun_out/quick.log
 done
-PESTO_LIB=paper_conf_middleware_hafeezsg021_b200/libpesto_pp.so timeout 1200 python -m pytest tests/test_gpu_parity.py -q -x > gpurun_out/pytest_pp.log 2>&1; echo "rc=$?" >> gpurun_out/pytest_pp.log
