@@ -296,6 +296,45 @@ __global__ void __launch_bounds__(kNdMaxWarps * 32, 3) nondelay_kernel(const NdP
             // ---- out-edges: FCFS prefix sums per link, arrivals, newly eligible ops ----
             const int64_t e0 = __ldg(reinterpret_cast<const long long *>(P.out_off) + v);
             const int64_t e1 = __ldg(reinterpret_cast<const long long *>(P.out_off) + v + 1);
+            if (e1 - e0 == 1) {
+                // a single out-edge (most ops): every lane computes the same values and lane 0
+                // stores them -- one edge cannot race, so no atomics, no ballots, no scan
+                const int32_t w = __ldg(edst + e0);
+                const int y = dev_of<PL>(X, words, w);
+                int64_t A = C;                                   // same device: C_v (L144)
+                if (y != d) {
+                    const int64_t t = __ldg(reinterpret_cast<const long long *>(et) +
+                                            e0 * P.n_classes + lclass[d * D + y]);
+                    if (P.link_queue) {                          // FCFS link d -> y
+                        const int li = d * D + y;
+                        const int64_t lf = __shfl_sync(kFull, li < 32 ? lk0 : lk1, li & 31);
+                        A = max(C, lf) + t;
+                        if (lane == (li & 31)) {
+                            if (li < 32) lk0 = A;
+                            else lk1 = A;
+                        }
+                    } else {
+                        A = C + t;                               // congestion-free (L113)
+                    }
+                }
+                const int64_t r = max((int64_t)__ldcg(reinterpret_cast<const long long *>(rdy + w)), A);
+                const int32_t rm = __ldcg(rem + w) - 1;
+                if (lane == 0) {
+                    __stcg(reinterpret_cast<long long *>(rdy + w), (long long)r);
+                    __stcg(rem + w, rm);
+                }
+                const int64_t fy = __shfl_sync(kFull, f, y & 31);
+                if (rm == 0) {
+                    const uint32_t pw = prio_of(w);
+                    if (r <= fy) {
+                        if (lane == 0) bm(y).set(pw);
+                    } else {
+                        heap_push(y, nd_key(r, pw, y));
+                    }
+                }
+                __syncwarp();
+                continue;
+            }
             for (int64_t b0 = e0; b0 < e1; b0 += 32) {
                 const int64_t i = b0 + lane;
                 const bool in = i < e1;
