@@ -174,3 +174,15 @@ def test_coarsen_matches_oracle(P):
     assert nc == rn == 8000 and (co == ro).all()
     with pytest.raises(P.PestoError):
         _host_graph(P, g).coarsen(0)
+
+
+def test_dispatch_and_link_model_validation(P):
+    """pesto_graph_set_dispatch / set_link_model accept their enums only (pesto.h)."""
+    g = dag.random_dag(5, 30, 1.5, D=2, beta0=10, beta1_fs=100)
+    G = _host_graph(P, g)
+    G.set_dispatch(P.DISPATCH_NONDELAY)
+    G.set_dispatch(P.DISPATCH_FIXED)
+    with pytest.raises(P.PestoError):
+        G.set_dispatch(2)
+    with pytest.raises(P.PestoError):
+        G.set_link_model(5)
