@@ -497,7 +497,7 @@ eval32_kernel(const EvalParams P) {
         const int nt = B->n_tiles32;
         // a task = TS consecutive candidate ids starting at a multiple of TS; a warp = CW of them
         constexpr int64_t TS = (int64_t)NW * CW;
-        const int64_t j0 = (MODE == 1 ? (P.j_begin & ~(TS - 1)) : 0) + local * TS + warp * CW;
+        const int64_t j0 = (MODE == 1 ? P.j_begin - P.j_begin % TS : 0) + local * TS + warp * CW;
         const int64_t gw = j0 >> 5;                                 // first 32-row group
 
         Place32<MODE, PL, CPL> place;

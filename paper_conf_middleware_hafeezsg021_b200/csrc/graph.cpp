@@ -287,10 +287,12 @@ int choose_cpl32(const pesto_graph *g, int64_t n_tasks) {
 }
 
 void plan_eval32(const pesto_graph *g, EvalParams &p, int64_t j0, int64_t j1, int n_bases) {
-    const int64_t t256 = (j1 - (j0 & ~(int64_t)255) + 255) / 256 * n_bases;
-    p.cpl32 = choose_cpl32(g, t256);
+    // CPL 1 when its tasks fit in one wave of 2 CTAs per SM (latency-bound: more warps), else 2
+    const int64_t ts1 = eval32_task_size(1);
+    const int64_t t1 = (j1 - (j0 - j0 % ts1) + ts1 - 1) / ts1 * n_bases;
+    p.cpl32 = choose_cpl32(g, t1);
     const int64_t ts = eval32_task_size(p.cpl32);
-    p.tasks_per_base = (j1 - (j0 & ~(ts - 1)) + ts - 1) / ts;
+    p.tasks_per_base = (j1 - (j0 - j0 % ts) + ts - 1) / ts;
     p.n_tasks = p.tasks_per_base * n_bases;
 }
 

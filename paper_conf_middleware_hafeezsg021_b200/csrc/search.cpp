@@ -237,7 +237,7 @@ pesto_status launch_search_eval(pesto_search *s, int b_first, int n_bases, int64
             const int c = (w && std::atoi(w) == 2) ? 2 : 1;
             p32.cpl32 = c;
             const int64_t ts = eval32_task_size(c);
-            p32.tasks_per_base = (j1 - (j0 & ~(ts - 1)) + ts - 1) / ts;
+            p32.tasks_per_base = (j1 - (j0 - j0 % ts) + ts - 1) / ts;
             p32.n_tasks = p32.tasks_per_base * n_bases;
         }
         if ((rc = ensure_state32(g, p32, 1, p32.n_tasks, &grid))) return rc;
