@@ -702,6 +702,35 @@ static int32_t alt_devices(const uint8_t *allowed, int32_t D, int32_t v, int32_t
     return c;
 }
 
+/* group moves over merged vertices (row f2, DESIGN §4 S9): global, test infrastructure */
+static struct {
+    int active;
+    int32_t n, n_coarse, pct;
+    int32_t *coarse_of;
+} g_coarse;
+
+void oracle_clear_coarse_moves(void) {
+    free(g_coarse.coarse_of);
+    memset(&g_coarse, 0, sizeof g_coarse);
+}
+
+int oracle_set_coarse_moves(int32_t n, const int32_t *coarse_of, int32_t n_coarse, int32_t pct) {
+    oracle_clear_coarse_moves();
+    if (n < 1 || n_coarse < 1 || n_coarse > 255 || pct < 0 || pct > 100 || !coarse_of)
+        return ORACLE_EINVAL;
+    g_coarse.coarse_of = malloc((size_t)n * sizeof(int32_t));
+    if (!g_coarse.coarse_of) return ORACLE_ENOMEM;
+    for (int32_t v = 0; v < n; v++) {
+        if (coarse_of[v] < 0 || coarse_of[v] >= n_coarse) { oracle_clear_coarse_moves(); return ORACLE_EINVAL; }
+        g_coarse.coarse_of[v] = coarse_of[v];
+    }
+    g_coarse.n = n;
+    g_coarse.n_coarse = n_coarse;
+    g_coarse.pct = pct;
+    g_coarse.active = 1;
+    return 0;
+}
+
 int oracle_candidate(int32_t n, int64_t m, const int32_t *src, const int32_t *dst, int32_t D,
                      const uint8_t *allowed, int32_t P, int32_t b, const uint8_t *base_x,
                      const int32_t *base_order, int64_t j, uint64_t seed, uint64_t step,
@@ -711,6 +740,17 @@ int oracle_candidate(int32_t n, int64_t m, const int32_t *src, const int32_t *ds
     memcpy(x_out, bx, (size_t)n);
     memcpy(order_out, bo, (size_t)n * sizeof(int32_t));
     int64_t g = j >> 7, lane = j & 127;      /* groups of 128 candidate ids (DESIGN §4 S2) */
+    /* S9: a coarse group moves one merged vertex per candidate and nothing else: vertex
+       k = draw(j, 10) mod n_coarse goes to device d = draw(j, 11) mod D (each of its ops whose
+       mask allows d); no order move, no region moves */
+    if (g_coarse.active && g_coarse.n == n && g != 0 && g_coarse.pct > 0 &&
+        (int64_t)(oracle_draw(seed, step, P, b, 128 * g, 12) % 100u) < g_coarse.pct) {
+        int32_t k = (int32_t)(oracle_draw(seed, step, P, b, j, 10) % (uint64_t)g_coarse.n_coarse);
+        int32_t d = (int32_t)(oracle_draw(seed, step, P, b, j, 11) % (uint64_t)D);
+        for (int32_t v = 0; v < n; v++)
+            if (g_coarse.coarse_of[v] == k && allowed_dev(allowed, v, d)) x_out[v] = (uint8_t)d;
+        return 1;
+    }
     int swap = 0;
     /* the group's region: positions [c, c + len) of the base order (DESIGN §4 S2) */
     int64_t c0 = (int64_t)(oracle_draw(seed, step, P, b, 128 * g, 13) % (uint64_t)n);

@@ -117,6 +117,14 @@ int64_t oracle_bruteforce(int32_t n, const int64_t *p, int64_t m, const int32_t 
 uint64_t oracle_mix64(uint64_t z);
 uint64_t oracle_draw(uint64_t seed, uint64_t step, int32_t P, int32_t b, int64_t j, int32_t k);
 
+/* Group moves over merged vertices (row f2; DESIGN.md §4 S9): while set, a coarse group of the
+ * search (draw(128g, 12) mod 100 < pct, g != 0) moves, per candidate j, every op of merged vertex
+ * draw(j, 10) mod n_coarse that allows device draw(j, 11) mod D to that device, and nothing
+ * else.  coarse_of [n] in [0, n_coarse), n_coarse <= 255.  Global (test infrastructure); applies
+ * to calls with the same n.  Returns 0 or ORACLE_EINVAL. */
+int oracle_set_coarse_moves(int32_t n, const int32_t *coarse_of, int32_t n_coarse, int32_t pct);
+void oracle_clear_coarse_moves(void);
+
 /* Decode candidate j of base b into (x_out, order_out); returns 1 valid, 0 invalid. */
 int oracle_candidate(int32_t n, int64_t m, const int32_t *src, const int32_t *dst, int32_t D,
                      const uint8_t *allowed, int32_t P, int32_t b, const uint8_t *base_x,

@@ -86,6 +86,10 @@ def lib():
         L.oracle_set_constraints.argtypes = [C.c_int32, C.c_int64, _i32p, _i32p, _i64p,
                                              C.c_int32, C.c_void_p, C.c_void_p, C.c_void_p]
         L.oracle_set_constraints.restype = C.c_int
+        L.oracle_set_coarse_moves.argtypes = [C.c_int32, _i32p, C.c_int32, C.c_int32]
+        L.oracle_set_coarse_moves.restype = C.c_int
+        L.oracle_clear_coarse_moves.argtypes = []
+        L.oracle_clear_coarse_moves.restype = None
         L.oracle_clear_constraints.argtypes = []
         L.oracle_clear_constraints.restype = None
         L.oracle_constraints_ok.argtypes = [C.c_int32, _u8p]
@@ -180,6 +184,24 @@ class constraints:
 
     def ok(self, x) -> bool:
         return bool(lib().oracle_constraints_ok(int(self.g.n), np.ascontiguousarray(x, np.uint8)))
+
+
+class coarse_moves:
+    """Group moves over merged vertices (row f2, DESIGN.md §4 S9), active inside `with`."""
+
+    def __init__(self, g, coarse_of, n_coarse, pct):
+        self.g = g
+        self.coarse_of = np.ascontiguousarray(coarse_of, np.int32)
+        self.n_coarse, self.pct = int(n_coarse), int(pct)
+
+    def __enter__(self):
+        rc = lib().oracle_set_coarse_moves(int(self.g.n), self.coarse_of, self.n_coarse, self.pct)
+        if rc != 0:
+            raise ValueError(f"oracle_set_coarse_moves: {rc}")
+        return self
+
+    def __exit__(self, *a):
+        lib().oracle_clear_coarse_moves()
 
 
 def makespan_nocongest(g, x, order) -> int:

@@ -137,3 +137,54 @@ def test_keys_equal_makespan_of_decoded_candidate(O):
         ok, x, o = O.candidate(g, 3, 1, xs, orders, j, 42, 9, MIX)
         assert ok
         assert int(keys[j]) == (O.makespan(g, x, o) << 24) | j
+
+
+def test_coarse_group_moves_spec(O):
+    """S9 (row f2): in a coarse group every candidate moves exactly the ops of one merged
+    vertex that allow the drawn device -- the vertex and device restated from the spec text --
+    with the order unchanged; other groups decode exactly as without coarse moves."""
+    g, xs, orders = _setup(seed=9, n=80, D=3, allowed_frac=0.3)
+    P, n = xs.shape
+    coarse_of = (np.arange(n) * 7 % 5).astype(np.int32)      # 5 merged vertices, interleaved
+    pct, seed, step = 40, 77, 2
+    plain = {}
+    for b in range(P):
+        for j in range(0, 1536):
+            plain[(b, j)] = O.candidate(g, P, b, xs, orders, j, seed, step, MIX)
+    n_coarse_groups = 0
+    with O.coarse_moves(g, coarse_of, 5, pct):
+        for b in range(P):
+            for j in range(0, 1536):
+                ok, x, o = O.candidate(g, P, b, xs, orders, j, seed, step, MIX)
+                grp = j >> 7
+                coarse = grp != 0 and O.draw(seed, step, P, b, 128 * grp, 12) % 100 < pct
+                if not coarse:
+                    pok, px, po = plain[(b, j)]
+                    assert ok == pok and (x == px).all() and (o == po).all()
+                    continue
+                n_coarse_groups += (j & 127) == 0
+                assert ok and (o == orders[b]).all()
+                k = O.draw(seed, step, P, b, j, 10) % 5
+                d = O.draw(seed, step, P, b, j, 11) % 3
+                want = xs[b].copy()
+                for v in range(n):
+                    if coarse_of[v] == k and (g.allowed is None or (g.allowed[v] >> d) & 1):
+                        want[v] = d
+                assert (x == want).all(), (b, j)
+    assert n_coarse_groups > 0
+
+
+def test_coarse_search_step_commits_best(O):
+    """a whole step with coarse groups: the committed base is the argmin candidate."""
+    g, xs, orders = _setup(seed=12, n=60, D=2)
+    coarse_of = (np.arange(g.n) // 12).astype(np.int32)
+    rx, ro = xs.copy(), orders.copy()
+    rmk = np.asarray([O.makespan(g, rx[b], ro[b]) for b in range(3)], np.int64)
+    with O.coarse_moves(g, coarse_of, 5, 60):
+        keys_all = [O.candidate_keys(g, 3, b, xs, orders, 0, 1024, 4, 0, MIX) for b in range(3)]
+        keys = O.search_step(g, rx, ro, rmk, 1024, 4, 0, MIX)
+        for b in range(3):
+            assert keys[b] == keys_all[b].min()
+            ok, x, o = O.candidate(g, 3, b, xs, orders, int(keys[b]) & ((1 << 24) - 1), 4, 0, MIX)
+            assert (rx[b] == x).all() and (ro[b] == o).all()
+            assert rmk[b] == int(keys[b]) >> 24 == O.makespan(g, x, o)
