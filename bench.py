@@ -45,6 +45,11 @@ def parse():
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
     ap.add_argument("--dispatch", default="fixed", choices=["fixed", "nondelay"],
                     help="row f4(i): nondelay = TF-style ready-queue dispatch by pi priority")
+    ap.add_argument("--coarse-pct", type=int, default=0,
+                    help="search spec S9 (row f2): %% of candidate groups that move merged "
+                         "vertices of a PAPER.md 3.3 coarsening (0 = off, the default mix)")
+    ap.add_argument("--coarse-target", type=int, default=200,
+                    help="merged vertices of that coarsening (L267: ~200)")
     return ap.parse_args()
 
 
@@ -134,9 +139,12 @@ def seeds_for(P, G, g, n_bases: int):
     return np.stack(xs[:n_bases]), np.stack(os_[:n_bases])
 
 
-def oracle_rate(g, xs, orders, k_per_base, seconds, threads, nondelay=False):
+def oracle_rate(g, xs, orders, k_per_base, seconds, threads, nondelay=False, coarse=None):
     """Oracle (as it stands) on a bounded sample of this workload's step-0 candidates."""
     from oracle import oracle as O
+    if coarse is not None:                   # the same S9 coarse groups as the timed search
+        with O.coarse_moves(g, *coarse):
+            return oracle_rate(g, xs, orders, k_per_base, seconds, threads, nondelay)
     P_ = xs.shape[0]
     mix = configs.MOVE_MIX
 
@@ -227,6 +235,11 @@ def run_pesto(args, rank, world, local):
         nid = obj[0]
     S = P.Search(G, xs, orders, k_per_base, configs.MOVE_MIX, configs.SEARCH_SEED, rank, world,
                  nid)
+    coarse = None
+    if args.coarse_pct > 0:                          # S9 group moves (host coarsening, untimed)
+        co, nc = G.coarsen(args.coarse_target)
+        S.set_coarse_moves(co, nc, args.coarse_pct)
+        coarse = (co, nc, args.coarse_pct)
     seed_mk = [S.get(b)[0] for b in range(n_bases)]
     stream = torch.cuda.current_stream()
     # L2 flush buffer (> 126 MB L2) written between timed steps
@@ -356,7 +369,9 @@ def run_pesto(args, rank, world, local):
                        "candidates_per_step": k_gpu * world, "candidates_per_gpu": k_gpu,
                        "bases": n_bases, "k_per_base": k_per_base, "move_mix": configs.MOVE_MIX,
                        "live_slots": st["live_slots"], "l2": "flushed between timed steps",
-                       "parallelism": f"candidate-dp{world}", "dispatch": args.dispatch},
+                       "parallelism": f"candidate-dp{world}", "dispatch": args.dispatch,
+                       "coarse_groups_pct": args.coarse_pct,
+                       "n_coarse": int(coarse[1]) if coarse else None},
             "op_relaxations_per_s": value * g.n, "edge_relaxations_per_s": value * g.m,
             "eval_kernel_ms": tot_eval_ms / args.steps,
             "roofline": {"bound": "alu", "achieved": achieved, "peak": peak_tops,
@@ -377,7 +392,7 @@ def run_pesto(args, rank, world, local):
     if not args.no_cpu_baseline:
         threads = len(os.sched_getaffinity(0))
         rate, done, dt = oracle_rate(g, xs, orders, k_per_base, args.cpu_seconds, threads,
-                                     nondelay=nd)
+                                     nondelay=nd, coarse=coarse)
         line["cpu_baseline"] = {"value": rate, "unit": "candidates/s", "cores": threads,
                                 "kind": "oracle",
                                 "sample": f"{done} step-0 neighbour candidates of the same "

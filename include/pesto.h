@@ -238,6 +238,21 @@ pesto_status pesto_search_commit(pesto_search *s, void *cuda_stream); /* K4 + st
 pesto_status pesto_search_candidate_keys(pesto_search *s, int32_t base, int64_t j0, int64_t j1,
                                          uint64_t *keys_out, void *cuda_stream);
 
+/* Search spec S9: group moves over merged vertices -- the
+ * placement unit of PAPER.md L269 ("all vertices that were merged ... to form v will be placed
+ * on GPU-0").  From the next step on, group g != 0 of every base is a coarse group iff
+ * draw(128g, 12) mod 100 < pct; its candidate j moves every op of merged vertex
+ * draw(j, 10) mod n_coarse whose mask allows device draw(j, 11) mod D to that device, with no
+ * order move and no region move.  Other groups decode as before.  All ranks must make the same
+ * call before the same step.
+ *   coarse_of: HOST [n_ops] merged vertex of each op in [0, n_coarse) (e.g. pesto_coarsen), copied;
+ *   n_coarse:  1 .. 255;   pct: 0 .. 100 (0 turns the moves off; coarse_of is then ignored).
+ * Synchronises.  Errors: EINVAL; ESTATE when the graph has row-f3 constraints (their local
+ * check does not cover a vertex spread over the whole order; constraints set later make the next
+ * step fail with ESTATE). */
+pesto_status pesto_search_set_coarse_moves(pesto_search *s, const int32_t *coarse_of,
+                                          int32_t n_coarse, int32_t pct);
+
 /* Current incumbent of `base` (synchronises): makespan, x (host [n_ops]) and order. */
 pesto_status pesto_search_get(pesto_search *s, int32_t base, int64_t *makespan,
                               uint8_t *x_host, int32_t *order_host);

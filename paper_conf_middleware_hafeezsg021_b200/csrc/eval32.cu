@@ -51,7 +51,7 @@ template <class T> constexpr uint32_t kSc = sizeof(T) / 4u;
 #ifndef PESTO_E32_W1
 #define PESTO_E32_W1 8
 #endif
-__host__ __device__ constexpr int warps_for(int cpl) { return cpl == 1 ? PESTO_E32_W1 : 4; }
+__host__ __device__ constexpr int warps_for(int cpl) { return cpl == 1 ? PESTO_E32_W1 : 8 / cpl; }
 
 // TMA ring depth and the occupancy target (resident CTAs per SM the register allocation aims
 // for), per candidates-per-lane
@@ -64,8 +64,13 @@ __host__ __device__ constexpr int warps_for(int cpl) { return cpl == 1 ? PESTO_E
 #ifndef PESTO_E32_MINB2
 #define PESTO_E32_MINB2 4
 #endif
+#ifndef PESTO_E32_MINB4
+#define PESTO_E32_MINB4 4
+#endif
 constexpr int kStages32 = PESTO_E32_STAGES;
-__host__ __device__ constexpr int min_blocks_for(int cpl) { return cpl == 1 ? PESTO_E32_MINB1 : PESTO_E32_MINB2; }
+__host__ __device__ constexpr int min_blocks_for(int cpl) {
+    return cpl == 1 ? PESTO_E32_MINB1 : (cpl == 2 ? PESTO_E32_MINB2 : PESTO_E32_MINB4);
+}
 
 // per-candidate device / link free times
 template <int CPL, class T>
@@ -174,6 +179,22 @@ __device__ __forceinline__ PackedMove pack_move(const LaneMove &mv, int32_t rc) 
         p.w1 |= ((uint32_t)(mv.ws - rc) << 12) | ((uint32_t)mv.wl << 18) | ((uint32_t)mv.wd << 25);
     return p;
 }
+// S9 coarse move (merged vertex k -> device d): w1 = k | d << 8 (w0 holds only the kind)
+__device__ __forceinline__ PackedMove pack_coarse(const LaneMove &mv) {
+    PackedMove p;
+    p.w0 = (uint32_t)kMoveCoarse << 27;
+    p.w1 = (uint32_t)mv.ws | ((uint32_t)mv.wd << 8);
+    return p;
+}
+__device__ __forceinline__ int coarse_apply_kept(const LaneMove &mv, int cq, int xb, unsigned aq) {
+    return apply_coarse(mv.ws, mv.wd, cq, xb, aq);
+}
+__device__ __forceinline__ int coarse_apply_kept(const PackedMove &mv, int cq, int xb, unsigned aq) {
+    return apply_coarse((int32_t)(mv.w1 & 255u), (int32_t)(mv.w1 >> 8), cq, xb, aq);
+}
+__device__ __forceinline__ void keep_coarse(LaneMove &dst, const LaneMove &mv) { dst = mv; }
+__device__ __forceinline__ void keep_coarse(PackedMove &dst, const LaneMove &mv) { dst = pack_coarse(mv); }
+
 // = apply_lane (moves.cuh) for offset o = q - rc of a position inside the region
 __device__ __forceinline__ int apply_packed(const PackedMove &p, uint32_t o, int xb, unsigned aq) {
     int x = xb;
@@ -213,10 +234,15 @@ struct Place32 {
     int32_t rc, rlen;            // MODE 1: the group's region [rc, rc + rlen)
     int all_allowed, lane, dmax;
     typename std::conditional<CPL == 1, LaneMove, PackedMove>::type mv[CPL];
-    const uint8_t *cpos;         // MODE 4: merged vertex of the op at each position
+    const uint8_t *cpos;         // MODE 4: merged vertex by position
     int cbits;                   // MODE 4: bits per merged vertex in the candidate index
     uint32_t jc[CPL];            // MODE 4: the lane's candidate indices
-    __device__ __forceinline__ void at(int32_t q, int xb, int (&x)[CPL]) const {
+    // MODE 5 (search with S9 coarse groups), coarse group: the region is the whole order, marked by a negative rlen (the
+    // unsigned range test still admits every position), so no flag register stays live
+    __device__ __forceinline__ bool coarse() const { return rlen < 0; }
+    // cfn(q): merged vertex of the op at position q (MODE 5 coarse groups only)
+    template <class CFn>
+    __device__ __forceinline__ void at(int32_t q, int xb, int (&x)[CPL], const CFn &cfn) const {
         if (MODE == 0) {
 #pragma unroll
             for (int c = 0; c < CPL; c++) x[c] = planes_dev_at<PL>(pl + c * pl_stride, q, lane, dmax);
@@ -232,6 +258,12 @@ struct Place32 {
         for (int c = 0; c < CPL; c++) x[c] = xb;
         if ((uint32_t)(q - rc) < (uint32_t)rlen) {             // warp-uniform branch
             const unsigned aq = all_allowed ? 0xFFu : (unsigned)__ldg(allowed_pos + q);
+            if (MODE == 5 && coarse()) {                       // S9: one merged vertex per lane
+                const int cq = cfn(q);
+#pragma unroll
+                for (int c = 0; c < CPL; c++) x[c] = coarse_apply_kept(mv[c], cq, xb, aq);
+                return;
+            }
 #pragma unroll
             for (int c = 0; c < CPL; c++) x[c] = apply_kept(mv[c], q, rc, xb, aq);
         }
@@ -384,6 +416,7 @@ __device__ __forceinline__ void begin32(const uint4 h, StateT &st, const T (&r)[
 template <int MODE, int PL, int CPL, class T>
 __global__ void __launch_bounds__((warps_for(CPL) + 1) * 32, min_blocks_for(CPL))
 eval32_kernel(const EvalParams P) {
+    constexpr bool kSearch = MODE == 1 || MODE == 5;   // 5: search with S9 coarse groups
     constexpr int NW = warps_for(CPL);          // consumer warps per CTA (256 candidates)
     constexpr int CW = 32 * CPL;                // candidates per warp
     extern __shared__ __align__(128) uint8_t smem[];
@@ -411,7 +444,7 @@ eval32_kernel(const EvalParams P) {
 
     auto runs_here = [&](int bl) {           // search: this kernel owns bases below saturation
         // (the wide instance, gate 2, owns the bases at or above saturation)
-        return MODE != 1 || P.gate == 0 ||
+        return !kSearch || P.gate == 0 ||
                (P.gate == 1 ? P.base_mk[bl] < (int64_t)kSat32 : P.base_mk[bl] >= (int64_t)kSat32);
     };
 
@@ -419,7 +452,7 @@ eval32_kernel(const EvalParams P) {
         if (lane == 0) {
             uint32_t it = 0;
             for (int64_t task = blockIdx.x; task < P.n_tasks; task += gridDim.x) {
-                const int bl = MODE == 1 ? (int)(task / P.tasks_per_base) : 0;
+                const int bl = kSearch ? (int)(task / P.tasks_per_base) : 0;
                 if (!runs_here(bl)) continue;
                 const BaseLayoutDev *B = &P.bases[bl];
                 const int nt = B->n_tiles32;
@@ -490,14 +523,14 @@ eval32_kernel(const EvalParams P) {
 
     uint32_t it = 0;
     for (int64_t task = blockIdx.x; task < P.n_tasks; task += gridDim.x) {
-        const int bl = MODE == 1 ? (int)(task / P.tasks_per_base) : 0;
+        const int bl = kSearch ? (int)(task / P.tasks_per_base) : 0;
         if (!runs_here(bl)) continue;
-        const int64_t local = MODE == 1 ? task % P.tasks_per_base : task;
+        const int64_t local = kSearch ? task % P.tasks_per_base : task;
         const BaseLayoutDev *B = &P.bases[bl];
         const int nt = B->n_tiles32;
         // a task = TS consecutive candidate ids starting at a multiple of TS; a warp = CW of them
         constexpr int64_t TS = (int64_t)NW * CW;
-        const int64_t j0 = (MODE == 1 ? P.j_begin - P.j_begin % TS : 0) + local * TS + warp * CW;
+        const int64_t j0 = (kSearch ? P.j_begin - P.j_begin % TS : 0) + local * TS + warp * CW;
         const int64_t gw = j0 >> 5;                                 // first 32-row group
 
         Place32<MODE, PL, CPL> place;
@@ -538,35 +571,52 @@ eval32_kernel(const EvalParams P) {
             const int breal = P.b_offset + bl;
             const uint64_t cb = ctr_base_of(P.step, P.P_total, breal);
             const int64_t grp = j0 >> kGroupShift;
-            const Region rg = decode_region(P.seed, cb, grp, P.n);
-            place.rc = rg.c;
-            place.rlen = rg.len;
             place.allowed_pos = B->allowed_pos;
+            const bool coarse = MODE == 5 && coarse_group(P.seed, cb, grp, P.coarse_pct, P.n_coarse);
+            if (coarse) {
+                // S9: every lane moves one merged vertex, anywhere in the order; no order move
+                place.rc = 0;
+                place.rlen = (int32_t)(0x80000000u | (uint32_t)P.n);
+#pragma unroll
+                for (int c = 0; c < CPL; c++) {
+                    const int64_t j = j0 + c * 32 + lane;
+                    valid[c] = active && j >= P.j_begin && j < P.j_end;
+                    keep_coarse(place.mv[c], decode_coarse_lane(P.seed, cb, j, P.n_coarse, P.D));
+                }
+            }
+            const Region rg = decode_region(P.seed, cb, grp, P.n);
+            if (!coarse) {
+                place.rc = rg.c;
+                place.rlen = rg.len;
+            }
             const uint8_t *blocked = B->swap_blocked;
-            ks = active ? decode_swap(P.seed, cb, grp, P.n, P.mix[3], rg,
-                                      [&](int32_t k) { return __ldg(blocked + k) != 0; })
-                        : -1;
+            ks = active && !coarse
+                     ? decode_swap(P.seed, cb, grp, P.n, P.mix[3], rg,
+                                   [&](int32_t k) { return __ldg(blocked + k) != 0; })
+                     : -1;
             const int32_t *ord = B->order;
             const uint32_t *bits = B->bits;
             const uint8_t *aop = P.allowed_op;
             const int words = P.words;
+            if (!coarse) {
 #pragma unroll
-            for (int c = 0; c < CPL; c++) {
-                const int64_t j = j0 + c * 32 + lane;
-                const bool in_range = active && j >= P.j_begin && j < P.j_end;
-                LaneMove mv = in_range
-                    ? decode_lane(P.seed, cb, j, ks >= 0 && (j & (kGroup - 1)) == 0, P.D, P.mix, rg,
-                                  [&](int32_t q) { return __ldg(ord + q); },
-                                  [&](int32_t q) { return ldg_bits_dev_at<PL>(bits, words, q); },
-                                  [&](int32_t op) { return (unsigned)__ldg(aop + op); })
-                    : no_move();
-                valid[c] = in_range && mv.kind != kMoveInvalid;
-                if (mv.kind == kMoveInvalid) mv = no_move();
-                if (valid[c] && (P.feas.has_cap || P.feas.has_coloc))   // row f3
-                    valid[c] = move_feasible<PL>(mv, rg, P.D, bits, words, ord,
-                                                 B->allowed_pos, P.all_allowed, P.feas,
-                                                 P.feas.fbase + (size_t)bl * 8);
-                keep_move(place.mv[c], mv, rg.c);
+                for (int c = 0; c < CPL; c++) {
+                    const int64_t j = j0 + c * 32 + lane;
+                    const bool in_range = active && j >= P.j_begin && j < P.j_end;
+                    LaneMove mv = in_range
+                        ? decode_lane(P.seed, cb, j, ks >= 0 && (j & (kGroup - 1)) == 0, P.D, P.mix, rg,
+                                      [&](int32_t q) { return __ldg(ord + q); },
+                                      [&](int32_t q) { return ldg_bits_dev_at<PL>(bits, words, q); },
+                                      [&](int32_t op) { return (unsigned)__ldg(aop + op); })
+                        : no_move();
+                    valid[c] = in_range && mv.kind != kMoveInvalid;
+                    if (mv.kind == kMoveInvalid) mv = no_move();
+                    if (valid[c] && (P.feas.has_cap || P.feas.has_coloc))   // row f3
+                        valid[c] = move_feasible<PL>(mv, rg, P.D, bits, words, ord,
+                                                     B->allowed_pos, P.all_allowed, P.feas,
+                                                     P.feas.fbase + (size_t)bl * 8);
+                    keep_move(place.mv[c], mv, rg.c);
+                }
             }
         }
         st.init();
@@ -581,8 +631,10 @@ eval32_kernel(const EvalParams P) {
 #pragma unroll
         for (int c = 0; c < CPL; c++) { x[c] = 0; cc[c] = 0u; fwd[c] = 0u; nfar[c] = 0u; nnear[c] = 0u; }
         // devices by direct lookup (search: base code + region moves; rows: plane words)
+        // S9 merged vertices by position of this base (P.coarse_pos = [local base][n])
+        auto cpos_at = [&](int32_t q) { return (int)__ldg(P.coarse_pos + (size_t)bl * P.n + q); };
         auto place_y = [&](int, const uint4 rec, int (&y)[CPL]) {
-            place.at((int32_t)(rec.y & kSuccPosMask), (int)((rec.y >> kSuccXShift) & 7u), y);
+            place.at((int32_t)(rec.y & kSuccPosMask), (int)((rec.y >> kSuccXShift) & 7u), y, cpos_at);
         };
         // explicit rows: the plane words of the next op are loaded one step ahead (consecutive
         // positions share cache lines); the successors' words come from K5's edge-slot stream
@@ -659,7 +711,7 @@ eval32_kernel(const EvalParams P) {
                     }
                     if (!(h.w & kStCont)) {
                         v++;
-                        if (MODE == 1 && v == ks) {
+                        if (kSearch && v == ks) {
                             // swapped pair: the op at ks+1 runs first, then the op at ks.  They
                             // share no producer, no consumer and no edge (DESIGN.md §4 S3), so
                             // every slot's first push is unchanged; only device and link queues
@@ -687,14 +739,14 @@ eval32_kernel(const EvalParams P) {
                             arrivals(h1.w, f1, g1, zero, r1);   // ks+1's distance-1 producer is ks: none
 #pragma unroll
                             for (int c = 0; c < CPL; c++) fwd[c] = 0u;
-                            place.at(v + 1, (int)(h1.w & kStXMask), x);
+                            place.at(v + 1, (int)(h1.w & kStXMask), x, cpos_at);
                             begin32<CPL, T>(h1, st, r1, x, cc);
                             for (int32_t q = 0; q < n1; q++) {
                                 const uint32_t a = sp1 + q * kStepBytes;
                                 edges32<PL, CPL, T>(cx, lds_u32(a + 12), lds_v4(a + 16), lds_v4(a + 32), x,
                                                  cc, place_y, st, fwd);
                             }
-                            place.at(v, (int)(h.w & kStXMask), x);
+                            place.at(v, (int)(h.w & kStXMask), x, cpos_at);
                             begin32<CPL, T>(h, st, r0, x, cc);
                             edges32<PL, CPL, T>(cx, h.w, e0, e1, x, cc, place_y, st, fwd);
                             for (int32_t q = 1; q < nk; q++) {
@@ -742,10 +794,10 @@ eval32_kernel(const EvalParams P) {
                             // outside the group's region every lane has the base device
                             // (CPL = 2 only: with one candidate per lane the launch is
                             // latency-bound and the branch-free selects schedule better)
-                            xu = (MODE == 1 && CPL == 2 &&
+                            xu = (kSearch && CPL >= 2 &&
                                   (uint32_t)(v - place.rc) >= (uint32_t)place.rlen)
                                      ? (int)(h.w & kStXMask) : -1;
-                            place.at(v, (int)(h.w & kStXMask), x);
+                            place.at(v, (int)(h.w & kStXMask), x, cpos_at);
                         }
                         if (MODE != 0 && xu >= 0) st.begin_u(xu, h.x, r, cc);
                         else begin32<CPL, T>(h, st, r, x, cc);
@@ -818,7 +870,7 @@ eval32_kernel(const EvalParams P) {
 template <int MODE, int PL, int CPL>
 auto kernel_for(const EvalParams &p) {
     // the wide (exact 64-bit) instance serves search bases at or above saturation only
-    if constexpr (MODE == 1) {
+    if constexpr (MODE == 1 || MODE == 5) {
         if (p.wide32) return eval32_kernel<MODE, PL, CPL, uint64_t>;
     }
     return eval32_kernel<MODE, PL, CPL, uint32_t>;
@@ -854,10 +906,10 @@ int planes_of32(int D) { return D <= 2 ? 1 : (D <= 4 ? 2 : 4); }
 int eval32_task_size(int cpl) { return warps_for(cpl) * 32 * cpl; }
 
 int eval32_smem_bytes(const EvalParams &p, int search_mode) {
-    const int cpl = p.cpl32 == 1 ? 1 : 2;
+    const int cpl = p.cpl32 == 1 ? 1 : (p.cpl32 == 4 ? 4 : 2);
     const int nw = warps_for(cpl);
     const int pl = planes_of32(p.D);
-    const size_t tb = (search_mode == 1 && p.wide32) ? 8 : 4;   // bytes per time value
+    const size_t tb = ((search_mode == 1 || search_mode == 5) && p.wide32) ? 8 : 4;   // bytes per time value
     size_t b = (size_t)kStages32 * (p.stage_bytes32 + kStepBytes) + 2 * kStages32 * 8;
     b = (b + 15) & ~size_t(15);
     b += (size_t)nw * kRing * 32 * cpl * tb;       // near ring
@@ -877,6 +929,10 @@ int eval32_smem_bytes(const EvalParams &p, int search_mode) {
             if (pl == 1) return FN<4, 1, C>(__VA_ARGS__);                                  \
             if (pl == 2) return FN<4, 2, C>(__VA_ARGS__);                                  \
             return FN<4, 4, C>(__VA_ARGS__);                                               \
+        } else if (search_mode && p.coarse_pct > 0) {   /* S9 coarse groups: own instance */ \
+            if (pl == 1) return FN<5, 1, C>(__VA_ARGS__);                                  \
+            if (pl == 2) return FN<5, 2, C>(__VA_ARGS__);                                  \
+            return FN<5, 4, C>(__VA_ARGS__);                                               \
         } else if (search_mode) {                                                          \
             if (pl == 1) return FN<1, 1, C>(__VA_ARGS__);                                  \
             if (pl == 2) return FN<1, 2, C>(__VA_ARGS__);                                  \
@@ -890,6 +946,10 @@ int eval32_smem_bytes(const EvalParams &p, int search_mode) {
 #define PESTO_DISPATCH32(FN, ...)                                                          \
     do {                                                                                   \
         if (p.cpl32 == 1) PESTO_DISPATCH32_C(FN, 1, __VA_ARGS__);                          \
+        if (p.cpl32 == 4 && search_mode == 1 && p.coarse_pct == 0) {  /* search only */    \
+            if (planes_of32(p.D) == 1) return FN<1, 1, 4>(__VA_ARGS__);                    \
+            if (planes_of32(p.D) == 2) return FN<1, 2, 4>(__VA_ARGS__);                    \
+        }                                                                                  \
         PESTO_DISPATCH32_C(FN, 2, __VA_ARGS__);                                            \
     } while (0)
 

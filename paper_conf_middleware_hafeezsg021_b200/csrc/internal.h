@@ -37,6 +37,8 @@ struct BaseLayoutDev {
     // producer's edges in (successor position, edge index) order -- the FCFS tie order R3
     const int32_t *nd_dst;      // [m] consumer op id
     const int64_t *nd_t;        // [m][n_classes] transfer time per link class
+    // search spec S9 (row f2 group moves): merged vertex of the op at each position, or null
+    const uint8_t *coarse_pos;
 };
 
 // Row f3 constraints as the kernels see them (PAPER.md L202 memory, L175 colocation).
@@ -100,6 +102,8 @@ struct EvalParams {
     // device (j >> (coarse_bits * k)) & (D - 1); every op takes its merged vertex's device
     const uint8_t *coarse_pos;          // [n] merged vertex of the op at each position
     int32_t coarse_bits, n_coarse;
+    int32_t coarse_pct;                 // search (mode 1): S9 coarse-group percentage (0 = off);
+                                        // merged vertices per position in bases[b].coarse_pos
     uint8_t coarse_allowed[32];         // device mask of each merged vertex (AND of members)
     // eval64 list mode (MODE 2): candidates list[0 .. *list_count)
     const int32_t *list;
@@ -134,6 +138,7 @@ struct NdParams {
     const uint8_t *allowed_op;
     uint64_t *keys, *keys_dbg;
     Feasibility feas;
+    int32_t n_coarse, coarse_pct;       // S9 coarse groups (0 = off)
 };
 
 struct TransposeParams {
@@ -163,6 +168,7 @@ struct CommitParams {
     int32_t *swap_out;                  // [P] committed swap position or -1
     int32_t patch32;                    // eval32 records carry base codes: patch them too
     Feasibility feas;                   // f3: the committed move updates fbase
+    int32_t n_coarse, coarse_pct;       // S9 coarse groups (0 = off)
 };
 
 // explicit rows: OR the candidates violating the f3 constraints into the per-group masks

@@ -77,6 +77,8 @@ struct Placement {
     LaneMove mv;
     int lane;
     int dmax;
+    const uint8_t *cpos;         // S9 coarse group: merged vertex by position (else unused)
+    bool coarse;
 
     __device__ __forceinline__ int operator()(int32_t q) const {
         // MODE 0: this warp's group words, bit `lane`; MODE 2 (fixup list): each lane's own
@@ -85,7 +87,8 @@ struct Placement {
         int x = ldg_bits_dev_at<PL>(bits, words, q);
         if ((uint32_t)(q - rc) < (uint32_t)rlen) {            // warp-uniform branch
             unsigned aq = all_allowed ? 0xFFu : (unsigned)__ldg(allowed_pos + q);
-            x = apply_lane(mv, q, x, aq);
+            x = coarse ? apply_coarse(mv.ws, mv.wd, (int)__ldg(cpos + q), x, aq)
+                       : apply_lane(mv, q, x, aq);
         }
         return x;
     }
@@ -297,6 +300,8 @@ eval_kernel(const EvalParams P) {
         place.dmax = P.D - 1;
         place.words = P.words;
         place.all_allowed = P.all_allowed;
+        place.coarse = false;
+        place.cpos = nullptr;
         bool active, valid = true;
         int64_t j = g * 32 + lane;
         int32_t ks = -1;
@@ -318,20 +323,25 @@ eval_kernel(const EvalParams P) {
             const uint64_t cb = ctr_base_of(P.step, P.P_total, breal);
             const int64_t grp = (g * 32) >> kGroupShift;          // spec group of this warp
             const Region rg = decode_region(P.seed, cb, grp, P.n);
-            place.rc = rg.c;
-            place.rlen = rg.len;
+            place.coarse = coarse_group(P.seed, cb, grp, P.coarse_pct, P.n_coarse);
+            place.rc = place.coarse ? 0 : rg.c;          // S9: a coarse group may move any op
+            place.rlen = place.coarse ? P.n : rg.len;
+            place.cpos = B->coarse_pos;
             place.bits = B->bits;
             place.allowed_pos = B->allowed_pos;
             const uint8_t *adj = B->swap_blocked;
-            ks = active ? decode_swap(P.seed, cb, grp, P.n, P.mix[3], rg,
-                                      [&](int32_t k) { return __ldg(adj + k) != 0; })
-                        : -1;
+            ks = active && !place.coarse
+                     ? decode_swap(P.seed, cb, grp, P.n, P.mix[3], rg,
+                                   [&](int32_t k) { return __ldg(adj + k) != 0; })
+                     : -1;
             const bool in_range = active && j >= P.j_begin && j < P.j_end;
             const int32_t *ord = B->order;
             const uint32_t *bits = B->bits;
             const uint8_t *aop = P.allowed_op;
             const int words = P.words;
-            place.mv = in_range
+            if (place.coarse)
+                place.mv = decode_coarse_lane(P.seed, cb, j, P.n_coarse, P.D);
+            else place.mv = in_range
                 ? decode_lane(P.seed, cb, j, ks >= 0 && (j & (kGroup - 1)) == 0, P.D, P.mix, rg,
                               [&](int32_t q) { return __ldg(ord + q); },
                               [&](int32_t q) { return ldg_bits_dev_at<PL>(bits, words, q); },
@@ -626,11 +636,13 @@ __global__ void commit_kernel(const CommitParams P) {
     const uint64_t cb = ctr_base_of(P.step, P.P, b);
     const uint8_t *adj = B.swap_blocked;
     const Region rg = decode_region(P.seed, cb, j >> kGroupShift, P.n);
-    const int32_t ks = j == 0 ? -1
+    const bool coarse = coarse_group(P.seed, cb, j >> kGroupShift, P.coarse_pct, P.n_coarse);
+    const int32_t ks = j == 0 || coarse ? -1
                               : decode_swap(P.seed, cb, j >> kGroupShift, P.n, P.mix[3], rg,
                                             [&](int32_t k) { return adj[k] != 0; });
     const int words = P.words;
     const LaneMove mv = j == 0 ? no_move()
+        : coarse ? decode_coarse_lane(P.seed, cb, j, P.n_coarse, P.D)
         : decode_lane(P.seed, cb, j, ks >= 0 && (j & (kGroup - 1)) == 0, P.D, P.mix, rg,
                       [&](int32_t q) { return B.order[q]; },
                       [&](int32_t q) { return get_dev_at<PL>(bits, words, q); },
@@ -675,6 +687,9 @@ __global__ void commit_kernel(const CommitParams P) {
     } else if (mv.kind == kMoveWindow) {
         for (int32_t q = mv.ws + lane; q < mv.ws + mv.wl; q += 32)
             if ((B.allowed_pos[q] >> mv.wd) & 1u) set_dev(q, mv.wd);
+    } else if (mv.kind == kMoveCoarse) {       // S9: every op of merged vertex ws that allows wd
+        for (int32_t q = lane; q < P.n; q += 32)
+            if (B.coarse_pos[q] == mv.ws && ((B.allowed_pos[q] >> mv.wd) & 1u)) set_dev(q, mv.wd);
     }
     __threadfence();                     // every lane's bit updates are performed ...
     __syncwarp();                        // ... before lane 0 reads the planes for the swap

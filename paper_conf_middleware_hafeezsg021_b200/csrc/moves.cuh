@@ -38,7 +38,7 @@ PESTO_HD int popc32(unsigned v) {
 #endif
 }
 
-enum MoveKind : int { kMoveNone = 0, kMoveFlip = 1, kMoveWindow = 2, kMoveInvalid = 3 };
+enum MoveKind : int { kMoveNone = 0, kMoveFlip = 1, kMoveWindow = 2, kMoveInvalid = 3, kMoveCoarse = 4 };
 
 struct LaneMove {
     int kind;
@@ -46,6 +46,7 @@ struct LaneMove {
     int32_t fpos[4];     // flipped positions (in the base order), applied in sequence
     int32_t fdev[4];
     int32_t ws, wl, wd;  // window: positions [ws, ws + wl) move to wd where allowed
+                         // coarse (S9): merged vertex ws moves to wd where allowed (wl = 0)
 };
 
 constexpr int kRegion = 64;     // positions a group of candidates may change (DESIGN §4 S2)
@@ -130,6 +131,28 @@ PESTO_HD LaneMove decode_lane(uint64_t seed, uint64_t cb, int64_t j, bool pure_s
         mv.wd = (int32_t)(draw(seed, cb, j, 4) % (uint64_t)D);
     }
     return mv;
+}
+
+// S9 (row f2): group g != 0 is a coarse group iff draw(128g, 12) mod 100 < pct.
+// A coarse group has no region, no order move and no region moves.
+PESTO_HD bool coarse_group(uint64_t seed, uint64_t cb, int64_t group, int pct, int n_coarse) {
+    return group != 0 && pct > 0 && n_coarse > 0 &&
+           (int)(draw(seed, cb, group * kGroup, 12) % 100u) < pct;
+}
+// candidate j of a coarse group: merged vertex draw(j, 10) mod n_coarse to device draw(j, 11) mod D
+PESTO_HD LaneMove decode_coarse_lane(uint64_t seed, uint64_t cb, int64_t j, int n_coarse, int D) {
+    LaneMove mv;
+    mv.kind = kMoveCoarse;
+    mv.nflip = 0;
+    for (int q = 0; q < 4; q++) { mv.fpos[q] = -1; mv.fdev[q] = 0; }
+    mv.ws = (int32_t)(draw(seed, cb, j, 10) % (uint64_t)n_coarse);
+    mv.wl = 0;
+    mv.wd = (int32_t)(draw(seed, cb, j, 11) % (uint64_t)D);
+    return mv;
+}
+// device of an op of merged vertex cq (base device xb, mask aq) under a coarse move
+PESTO_HD int apply_coarse(int32_t k, int32_t d, int cq, int xb, unsigned aq) {
+    return (cq == k && ((aq >> d) & 1u)) ? d : xb;
 }
 
 // device of position q under move mv (base device xb, op mask at q for the window check)

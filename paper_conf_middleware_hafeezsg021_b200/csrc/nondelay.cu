@@ -151,18 +151,21 @@ __global__ void __launch_bounds__(kNdMaxWarps * 32, 3) nondelay_kernel(const NdP
             et = B->nd_t;
             const uint64_t cb = ctr_base_of(P.step, P.P_total, P.b_offset + bl);
             const int64_t grp = j >> kGroupShift;
-            const Region rg = decode_region(P.seed, cb, grp, n);
+            const bool coarse = coarse_group(P.seed, cb, grp, P.coarse_pct, P.n_coarse);   // S9
+            Region rg = decode_region(P.seed, cb, grp, n);
             const uint8_t *adj = B->swap_blocked;
-            ks = decode_swap(P.seed, cb, grp, n, P.mix[3], rg,
-                             [&](int32_t k) { return __ldg(adj + k) != 0; });
+            ks = coarse ? -1
+                        : decode_swap(P.seed, cb, grp, n, P.mix[3], rg,
+                                      [&](int32_t k) { return __ldg(adj + k) != 0; });
             const uint32_t *bits = B->bits;
             const uint8_t *aop = P.allowed_op;
-            LaneMove mv = decode_lane(P.seed, cb, j, ks >= 0 && (j & (kGroup - 1)) == 0, D, P.mix,
+            LaneMove mv = coarse ? decode_coarse_lane(P.seed, cb, j, P.n_coarse, D) : decode_lane(P.seed, cb, j, ks >= 0 && (j & (kGroup - 1)) == 0, D, P.mix,
                                       rg, [&](int32_t q) { return __ldg(order + q); },
                                       [&](int32_t q) { return ldg_bits_dev_at<PL>(bits, words, q); },
                                       [&](int32_t op) { return (unsigned)__ldg(aop + op); });
             valid = mv.kind != kMoveInvalid;
             if (!valid) mv = no_move();
+            if (coarse) rg = Region{0, n};                        // any op may move
             if (valid && (P.feas.has_cap || P.feas.has_coloc))    // row f3
                 valid = move_feasible<PL>(mv, rg, D, bits, words, order, B->allowed_pos,
                                           P.all_allowed, P.feas, P.feas.fbase + (size_t)bl * 8);
@@ -175,7 +178,8 @@ __global__ void __launch_bounds__(kNdMaxWarps * 32, 3) nondelay_kernel(const NdP
                         x = ldg_bits_dev_at<PL>(bits, words, q);
                         if ((uint32_t)(q - rg.c) < (uint32_t)rg.len) {
                             const unsigned aq = P.all_allowed ? 0xFFu : (unsigned)__ldg(B->allowed_pos + q);
-                            x = apply_lane(mv, q, x, aq);
+                            x = coarse ? apply_coarse(mv.ws, mv.wd, (int)__ldg(B->coarse_pos + q), x, aq)
+                                       : apply_lane(mv, q, x, aq);
                         }
                     }
 #pragma unroll

@@ -82,6 +82,12 @@ struct pesto_search {
     // committed swaps: patched in place on the device vs. layout rebuilt on the host
     DevBuf d_patch;
     int64_t n_swap_inplace = 0, n_swap_rebuilt = 0;
+    // search spec S9 (row f2 group moves): merged vertex of every op, and per base the merged
+    // vertex of the op at each position ([P][n], kept in step with committed swaps)
+    int32_t n_coarse = 0, coarse_pct = 0;
+    std::vector<int32_t> coarse_of;
+    std::vector<uint8_t> cpos;
+    DevBuf d_cpos;
 };
 
 namespace {
@@ -96,6 +102,7 @@ void refresh_views(pesto_search *s) {
         if (s->layouts[b]->W32 == 0) s->use32 = false;
         s->views[b] = layout_view(*s->layouts[b]);
         s->views[b].bits = s->d_bits.as<uint32_t>() + (size_t)b * s->g->planes * s->g->words;
+        s->views[b].coarse_pos = s->cpos.empty() ? nullptr : s->d_cpos.as<uint8_t>() + (size_t)b * s->g->n;
         s->max_W = std::max(s->max_W, s->layouts[b]->W);
         s->stage_bytes = std::max(s->stage_bytes, s->layouts[b]->stage_bytes);
         s->max_W32 = std::max(s->max_W32, s->layouts[b]->W32);
@@ -172,6 +179,8 @@ pesto_status launch_search_nondelay(pesto_search *s, int b_first, int n_bases, i
     p.allowed_op = g->d_allowed.as<uint8_t>();
     p.keys = keys;
     p.keys_dbg = keys_dbg;
+    p.n_coarse = s->n_coarse;
+    p.coarse_pct = s->coarse_pct;
     if ((e = launch_nondelay(p, 1, grid, st)) != cudaSuccess) return cuda_fail(e, "launch non-delay search");
     return PESTO_OK;
 }
@@ -185,6 +194,8 @@ pesto_status launch_search_eval(pesto_search *s, int b_first, int n_bases, int64
     if (j1 <= j0) return PESTO_OK;
     pesto_status rc0 = sync_constraints(s);
     if (rc0) return rc0;
+    if (s->coarse_pct > 0 && (g->has_cap || g->has_coloc))
+        return fail(PESTO_ESTATE, "coarse group moves (S9) cannot be combined with row-f3 constraints");
     if (g->dispatch == PESTO_DISPATCH_NONDELAY)
         return launch_search_nondelay(s, b_first, n_bases, j0, j1, keys, keys_dbg, st);
     EvalParams p;
@@ -208,6 +219,9 @@ pesto_status launch_search_eval(pesto_search *s, int b_first, int n_bases, int64
     p.allowed_op = g->d_allowed.as<uint8_t>();
     p.keys = keys;
     p.keys_dbg = keys_dbg;
+    p.n_coarse = s->n_coarse;
+    p.coarse_pct = s->coarse_pct;
+    p.coarse_pos = s->cpos.empty() ? nullptr : s->d_cpos.as<uint8_t>() + (size_t)b_first * g->n;
     p.group_begin = j0 >> 5;
     p.groups_per_base = ((j1 - 1) >> 5) - p.group_begin + 1;
     p.tasks_per_base = (p.groups_per_base + kWarps - 1) / kWarps;
@@ -222,6 +236,13 @@ pesto_status launch_search_eval(pesto_search *s, int b_first, int n_bases, int64
         EvalParams p32 = p;
         p32.gate = 1;
         plan_eval32(g, p32, j0, j1, n_bases);
+        // four candidates per lane (2-warp CTAs, the same 256-candidate task) for multi-wave
+        // search launches: PESTO_EVAL32_CPL=4 (experiment; D <= 4, no S9 coarse groups)
+        static const bool cpl4 = [] {
+            const char *e = std::getenv("PESTO_EVAL32_CPL");
+            return e && std::atoi(e) == 4;
+        }();
+        if (cpl4 && p32.cpl32 == 2 && g->planes <= 2 && s->coarse_pct == 0) p32.cpl32 = 4;
         if ((rc = ensure_state32(g, p32, 1, p32.n_tasks, &grid))) return rc;
         p32.state32 = g->d_state32.as<uint32_t>();
         if ((e = launch_eval32(p32, 1, grid, st)) != cudaSuccess) return cuda_fail(e, "launch eval32");
@@ -654,6 +675,8 @@ pesto_status pesto_search_commit(pesto_search *s, void *stream) {
     cp.patch32 = s->use32 ? 1 : 0;
     cp.feas = feasibility_view(g);
     cp.feas.fbase = s->d_fbase.as<int64_t>();
+    cp.n_coarse = s->n_coarse;
+    cp.coarse_pct = s->coarse_pct;
     cudaError_t e = launch_commit(cp, st);
     if (e != cudaSuccess) return cuda_fail(e, "launch commit");
     s->step++;
@@ -671,6 +694,11 @@ pesto_status pesto_search_commit(pesto_search *s, void *stream) {
             const int32_t k = s->h_swap[b];
             if (k < 0) continue;
             std::swap(s->order[b][k], s->order[b][k + 1]);
+            if (!s->cpos.empty()) {           // S9 merged vertices by position follow the order
+                const size_t r = (size_t)b * g->n;
+                pt.set_elem(s->d_cpos, s->cpos, r + k, (uint8_t)s->coarse_of[s->order[b][k]]);
+                pt.set_elem(s->d_cpos, s->cpos, r + k + 1, (uint8_t)s->coarse_of[s->order[b][k + 1]]);
+            }
             if (swap_in_place(s, b, k, pt)) {
                 s->n_swap_inplace++;
                 continue;
@@ -699,6 +727,43 @@ pesto_status pesto_search_commit(pesto_search *s, void *stream) {
                 return cuda_fail(e, "upload views");
         }
     }
+    return PESTO_OK;
+}
+
+pesto_status pesto_search_set_coarse_moves(pesto_search *s, const int32_t *coarse_of, int32_t n_coarse,
+                                          int32_t pct) {
+    if (!s) return fail(PESTO_EINVAL, "NULL search");
+    pesto_graph *g = s->g;
+    if (pct < 0 || pct > 100) return fail(PESTO_EINVAL, "coarse percentage out of 0..100");
+    if (pct == 0) {                       // off; the position arrays are kept (cheap) but unused
+        s->coarse_pct = 0;
+        return PESTO_OK;
+    }
+    if (!coarse_of) return fail(PESTO_EINVAL, "NULL coarse_of");
+    if (n_coarse < 1 || n_coarse > 255) return fail(PESTO_EINVAL, "n_coarse must be in 1..255");
+    for (int32_t v = 0; v < g->n; v++)
+        if (coarse_of[v] < 0 || coarse_of[v] >= n_coarse)
+            return fail(PESTO_EINVAL, "coarse_of[" + std::to_string(v) + "] out of range");
+    if (g->has_cap || g->has_coloc)
+        return fail(PESTO_ESTATE, "coarse group moves (S9) cannot be combined with row-f3 constraints");
+    DeviceGuard guard(g->device);
+    cudaError_t e;
+    if (s->last_stream && (e = cudaStreamSynchronize(s->last_stream)) != cudaSuccess)
+        return cuda_fail(e, "synchronise");
+    s->coarse_of.assign(coarse_of, coarse_of + g->n);
+    s->cpos.resize((size_t)s->P * g->n);
+    for (int b = 0; b < s->P; b++)
+        for (int32_t q = 0; q < g->n; q++)
+            s->cpos[(size_t)b * g->n + q] = (uint8_t)coarse_of[s->order[b][q]];
+    if ((e = s->d_cpos.ensure(s->cpos.size())) != cudaSuccess ||
+        (e = cudaMemcpy(s->d_cpos.ptr, s->cpos.data(), s->cpos.size(), cudaMemcpyHostToDevice)) != cudaSuccess)
+        return cuda_fail(e, "upload merged vertices");
+    refresh_views(s);
+    if ((e = cudaMemcpy(s->d_views.ptr, s->views.data(), sizeof(BaseLayoutDev) * s->P,
+                        cudaMemcpyHostToDevice)) != cudaSuccess)
+        return cuda_fail(e, "upload views");
+    s->n_coarse = n_coarse;
+    s->coarse_pct = pct;
     return PESTO_OK;
 }
 

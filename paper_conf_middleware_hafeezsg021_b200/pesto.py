@@ -79,6 +79,7 @@ SIGNATURES = {
     "pesto_search_set_keys": (_I32, [_VP, _VP, _VP]),
     "pesto_search_commit": (_I32, [_VP, _VP]),
     "pesto_search_candidate_keys": (_I32, [_VP, _I32, _I64, _I64, _VP, _VP]),
+    "pesto_search_set_coarse_moves": (_I32, [_VP, _VP, _I32, _I32]),
     "pesto_search_get": (_I32, [_VP, _I32, _VP, _VP, _VP]),
     "pesto_search_step_count": (_I64, [_VP]),
     "pesto_search_swap_stats": (_I32, [_VP, _VP, _VP]),
@@ -313,6 +314,13 @@ class Search:
 
     def commit(self, stream=None):
         _check(_L.pesto_search_commit(self._h, _stream(stream)))
+
+    def set_coarse_moves(self, coarse_of, n_coarse: int, pct: int):
+        """search spec S9: coarse groups move merged vertices (pesto_search_set_coarse_moves)"""
+        c = np.ascontiguousarray(coarse_of, dtype=np.int32)
+        if c.shape != (self.graph.n,):
+            raise ValueError("coarse_of must have one entry per op")
+        _check(_L.pesto_search_set_coarse_moves(self._h, c.ctypes.data, int(n_coarse), int(pct)))
 
     def candidate_keys(self, base: int, j0: int, j1: int, stream=None) -> np.ndarray:
         import torch

@@ -227,6 +227,32 @@ def test_search_steps_match_reference(P, O):
         del keys
 
 
+@pytest.mark.parametrize("D", [2, 4])
+def test_multiwave_search_steps(P, O, D):
+    """search launches of more than one wave (2 x 131,072 candidates = 1,024 eval32 tasks: the
+    multi-candidate-per-lane instances): each step's keys equal the oracle's
+    reference step, and the per-base minimum of the independent eval64 kernel's keys"""
+    g = dag.random_dag(301 + D, 1500, 1.6, D=D, p_max=4000, max_bytes=300_000, beta0=700,
+                       beta1_fs=30_000)
+    G = P.Graph.from_arrays(g)
+    xs, orders = _bases(g, 2, seed=29)
+    K, mix, seed = 131072, (40, 20, 20, 20), 8
+    S = P.Search(G, xs, orders, K, mix, seed=seed)
+    rx, ro = xs.copy(), orders.copy()
+    rmk = np.asarray([O.makespan(g, rx[b], ro[b]) for b in range(2)], np.int64)
+    for step in range(3):
+        S.eval()
+        gkeys = S.keys()
+        for b in range(2):
+            assert int(gkeys[b]) == int(S.candidate_keys(b, 0, K).min()), (step, b)
+        keys = O.search_step(g, rx, ro, rmk, K, seed, step, mix)
+        assert [int(k) for k in gkeys] == [int(k) for k in keys], step
+        S.commit()
+        for b in range(2):
+            mk, x, o = S.get(b)
+            assert mk == rmk[b] and (x == rx[b]).all() and (o == ro[b]).all(), (step, b)
+
+
 @pytest.mark.parametrize("D,mix,steps", [(2, (0, 0, 0, 100), 24), (2, (30, 10, 10, 50), 12),
                                          (4, (20, 10, 10, 60), 10)])
 def test_committed_swaps_patch_layouts(P, O, D, mix, steps):
