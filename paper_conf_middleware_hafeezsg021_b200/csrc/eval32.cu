@@ -51,7 +51,7 @@ template <class T> constexpr uint32_t kSc = sizeof(T) / 4u;
 #ifndef PESTO_E32_W1
 #define PESTO_E32_W1 8
 #endif
-__host__ __device__ constexpr int warps_for(int cpl) { return cpl == 1 ? PESTO_E32_W1 : 8 / cpl; }
+__host__ __device__ constexpr int warps_for(int cpl) { return cpl == 1 ? PESTO_E32_W1 : 4; }
 
 // TMA ring depth and the occupancy target (resident CTAs per SM the register allocation aims
 // for), per candidates-per-lane
@@ -64,13 +64,9 @@ __host__ __device__ constexpr int warps_for(int cpl) { return cpl == 1 ? PESTO_E
 #ifndef PESTO_E32_MINB2
 #define PESTO_E32_MINB2 4
 #endif
-#ifndef PESTO_E32_MINB4
-#define PESTO_E32_MINB4 4
-#endif
+
 constexpr int kStages32 = PESTO_E32_STAGES;
-__host__ __device__ constexpr int min_blocks_for(int cpl) {
-    return cpl == 1 ? PESTO_E32_MINB1 : (cpl == 2 ? PESTO_E32_MINB2 : PESTO_E32_MINB4);
-}
+__host__ __device__ constexpr int min_blocks_for(int cpl) { return cpl == 1 ? PESTO_E32_MINB1 : PESTO_E32_MINB2; }
 
 // per-candidate device / link free times
 template <int CPL, class T>
@@ -794,7 +790,7 @@ eval32_kernel(const EvalParams P) {
                             // outside the group's region every lane has the base device
                             // (CPL = 2 only: with one candidate per lane the launch is
                             // latency-bound and the branch-free selects schedule better)
-                            xu = (kSearch && CPL >= 2 &&
+                            xu = (kSearch && CPL == 2 &&
                                   (uint32_t)(v - place.rc) >= (uint32_t)place.rlen)
                                      ? (int)(h.w & kStXMask) : -1;
                             place.at(v, (int)(h.w & kStXMask), x, cpos_at);
@@ -906,7 +902,7 @@ int planes_of32(int D) { return D <= 2 ? 1 : (D <= 4 ? 2 : 4); }
 int eval32_task_size(int cpl) { return warps_for(cpl) * 32 * cpl; }
 
 int eval32_smem_bytes(const EvalParams &p, int search_mode) {
-    const int cpl = p.cpl32 == 1 ? 1 : (p.cpl32 == 4 ? 4 : 2);
+    const int cpl = p.cpl32 == 1 ? 1 : 2;
     const int nw = warps_for(cpl);
     const int pl = planes_of32(p.D);
     const size_t tb = ((search_mode == 1 || search_mode == 5) && p.wide32) ? 8 : 4;   // bytes per time value
@@ -946,10 +942,6 @@ int eval32_smem_bytes(const EvalParams &p, int search_mode) {
 #define PESTO_DISPATCH32(FN, ...)                                                          \
     do {                                                                                   \
         if (p.cpl32 == 1) PESTO_DISPATCH32_C(FN, 1, __VA_ARGS__);                          \
-        if (p.cpl32 == 4 && search_mode == 1 && p.coarse_pct == 0) {  /* search only */    \
-            if (planes_of32(p.D) == 1) return FN<1, 1, 4>(__VA_ARGS__);                    \
-            if (planes_of32(p.D) == 2) return FN<1, 2, 4>(__VA_ARGS__);                    \
-        }                                                                                  \
         PESTO_DISPATCH32_C(FN, 2, __VA_ARGS__);                                            \
     } while (0)
 

@@ -236,13 +236,6 @@ pesto_status launch_search_eval(pesto_search *s, int b_first, int n_bases, int64
         EvalParams p32 = p;
         p32.gate = 1;
         plan_eval32(g, p32, j0, j1, n_bases);
-        // four candidates per lane (2-warp CTAs, the same 256-candidate task) for multi-wave
-        // search launches: PESTO_EVAL32_CPL=4 (experiment; D <= 4, no S9 coarse groups)
-        static const bool cpl4 = [] {
-            const char *e = std::getenv("PESTO_EVAL32_CPL");
-            return e && std::atoi(e) == 4;
-        }();
-        if (cpl4 && p32.cpl32 == 2 && g->planes <= 2 && s->coarse_pct == 0) p32.cpl32 = 4;
         if ((rc = ensure_state32(g, p32, 1, p32.n_tasks, &grid))) return rc;
         p32.state32 = g->d_state32.as<uint32_t>();
         if ((e = launch_eval32(p32, 1, grid, st)) != cudaSuccess) return cuda_fail(e, "launch eval32");
