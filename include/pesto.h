@@ -203,6 +203,24 @@ pesto_status pesto_eval_batch_host(pesto_graph *g, const int32_t *order,
                                    const void *placements_host, int64_t row_stride_bytes,
                                    int64_t n_cand, int64_t *makespans_host, void *cuda_stream);
 
+/* Asynchronous host-buffer evaluation.  A workspace owns a private set of evaluation scratch
+ * (rows and makespans staging, bit-sliced rows, slot state) on the graph's GPU, so calls on
+ * different workspaces (on different streams) may be in flight at once -- e.g. the host->device
+ * copy of one batch overlapping the evaluation of the previous one (double buffering).
+ * pesto_eval_batch_host_async = pesto_eval_batch_host on the workspace's scratch, enqueued on
+ * cuda_stream WITHOUT synchronising: the caller synchronises that stream before reading
+ * makespans_host, before reusing placements_host, and before the next call on the same
+ * workspace from another stream.  placements_host should be pinned (else the copy is
+ * synchronous).  The graph and its layouts are shared (not thread-safe: one host thread).
+ * Errors as pesto_eval_batch_host; create: EINVAL, ESTATE (host-only graph), ENOMEM. */
+typedef struct pesto_workspace pesto_workspace;
+pesto_status pesto_workspace_create(pesto_graph *g, pesto_workspace **out);
+void pesto_workspace_destroy(pesto_workspace *w);                      /* NULL-safe */
+pesto_status pesto_eval_batch_host_async(pesto_workspace *w, const int32_t *order,
+                                         const void *placements_host, int64_t row_stride_bytes,
+                                         int64_t n_cand, int64_t *makespans_host,
+                                         void *cuda_stream);
+
 /* ------------------------------------------------------------------------------------------ */
 /* Parallel local search (DESIGN.md §4 for the move spec)         */
 /* ------------------------------------------------------------------------------------------ */

@@ -258,8 +258,8 @@ pesto_status pesto_eval_coarse_exhaustive(pesto_graph *g, const int32_t *order,
     std::copy(cmask.begin(), cmask.end(), p.coarse_allowed);
     plan_eval32(g, p, 0, total, 1);
     int grid = 0;
-    if ((s = ensure_state32(g, p, 4, p.n_tasks, &grid))) return s;
-    p.state32 = g->d_state32.as<uint32_t>();
+    if ((s = ensure_state32(g, g->ws, p, 4, p.n_tasks, &grid))) return s;
+    p.state32 = g->ws.state32.as<uint32_t>();
     if ((e = launch_eval32(p, 4, grid, st)) != cudaSuccess) return cuda_fail(e, "launch exhaustive coarse search");
     uint64_t key = ~0ull;
     if ((e = cudaMemcpyAsync(&key, g->d_ckey.ptr, 8, cudaMemcpyDeviceToHost, st)) != cudaSuccess ||

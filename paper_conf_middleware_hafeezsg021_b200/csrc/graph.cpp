@@ -3,6 +3,7 @@
 #include <algorithm>
 #include <cstdlib>
 #include <cstring>
+#include <new>
 #include <queue>
 #include <string>
 
@@ -205,7 +206,7 @@ pesto_status nd_ensure_layout(pesto_graph *g, Layout &L) {
     return PESTO_OK;
 }
 
-pesto_status nd_fill(pesto_graph *g, NdParams &p, int64_t n_tasks, int *grid_out) {
+pesto_status nd_fill(pesto_graph *g, Scratch &ws, NdParams &p, int64_t n_tasks, int *grid_out) {
     std::memset(&p, 0, sizeof p);
     p.n = g->n;
     p.D = g->D;
@@ -236,13 +237,13 @@ pesto_status nd_fill(pesto_graph *g, NdParams &p, int64_t n_tasks, int *grid_out
     grid = std::max<int64_t>(grid, 1);
     const size_t slots = (size_t)grid * p.warps_per_cta;
     cudaError_t e;
-    if ((e = g->d_nd_rem.ensure(slots * g->n * 4)) != cudaSuccess ||
-        (e = g->d_nd_rdy.ensure(slots * g->n * 8)) != cudaSuccess ||
-        (e = g->d_nd_pend.ensure(slots * g->n * g->D * 8)) != cudaSuccess)
+    if ((e = ws.nd_rem.ensure(slots * g->n * 4)) != cudaSuccess ||
+        (e = ws.nd_rdy.ensure(slots * g->n * 8)) != cudaSuccess ||
+        (e = ws.nd_pend.ensure(slots * g->n * g->D * 8)) != cudaSuccess)
         return cuda_fail(e, "allocate non-delay scratch");
-    p.rem = g->d_nd_rem.as<int32_t>();
-    p.rdy = g->d_nd_rdy.as<int64_t>();
-    p.pend = g->d_nd_pend.as<uint64_t>();
+    p.rem = ws.nd_rem.as<int32_t>();
+    p.rdy = ws.nd_rdy.as<int64_t>();
+    p.pend = ws.nd_pend.as<uint64_t>();
     *grid_out = (int)grid;
     return PESTO_OK;
 }
@@ -262,8 +263,8 @@ void fill_eval_common(const pesto_graph *g, EvalParams &p) {
     p.all_allowed = g->all_allowed ? 1 : 0;
 }
 
-pesto_status ensure_state(pesto_graph *g, const EvalParams &p, int search_mode, int64_t n_tasks,
-                          int *grid_out) {
+pesto_status ensure_state(pesto_graph *g, Scratch &ws, const EvalParams &p, int search_mode,
+                          int64_t n_tasks, int *grid_out) {
     int per_sm = eval_max_ctas_per_sm(p, search_mode);
     if (per_sm <= 0)
         return fail(PESTO_ECUDA, "eval kernel does not fit on an SM (smem " +
@@ -271,7 +272,7 @@ pesto_status ensure_state(pesto_graph *g, const EvalParams &p, int search_mode, 
     int64_t grid = std::min<int64_t>(n_tasks, (int64_t)g->sms * per_sm);
     grid = std::max<int64_t>(grid, 1);
     size_t bytes = (size_t)grid * kWarps * (size_t)std::max(p.max_W, 1) * 32 * sizeof(int64_t);
-    cudaError_t e = g->d_state.ensure(bytes);
+    cudaError_t e = ws.state.ensure(bytes);
     if (e != cudaSuccess) return cuda_fail(e, "allocate slot state");
     *grid_out = (int)grid;
     return PESTO_OK;
@@ -296,8 +297,8 @@ void plan_eval32(const pesto_graph *g, EvalParams &p, int64_t j0, int64_t j1, in
     p.n_tasks = p.tasks_per_base * n_bases;
 }
 
-pesto_status ensure_state32(pesto_graph *g, const EvalParams &p, int search_mode, int64_t n_tasks,
-                            int *grid_out) {
+pesto_status ensure_state32(pesto_graph *g, Scratch &ws, const EvalParams &p, int search_mode,
+                            int64_t n_tasks, int *grid_out) {
     int per_sm = eval32_max_ctas_per_sm(p, search_mode);
     if (per_sm <= 0)
         return fail(PESTO_ECUDA, "eval32 kernel does not fit on an SM (smem " +
@@ -306,7 +307,7 @@ pesto_status ensure_state32(pesto_graph *g, const EvalParams &p, int search_mode
     grid = std::max<int64_t>(grid, 1);
     size_t bytes = (size_t)grid * eval32_task_size(p.cpl32) * (size_t)std::max(p.max_W32, 1) *
                    (p.wide32 ? sizeof(uint64_t) : sizeof(uint32_t));
-    cudaError_t e = g->d_state32.ensure(bytes);
+    cudaError_t e = ws.state32.ensure(bytes);
     if (e != cudaSuccess) return cuda_fail(e, "allocate cold slot state");
     *grid_out = (int)grid;
     return PESTO_OK;
@@ -715,8 +716,13 @@ pesto_status pesto_seed_placement(pesto_graph *g, int32_t kind, const int32_t *o
     return PESTO_OK;
 }
 
-pesto_status pesto_eval_batch(pesto_graph *g, const int32_t *order, const void *placements,
-                              int64_t stride, int64_t n_cand, int64_t *makespans, void *stream) {
+}  // extern "C"
+
+namespace {
+
+// pesto_eval_batch on the scratch set ws (the graph's own, or a workspace's)
+pesto_status eval_batch_ws(pesto_graph *g, Scratch &ws, const int32_t *order, const void *placements,
+                           int64_t stride, int64_t n_cand, int64_t *makespans, void *stream) {
     if (!g) return fail(PESTO_EINVAL, "NULL graph");
     if (g->device < 0) return fail(PESTO_ESTATE, "host-only graph handle");
     if (n_cand < 0) return fail(PESTO_EINVAL, "n_cand < 0");
@@ -732,9 +738,9 @@ pesto_status pesto_eval_batch(pesto_graph *g, const int32_t *order, const void *
     if ((s = upload_layout(g, *L))) return s;
     cudaStream_t st = (cudaStream_t)stream;
     const int64_t n_groups = (n_cand + 31) / 32;
-    cudaError_t e = g->d_planes.ensure((size_t)n_groups * g->n * g->planes * 4);
+    cudaError_t e = ws.planes.ensure((size_t)n_groups * g->n * g->planes * 4);
     if (e != cudaSuccess) return cuda_fail(e, "allocate bit-sliced placements");
-    if ((e = g->d_invalid.ensure((size_t)n_groups * 4)) != cudaSuccess) return cuda_fail(e, "allocate");
+    if ((e = ws.invalid.ensure((size_t)n_groups * 4)) != cudaSuccess) return cuda_fail(e, "allocate");
     TransposeParams tp{};
     tp.rows = static_cast<const uint8_t *>(placements);
     tp.stride = stride;
@@ -744,8 +750,8 @@ pesto_status pesto_eval_batch(pesto_graph *g, const int32_t *order, const void *
     tp.planes = g->planes;
     tp.pos_of = L->d_pos.as<int32_t>();
     tp.fmask = g->d_fmask.as<uint16_t>();
-    tp.planes_out = g->d_planes.as<uint32_t>();
-    tp.invalid_out = g->d_invalid.as<uint32_t>();
+    tp.planes_out = ws.planes.as<uint32_t>();
+    tp.invalid_out = ws.invalid.as<uint32_t>();
     // the successors' codes in eval32 walk order (edge slots), for the explicit-row walk
     const bool nondelay = g->dispatch == PESTO_DISPATCH_NONDELAY;
     if (nondelay) {
@@ -756,15 +762,15 @@ pesto_status pesto_eval_batch(pesto_graph *g, const int32_t *order, const void *
     if (ystream) {
         tp.slot_succ = L->d_slot_succ.as<int32_t>();
         tp.n_slots = (int64_t)L->slot_succ.size();
-        if ((e = g->d_yplanes.ensure((size_t)n_groups * tp.n_slots * g->planes * 4)) != cudaSuccess)
+        if ((e = ws.yplanes.ensure((size_t)n_groups * tp.n_slots * g->planes * 4)) != cudaSuccess)
             return cuda_fail(e, "allocate edge-slot stream");
-        tp.yplanes_out = g->d_yplanes.as<uint32_t>();
+        tp.yplanes_out = ws.yplanes.as<uint32_t>();
     }
     if ((e = launch_transpose(tp, st)) != cudaSuccess) return cuda_fail(e, "launch transpose");
     if (g->has_cap || g->has_coloc) {                 // row f3: mark infeasible rows
         FeasParams fp{};
-        fp.planes = g->d_planes.as<uint32_t>();
-        fp.invalid = g->d_invalid.as<uint32_t>();
+        fp.planes = ws.planes.as<uint32_t>();
+        fp.invalid = ws.invalid.as<uint32_t>();
         fp.n_groups = n_groups;
         fp.n = g->n;
         fp.D = g->D;
@@ -777,11 +783,11 @@ pesto_status pesto_eval_batch(pesto_graph *g, const int32_t *order, const void *
     if (nondelay) {                                   // row f4(i): one warp per row
         NdParams np;
         int grid = 0;
-        if ((s = nd_fill(g, np, n_cand, &grid))) return s;
+        if ((s = nd_fill(g, ws, np, n_cand, &grid))) return s;
         np.rows = tp.rows;
         np.stride = stride;
         np.n_cand = n_cand;
-        np.invalid = g->d_invalid.as<uint32_t>();
+        np.invalid = ws.invalid.as<uint32_t>();
         np.makespans = makespans;
         np.nd_dst = L->d_nd_dst.as<int32_t>();
         np.nd_t = L->d_nd_t.as<int64_t>();
@@ -796,10 +802,10 @@ pesto_status pesto_eval_batch(pesto_graph *g, const int32_t *order, const void *
     p.max_W = L->W;
     p.stage_bytes32 = L->stage_bytes32;
     p.max_W32 = L->W32;
-    p.planes_in = g->d_planes.as<uint32_t>();
-    p.yplanes = g->d_yplanes.as<uint32_t>();
+    p.planes_in = ws.planes.as<uint32_t>();
+    p.yplanes = ws.yplanes.as<uint32_t>();
     p.n_slots = (int64_t)L->slot_succ.size();
-    p.invalid = g->d_invalid.as<uint32_t>();
+    p.invalid = ws.invalid.as<uint32_t>();
     p.n_cand = n_cand;
     p.makespans = makespans;
     p.bases = L->d_view.as<BaseLayoutDev>();
@@ -811,51 +817,100 @@ pesto_status pesto_eval_batch(pesto_graph *g, const int32_t *order, const void *
     // 64-bit path for every row: ineligible durations, no eval32 stream, or congestion-free
     // links (row f4(ii) is a modelling variant; eval32 carries only the FCFS link queues)
     if (!g->eligible32 || L->W32 == 0 || g->link_model != PESTO_LINKS_FCFS) {
-        if ((s = ensure_state(g, p, 0, p.n_tasks, &grid))) return s;
-        p.state = g->d_state.as<int64_t>();
+        if ((s = ensure_state(g, ws, p, 0, p.n_tasks, &grid))) return s;
+        p.state = ws.state.as<int64_t>();
         if ((e = launch_eval(p, 0, grid, st)) != cudaSuccess) return cuda_fail(e, "launch eval");
         return PESTO_OK;
     }
     // fast path: 32-bit saturating K1; rows that saturate are listed and re-run in 64-bit
-    if ((e = g->d_flags.ensure((size_t)(n_cand + 4) * 4)) != cudaSuccess) return cuda_fail(e, "allocate");
-    if ((e = cudaMemsetAsync(g->d_flags.ptr, 0, 4, st)) != cudaSuccess) return cuda_fail(e, "reset flags");
-    p.flag_count = g->d_flags.as<int32_t>();
-    p.flag_list = g->d_flags.as<int32_t>() + 4;
+    if ((e = ws.flags.ensure((size_t)(n_cand + 4) * 4)) != cudaSuccess) return cuda_fail(e, "allocate");
+    if ((e = cudaMemsetAsync(ws.flags.ptr, 0, 4, st)) != cudaSuccess) return cuda_fail(e, "reset flags");
+    p.flag_count = ws.flags.as<int32_t>();
+    p.flag_list = ws.flags.as<int32_t>() + 4;
     {
         EvalParams p32 = p;
         plan_eval32(g, p32, 0, n_cand, 1);
-        if ((s = ensure_state32(g, p32, 0, p32.n_tasks, &grid))) return s;
-        p32.state32 = g->d_state32.as<uint32_t>();
+        if ((s = ensure_state32(g, ws, p32, 0, p32.n_tasks, &grid))) return s;
+        p32.state32 = ws.state32.as<uint32_t>();
         if ((e = launch_eval32(p32, 0, grid, st)) != cudaSuccess) return cuda_fail(e, "launch eval32");
     }
     p.list = p.flag_list;
     p.list_count = p.flag_count;
     const int64_t fix_tasks = std::min<int64_t>(p.n_tasks, g->sms);
-    if ((s = ensure_state(g, p, 2, fix_tasks, &grid))) return s;
-    p.state = g->d_state.as<int64_t>();
+    if ((s = ensure_state(g, ws, p, 2, fix_tasks, &grid))) return s;
+    p.state = ws.state.as<int64_t>();
     if ((e = launch_eval(p, 2, grid, st)) != cudaSuccess) return cuda_fail(e, "launch eval fixup");
     return PESTO_OK;
 }
 
-pesto_status pesto_eval_batch_host(pesto_graph *g, const int32_t *order, const void *rows,
-                                   int64_t stride, int64_t n_cand, int64_t *mk_host, void *stream) {
+// rows copied in from host memory, evaluated, makespans copied out -- all enqueued on stream
+pesto_status eval_batch_host_ws(pesto_graph *g, Scratch &ws, const int32_t *order, const void *rows,
+                                int64_t stride, int64_t n_cand, int64_t *mk_host, void *stream) {
     if (!g) return fail(PESTO_EINVAL, "NULL graph");
     if (g->device < 0) return fail(PESTO_ESTATE, "host-only graph handle");
     if (n_cand <= 0) return n_cand == 0 ? PESTO_OK : fail(PESTO_EINVAL, "n_cand < 0");
     if (!rows || !mk_host) return fail(PESTO_EINVAL, "NULL buffer");
     DeviceGuard guard(g->device);
     cudaStream_t st = (cudaStream_t)stream;
-    cudaError_t e = g->d_rows.ensure((size_t)n_cand * stride);
+    cudaError_t e = ws.rows.ensure((size_t)n_cand * stride);
     if (e != cudaSuccess) return cuda_fail(e, "allocate rows");
-    if ((e = g->d_out.ensure((size_t)n_cand * 8)) != cudaSuccess) return cuda_fail(e, "allocate out");
-    if ((e = cudaMemcpyAsync(g->d_rows.ptr, rows, (size_t)n_cand * stride, cudaMemcpyHostToDevice, st)) != cudaSuccess)
+    if ((e = ws.out.ensure((size_t)n_cand * 8)) != cudaSuccess) return cuda_fail(e, "allocate out");
+    if ((e = cudaMemcpyAsync(ws.rows.ptr, rows, (size_t)n_cand * stride, cudaMemcpyHostToDevice, st)) != cudaSuccess)
         return cuda_fail(e, "copy rows in");
-    pesto_status s = pesto_eval_batch(g, order, g->d_rows.ptr, stride, n_cand, g->d_out.as<int64_t>(), stream);
+    pesto_status s = eval_batch_ws(g, ws, order, ws.rows.ptr, stride, n_cand, ws.out.as<int64_t>(), stream);
     if (s) return s;
-    if ((e = cudaMemcpyAsync(mk_host, g->d_out.ptr, (size_t)n_cand * 8, cudaMemcpyDeviceToHost, st)) != cudaSuccess)
+    if ((e = cudaMemcpyAsync(mk_host, ws.out.ptr, (size_t)n_cand * 8, cudaMemcpyDeviceToHost, st)) != cudaSuccess)
         return cuda_fail(e, "copy makespans out");
-    if ((e = cudaStreamSynchronize(st)) != cudaSuccess) return cuda_fail(e, "eval_batch_host");
     return PESTO_OK;
+}
+
+}  // namespace
+
+struct pesto_workspace {
+    pesto_graph *g = nullptr;
+    Scratch ws;
+};
+
+extern "C" {
+
+pesto_status pesto_eval_batch(pesto_graph *g, const int32_t *order, const void *placements,
+                              int64_t stride, int64_t n_cand, int64_t *makespans, void *stream) {
+    if (!g) return fail(PESTO_EINVAL, "NULL graph");
+    return eval_batch_ws(g, g->ws, order, placements, stride, n_cand, makespans, stream);
+}
+
+pesto_status pesto_eval_batch_host(pesto_graph *g, const int32_t *order, const void *rows,
+                                   int64_t stride, int64_t n_cand, int64_t *mk_host, void *stream) {
+    if (!g) return fail(PESTO_EINVAL, "NULL graph");
+    pesto_status s = eval_batch_host_ws(g, g->ws, order, rows, stride, n_cand, mk_host, stream);
+    if (s || n_cand == 0) return s;
+    DeviceGuard guard(g->device);
+    cudaError_t e = cudaStreamSynchronize((cudaStream_t)stream);
+    return e == cudaSuccess ? PESTO_OK : cuda_fail(e, "eval_batch_host");
+}
+
+pesto_status pesto_workspace_create(pesto_graph *g, pesto_workspace **out) {
+    if (!g || !out) return fail(PESTO_EINVAL, "NULL argument");
+    *out = nullptr;
+    if (g->device < 0) return fail(PESTO_ESTATE, "host-only graph handle");
+    pesto_workspace *w = new (std::nothrow) pesto_workspace();
+    if (!w) return fail(PESTO_ENOMEM, "workspace");
+    w->g = g;
+    *out = w;
+    return PESTO_OK;
+}
+
+void pesto_workspace_destroy(pesto_workspace *w) {
+    if (!w) return;
+    DeviceGuard guard(w->g->device);
+    delete w;                           // DevBuf frees synchronise with the device
+}
+
+pesto_status pesto_eval_batch_host_async(pesto_workspace *w, const int32_t *order, const void *rows,
+                                         int64_t stride, int64_t n_cand, int64_t *mk_host,
+                                         void *stream) {
+    if (!w) return fail(PESTO_EINVAL, "NULL workspace");
+    return eval_batch_host_ws(w->g, w->ws, order, rows, stride, n_cand, mk_host, stream);
 }
 
 }  // extern "C"

@@ -75,6 +75,18 @@ struct Layout {
     bool on_device = false;
 };
 
+// Evaluation scratch (device): one set per graph for the synchronous calls and the search, one
+// per pesto_workspace for asynchronous host-buffer evaluations that may overlap each other.
+struct Scratch {
+    DevBuf state;                 // eval64 ready-time slots
+    DevBuf state32;               // eval32 cold slots
+    DevBuf planes, invalid;       // K5: bit-sliced rows, per-group infeasible-lane masks
+    DevBuf yplanes;               // K5: codes per eval32 edge slot (explicit rows)
+    DevBuf flags;                 // [count | list of saturated candidates]
+    DevBuf rows, out;             // host-buffer calls: rows copied in, makespans copied out
+    DevBuf nd_rem, nd_rdy, nd_pend;   // row f4(i) per-warp scratch
+};
+
 }  // namespace pesto
 
 struct pesto_graph {
@@ -107,12 +119,12 @@ struct pesto_graph {
     // layout cache (most recent first)
     std::list<std::shared_ptr<pesto::Layout>> cache;
     // device buffers
-    pesto::DevBuf d_state, d_planes, d_invalid, d_fmask, d_movable, d_allowed, d_bases, d_rows,
-        d_out, d_state32, d_flags;        // d_flags: [count | list of saturated candidates]
+    pesto::DevBuf d_fmask, d_movable, d_allowed, d_bases;
+    pesto::Scratch ws;                    // scratch of the synchronous calls and the search
     int32_t sms = 148;
     int32_t link_model = 0;               // PESTO_LINKS_FCFS / PESTO_LINKS_UNLIMITED
     int32_t dispatch = 0;                 // PESTO_DISPATCH_FIXED / PESTO_DISPATCH_NONDELAY
-    pesto::DevBuf d_nd_p, d_nd_indeg, d_nd_off, d_nd_rem, d_nd_rdy, d_nd_pend;
+    pesto::DevBuf d_nd_p, d_nd_indeg, d_nd_off;
     bool nd_graph_ready = false;
     // row f3 constraints (host copies + device arrays); cons_gen counts changes
     bool has_cap = false, has_coloc = false;
@@ -122,7 +134,6 @@ struct pesto_graph {
     int64_t cons_gen = 0;
     pesto::DevBuf d_mem, d_cap, d_coloc, d_coloc_size, d_coloc_pairs;
     pesto::DevBuf d_cpos, d_ckey;         // row f2 exhaustive coarse search
-    pesto::DevBuf d_yplanes;              // explicit rows: codes per eval32 edge slot
 };
 
 namespace pesto {
@@ -138,7 +149,7 @@ bool pair_blocked(const pesto_graph *g, int32_t a, int32_t c);
 // check (positive durations, n <= 2^20) and the scratch for `slots` resident warps
 pesto_status nd_check(pesto_graph *g);
 pesto_status nd_ensure_layout(pesto_graph *g, Layout &L);
-pesto_status nd_fill(pesto_graph *g, NdParams &p, int64_t n_tasks, int *grid_out);
+pesto_status nd_fill(pesto_graph *g, Scratch &ws, NdParams &p, int64_t n_tasks, int *grid_out);
 // row f2: PAPER.md §3.3 coarsening to at most `target` merged vertices (coarsen.cpp)
 pesto_status coarsen_graph(const pesto_graph *g, int32_t target, std::vector<int32_t> &coarse_of,
                            int32_t &n_coarse);
@@ -147,16 +158,16 @@ Feasibility feasibility_view(const pesto_graph *g);
 bool placement_feasible(const pesto_graph *g, const uint8_t *x, int64_t *footprint8);
 BaseLayoutDev layout_view(const Layout &L);
 void fill_eval_common(const pesto_graph *g, EvalParams &p);
-pesto_status ensure_state(pesto_graph *g, const EvalParams &p, int search_mode, int64_t n_tasks,
-                          int *grid_out);
+pesto_status ensure_state(pesto_graph *g, Scratch &ws, const EvalParams &p, int search_mode,
+                          int64_t n_tasks, int *grid_out);
 // eval32 candidates per lane for a launch of n_tasks 256-candidate tasks:
 // 1 when every task is resident at once (latency-bound: more warps), else 2
 int choose_cpl32(const pesto_graph *g, int64_t n_tasks);
 // eval32 launch plan for candidate ids [j0, j1) of n_bases bases: p.cpl32 (from the launch size
 // in 256-candidate units), p.tasks_per_base and p.n_tasks in tasks of eval32_task_size(cpl)
 void plan_eval32(const pesto_graph *g, EvalParams &p, int64_t j0, int64_t j1, int n_bases);
-pesto_status ensure_state32(pesto_graph *g, const EvalParams &p, int search_mode, int64_t n_tasks,
-                            int *grid_out);
+pesto_status ensure_state32(pesto_graph *g, Scratch &ws, const EvalParams &p, int search_mode,
+                            int64_t n_tasks, int *grid_out);
 struct DeviceGuard {
     int prev = -1;
     explicit DeviceGuard(int dev) {

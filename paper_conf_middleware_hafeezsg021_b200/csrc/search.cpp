@@ -165,7 +165,7 @@ pesto_status launch_search_nondelay(pesto_search *s, int b_first, int n_bases, i
     NdParams p;
     int grid = 0;
     const int64_t n_tasks = (int64_t)n_bases * (j1 - j0);
-    if ((rc = nd_fill(g, p, n_tasks, &grid))) return rc;
+    if ((rc = nd_fill(g, g->ws, p, n_tasks, &grid))) return rc;
     p.feas.fbase = s->d_fbase.as<int64_t>() + (size_t)b_first * 8;
     p.bases = s->d_views.as<BaseLayoutDev>() + b_first;
     p.n_bases = n_bases;
@@ -236,8 +236,8 @@ pesto_status launch_search_eval(pesto_search *s, int b_first, int n_bases, int64
         EvalParams p32 = p;
         p32.gate = 1;
         plan_eval32(g, p32, j0, j1, n_bases);
-        if ((rc = ensure_state32(g, p32, 1, p32.n_tasks, &grid))) return rc;
-        p32.state32 = g->d_state32.as<uint32_t>();
+        if ((rc = ensure_state32(g, g->ws, p32, 1, p32.n_tasks, &grid))) return rc;
+        p32.state32 = g->ws.state32.as<uint32_t>();
         if ((e = launch_eval32(p32, 1, grid, st)) != cudaSuccess) return cuda_fail(e, "launch eval32");
         if (s->all_below) return PESTO_OK;
         // bases at or above saturation: the wide eval32 instance (exact 64-bit times, the
@@ -254,13 +254,13 @@ pesto_status launch_search_eval(pesto_search *s, int b_first, int n_bases, int64
             p32.tasks_per_base = (j1 - (j0 - j0 % ts) + ts - 1) / ts;
             p32.n_tasks = p32.tasks_per_base * n_bases;
         }
-        if ((rc = ensure_state32(g, p32, 1, p32.n_tasks, &grid))) return rc;
-        p32.state32 = g->d_state32.as<uint32_t>();
+        if ((rc = ensure_state32(g, g->ws, p32, 1, p32.n_tasks, &grid))) return rc;
+        p32.state32 = g->ws.state32.as<uint32_t>();
         if ((e = launch_eval32(p32, 1, grid, st)) != cudaSuccess) return cuda_fail(e, "launch wide eval32");
         return PESTO_OK;
     }
-    if ((rc = ensure_state(g, p, 1, p.n_tasks, &grid))) return rc;
-    p.state = g->d_state.as<int64_t>();
+    if ((rc = ensure_state(g, g->ws, p, 1, p.n_tasks, &grid))) return rc;
+    p.state = g->ws.state.as<int64_t>();
     if ((e = launch_eval(p, 1, grid, st)) != cudaSuccess) return cuda_fail(e, "launch search eval");
     return PESTO_OK;
 }

@@ -71,6 +71,9 @@ SIGNATURES = {
     "pesto_seed_placement": (_I32, [_VP, _I32, _VP, _VP, _U64, _VP]),
     "pesto_eval_batch": (_I32, [_VP, _VP, _VP, _I64, _I64, _VP, _VP]),
     "pesto_eval_batch_host": (_I32, [_VP, _VP, _VP, _I64, _I64, _VP, _VP]),
+    "pesto_workspace_create": (_I32, [_VP, C.POINTER(_VP)]),
+    "pesto_workspace_destroy": (None, [_VP]),
+    "pesto_eval_batch_host_async": (_I32, [_VP, _VP, _VP, _I64, _I64, _VP, _VP]),
     "pesto_search_create": (_I32, [_VP, C.POINTER(SearchDesc), C.POINTER(_VP)]),
     "pesto_search_step": (_I32, [_VP, _VP]),
     "pesto_search_eval": (_I32, [_VP, _VP]),
@@ -266,6 +269,36 @@ class Graph:
             out = np.empty(n_cand, dtype=np.int64)
         _check(_L.pesto_eval_batch_host(self._h, _ptr(o), rows.ctypes.data, stride, n_cand,
                                         out.ctypes.data, _stream(stream)))
+        return out
+
+    def workspace(self) -> "Workspace":
+        return Workspace(self)
+
+
+class Workspace:
+    """Private evaluation scratch (pesto_workspace) for asynchronous host-buffer batches."""
+
+    def __init__(self, graph: Graph):
+        self.graph = graph
+        h = _VP()
+        _check(_L.pesto_workspace_create(graph._h, C.byref(h)))
+        self._h = h
+
+    def __del__(self):
+        h = getattr(self, "_h", None)
+        if h:
+            _L.pesto_workspace_destroy(h)
+            self._h = None
+
+    def eval_host_async(self, order, rows: np.ndarray, out: np.ndarray, stream=None):
+        """Enqueue rows (pinned host) -> out (pinned host int64) on `stream`; no synchronisation:
+        synchronise the stream before reading `out` or reusing `rows`."""
+        o = np.ascontiguousarray(order, dtype=np.int32)
+        n_cand, stride = rows.shape
+        if out.shape != (n_cand,) or out.dtype != np.int64:
+            raise ValueError("out must be an int64 array with one entry per row")
+        _check(_L.pesto_eval_batch_host_async(self._h, _ptr(o), rows.ctypes.data, stride, n_cand,
+                                              out.ctypes.data, _stream(stream)))
         return out
 
 

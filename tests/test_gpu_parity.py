@@ -228,6 +228,35 @@ def test_search_steps_match_reference(P, O):
 
 
 @pytest.mark.parametrize("D", [2, 4])
+def test_async_workspaces_double_buffered(P, O, D):
+    """pesto_eval_batch_host_async: four batches on two workspaces / two streams in flight at
+    once (the e2e pattern of bench.py); every makespan equals the oracle's"""
+    import torch
+    g = dag.random_dag(321 + D, 900, 1.5, D=D, p_max=4000, max_bytes=300_000, beta0=700,
+                       beta1_fs=30_000, allowed_frac=0.3)
+    G = P.Graph.from_arrays(g)
+    order = dag.random_topo_order(g, 5)
+    xs = [dag.random_placements(g, 40 + i, 700 + 37 * i) for i in range(4)]
+    rows = [torch.from_numpy(P.pack_rows(x, g.D)).pin_memory().numpy() for x in xs]
+    outs = [torch.empty(len(x), dtype=torch.int64).pin_memory().numpy() for x in xs]
+    wss = [G.workspace(), G.workspace()]
+    sts = [torch.cuda.Stream(), torch.cuda.Stream()]
+    got = []
+    for i in range(4):
+        k = i & 1
+        if i >= 2:
+            sts[k].synchronize()
+            got.append(outs[i - 2].copy())
+        wss[k].eval_host_async(order, rows[i], outs[i], stream=sts[k])
+    for st in sts:
+        st.synchronize()
+    got += [outs[2].copy(), outs[3].copy()]
+    for i in range(4):
+        ref, _ = O.makespan_batch(g, xs[i], order)
+        assert (got[i] == ref).all(), i
+
+
+@pytest.mark.parametrize("D", [2, 4])
 def test_multiwave_search_steps(P, O, D):
     """search launches of more than one wave (2 x 131,072 candidates = 1,024 eval32 tasks: the
     multi-candidate-per-lane instances): each step's keys equal the oracle's
