@@ -684,10 +684,11 @@ eval32_kernel(const EvalParams P) {
                 const uint32_t tile = (uint32_t)s * sb;
                 const int32_t nsteps = (int32_t)lds_u32(cx.smem + tile);
                 uint32_t sp = cx.smem + tile + kTileHeader + (uint32_t)skip * kStepBytes;
-                int32_t i = skip;
+                // the tile's steps end at spe: the walk compares step addresses (no step counter)
+                const uint32_t spe = cx.smem + tile + kTileHeader + (uint32_t)nsteps * kStepBytes;
                 skip = 0;
                 uint4 h = lds_v4(sp), e0 = lds_v4(sp + 16), e1 = lds_v4(sp + 32);
-                while (i < nsteps) {
+                while (sp < spe) {
                     // the next step's head (past the tile's end: padding, never used); this
                     // step's edge records (their first use is after the head's work)
                     // (CPL = 1 reads its own head here: the read-ahead copy costs more than the
@@ -713,7 +714,7 @@ eval32_kernel(const EvalParams P) {
                             // every slot's first push is unchanged; only device and link queues
                             // see the new order.
                             const int32_t nk = (int32_t)(h.w >> kStStepsShift);
-                            const bool straddle = i + nk >= nsteps;
+                            const bool straddle = sp + (uint32_t)nk * kStepBytes >= spe;
                             uint32_t sp1;
                             if (straddle) {
                                 const int s2 = (it + 1) % kStages32;
@@ -758,7 +759,6 @@ eval32_kernel(const EvalParams P) {
                                 break;
                             }
                             sp = sp1 + (uint32_t)n1 * kStepBytes;
-                            i += nk + n1;
                             h = lds_v4(sp);
                             e0 = lds_v4(sp + 16);
                             e1 = lds_v4(sp + 32);
@@ -821,7 +821,6 @@ eval32_kernel(const EvalParams P) {
                         }
                     }
                     sp += kStepBytes;
-                    i++;
                     if constexpr (CPL != 1) h = hn;
                 }
             }
