@@ -538,6 +538,7 @@ eval32_kernel(const EvalParams P) {
         bool active;
         bool valid[CPL];
         int32_t ks = -1;
+        uint32_t off_ks = 0;         // search: byte offset of the op at ks in the step stream
         if (MODE == 4) {
             // exhaustive coarse placements (row f2): candidate j is its own placement code
             active = j0 < P.n_cand;
@@ -590,6 +591,7 @@ eval32_kernel(const EvalParams P) {
                      ? decode_swap(P.seed, cb, grp, P.n, P.mix[3], rg,
                                    [&](int32_t k) { return __ldg(blocked + k) != 0; })
                      : -1;
+            if (ks >= 0) off_ks = __ldg(B->op_off32 + ks);
             const int32_t *ord = B->order;
             const uint32_t *bits = B->bits;
             const uint8_t *aop = P.allowed_op;
@@ -688,140 +690,157 @@ eval32_kernel(const EvalParams P) {
                 const uint32_t spe = cx.smem + tile + kTileHeader + (uint32_t)nsteps * kStepBytes;
                 skip = 0;
                 uint4 h = lds_v4(sp), e0 = lds_v4(sp + 16), e1 = lds_v4(sp + 32);
-                while (sp < spe) {
-                    // the next step's head (past the tile's end: padding, never used); this
-                    // step's edge records (their first use is after the head's work)
-                    // (CPL = 1 reads its own head here: the read-ahead copy costs more than the
-                    // LDS latency it hides there -- measured 5.86 vs 5.77 ms on inception)
-                    uint4 hn;
-                    if constexpr (CPL == 1) h = lds_v4(sp);
-                    else hn = lds_v4(sp + 48);
-                    e0 = lds_v4(sp + 16);
-                    e1 = lds_v4(sp + 32);
-                    if constexpr (MODE == 0) {
-                        if (slot0 >= ywb + SW) {               // next window; prefetch the one after
+                // the search group's swapped pair (ks, ks+1): when the op at ks starts in this
+                // tile the walk's step limit is its first step, where the pair is walked in
+                // swapped order -- no per-op position test in the loop
+                uint32_t lim = spe;
+                if (kSearch && ks >= 0) {
+                    const uint32_t rel = off_ks - lds_u32(cx.smem + tile + 4);   // tile's blob offset
+                    if (rel < lds_u32(cx.smem + tile + 8)) lim = min(spe, cx.smem + tile + rel);
+                }
+                for (;;) {
+                    while (sp < lim) {
+                        // the next step's head (past the tile's end: padding, never used); this
+                        // step's edge records (their first use is after the head's work)
+                        // (CPL = 1 reads its own head here: the read-ahead copy costs more than the
+                        // LDS latency it hides there -- measured 5.86 vs 5.77 ms on inception)
+                        uint4 hn;
+                        if constexpr (CPL == 1) h = lds_v4(sp);
+                        else hn = lds_v4(sp + 48);
+                        e0 = lds_v4(sp + 16);
+                        e1 = lds_v4(sp + 32);
+                        if constexpr (MODE == 0) {
+                            if (slot0 >= ywb + SW) {               // next window; prefetch the one after
 #pragma unroll
-                            for (int c = 0; c < CPL; c++) yw[c] = yn[c];
-                            ywb += SW;
-                            y_load(ywb + SW, yn);
-                        }
-                    }
-                    if (!(h.w & kStCont)) {
-                        v++;
-                        if (kSearch && v == ks) {
-                            // swapped pair: the op at ks+1 runs first, then the op at ks.  They
-                            // share no producer, no consumer and no edge (DESIGN.md §4 S3), so
-                            // every slot's first push is unchanged; only device and link queues
-                            // see the new order.
-                            const int32_t nk = (int32_t)(h.w >> kStStepsShift);
-                            const bool straddle = sp + (uint32_t)nk * kStepBytes >= spe;
-                            uint32_t sp1;
-                            if (straddle) {
-                                const int s2 = (it + 1) % kStages32;
-                                mbar_wait(&full[s2], ((it + 1) / kStages32) & 1);
-                                sp1 = cx.smem + (uint32_t)s2 * sb + kTileHeader;
-                            } else {
-                                sp1 = sp + (uint32_t)nk * kStepBytes;
+                                for (int c = 0; c < CPL; c++) yw[c] = yn[c];
+                                ywb += SW;
+                                y_load(ywb + SW, yn);
                             }
-                            const uint4 h1 = lds_v4(sp1);
-                            const int32_t n1 = (int32_t)(h1.w >> kStStepsShift);
+                        }
+                        if (!(h.w & kStCont)) {
+                            v++;
                             issue_far(h, v);
-                            issue_far(h1, v + 1);
-                            cp_async_wait<kPrefetchDist - 1>();  // v+1 and v+2 have landed
-                            T r0[CPL], r1[CPL], f1[CPL], g1[CPL], zero[CPL];
-#pragma unroll
-                            for (int c = 0; c < CPL; c++) zero[c] = 0u;
-                            arrivals(h.w, nfar, nnear, fwd, r0);
-                            load_next(v + 1, f1, g1);
-                            arrivals(h1.w, f1, g1, zero, r1);   // ks+1's distance-1 producer is ks: none
+                            cp_async_wait<kPrefetchDist - 1>();      // v+1 has landed
+                            T r[CPL];
+                            arrivals(h.w, nfar, nnear, fwd, r);
+                            load_next(v + 1, nfar, nnear);
 #pragma unroll
                             for (int c = 0; c < CPL; c++) fwd[c] = 0u;
-                            place.at(v + 1, (int)(h1.w & kStXMask), x, cpos_at);
-                            begin32<CPL, T>(h1, st, r1, x, cc);
-                            for (int32_t q = 0; q < n1; q++) {
-                                const uint32_t a = sp1 + q * kStepBytes;
-                                edges32<PL, CPL, T>(cx, lds_u32(a + 12), lds_v4(a + 16), lds_v4(a + 32), x,
-                                                 cc, place_y, st, fwd);
+                            if constexpr (MODE == 0) {
+                                if (v >= xwb + SW) {               // next window; prefetch the one after
+#pragma unroll
+                                    for (int c = 0; c < CPL; c++) xw[c] = xn[c];
+                                    xwb += SW;
+                                    x_load(xwb + SW, xn);
+                                }
+#pragma unroll
+                                for (int c = 0; c < CPL; c++) {
+                                    PlaneWords<PL> w;
+#pragma unroll
+                                    for (int p = 0; p < PL; p++)
+                                        w.w[p] = __shfl_sync(0xffffffffu, xw[c], (v - xwb) * PL + p);
+                                    x[c] = plane_dev<PL>(w, lane, place.dmax);
+                                }
+                            } else {
+                                // outside the group's region every lane has the base device
+                                // (CPL = 2 only: with one candidate per lane the launch is
+                                // latency-bound and the branch-free selects schedule better)
+                                xu = (kSearch && CPL == 2 &&
+                                      (uint32_t)(v - place.rc) >= (uint32_t)place.rlen)
+                                         ? (int)(h.w & kStXMask) : -1;
+                                place.at(v, (int)(h.w & kStXMask), x, cpos_at);
                             }
-                            place.at(v, (int)(h.w & kStXMask), x, cpos_at);
-                            begin32<CPL, T>(h, st, r0, x, cc);
-                            edges32<PL, CPL, T>(cx, h.w, e0, e1, x, cc, place_y, st, fwd);
-                            for (int32_t q = 1; q < nk; q++) {
-                                const uint32_t a = sp + q * kStepBytes;
-                                edges32<PL, CPL, T>(cx, lds_u32(a + 12), lds_v4(a + 16), lds_v4(a + 32), x,
-                                                 cc, place_y, st, fwd);
-                            }
-                            v++;
-                            xu = -1;
-                            load_next(v + 1, nfar, nnear);
-                            if (straddle) {
-                                skip = n1;
-                                break;
-                            }
-                            sp = sp1 + (uint32_t)n1 * kStepBytes;
-                            h = lds_v4(sp);
-                            e0 = lds_v4(sp + 16);
-                            e1 = lds_v4(sp + 32);
-                            continue;
+                            if (MODE != 0 && xu >= 0) st.begin_u(xu, h.x, r, cc);
+                            else begin32<CPL, T>(h, st, r, x, cc);
                         }
+                        if constexpr (MODE == 0) {
+                            edges32<PL, CPL, T>(cx, h.w, e0, e1, x, cc, pw_y, st, fwd);
+                            slot0 += 2;
+                        } else {
+                            const uint32_t ne = (h.w >> kStEdgeShift) & 3u;
+                            if (xu >= 0) {
+                                if (ne >= 1) {
+                                    const int32_t q0 = (int32_t)(e0.y & kSuccPosMask);
+                                    if ((uint32_t)(q0 - place.rc) >= (uint32_t)place.rlen)
+                                        push32_u<PL, CPL, T>(cx, e0, xu, (int)((e0.y >> kSuccXShift) & 7u), cc, st, fwd);
+                                    else { int y[CPL]; place_y(0, e0, y); push32<PL, CPL, T>(cx, e0, x, y, cc, st, fwd); }
+                                }
+                                if (ne >= 2) {
+                                    const int32_t q1 = (int32_t)(e1.y & kSuccPosMask);
+                                    if ((uint32_t)(q1 - place.rc) >= (uint32_t)place.rlen)
+                                        push32_u<PL, CPL, T>(cx, e1, xu, (int)((e1.y >> kSuccXShift) & 7u), cc, st, fwd);
+                                    else { int y[CPL]; place_y(1, e1, y); push32<PL, CPL, T>(cx, e1, x, y, cc, st, fwd); }
+                                }
+                            } else {
+                                edges32<PL, CPL, T>(cx, h.w, e0, e1, x, cc, place_y, st, fwd);
+                            }
+                        }
+                        sp += kStepBytes;
+                        if constexpr (CPL != 1) h = hn;
+                    }
+                    if (!kSearch || sp >= spe) break;
+                    // sp = the first step of the op at ks (a walk stops there only for ks)
+                    lim = spe;
+                    if constexpr (CPL == 1) h = lds_v4(sp);
+                    e0 = lds_v4(sp + 16);
+                    e1 = lds_v4(sp + 32);
+                    v++;
+                    {
+                        // swapped pair: the op at ks+1 runs first, then the op at ks.  They
+                        // share no producer, no consumer and no edge (DESIGN.md §4 S3), so
+                        // every slot's first push is unchanged; only device and link queues
+                        // see the new order.
+                        const int32_t nk = (int32_t)(h.w >> kStStepsShift);
+                        const bool straddle = sp + (uint32_t)nk * kStepBytes >= spe;
+                        uint32_t sp1;
+                        if (straddle) {
+                            const int s2 = (it + 1) % kStages32;
+                            mbar_wait(&full[s2], ((it + 1) / kStages32) & 1);
+                            sp1 = cx.smem + (uint32_t)s2 * sb + kTileHeader;
+                        } else {
+                            sp1 = sp + (uint32_t)nk * kStepBytes;
+                        }
+                        const uint4 h1 = lds_v4(sp1);
+                        const int32_t n1 = (int32_t)(h1.w >> kStStepsShift);
                         issue_far(h, v);
-                        cp_async_wait<kPrefetchDist - 1>();      // v+1 has landed
-                        T r[CPL];
-                        arrivals(h.w, nfar, nnear, fwd, r);
-                        load_next(v + 1, nfar, nnear);
+                        issue_far(h1, v + 1);
+                        cp_async_wait<kPrefetchDist - 1>();  // v+1 and v+2 have landed
+                        T r0[CPL], r1[CPL], f1[CPL], g1[CPL], zero[CPL];
+#pragma unroll
+                        for (int c = 0; c < CPL; c++) zero[c] = 0u;
+                        arrivals(h.w, nfar, nnear, fwd, r0);
+                        load_next(v + 1, f1, g1);
+                        arrivals(h1.w, f1, g1, zero, r1);   // ks+1's distance-1 producer is ks: none
 #pragma unroll
                         for (int c = 0; c < CPL; c++) fwd[c] = 0u;
-                        if constexpr (MODE == 0) {
-                            if (v >= xwb + SW) {               // next window; prefetch the one after
-#pragma unroll
-                                for (int c = 0; c < CPL; c++) xw[c] = xn[c];
-                                xwb += SW;
-                                x_load(xwb + SW, xn);
-                            }
-#pragma unroll
-                            for (int c = 0; c < CPL; c++) {
-                                PlaneWords<PL> w;
-#pragma unroll
-                                for (int p = 0; p < PL; p++)
-                                    w.w[p] = __shfl_sync(0xffffffffu, xw[c], (v - xwb) * PL + p);
-                                x[c] = plane_dev<PL>(w, lane, place.dmax);
-                            }
-                        } else {
-                            // outside the group's region every lane has the base device
-                            // (CPL = 2 only: with one candidate per lane the launch is
-                            // latency-bound and the branch-free selects schedule better)
-                            xu = (kSearch && CPL == 2 &&
-                                  (uint32_t)(v - place.rc) >= (uint32_t)place.rlen)
-                                     ? (int)(h.w & kStXMask) : -1;
-                            place.at(v, (int)(h.w & kStXMask), x, cpos_at);
+                        place.at(v + 1, (int)(h1.w & kStXMask), x, cpos_at);
+                        begin32<CPL, T>(h1, st, r1, x, cc);
+                        for (int32_t q = 0; q < n1; q++) {
+                            const uint32_t a = sp1 + q * kStepBytes;
+                            edges32<PL, CPL, T>(cx, lds_u32(a + 12), lds_v4(a + 16), lds_v4(a + 32), x,
+                                             cc, place_y, st, fwd);
                         }
-                        if (MODE != 0 && xu >= 0) st.begin_u(xu, h.x, r, cc);
-                        else begin32<CPL, T>(h, st, r, x, cc);
-                    }
-                    if constexpr (MODE == 0) {
-                        edges32<PL, CPL, T>(cx, h.w, e0, e1, x, cc, pw_y, st, fwd);
-                        slot0 += 2;
-                    } else {
-                        const uint32_t ne = (h.w >> kStEdgeShift) & 3u;
-                        if (xu >= 0) {
-                            if (ne >= 1) {
-                                const int32_t q0 = (int32_t)(e0.y & kSuccPosMask);
-                                if ((uint32_t)(q0 - place.rc) >= (uint32_t)place.rlen)
-                                    push32_u<PL, CPL, T>(cx, e0, xu, (int)((e0.y >> kSuccXShift) & 7u), cc, st, fwd);
-                                else { int y[CPL]; place_y(0, e0, y); push32<PL, CPL, T>(cx, e0, x, y, cc, st, fwd); }
-                            }
-                            if (ne >= 2) {
-                                const int32_t q1 = (int32_t)(e1.y & kSuccPosMask);
-                                if ((uint32_t)(q1 - place.rc) >= (uint32_t)place.rlen)
-                                    push32_u<PL, CPL, T>(cx, e1, xu, (int)((e1.y >> kSuccXShift) & 7u), cc, st, fwd);
-                                else { int y[CPL]; place_y(1, e1, y); push32<PL, CPL, T>(cx, e1, x, y, cc, st, fwd); }
-                            }
-                        } else {
-                            edges32<PL, CPL, T>(cx, h.w, e0, e1, x, cc, place_y, st, fwd);
+                        place.at(v, (int)(h.w & kStXMask), x, cpos_at);
+                        begin32<CPL, T>(h, st, r0, x, cc);
+                        edges32<PL, CPL, T>(cx, h.w, e0, e1, x, cc, place_y, st, fwd);
+                        for (int32_t q = 1; q < nk; q++) {
+                            const uint32_t a = sp + q * kStepBytes;
+                            edges32<PL, CPL, T>(cx, lds_u32(a + 12), lds_v4(a + 16), lds_v4(a + 32), x,
+                                             cc, place_y, st, fwd);
                         }
+                        v++;
+                        xu = -1;
+                        load_next(v + 1, nfar, nnear);
+                        if (straddle) {
+                            skip = n1;
+                            break;
+                        }
+                        sp = sp1 + (uint32_t)n1 * kStepBytes;
+                        h = lds_v4(sp);
+                        e0 = lds_v4(sp + 16);
+                        e1 = lds_v4(sp + 32);
+                        continue;
                     }
-                    sp += kStepBytes;
-                    if constexpr (CPL != 1) h = hn;
                 }
             }
             __syncwarp();

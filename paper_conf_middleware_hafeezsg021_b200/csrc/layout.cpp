@@ -291,7 +291,8 @@ pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<
             td.byte_off = (int64_t)t_start;
             td.bytes = (int32_t)(blob.size() - t_start);
             td.pos_begin = t_steps;                  // (steps in the tile)
-            const int32_t hdr[4] = {t_steps, 0, td.bytes, 0};
+            // {steps, blob offset of the tile (the walk locates a swapped pair with it), bytes, 0}
+            const int32_t hdr[4] = {t_steps, (int32_t)(uint32_t)t_start, td.bytes, 0};
             std::memcpy(blob.data() + t_start, hdr, 16);
             L->tiles32.push_back(td);
             L->stage_bytes32 = std::max(L->stage_bytes32, td.bytes);
