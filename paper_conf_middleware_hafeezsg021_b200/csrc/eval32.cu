@@ -188,6 +188,8 @@ __device__ __forceinline__ int coarse_apply_kept(const LaneMove &mv, int cq, int
 __device__ __forceinline__ int coarse_apply_kept(const PackedMove &mv, int cq, int xb, unsigned aq) {
     return apply_coarse((int32_t)(mv.w1 & 255u), (int32_t)(mv.w1 >> 8), cq, xb, aq);
 }
+__device__ __forceinline__ int coarse_k(const LaneMove &mv) { return mv.ws; }
+__device__ __forceinline__ int coarse_k(const PackedMove &mv) { return (int)(mv.w1 & 255u); }
 __device__ __forceinline__ void keep_coarse(LaneMove &dst, const LaneMove &mv) { dst = mv; }
 __device__ __forceinline__ void keep_coarse(PackedMove &dst, const LaneMove &mv) { dst = pack_coarse(mv); }
 
@@ -236,33 +238,42 @@ struct Place32 {
     // MODE 5 (search with S9 coarse groups), coarse group: the region is the whole order, marked by a negative rlen (the
     // unsigned range test still admits every position), so no flag register stays live
     __device__ __forceinline__ bool coarse() const { return rlen < 0; }
-    // cfn(q): merged vertex of the op at position q (MODE 5 coarse groups only)
+    // cfn(q): merged vertex of the op at position q (MODE 5 coarse groups only).  Returns true
+    // when every lane keeps the base code xb (search: outside the region; a coarse group: no
+    // lane moves the op's merged vertex -- a warp vote), false otherwise or when unknown.
     template <class CFn>
-    __device__ __forceinline__ void at(int32_t q, int xb, int (&x)[CPL], const CFn &cfn) const {
+    __device__ __forceinline__ bool at(int32_t q, int xb, int (&x)[CPL], const CFn &cfn) const {
         if (MODE == 0) {
 #pragma unroll
             for (int c = 0; c < CPL; c++) x[c] = planes_dev_at<PL>(pl + c * pl_stride, q, lane, dmax);
-            return;
+            return false;
         }
         if (MODE == 4) {                                       // digit of the merged vertex
             const int sh = cbits * (int)__ldg(cpos + q);
 #pragma unroll
             for (int c = 0; c < CPL; c++) x[c] = (int)((jc[c] >> sh) & (uint32_t)dmax);
-            return;
+            return false;
         }
 #pragma unroll
         for (int c = 0; c < CPL; c++) x[c] = xb;
         if ((uint32_t)(q - rc) < (uint32_t)rlen) {             // warp-uniform branch
-            const unsigned aq = all_allowed ? 0xFFu : (unsigned)__ldg(allowed_pos + q);
             if (MODE == 5 && coarse()) {                       // S9: one merged vertex per lane
                 const int cq = cfn(q);
+                bool hit = false;
+#pragma unroll
+                for (int c = 0; c < CPL; c++) hit = hit || coarse_k(mv[c]) == cq;
+                if (!__any_sync(0xffffffffu, hit)) return true;   // no lane moves this vertex
+                const unsigned aq = all_allowed ? 0xFFu : (unsigned)__ldg(allowed_pos + q);
 #pragma unroll
                 for (int c = 0; c < CPL; c++) x[c] = coarse_apply_kept(mv[c], cq, xb, aq);
-                return;
+                return false;
             }
+            const unsigned aq = all_allowed ? 0xFFu : (unsigned)__ldg(allowed_pos + q);
 #pragma unroll
             for (int c = 0; c < CPL; c++) x[c] = apply_kept(mv[c], q, rc, xb, aq);
+            return false;
         }
+        return true;
     }
 };
 
@@ -745,10 +756,16 @@ eval32_kernel(const EvalParams P) {
                                 // outside the group's region every lane has the base device
                                 // (CPL = 2 only: with one candidate per lane the launch is
                                 // latency-bound and the branch-free selects schedule better)
-                                xu = (kSearch && CPL == 2 &&
-                                      (uint32_t)(v - place.rc) >= (uint32_t)place.rlen)
-                                         ? (int)(h.w & kStXMask) : -1;
-                                place.at(v, (int)(h.w & kStXMask), x, cpos_at);
+                                if constexpr (MODE == 5) {
+                                    // coarse groups: uniform wherever no lane moves the op's merged vertex
+                                    const bool uni = place.at(v, (int)(h.w & kStXMask), x, cpos_at);
+                                    xu = (CPL == 2 && uni) ? (int)(h.w & kStXMask) : -1;
+                                } else {
+                                    xu = (kSearch && CPL == 2 &&
+                                          (uint32_t)(v - place.rc) >= (uint32_t)place.rlen)
+                                             ? (int)(h.w & kStXMask) : -1;
+                                    place.at(v, (int)(h.w & kStXMask), x, cpos_at);
+                                }
                             }
                             if (MODE != 0 && xu >= 0) st.begin_u(xu, h.x, r, cc);
                             else begin32<CPL, T>(h, st, r, x, cc);
@@ -758,7 +775,23 @@ eval32_kernel(const EvalParams P) {
                             slot0 += 2;
                         } else {
                             const uint32_t ne = (h.w >> kStEdgeShift) & 3u;
-                            if (xu >= 0) {
+                            if (MODE == 5 && xu >= 0) {
+                                // successors: the uniform push wherever no lane moves them
+                                if (ne >= 1) {
+                                    int y[CPL];
+                                    const int yb = (int)((e0.y >> kSuccXShift) & 7u);
+                                    if (place.at((int32_t)(e0.y & kSuccPosMask), yb, y, cpos_at))
+                                        push32_u<PL, CPL, T>(cx, e0, xu, yb, cc, st, fwd);
+                                    else push32<PL, CPL, T>(cx, e0, x, y, cc, st, fwd);
+                                }
+                                if (ne >= 2) {
+                                    int y[CPL];
+                                    const int yb = (int)((e1.y >> kSuccXShift) & 7u);
+                                    if (place.at((int32_t)(e1.y & kSuccPosMask), yb, y, cpos_at))
+                                        push32_u<PL, CPL, T>(cx, e1, xu, yb, cc, st, fwd);
+                                    else push32<PL, CPL, T>(cx, e1, x, y, cc, st, fwd);
+                                }
+                            } else if (xu >= 0) {
                                 if (ne >= 1) {
                                     const int32_t q0 = (int32_t)(e0.y & kSuccPosMask);
                                     if ((uint32_t)(q0 - place.rc) >= (uint32_t)place.rlen)
