@@ -438,6 +438,12 @@ eval32_kernel(const EvalParams P) {
     T *stage_all = reinterpret_cast<T *>(cur);                        // far-arrival staging
     cur = align16(cur + (size_t)NW * kRing * CW * sizeof(T));
     T *dstate = reinterpret_cast<T *>(cur);
+    // MODE 5, CPL 1: the merged vertex of every position of the current task's base in shared
+    // memory (S9 coarse groups look one up per op and per successor; from global memory those
+    // lookups missed L1 behind the cold-slot traffic and made a coarse warp ~1.7x slower).  Not
+    // for CPL 2: n more bytes per CTA cost a resident CTA per SM there (measured slower).
+    constexpr bool kCposSmem = MODE == 5 && CPL == 1;
+    const uint32_t cpos_s = su32_reg(align16(cur + (PL != 1 ? (size_t)NW * (P.D + P.D * P.D) * CW * sizeof(T) : 0)));
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     if (threadIdx.x == 0) {
@@ -529,9 +535,19 @@ eval32_kernel(const EvalParams P) {
     };
 
     uint32_t it = 0;
+    int prev_bl = -1;
     for (int64_t task = blockIdx.x; task < P.n_tasks; task += gridDim.x) {
         const int bl = kSearch ? (int)(task / P.tasks_per_base) : 0;
         if (!runs_here(bl)) continue;
+        if constexpr (kCposSmem) {
+            if (bl != prev_bl) {         // the consumer warps copy the base's merged vertices
+                named_bar_sync(1, NW * 32);                   // previous walks are done
+                const uint8_t *src = P.coarse_pos + (size_t)bl * P.n;
+                for (int q = threadIdx.x; q < P.n; q += NW * 32) sts_u8(cpos_s + q, __ldg(src + q));
+                named_bar_sync(1, NW * 32);
+                prev_bl = bl;
+            }
+        }
         const int64_t local = kSearch ? task % P.tasks_per_base : task;
         const BaseLayoutDev *B = &P.bases[bl];
         const int nt = B->n_tiles32;
@@ -640,8 +656,12 @@ eval32_kernel(const EvalParams P) {
 #pragma unroll
         for (int c = 0; c < CPL; c++) { x[c] = 0; cc[c] = 0u; fwd[c] = 0u; nfar[c] = 0u; nnear[c] = 0u; }
         // devices by direct lookup (search: base code + region moves; rows: plane words)
-        // S9 merged vertices by position of this base (P.coarse_pos = [local base][n])
-        auto cpos_at = [&](int32_t q) { return (int)__ldg(P.coarse_pos + (size_t)bl * P.n + q); };
+        // S9 merged vertices by position of this base (shared copy of P.coarse_pos[bl][.])
+        // (a non-volatile shared load: the compiler may issue it early)
+        auto cpos_at = [&](int32_t q) {
+            if constexpr (kCposSmem) return (int)lds_u8_nv(cpos_s + (uint32_t)q);
+            else return (int)__ldg(P.coarse_pos + (size_t)bl * P.n + q);
+        };
         auto place_y = [&](int, const uint4 rec, int (&y)[CPL]) {
             place.at((int32_t)(rec.y & kSuccPosMask), (int)((rec.y >> kSuccXShift) & 7u), y, cpos_at);
         };
@@ -964,6 +984,8 @@ int eval32_smem_bytes(const EvalParams &p, int search_mode) {
     b += (size_t)nw * kRing * 32 * cpl * tb;       // far-arrival staging
     b = (b + 15) & ~size_t(15);
     if (pl != 1) b += (size_t)nw * (p.D + p.D * p.D) * 32 * cpl * tb;
+    b = (b + 15) & ~size_t(15);
+    if (search_mode == 5 && cpl == 1) b += (size_t)p.n;   // merged vertex per position (S9)
     return (int)b + 128;
 }
 
