@@ -186,3 +186,17 @@ def test_dispatch_and_link_model_validation(P):
         G.set_dispatch(2)
     with pytest.raises(P.PestoError):
         G.set_link_model(5)
+
+
+def test_workspace_and_async_validation(P):
+    """pesto.h: a workspace needs a device graph (ESTATE on a host-only handle); NULL -> EINVAL;
+    the async call validates like pesto_eval_batch_host before touching a GPU."""
+    import ctypes as C
+    g = dag.random_dag(3, 20, 1.5, D=2)
+    G = _host_graph(P, g)
+    h = C.c_void_p()
+    assert P.lib().pesto_workspace_create(G.handle, C.byref(h)) == P.ESTATE
+    assert not h.value
+    assert P.lib().pesto_workspace_create(None, C.byref(h)) == P.EINVAL
+    assert P.lib().pesto_eval_batch_host_async(None, None, None, 16, 1, None, None) == P.EINVAL
+    P.lib().pesto_workspace_destroy(None)                      # NULL-safe
