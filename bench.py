@@ -163,13 +163,16 @@ def oracle_rate(g, xs, orders, k_per_base, seconds, threads, nondelay=False, coa
     sample = int(max(probe, min(k_per_base, seconds / max(per, 1e-9))))
     t0 = time.perf_counter()
     done = 0
+    sample_keys = []
     for b in range(P_):
         cnt = sample // P_
         if cnt <= 0:
+            sample_keys.append(np.zeros(0, np.uint64))
             continue
-        keys(b, cnt)
+        sample_keys.append(keys(b, cnt))
         done += cnt
     dt = time.perf_counter() - t0
+    oracle_rate.sample_keys = sample_keys           # the timed sample's keys, for parity
     return done / dt, done, dt
 
 
@@ -219,6 +222,8 @@ def run_pesto(args, rank, world, local):
     if world > 1:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     cfg = configs.CONFIGS[args.config]
+    # SURVEY 8(d) roof microbenchmarks on this GPU (integer issue, L2, HBM), before anything else
+    roofs = P.measure_roofs(local, 5)
     g = configs.graph_for(cfg)
     G = P.Graph.from_arrays(g, device=local)
     nd = args.dispatch == "nondelay"
@@ -400,13 +405,16 @@ def run_pesto(args, rank, world, local):
                          "note": "algorithmic int ops (2n+m+2*cross per candidate) / K1 time; "
                                  "traffic = ncu DRAM bytes per K1 launch (profiles/)"},
             "issue_roof": issue_roof,
+            "roofs": dict(roofs, source="pesto_measure_roofs (csrc/roofs.cu): K1's max/add/"
+                          "saturate chains on all SMs, L2-resident sweeps, 1 GiB copy; best of 5",
+                          k1_frac_of_measured_int_roof=achieved * 1e12 / roofs["int_ops_per_s"]),
             "gpu_launches": int(launches),
             "wall_s_timed_region": wall,
             "search": {"seed_makespans": seed_mk, "best_makespans": best_mk,
                        "swaps_patched_in_place": swap_stats[0], "swaps_rebuilt": swap_stats[1]},
             "e2e": e2e}
     line["clocks"] = clk.summary()
-    if not args.no_cpu_baseline:
+    if not args.no_cpu_baseline and world == 1:
         threads = len(os.sched_getaffinity(0))
         rate, done, dt = oracle_rate(g, xs, orders, k_per_base, args.cpu_seconds, threads,
                                      nondelay=nd, coarse=coarse)
@@ -414,6 +422,18 @@ def run_pesto(args, rank, world, local):
                                 "kind": "oracle",
                                 "sample": f"{done} step-0 neighbour candidates of the same "
                                           f"{n_bases} bases ({dt:.1f}s)"}
+        # the same sample on the GPU (a fresh search at step 0, every candidate's key from the
+        # independent 64-bit kernel), compared key by key with the oracle's
+        S0 = P.Search(G, xs, orders, k_per_base, configs.MOVE_MIX, configs.SEARCH_SEED)
+        if coarse is not None:
+            S0.set_coarse_moves(*coarse)
+        mism = 0
+        for b, ok in enumerate(oracle_rate.sample_keys):
+            if len(ok):
+                mism += int((S0.candidate_keys(b, 0, len(ok)) != ok).sum())
+        line["parity"] = {"checked": int(done), "mismatches": mism,
+                          "what": "keys (makespan << 24 | j) of the cpu_baseline sample, GPU "
+                                  "(pesto_search_candidate_keys) vs oracle, bit-exact"}
     print(json.dumps(line), flush=True)
     if world > 1:
         dist.destroy_process_group()

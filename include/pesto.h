@@ -286,6 +286,21 @@ pesto_status pesto_search_swap_stats(const pesto_search *s, int64_t *in_place, i
 pesto_status pesto_nccl_unique_id(uint8_t *out128);
 void pesto_search_destroy(pesto_search *s);                        /* NULL-safe */
 
+/* Roof microbenchmarks on `device`, best of `reps` CUDA-event-timed runs each:
+ * the ceilings K1 is reported against, measured on the box that runs the bench.  Synchronises;
+ * ~1 s.  Errors: EINVAL (NULL out, reps < 1), ESTATE (no such device), ECUDA. */
+typedef struct {
+    double int_ops_per_s;          /* K1's per-op arithmetic c = min(max(r, d) + p, sat) on 8
+                                      independent uint32 chains per thread, all SMs full:
+                                      algorithmic ops (max, add, saturate) per second          */
+    double int_chain_steps_per_s;  /* the same in chain steps (3 ops each) per second           */
+    double l2_read_gbs;            /* L2-resident buffer (a quarter of the L2), 128-bit reads   */
+    double l2_rmw_gbs;             /* same buffer, 4-byte lanes read + written (K1's cold slots)*/
+    int64_t l2_buffer_bytes;
+    double hbm_copy_gbs;           /* 1 GiB copy kernel, read + write bytes                     */
+} pesto_roofs;
+pesto_status pesto_measure_roofs(int32_t device, int32_t reps, pesto_roofs *out);
+
 /* ------------------------------------------------------------------------------------------ */
 const char *pesto_last_error(void);       /* thread-local detail of the last failure */
 const char *pesto_status_str(pesto_status s);

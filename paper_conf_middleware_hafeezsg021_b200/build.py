@@ -15,7 +15,7 @@ CUDA = os.environ.get("CUDA_HOME", "/usr/local/cuda")
 NVCC = os.path.join(CUDA, "bin", "nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 
-CU_SOURCES = ["kernels.cu", "eval32.cu", "nondelay.cu"]
+CU_SOURCES = ["kernels.cu", "eval32.cu", "nondelay.cu", "roofs.cu"]
 CPP_SOURCES = ["graph.cpp", "layout.cpp", "search.cpp", "coarsen.cpp"]
 HEADERS = ["internal.h", "host.h", "layout_format.h", "moves.cuh", "device_common.cuh",
            "feasibility.cuh"]

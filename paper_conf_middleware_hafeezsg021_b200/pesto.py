@@ -49,6 +49,12 @@ class GraphStats(C.Structure):
                 ("link_classes", C.c_int32), ("time32_exact", C.c_int32)]
 
 
+class Roofs(C.Structure):
+    _fields_ = [("int_ops_per_s", C.c_double), ("int_chain_steps_per_s", C.c_double),
+                ("l2_read_gbs", C.c_double), ("l2_rmw_gbs", C.c_double),
+                ("l2_buffer_bytes", C.c_int64), ("hbm_copy_gbs", C.c_double)]
+
+
 class SearchDesc(C.Structure):
     _fields_ = [("n_bases", C.c_int32), ("base_x", C.c_void_p), ("base_order", C.c_void_p),
                 ("k_per_base", C.c_int64), ("mix", C.c_int32 * 4), ("seed", C.c_uint64),
@@ -92,6 +98,7 @@ SIGNATURES = {
     "pesto_status_str": (C.c_char_p, [_I32]),
     "pesto_version": (_I32, []),
     "pesto_launch_count": (_I64, []),
+    "pesto_measure_roofs": (_I32, [_I32, _I32, _VP]),
 }
 
 if not os.path.exists(LIB_PATH):
@@ -379,3 +386,10 @@ class Search:
         a, b = C.c_int64(), C.c_int64()
         _check(_L.pesto_search_swap_stats(self._h, C.byref(a), C.byref(b)))
         return int(a.value), int(b.value)
+
+
+def measure_roofs(device: int = 0, reps: int = 5) -> dict:
+    """SURVEY 8(d) roof microbenchmarks on `device` (pesto_measure_roofs)."""
+    r = Roofs()
+    _check(_L.pesto_measure_roofs(device, reps, C.byref(r)))
+    return {k: getattr(r, k) for k, _ in Roofs._fields_}
