@@ -681,24 +681,33 @@ eval32_kernel(const EvalParams P) {
         constexpr int SW = 32 / PL;                    // edge slots per 32-word window
         const int64_t ywords = P.n_slots * PL;         // words of one group's slot stream
         uint32_t yw[CPL], yn[CPL];                     // this window / the next, per candidate
-        int64_t ywb = 0;                               // first slot of this window
-        int64_t slot0 = 0;                             // first slot of the current step
-        auto y_load = [&](int64_t slot, uint32_t (&w)[CPL]) {
-            const int64_t wi = slot * PL + lane;
+        int32_t ywb = 0;                               // first slot of this window
+        int32_t slot0 = 0;                             // first slot of the current step
+        auto y_load = [&](int32_t slot, uint32_t (&w)[CPL]) {
+            const int64_t wi = (int64_t)slot * PL + lane;
 #pragma unroll
             for (int c = 0; c < CPL; c++)
                 w[c] = wi < ywords ? __ldg(P.yplanes + (size_t)(gw + c) * ywords + wi) : 0u;
         };
-        auto pw_y = [&](int k, const uint4, int (&y)[CPL]) {
-            const int base = (int)((slot0 + k - ywb) * PL);
+        // the codes of a position's / an edge slot's word, by shuffle from a window
+        auto shfl_dev = [&](const uint32_t (&win)[CPL], int base, int (&out)[CPL]) {
 #pragma unroll
             for (int c = 0; c < CPL; c++) {
                 PlaneWords<PL> w;
 #pragma unroll
-                for (int p = 0; p < PL; p++) w.w[p] = __shfl_sync(0xffffffffu, yw[c], base + p);
-                y[c] = plane_dev<PL>(w, lane, place.dmax);
+                for (int p = 0; p < PL; p++) w.w[p] = __shfl_sync(0xffffffffu, win[c], base + p);
+                out[c] = plane_dev<PL>(w, lane, place.dmax);
             }
         };
+        // both successor slots of a step are shuffled at the step's top (off the edges' chains;
+        // slot0 is even and a window holds an even number of slots, so both are in window yw)
+        int ys[2][CPL];
+        auto pw_y = [&](int k, const uint4, int (&y)[CPL]) {
+#pragma unroll
+            for (int c = 0; c < CPL; c++) y[c] = ys[k][c];
+        };
+        // the next op's codes, shuffled one op ahead
+        int xnext[CPL];
         if constexpr (MODE == 0) {
             if (active) {
                 x_load(0, xw);
@@ -706,6 +715,7 @@ eval32_kernel(const EvalParams P) {
                 y_load(0, yw);
                 y_load(SW, yn);
             }
+            shfl_dev(xw, 0, xnext);
         }
         int32_t v = -1;
         int xu = -1;                 // search: the walked op's device if warp-uniform, else -1
@@ -747,6 +757,8 @@ eval32_kernel(const EvalParams P) {
                                 ywb += SW;
                                 y_load(ywb + SW, yn);
                             }
+                            shfl_dev(yw, (slot0 - ywb) * PL, ys[0]);
+                            shfl_dev(yw, (slot0 + 1 - ywb) * PL, ys[1]);
                         }
                         if (!(h.w & kStCont)) {
                             v++;
@@ -758,20 +770,15 @@ eval32_kernel(const EvalParams P) {
 #pragma unroll
                             for (int c = 0; c < CPL; c++) fwd[c] = 0u;
                             if constexpr (MODE == 0) {
-                                if (v >= xwb + SW) {               // next window; prefetch the one after
+#pragma unroll
+                                for (int c = 0; c < CPL; c++) x[c] = xnext[c];
+                                if (v + 1 >= xwb + SW) {           // next window; prefetch the one after
 #pragma unroll
                                     for (int c = 0; c < CPL; c++) xw[c] = xn[c];
                                     xwb += SW;
                                     x_load(xwb + SW, xn);
                                 }
-#pragma unroll
-                                for (int c = 0; c < CPL; c++) {
-                                    PlaneWords<PL> w;
-#pragma unroll
-                                    for (int p = 0; p < PL; p++)
-                                        w.w[p] = __shfl_sync(0xffffffffu, xw[c], (v - xwb) * PL + p);
-                                    x[c] = plane_dev<PL>(w, lane, place.dmax);
-                                }
+                                shfl_dev(xw, (v + 1 - xwb) * PL, xnext);
                             } else {
                                 // outside the group's region every lane has the base device
                                 // (CPL = 2 only: with one candidate per lane the launch is

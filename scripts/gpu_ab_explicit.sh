@@ -1,0 +1,14 @@
+# A/B of the explicit-row path (K5 + eval32 mode 0): default lib vs libpesto_$B.so
+cd $GRAFT_REPO_ROOT
+mkdir -p gpurun_out
+B=${B:-b3}
+: > gpurun_out/abx.log
+timeout 900 python -m pytest tests/test_gpu_parity.py -q -x > gpurun_out/pytest_abx.log 2>&1; echo "rc=$?" >> gpurun_out/pytest_abx.log
+for rep in 1 2; do
+ for v in new $B; do
+  if [ $v = new ]; then L=""; else L=paper_conf_middleware_hafeezsg021_b200/libpesto_$v.so; fi
+  r=$(PESTO_LIB=$L timeout 300 python scripts/time_explicit.py inception_v3_2dev 2>&1 | head -1)
+  e=$(PESTO_LIB=$L timeout 300 python bench.py --steps 5 --warmup 3 --no-cpu-baseline 2>&1 | grep '^{' | tail -1 | python -c "import json,sys; d=json.loads(sys.stdin.read()); print('e2e', round(d['e2e']['value']/1e6,3), 'search', round(d['value']/1e6,3))" 2>&1)
+  echo "$v $r | $e" >> gpurun_out/abx.log
+ done
+done
