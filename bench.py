@@ -391,6 +391,13 @@ def run_pesto(args, rank, world, local):
                        "candidates_per_step": k_gpu * world, "candidates_per_gpu": k_gpu,
                        "bases": n_bases, "k_per_base": k_per_base, "move_mix": configs.MOVE_MIX,
                        "live_slots": st["live_slots"], "l2": "flushed between timed steps",
+                       "f_x_seeds": [round(float((xs[b][g.src] != xs[b][g.dst]).mean()), 4)
+                                     for b in range(n_bases)],
+                       "time_t": "uint32 saturating at 4.03 s (eval32), exact 64-bit for bases "
+                                 "above it (wide eval32 / eval64)",
+                       "state_tier": "near ring + far staging in shared memory, cold slots in "
+                                     "global memory (L2/HBM), device/link state in registers "
+                                     "(D = 2) or shared memory (D > 2)",
                        "parallelism": f"candidate-dp{world}", "dispatch": args.dispatch,
                        "coarse_groups_pct": args.coarse_pct,
                        "n_coarse": int(coarse[1]) if coarse else None},
