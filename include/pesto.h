@@ -212,6 +212,9 @@ pesto_status pesto_eval_batch_host(pesto_graph *g, const int32_t *order,
  * makespans_host, before reusing placements_host, and before the next call on the same
  * workspace from another stream.  placements_host should be pinned (else the copy is
  * synchronous).  The graph and its layouts are shared (not thread-safe: one host thread).
+ * A workspace must be destroyed before its graph.  (pesto_eval_batch, pesto_eval_batch_host and
+ * the search steps share the graph's own scratch: calls of those on different streams must be
+ * ordered by the caller.)
  * Errors as pesto_eval_batch_host; create: EINVAL, ESTATE (host-only graph), ENOMEM. */
 typedef struct pesto_workspace pesto_workspace;
 pesto_status pesto_workspace_create(pesto_graph *g, pesto_workspace **out);
