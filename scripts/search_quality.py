@@ -50,7 +50,7 @@ def main():
             t0 = time.perf_counter()
             for s in range(1, a.steps + 1):
                 S.step()
-                if s in (10, 30, 100, 300, 1000, a.steps):
+                if s in (10, 30, 100, 300, 1000, 2000, a.steps):
                     traj[s] = [S.get(b)[0] for b in range(cfg.bases)]
             torch.cuda.synchronize()
             dt = time.perf_counter() - t0
