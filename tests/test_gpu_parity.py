@@ -526,3 +526,13 @@ def test_exhaustive_coarse_search_inception(P, O):
     xs = np.stack([OC.expand(co, 2, int(c)) for c in sample])
     ref, _ = O.makespan_batch(g, xs, order)
     assert (ref >= mk).all()
+
+
+def test_roofs_microbenchmarks(P):
+    """pesto_measure_roofs: positive, physically plausible ceilings on a B200"""
+    r = P.measure_roofs(0, 2)
+    assert 1e12 < r["int_ops_per_s"] < 1e14
+    assert abs(r["int_ops_per_s"] - 3 * r["int_chain_steps_per_s"]) < 1e-6 * r["int_ops_per_s"]
+    assert 1e3 < r["l2_read_gbs"] < 1e5 and 1e3 < r["l2_rmw_gbs"] < 1e5
+    assert 1e3 < r["hbm_copy_gbs"] < 1e4
+    assert r["l2_buffer_bytes"] > 0
