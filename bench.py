@@ -293,29 +293,33 @@ def run_pesto(args, rank, world, local):
 
     # ---- end to end through the public API with host buffers ----
     # every step copies its batch of explicit placement rows in from pinned host memory,
-    # evaluates it and copies the makespans out; two workspaces on two streams double-buffer
-    # the steps (pesto_eval_batch_host_async), so step i+1's copy-in overlaps step i's kernels
+    # evaluates it and copies the makespans out; four workspaces on four streams keep four steps
+    # in flight (pesto_eval_batch_host_async), so copies overlap kernels and the kernels of
+    # consecutive batches overlap each other
     e2e = None
     if not args.no_e2e:
         rows_h = []
         for r in range(2):                           # two distinct input batches, alternating
             rows = P.pack_rows(dag.random_placements(g, 11 + 2 * rank + r, k_gpu), g.D)
             rows_h.append(torch.from_numpy(rows).pin_memory().numpy())
-        outs = [torch.empty(k_gpu, dtype=torch.int64).pin_memory().numpy() for _ in range(2)]
-        wss = [G.workspace(), G.workspace()]
-        sts = [torch.cuda.Stream(), torch.cuda.Stream()]
+        nbuf = int(os.environ.get("PESTO_E2E_BUFFERS", "4"))     # batches in flight
+        outs = [torch.empty(k_gpu, dtype=torch.int64).pin_memory().numpy() for _ in range(nbuf)]
+        wss = [G.workspace() for _ in range(nbuf)]
+        sts = [torch.cuda.Stream() for _ in range(nbuf)]
         o = orders[0]
 
         def e2e_run(n):
             for i in range(n):
-                k = i & 1
-                if i >= 2:
-                    sts[k].synchronize()             # batch i-2 is done and its makespans read
-                wss[k].eval_host_async(o, rows_h[k], outs[k], stream=sts[k])
+                k = i % nbuf
+                if i >= nbuf:
+                    sts[k].synchronize()             # batch i-nbuf is done and its makespans read
+                wss[k].eval_host_async(o, rows_h[i & 1], outs[k], stream=sts[k])
             for st_ in sts:
                 st_.synchronize()
-        e2e_run(max(2, args.warmup))
-        ref0 = G.eval_host(o, rows_h[0])             # the synchronous API agrees
+        nw = max(nbuf, args.warmup)
+        e2e_run(nw)
+        last0 = max(i for i in range(nw) if i % nbuf == 0)   # the batch buffer 0 holds
+        ref0 = G.eval_host(o, rows_h[last0 & 1])     # the synchronous API agrees
         assert (ref0 == outs[0]).all(), "async host-buffer evaluation disagrees"
         if world > 1:
             dist.barrier()
@@ -329,8 +333,8 @@ def run_pesto(args, rank, world, local):
         e2e = {"value": k_gpu * world * e2e_steps / float(e2e_s[0]), "unit": "candidates/s",
                "h2d_bytes_per_step": int(rows_h[0].nbytes), "d2h_bytes_per_step": int(8 * k_gpu),
                "api": "pesto_eval_batch_host_async (explicit placement rows from pinned host "
-                      "memory, makespans back to pinned host memory; 2 workspaces on 2 streams, "
-                      "double-buffered)"}
+                      f"memory, makespans back to pinned host memory; {nbuf} workspaces on "
+                      f"{nbuf} streams, {nbuf} batches in flight)"}
 
     if rank != 0:
         if world > 1:
