@@ -298,7 +298,7 @@ void plan_eval32(const pesto_graph *g, EvalParams &p, int64_t j0, int64_t j1, in
 }
 
 pesto_status ensure_state32(pesto_graph *g, Scratch &ws, const EvalParams &p, int search_mode,
-                            int64_t n_tasks, int *grid_out) {
+                            int64_t n_tasks, int *grid_out, bool wide_buf) {
     int per_sm = eval32_max_ctas_per_sm(p, search_mode);
     if (per_sm <= 0)
         return fail(PESTO_ECUDA, "eval32 kernel does not fit on an SM (smem " +
@@ -307,7 +307,7 @@ pesto_status ensure_state32(pesto_graph *g, Scratch &ws, const EvalParams &p, in
     grid = std::max<int64_t>(grid, 1);
     size_t bytes = (size_t)grid * eval32_task_size(p.cpl32) * (size_t)std::max(p.max_W32, 1) *
                    (p.wide32 ? sizeof(uint64_t) : sizeof(uint32_t));
-    cudaError_t e = ws.state32.ensure(bytes);
+    cudaError_t e = (wide_buf ? ws.state32w : ws.state32).ensure(bytes);
     if (e != cudaSuccess) return cuda_fail(e, "allocate cold slot state");
     *grid_out = (int)grid;
     return PESTO_OK;

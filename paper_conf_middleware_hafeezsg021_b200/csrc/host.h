@@ -80,6 +80,7 @@ struct Layout {
 struct Scratch {
     DevBuf state;                 // eval64 ready-time slots
     DevBuf state32;               // eval32 cold slots
+    DevBuf state32w;              // the search's wide eval32 launch (runs beside the 32-bit one)
     DevBuf planes, invalid;       // K5: bit-sliced rows, per-group infeasible-lane masks
     DevBuf yplanes;               // K5: codes per eval32 edge slot (explicit rows)
     DevBuf flags;                 // [count | list of saturated candidates]
@@ -167,7 +168,7 @@ int choose_cpl32(const pesto_graph *g, int64_t n_tasks);
 // in 256-candidate units), p.tasks_per_base and p.n_tasks in tasks of eval32_task_size(cpl)
 void plan_eval32(const pesto_graph *g, EvalParams &p, int64_t j0, int64_t j1, int n_bases);
 pesto_status ensure_state32(pesto_graph *g, Scratch &ws, const EvalParams &p, int search_mode,
-                            int64_t n_tasks, int *grid_out);
+                            int64_t n_tasks, int *grid_out, bool wide_buf = false);
 struct DeviceGuard {
     int prev = -1;
     explicit DeviceGuard(int dev) {

@@ -88,6 +88,10 @@ struct pesto_search {
     std::vector<int32_t> coarse_of;
     std::vector<uint8_t> cpos;
     DevBuf d_cpos;
+    // the wide eval32 launch (bases at or above saturation) runs on `aux`, forked from and
+    // joined back into the caller's stream, beside the 32-bit launch
+    cudaStream_t aux = nullptr;
+    cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
 };
 
 namespace {
@@ -238,8 +242,22 @@ pesto_status launch_search_eval(pesto_search *s, int b_first, int n_bases, int64
         plan_eval32(g, p32, j0, j1, n_bases);
         if ((rc = ensure_state32(g, g->ws, p32, 1, p32.n_tasks, &grid))) return rc;
         p32.state32 = g->ws.state32.as<uint32_t>();
+        if (s->all_below) {
+            if ((e = launch_eval32(p32, 1, grid, st)) != cudaSuccess) return cuda_fail(e, "launch eval32");
+            return PESTO_OK;
+        }
+        // some bases are at or above saturation: their wide launch runs on the auxiliary
+        // stream beside this one (own cold-slot buffer; disjoint bases, so disjoint keys)
+        if (!s->aux) {
+            if ((e = cudaStreamCreateWithFlags(&s->aux, cudaStreamNonBlocking)) != cudaSuccess ||
+                (e = cudaEventCreateWithFlags(&s->ev_fork, cudaEventDisableTiming)) != cudaSuccess ||
+                (e = cudaEventCreateWithFlags(&s->ev_join, cudaEventDisableTiming)) != cudaSuccess)
+                return cuda_fail(e, "auxiliary stream");
+        }
+        if ((e = cudaEventRecord(s->ev_fork, st)) != cudaSuccess ||
+            (e = cudaStreamWaitEvent(s->aux, s->ev_fork, 0)) != cudaSuccess)
+            return cuda_fail(e, "fork");
         if ((e = launch_eval32(p32, 1, grid, st)) != cudaSuccess) return cuda_fail(e, "launch eval32");
-        if (s->all_below) return PESTO_OK;
         // bases at or above saturation: the wide eval32 instance (exact 64-bit times, the
         // same step records) -- about 2x the throughput of eval64 there
         p32.gate = 2;
@@ -254,9 +272,12 @@ pesto_status launch_search_eval(pesto_search *s, int b_first, int n_bases, int64
             p32.tasks_per_base = (j1 - (j0 - j0 % ts) + ts - 1) / ts;
             p32.n_tasks = p32.tasks_per_base * n_bases;
         }
-        if ((rc = ensure_state32(g, g->ws, p32, 1, p32.n_tasks, &grid))) return rc;
-        p32.state32 = g->ws.state32.as<uint32_t>();
-        if ((e = launch_eval32(p32, 1, grid, st)) != cudaSuccess) return cuda_fail(e, "launch wide eval32");
+        if ((rc = ensure_state32(g, g->ws, p32, 1, p32.n_tasks, &grid, true))) return rc;
+        p32.state32 = g->ws.state32w.as<uint32_t>();
+        if ((e = launch_eval32(p32, 1, grid, s->aux)) != cudaSuccess) return cuda_fail(e, "launch wide eval32");
+        if ((e = cudaEventRecord(s->ev_join, s->aux)) != cudaSuccess ||
+            (e = cudaStreamWaitEvent(st, s->ev_join, 0)) != cudaSuccess)
+            return cuda_fail(e, "join");
         return PESTO_OK;
     }
     if ((rc = ensure_state(g, g->ws, p, 1, p.n_tasks, &grid))) return rc;
@@ -822,6 +843,10 @@ void pesto_search_destroy(pesto_search *s) {
     if (!s) return;
     DeviceGuard guard(s->g->device);
     if (s->comm && nccl().comm_destroy) nccl().comm_destroy(s->comm);
+    if (s->aux) cudaStreamSynchronize(s->aux);
+    if (s->ev_fork) cudaEventDestroy(s->ev_fork);
+    if (s->ev_join) cudaEventDestroy(s->ev_join);
+    if (s->aux) cudaStreamDestroy(s->aux);
     if (s->h_swap) cudaFreeHost(s->h_swap);
     if (s->h_keys) cudaFreeHost(s->h_keys);
     delete s;
