@@ -536,8 +536,6 @@ eval32_kernel(const EvalParams P) {
 
     uint32_t it = 0;
     int prev_bl = -1;
-    __shared__ unsigned long long red_s[2][8];   // K3: per-warp minima, by task parity
-    int tpar = 0;
     for (int64_t task = blockIdx.x; task < P.n_tasks; task += gridDim.x) {
         const int bl = kSearch ? (int)(task / P.tasks_per_base) : 0;
         if (!runs_here(bl)) continue;
@@ -910,32 +908,6 @@ eval32_kernel(const EvalParams P) {
         }
         cp_async_wait<0>();
 
-        if constexpr (MODE != 0) {       // search (1, 5) and exhaustive coarse (4): keys
-            // K3: warp min, then the CTA's minimum over its consumer warps (shared memory, one
-            // named barrier), one atomicMin per CTA and task.  A saturated candidate's true
-            // makespan is >= kSat32 > this base's makespan, so it never wins the argmin; its
-            // clamped key still sorts after the base's (exact) key.
-            uint64_t key = ~0ull;
-            if (active) {
-#pragma unroll
-                for (int c = 0; c < CPL; c++) {
-                    const int64_t j = j0 + c * 32 + lane;
-                    const uint64_t kc = valid[c] ? (((uint64_t)st.makespan(c) << 24) | (uint64_t)j) : ~0ull;
-                    key = kc < key ? kc : key;
-                }
-            }
-            key = warp_min_u64(key);
-            if (lane == 0) red_s[tpar][warp] = key;
-            named_bar_sync(2, NW * 32);
-            if (warp == 0) {
-                uint64_t k2 = lane < NW ? red_s[tpar][lane] : ~0ull;
-                k2 = warp_min_u64(k2);
-                if (lane == 0 && k2 != ~0ull)
-                    atomicMin(reinterpret_cast<unsigned long long *>(P.keys + bl), (unsigned long long)k2);
-            }
-            tpar ^= 1;                   // double-buffered: no barrier before the next write
-            continue;
-        }
         if (!active) continue;
         if (MODE == 0) {
 #pragma unroll
@@ -952,6 +924,19 @@ eval32_kernel(const EvalParams P) {
                     P.flag_list[atomicAdd(P.flag_count, 1)] = (int32_t)j;
                 }
             }
+        } else {
+            // a saturated candidate's true makespan is >= kSat32 > this base's makespan, so it
+            // never wins the argmin; its clamped key still sorts after the base's (exact) key
+            uint64_t key = ~0ull;
+#pragma unroll
+            for (int c = 0; c < CPL; c++) {
+                const int64_t j = j0 + c * 32 + lane;
+                const uint64_t kc = valid[c] ? (((uint64_t)st.makespan(c) << 24) | (uint64_t)j) : ~0ull;
+                key = kc < key ? kc : key;
+            }
+            key = warp_min_u64(key);
+            if (lane == 0 && key != ~0ull)
+                atomicMin(reinterpret_cast<unsigned long long *>(P.keys + bl), (unsigned long long)key);
         }
     }
 }
