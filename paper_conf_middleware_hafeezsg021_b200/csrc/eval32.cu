@@ -491,7 +491,12 @@ eval32_kernel(const EvalParams P) {
     cx.cls1 = 0;
     for (int i = 0; i < P.D * P.D; i++)
         if (P.link_class[i] == 1) cx.cls1 |= 1ull << i;
-    const uint32_t stage = su32_reg(stage_all + (size_t)warp * kRing * CW + lane);
+    // the staging ring sits a compile-time distance after the near ring (both NW x kRing x CW
+    // times, 16-byte multiples): derived from cx.ring so that the pair of loads per position
+    // shares one address register (the second load takes an immediate offset)
+    static_assert((NW * kRing * CW * sizeof(T)) % 16 == 0, "ring and staging are adjacent");
+    const uint32_t stage = cx.ring + (uint32_t)(NW * kRing * CW * sizeof(T));
+    (void)stage_all;
 
     using StateT = typename std::conditional<PL == 1, RegState32<CPL, T>, SmemState32<CPL, T>>::type;
     StateT st;
