@@ -5,10 +5,12 @@ step on B200 (BASELINE.json metric).  One JSON line on rank 0.
   python bench.py [--gpus N] [--steps K] [--warmup W] [--config NAME] [--impl pesto|reference]
 
 A step = one pass of the whole hot path over one batch: K2 neighbour decode + K1 makespan of
-every candidate + K3 argmin (one kernel) -> N1 allreduce-MIN over ranks -> K4 commit.  At N=1 the
-workload is BASELINE.json configs[1] (inception_v3_2dev: 65,536 candidates/step); per-GPU work
+every candidate + K3 argmin (one kernel) -> N1 allreduce-MIN over ranks -> K4 commit.  Per-GPU work
 is fixed as N grows (weak scaling).  `--impl reference` times the CPU oracle on the same
 workload (the reference arm of this tier).
+
+Default workload: transformer_2dev (BASELINE.json configs[3], 1,048,576 candidates per step, the
+largest single-GPU config; Table 1's Transformer-6 row).
 """
 
 from __future__ import annotations
@@ -27,10 +29,10 @@ import numpy as np
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
-from workloads import configs, dag  # noqa: E402
+from workloads import configs, dag, seeds  # noqa: E402
 
 METRIC = "placement candidates evaluated/sec (and op-relaxations/sec) at 1/2/4/8 B200"
-DEFAULT_CONFIG = "inception_v3_2dev"
+DEFAULT_CONFIG = "transformer_2dev"
 
 
 def parse():
@@ -126,21 +128,41 @@ class ClockSampler:
 
 
 def seeds_for(P, G, g, n_bases: int):
-    """Search incumbents (row a1): expert, topological split, single-device, random."""
+    """Search incumbents (row a1) from libpesto's generators: expert, topological split,
+    single-device, random.  They must equal workloads/seeds.py's plain-Python restatement, which
+    the CPU reference arm starts from (so both arms search the same four bases)."""
     o_cp = G.seed_order(P.ORDER_CRITICAL_PATH)
     o_fifo = G.seed_order(P.ORDER_FIFO)
-    o_rand = G.seed_order(P.ORDER_RANDOM, 2021)
+    o_rand = G.seed_order(P.ORDER_RANDOM, configs.SEARCH_SEED)
     xs = [G.seed_placement(P.PLACE_EXPERT, layer=g.layer) if g.layer is not None
           else G.seed_placement(P.PLACE_TOPO_SPLIT, order=o_cp),
           G.seed_placement(P.PLACE_TOPO_SPLIT, order=o_cp),
           G.seed_placement(P.PLACE_SINGLE),
-          G.seed_placement(P.PLACE_RANDOM, seed=2021)]
+          G.seed_placement(P.PLACE_RANDOM, seed=configs.SEARCH_SEED)]
     os_ = [o_cp, o_cp, o_fifo, o_rand]
-    return np.stack(xs[:n_bases]), np.stack(os_[:n_bases])
+    xs, os_ = np.stack(xs[:n_bases]), np.stack(os_[:n_bases])
+    px, po = seeds.bench_seeds(g, n_bases, configs.SEARCH_SEED)
+    assert (px == xs).all() and (po == os_).all(), "library seeds differ from workloads/seeds.py"
+    return xs, os_
+
+
+def common_config(args, cfg, g, world):
+    """The `config` object both arms print (same keys and values, so the driver can match them)."""
+    k_gpu = cfg.candidates_per_gpu
+    return {"workload": args.config, "n_ops": g.n, "n_edges": g.m, "D": g.D,
+            "candidates_per_step": k_gpu * world, "candidates_per_gpu": k_gpu,
+            "bases": cfg.bases, "k_per_base": (k_gpu * world) // cfg.bases,
+            "move_mix": list(configs.MOVE_MIX), "search_seed": configs.SEARCH_SEED,
+            "seeds": "expert / topological split on the critical-path order, single device on "
+                     "the FIFO order, random placement on a random order (workloads/seeds.py)",
+            "l2": "GPU arm: flushed (256 MiB write) between timed steps",
+            "parallelism": f"candidate-dp{world}", "dispatch": args.dispatch,
+            "coarse_groups_pct": args.coarse_pct}
 
 
 def oracle_rate(g, xs, orders, k_per_base, seconds, threads, nondelay=False, coarse=None):
-    """Oracle (as it stands) on a bounded sample of this workload's step-0 candidates."""
+    """Oracle (as it stands) on a bounded sample of this workload's step-0 candidates: the
+    first ids of every base (they span whole 128-id groups, swap groups included)."""
     from oracle import oracle as O
     if coarse is not None:                   # the same S9 coarse groups as the timed search
         with O.coarse_moves(g, *coarse):
@@ -160,15 +182,12 @@ def oracle_rate(g, xs, orders, k_per_base, seconds, threads, nondelay=False, coa
     keys(0, probe)
     dt = time.perf_counter() - t0
     per = dt / probe
-    sample = int(max(probe, min(k_per_base, seconds / max(per, 1e-9))))
+    sample = int(max(probe * P_, min(k_per_base * P_, seconds / max(per, 1e-9))))
     t0 = time.perf_counter()
     done = 0
     sample_keys = []
     for b in range(P_):
         cnt = sample // P_
-        if cnt <= 0:
-            sample_keys.append(np.zeros(0, np.uint64))
-            continue
         sample_keys.append(keys(b, cnt))
         done += cnt
     dt = time.perf_counter() - t0
@@ -177,37 +196,41 @@ def oracle_rate(g, xs, orders, k_per_base, seconds, threads, nondelay=False, coa
 
 
 def run_reference(args, rank, world):
+    """This tier's reference arm: the CPU oracle as it stands, on the same workload, the same
+    four bases (workloads/seeds.py) and the same step-0 candidates; each step is a bounded
+    sample, timed on the wall clock (ms_per_step is the measured sample step)."""
     if rank != 0:
         return
     cfg = configs.CONFIGS[args.config]
     g = configs.graph_for(cfg)
     from oracle import oracle as O  # noqa: F401  (TEST INFRASTRUCTURE: the reference arm)
     threads = len(os.sched_getaffinity(0))
-    # seeds via plain host code shared with nothing: CP order from the generator's Kahn
-    order = dag.random_topo_order(g, 0)
-    xs = np.stack([np.zeros(g.n, np.uint8), dag.random_placements(g, 1, 1)[0]])
-    orders = np.stack([order, order])
-    per_step_budget = max(1.0, args.cpu_seconds / max(1, args.steps + args.warmup))
-    rates, times = [], []
+    xs, orders = seeds.bench_seeds(g, cfg.bases, configs.SEARCH_SEED)
+    k_per_base = cfg.candidates_per_gpu // cfg.bases
+    per_step_budget = max(0.5, args.cpu_seconds / max(1, args.steps + args.warmup))
+    rates, times, counts = [], [], []
     nd = args.dispatch == "nondelay"
     for i in range(args.warmup + args.steps):
-        rate, done, dt = oracle_rate(g, xs, orders, cfg.candidates_per_gpu // 2, per_step_budget,
-                                     threads, nondelay=nd)
+        rate, done, dt = oracle_rate(g, xs, orders, k_per_base, per_step_budget, threads,
+                                     nondelay=nd)
         if i >= args.warmup:
             rates.append(rate)
             times.append(dt)
-    value = statistics.median(rates)
+            counts.append(done)
+    value = sum(counts) / sum(times)
     line = {"impl": "reference", "metric": METRIC, "value": value, "unit": "candidates/s",
             "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
-            "ms_per_step": 1e3 * cfg.candidates_per_gpu / value, "higher_is_better": True,
+            "ms_per_step": 1e3 * statistics.median(times), "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "int64", "data": "synthetic",
-            "config": {"workload": args.config, "n_ops": g.n, "n_edges": g.m, "D": g.D,
-                       "candidates_per_step": cfg.candidates_per_gpu, "dispatch": args.dispatch},
+            "config": common_config(args, cfg, g, 1),
             "op_relaxations_per_s": value * g.n,
             "cpu_baseline": {"value": value, "unit": "candidates/s", "cores": threads,
                              "kind": "oracle",
-                             "sample": f"{args.steps} steps x ~{per_step_budget:.1f}s of step-0 "
-                                       "neighbour candidates, event-driven simulator"},
+                             "sample": f"each step: the first {counts[0] // cfg.bases} step-0 "
+                                       f"neighbour ids of each of the {cfg.bases} bases "
+                                       f"({counts[0]} candidates, ~{per_step_budget:.1f} s), "
+                                       "event-driven simulator; ms_per_step is that sample's "
+                                       "measured wall time"},
             "e2e": {"value": value, "unit": "candidates/s", "h2d_bytes_per_step": 0,
                     "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
@@ -300,9 +323,14 @@ def run_pesto(args, rank, world, local):
     if not args.no_e2e:
         rows_h = []
         for r in range(2):                           # two distinct input batches, alternating
-            rows = P.pack_rows(dag.random_placements(g, 11 + 2 * rank + r, k_gpu), g.D)
+            rows = dag.random_packed_rows(g, 11 + 2 * rank + r, k_gpu)
             rows_h.append(torch.from_numpy(rows).pin_memory().numpy())
-        nbuf = int(os.environ.get("PESTO_E2E_BUFFERS", "4"))     # batches in flight
+            del rows
+        # batches in flight: 4 for one-wave batches (inception's 64 K rows: their kernels overlap
+        # each other), 2 for multi-wave ones (1 M rows: the copy-in of one batch overlaps the
+        # evaluation of the other; each workspace holds ~14 GB of scratch at that size)
+        nbuf = int(os.environ.get("PESTO_E2E_BUFFERS",
+                                  "4" if rows_h[0].nbytes < (1 << 30) else "2"))
         outs = [torch.empty(k_gpu, dtype=torch.int64).pin_memory().numpy() for _ in range(nbuf)]
         wss = [G.workspace() for _ in range(nbuf)]
         sts = [torch.cuda.Stream() for _ in range(nbuf)]
@@ -357,54 +385,45 @@ def run_pesto(args, rank, world, local):
     achieved = alg_ops_launch / eval_avg_s / 1e12
     traffic = None
     issue = None
-    prof = os.path.join(ROOT, "profiles", f"r1_eval32_{args.config.split('_')[0]}_ncu.json")
-    if os.path.exists(prof) and world == 1 and not nd:
+    prof = None
+    for cand in (f"r2_eval32_{args.config}_ncu.json",
+                 f"r1_eval32_{args.config.split('_')[0]}_ncu.json"):
+        if os.path.exists(os.path.join(ROOT, "profiles", cand)):
+            prof = os.path.join(ROOT, "profiles", cand)
+            break
+    if prof and world == 1 and not nd:
         try:
             pj = json.load(open(prof))
             if pj.get("config") == args.config:
                 traffic = pj["dram_bytes_per_launch"]
                 m = pj["metrics"]
+                inst = m["smsp__inst_executed.sum"]["value"]
                 issue = {"issue_slots_busy_pct": m["smsp__issue_active.avg.pct_of_peak_sustained_active"]["value"],
                          "warps_per_smsp": m["smsp__warps_active.avg.per_cycle_active"]["value"],
                          "dram_GBps": pj.get("dram_GBps"),
-                         "source": os.path.relpath(prof, ROOT)}
+                         "l2_bytes_per_launch": pj.get("lts_bytes_per_launch"),
+                         "warp_instr_per_op_relax": inst / (k_gpu * g.n),
+                         "source": os.path.relpath(prof, ROOT),
+                         "note": "ncu capture of the same kernel on the same config (cold cache, "
+                                 "one launch); its duration is not this run's"}
         except Exception:
             traffic = None
-    # SURVEY §8(d) issue roof: 148 SMs x 4 warp-instr/clk at sm_max_mhz, at the survey's
-    # estimate of 2 warp instructions per op-relaxation; the measured instructions per
-    # op-relaxation come from the ncu capture of the same kernel (profiles/)
-    issue_peak = 148 * 4 * sm_mhz * 1e6
-    op_relax_k1 = k_gpu * g.n / eval_avg_s
-    issue_roof = {"unit": "op-relax/s", "achieved": op_relax_k1, "peak": issue_peak / 2.0,
-                  "frac": op_relax_k1 / (issue_peak / 2.0),
-                  "peak_source": "148 SMs x 4 warp-instr/clk x sm_max_mhz / 2 warp-instr per "
-                                 "op-relax (SURVEY 8(d) estimate)",
-                  "measured_warp_instr_per_op_relax": None}
-    if issue is not None:
-        try:
-            inst = json.load(open(prof))["metrics"]["smsp__inst_executed.sum"]["value"]
-            issue_roof["measured_warp_instr_per_op_relax"] = inst / (k_gpu * g.n)
-        except Exception:
-            pass
     st = G.stats(orders[0])
     line = {"metric": METRIC, "value": value, "unit": "candidates/s", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": tot_ms / args.steps,
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int64",
             "data": "synthetic",
-            "config": {"workload": args.config, "n_ops": g.n, "n_edges": g.m, "D": g.D,
-                       "candidates_per_step": k_gpu * world, "candidates_per_gpu": k_gpu,
-                       "bases": n_bases, "k_per_base": k_per_base, "move_mix": configs.MOVE_MIX,
-                       "live_slots": st["live_slots"], "l2": "flushed between timed steps",
-                       "f_x_seeds": [round(float((xs[b][g.src] != xs[b][g.dst]).mean()), 4)
-                                     for b in range(n_bases)],
-                       "time_t": "uint32 saturating at 4.03 s (eval32), exact 64-bit for bases "
-                                 "above it (wide eval32 / eval64)",
-                       "state_tier": "near ring + far staging in shared memory, cold slots in "
-                                     "global memory (L2/HBM), device/link state in registers "
-                                     "(D = 2) or shared memory (D > 2)",
-                       "parallelism": f"candidate-dp{world}", "dispatch": args.dispatch,
-                       "coarse_groups_pct": args.coarse_pct,
-                       "n_coarse": int(coarse[1]) if coarse else None},
+            "config": common_config(args, cfg, g, world),
+            "workload_details": {
+                "live_slots": st["live_slots"],
+                "f_x_seeds": [round(float((xs[b][g.src] != xs[b][g.dst]).mean()), 4)
+                              for b in range(n_bases)],
+                "time_t": "uint32 saturating at 4.03 s (eval32), exact 64-bit for bases "
+                          "above it (wide eval32 / eval64)",
+                "state_tier": "near ring + far staging in shared memory, cold slots in global "
+                              "memory (L2/HBM), device/link state in registers (D = 2) or "
+                              "shared memory (D > 2)",
+                "n_coarse": int(coarse[1]) if coarse else None},
             "op_relaxations_per_s": value * g.n, "edge_relaxations_per_s": value * g.m,
             "eval_kernel_ms": tot_eval_ms / args.steps,
             "roofline": {"bound": "alu", "achieved": achieved, "peak": peak_tops,
@@ -415,7 +434,6 @@ def run_pesto(args, rank, world, local):
                          "kernel": "nondelay_kernel (row f4(i))" if nd else "eval32_kernel (K1)",
                          "note": "algorithmic int ops (2n+m+2*cross per candidate) / K1 time; "
                                  "traffic = ncu DRAM bytes per K1 launch (profiles/)"},
-            "issue_roof": issue_roof,
             "roofs": dict(roofs, source="pesto_measure_roofs (csrc/roofs.cu): K1's max/add/"
                           "saturate chains on all SMs, L2-resident sweeps, 1 GiB copy; best of 5",
                           k1_frac_of_measured_int_roof=achieved * 1e12 / roofs["int_ops_per_s"]),
@@ -433,18 +451,30 @@ def run_pesto(args, rank, world, local):
                                 "kind": "oracle",
                                 "sample": f"{done} step-0 neighbour candidates of the same "
                                           f"{n_bases} bases ({dt:.1f}s)"}
-        # the same sample on the GPU (a fresh search at step 0, every candidate's key from the
-        # independent 64-bit kernel), compared key by key with the oracle's
+        # the same sample on the GPU (a fresh search at step 0): every candidate's key from the
+        # kernel instantiation the timed step launches (pesto_search_candidate_keys_ex,
+        # PESTO_KEYS_TIMED), compared key by key with the oracle's; saturated 32-bit walks are
+        # re-run by the 64-bit kernel there, and the raw timed output is checked on the rest
         S0 = P.Search(G, xs, orders, k_per_base, configs.MOVE_MIX, configs.SEARCH_SEED)
         if coarse is not None:
             S0.set_coarse_moves(*coarse)
-        mism = 0
+        mism = mism_raw = n_sat = 0
         for b, ok in enumerate(oracle_rate.sample_keys):
             if len(ok):
-                mism += int((S0.candidate_keys(b, 0, len(ok)) != ok).sum())
+                gk = S0.candidate_keys(b, 0, len(ok), kernel=P.KEYS_TIMED)
+                raw = S0.candidate_keys(b, 0, len(ok), kernel=P.KEYS_TIMED_RAW)
+                mism += int((gk != ok).sum())
+                sat = (raw != P.KEY_INVALID) & ((raw >> np.uint64(24)) >= np.uint64(0xF0000000))
+                n_sat += int(sat.sum())
+                mism_raw += int((raw[~sat] != ok[~sat]).sum())
+                # a clamped walk's exact makespan is at least the clamp
+                mism_raw += int(((ok[sat] >> np.uint64(24)) < np.uint64(0xF0000000)).sum())
         line["parity"] = {"checked": int(done), "mismatches": mism,
-                          "what": "keys (makespan << 24 | j) of the cpu_baseline sample, GPU "
-                                  "(pesto_search_candidate_keys) vs oracle, bit-exact"}
+                          "raw_mismatches": mism_raw, "saturated_walks": n_sat,
+                          "what": "keys (makespan << 24 | j) of the cpu_baseline sample from the "
+                                  "timed eval32 instantiation (pesto_search_candidate_keys_ex "
+                                  "PESTO_KEYS_TIMED: same kernel, CPL and 32-bit/wide split as "
+                                  "the step) vs the oracle, bit-exact"}
     print(json.dumps(line), flush=True)
     if world > 1:
         dist.destroy_process_group()

@@ -239,6 +239,9 @@ typedef struct {
                                     /* NULL and world > 1 the caller reduces keys itself          */
 } pesto_search_desc;
 
+/* The search snapshots the graph's comm model (its layouts hold the transfer times): a later
+ * pesto_comm_model on the same graph makes pesto_search_eval / _commit / _step /
+ * _candidate_keys return PESTO_ESTATE -- create a new search after changing the comm model. */
 pesto_status pesto_search_create(pesto_graph *g, const pesto_search_desc *desc,
                                  pesto_search **out);
 
@@ -254,8 +257,22 @@ pesto_status pesto_search_keys(pesto_search *s, uint64_t *keys_host, void *cuda_
 pesto_status pesto_search_set_keys(pesto_search *s, const uint64_t *keys_host, void *cuda_stream);
 pesto_status pesto_search_commit(pesto_search *s, void *cuda_stream); /* K4 + step += 1        */
 
-/* Keys (makespan << 24 | j, UINT64_MAX if invalid) of candidates j in [j0, j1) of `base` at
- * the current step, into DEVICE keys_out[j1 - j0] (parity/debug; ignores rank/world). */
+/* Per-candidate keys (makespan << 24 | j, UINT64_MAX if invalid) of candidates j in [j0, j1)
+ * of `base` at the current step, into DEVICE keys_out[j1 - j0] (parity/debug; ignores
+ * rank/world).  `kernel` says which kernel computes them:
+ *   PESTO_KEYS_TIMED     the instantiation pesto_search_eval launches for this step (same
+ *                        kernel, candidates per lane, 32-bit / wide split), each walk storing
+ *                        its own key after the argmin epilogue; walks that saturated the 32-bit
+ *                        time (makespan field >= 0xF0000000) are re-run by the exact 64-bit
+ *                        kernel, so every key is exact.  Synchronises the stream.
+ *   PESTO_KEYS_EVAL64    the independent exact 64-bit kernel (eval64) for every candidate.
+ *   PESTO_KEYS_TIMED_RAW the timed instantiation's own output, saturated walks left clamped
+ *                        (makespan field 0xF0000000).
+ * pesto_search_candidate_keys = _ex with PESTO_KEYS_TIMED.  Errors: EINVAL (range outside
+ * [0, K], unknown kernel), ESTATE, ECUDA. */
+enum { PESTO_KEYS_TIMED = 0, PESTO_KEYS_EVAL64 = 1, PESTO_KEYS_TIMED_RAW = 2 };
+pesto_status pesto_search_candidate_keys_ex(pesto_search *s, int32_t base, int64_t j0, int64_t j1,
+                                            uint64_t *keys_out, int32_t kernel, void *cuda_stream);
 pesto_status pesto_search_candidate_keys(pesto_search *s, int32_t base, int64_t j0, int64_t j1,
                                          uint64_t *keys_out, void *cuda_stream);
 

@@ -938,6 +938,9 @@ eval32_kernel(const EvalParams P) {
                 const int64_t j = j0 + c * 32 + lane;
                 const uint64_t kc = valid[c] ? (((uint64_t)st.makespan(c) << 24) | (uint64_t)j) : ~0ull;
                 key = kc < key ? kc : key;
+                // parity output (pesto_search_candidate_keys): this walk's own key of every
+                // candidate, after the walk -- a saturated one carries kSat32 as its makespan
+                if (P.keys_dbg && j >= P.j_begin && j < P.j_end) P.keys_dbg[j - P.j_begin] = kc;
             }
             key = warp_min_u64(key);
             if (lane == 0 && key != ~0ull)

@@ -166,7 +166,6 @@ struct CommitParams {
     const uint64_t *keys;
     int64_t *base_mk;
     int32_t *swap_out;                  // [P] committed swap position or -1
-    int32_t patch32;                    // eval32 records carry base codes: patch them too
     Feasibility feas;                   // f3: the committed move updates fbase
     int32_t n_coarse, coarse_pct;       // S9 coarse groups (0 = off)
 };

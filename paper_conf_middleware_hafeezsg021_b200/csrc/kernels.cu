@@ -667,7 +667,7 @@ __global__ void commit_kernel(const CommitParams P) {
                       (unsigned long long)m);
         }
         set_dev_at<PL>(bits, words, q, x);
-        if (!P.patch32) return;
+        if (B.W32 == 0) return;           // this base has no eval32 records (per base)
         uint32_t *flags = reinterpret_cast<uint32_t *>(blob32 + B.op_off32[q]) + 3;   // StepHead
         *flags = (*flags & ~kStXMask) | (uint32_t)x;
         for (uint32_t i = B.pin_off[q]; i < B.pin_off[q + 1]; i++) {

@@ -79,6 +79,10 @@ struct pesto_search {
     // row f3: footprint of each base per device ([P][8]), for the constraints of cons_gen
     DevBuf d_fbase;
     int64_t cons_gen = -1;
+    // the comm model the bases' layouts were built with (their edge records hold the transfer
+    // times); a later pesto_comm_model makes the search fail with ESTATE instead of walking
+    // stale records
+    int64_t comm_gen = -1;
     // committed swaps: patched in place on the device vs. layout rebuilt on the host
     DevBuf d_patch;
     int64_t n_swap_inplace = 0, n_swap_rebuilt = 0;
@@ -191,11 +195,15 @@ pesto_status launch_search_nondelay(pesto_search *s, int b_first, int n_bases, i
 
 // fast: eval32 for the bases below saturation (+ eval64 for the others while any may exist);
 // otherwise (debug keys, initial makespans, ineligible graphs) eval64 for all candidates
+// cpl_force (1 or 2): the candidates-per-lane instance to launch instead of the one this range
+// alone would choose -- the parity path runs the instance the full step launches
 pesto_status launch_search_eval(pesto_search *s, int b_first, int n_bases, int64_t j0, int64_t j1,
                                 uint64_t *keys, uint64_t *keys_dbg, cudaStream_t st,
-                                bool fast = false) {
+                                bool fast = false, int cpl_force = 0) {
     pesto_graph *g = s->g;
     if (j1 <= j0) return PESTO_OK;
+    if (s->comm_gen >= 0 && s->comm_gen != g->comm_gen)
+        return fail(PESTO_ESTATE, "the comm model changed after the search was created");
     pesto_status rc0 = sync_constraints(s);
     if (rc0) return rc0;
     if (s->coarse_pct > 0 && (g->has_cap || g->has_coloc))
@@ -233,13 +241,18 @@ pesto_status launch_search_eval(pesto_search *s, int b_first, int n_bases, int64
     int grid = 0;
     pesto_status rc;
     cudaError_t e;
-    const bool use32 = fast && s->use32 && keys_dbg == nullptr &&
-                       g->link_model == PESTO_LINKS_FCFS;   // f4(ii) runs on eval64
+    const bool use32 = fast && s->use32 && g->link_model == PESTO_LINKS_FCFS;   // f4(ii): eval64
     if (use32) {
         // eval32 tasks: consecutive ids from a multiple of the task size
         EvalParams p32 = p;
         p32.gate = 1;
         plan_eval32(g, p32, j0, j1, n_bases);
+        if (cpl_force == 1 || cpl_force == 2) {
+            p32.cpl32 = cpl_force;
+            const int64_t ts = eval32_task_size(cpl_force);
+            p32.tasks_per_base = (j1 - (j0 - j0 % ts) + ts - 1) / ts;
+            p32.n_tasks = p32.tasks_per_base * n_bases;
+        }
         if ((rc = ensure_state32(g, g->ws, p32, 1, p32.n_tasks, &grid))) return rc;
         p32.state32 = g->ws.state32.as<uint32_t>();
         if (s->all_below) {
@@ -593,6 +606,7 @@ pesto_status pesto_search_create(pesto_graph *g, const pesto_search_desc *d, pes
         if ((rc = upload_layout(g, *s->layouts[b]))) return rc;
         if ((rc = upload_bits(s.get(), b, d->base_x + (size_t)b * n))) return rc;
     }
+    s->comm_gen = g->comm_gen;
     if ((e = s->d_views.ensure(sizeof(BaseLayoutDev) * s->P)) != cudaSuccess) return cuda_fail(e, "allocate");
     refresh_views(s.get());
     if ((e = cudaMemcpy(s->d_views.ptr, s->views.data(), sizeof(BaseLayoutDev) * s->P,
@@ -666,6 +680,8 @@ pesto_status pesto_search_set_keys(pesto_search *s, const uint64_t *keys_host, v
 pesto_status pesto_search_commit(pesto_search *s, void *stream) {
     if (!s) return fail(PESTO_EINVAL, "NULL search");
     pesto_graph *g = s->g;
+    if (s->comm_gen != g->comm_gen)
+        return fail(PESTO_ESTATE, "the comm model changed after the search was created");
     DeviceGuard guard(g->device);
     cudaStream_t st = (cudaStream_t)stream;
     s->last_stream = st;
@@ -686,7 +702,6 @@ pesto_status pesto_search_commit(pesto_search *s, void *stream) {
     cp.keys = s->d_keys.as<uint64_t>();
     cp.base_mk = s->d_mk.as<int64_t>();
     cp.swap_out = s->d_swap.as<int32_t>();
-    cp.patch32 = s->use32 ? 1 : 0;
     cp.feas = feasibility_view(g);
     cp.feas.fbase = s->d_fbase.as<int64_t>();
     cp.n_coarse = s->n_coarse;
@@ -800,16 +815,47 @@ pesto_status pesto_search_step(pesto_search *s, void *stream) {
     return pesto_search_commit(s, stream);
 }
 
-pesto_status pesto_search_candidate_keys(pesto_search *s, int32_t base, int64_t j0, int64_t j1,
-                                         uint64_t *keys_out, void *stream) {
+pesto_status pesto_search_candidate_keys_ex(pesto_search *s, int32_t base, int64_t j0, int64_t j1,
+                                            uint64_t *keys_out, int32_t kernel, void *stream) {
     if (!s || !keys_out) return fail(PESTO_EINVAL, "NULL argument");
     if (base < 0 || base >= s->P) return fail(PESTO_EINVAL, "base out of range");
     if (j0 < 0 || j1 < j0 || j1 > s->K) return fail(PESTO_EINVAL, "candidate range out of [0, K]");
-    DeviceGuard guard(s->g->device);
+    if (kernel < PESTO_KEYS_TIMED || kernel > PESTO_KEYS_TIMED_RAW)
+        return fail(PESTO_EINVAL, "unknown key kernel");
+    if (j1 == j0) return PESTO_OK;
+    pesto_graph *g = s->g;
+    DeviceGuard guard(g->device);
     cudaStream_t st = (cudaStream_t)stream;
     cudaError_t e = cudaMemsetAsync(s->d_dbg_key.ptr, 0xFF, 8, st);
     if (e != cudaSuccess) return cuda_fail(e, "reset");
-    return launch_search_eval(s, base, 1, j0, j1, s->d_dbg_key.as<uint64_t>(), keys_out, st);
+    if (kernel == PESTO_KEYS_EVAL64)
+        return launch_search_eval(s, base, 1, j0, j1, s->d_dbg_key.as<uint64_t>(), keys_out, st);
+    // the instance the timed step launches: its candidates-per-lane choice is the full step's
+    EvalParams plan;
+    fill_eval_common(g, plan);
+    plan_eval32(g, plan, s->j_begin, s->j_end, s->P);
+    pesto_status rc = launch_search_eval(s, base, 1, j0, j1, s->d_dbg_key.as<uint64_t>(), keys_out,
+                                         st, true, plan.cpl32);
+    if (rc || kernel == PESTO_KEYS_TIMED_RAW || !s->use32 || g->dispatch != PESTO_DISPATCH_FIXED ||
+        g->link_model != PESTO_LINKS_FCFS)
+        return rc;                                   // (those paths are exact 64-bit already)
+    // saturated 32-bit walks (makespan field kSat32): exact keys from the 64-bit kernel
+    std::vector<uint64_t> h((size_t)(j1 - j0));
+    if ((e = cudaMemcpyAsync(h.data(), keys_out, h.size() * 8, cudaMemcpyDeviceToHost, st)) != cudaSuccess ||
+        (e = cudaStreamSynchronize(st)) != cudaSuccess)
+        return cuda_fail(e, "read keys");
+    for (size_t i = 0; i < h.size(); i++) {
+        if (h[i] == ~0ull || (h[i] >> 24) < (uint64_t)kSat32) continue;
+        const int64_t j = j0 + (int64_t)i;
+        if ((rc = launch_search_eval(s, base, 1, j, j + 1, s->d_dbg_key.as<uint64_t>(), keys_out + i, st)))
+            return rc;
+    }
+    return PESTO_OK;
+}
+
+pesto_status pesto_search_candidate_keys(pesto_search *s, int32_t base, int64_t j0, int64_t j1,
+                                         uint64_t *keys_out, void *stream) {
+    return pesto_search_candidate_keys_ex(s, base, j0, j1, keys_out, PESTO_KEYS_TIMED, stream);
 }
 
 pesto_status pesto_search_get(pesto_search *s, int32_t base, int64_t *mk, uint8_t *x_host,

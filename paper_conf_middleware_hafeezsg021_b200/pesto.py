@@ -23,6 +23,7 @@ ORDER_CRITICAL_PATH, ORDER_FIFO, ORDER_RANDOM = 0, 1, 2
 LINKS_FCFS, LINKS_UNLIMITED = 0, 1
 DISPATCH_FIXED, DISPATCH_NONDELAY = 0, 1
 PLACE_SINGLE, PLACE_EXPERT, PLACE_TOPO_SPLIT, PLACE_RANDOM = 0, 1, 2, 3
+KEYS_TIMED, KEYS_EVAL64, KEYS_TIMED_RAW = 0, 1, 2
 
 
 class PestoError(RuntimeError):
@@ -88,6 +89,7 @@ SIGNATURES = {
     "pesto_search_set_keys": (_I32, [_VP, _VP, _VP]),
     "pesto_search_commit": (_I32, [_VP, _VP]),
     "pesto_search_candidate_keys": (_I32, [_VP, _I32, _I64, _I64, _VP, _VP]),
+    "pesto_search_candidate_keys_ex": (_I32, [_VP, _I32, _I64, _I64, _VP, _I32, _VP]),
     "pesto_search_set_coarse_moves": (_I32, [_VP, _VP, _I32, _I32]),
     "pesto_search_get": (_I32, [_VP, _I32, _VP, _VP, _VP]),
     "pesto_search_step_count": (_I64, [_VP]),
@@ -362,11 +364,15 @@ class Search:
             raise ValueError("coarse_of must have one entry per op")
         _check(_L.pesto_search_set_coarse_moves(self._h, c.ctypes.data, int(n_coarse), int(pct)))
 
-    def candidate_keys(self, base: int, j0: int, j1: int, stream=None) -> np.ndarray:
+    def candidate_keys(self, base: int, j0: int, j1: int, stream=None,
+                       kernel: int = KEYS_TIMED) -> np.ndarray:
+        """Per-candidate keys of [j0, j1) (pesto_search_candidate_keys_ex): KEYS_TIMED = the
+        instantiation the step launches (exact), KEYS_EVAL64 = the independent 64-bit kernel,
+        KEYS_TIMED_RAW = the timed kernel's own output (saturated walks clamped)."""
         import torch
         out = torch.empty(max(1, j1 - j0), dtype=torch.int64, device=f"cuda:{self.graph.device}")
-        _check(_L.pesto_search_candidate_keys(self._h, base, j0, j1, out.data_ptr(),
-                                              _stream(stream)))
+        _check(_L.pesto_search_candidate_keys_ex(self._h, base, j0, j1, out.data_ptr(), kernel,
+                                                 _stream(stream)))
         torch.cuda.synchronize(self.graph.device)
         return out[:j1 - j0].cpu().numpy().view(np.uint64)
 

@@ -8,7 +8,13 @@ WANT = ['gpu__time_duration.sum', 'dram__bytes_read.sum', 'dram__bytes_write.sum
         'launch__registers_per_thread', 'launch__grid_size', 'launch__block_size',
         'sm__throughput.avg.pct_of_peak_sustained_elapsed',
         'dram__throughput.avg.pct_of_peak_sustained_elapsed',
-        'smsp__warps_active.avg.per_cycle_active']
+        'smsp__warps_active.avg.per_cycle_active', 'lts__t_bytes.sum',
+        'lts__t_sectors_srcunit_tex_op_read.sum', 'lts__t_sectors_srcunit_tex_op_write.sum',
+        'l1tex__t_bytes.sum', 'sm__cycles_active.avg', 'smsp__cycles_active.avg',
+        'sm__inst_executed_pipe_alu.avg.pct_of_peak_sustained_active',
+        'sm__inst_executed_pipe_lsu.avg.pct_of_peak_sustained_active',
+        'smsp__inst_executed_op_shared_ld.sum', 'smsp__inst_executed_op_shared_st.sum',
+        'smsp__inst_executed_op_global_red.sum', 'smsp__inst_executed_op_global_st.sum']
 STALLS = ['long_scoreboard', 'short_scoreboard', 'wait', 'mio_throttle', 'lg_throttle', 'barrier',
           'math_pipe_throttle', 'not_selected', 'selected', 'dispatch_stall', 'no_instruction',
           'branch_resolving', 'drain', 'membar', 'sleeping', 'tex_throttle', 'imc_miss']

@@ -22,6 +22,7 @@ def test_reference_arm_json_contract():
               "cpu_baseline", "e2e", "impl"):
         assert k in d, k
     assert d["impl"] == "reference" and d["value"] > 0 and d["higher_is_better"] is True
-    assert d["config"]["workload"] == "inception_v3_2dev"
+    assert d["config"]["workload"] == "transformer_2dev"
+    assert d["config"]["bases"] == 4 and d["ms_per_step"] > 0
     assert d["cpu_baseline"]["kind"] == "oracle" and d["cpu_baseline"]["cores"] >= 1
     assert d["e2e"]["h2d_bytes_per_step"] == 0 and d["e2e"]["value"] == d["value"]

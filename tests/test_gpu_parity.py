@@ -171,10 +171,8 @@ def test_full_size_sampled(P, O, name):
              G.seed_placement(P.PLACE_SINGLE)]
     x = np.concatenate([np.stack(seeds), dag.random_placements(g, 5, 4093)])
     gpu = _gpu_eval(P, G, g, order, x)
-    idx = np.concatenate([np.arange(3), np.random.default_rng(1).choice(np.arange(3, 4096), 45,
-                                                                         replace=False)])
-    ref, _ = O.makespan_batch(g, x[idx], order)
-    assert (gpu[idx] == ref).all()
+    ref, _ = O.makespan_batch(g, x, order, threads=os.cpu_count())
+    assert (gpu == ref).all(), np.nonzero(gpu != ref)[0][:5]  # all 4096 rows
     assert gpu[2] == int(g.p.sum())                           # single device = sum p
 
 
@@ -190,20 +188,36 @@ def _bases(g, P_, seed=0):
     return xs, orders
 
 
+SAT32 = np.uint64(0xF0000000)
+
+
+def _check_raw(P, raw, ok):
+    """the timed kernel's own keys: exact where its 32-bit walk did not saturate; a clamped walk
+    (makespan field 0xF0000000) must belong to a candidate whose exact makespan is >= the clamp"""
+    sat = (raw != np.uint64(P.KEY_INVALID)) & ((raw >> np.uint64(24)) >= SAT32)
+    assert (raw[~sat] == ok[~sat]).all(), np.nonzero((raw != ok) & ~sat)[0][:5]
+    assert ((ok[sat] >> np.uint64(24)) >= SAT32).all()
+    return int(sat.sum())
+
+
 @pytest.mark.parametrize("D,allowed_frac", [(2, 0.0), (4, 0.5)])
 def test_search_candidate_keys(P, O, D, allowed_frac):
+    """per-candidate keys of the timed eval32 instantiation, of its raw output and of the
+    independent 64-bit kernel, each equal to the oracle's decode + makespan"""
     g = _search_graph(D=D, allowed_frac=allowed_frac)
     G = P.Graph.from_arrays(g)
     xs, orders = _bases(g, 3)
     K = 1500
     S = P.Search(G, xs, orders, K, MIX, seed=99)
     for b in range(3):
-        gk = S.candidate_keys(b, 0, K)
         ok = O.candidate_keys(g, 3, b, xs, orders, 0, K, 99, 0, MIX)
-        assert (gk == ok).all(), (b, np.nonzero(gk != ok)[0][:5])
-    gk = S.candidate_keys(1, 77, 1013)                       # unaligned range
+        for kern in (P.KEYS_TIMED, P.KEYS_EVAL64):
+            gk = S.candidate_keys(b, 0, K, kernel=kern)
+            assert (gk == ok).all(), (kern, b, np.nonzero(gk != ok)[0][:5])
+        _check_raw(P, S.candidate_keys(b, 0, K, kernel=P.KEYS_TIMED_RAW), ok)
     ok = O.candidate_keys(g, 3, 1, xs, orders, 77, 1013, 99, 0, MIX)
-    assert (gk == ok).all()
+    for kern in (P.KEYS_TIMED, P.KEYS_EVAL64):               # unaligned range
+        assert (S.candidate_keys(1, 77, 1013, kernel=kern) == ok).all(), kern
 
 
 def test_search_steps_match_reference(P, O):
@@ -273,7 +287,13 @@ def test_multiwave_search_steps(P, O, D):
         S.eval()
         gkeys = S.keys()
         for b in range(2):
-            assert int(gkeys[b]) == int(S.candidate_keys(b, 0, K).min()), (step, b)
+            # every candidate of the step from the timed instantiation (CPL 2 here) vs the oracle
+            tk = S.candidate_keys(b, 0, K, kernel=P.KEYS_TIMED)
+            ok = O.candidate_keys(g, 2, b, rx, ro, 0, K, seed, step, mix, os.cpu_count())
+            assert (tk == ok).all(), (step, b, np.nonzero(tk != ok)[0][:5])
+            _check_raw(P, S.candidate_keys(b, 0, K, kernel=P.KEYS_TIMED_RAW), ok)
+            assert int(gkeys[b]) == int(tk.min()), (step, b)
+            assert int(gkeys[b]) == int(S.candidate_keys(b, 0, K, kernel=P.KEYS_EVAL64).min())
         keys = O.search_step(g, rx, ro, rmk, K, seed, step, mix)
         assert [int(k) for k in gkeys] == [int(k) for k in keys], step
         S.commit()
@@ -394,22 +414,43 @@ def test_nccl_allreduce_path_single_rank(P, O):
             assert a[0] == c[0] and (a[1] == c[1]).all() and (a[2] == c[2]).all()
 
 
-def test_search_full_size_sampled(P, O):
-    """transformer_2dev at full size: a sample of search candidates checked one by one."""
-    cfg = configs.CONFIGS["transformer_2dev"]
+def _full_size_ids(K):
+    """>= 4,096 candidate ids of one base: the first 2,048 (16 whole 128-id groups, group 0's
+    identity included) and 16 whole groups spread over [0, K) (swap groups among them)"""
+    spread = np.linspace(16, K // 128 - 1, 16).astype(np.int64)
+    return np.unique(np.concatenate([np.arange(2048)] +
+                                    [np.arange(128 * g, 128 * g + 128) for g in spread]))
+
+
+@pytest.mark.parametrize("name", ["inception_v3_2dev", "nmt4_2dev_commheavy",
+                                  "transformer_2dev", "transformer_4dev_8gpu"])
+def test_search_full_size_parity(P, O, name):
+    """every BASELINE config at full size, the bench's four seeds (nmt4 includes bases above the
+    32-bit saturation, walked by the wide instance), the full step's K per base: per-candidate
+    keys of the timed instantiation over all K ids of each base, the >= 4,096-id sample of each
+    base compared element by element with the oracle; the step's argmin equals their minimum"""
+    from workloads import seeds
+    cfg = configs.CONFIGS[name]
     g = configs.graph_for(cfg)
     G = P.Graph.from_arrays(g)
-    order = G.seed_order(P.ORDER_CRITICAL_PATH)
-    xs = np.stack([G.seed_placement(P.PLACE_EXPERT, layer=g.layer),
-                   G.seed_placement(P.PLACE_TOPO_SPLIT, order=order)])
-    orders = np.stack([order, order])
-    S = P.Search(G, xs, orders, 1 << 20, MIX, seed=2021)
-    for b in range(2):
-        sample = [0, 1, 31, 32, 33, 4097, 65535, 524287, (1 << 20) - 1]
-        for j in sample:
-            gk = S.candidate_keys(b, j, j + 1)
-            ok = O.candidate_keys(g, 2, b, xs, orders, j, j + 1, 2021, 0, MIX)
-            assert (gk == ok).all(), (b, j)
+    xs, orders = seeds.bench_seeds(g, cfg.bases, configs.SEARCH_SEED)
+    K = cfg.candidates_per_gpu // cfg.bases
+    S = P.Search(G, xs, orders, K, configs.MOVE_MIX, configs.SEARCH_SEED)
+    S.eval()
+    gkeys = S.keys()
+    ids = _full_size_ids(K)
+    for b in range(cfg.bases):
+        tk = S.candidate_keys(b, 0, K, kernel=P.KEYS_TIMED)
+        assert int(gkeys[b]) == int(tk.min()), b
+        ok = np.empty(len(ids), np.uint64)
+        for lo in range(0, len(ids), 128):                  # whole groups, contiguous ids
+            j0 = int(ids[lo])
+            ok[lo:lo + 128] = O.candidate_keys(g, cfg.bases, b, xs, orders, j0, j0 + 128,
+                                               configs.SEARCH_SEED, 0, configs.MOVE_MIX,
+                                               os.cpu_count())
+        assert (tk[ids] == ok).all(), (b, ids[np.nonzero(tk[ids] != ok)[0][:5]])
+        raw = S.candidate_keys(b, 0, K, kernel=P.KEYS_TIMED_RAW)
+        _check_raw(P, raw[ids], ok)
 
 
 # ---------------------------------------------------------------------------------------------

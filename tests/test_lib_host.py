@@ -200,3 +200,27 @@ def test_workspace_and_async_validation(P):
     assert P.lib().pesto_workspace_create(None, C.byref(h)) == P.EINVAL
     assert P.lib().pesto_eval_batch_host_async(None, None, None, 16, 1, None, None) == P.EINVAL
     P.lib().pesto_workspace_destroy(None)                      # NULL-safe
+
+
+@pytest.mark.parametrize("name", ["inception_v3_2dev", "nmt4_2dev_commheavy",
+                                  "transformer_4dev_8gpu", "random_masked"])
+def test_python_seeds_equal_library_seeds(P, name):
+    """workloads/seeds.py (the CPU reference arm's incumbents) restates libpesto's row-a1 seed
+    generators: every order and placement agrees op for op."""
+    from workloads import seeds
+    if name == "random_masked":
+        g = dag.random_dag(77, 500, 1.5, D=3, p_max=3000, max_bytes=10_000, beta0=100,
+                           beta1_fs=1000, allowed_frac=0.4)
+        g.layer = (np.arange(g.n) * 7) // g.n
+    else:
+        g = configs.graph_for(configs.CONFIGS[name])
+    G = _host_graph(P, g)
+    o_cp = G.seed_order(P.ORDER_CRITICAL_PATH)
+    assert (o_cp == seeds.order_critical_path(g)).all()
+    assert (G.seed_order(P.ORDER_FIFO) == seeds.order_fifo(g)).all()
+    assert (G.seed_order(P.ORDER_RANDOM, 2021) == seeds.order_random(g, 2021)).all()
+    assert (G.seed_placement(P.PLACE_SINGLE) == seeds.place_single(g)).all()
+    assert (G.seed_placement(P.PLACE_EXPERT, layer=g.layer) == seeds.place_expert(g, g.layer)).all()
+    assert (G.seed_placement(P.PLACE_TOPO_SPLIT, order=o_cp) ==
+            seeds.place_topo_split(g, o_cp)).all()
+    assert (G.seed_placement(P.PLACE_RANDOM, seed=2021) == seeds.place_random(g, 2021)).all()

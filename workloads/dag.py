@@ -266,3 +266,27 @@ def pack_placements(x: np.ndarray, D: int, row_stride: Optional[int] = None) -> 
             # each byte index appears once for a fixed bit index i, so fancy-index OR is exact
             out[:, byte_idx[sel]] |= contrib
     return out
+
+
+def random_packed_rows(g: Graph, seed: int, count: int, chunk: int = 65536) -> np.ndarray:
+    """[count, stride] packed rows (the `pesto_eval_batch` format of `pack_placements`) of
+    placements uniform over all device codes, drawn directly as random bits so that 1M-row
+    batches need no [count, n] intermediate.  For graphs whose every op allows all devices and
+    D a power of two (every code < D) this is the distribution of `random_placements`."""
+    if g.allowed is not None and (np.asarray(g.allowed) != (1 << g.D) - 1).any():
+        raise ValueError("random_packed_rows needs all-allowed masks")
+    if g.D & (g.D - 1):
+        raise ValueError("random_packed_rows needs D a power of two")
+    b = 1 if g.D <= 2 else (2 if g.D <= 4 else 4)
+    nbits = g.n * b
+    stride = ((nbits + 7) // 8 + 15) // 16 * 16
+    out = np.empty((count, stride), dtype=np.uint8)
+    rng = np.random.default_rng(seed)
+    tail = np.zeros(stride, dtype=np.uint8)              # keep only the row's nbits
+    tail[: nbits // 8] = 0xFF
+    if nbits % 8:
+        tail[nbits // 8] = (1 << (nbits % 8)) - 1
+    for a in range(0, count, chunk):
+        e = min(count, a + chunk)
+        out[a:e] = rng.integers(0, 256, size=(e - a, stride), dtype=np.uint8) & tail
+    return out
