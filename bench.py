@@ -313,6 +313,14 @@ def run_pesto(args, rank, world, local):
     value = total_cands / (tot_ms / 1e3)
     best_mk = [S.get(b)[0] for b in range(n_bases)]
     swap_stats = S.swap_stats()
+    # the neighbourhood the next step evaluates (DESIGN §4 v6): distinct (placement, order)
+    # pairs among this rank's candidates, decoded on the host by the kernels' spec code
+    ms = [S.move_stats(b, k_per_base * rank // world, k_per_base * (rank + 1) // world)
+          for b in range(n_bases)]
+    tot = {k: sum(m[k] for m in ms) for k in ms[0]}
+    move_stats = dict(tot, step=S.step_count,
+                      distinct_fraction=tot["distinct"] / tot["candidates"],
+                      duplicate_fraction=1.0 - (tot["distinct"] + tot["invalid"]) / tot["candidates"])
 
     # ---- end to end through the public API with host buffers ----
     # every step copies its batch of explicit placement rows in from pinned host memory,
@@ -439,6 +447,7 @@ def run_pesto(args, rank, world, local):
                           k1_frac_of_measured_int_roof=achieved * 1e12 / roofs["int_ops_per_s"]),
             "gpu_launches": int(launches),
             "wall_s_timed_region": wall,
+            "candidates": move_stats,
             "search": {"seed_makespans": seed_mk, "best_makespans": best_mk,
                        "swaps_patched_in_place": swap_stats[0], "swaps_rebuilt": swap_stats[1]},
             "e2e": e2e}

@@ -291,6 +291,17 @@ pesto_status pesto_search_candidate_keys(pesto_search *s, int32_t base, int64_t 
 pesto_status pesto_search_set_coarse_moves(pesto_search *s, const int32_t *coarse_of,
                                           int32_t n_coarse, int32_t pct);
 
+/* Neighbourhood statistics of candidates j in [j0, j1) of `base` at the current step, decoded
+ * on the host by the same spec code the kernels use: how many are invalid, how
+ * many valid ones are identical to the base (no placement change, no order move; j = 0
+ * included) and how many distinct (placement, order) pairs the valid ones form.  Synchronises.
+ * Errors: EINVAL. */
+typedef struct {
+    int64_t candidates, invalid, identical_to_base, distinct;
+} pesto_move_stats;
+pesto_status pesto_search_move_stats(pesto_search *s, int32_t base, int64_t j0, int64_t j1,
+                                     pesto_move_stats *out);
+
 /* Current incumbent of `base` (synchronises): makespan, x (host [n_ops]) and order. */
 pesto_status pesto_search_get(pesto_search *s, int32_t base, int64_t *makespan,
                               uint8_t *x_host, int32_t *order_host);

@@ -752,19 +752,23 @@ int oracle_candidate(int32_t n, int64_t m, const int32_t *src, const int32_t *ds
         return 1;
     }
     int swap = 0;
-    /* the group's region: positions [c, c + len) of the base order (DESIGN §4 S2) */
-    int64_t c0 = (int64_t)(oracle_draw(seed, step, P, b, 128 * g, 13) % (uint64_t)n);
+    /* S2 (v6): the regions tile the base order, R = ceil(n/64), rotated by o = draw(0, 13)
+       mod R; group g takes region (g + o) mod R = positions [c, c + len), in pass g / R */
+    int64_t R = ((int64_t)n + 63) / 64;
+    int64_t rot = (int64_t)(oracle_draw(seed, step, P, b, 0, 13) % (uint64_t)R);
+    int64_t c0 = 64 * ((g + rot) % R);
     int64_t rlen = n - c0 < 64 ? n - c0 : 64;
-    /* order move: one adjacent swap per group (DESIGN §4 S3) */
+    int64_t pass = g / R;
+    /* S3: order move, one adjacent swap per group */
     if (g != 0 && mix[3] > 0 && n >= 2) {
         uint64_t u = oracle_draw(seed, step, P, b, 128 * g, 15);
         if ((int64_t)(u % 100u) < mix[3]) {
             int64_t k = c0 + (int64_t)(oracle_draw(seed, step, P, b, 128 * g, 14) % (uint64_t)rlen);
             if (k > n - 2) k = n - 2;
             int32_t a = bo[k], c = bo[k + 1];
-            /* blocked (S3): an edge joins them, they share a producer or a consumer, or
-               either has more than 64 successors */
-            int joined = 0;
+            /* blocked: an edge joins them, they share a producer or a consumer, either has more
+               than 64 out-edges, or their base devices differ */
+            int joined = bx[a] != bx[c];
             int64_t out_a = 0, out_c = 0;
             for (int64_t e = 0; e < m; e++) {
                 if ((src[e] == a && dst[e] == c) || (src[e] == c && dst[e] == a)) joined = 1;
@@ -789,27 +793,55 @@ int oracle_candidate(int32_t n, int64_t m, const int32_t *src, const int32_t *ds
             }
         }
     }
+    /* S4: placement move */
     if (j == 0 || (swap && lane == 0)) return 1;
     int32_t wsum = mix[0] + mix[1] + mix[2];
     if (wsum <= 0) return 1;
+    int64_t b1 = (128 * (int64_t)mix[0]) / wsum, b2 = (128 * (int64_t)(mix[0] + mix[1])) / wsum;
     int32_t alts[8];
-    int64_t r = (int64_t)(oracle_draw(seed, step, P, b, j, 0) % (uint64_t)wsum);
-    if (r < mix[0] + mix[1]) {                               /* FLIP1 or FLIPk (S4) */
-        int32_t flips = 1;
-        if (r >= mix[0]) flips = 2 + (int32_t)(oracle_draw(seed, step, P, b, j, 1) % 3u);
-        for (int32_t q = 0; q < flips; q++) {
-            int64_t pos = c0 + (int64_t)(oracle_draw(seed, step, P, b, j, 2 + 2 * q) % (uint64_t)rlen);
-            int32_t v = bo[pos];
-            unsigned msk = allowed ? (unsigned)allowed[v] : 0xFFu;
-            if (popcount8(msk & ((1u << D) - 1u)) < 2) return 0;   /* op cannot move: invalid */
-            int32_t na = alt_devices(allowed, D, v, x_out[v], alts);
-            x_out[v] = (uint8_t)alts[oracle_draw(seed, step, P, b, j, 3 + 2 * q) % (uint64_t)na];
+    if (lane < b1) {                                         /* FLIP1: enumerated */
+        int64_t t = pass * b1 + lane;
+        if (t < rlen * (D - 1)) {
+            int64_t q = c0 + t % rlen, a = t / rlen;
+            int32_t v = bo[q];
+            int32_t na = alt_devices(allowed, D, v, bx[v], alts);
+            if (a >= na) return 0;                           /* no such alternative: invalid */
+            x_out[v] = (uint8_t)alts[a];
+            return 1;
         }
-    } else {                                                 /* WINDOW (S4) */
-        int64_t s = c0 + (int64_t)(oracle_draw(seed, step, P, b, j, 2) % (uint64_t)rlen);
-        int64_t len = 1 + (int64_t)(oracle_draw(seed, step, P, b, j, 3) % 64u);
-        int32_t d = (int32_t)(oracle_draw(seed, step, P, b, j, 4) % (uint64_t)D);
-        for (int64_t q = s; q < s + len && q < c0 + rlen; q++) {
+        /* the region's single-op moves are used up: a FLIPk lane */
+    }
+    if (lane < b2) {                                         /* FLIPk: distinct positions */
+        int64_t f = 2 + (int64_t)(oracle_draw(seed, step, P, b, j, 1) % 3u);
+        if (f > rlen) f = rlen;
+        int64_t taken[4];
+        for (int64_t i = 0; i < f; i++) {
+            int64_t r = (int64_t)(oracle_draw(seed, step, P, b, j, 2 + 2 * i) % (uint64_t)(rlen - i));
+            int64_t q = -1;                                  /* r-th free position, ascending */
+            for (int64_t cand = c0; cand < c0 + rlen; cand++) {
+                int used = 0;
+                for (int64_t u = 0; u < i; u++) used |= taken[u] == cand;
+                if (used) continue;
+                if (r == 0) { q = cand; break; }
+                r--;
+            }
+            taken[i] = q;
+            int32_t v = bo[q];
+            int32_t na = alt_devices(allowed, D, v, bx[v], alts);
+            if (na == 0) return 0;                           /* op cannot move: invalid */
+            x_out[v] = (uint8_t)alts[oracle_draw(seed, step, P, b, j, 3 + 2 * i) % (uint64_t)na];
+        }
+        return 1;
+    }
+    {                                                        /* WINDOW: enumerated starts */
+        int64_t i = lane - b2, nw = 128 - b2;
+        int64_t s = c0 + (pass * nw + i) % rlen;
+        int64_t e = s + 1 + (int64_t)(oracle_draw(seed, step, P, b, j, 3) % 64u);
+        if (e > c0 + rlen) e = c0 + rlen;
+        int32_t na = alt_devices(allowed, D, bo[s], bx[bo[s]], alts);
+        if (na == 0) return 0;
+        int32_t d = alts[oracle_draw(seed, step, P, b, j, 4) % (uint64_t)na];
+        for (int64_t q = s; q < e; q++) {
             int32_t v = bo[q];
             if (allowed_dev(allowed, v, d)) x_out[v] = (uint8_t)d;
         }

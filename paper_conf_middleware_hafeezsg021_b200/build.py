@@ -42,22 +42,26 @@ def build(force: bool = False, verbose: bool = False) -> str:
     if not force and not _stale():
         return OUT
     os.makedirs(BUILD, exist_ok=True)
-    objs = []
+    jobs = []
     for f in CU_SOURCES:
         o = os.path.join(BUILD, f + ".o")
-        extra = []
-        cmd = [NVCC, *ARCH, "-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC", *extra,
+        cmd = [NVCC, *ARCH, "-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC",
                "-Xptxas", "-v" if verbose else "-O3", "-I", INC, "-I", CSRC, "-c",
                os.path.join(CSRC, f), "-o", o]
-        r = _run(cmd)
-        if verbose:
-            sys.stderr.write(r.stderr)
-        objs.append(o)
+        jobs.append((cmd, o))
     for f in CPP_SOURCES:
         o = os.path.join(BUILD, f + ".o")
-        _run(["g++", "-O2", "-std=c++17", "-fPIC", "-Wall", "-I", os.path.join(CUDA, "include"),
-              "-I", INC, "-I", CSRC, "-c", os.path.join(CSRC, f), "-o", o])
-        objs.append(o)
+        jobs.append((["g++", "-O2", "-std=c++17", "-fPIC", "-Wall", "-I",
+                      os.path.join(CUDA, "include"), "-I", INC, "-I", CSRC, "-c",
+                      os.path.join(CSRC, f), "-o", o], o))
+    # the translation units are independent: compile them concurrently
+    from concurrent.futures import ThreadPoolExecutor
+    with ThreadPoolExecutor(max_workers=min(len(jobs), os.cpu_count() or 1)) as ex:
+        results = list(ex.map(lambda jc: _run(jc[0]), jobs))
+    if verbose:
+        for r in results:
+            sys.stderr.write(r.stderr)
+    objs = [o for _, o in jobs]
     tmp = OUT + ".tmp"
     _run([NVCC, *ARCH, "-shared", "-cudart", "static", "-o", tmp, *objs, "-ldl", "-lpthread",
           "-lrt"])

@@ -619,15 +619,16 @@ eval32_kernel(const EvalParams P) {
                 place.rlen = rg.len;
             }
             const uint8_t *blocked = B->swap_blocked;
-            ks = active && !coarse
-                     ? decode_swap(P.seed, cb, grp, P.n, P.mix[3], rg,
-                                   [&](int32_t k) { return __ldg(blocked + k) != 0; })
-                     : -1;
-            if (ks >= 0) off_ks = __ldg(B->op_off32 + ks);
             const int32_t *ord = B->order;
             const uint32_t *bits = B->bits;
             const uint8_t *aop = P.allowed_op;
             const int words = P.words;
+            ks = active && !coarse
+                     ? decode_swap(P.seed, cb, grp, P.n, P.mix[3], rg,
+                                   [&](int32_t k) { return __ldg(blocked + k) != 0; },
+                                   [&](int32_t q) { return ldg_bits_dev_at<PL>(bits, words, q); })
+                     : -1;
+            if (ks >= 0) off_ks = __ldg(B->op_off32 + ks);
             if (!coarse) {
 #pragma unroll
                 for (int c = 0; c < CPL; c++) {

@@ -330,15 +330,16 @@ eval_kernel(const EvalParams P) {
             place.bits = B->bits;
             place.allowed_pos = B->allowed_pos;
             const uint8_t *adj = B->swap_blocked;
-            ks = active && !place.coarse
-                     ? decode_swap(P.seed, cb, grp, P.n, P.mix[3], rg,
-                                   [&](int32_t k) { return __ldg(adj + k) != 0; })
-                     : -1;
-            const bool in_range = active && j >= P.j_begin && j < P.j_end;
             const int32_t *ord = B->order;
             const uint32_t *bits = B->bits;
             const uint8_t *aop = P.allowed_op;
             const int words = P.words;
+            ks = active && !place.coarse
+                     ? decode_swap(P.seed, cb, grp, P.n, P.mix[3], rg,
+                                   [&](int32_t k) { return __ldg(adj + k) != 0; },
+                                   [&](int32_t q) { return ldg_bits_dev_at<PL>(bits, words, q); })
+                     : -1;
+            const bool in_range = active && j >= P.j_begin && j < P.j_end;
             if (place.coarse)
                 place.mv = decode_coarse_lane(P.seed, cb, j, P.n_coarse, P.D);
             else place.mv = in_range
@@ -639,7 +640,8 @@ __global__ void commit_kernel(const CommitParams P) {
     const bool coarse = coarse_group(P.seed, cb, j >> kGroupShift, P.coarse_pct, P.n_coarse);
     const int32_t ks = j == 0 || coarse ? -1
                               : decode_swap(P.seed, cb, j >> kGroupShift, P.n, P.mix[3], rg,
-                                            [&](int32_t k) { return adj[k] != 0; });
+                                            [&](int32_t k) { return adj[k] != 0; },
+                                            [&](int32_t q) { return get_dev_at<PL>(bits, P.words, q); });
     const int words = P.words;
     const LaneMove mv = j == 0 ? no_move()
         : coarse ? decode_coarse_lane(P.seed, cb, j, P.n_coarse, P.D)

@@ -53,33 +53,50 @@ constexpr int kRegion = 64;     // positions a group of candidates may change (D
 constexpr int kGroupShift = 7;  // a group = 128 consecutive candidate ids
 constexpr int kGroup = 1 << kGroupShift;
 
-// The group's region [c, c + len) of the base order.
+// The group's region [c, c + len) of the base order and its pass over the regions.
 struct Region {
-    int32_t c, len;
+    int32_t c, len, pass;
 };
+// S2 (v6): the regions tile the order (R = ceil(n/64)); group g takes region (g + o) mod R with
+// the per-(step, base) rotation o = draw(0, 13) mod R, in pass g / R
 PESTO_HD Region decode_region(uint64_t seed, uint64_t cb, int64_t group, int n) {
+    const int64_t R = ((int64_t)n + kRegion - 1) / kRegion;
+    const int64_t rot = (int64_t)(draw(seed, cb, 0, 13) % (uint64_t)R);
     Region r;
-    r.c = (int32_t)(draw(seed, cb, group * kGroup, 13) % (uint64_t)n);
+    r.c = (int32_t)(kRegion * ((group + rot) % R));
     r.len = n - r.c < kRegion ? n - r.c : kRegion;
+    r.pass = (int32_t)(group / R);
     return r;
 }
 
-// Group order move: adjacent swap of positions (k, k+1) of the base order, or -1.
-// blocked(k) says whether (k, k+1) may not be swapped: an edge joins them, they share a
-// producer or a consumer, or either has more than kSwapMaxOut successors (DESIGN §4 S3).
+// Group order move (S3): adjacent swap of positions (k, k+1) of the base order, or -1.
+// blocked(k) says whether (k, k+1) may not be swapped for structural reasons (an edge joins
+// them, they share a producer or a consumer, or either has more than kSwapMaxOut out-edges);
+// base_dev(q) is the base device at q -- a pair on different devices is blocked too (v6).
 constexpr int kSwapMaxOut = 64;
-template <class Blocked>
+template <class Blocked, class BaseDev>
 PESTO_HD int32_t decode_swap(uint64_t seed, uint64_t cb, int64_t group, int n, int swap_pct,
-                             Region rg, Blocked blocked) {
+                             Region rg, Blocked blocked, BaseDev base_dev) {
     if (group == 0 || swap_pct <= 0 || n < 2) return -1;
     int64_t j0 = group * kGroup;
     if ((int)(draw(seed, cb, j0, 15) % 100u) >= swap_pct) return -1;
     int32_t k = rg.c + (int32_t)(draw(seed, cb, j0, 14) % (uint64_t)rg.len);
     if (k > n - 2) k = n - 2;
-    return blocked(k) ? -1 : k;
+    return (blocked(k) || base_dev(k) != base_dev(k + 1)) ? -1 : k;
 }
 
-// Lane placement move of candidate j inside region rg.  Callbacks:
+// the a-th (0-based, ascending) device of mask msk, or -1
+PESTO_HD int nth_device(unsigned msk, int a, int D) {
+    for (int d = 0; d < D; d++) {
+        if ((msk >> d) & 1u) {
+            if (a == 0) return d;
+            a--;
+        }
+    }
+    return -1;
+}
+
+// Lane placement move of candidate j inside region rg (S4, v6).  Callbacks:
 //   op_at(pos) -> op id at a position of the base order;  base_dev(pos) -> base device there;
 //   allowed(op) -> device mask.
 template <class OpAt, class BaseDev, class Allowed>
@@ -92,44 +109,65 @@ PESTO_HD LaneMove decode_lane(uint64_t seed, uint64_t cb, int64_t j, bool pure_s
     mv.ws = 0; mv.wl = 0; mv.wd = 0;
     for (int q = 0; q < 4; q++) { mv.fpos[q] = -1; mv.fdev[q] = 0; }
     if (j == 0 || pure_swap) return mv;
-    int wsum = mix[0] + mix[1] + mix[2];
+    const int wsum = mix[0] + mix[1] + mix[2];
     if (wsum <= 0) return mv;
-    int r = (int)(draw(seed, cb, j, 0) % (uint64_t)wsum);
-    if (r < mix[0] + mix[1]) {
-        int flips = 1;
-        if (r >= mix[0]) flips = 2 + (int)(draw(seed, cb, j, 1) % 3u);
-        mv.kind = kMoveFlip;
-        mv.nflip = flips;
-        for (int q = 0; q < flips; q++) {
-            int32_t pos = rg.c + (int32_t)(draw(seed, cb, j, 2 + 2 * q) % (uint64_t)rg.len);
-            int32_t op = op_at(pos);
-            const unsigned am = allowed(op) & ((1u << D) - 1u);
-            if (popc32(am) < 2) { mv.kind = kMoveInvalid; return mv; }   // op cannot move
-            int cur = base_dev(pos);
-            for (int e = 0; e < q; e++)
-                if (mv.fpos[e] == pos) cur = mv.fdev[e];      // device after earlier flips
-            unsigned msk = am & ~(1u << cur);
-            int na = popc32(msk);
-            int pick = (int)(draw(seed, cb, j, 3 + 2 * q) % (uint64_t)na);
-            int dev = 0;
-            for (int d = 0; d < D; d++) {                      // pick-th set bit, ascending
-                if ((msk >> d) & 1u) {
-                    if (pick == 0) { dev = d; break; }
-                    pick--;
-                }
-            }
-            mv.fpos[q] = pos;
-            mv.fdev[q] = dev;
+    const int lane = (int)(j & (kGroup - 1));
+    const int b1 = (kGroup * mix[0]) / wsum, b2 = (kGroup * (mix[0] + mix[1])) / wsum;
+    const unsigned dmask = (1u << D) - 1u;
+    // A_q: allowed devices of the op at q without its base device
+    auto alts = [&](int32_t q) { return allowed(op_at(q)) & dmask & ~(1u << base_dev(q)); };
+    if (lane < b1) {                                   // FLIP1: enumerated single-op moves
+        const int64_t t = (int64_t)rg.pass * b1 + lane;
+        if (t < (int64_t)rg.len * (D - 1)) {
+            const int32_t q = rg.c + (int32_t)(t % rg.len);
+            const int a = (int)(t / rg.len);
+            const unsigned am = alts(q);
+            if (a >= popc32(am)) { mv.kind = kMoveInvalid; return mv; }
+            mv.kind = kMoveFlip;
+            mv.nflip = 1;
+            mv.fpos[0] = q;
+            mv.fdev[0] = nth_device(am, a, D);
+            return mv;
         }
-    } else {
-        mv.kind = kMoveWindow;
-        int32_t s = rg.c + (int32_t)(draw(seed, cb, j, 2) % (uint64_t)rg.len);
-        int32_t len = 1 + (int32_t)(draw(seed, cb, j, 3) % 64u);
-        if (s + len > rg.c + rg.len) len = rg.c + rg.len - s;
-        mv.ws = s;
-        mv.wl = len;
-        mv.wd = (int32_t)(draw(seed, cb, j, 4) % (uint64_t)D);
+        // the region's single-op moves are used up: a FLIPk lane
     }
+    if (lane < b2) {                                   // FLIPk (or a used-up FLIP1 lane)
+        int f = 2 + (int)(draw(seed, cb, j, 1) % 3u);
+        if (f > rg.len) f = rg.len;
+        mv.kind = kMoveFlip;
+        mv.nflip = f;
+        for (int i = 0; i < f; i++) {
+            int r = (int)(draw(seed, cb, j, 2 + 2 * i) % (uint64_t)(rg.len - i));
+            // the r-th free offset of the region: the least fixed point of
+            // off = r + #{taken offsets <= off} (at most i <= 3 increases)
+            int32_t off = r;
+            for (int it = 0; it < 4; it++) {
+                int32_t cnt = 0;
+                for (int e = 0; e < i; e++) cnt += (mv.fpos[e] - rg.c) <= off ? 1 : 0;
+                if (r + cnt == off) break;
+                off = r + cnt;
+            }
+            const int32_t q = rg.c + off;
+            const unsigned am = alts(q);
+            const int na = popc32(am);
+            if (na == 0) { mv.kind = kMoveInvalid; return mv; }
+            mv.fpos[i] = q;
+            mv.fdev[i] = nth_device(am, (int)(draw(seed, cb, j, 3 + 2 * i) % (uint64_t)na), D);
+        }
+        return mv;
+    }
+    // WINDOW: enumerated starts; the op at s always changes
+    const int i = lane - b2, nw = kGroup - b2;
+    const int32_t s = rg.c + (int32_t)(((int64_t)rg.pass * nw + i) % rg.len);
+    int32_t len = 1 + (int32_t)(draw(seed, cb, j, 3) % 64u);
+    if (s + len > rg.c + rg.len) len = rg.c + rg.len - s;
+    const unsigned am = alts(s);
+    const int na = popc32(am);
+    if (na == 0) { mv.kind = kMoveInvalid; return mv; }
+    mv.kind = kMoveWindow;
+    mv.ws = s;
+    mv.wl = len;
+    mv.wd = nth_device(am, (int)(draw(seed, cb, j, 4) % (uint64_t)na), D);
     return mv;
 }
 

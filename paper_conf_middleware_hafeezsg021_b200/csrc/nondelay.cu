@@ -154,10 +154,11 @@ __global__ void __launch_bounds__(kNdMaxWarps * 32, 3) nondelay_kernel(const NdP
             const bool coarse = coarse_group(P.seed, cb, grp, P.coarse_pct, P.n_coarse);   // S9
             Region rg = decode_region(P.seed, cb, grp, n);
             const uint8_t *adj = B->swap_blocked;
+            const uint32_t *bits = B->bits;
             ks = coarse ? -1
                         : decode_swap(P.seed, cb, grp, n, P.mix[3], rg,
-                                      [&](int32_t k) { return __ldg(adj + k) != 0; });
-            const uint32_t *bits = B->bits;
+                                      [&](int32_t k) { return __ldg(adj + k) != 0; },
+                                      [&](int32_t q) { return ldg_bits_dev_at<PL>(bits, words, q); });
             const uint8_t *aop = P.allowed_op;
             LaneMove mv = coarse ? decode_coarse_lane(P.seed, cb, j, P.n_coarse, D) : decode_lane(P.seed, cb, j, ks >= 0 && (j & (kGroup - 1)) == 0, D, P.mix,
                                       rg, [&](int32_t q) { return __ldg(order + q); },
@@ -165,7 +166,7 @@ __global__ void __launch_bounds__(kNdMaxWarps * 32, 3) nondelay_kernel(const NdP
                                       [&](int32_t op) { return (unsigned)__ldg(aop + op); });
             valid = mv.kind != kMoveInvalid;
             if (!valid) mv = no_move();
-            if (coarse) rg = Region{0, n};                        // any op may move
+            if (coarse) rg = Region{0, n, 0};                        // any op may move
             if (valid && (P.feas.has_cap || P.feas.has_coloc))    // row f3
                 valid = move_feasible<PL>(mv, rg, D, bits, words, order, B->allowed_pos,
                                           P.all_allowed, P.feas, P.feas.fbase + (size_t)bl * 8);

@@ -858,6 +858,77 @@ pesto_status pesto_search_candidate_keys(pesto_search *s, int32_t base, int64_t 
     return pesto_search_candidate_keys_ex(s, base, j0, j1, keys_out, PESTO_KEYS_TIMED, stream);
 }
 
+pesto_status pesto_search_move_stats(pesto_search *s, int32_t base, int64_t j0, int64_t j1,
+                                     pesto_move_stats *out) {
+    if (!s || !out) return fail(PESTO_EINVAL, "NULL argument");
+    if (base < 0 || base >= s->P) return fail(PESTO_EINVAL, "base out of range");
+    if (j0 < 0 || j1 < j0 || j1 > s->K) return fail(PESTO_EINVAL, "candidate range out of [0, K]");
+    pesto_graph *g = s->g;
+    DeviceGuard guard(g->device);
+    cudaError_t e = s->last_stream ? cudaStreamSynchronize(s->last_stream) : cudaDeviceSynchronize();
+    if (e != cudaSuccess) return cuda_fail(e, "synchronise");
+    const int32_t n = g->n;
+    std::vector<uint8_t> x_op(n), xq(n);
+    pesto_status rc = download_x(s, base, x_op.data());
+    if (rc) return rc;
+    const std::vector<int32_t> &ord = s->order[base];
+    for (int32_t q = 0; q < n; q++) xq[q] = x_op[ord[q]];
+    const std::vector<uint8_t> &blocked = s->layouts[base]->swap_blocked;
+    const uint64_t cb = ctr_base_of((uint64_t)s->step, s->P, base);
+    // a candidate's signature: its order move and every (position, new device) that differs
+    // from the base, hashed; equal signatures = identical (placement, order) pairs
+    std::vector<uint64_t> sig;
+    sig.reserve((size_t)(j1 - j0));
+    pesto_move_stats st{};
+    for (int64_t j = j0; j < j1; j++) {
+        const int64_t grp = j >> kGroupShift;
+        const bool coarse = coarse_group(s->seed, cb, grp, s->coarse_pct, s->n_coarse);
+        const Region rg = decode_region(s->seed, cb, grp, n);
+        const int32_t ks = coarse ? -1
+            : decode_swap(s->seed, cb, grp, n, s->mix[3], rg,
+                          [&](int32_t k) { return blocked[k] != 0; },
+                          [&](int32_t q) { return (int)xq[q]; });
+        const LaneMove mv = j == 0 ? LaneMove{kMoveNone, 0, {-1, -1, -1, -1}, {0, 0, 0, 0}, 0, 0, 0}
+            : coarse ? decode_coarse_lane(s->seed, cb, j, s->n_coarse, g->D)
+            : decode_lane(s->seed, cb, j, ks >= 0 && (j & (kGroup - 1)) == 0, g->D, s->mix, rg,
+                          [&](int32_t q) { return ord[q]; }, [&](int32_t q) { return (int)xq[q]; },
+                          [&](int32_t op) { return (unsigned)g->allowed[op]; });
+        st.candidates++;
+        if (mv.kind == kMoveInvalid) { st.invalid++; continue; }
+        uint64_t h = mix64(0x5045535430ull + (uint64_t)(ks + 1));
+        int changed = 0;
+        auto add = [&](int32_t q, int d) {
+            if (d == (int)xq[q]) return;
+            h = mix64(h ^ mix64(((uint64_t)q << 8) | (uint64_t)d));
+            changed++;
+        };
+        if (mv.kind == kMoveFlip) {
+            int32_t qs[4];
+            int m = 0;
+            for (int f = 0; f < mv.nflip; f++) {           // a later flip of a position wins
+                bool last = true;
+                for (int f2 = f + 1; f2 < mv.nflip; f2++) last = last && mv.fpos[f2] != mv.fpos[f];
+                if (last) qs[m++] = f;
+            }
+            for (int a = 1; a < m; a++)                      // ascending position
+                for (int b = a; b > 0 && mv.fpos[qs[b]] < mv.fpos[qs[b - 1]]; b--) std::swap(qs[b], qs[b - 1]);
+            for (int i = 0; i < m; i++) add(mv.fpos[qs[i]], mv.fdev[qs[i]]);
+        } else if (mv.kind == kMoveWindow) {
+            for (int32_t q = mv.ws; q < mv.ws + mv.wl; q++)
+                if ((g->allowed[ord[q]] >> mv.wd) & 1) add(q, mv.wd);
+        } else if (mv.kind == kMoveCoarse) {
+            for (int32_t q = 0; q < n; q++)
+                if (s->coarse_of[ord[q]] == mv.ws && ((g->allowed[ord[q]] >> mv.wd) & 1)) add(q, mv.wd);
+        }
+        if (changed == 0 && ks < 0) st.identical_to_base++;
+        sig.push_back(h);
+    }
+    std::sort(sig.begin(), sig.end());
+    st.distinct = (int64_t)(std::unique(sig.begin(), sig.end()) - sig.begin());
+    *out = st;
+    return PESTO_OK;
+}
+
 pesto_status pesto_search_get(pesto_search *s, int32_t base, int64_t *mk, uint8_t *x_host,
                               int32_t *order_host) {
     if (!s) return fail(PESTO_EINVAL, "NULL search");

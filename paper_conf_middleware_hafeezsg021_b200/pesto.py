@@ -56,6 +56,11 @@ class Roofs(C.Structure):
                 ("l2_buffer_bytes", C.c_int64), ("hbm_copy_gbs", C.c_double)]
 
 
+class MoveStats(C.Structure):
+    _fields_ = [("candidates", C.c_int64), ("invalid", C.c_int64),
+                ("identical_to_base", C.c_int64), ("distinct", C.c_int64)]
+
+
 class SearchDesc(C.Structure):
     _fields_ = [("n_bases", C.c_int32), ("base_x", C.c_void_p), ("base_order", C.c_void_p),
                 ("k_per_base", C.c_int64), ("mix", C.c_int32 * 4), ("seed", C.c_uint64),
@@ -91,6 +96,7 @@ SIGNATURES = {
     "pesto_search_candidate_keys": (_I32, [_VP, _I32, _I64, _I64, _VP, _VP]),
     "pesto_search_candidate_keys_ex": (_I32, [_VP, _I32, _I64, _I64, _VP, _I32, _VP]),
     "pesto_search_set_coarse_moves": (_I32, [_VP, _VP, _I32, _I32]),
+    "pesto_search_move_stats": (_I32, [_VP, _I32, _I64, _I64, _VP]),
     "pesto_search_get": (_I32, [_VP, _I32, _VP, _VP, _VP]),
     "pesto_search_step_count": (_I64, [_VP]),
     "pesto_search_swap_stats": (_I32, [_VP, _VP, _VP]),
@@ -375,6 +381,14 @@ class Search:
                                                  _stream(stream)))
         torch.cuda.synchronize(self.graph.device)
         return out[:j1 - j0].cpu().numpy().view(np.uint64)
+
+    def move_stats(self, base: int, j0: int = 0, j1: int = None) -> dict:
+        """Distinct / identical / invalid counts of the step's candidates [j0, j1) of `base`
+        (pesto_search_move_stats)."""
+        st = MoveStats()
+        _check(_L.pesto_search_move_stats(self._h, base, j0, self.K if j1 is None else j1,
+                                          C.byref(st)))
+        return {f: getattr(st, f) for f, _ in MoveStats._fields_}
 
     def get(self, base: int):
         mk = C.c_int64()

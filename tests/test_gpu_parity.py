@@ -577,3 +577,41 @@ def test_roofs_microbenchmarks(P):
     assert 1e3 < r["l2_read_gbs"] < 1e5 and 1e3 < r["l2_rmw_gbs"] < 1e5
     assert 1e3 < r["hbm_copy_gbs"] < 1e4
     assert r["l2_buffer_bytes"] > 0
+
+
+@pytest.mark.parametrize("D,allowed_frac,mix", [(2, 0.0, (50, 20, 20, 10)),
+                                                 (3, 0.4, (40, 20, 20, 40))])
+def test_move_stats_count_distinct_candidates(P, O, D, allowed_frac, mix):
+    """pesto_search_move_stats (host decode by the product's spec code) counts the same
+    invalid / identical-to-base / distinct (placement, order) candidates as the oracle's decode,
+    over several passes of the region tiling (n = 300: 5 regions, K = 2048: 16 groups)"""
+    g = dag.random_dag(140 + D, 300, 1.5, D=D, p_max=3000, max_bytes=100_000, beta0=500,
+                       beta1_fs=25_000, allowed_frac=allowed_frac)
+    G = P.Graph.from_arrays(g)
+    xs, orders = _bases(g, 2, seed=3)
+    K = 2048
+    S = P.Search(G, xs, orders, K, mix, seed=31)
+    for step in range(2):
+        for b in range(2):
+            st = S.move_stats(b)
+            seen, inval, ident = set(), 0, 0
+            cur_x, cur_o = _cur(S)
+            for j in range(K):
+                ok, x, o = O.candidate(g, 2, b, cur_x, cur_o, j, 31, step, mix)
+                if not ok:
+                    inval += 1
+                    continue
+                ident += int((x == cur_x[b]).all() and (o == cur_o[b]).all())
+                seen.add((x.tobytes(), o.tobytes()))
+            assert st == {"candidates": K, "invalid": inval, "identical_to_base": ident,
+                          "distinct": len(seen)}, (step, b, st)
+        S.step()
+
+
+def _cur(S):
+    xs, os_ = [], []
+    for b in range(S.P):
+        _, x, o = S.get(b)
+        xs.append(x)
+        os_.append(o)
+    return np.stack(xs), np.stack(os_)

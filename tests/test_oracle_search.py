@@ -6,6 +6,7 @@ candidate, the min/commit rule, and that W simulated ranks give the single-rank 
 """
 
 import numpy as np
+import pytest
 
 from workloads import dag
 from workloads.rng import mix64
@@ -33,11 +34,12 @@ def test_identity_and_move_shapes(O):
     edges = set(zip(g.src.tolist(), g.dst.tolist()))
     P, n = xs.shape
     seen = {"flip": 0, "window": 0, "swap": 0}
-    for b in range(P):
-        ok, x, o = O.candidate(g, P, b, xs, orders, 0, 2021, 3, MIX)
+    mix = (50, 20, 20, 60)                                # swap-heavy (v6 blocks pairs on
+    for b in range(P):                                    # different base devices)
+        ok, x, o = O.candidate(g, P, b, xs, orders, 0, 2021, 3, mix)
         assert ok and (x == xs[b]).all() and (o == orders[b]).all()
         for j in range(1, 2048):
-            ok, x, o = O.candidate(g, P, b, xs, orders, j, 2021, 3, MIX)
+            ok, x, o = O.candidate(g, P, b, xs, orders, j, 2021, 3, mix)
             assert ok
             diff_pos = np.nonzero(o != orders[b])[0]
             if len(diff_pos):
@@ -52,6 +54,7 @@ def test_identity_and_move_shapes(O):
                 succs = lambda v: {d for s, d in edges if s == v}
                 assert not (preds(a) & preds(c)) and not (succs(a) & succs(c))
                 assert len(succs(a)) <= 64 and len(succs(c)) <= 64
+                assert xs[b][a] == xs[b][c]                  # same base device (v6)
                 assert O.makespan(g, x, o) >= 0           # still topological
                 if j % 128 == 0:
                     assert (x == xs[b]).all()              # lane 0 of a swap group: pure swap
@@ -69,12 +72,15 @@ def test_identity_and_move_shapes(O):
 
 
 def test_group_changes_stay_in_its_region(O):
-    """every change a group of 32 candidates makes lies in [c_g, c_g + 64) (DESIGN §4 S2)."""
+    """every change a group of 128 candidates makes lies in its region [c_g, c_g + 64), the
+    regions of consecutive groups tile the order (DESIGN §4 S2, v6)."""
     g, xs, orders = _setup(seed=6, n=300)
     P = xs.shape[0]
+    R = (g.n + 63) // 64
     for b in range(P):
+        rot = O.draw(2021, 2, P, b, 0, 13) % R
         for grp in range(1, 12):
-            c = O.draw(2021, 2, P, b, 128 * grp, 13) % g.n
+            c = 64 * ((grp + rot) % R)
             hi = min(g.n, c + 64)
             for lane in range(128):
                 j = 128 * grp + lane
@@ -188,3 +194,118 @@ def test_coarse_search_step_commits_best(O):
             ok, x, o = O.candidate(g, 3, b, xs, orders, int(keys[b]) & ((1 << 24) - 1), 4, 0, MIX)
             assert (rx[b] == x).all() and (ro[b] == o).all()
             assert rmk[b] == int(keys[b]) >> 24 == O.makespan(g, x, o)
+
+
+# ---------------------------------------------------------------------------------------------
+# Exact restatement of DESIGN.md §4 S2-S4 (spec v6) in plain Python, written from the text and
+# compared element by element with the oracle's decode (oracle_candidate).
+# ---------------------------------------------------------------------------------------------
+def _py_draw(seed, step, P, b, j, k):
+    ctr = (((step * P + b) * (1 << 24) + j) * 16 + k) & ((1 << 64) - 1)
+    return mix64(seed ^ mix64(ctr))
+
+
+def _py_candidate(g, P, b, xs, orders, j, seed, step, mix, edges, preds, succs):
+    n, D = g.n, g.D
+    bx, bo = xs[b], orders[b]
+    x, o = bx.copy(), bo.copy()
+    dr = lambda jj, k: _py_draw(seed, step, P, b, jj, k)
+    allowed = lambda v: [d for d in range(D)
+                         if g.allowed is None or (int(g.allowed[v]) >> d) & 1]
+    A = lambda q: [d for d in allowed(int(bo[q])) if d != int(bx[bo[q]])]
+    grp, lane = j // 128, j % 128
+    R = (n + 63) // 64                                         # S2
+    r = (grp + dr(0, 13) % R) % R
+    c, ln, ps = 64 * r, min(64, n - 64 * r), grp // R
+    swap = False                                               # S3
+    if grp != 0 and mix[3] > 0 and n >= 2 and dr(128 * grp, 15) % 100 < mix[3]:
+        k = min(c + dr(128 * grp, 14) % ln, n - 2)
+        a, cc = int(bo[k]), int(bo[k + 1])
+        blocked = ((a, cc) in edges or (cc, a) in edges or (preds[a] & preds[cc]) or
+                   (succs[a] & succs[cc]) or len(succs[a]) > 64 or len(succs[cc]) > 64 or
+                   bx[a] != bx[cc])
+        if not blocked:
+            o[k], o[k + 1] = cc, a
+            swap = True
+    if j == 0 or (swap and lane == 0):                         # S4
+        return True, x, o
+    W = mix[0] + mix[1] + mix[2]
+    if W <= 0:
+        return True, x, o
+    b1, b2 = (128 * mix[0]) // W, (128 * (mix[0] + mix[1])) // W
+    kind = "flip1" if lane < b1 else ("flipk" if lane < b2 else "window")
+    if kind == "flip1":
+        t = ps * b1 + lane
+        if t < ln * (D - 1):
+            q = c + t % ln
+            aq = A(q)
+            if t // ln >= len(aq):
+                return False, x, o
+            x[bo[q]] = aq[t // ln]
+            return True, x, o
+        kind = "flipk"
+    if kind == "flipk":
+        f = min(2 + dr(j, 1) % 3, ln)
+        taken = []
+        for i in range(f):
+            free = [q for q in range(c, c + ln) if q not in taken]
+            q = free[dr(j, 2 + 2 * i) % (ln - i)]
+            taken.append(q)
+            aq = A(q)
+            if not aq:
+                return False, x, o
+            x[bo[q]] = aq[dr(j, 3 + 2 * i) % len(aq)]
+        return True, x, o
+    i, nw = lane - b2, 128 - b2
+    s = c + (ps * nw + i) % ln
+    e = min(s + 1 + dr(j, 3) % 64, c + ln)
+    aq = A(s)
+    if not aq:
+        return False, x, o
+    d = aq[dr(j, 4) % len(aq)]
+    for q in range(s, e):
+        if d in allowed(int(bo[q])):
+            x[bo[q]] = d
+    return True, x, o
+
+
+@pytest.mark.parametrize("seed,n,D,allowed_frac,mix,P", [
+    (21, 150, 2, 0.0, (50, 20, 20, 10), 3),          # R = 3 regions: passes 0..10 in 4096 ids
+    (22, 333, 2, 0.0, (40, 20, 20, 60), 2),          # swap-heavy, clipped last region (13)
+    (23, 200, 3, 0.4, (50, 20, 20, 30), 2),          # masks: invalid and used-up flips
+    (24, 260, 4, 0.0, (10, 30, 60, 20), 2),          # D = 4, window-heavy
+    (25, 90, 4, 0.5, (80, 0, 0, 50), 1),             # FLIP1 only: enumerations run out
+    (26, 70, 2, 0.0, (0, 0, 1, 0), 2)])              # WINDOW only
+def test_decode_equals_spec_restatement(O, seed, n, D, allowed_frac, mix, P):
+    """oracle_candidate (C) = the plain-Python restatement of DESIGN §4 S2-S4, x and order
+    element by element, for 4096 ids per base (groups of every pass, swap groups, lane 0)."""
+    g = dag.random_dag(seed, n, 1.5, D=D, p_max=2000, max_bytes=50_000, beta0=300,
+                       beta1_fs=20_000, allowed_frac=allowed_frac)
+    orders = np.stack([dag.random_topo_order(g, 5 + b) for b in range(P)]).astype(np.int32)
+    xs = dag.random_placements(g, 9, P)
+    edges = set(zip(g.src.tolist(), g.dst.tolist()))
+    preds = [set() for _ in range(n)]
+    succs = [set() for _ in range(n)]
+    for s_, d_ in edges:
+        preds[d_].add(s_)
+        succs[s_].add(d_)
+    for s_ in range(n):                       # S3 counts out-edges (parallel edges included)
+        if int((g.src == s_).sum()) > 64:
+            succs[s_] = succs[s_] | {-1 - k for k in range(65)}
+    counts = {"valid": 0, "invalid": 0, "swapped": 0}
+    for step in (0, 3):
+        for b in range(P):
+            for j in range(4096):
+                ok, x, o = O.candidate(g, P, b, xs, orders, j, 77, step, mix)
+                pok, px, po = _py_candidate(g, P, b, xs, orders, j, 77, step, mix, edges, preds,
+                                            succs)
+                assert ok == pok, (step, b, j)
+                if ok:
+                    assert (x == px).all() and (o == po).all(), (step, b, j)
+                counts["valid" if ok else "invalid"] += 1
+                counts["swapped"] += int((o != orders[b]).any())
+    assert counts["valid"] > 0
+    if mix[3]:
+        assert counts["swapped"] > 0
+    if allowed_frac:
+        assert counts["invalid"] > 0
