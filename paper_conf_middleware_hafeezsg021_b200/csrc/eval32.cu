@@ -66,6 +66,15 @@ __host__ __device__ constexpr int warps_for(int cpl) { return cpl == 1 ? PESTO_E
 #endif
 
 constexpr int kStages32 = PESTO_E32_STAGES;
+#ifndef PESTO_UNI_SWITCH
+#define PESTO_UNI_SWITCH 0
+#endif
+// CPL = 2 reads the next step's head one step ahead (1) or its own head at the step's top (0)
+#ifndef PESTO_HEAD_AHEAD2
+#define PESTO_HEAD_AHEAD2 1
+#endif
+constexpr bool kHeadAhead = PESTO_HEAD_AHEAD2 != 0;
+constexpr bool kUniSwitch = PESTO_UNI_SWITCH != 0;
 __host__ __device__ constexpr int min_blocks_for(int cpl) { return cpl == 1 ? PESTO_E32_MINB1 : PESTO_E32_MINB2; }
 
 // per-candidate device / link free times
@@ -388,6 +397,84 @@ __device__ __forceinline__ void push32_u(const Ctx32 &cx, const uint4 rec, int x
     }
     push_tail<CPL, T>(cx, rec.z, a, fwd);
 }
+
+// D = 2 (register state), both devices warp-uniform: the edge's whole path -- link or not, which
+// direction, register / ring / cold slot, first push or max -- is selected by one jump-table
+// dispatch on idx = target class << 2 | xu << 1 | (xu != yu), taken from one record word
+// (succ_pos: successor code at bit 24, class code at bits 27-29) and xm = xu * 3
+template <uint32_t TC, int XU, int CROSS, int CPL, class T>
+__device__ __forceinline__ void uni_edge(const Ctx32 &cx, const uint4 rec, const T (&cc)[CPL],
+                                         RegState32<CPL, T> &st, T (&fwd)[CPL]) {
+    T a[CPL];
+#pragma unroll
+    for (int c = 0; c < CPL; c++) {
+        if constexpr (CROSS) {                               // FCFS link xu -> 1 - xu
+            T &l = XU ? st.l10[c] : st.l01[c];
+            a[c] = add_sat(max(cc[c], l), (T)(XU ? rec.w : rec.x));
+            l = a[c];
+        } else {
+            a[c] = cc[c];                                    // same device: C_v (L144)
+        }
+    }
+    constexpr uint32_t F = TC << 29;
+    if constexpr ((F & kT32Next) != 0) {
+#pragma unroll
+        for (int c = 0; c < CPL; c++) fwd[c] = max(fwd[c], a[c]);
+    } else {
+        const uint32_t bytes = (rec.z & kT32SlotMask) * CPL * kSc<T>;
+        if constexpr ((F & kT32Near) != 0) {
+#pragma unroll
+            for (int c = 0; c < CPL; c++) {
+                const uint32_t slot = cx.ring + bytes + c * kColB<T>;
+                T v = a[c];
+                if constexpr ((F & kT32First) == 0) v = max(v, lds_t<T>(slot));
+                sts_t(slot, v);
+            }
+        } else {
+#pragma unroll
+            for (int c = 0; c < CPL; c++) {
+                T *slot = reinterpret_cast<T *>(cx.cold + bytes + c * kColB<T>);
+                if constexpr ((F & kT32First) != 0) *slot = a[c];
+                else if constexpr (sizeof(T) == 4) atomicMax(slot, a[c]);
+                else atomicMax(reinterpret_cast<unsigned long long *>(slot), (unsigned long long)a[c]);
+            }
+        }
+    }
+}
+#include "uni_push_ptx.inc"
+template <int CPL, class T>
+__device__ __forceinline__ void push_uni(const Ctx32 &cx, const uint4 rec, uint32_t xm,
+                                         const T (&cc)[CPL], RegState32<CPL, T> &st, T (&fwd)[CPL]) {
+    if constexpr (PESTO_UNI_SWITCH == 2 && CPL == 2 && sizeof(T) == 4) {
+        const uint32_t idx = ((((rec.y >> (kSuccTcShift - 2)) & 0x1Cu) | ((rec.y >> kSuccXShift) & 1u)) ^ xm);
+        asm volatile(PESTO_UNI_PUSH_PTX
+                     : "+r"(st.l01[0]), "+r"(st.l01[1]), "+r"(st.l10[0]), "+r"(st.l10[1]),
+                       "+r"(fwd[0]), "+r"(fwd[1])
+                     : "r"(idx), "r"(rec.x), "r"(rec.w), "r"(rec.z), "r"(cc[0]), "r"(cc[1]),
+                       "r"(cx.ring), "l"(cx.cold)
+                     : "memory");
+        return;
+    }
+    // idx = class << 2 | xu << 1 | (xu != yu): 20 dense entries, one jump table
+    const uint32_t idx = ((((rec.y >> (kSuccTcShift - 2)) & 0x1Cu) | ((rec.y >> kSuccXShift) & 1u)) ^ xm);
+    switch (idx) {
+#define PESTO_UNI_CASES(TC, FL)                                                          \
+    case (TC) * 4 + 0: uni_edge<FL, 0, 0, CPL, T>(cx, rec, cc, st, fwd); break;          \
+    case (TC) * 4 + 1: uni_edge<FL, 0, 1, CPL, T>(cx, rec, cc, st, fwd); break;          \
+    case (TC) * 4 + 2: uni_edge<FL, 1, 0, CPL, T>(cx, rec, cc, st, fwd); break;          \
+    case (TC) * 4 + 3: uni_edge<FL, 1, 1, CPL, T>(cx, rec, cc, st, fwd); break;
+        PESTO_UNI_CASES(0u, 0u)      // far, later push: RED.MAX
+        PESTO_UNI_CASES(1u, 4u)      // far, first push: STG
+        PESTO_UNI_CASES(2u, 2u)      // near ring, later push
+        PESTO_UNI_CASES(3u, 6u)      // near ring, first push
+        PESTO_UNI_CASES(4u, 1u)      // next position: register
+#undef PESTO_UNI_CASES
+        default: __builtin_unreachable();
+    }
+}
+template <int CPL, class T>
+__device__ __forceinline__ void push_uni(const Ctx32 &, const uint4, uint32_t, const T (&)[CPL],
+                                         SmemState32<CPL, T> &, T (&)[CPL]) {}
 
 // the (up to two) out-edges of one step, records already in registers; yfn(k, rec, y) gives
 // the successor's devices of edge k
@@ -752,7 +839,7 @@ eval32_kernel(const EvalParams P) {
                         // (CPL = 1 reads its own head here: the read-ahead copy costs more than the
                         // LDS latency it hides there -- measured 5.86 vs 5.77 ms on inception)
                         uint4 hn;
-                        if constexpr (CPL == 1) h = lds_v4(sp);
+                        if constexpr (CPL == 1 || !kHeadAhead) h = lds_v4(sp);
                         else hn = lds_v4(sp + 48);
                         e0 = lds_v4(sp + 16);
                         e1 = lds_v4(sp + 32);
@@ -825,29 +912,32 @@ eval32_kernel(const EvalParams P) {
                                     else push32<PL, CPL, T>(cx, e1, x, y, cc, st, fwd);
                                 }
                             } else if (xu >= 0) {
+                                const uint32_t xm = (uint32_t)xu * 3u;
                                 if (ne >= 1) {
                                     const int32_t q0 = (int32_t)(e0.y & kSuccPosMask);
-                                    if ((uint32_t)(q0 - place.rc) >= (uint32_t)place.rlen)
-                                        push32_u<PL, CPL, T>(cx, e0, xu, (int)((e0.y >> kSuccXShift) & 7u), cc, st, fwd);
-                                    else { int y[CPL]; place_y(0, e0, y); push32<PL, CPL, T>(cx, e0, x, y, cc, st, fwd); }
+                                    if ((uint32_t)(q0 - place.rc) >= (uint32_t)place.rlen) {
+                                        if constexpr (PL == 1 && kUniSwitch) push_uni<CPL, T>(cx, e0, xm, cc, st, fwd);
+                                        else push32_u<PL, CPL, T>(cx, e0, xu, (int)((e0.y >> kSuccXShift) & 7u), cc, st, fwd);
+                                    } else { int y[CPL]; place_y(0, e0, y); push32<PL, CPL, T>(cx, e0, x, y, cc, st, fwd); }
                                 }
                                 if (ne >= 2) {
                                     const int32_t q1 = (int32_t)(e1.y & kSuccPosMask);
-                                    if ((uint32_t)(q1 - place.rc) >= (uint32_t)place.rlen)
-                                        push32_u<PL, CPL, T>(cx, e1, xu, (int)((e1.y >> kSuccXShift) & 7u), cc, st, fwd);
-                                    else { int y[CPL]; place_y(1, e1, y); push32<PL, CPL, T>(cx, e1, x, y, cc, st, fwd); }
+                                    if ((uint32_t)(q1 - place.rc) >= (uint32_t)place.rlen) {
+                                        if constexpr (PL == 1 && kUniSwitch) push_uni<CPL, T>(cx, e1, xm, cc, st, fwd);
+                                        else push32_u<PL, CPL, T>(cx, e1, xu, (int)((e1.y >> kSuccXShift) & 7u), cc, st, fwd);
+                                    } else { int y[CPL]; place_y(1, e1, y); push32<PL, CPL, T>(cx, e1, x, y, cc, st, fwd); }
                                 }
                             } else {
                                 edges32<PL, CPL, T>(cx, h.w, e0, e1, x, cc, place_y, st, fwd);
                             }
                         }
                         sp += kStepBytes;
-                        if constexpr (CPL != 1) h = hn;
+                        if constexpr (CPL != 1 && kHeadAhead) h = hn;
                     }
                     if (!kSearch || sp >= spe) break;
                     // sp = the first step of the op at ks (a walk stops there only for ks)
                     lim = spe;
-                    if constexpr (CPL == 1) h = lds_v4(sp);
+                    if constexpr (CPL == 1 || !kHeadAhead) h = lds_v4(sp);
                     e0 = lds_v4(sp + 16);
                     e1 = lds_v4(sp + 32);
                     v++;

@@ -277,6 +277,7 @@ pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<
                      : (near_edge(e) ? (kT32Near | (uint32_t)(pos[w] & (kRing - 1)) * 128u)
                                      : (uint32_t)cslot[w] * 128u) |
                        (first32[e] ? kT32First : 0u);
+            r.succ_pos = (int32_t)((uint32_t)r.succ_pos | (target_class32(r.target) << kSuccTcShift));
             L->pin_ref[pfill[pos[w]]++] = (uint32_t)at;
             L->eloc32[e] = (uint32_t)at;
             return r;

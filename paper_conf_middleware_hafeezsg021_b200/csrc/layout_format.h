@@ -70,6 +70,14 @@ constexpr int kOpXShift = 25;                   // OpRec32.nout bits 25-27: base
 constexpr uint32_t kOpAdj = 1u << 28;           // producer feeds two adjacent positions
 constexpr int kSuccXShift = 24;                 // EdgeRec32.succ_pos bits 24-26: base device
 constexpr uint32_t kSuccPosMask = (1u << 24) - 1;
+// EdgeRec32.succ_pos bits 27-29: the target's class as a dense code (0 far, 1 far first,
+// 2 near, 3 near first, 4 next), so that the walk's uniform-device push finds (class, successor
+// code) in one word and dispatches on them with a single jump table (eval32.cu push_uni)
+constexpr int kSuccTcShift = 27;
+constexpr uint32_t kSuccTcMask = 7u << kSuccTcShift;
+constexpr uint32_t target_class32(uint32_t target) {
+    return (target & (1u << 29)) ? 4u : (((target >> 30) & 1u) << 1 | (target >> 31));
+}
 constexpr uint32_t kPinHeavy = 1u << 31;        // patch reference into the out-of-line array
 constexpr uint32_t kT32First = 1u << 31;        // EdgeRec32.target: first push into its slot
 constexpr uint32_t kT32Near = 1u << 30;         // push into the near ring (slot = succ & 15)

@@ -526,7 +526,8 @@ bool swap_in_place(pesto_search *s, int b, int32_t k, Patcher &pt) {
                                                 (e == near_first ? kT32First : 0u))
                                              : ((uint32_t)L.cslot[w] * 128u | (e == far_first ? kT32First : 0u));
                 const uint32_t loc = L.eloc32[e];
-                pt.set32(L.d_blob32, L.blob32.data(), loc + 4, kSuccPosMask, (uint32_t)q);
+                pt.set32(L.d_blob32, L.blob32.data(), loc + 4, kSuccPosMask | kSuccTcMask,
+                         (uint32_t)q | (target_class32(tgt) << kSuccTcShift));
                 pt.set32(L.d_blob32, L.blob32.data(), loc + 8, ~0u, tgt);
             }
             pt.set32(L.d_blob32, L.blob32.data(), L.op_off32[q] + 12, kStHasNear,

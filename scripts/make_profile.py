@@ -16,12 +16,17 @@ dram = sum(s[k] * scale[s[k + '.unit']] for k in ('dram__bytes_read.sum', 'dram_
 lts = None
 if s.get('lts__t_bytes.sum') is not None:
     lts = s['lts__t_bytes.sum'] * scale.get(s['lts__t_bytes.sum.unit'], 1.0)
+if lts is None and s.get('lts__t_sectors_srcunit_tex_op_read.sum') is not None:
+    # L2 traffic from the SMs (L1 misses, stores and reductions): 32-byte sectors
+    lts = 32.0 * (s['lts__t_sectors_srcunit_tex_op_read.sum'] +
+                  s['lts__t_sectors_srcunit_tex_op_write.sum'])
 dur = s['gpu__time_duration.sum'] * {'ms': 1e-3, 'us': 1e-6, 'ns': 1e-9}[s['gpu__time_duration.sum.unit']]
 tag = sys.argv[5] if len(sys.argv) > 5 else 'r2'
 out = {'kernel': s['kernel'], 'config': cfg, 'command': cmd, 'round': int(tag[1]), 'metrics': metrics,
        'stall_cycles_per_issue': s['stall_cycles_per_issue'],
        'dram_bytes_per_launch': dram, 'duration_s': dur, 'lts_bytes_per_launch': lts,
        'dram_GBps': dram / dur / 1e9,
+       'l2_GBps': (lts / dur / 1e9) if lts else None,
        'note': 'one launch, ncu --set full --clock-control none (cold, serialised): compare '
                'shares and counters, not the absolute time, with bench.py'}
 name = os.path.join('profiles', f"{tag}_eval32_{cfg}_ncu.json")
