@@ -18,7 +18,7 @@ ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 CU_SOURCES = ["kernels.cu", "eval32.cu", "nondelay.cu", "roofs.cu"]
 CPP_SOURCES = ["graph.cpp", "layout.cpp", "search.cpp", "coarsen.cpp"]
 HEADERS = ["internal.h", "host.h", "layout_format.h", "moves.cuh", "device_common.cuh",
-           "feasibility.cuh", "uni_push_ptx.inc"]
+           "feasibility.cuh", "uni_push_ptx.inc", "fast_walk_ptx.inc"]
 
 
 def _stale() -> bool:

@@ -51,7 +51,10 @@ template <class T> constexpr uint32_t kSc = sizeof(T) / 4u;
 #ifndef PESTO_E32_W1
 #define PESTO_E32_W1 8
 #endif
-__host__ __device__ constexpr int warps_for(int cpl) { return cpl == 1 ? PESTO_E32_W1 : 4; }
+#ifndef PESTO_E32_W2
+#define PESTO_E32_W2 4
+#endif
+__host__ __device__ constexpr int warps_for(int cpl) { return cpl == 1 ? PESTO_E32_W1 : PESTO_E32_W2; }
 
 // TMA ring depth and the occupancy target (resident CTAs per SM the register allocation aims
 // for), per candidates-per-lane
@@ -67,15 +70,27 @@ __host__ __device__ constexpr int warps_for(int cpl) { return cpl == 1 ? PESTO_E
 
 constexpr int kStages32 = PESTO_E32_STAGES;
 #ifndef PESTO_UNI_SWITCH
-#define PESTO_UNI_SWITCH 0
+#define PESTO_UNI_SWITCH 2
 #endif
 // CPL = 2 reads the next step's head one step ahead (1) or its own head at the step's top (0)
 #ifndef PESTO_HEAD_AHEAD2
 #define PESTO_HEAD_AHEAD2 1
 #endif
 constexpr bool kHeadAhead = PESTO_HEAD_AHEAD2 != 0;
+// search walk, D = 2, two candidates per lane, uint32 time: uniform steps run in the PTX fast
+// segment (fast_walk_ptx.inc), special positions in the C++ step below
+#ifndef PESTO_FAST_WALK
+#define PESTO_FAST_WALK 1
+#endif
 constexpr bool kUniSwitch = PESTO_UNI_SWITCH != 0;
 __host__ __device__ constexpr int min_blocks_for(int cpl) { return cpl == 1 ? PESTO_E32_MINB1 : PESTO_E32_MINB2; }
+// tile loads: a producer warp per CTA (0), or issued by the consumer warp that releases a stage
+// last (1: no warp slot and no registers spent on a warp that mostly sleeps)
+#ifndef PESTO_E32_NOPROD
+#define PESTO_E32_NOPROD 0
+#endif
+constexpr bool kProducerWarp = PESTO_E32_NOPROD == 0;
+__host__ __device__ constexpr int threads_for(int cpl) { return (warps_for(cpl) + (kProducerWarp ? 1 : 0)) * 32; }
 
 // per-candidate device / link free times
 template <int CPL, class T>
@@ -442,6 +457,49 @@ __device__ __forceinline__ void uni_edge(const Ctx32 &cx, const uint4 rec, const
     }
 }
 #include "uni_push_ptx.inc"
+#include "fast_walk_ptx.inc"
+
+// the uniform steps from sp on (until lim or the first step of the special position nspec),
+// state in registers; returns with sp at the first step it did not take
+__device__ __forceinline__ void fast_segment(uint32_t &sp, int32_t &v, uint32_t &fxu,
+                                             RegState32<2, uint32_t> &st,
+                                             uint32_t (&fwd)[2], uint32_t (&nfar)[2],
+                                             uint32_t (&nnear)[2], uint32_t lim, int32_t nspec,
+                                             uint32_t ring, uint32_t stage, const uint8_t *cold) {
+    asm volatile(PESTO_FAST_WALK_PTX2
+                 : "+r"(sp), "+r"(v), "+r"(fxu), "+r"(st.d0[0]), "+r"(st.d0[1]), "+r"(st.d1[0]), "+r"(st.d1[1]),
+                   "+r"(st.l01[0]), "+r"(st.l01[1]), "+r"(st.l10[0]), "+r"(st.l10[1]),
+                   "+r"(fwd[0]), "+r"(fwd[1]), "+r"(nfar[0]), "+r"(nfar[1]), "+r"(nnear[0]),
+                   "+r"(nnear[1])
+                 : "r"(lim), "r"(nspec), "r"(ring), "r"(stage), "l"(cold)
+                 : "memory");
+}
+__device__ __forceinline__ void fast_segment(uint32_t &sp, int32_t &v, uint32_t &fxu,
+                                             RegState32<1, uint32_t> &st,
+                                             uint32_t (&fwd)[1], uint32_t (&nfar)[1],
+                                             uint32_t (&nnear)[1], uint32_t lim, int32_t nspec,
+                                             uint32_t ring, uint32_t stage, const uint8_t *cold) {
+    asm volatile(PESTO_FAST_WALK_PTX1
+                 : "+r"(sp), "+r"(v), "+r"(fxu), "+r"(st.d0[0]), "+r"(st.d1[0]), "+r"(st.l01[0]),
+                   "+r"(st.l10[0]), "+r"(fwd[0]), "+r"(nfar[0]), "+r"(nnear[0])
+                 : "r"(lim), "r"(nspec), "r"(ring), "r"(stage), "l"(cold)
+                 : "memory");
+}
+__device__ __forceinline__ void fast_segment(uint32_t &sp, int32_t &v, uint32_t &fxu,
+                                             RegState32<1, uint64_t> &st,
+                                             uint64_t (&fwd)[1], uint64_t (&nfar)[1],
+                                             uint64_t (&nnear)[1], uint32_t lim, int32_t nspec,
+                                             uint32_t ring, uint32_t stage, const uint8_t *cold) {
+    asm volatile(PESTO_FAST_WALK_PTX1W
+                 : "+r"(sp), "+r"(v), "+r"(fxu), "+l"(st.d0[0]), "+l"(st.d1[0]), "+l"(st.l01[0]),
+                   "+l"(st.l10[0]), "+l"(fwd[0]), "+l"(nfar[0]), "+l"(nnear[0])
+                 : "r"(lim), "r"(nspec), "r"(ring), "r"(stage), "l"(cold)
+                 : "memory");
+}
+template <int CPL, class T, class ST>
+__device__ __forceinline__ void fast_segment(uint32_t &, int32_t &, uint32_t &, ST &, T (&)[CPL], T (&)[CPL],
+                                             T (&)[CPL], uint32_t, int32_t, uint32_t, uint32_t,
+                                             const uint8_t *) {}
 template <int CPL, class T>
 __device__ __forceinline__ void push_uni(const Ctx32 &cx, const uint4 rec, uint32_t xm,
                                          const T (&cc)[CPL], RegState32<CPL, T> &st, T (&fwd)[CPL]) {
@@ -508,9 +566,12 @@ __device__ __forceinline__ void begin32(const uint4 h, StateT &st, const T (&r)[
 }
 
 template <int MODE, int PL, int CPL, class T>
-__global__ void __launch_bounds__((warps_for(CPL) + 1) * 32, min_blocks_for(CPL))
+__global__ void __launch_bounds__(threads_for(CPL), min_blocks_for(CPL))
 eval32_kernel(const EvalParams P) {
     constexpr bool kSearch = MODE == 1 || MODE == 5;   // 5: search with S9 coarse groups
+    // uniform steps through the PTX fast segment (D = 2, CPL 2, 32-bit time, search)
+    constexpr bool kFast = PESTO_FAST_WALK != 0 && MODE == 1 && PL == 1 &&
+                           (sizeof(T) == 4 || CPL == 1);
     constexpr int NW = warps_for(CPL);          // consumer warps per CTA (256 candidates)
     constexpr int CW = 32 * CPL;                // candidates per warp
     extern __shared__ __align__(128) uint8_t smem[];
@@ -533,22 +594,52 @@ eval32_kernel(const EvalParams P) {
     const uint32_t cpos_s = su32_reg(align16(cur + (PL != 1 ? (size_t)NW * (P.D + P.D * P.D) * CW * sizeof(T) : 0)));
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    if (threadIdx.x == 0) {
-        for (int s = 0; s < kStages32; s++) {
-            mbar_init(&full[s], 1);
-            mbar_init(&empty[s], NW);
-        }
-        mbar_fence_init();
-    }
-    __syncthreads();
-
     auto runs_here = [&](int bl) {           // search: this kernel owns bases below saturation
         // (the wide instance, gate 2, owns the bases at or above saturation)
         return !kSearch || P.gate == 0 ||
                (P.gate == 1 ? P.base_mk[bl] < (int64_t)kSat32 : P.base_mk[bl] >= (int64_t)kSat32);
     };
+    // the CTA's tile sequence: (task, tile) over its tasks, tiles in order (no-producer mode)
+    auto first_task = [&](int64_t task) {
+        for (; task < P.n_tasks; task += gridDim.x)
+            if (runs_here(kSearch ? (int)(task / P.tasks_per_base) : 0)) break;
+        return task;
+    };
+    auto advance = [&](int64_t &task, int &t) {
+        if (task >= P.n_tasks) return;
+        const int bl = kSearch ? (int)(task / P.tasks_per_base) : 0;
+        if (++t < P.bases[bl].n_tiles32) return;
+        t = 0;
+        task = first_task(task + gridDim.x);
+    };
+    auto load_tile = [&](int64_t task, int t, int s) {      // one lane
+        if (task >= P.n_tasks) return;
+        const BaseLayoutDev *B = &P.bases[kSearch ? (int)(task / P.tasks_per_base) : 0];
+        const TileDesc td = B->tiles32[t];
+        mbar_expect_tx(&full[s], (uint32_t)td.bytes);
+        bulk_g2s(smem + (size_t)s * sb, B->blob32 + td.byte_off, (uint32_t)td.bytes, &full[s]);
+    };
+    // stage release counters (no-producer mode), in the space of the empty barriers
+    const uint32_t rel0 = su32(empty);
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < kStages32; s++) {
+            mbar_init(&full[s], 1);
+            if constexpr (kProducerWarp) mbar_init(&empty[s], NW);
+            else empty[s] = 0;
+        }
+        mbar_fence_init();
+        if constexpr (!kProducerWarp) {
+            int64_t task = first_task(blockIdx.x);
+            int t = 0;
+            for (int s = 0; s < kStages32; s++) {
+                load_tile(task, t, s);
+                advance(task, t);
+            }
+        }
+    }
+    __syncthreads();
 
-    if (warp == NW) {
+    if (kProducerWarp && warp == NW) {
         if (lane == 0) {
             uint32_t it = 0;
             for (int64_t task = blockIdx.x; task < P.n_tasks; task += gridDim.x) {
@@ -656,6 +747,11 @@ eval32_kernel(const EvalParams P) {
         place.rlen = 0;
         bool active;
         bool valid[CPL];
+        // fast walk: the group's next special position (spec_pos list of its region)
+        int32_t nspec = INT32_MAX;
+        uint32_t spi = 0;
+        bool fast_ok = false, gen_op = false;
+        uint32_t fxu = 0;            // the fast segment's current op device (across segments)
         int32_t ks = -1;
         uint32_t off_ks = 0;         // search: byte offset of the op at ks in the step stream
         if (MODE == 4) {
@@ -704,6 +800,13 @@ eval32_kernel(const EvalParams P) {
             if (!coarse) {
                 place.rc = rg.c;
                 place.rlen = rg.len;
+            }
+            if constexpr (kFast) {
+                fast_ok = B->spec_pos != nullptr;
+                if (fast_ok) {
+                    spi = __ldg(B->spec_off + rg.c / kRegion);
+                    nspec = __ldg(B->spec_pos + spi);
+                }
             }
             const uint8_t *blocked = B->swap_blocked;
             const int32_t *ord = B->order;
@@ -834,12 +937,26 @@ eval32_kernel(const EvalParams P) {
                 }
                 for (;;) {
                     while (sp < lim) {
+                        if constexpr (kFast) {
+                            // uniform steps: the PTX segment; a special position's first step
+                            // (and its continuation steps) take the C++ step below
+                            if (fast_ok) {
+                                const bool is_cont = (lds_u32(sp + 12) & kStCont) != 0;
+                                if (is_cont ? !gen_op : (v + 1 != nspec)) {
+                                    fast_segment(sp, v, fxu, st, fwd, nfar, nnear, lim, nspec,
+                                                 cx.ring, stage, cx.cold);
+                                    gen_op = false;
+                                    continue;
+                                }
+                                gen_op = true;
+                            }
+                        }
                         // the next step's head (past the tile's end: padding, never used); this
                         // step's edge records (their first use is after the head's work)
                         // (CPL = 1 reads its own head here: the read-ahead copy costs more than the
                         // LDS latency it hides there -- measured 5.86 vs 5.77 ms on inception)
                         uint4 hn;
-                        if constexpr (CPL == 1 || !kHeadAhead) h = lds_v4(sp);
+                        if constexpr (CPL == 1 || !kHeadAhead || kFast) h = lds_v4(sp);
                         else hn = lds_v4(sp + 48);
                         e0 = lds_v4(sp + 16);
                         e1 = lds_v4(sp + 32);
@@ -855,6 +972,10 @@ eval32_kernel(const EvalParams P) {
                         }
                         if (!(h.w & kStCont)) {
                             v++;
+                            if constexpr (kFast) {
+                                if (fast_ok)
+                                    while (nspec <= v) nspec = __ldg(P.bases[bl].spec_pos + ++spi);
+                            }
                             issue_far(h, v);
                             cp_async_wait<kPrefetchDist - 1>();      // v+1 has landed
                             T r[CPL];
@@ -932,12 +1053,12 @@ eval32_kernel(const EvalParams P) {
                             }
                         }
                         sp += kStepBytes;
-                        if constexpr (CPL != 1 && kHeadAhead) h = hn;
+                        if constexpr (CPL != 1 && kHeadAhead && !kFast) h = hn;
                     }
                     if (!kSearch || sp >= spe) break;
                     // sp = the first step of the op at ks (a walk stops there only for ks)
                     lim = spe;
-                    if constexpr (CPL == 1 || !kHeadAhead) h = lds_v4(sp);
+                    if constexpr (CPL == 1 || !kHeadAhead || kFast) h = lds_v4(sp);
                     e0 = lds_v4(sp + 16);
                     e1 = lds_v4(sp + 32);
                     v++;
@@ -987,6 +1108,11 @@ eval32_kernel(const EvalParams P) {
                         v++;
                         xu = -1;
                         load_next(v + 1, nfar, nnear);
+                        if constexpr (kFast) {
+                            if (fast_ok)
+                                while (nspec <= v) nspec = __ldg(P.bases[bl].spec_pos + ++spi);
+                            gen_op = false;       // the walk continues at a first step
+                        }
                         if (straddle) {
                             skip = n1;
                             break;
@@ -1000,7 +1126,22 @@ eval32_kernel(const EvalParams P) {
                 }
             }
             __syncwarp();
-            if (lane == 0) mbar_arrive(&empty[s]);
+            if constexpr (kProducerWarp) {
+                if (lane == 0) mbar_arrive(&empty[s]);
+            } else if (lane == 0) {
+                // the warp that releases stage s last loads the CTA's tile kStages32 iterations
+                // ahead into it (acq_rel: every warp's reads of the stage precede the load)
+                uint32_t old;
+                asm volatile("atom.acq_rel.cta.shared::cta.add.u32 %0, [%1], 1;"
+                             : "=r"(old) : "r"(rel0 + 8u * (uint32_t)s) : "memory");
+                if ((old + 1u) % (uint32_t)NW == 0u) {
+                    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+                    int64_t nt_task = task;
+                    int nt_t = t;
+                    for (int k = 0; k < kStages32; k++) advance(nt_task, nt_t);
+                    load_tile(nt_task, nt_t, s);
+                }
+            }
         }
         cp_async_wait<0>();
 
@@ -1062,7 +1203,7 @@ cudaError_t launch_one32(const EvalParams &p, int grid, cudaStream_t st) {
         (e = cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout,
                                   cudaSharedmemCarveoutMaxShared)) != cudaSuccess)
         return e;
-    kern<<<grid, (warps_for(CPL) + 1) * 32, smem, st>>>(p);
+    kern<<<grid, threads_for(CPL), smem, st>>>(p);
     return cudaGetLastError();
 }
 
@@ -1073,7 +1214,7 @@ int occupancy_one32(const EvalParams &p) {
     if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) != cudaSuccess)
         return 0;
     int n = 0;
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kern, (warps_for(CPL) + 1) * 32, smem) !=
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kern, threads_for(CPL), smem) !=
         cudaSuccess)
         return 0;
     return n;

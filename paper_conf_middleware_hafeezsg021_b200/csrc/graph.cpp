@@ -126,6 +126,8 @@ pesto_status upload_layout(pesto_graph *g, Layout &L) {
     if ((e = upload_vec(L.d_pin_off, L.pin_off)) != cudaSuccess) return cuda_fail(e, "upload layout");
     if ((e = upload_vec(L.d_pin_ref, L.pin_ref)) != cudaSuccess) return cuda_fail(e, "upload layout");
     if ((e = upload_vec(L.d_slot_succ, L.slot_succ)) != cudaSuccess) return cuda_fail(e, "upload layout");
+    if ((e = upload_vec(L.d_spec_off, L.spec_off)) != cudaSuccess) return cuda_fail(e, "upload layout");
+    if ((e = upload_vec(L.d_spec_pos, L.spec_pos)) != cudaSuccess) return cuda_fail(e, "upload layout");
     L.on_device = true;
     std::vector<BaseLayoutDev> view{layout_view(L)};
     if ((e = upload_vec(L.d_view, view)) != cudaSuccess) return cuda_fail(e, "upload layout");
@@ -154,6 +156,8 @@ BaseLayoutDev layout_view(const Layout &L) {
     v.pin_ref = L.d_pin_ref.as<uint32_t>();
     v.nd_dst = L.d_nd_dst.as<int32_t>();
     v.nd_t = L.d_nd_t.as<int64_t>();
+    v.spec_off = L.spec_off.empty() ? nullptr : L.d_spec_off.as<uint32_t>();
+    v.spec_pos = L.spec_pos.empty() ? nullptr : L.d_spec_pos.as<int32_t>();
     return v;
 }
 

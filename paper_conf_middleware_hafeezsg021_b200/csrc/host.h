@@ -65,10 +65,17 @@ struct Layout {
     std::vector<uint32_t> eloc64, eloc32;           // [edge] record offset (| kPinHeavy: heavy)
     std::vector<int32_t> slot_succ;                 // [2 * steps] successor position of each
                                                     // eval32 edge slot, -1 = empty (K5 y stream)
+    // eval32 search fast walk: per region r (positions [64r, 64r + 64)), the
+    // sorted positions where a group of that region is not warp-uniform -- the region itself and
+    // every producer before it of an op inside it -- followed by INT32_MAX sentinels (slack, so a
+    // committed swap can rewrite a region's list in place); CSR by region
+    std::vector<uint32_t> spec_off;
+    std::vector<int32_t> spec_pos;
     int64_t comm_gen = -1;
     // device copies
     DevBuf d_blob, d_heavy, d_tiles, d_pos, d_adj, d_allowed_pos, d_view, d_order;
     DevBuf d_blob32, d_heavy32, d_tiles32, d_op_off32, d_pin_off, d_pin_ref, d_slot_succ;
+    DevBuf d_spec_off, d_spec_pos;
     // row f4(i): producer-grouped out-edges in this order's FCFS tie order (built on demand)
     DevBuf d_nd_dst, d_nd_t;
     int64_t nd_gen = -1;                // comm tables generation the nd arrays were built for
@@ -146,6 +153,9 @@ pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<
 pesto_status upload_layout(pesto_graph *g, Layout &L);
 // v4 swap rule (DESIGN.md §4 S3) for the ops a (first) and c (second) of an adjacent pair
 bool pair_blocked(const pesto_graph *g, int32_t a, int32_t c);
+// the special positions of region r under L's order (see Layout::spec_pos), sorted, unique
+void spec_region(const pesto_graph *g, const Layout &L, int32_t r, std::vector<int32_t> &out);
+constexpr int kSpecSlack = 8;       // sentinels after each region's list
 // row f4(i): device arrays of the non-delay kernel (graph-level and per order), the domain
 // check (positive durations, n <= 2^20) and the scratch for `slots` resident warps
 pesto_status nd_check(pesto_graph *g);

@@ -39,6 +39,9 @@ struct BaseLayoutDev {
     const int64_t *nd_t;        // [m][n_classes] transfer time per link class
     // search spec S9 (row f2 group moves): merged vertex of the op at each position, or null
     const uint8_t *coarse_pos;
+    // eval32 search fast walk: special positions per region (Layout::spec_pos), CSR by region
+    const uint32_t *spec_off;
+    const int32_t *spec_pos;
 };
 
 // Row f3 constraints as the kernels see them (PAPER.md L202 memory, L175 colocation).

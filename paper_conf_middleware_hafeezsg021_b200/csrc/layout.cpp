@@ -8,6 +8,7 @@
 //           (search bases only; patched in place by K4 when a placement move is committed).
 // Everything is O(n + m): counting sorts by position, flat CSR arrays, one pass per field.
 #include <algorithm>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 
@@ -298,7 +299,13 @@ pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<
             L->tiles32.push_back(td);
             L->stage_bytes32 = std::max(L->stage_bytes32, td.bytes);
         };
-        const size_t budget = (size_t)kTileTarget;
+        // eval32 tile budget: kTileTarget, or PESTO_TILE32_BYTES (occupancy experiments: a smaller
+        // tile lets more CTAs' stages fit in shared memory)
+        static const size_t budget = [] {
+            const char *e = std::getenv("PESTO_TILE32_BYTES");
+            const long v = e ? std::atol(e) : 0;
+            return (size_t)(v >= 1024 && v <= 65536 ? (v & ~15L) : kTileTarget);
+        }();
         open();
         for (int32_t k = 0; k < n; k++) {
             const int32_t u = order[k];
@@ -330,9 +337,11 @@ pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<
                     h.flags = kStCont | ((uint32_t)ne << kStEdgeShift);
                 }
                 std::memcpy(blob.data() + at, &h, 16);
-                for (int64_t q = 0; q < ne; q++) {
+                for (int64_t q = 0; q < 2; q++) {
                     const size_t eo = at + 16 + 16 * q;
-                    const EdgeRec32 r = edge_rec(sorted[b0 + 2 * s + q], eo);
+                    EdgeRec32 r{};
+                    if (q < ne) r = edge_rec(sorted[b0 + 2 * s + q], eo);
+                    else r.succ_pos = (int32_t)(kSuccClassNone << kSuccTcShift);   // empty slot
                     std::memcpy(blob.data() + eo, &r, 16);
                 }
                 for (int64_t q = 0; q < 2; q++)       // explicit rows: successor of each slot
@@ -366,6 +375,19 @@ pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<
             L->swap_blocked[k] = blocked ? 1 : 0;
         }
     }
+    if (L->W32 > 0) {
+        const int32_t R = (n + kRegion - 1) / kRegion;
+        L->spec_off.assign((size_t)R + 1, 0);
+        L->spec_pos.clear();
+        std::vector<int32_t> lst;
+        for (int32_t r = 0; r < R; r++) {
+            L->spec_off[r] = (uint32_t)L->spec_pos.size();
+            spec_region(g, *L, r, lst);
+            L->spec_pos.insert(L->spec_pos.end(), lst.begin(), lst.end());
+            L->spec_pos.insert(L->spec_pos.end(), (size_t)kSpecSlack, INT32_MAX);
+        }
+        L->spec_off[R] = (uint32_t)L->spec_pos.size();
+    }
     L->allowed_pos.resize(n);
     for (int32_t k = 0; k < n; k++) L->allowed_pos[k] = g->allowed[order[k]];
     if (use_cache && !x_op) {
@@ -374,6 +396,21 @@ pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<
     }
     out = L;
     return PESTO_OK;
+}
+
+void spec_region(const pesto_graph *g, const Layout &L, int32_t r, std::vector<int32_t> &out) {
+    const int32_t c = r * kRegion, e = std::min(g->n, c + kRegion);
+    out.clear();
+    for (int32_t q = c; q < e; q++) {
+        out.push_back(q);
+        const int32_t w = L.order[q];
+        for (int64_t i = g->in_off[w]; i < g->in_off[w + 1]; i++) {
+            const int32_t pq = L.pos[g->src[g->in_edges[i]]];
+            if (pq < c) out.push_back(pq);
+        }
+    }
+    std::sort(out.begin(), out.end());
+    out.erase(std::unique(out.begin(), out.end()), out.end());
 }
 
 bool pair_blocked(const pesto_graph *g, int32_t a, int32_t c) {

@@ -75,6 +75,7 @@ constexpr uint32_t kSuccPosMask = (1u << 24) - 1;
 // code) in one word and dispatches on them with a single jump table (eval32.cu push_uni)
 constexpr int kSuccTcShift = 27;
 constexpr uint32_t kSuccTcMask = 7u << kSuccTcShift;
+constexpr uint32_t kSuccClassNone = 5;          // class code of an empty edge slot of a step
 constexpr uint32_t target_class32(uint32_t target) {
     return (target & (1u << 29)) ? 4u : (((target >> 30) & 1u) << 1 | (target >> 31));
 }

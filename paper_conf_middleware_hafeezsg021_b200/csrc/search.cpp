@@ -96,6 +96,8 @@ struct pesto_search {
     // joined back into the caller's stream, beside the 32-bit launch
     cudaStream_t aux = nullptr;
     cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
+    // bases whose special-position lists overflowed during an in-place swap patch
+    std::vector<int> spec_rebuild;
 };
 
 namespace {
@@ -543,8 +545,62 @@ bool swap_in_place(pesto_search *s, int b, int32_t k, Patcher &pt) {
             const int32_t pf = ahead < n ? L.cslot[L.order[ahead]] : -1;
             pt.set32(L.d_blob32, L.blob32.data(), L.op_off32[q] + 8, ~0u, (uint32_t)pf);
         }
+        // special positions of the regions the swap can touch: the regions of k and k+1 (a and c
+        // change region when they straddle a boundary) and those of every successor of a or c
+        // (their producer positions changed); rewritten in place within each list's capacity
+        if (!L.spec_off.empty()) {
+            std::vector<int32_t> regs{k / kRegion, (k + 1) / kRegion};
+            for (int32_t op : {a, c})
+                for (int64_t i = g->out_off[op]; i < g->out_off[op + 1]; i++)
+                    regs.push_back(L.pos[g->dst[g->out_edges[i]]] / kRegion);
+            std::sort(regs.begin(), regs.end());
+            regs.erase(std::unique(regs.begin(), regs.end()), regs.end());
+            std::vector<int32_t> lst;
+            bool fits = true;
+            for (int32_t r : regs) {
+                spec_region(g, L, r, lst);
+                if (lst.size() + 1 > (size_t)(L.spec_off[r + 1] - L.spec_off[r])) fits = false;
+            }
+            if (!fits) {                     // rare: rebuild this base's lists (host + upload)
+                s->spec_rebuild.push_back(b);
+            } else {
+                for (int32_t r : regs) {
+                    spec_region(g, L, r, lst);
+                    const uint32_t o = L.spec_off[r], cap = L.spec_off[r + 1] - o;
+                    for (uint32_t i = 0; i < cap; i++) {
+                        const int32_t val = i < lst.size() ? lst[i] : INT32_MAX;
+                        if (L.spec_pos[o + i] != val) pt.set_elem(L.d_spec_pos, L.spec_pos, o + i, val);
+                    }
+                }
+            }
+        }
     }
     return true;
+}
+
+// rebuild the special-position lists of a layout whose in-place rewrite overflowed a region's
+// capacity (fresh slack everywhere), and upload them
+pesto_status rebuild_spec(pesto_graph *g, Layout &L) {
+    const int32_t n = g->n, R = (n + kRegion - 1) / kRegion;
+    L.spec_off.assign((size_t)R + 1, 0);
+    L.spec_pos.clear();
+    std::vector<int32_t> lst;
+    for (int32_t r = 0; r < R; r++) {
+        L.spec_off[r] = (uint32_t)L.spec_pos.size();
+        spec_region(g, L, r, lst);
+        L.spec_pos.insert(L.spec_pos.end(), lst.begin(), lst.end());
+        L.spec_pos.insert(L.spec_pos.end(), (size_t)kSpecSlack, INT32_MAX);
+    }
+    L.spec_off[R] = (uint32_t)L.spec_pos.size();
+    cudaError_t e;
+    if ((e = L.d_spec_off.ensure(L.spec_off.size() * 4)) != cudaSuccess ||
+        (e = cudaMemcpy(L.d_spec_off.ptr, L.spec_off.data(), L.spec_off.size() * 4,
+                        cudaMemcpyHostToDevice)) != cudaSuccess ||
+        (e = L.d_spec_pos.ensure(L.spec_pos.size() * 4)) != cudaSuccess ||
+        (e = cudaMemcpy(L.d_spec_pos.ptr, L.spec_pos.data(), L.spec_pos.size() * 4,
+                        cudaMemcpyHostToDevice)) != cudaSuccess)
+        return cuda_fail(e, "upload special positions");
+    return PESTO_OK;
 }
 
 }  // namespace
@@ -741,6 +797,12 @@ pesto_status pesto_search_commit(pesto_search *s, void *stream) {
             if ((rc = upload_layout(g, *s->layouts[b]))) return rc;
             changed = true;
         }
+        for (int b : s->spec_rebuild) {
+            pesto_status rc = rebuild_spec(g, *s->layouts[b]);
+            if (rc) return rc;
+            changed = true;                  // the list buffers may have moved: refresh views
+        }
+        s->spec_rebuild.clear();
         if (!pt.ops.empty()) {
             const size_t bytes = pt.ops.size() * sizeof(PatchOp);
             if ((e = s->d_patch.ensure(bytes)) != cudaSuccess ||

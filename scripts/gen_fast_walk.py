@@ -1,0 +1,203 @@
+"""Generates paper_conf_middleware_hafeezsg021_b200/csrc/fast_walk_ptx.inc: the eval32 search
+walk's uniform segment (D = 2, two candidates per lane, uint32 time; DESIGN.md §3.4 "fast walk")
+as one inline-PTX loop with `brx.idx.uni` jump tables.
+
+Outside its group's special positions (the region and the producers of region ops, the
+Layout::spec_pos lists) every lane of a warp has the base device of every op and successor, so a
+step's whole control path -- begin on device xu or a continuation step, then per edge: link or
+not, register / ring / cold slot, first push or max -- is a function of (xu, class, cross) of its
+<= 2 edges.  The loop runs steps until the tile's limit or the next special position and
+dispatches each step through two warp-uniform jump tables:
+  TA[first ? xu*12 + k0 : 24 + xu*12 + k0]  begin (first steps) + edge 0
+  TB[xu*12 + k1]                            edge 1
+with k = class*2 + yu (the handler knows cross = yu != xu), class 0 far, 1 far first, 2 near, 3 near first, 4 next, 5 empty slot
+(layout_format.h kSuccTcShift / kSuccClassNone).  Same arithmetic as eval32.cu's C++ step
+(PAPER.md L142-146, L188-198): C_v = min(max(r, dev_free[xu]) + p_v, SAT); a crossing edge
+A = min(max(C_v, link_free[xu -> 1-xu]) + t, SAT), link_free = A; else A = C_v.
+
+usage: python scripts/gen_fast_walk.py  (rewrites the .inc; commit both)
+"""
+import os
+
+HERE = os.path.dirname(os.path.abspath(__file__))
+OUT = os.path.join(HERE, "..", "paper_conf_middleware_hafeezsg021_b200", "csrc", "fast_walk_ptx.inc")
+
+SAT = "0xF0000000"
+
+
+def operands(cpl, wide):
+    """read-write %0 sp, %1 v, %2 xu (the walked op's base device: continuation steps carry no
+    code, so it is kept across steps and segments), then per candidate c: d0[c], d1[c], l01[c],
+    l10[c], fwd[c], nfar[c], nnear[c] (each group of cpl consecutive); inputs lim, nspec, ring,
+    stage (shared u32), cold (global u64).  wide: the exact 64-bit instance (times u64)."""
+    global SP, V, XU, D, L, FWD, NFAR, NNEAR, LIM, NSPEC, RING, STAGE, COLD, CPL, W, TY, TB_, CB
+    CPL, W = cpl, wide
+    TY = "u64" if wide else "u32"       # time type
+    TB_ = 8 if wide else 4              # bytes per time value
+    CB = 32 * TB_                       # bytes of one 32-lane column
+    k = iter(range(3, 3 + 7 * cpl + 5))
+    grp = lambda: tuple(f"%{next(k)}" for _ in range(cpl))   # noqa: E731
+    SP, V, XU = "%0", "%1", "%2"
+    D = (grp(), grp())
+    L = (grp(), grp())                 # l01 (xu 0 -> 1), l10 (xu 1 -> 0)
+    FWD, NFAR, NNEAR = grp(), grp(), grp()
+    LIM, NSPEC, RING, STAGE, COLD = (f"%{next(k)}" for _ in range(5))
+
+
+def tadd(dst, a, dur):
+    """dst = a + dur, saturated at SAT for uint32 (every duration < 2^28 so it never wraps),
+    exact for uint64; dur is a u32 record field"""
+    if W:
+        return [f"cvt.u64.u32 z, {dur};", f"add.u64 {dst}, {a}, z;"]
+    return [f"add.u32 {dst}, {a}, {dur};", f"min.u32 {dst}, {dst}, {SAT};"]
+
+
+def log2(x):
+    return x.bit_length() - 1
+
+
+def edge(xu, cls, cross, rec):
+    """PTX of one uniform edge (record registers rec = (t0, succ, target, t1))."""
+    if cls == 5:
+        return []
+    C = D[xu]
+    out = []
+    if cross:
+        t = rec[3] if xu else rec[0]
+        for c in range(CPL):
+            out += [f"max.{TY} w{c}, {C[c]}, {L[xu][c]};"] + tadd(f"w{c}", f"w{c}", t) + \
+                   [f"mov.{TY} {L[xu][c]}, w{c};"]
+        a = ("w0", "w1")[:CPL]
+    else:
+        a = C
+    if cls == 4:
+        out += [f"max.{TY} {FWD[c]}, {FWD[c]}, {a[c]};" for c in range(CPL)]
+        return out
+    # slot byte offset of the lane's column: (target & mask) x CPL x sizeof(T)/4 (the records
+    # hold offsets of 4-byte columns)
+    sh = log2(CPL * TB_ // 4)
+    out += [f"and.b32 o, {rec[2]}, 0x1FFFFFFF;"] + ([f"shl.b32 o, o, {sh};"] if sh else [])
+    if cls in (2, 3):
+        out += [f"add.u32 s, {RING}, o;"]
+        for c in range(CPL):
+            if cls == 2:
+                out += [f"ld.shared.{TY} y{c}, [s+{CB * c}];", f"max.{TY} y{c}, y{c}, {a[c]};",
+                        f"st.shared.{TY} [s+{CB * c}], y{c};"]
+            else:
+                out += [f"st.shared.{TY} [s+{CB * c}], {a[c]};"]
+    else:
+        out += ["cvt.u64.u32 g, o;", f"add.u64 g, {COLD}, g;"]
+        for c in range(CPL):
+            if cls == 1:
+                out += [f"st.global.{TY} [g+{CB * c}], {a[c]};"]
+            else:
+                out += [f"red.relaxed.gpu.global.max.{TY} [g+{CB * c}], {a[c]};"]
+    return out
+
+
+def begin(xu):
+    """C_v = min(max(r, dev_free[xu]) + p, SAT); dev_free[xu] = C_v (arrivals in r0/r1)."""
+    out = []
+    for c in range(CPL):
+        out += [f"max.{TY} w{c}, r{c}, {D[xu][c]};"] + tadd(D[xu][c], f"w{c}", "h0")
+    return out
+
+
+def kind(rec_succ, k):
+    """k = class*2 + yu: class from bits 27-29, the successor's base code yu from bit 24 (D = 2;
+    bits 25-26 are zero, so the shift leaves class*2); the handler knows cross = (yu != xu)"""
+    return [f"shr.u32 {k}, {rec_succ}, 26;", f"shr.u32 t, {rec_succ}, 24;", "and.b32 t, t, 1;",
+            f"or.b32 {k}, {k}, t;"]
+
+
+def segment(cpl, wide=False):
+    operands(cpl, wide)
+    cb = CB * cpl                       # bytes of one ring slot (cpl columns of 32 lanes)
+    sh = log2(cb)
+    A = ("a0", "a1", "a2", "a3")
+    B = ("b0", "b1", "b2", "b3")
+    ta = [f"FA{i}" for i in range(48)]
+    tb = [f"FB{i}" for i in range(24)]
+    P = []
+    P += ["{",
+          ".reg .pred p, q, q2;",
+          ".reg .u32 h0, h1, h2, h3, a0, a1, a2, a3, b0, b1, b2, b3, t, k0, k1, o, s, sz;",
+          f".reg .{TY} r0, r1, w0, w1, y0, y1;",
+          ".reg .u64 g, z;",
+          "TA: .branchtargets " + ", ".join(ta) + ";",
+          "TB: .branchtargets " + ", ".join(tb) + ";",
+          "FLOOP:",
+          f"setp.ge.u32 p, {SP}, {LIM};",
+          "@p bra.uni FDONE;",
+          f"ld.shared.v4.u32 {{h0, h1, h2, h3}}, [{SP}];",
+          f"ld.shared.v4.u32 {{a0, a1, a2, a3}}, [{SP}+16];",
+          f"ld.shared.v4.u32 {{b0, b1, b2, b3}}, [{SP}+32];",
+          "and.b32 t, h3, 16;",
+          "setp.ne.u32 q, t, 0;",
+          f"@!q and.b32 {XU}, h3, 1;"]          # first step: the op's base code (D = 2)
+    P += kind("a1", "k0") + kind("b1", "k1")
+    P += ["setp.ge.u32 q2, k1, 10;",          # step without a second edge: no TB dispatch
+          f"mad.lo.u32 k1, {XU}, 12, k1;",
+          f"mad.lo.u32 k0, {XU}, 12, k0;",
+          "@q bra.uni FCONT;",
+          # first step of the op at v + 1: leave special positions to the generic walk
+          f"add.u32 t, {V}, 1;",
+          f"setp.eq.u32 p, t, {NSPEC};",
+          "@p bra.uni FDONE;",
+          f"mov.u32 {V}, t;",
+          # far arrivals of v + 11 -> staging ring (zero-filled when the op has no far producer)
+          f"add.u32 t, {V}, 11;", "and.b32 t, t, 15;", f"shl.b32 t, t, {sh};", f"add.u32 s, {STAGE}, t;",
+          "setp.ge.s32 p, h2, 0;", "max.s32 t, h2, 0;", f"mul.wide.u32 g, t, {cb};",
+          f"add.u64 g, {COLD}, g;", f"selp.u32 sz, {TB_}, 0, p;"]
+    P += [f"cp.async.ca.shared.global [s+{CB * c}], [g+{CB * c}], {TB_}, sz;" for c in range(cpl)]
+    P += ["cp.async.commit_group;",
+          "cp.async.wait_group 10;",
+          # arrivals of v: staged far, forwarded (distance 1), near ring when flagged
+          "and.b32 t, h3, 8;", "setp.ne.u32 p, t, 0;"]
+    for c in range(cpl):
+        P += [f"selp.{TY} r{c}, {NNEAR[c]}, 0, p;", f"max.{TY} r{c}, r{c}, {NFAR[c]};",
+              f"max.{TY} r{c}, r{c}, {FWD[c]};"]
+    # read ahead the far / near arrivals of v + 1 (final once v starts)
+    P += [f"add.u32 t, {V}, 1;", "and.b32 t, t, 15;", f"shl.b32 t, t, {sh};",
+          f"add.u32 s, {STAGE}, t;"]
+    P += [f"ld.shared.{TY} {NFAR[c]}, [s+{CB * c}];" for c in range(cpl)]
+    P += [f"add.u32 s, {RING}, t;"]
+    P += [f"ld.shared.{TY} {NNEAR[c]}, [s+{CB * c}];" for c in range(cpl)]
+    P += [f"mov.{TY} {FWD[c]}, 0;" for c in range(cpl)]
+    P += ["brx.idx.uni k0, TA;",
+          "FCONT:",
+          "add.u32 k0, k0, 24;",
+          "brx.idx.uni k0, TA;"]
+    for i in range(48):
+        cont, xu, k = i // 24, (i // 12) & 1, i % 12
+        cls, cross = k // 2, int((k & 1) != xu)
+        P.append(f"FA{i}:")
+        if not cont:
+            P += begin(xu)
+        P += edge(xu, cls, cross, A)
+        P.append("@q2 bra.uni FNEXT;")
+        P.append("brx.idx.uni k1, TB;")
+    for i in range(24):
+        xu, k = i // 12, i % 12
+        cls, cross = k // 2, int((k & 1) != xu)
+        P.append(f"FB{i}:")
+        P += edge(xu, cls, cross, B)
+        if i < 23:
+            P.append("bra.uni FNEXT;")
+    P += ["FNEXT:", f"add.u32 {SP}, {SP}, 48;", "bra.uni FLOOP;", "FDONE:", "}"]
+    return P
+
+
+def main():
+    with open(OUT, "w") as f:
+        f.write("// generated by scripts/gen_fast_walk.py -- do not edit\n")
+        f.write("// eval32.cu fast_segment (DESIGN.md §3.4 fast walk): uniform steps in one PTX loop\n")
+        for cpl, wide, name in ((1, False, "1"), (2, False, "2"), (1, True, "1W")):
+            P = segment(cpl, wide)
+            f.write(f"#define PESTO_FAST_WALK_PTX{name} \\\n" +
+                    " \\\n".join('    "' + l + '\\n"' for l in P) + "\n")
+            print(OUT, name, len(P), "PTX lines")
+
+
+if __name__ == "__main__":
+    main()

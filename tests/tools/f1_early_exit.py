@@ -11,7 +11,7 @@ has.  Lower bounds after the op at position v of the candidate's order (all mono
 Prints, per config and base, the mean fraction of warp walks (positions) an exit at the first
 position where all lanes' max(LB1, LB2, LB3) >= M_b would skip, from the oracle's trace.
 
-usage: python scripts/f1_early_exit.py [config ...]  (CPU, test infrastructure: uses oracle/)
+usage: python tests/tools/f1_early_exit.py [config ...] [config=bases.npz ...]\n(CPU, test infrastructure: uses oracle/; bases.npz from tests/tools/dump_bases.py on the GPU)
 """
 import json
 import sys
@@ -55,17 +55,23 @@ def exit_position(g, tail, x, order, mk_base):
     return (int(hit[0]) + 1 if len(hit) else g.n), mk
 
 
-def main(names):
+def main(names, bases_npz=None, out_name="profiles/r2_f1_early_exit.json"):
+    """bases_npz: {config: file written by tests/tools/dump_bases.py} -- the bases after s steps
+    of the GPU search (key "x_s"/"order_s"), else the step-0 seeds"""
     out = {}
     for name in names:
         cfg = configs.CONFIGS[name]
         g = configs.graph_for(cfg)
         tail = tails(g)
-        xs, orders = seeds.bench_seeds(g, cfg.bases, configs.SEARCH_SEED)
         K = cfg.candidates_per_gpu // cfg.bases
-        rng = np.random.default_rng(0)
+        stages = [(0, seeds.bench_seeds(g, cfg.bases, configs.SEARCH_SEED))]
+        if bases_npz and name in bases_npz:
+            z = np.load(bases_npz[name])
+            stages = [(int(s), (z[f"x_{int(s)}"], z[f"order_{int(s)}"])) for s in z["steps"]]
         res = {}
-        for b in range(cfg.bases):
+        for step, (xs, orders) in stages:
+          rng = np.random.default_rng(0)
+          for b in range(cfg.bases):
             mk_b = O.makespan(g, xs[b], orders[b])
             fr, worse = [], 0
             groups = rng.choice(np.arange(1, K // 128), 6, replace=False)
@@ -74,7 +80,7 @@ def main(names):
                     pos = []
                     for j in range(128 * grp + 64 * w, 128 * grp + 64 * w + 64):
                         ok, x, o = O.candidate(g, cfg.bases, b, xs, orders, int(j),
-                                               configs.SEARCH_SEED, 0, configs.MOVE_MIX)
+                                               configs.SEARCH_SEED, step, configs.MOVE_MIX)
                         if not ok:
                             pos.append(0)
                             continue
@@ -82,12 +88,22 @@ def main(names):
                         worse += mk >= mk_b
                         pos.append(e)
                     fr.append(1.0 - max(pos) / g.n)
-            res[b] = {"base_mk": int(mk_b), "skippable_warp_fraction": float(np.mean(fr)),
-                      "warps": len(fr), "lanes_not_better": worse / (len(fr) * 64)}
-            print(name, b, res[b], flush=True)
+            res[f"step{step}_base{b}"] = {
+                "step": step, "base": b, "base_mk": int(mk_b),
+                "skippable_warp_fraction": float(np.mean(fr)), "warps": len(fr),
+                "lanes_not_better": worse / (len(fr) * 64)}
+            print(name, step, b, res[f"step{step}_base{b}"], flush=True)
         out[name] = res
-    json.dump(out, open("profiles/r2_f1_early_exit.json", "w"), indent=1)
+    json.dump(out, open(out_name, "w"), indent=1)
 
 
 if __name__ == "__main__":
-    main(sys.argv[1:] or ["inception_v3_2dev", "transformer_2dev"])
+    args = sys.argv[1:]
+    npz = {}
+    for a in list(args):
+        if a.endswith(".npz"):          # CONFIG=FILE.npz
+            k, v = a.split("=", 1)
+            npz[k] = v
+            args.remove(a)
+    main(args or ["inception_v3_2dev", "transformer_2dev"], npz,
+         "profiles/r2_f1_early_exit_steps.json" if npz else "profiles/r2_f1_early_exit.json")
