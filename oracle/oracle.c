@@ -833,17 +833,29 @@ int oracle_candidate(int32_t n, int64_t m, const int32_t *src, const int32_t *ds
         }
         return 1;
     }
-    {                                                        /* WINDOW: enumerated starts */
+    {   /* WINDOW (v7): start s enumerated over the region (visit = how many times the
+           enumeration has passed s); device d = A_s[draw(j, 4) mod |A_s|]; the window moves
+           the first L ops from s that allow d and are not on d in the base (the "eligible"
+           ops, M of them in [s, c + len)), L = 2 + (visit + draw(s, 0)) mod (M - 1): distinct
+           for every visit of s; invalid if M < 2 or every length is used */
         int64_t i = lane - b2, nw = 128 - b2;
-        int64_t s = c0 + (pass * nw + i) % rlen;
-        int64_t e = s + 1 + (int64_t)(oracle_draw(seed, step, P, b, j, 3) % 64u);
-        if (e > c0 + rlen) e = c0 + rlen;
+        int64_t w = pass * nw + i;
+        int64_t s = c0 + w % rlen, visit = w / rlen;
         int32_t na = alt_devices(allowed, D, bo[s], bx[bo[s]], alts);
         if (na == 0) return 0;
         int32_t d = alts[oracle_draw(seed, step, P, b, j, 4) % (uint64_t)na];
-        for (int64_t q = s; q < e; q++) {
+        int64_t M = 0;
+        for (int64_t q = s; q < c0 + rlen; q++)
+            if (allowed_dev(allowed, bo[q], d) && bx[bo[q]] != d) M++;
+        if (M < 2 || visit >= M - 1) return 0;
+        int64_t L = 2 + (int64_t)(((uint64_t)visit + oracle_draw(seed, step, P, b, s, 0)) %
+                                  (uint64_t)(M - 1));
+        for (int64_t q = s; L > 0; q++) {
             int32_t v = bo[q];
-            if (allowed_dev(allowed, v, d)) x_out[v] = (uint8_t)d;
+            if (allowed_dev(allowed, v, d) && bx[v] != d) {
+                x_out[v] = (uint8_t)d;
+                L--;
+            }
         }
     }
     return 1;

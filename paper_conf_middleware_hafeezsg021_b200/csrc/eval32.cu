@@ -43,6 +43,16 @@ __device__ __forceinline__ void sts_t(uint32_t addr, uint32_t v) { sts_u32(addr,
 __device__ __forceinline__ void sts_t(uint32_t addr, uint64_t v) { sts_u64(addr, v); }
 // bytes of one 32-lane column of T; record slot offsets are written for 4-byte columns
 template <class T> constexpr uint32_t kColB = 32u * sizeof(T);
+// slot layout of the ring, the staging ring and the cold slots: a slot holds 32 lanes x CPL
+// values; with two candidates per lane in 32-bit time the lane's pair sits side by side
+// (interleaved: lane base lane x 8, candidate c at +4c) so the fast walk moves the pair with one
+// 8-byte access; otherwise one 32-lane column per candidate (lane base lane x sizeof(T),
+// candidate c at +c x kColB).  A slot's byte size is CPL x kColB either way, so the records'
+// slot offsets are the same.
+constexpr bool kInterleave2 = true;
+template <int CPL, class T> constexpr bool kIL = kInterleave2 && CPL == 2 && sizeof(T) == 4;
+template <int CPL, class T> constexpr uint32_t kCandB = kIL<CPL, T> ? (uint32_t)sizeof(T) : kColB<T>;
+template <int CPL, class T> constexpr uint32_t kLaneMul = kIL<CPL, T> ? (uint32_t)CPL : 1u;
 template <class T> constexpr uint32_t kSc = sizeof(T) / 4u;
 
 // consumer warps per CTA: 256 candidates either way.  (Measured: 2-warp CTAs for CPL = 1, to
@@ -379,7 +389,7 @@ __device__ __forceinline__ void push_tail(const Ctx32 &cx, const uint32_t tgt, c
     if (tgt & kT32Near) {
 #pragma unroll
         for (int c = 0; c < CPL; c++) {
-            const uint32_t slot = cx.ring + bytes + c * kColB<T>;
+            const uint32_t slot = cx.ring + bytes + c * kCandB<CPL, T>;
             T v = a[c];
             if (!(tgt & kT32First)) v = max(v, lds_t<T>(slot));
             sts_t(slot, v);
@@ -387,7 +397,7 @@ __device__ __forceinline__ void push_tail(const Ctx32 &cx, const uint32_t tgt, c
     } else {
 #pragma unroll
         for (int c = 0; c < CPL; c++) {
-            T *slot = reinterpret_cast<T *>(cx.cold + bytes + c * kColB<T>);
+            T *slot = reinterpret_cast<T *>(cx.cold + bytes + c * kCandB<CPL, T>);
             if (tgt & kT32First) *slot = a[c];                   // first far push: plain store
             else if constexpr (sizeof(T) == 4) atomicMax(slot, a[c]);   // RED.MAX, no reply
             else atomicMax(reinterpret_cast<unsigned long long *>(slot), (unsigned long long)a[c]);
@@ -440,7 +450,7 @@ __device__ __forceinline__ void uni_edge(const Ctx32 &cx, const uint4 rec, const
         if constexpr ((F & kT32Near) != 0) {
 #pragma unroll
             for (int c = 0; c < CPL; c++) {
-                const uint32_t slot = cx.ring + bytes + c * kColB<T>;
+                const uint32_t slot = cx.ring + bytes + c * kCandB<CPL, T>;
                 T v = a[c];
                 if constexpr ((F & kT32First) == 0) v = max(v, lds_t<T>(slot));
                 sts_t(slot, v);
@@ -448,7 +458,7 @@ __device__ __forceinline__ void uni_edge(const Ctx32 &cx, const uint4 rec, const
         } else {
 #pragma unroll
             for (int c = 0; c < CPL; c++) {
-                T *slot = reinterpret_cast<T *>(cx.cold + bytes + c * kColB<T>);
+                T *slot = reinterpret_cast<T *>(cx.cold + bytes + c * kCandB<CPL, T>);
                 if constexpr ((F & kT32First) != 0) *slot = a[c];
                 else if constexpr (sizeof(T) == 4) atomicMax(slot, a[c]);
                 else atomicMax(reinterpret_cast<unsigned long long *>(slot), (unsigned long long)a[c]);
@@ -458,47 +468,60 @@ __device__ __forceinline__ void uni_edge(const Ctx32 &cx, const uint4 rec, const
 }
 #include "uni_push_ptx.inc"
 #include "fast_walk_ptx.inc"
+// the fast segment reads the next step's head one step ahead (1) or at the step's top (0)
+#ifndef PESTO_FAST_RA
+#define PESTO_FAST_RA 0
+#endif
+#if PESTO_FAST_RA
+#define PESTO_FW1 PESTO_FAST_WALK_PTX1_RA
+#define PESTO_FW2 PESTO_FAST_WALK_PTX2_RA
+#define PESTO_FW1W PESTO_FAST_WALK_PTX1W_RA
+#else
+#define PESTO_FW1 PESTO_FAST_WALK_PTX1
+#define PESTO_FW2 PESTO_FAST_WALK_PTX2
+#define PESTO_FW1W PESTO_FAST_WALK_PTX1W
+#endif
 
 // the uniform steps from sp on (until lim or the first step of the special position nspec),
 // state in registers; returns with sp at the first step it did not take
-__device__ __forceinline__ void fast_segment(uint32_t &sp, int32_t &v, uint32_t &fxu,
+__device__ __forceinline__ void fast_segment(uint32_t &sp, int32_t &v,
                                              RegState32<2, uint32_t> &st,
                                              uint32_t (&fwd)[2], uint32_t (&nfar)[2],
-                                             uint32_t (&nnear)[2], uint32_t lim, int32_t nspec,
+                                             uint32_t (&nnear)[2], uint32_t lim,
                                              uint32_t ring, uint32_t stage, const uint8_t *cold) {
-    asm volatile(PESTO_FAST_WALK_PTX2
-                 : "+r"(sp), "+r"(v), "+r"(fxu), "+r"(st.d0[0]), "+r"(st.d0[1]), "+r"(st.d1[0]), "+r"(st.d1[1]),
+    asm volatile(PESTO_FW2
+                 : "+r"(sp), "+r"(v), "+r"(st.d0[0]), "+r"(st.d0[1]), "+r"(st.d1[0]), "+r"(st.d1[1]),
                    "+r"(st.l01[0]), "+r"(st.l01[1]), "+r"(st.l10[0]), "+r"(st.l10[1]),
                    "+r"(fwd[0]), "+r"(fwd[1]), "+r"(nfar[0]), "+r"(nfar[1]), "+r"(nnear[0]),
                    "+r"(nnear[1])
-                 : "r"(lim), "r"(nspec), "r"(ring), "r"(stage), "l"(cold)
+                 : "r"(lim), "r"(ring), "r"(stage), "l"(cold)
                  : "memory");
 }
-__device__ __forceinline__ void fast_segment(uint32_t &sp, int32_t &v, uint32_t &fxu,
+__device__ __forceinline__ void fast_segment(uint32_t &sp, int32_t &v,
                                              RegState32<1, uint32_t> &st,
                                              uint32_t (&fwd)[1], uint32_t (&nfar)[1],
-                                             uint32_t (&nnear)[1], uint32_t lim, int32_t nspec,
+                                             uint32_t (&nnear)[1], uint32_t lim,
                                              uint32_t ring, uint32_t stage, const uint8_t *cold) {
-    asm volatile(PESTO_FAST_WALK_PTX1
-                 : "+r"(sp), "+r"(v), "+r"(fxu), "+r"(st.d0[0]), "+r"(st.d1[0]), "+r"(st.l01[0]),
+    asm volatile(PESTO_FW1
+                 : "+r"(sp), "+r"(v), "+r"(st.d0[0]), "+r"(st.d1[0]), "+r"(st.l01[0]),
                    "+r"(st.l10[0]), "+r"(fwd[0]), "+r"(nfar[0]), "+r"(nnear[0])
-                 : "r"(lim), "r"(nspec), "r"(ring), "r"(stage), "l"(cold)
+                 : "r"(lim), "r"(ring), "r"(stage), "l"(cold)
                  : "memory");
 }
-__device__ __forceinline__ void fast_segment(uint32_t &sp, int32_t &v, uint32_t &fxu,
+__device__ __forceinline__ void fast_segment(uint32_t &sp, int32_t &v,
                                              RegState32<1, uint64_t> &st,
                                              uint64_t (&fwd)[1], uint64_t (&nfar)[1],
-                                             uint64_t (&nnear)[1], uint32_t lim, int32_t nspec,
+                                             uint64_t (&nnear)[1], uint32_t lim,
                                              uint32_t ring, uint32_t stage, const uint8_t *cold) {
-    asm volatile(PESTO_FAST_WALK_PTX1W
-                 : "+r"(sp), "+r"(v), "+r"(fxu), "+l"(st.d0[0]), "+l"(st.d1[0]), "+l"(st.l01[0]),
+    asm volatile(PESTO_FW1W
+                 : "+r"(sp), "+r"(v), "+l"(st.d0[0]), "+l"(st.d1[0]), "+l"(st.l01[0]),
                    "+l"(st.l10[0]), "+l"(fwd[0]), "+l"(nfar[0]), "+l"(nnear[0])
-                 : "r"(lim), "r"(nspec), "r"(ring), "r"(stage), "l"(cold)
+                 : "r"(lim), "r"(ring), "r"(stage), "l"(cold)
                  : "memory");
 }
 template <int CPL, class T, class ST>
-__device__ __forceinline__ void fast_segment(uint32_t &, int32_t &, uint32_t &, ST &, T (&)[CPL], T (&)[CPL],
-                                             T (&)[CPL], uint32_t, int32_t, uint32_t, uint32_t,
+__device__ __forceinline__ void fast_segment(uint32_t &, int32_t &, ST &, T (&)[CPL], T (&)[CPL],
+                                             T (&)[CPL], uint32_t, uint32_t, uint32_t,
                                              const uint8_t *) {}
 template <int CPL, class T>
 __device__ __forceinline__ void push_uni(const Ctx32 &cx, const uint4 rec, uint32_t xm,
@@ -662,9 +685,10 @@ eval32_kernel(const EvalParams P) {
 
     Ctx32 cx;
     cx.smem = su32_reg(smem);
-    cx.ring = su32_reg(ring_all + (size_t)warp * kRing * CW + lane);
+    cx.ring = su32_reg(ring_all + (size_t)warp * kRing * CW + lane * kLaneMul<CPL, T>);
     cx.cold = reinterpret_cast<uint8_t *>(reinterpret_cast<T *>(P.state32) +
-                                          ((size_t)(blockIdx.x * NW + warp) * P.max_W32) * CW + lane);
+                                          ((size_t)(blockIdx.x * NW + warp) * P.max_W32) * CW +
+                                          lane * kLaneMul<CPL, T>);
     cx.D = P.D;
     cx.cls1 = 0;
     for (int i = 0; i < P.D * P.D; i++)
@@ -694,8 +718,8 @@ eval32_kernel(const EvalParams P) {
         const uint8_t *src = cx.cold + (size_t)(have ? h.z : 0) * CW * sizeof(T);
 #pragma unroll
         for (int c = 0; c < CPL; c++) {
-            if constexpr (sizeof(T) == 4) cp_async4_zfill(dst + c * kColB<T>, src + c * kColB<T>, have);
-            else cp_async8_zfill(dst + c * kColB<T>, src + c * kColB<T>, have);
+            if constexpr (sizeof(T) == 4) cp_async4_zfill(dst + c * kCandB<CPL, T>, src + c * kCandB<CPL, T>, have);
+            else cp_async8_zfill(dst + c * kCandB<CPL, T>, src + c * kCandB<CPL, T>, have);
         }
         cp_async_commit();
     };
@@ -706,8 +730,8 @@ eval32_kernel(const EvalParams P) {
         const uint32_t o = (uint32_t)((q & (kRing - 1)) * CPL) * kColB<T>;
 #pragma unroll
         for (int c = 0; c < CPL; c++) {
-            nfar[c] = lds_t<T>(stage + o + c * kColB<T>);
-            nnear[c] = lds_t<T>(cx.ring + o + c * kColB<T>);
+            nfar[c] = lds_t<T>(stage + o + c * kCandB<CPL, T>);
+            nnear[c] = lds_t<T>(cx.ring + o + c * kCandB<CPL, T>);
         }
     };
     auto arrivals = [&](uint32_t flags, const T (&nfar)[CPL], const T (&nnear)[CPL],
@@ -751,7 +775,6 @@ eval32_kernel(const EvalParams P) {
         int32_t nspec = INT32_MAX;
         uint32_t spi = 0;
         bool fast_ok = false, gen_op = false;
-        uint32_t fxu = 0;            // the fast segment's current op device (across segments)
         int32_t ks = -1;
         uint32_t off_ks = 0;         // search: byte offset of the op at ks in the step stream
         if (MODE == 4) {
@@ -843,7 +866,9 @@ eval32_kernel(const EvalParams P) {
         st.init();
         // positions 0 .. kPrefetchDist - 1 are never prefetched (they have no far producer)
 #pragma unroll
-        for (int q = 0; q < kRing * CPL; q++) sts_t(stage + q * kColB<T>, (T)0);
+        for (int q = 0; q < kRing; q++)
+#pragma unroll
+            for (int c = 0; c < CPL; c++) sts_t(stage + (q * CPL) * kColB<T> + c * kCandB<CPL, T>, (T)0);
 
         // the op being walked (its devices and C_v), the arrivals it forwards to v + 1, and the
         // far / near arrivals of v + 1 read ahead
@@ -943,8 +968,17 @@ eval32_kernel(const EvalParams P) {
                             if (fast_ok) {
                                 const bool is_cont = (lds_u32(sp + 12) & kStCont) != 0;
                                 if (is_cont ? !gen_op : (v + 1 != nspec)) {
-                                    fast_segment(sp, v, fxu, st, fwd, nfar, nnear, lim, nspec,
-                                                 cx.ring, stage, cx.cold);
+                                    // stop at the first step of the next special position when
+                                    // it starts in this tile (found by address, like the pair)
+                                    uint32_t flim = lim;
+                                    if (nspec < P.n) {
+                                        const uint32_t rel = __ldg(P.bases[bl].op_off32 + nspec) -
+                                                             lds_u32(cx.smem + tile + 4);
+                                        if (rel < lds_u32(cx.smem + tile + 8))
+                                            flim = min(flim, cx.smem + tile + rel);
+                                    }
+                                    fast_segment(sp, v, st, fwd, nfar, nnear, flim, cx.ring,
+                                                 stage, cx.cold);
                                     gen_op = false;
                                     continue;
                                 }

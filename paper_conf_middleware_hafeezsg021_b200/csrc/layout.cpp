@@ -262,7 +262,7 @@ pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<
         for (int64_t e = 0; e < m; e++) L->pin_off[pos[g->dst[e]] + 1]++;
         for (int32_t q = 0; q < n; q++) L->pin_off[q + 1] += L->pin_off[q];
         std::vector<uint32_t> pfill(L->pin_off.begin(), L->pin_off.end() - 1);
-        auto edge_rec = [&](int64_t e, size_t at) {
+        auto edge_rec = [&](int64_t e, size_t at, uint32_t slot) {
             EdgeRec32 r;
             if (g->D == 2) {             // by direction: t0 on link 0 -> 1, t1 on link 1 -> 0
                 r.t0 = t32(e, g->link_class[1]);
@@ -279,8 +279,8 @@ pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<
                                      : (uint32_t)cslot[w] * 128u) |
                        (first32[e] ? kT32First : 0u);
             r.succ_pos = (int32_t)((uint32_t)r.succ_pos | (target_class32(r.target) << kSuccTcShift));
-            L->pin_ref[pfill[pos[w]]++] = (uint32_t)at;
-            L->eloc32[e] = (uint32_t)at;
+            L->pin_ref[pfill[pos[w]]++] = (uint32_t)at | (slot ? kPinSlot : 0u);
+            L->eloc32[e] = (uint32_t)at | (slot ? kPinSlot : 0u);
             return r;
         };
         // tiles hold whole ops, except an op larger than a tile, which continues in the next
@@ -320,11 +320,10 @@ pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<
                 if (t_steps > 0 && blob.size() - t_start + kStepBytes > budget) { close(); open(); }
                 const size_t at = blob.size();
                 blob.resize(at + kStepBytes, 0);
-                StepHead h;
+                StepHead h{};
                 const int64_t ne = std::min<int64_t>(2, nout - 2 * s);
                 if (s == 0) {
                     h.p = (uint32_t)g->p[u];
-                    h.cold_slot = cslot[u];
                     const int32_t ahead = k + kPrefetchDist;
                     h.pf_slot = ahead < n ? cslot[order[ahead]] : -1;
                     h.flags = xcode(u) | (has_near[u] ? kStHasNear : 0u) |
@@ -332,18 +331,24 @@ pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<
                               ((uint32_t)nsteps << kStStepsShift);
                 } else {
                     h.p = 0;
-                    h.cold_slot = -1;
                     h.pf_slot = -1;
                     h.flags = kStCont | ((uint32_t)ne << kStEdgeShift);
                 }
                 std::memcpy(blob.data() + at, &h, 16);
+                uint32_t kinds = 0;
                 for (int64_t q = 0; q < 2; q++) {
                     const size_t eo = at + 16 + 16 * q;
                     EdgeRec32 r{};
-                    if (q < ne) r = edge_rec(sorted[b0 + 2 * s + q], eo);
+                    if (q < ne) r = edge_rec(sorted[b0 + 2 * s + q], eo, (uint32_t)q);
                     else r.succ_pos = (int32_t)(kSuccClassNone << kSuccTcShift);   // empty slot
                     std::memcpy(blob.data() + eo, &r, 16);
+                    // the fast walk's dispatch entry of this slot (D = 2 only)
+                    const uint32_t yu = ((uint32_t)r.succ_pos >> kSuccXShift) & 1u;
+                    const uint32_t cls = ((uint32_t)r.succ_pos >> kSuccTcShift) & 7u;
+                    if (g->D == 2)
+                        kinds |= (yu | cls << kKindClassShift | (xcode(u) ? kKindXu : 0u)) << (8 * q);
                 }
+                std::memcpy(blob.data() + at + 4, &kinds, 4);
                 for (int64_t q = 0; q < 2; q++)       // explicit rows: successor of each slot
                     L->slot_succ.push_back(q < ne ? pos[g->dst[sorted[b0 + 2 * s + q]]] : -1);
                 t_steps++;

@@ -80,6 +80,8 @@ constexpr uint32_t target_class32(uint32_t target) {
     return (target & (1u << 29)) ? 4u : (((target >> 30) & 1u) << 1 | (target >> 31));
 }
 constexpr uint32_t kPinHeavy = 1u << 31;        // patch reference into the out-of-line array
+constexpr uint32_t kPinSlot = 1u << 30;         // eval32 edge record in slot 1 of its step (else 0)
+constexpr uint32_t kPinOffMask = kPinSlot - 1;  // byte offset part of a patch reference
 constexpr uint32_t kT32First = 1u << 31;        // EdgeRec32.target: first push into its slot
 constexpr uint32_t kT32Near = 1u << 30;         // push into the near ring (slot = succ & 15)
 constexpr uint32_t kT32Next = 1u << 29;         // consumer is the next position: register
@@ -109,10 +111,16 @@ inline int edge_stride32_for(int classes) {
 // more than two distinct link classes use eval64.
 struct alignas(16) StepHead {
     uint32_t p;          // p_v (< kMaxDur32)
-    int32_t cold_slot;   // this op's cold slot (far arrivals); -1 = none
+    uint32_t kinds;      // D = 2: the fast walk's jump-table entry of each edge slot (byte k for
+                         // slot k): yu | class << 1 | xu << 4 (kKind*); 0 for D > 2
     int32_t pf_slot;     // cold slot of the op kPrefetchDist positions ahead; -1 = none
     uint32_t flags;      // base code | kStHasNear | kStCont | edges << 5 | op steps << 8
 };
+// StepHead.kinds, per slot byte: bit 0 the successor's base code yu, bits 1-3 the edge's class
+// (kSuccTcShift codes, kSuccClassNone for an empty slot), bit 4 the op's base code xu.  The
+// layout writes them; K4 keeps the yu / xu bits in step with committed placement moves, a
+// committed swap's retarget the class bits (each owner touches only its bits)
+constexpr uint32_t kKindYu = 1u, kKindClassShift = 1, kKindClassMask = 7u << 1, kKindXu = 1u << 4;
 constexpr int kStepBytes = 48;
 constexpr uint32_t kStXMask = 7u;               // bits 0-2: base device code of the op
 constexpr uint32_t kStHasNear = 1u << 3;        // read the near ring

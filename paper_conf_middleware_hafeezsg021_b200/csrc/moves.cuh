@@ -156,18 +156,32 @@ PESTO_HD LaneMove decode_lane(uint64_t seed, uint64_t cb, int64_t j, bool pure_s
         }
         return mv;
     }
-    // WINDOW: enumerated starts; the op at s always changes
+    // WINDOW (v7): enumerated starts s, the visit of s = how many times the enumeration has
+    // passed it; the window moves the first L "eligible" ops from s (allow d, not on d in the
+    // base; M of them in [s, c + len)), L = 2 + (visit + draw(s, 0)) mod (M - 1): every visit
+    // of s changes a different number of ops, so no two WINDOW candidates coincide (v6 drew the
+    // length in positions and clipped it at the region's end: 7% duplicates at 1 M per step)
     const int i = lane - b2, nw = kGroup - b2;
-    const int32_t s = rg.c + (int32_t)(((int64_t)rg.pass * nw + i) % rg.len);
-    int32_t len = 1 + (int32_t)(draw(seed, cb, j, 3) % 64u);
-    if (s + len > rg.c + rg.len) len = rg.c + rg.len - s;
+    const int64_t w = (int64_t)rg.pass * nw + i;
+    const int32_t s = rg.c + (int32_t)(w % rg.len);
+    const int64_t visit = w / rg.len;
     const unsigned am = alts(s);
     const int na = popc32(am);
     if (na == 0) { mv.kind = kMoveInvalid; return mv; }
+    const int d = nth_device(am, (int)(draw(seed, cb, j, 4) % (uint64_t)na), D);
+    auto eligible = [&](int32_t q) {
+        return ((allowed(op_at(q)) >> d) & 1u) != 0 && base_dev(q) != d;
+    };
+    int32_t M = 0;
+    for (int32_t q = s; q < rg.c + rg.len; q++) M += eligible(q) ? 1 : 0;
+    if (M < 2 || visit >= M - 1) { mv.kind = kMoveInvalid; return mv; }
+    int32_t L = 2 + (int32_t)(((uint64_t)visit + draw(seed, cb, s, 0)) % (uint64_t)(M - 1));
+    int32_t e = s;
+    while (L > 0) L -= eligible(e++) ? 1 : 0;
     mv.kind = kMoveWindow;
     mv.ws = s;
-    mv.wl = len;
-    mv.wd = nth_device(am, (int)(draw(seed, cb, j, 4) % (uint64_t)na), D);
+    mv.wl = e - s;
+    mv.wd = d;
     return mv;
 }
 

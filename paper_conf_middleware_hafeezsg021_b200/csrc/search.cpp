@@ -98,6 +98,12 @@ struct pesto_search {
     cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
     // bases whose special-position lists overflowed during an in-place swap patch
     std::vector<int> spec_rebuild;
+    // without swap moves a commit does not read the base makespans back synchronously: it
+    // copies them into pinned h_mk_async and the next eval picks them up once the copy is done
+    // (the device gates every base itself; this only stops the wide launch when none needs it)
+    int64_t *h_mk_async = nullptr;
+    cudaEvent_t ev_mk = nullptr;
+    bool mk_pending = false;
 };
 
 namespace {
@@ -201,7 +207,7 @@ pesto_status launch_search_nondelay(pesto_search *s, int b_first, int n_bases, i
 // alone would choose -- the parity path runs the instance the full step launches
 pesto_status launch_search_eval(pesto_search *s, int b_first, int n_bases, int64_t j0, int64_t j1,
                                 uint64_t *keys, uint64_t *keys_dbg, cudaStream_t st,
-                                bool fast = false, int cpl_force = 0) {
+                                bool fast = false, int cpl_force = 0, bool wide_all = false) {
     pesto_graph *g = s->g;
     if (j1 <= j0) return PESTO_OK;
     if (s->comm_gen >= 0 && s->comm_gen != g->comm_gen)
@@ -243,6 +249,11 @@ pesto_status launch_search_eval(pesto_search *s, int b_first, int n_bases, int64
     int grid = 0;
     pesto_status rc;
     cudaError_t e;
+    if (s->mk_pending && cudaEventQuery(s->ev_mk) == cudaSuccess) {   // non-blocking refresh
+        std::memcpy(s->h_mk.data(), s->h_mk_async, 8 * s->P);
+        s->mk_pending = false;
+        update_all_below(s);
+    }
     const bool use32 = fast && s->use32 && g->link_model == PESTO_LINKS_FCFS;   // f4(ii): eval64
     if (use32) {
         // eval32 tasks: consecutive ids from a multiple of the task size
@@ -254,6 +265,20 @@ pesto_status launch_search_eval(pesto_search *s, int b_first, int n_bases, int64
             const int64_t ts = eval32_task_size(cpl_force);
             p32.tasks_per_base = (j1 - (j0 - j0 % ts) + ts - 1) / ts;
             p32.n_tasks = p32.tasks_per_base * n_bases;
+        }
+        if (wide_all) {
+            // every candidate of the range on the wide (exact 64-bit) instance, whatever its
+            // base's makespan: the parity path's exact keys of saturated 32-bit walks
+            p32.gate = 0;
+            p32.wide32 = 1;
+            p32.cpl32 = 1;
+            const int64_t ts = eval32_task_size(1);
+            p32.tasks_per_base = (j1 - (j0 - j0 % ts) + ts - 1) / ts;
+            p32.n_tasks = p32.tasks_per_base * n_bases;
+            if ((rc = ensure_state32(g, g->ws, p32, 1, p32.n_tasks, &grid, true))) return rc;
+            p32.state32 = g->ws.state32w.as<uint32_t>();
+            if ((e = launch_eval32(p32, 1, grid, st)) != cudaSuccess) return cuda_fail(e, "launch wide eval32");
+            return PESTO_OK;
         }
         if ((rc = ensure_state32(g, g->ws, p32, 1, p32.n_tasks, &grid))) return rc;
         p32.state32 = g->ws.state32.as<uint32_t>();
@@ -491,7 +516,7 @@ bool swap_in_place(pesto_search *s, int b, int32_t k, Patcher &pt) {
             succ_q.erase(std::unique(succ_q.begin(), succ_q.end()), succ_q.end());
             for (int32_t q : succ_q)                  // entries into op's old block move with it
                 for (uint32_t r = L.pin_off[q]; r < L.pin_off[q + 1]; r++)
-                    if (L.pin_ref[r] >= base && L.pin_ref[r] < base + len)
+                    if ((L.pin_ref[r] & kPinOffMask) >= base && (L.pin_ref[r] & kPinOffMask) < base + len)
                         pt.set_elem(L.d_pin_ref, L.pin_ref, r, L.pin_ref[r] + shift);
             for (int64_t i = g->out_off[op]; i < g->out_off[op + 1]; i++)
                 L.eloc32[g->out_edges[i]] += shift;
@@ -527,10 +552,15 @@ bool swap_in_place(pesto_search *s, int b, int32_t k, Patcher &pt) {
                                    : cl == 1 ? (kT32Near | (uint32_t)(q & (kRing - 1)) * 128u |
                                                 (e == near_first ? kT32First : 0u))
                                              : ((uint32_t)L.cslot[w] * 128u | (e == far_first ? kT32First : 0u));
-                const uint32_t loc = L.eloc32[e];
+                const uint32_t loc = L.eloc32[e] & kPinOffMask;
+                const uint32_t slot = (L.eloc32[e] & kPinSlot) ? 1u : 0u;
                 pt.set32(L.d_blob32, L.blob32.data(), loc + 4, kSuccPosMask | kSuccTcMask,
                          (uint32_t)q | (target_class32(tgt) << kSuccTcShift));
                 pt.set32(L.d_blob32, L.blob32.data(), loc + 8, ~0u, tgt);
+                if (g->D == 2)        // the fast walk's dispatch entry of the slot: class bits
+                    pt.set32(L.d_blob32, L.blob32.data(), loc - 16 * (slot + 1) + 4,
+                             kKindClassMask << (8 * slot),
+                             (target_class32(tgt) << kKindClassShift) << (8 * slot));
             }
             pt.set32(L.d_blob32, L.blob32.data(), L.op_off32[q] + 12, kStHasNear,
                      near_first >= 0 ? kStHasNear : 0u);
@@ -766,6 +796,18 @@ pesto_status pesto_search_commit(pesto_search *s, void *stream) {
     cudaError_t e = launch_commit(cp, st);
     if (e != cudaSuccess) return cuda_fail(e, "launch commit");
     s->step++;
+    if (s->mix[3] == 0 && !s->all_below) {
+        // bases may have dropped below the 32-bit saturation point: read their makespans back
+        // asynchronously (without this the wide launch ran every step)
+        if (!s->ev_mk && (e = cudaEventCreateWithFlags(&s->ev_mk, cudaEventDisableTiming)) != cudaSuccess)
+            return cuda_fail(e, "event");
+        if (!s->h_mk_async && (e = cudaMallocHost((void **)&s->h_mk_async, 8 * s->P)) != cudaSuccess)
+            return cuda_fail(e, "pinned");
+        if ((e = cudaMemcpyAsync(s->h_mk_async, s->d_mk.ptr, 8 * s->P, cudaMemcpyDeviceToHost, st)) != cudaSuccess ||
+            (e = cudaEventRecord(s->ev_mk, st)) != cudaSuccess)
+            return cuda_fail(e, "read base makespans");
+        s->mk_pending = true;
+    }
     if (s->mix[3] > 0) {
         // a committed adjacent swap changes a base's order: rebuild its position-space layout
         if ((e = cudaMemcpyAsync(s->h_swap, s->d_swap.ptr, 4 * s->P, cudaMemcpyDeviceToHost, st)) != cudaSuccess ||
@@ -902,17 +944,31 @@ pesto_status pesto_search_candidate_keys_ex(pesto_search *s, int32_t base, int64
     if (rc || kernel == PESTO_KEYS_TIMED_RAW || !s->use32 || g->dispatch != PESTO_DISPATCH_FIXED ||
         g->link_model != PESTO_LINKS_FCFS)
         return rc;                                   // (those paths are exact 64-bit already)
-    // saturated 32-bit walks (makespan field kSat32): exact keys from the 64-bit kernel
+    // saturated 32-bit walks (makespan field kSat32): exact keys from one launch of the wide
+    // (exact 64-bit) instance over the range (round 1 re-ran each on eval64: ~1 launch per
+    // saturated id, 33 minutes on nmt4's full K)
     std::vector<uint64_t> h((size_t)(j1 - j0));
     if ((e = cudaMemcpyAsync(h.data(), keys_out, h.size() * 8, cudaMemcpyDeviceToHost, st)) != cudaSuccess ||
         (e = cudaStreamSynchronize(st)) != cudaSuccess)
         return cuda_fail(e, "read keys");
-    for (size_t i = 0; i < h.size(); i++) {
-        if (h[i] == ~0ull || (h[i] >> 24) < (uint64_t)kSat32) continue;
-        const int64_t j = j0 + (int64_t)i;
-        if ((rc = launch_search_eval(s, base, 1, j, j + 1, s->d_dbg_key.as<uint64_t>(), keys_out + i, st)))
-            return rc;
-    }
+    bool any = false;
+    for (size_t i = 0; i < h.size() && !any; i++)
+        any = h[i] != ~0ull && (h[i] >> 24) >= (uint64_t)kSat32;
+    if (!any) return PESTO_OK;
+    DevBuf wide;
+    if ((e = wide.ensure(h.size() * 8)) != cudaSuccess) return cuda_fail(e, "alloc");
+    if ((rc = launch_search_eval(s, base, 1, j0, j1, s->d_dbg_key.as<uint64_t>(), wide.as<uint64_t>(), st,
+                                 true, 0, true)))
+        return rc;
+    std::vector<uint64_t> hw(h.size());
+    if ((e = cudaMemcpyAsync(hw.data(), wide.ptr, hw.size() * 8, cudaMemcpyDeviceToHost, st)) != cudaSuccess ||
+        (e = cudaStreamSynchronize(st)) != cudaSuccess)
+        return cuda_fail(e, "read keys");
+    for (size_t i = 0; i < h.size(); i++)
+        if (h[i] != ~0ull && (h[i] >> 24) >= (uint64_t)kSat32) h[i] = hw[i];
+    if ((e = cudaMemcpyAsync(keys_out, h.data(), h.size() * 8, cudaMemcpyHostToDevice, st)) != cudaSuccess ||
+        (e = cudaStreamSynchronize(st)) != cudaSuccess)
+        return cuda_fail(e, "write keys");
     return PESTO_OK;
 }
 
@@ -1029,6 +1085,8 @@ void pesto_search_destroy(pesto_search *s) {
     if (s->aux) cudaStreamDestroy(s->aux);
     if (s->h_swap) cudaFreeHost(s->h_swap);
     if (s->h_keys) cudaFreeHost(s->h_keys);
+    if (s->h_mk_async) cudaFreeHost(s->h_mk_async);
+    if (s->ev_mk) cudaEventDestroy(s->ev_mk);
     delete s;
 }
 

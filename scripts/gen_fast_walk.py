@@ -1,17 +1,21 @@
 """Generates paper_conf_middleware_hafeezsg021_b200/csrc/fast_walk_ptx.inc: the eval32 search
 walk's uniform segment (D = 2, two candidates per lane, uint32 time; DESIGN.md §3.4 "fast walk")
-as one inline-PTX loop with `brx.idx.uni` jump tables.
+as one inline-PTX loop with `brx.idx.uni` jump tables.  With two candidates per lane (uint32)
+the lane's two values of a slot sit side by side (eval32.cu kInterleave2), so every ring,
+staging and cold access of the pair is one 8-byte access (cold-slot reductions stay 4-byte).
 
 Outside its group's special positions (the region and the producers of region ops, the
 Layout::spec_pos lists) every lane of a warp has the base device of every op and successor, so a
 step's whole control path -- begin on device xu or a continuation step, then per edge: link or
 not, register / ring / cold slot, first push or max -- is a function of (xu, class, cross) of its
-<= 2 edges.  The loop runs steps until the tile's limit or the next special position and
+<= 2 edges.  The loop runs steps until a limit address (the tile's end, the swapped pair, or
+the first step of the next special position, which the caller looks up in op_off32) and
 dispatches each step through two warp-uniform jump tables:
-  TA[first ? xu*12 + k0 : 24 + xu*12 + k0]  begin (first steps) + edge 0
-  TB[xu*12 + k1]                            edge 1
-with k = class*2 + yu (the handler knows cross = yu != xu), class 0 far, 1 far first, 2 near, 3 near first, 4 next, 5 empty slot
-(layout_format.h kSuccTcShift / kSuccClassNone).  Same arithmetic as eval32.cu's C++ step
+  TA[(continuation << 5) | k0]  begin (first steps) + edge 0
+  TB[k1]                        edge 1
+with k = yu | class << 1 | xu << 4 read from the step head (StepHead.kinds, one byte per slot,
+kept by the layout, K4 and the swap patch); the handler knows cross = (yu != xu); class 0 far,
+1 far first, 2 near, 3 near first, 4 next, 5 empty slot (layout_format.h).  Same arithmetic as eval32.cu's C++ step
 (PAPER.md L142-146, L188-198): C_v = min(max(r, dev_free[xu]) + p_v, SAT); a crossing edge
 A = min(max(C_v, link_free[xu -> 1-xu]) + t, SAT), link_free = A; else A = C_v.
 
@@ -26,22 +30,23 @@ SAT = "0xF0000000"
 
 
 def operands(cpl, wide):
-    """read-write %0 sp, %1 v, %2 xu (the walked op's base device: continuation steps carry no
-    code, so it is kept across steps and segments), then per candidate c: d0[c], d1[c], l01[c],
-    l10[c], fwd[c], nfar[c], nnear[c] (each group of cpl consecutive); inputs lim, nspec, ring,
-    stage (shared u32), cold (global u64).  wide: the exact 64-bit instance (times u64)."""
-    global SP, V, XU, D, L, FWD, NFAR, NNEAR, LIM, NSPEC, RING, STAGE, COLD, CPL, W, TY, TB_, CB
+    """read-write %0 sp, %1 v, then per candidate c: d0[c], d1[c], l01[c], l10[c], fwd[c],
+    nfar[c], nnear[c] (each group of cpl consecutive); inputs lim (the step address where the
+    segment must stop: the tile's end, the swapped pair or the first step of the next special
+    position), ring, stage (shared u32), cold (global u64).  wide: the exact 64-bit instance."""
+    global SP, V, D, L, FWD, NFAR, NNEAR, LIM, RING, STAGE, COLD, CPL, W, TY, TB_, CB, IL
     CPL, W = cpl, wide
+    IL = cpl == 2 and not wide          # a lane's two candidates side by side (8 bytes per slot)
     TY = "u64" if wide else "u32"       # time type
     TB_ = 8 if wide else 4              # bytes per time value
     CB = 32 * TB_                       # bytes of one 32-lane column
-    k = iter(range(3, 3 + 7 * cpl + 5))
+    k = iter(range(2, 2 + 7 * cpl + 4))
     grp = lambda: tuple(f"%{next(k)}" for _ in range(cpl))   # noqa: E731
-    SP, V, XU = "%0", "%1", "%2"
+    SP, V = "%0", "%1"
     D = (grp(), grp())
     L = (grp(), grp())                 # l01 (xu 0 -> 1), l10 (xu 1 -> 0)
     FWD, NFAR, NNEAR = grp(), grp(), grp()
-    LIM, NSPEC, RING, STAGE, COLD = (f"%{next(k)}" for _ in range(5))
+    LIM, RING, STAGE, COLD = (f"%{next(k)}" for _ in range(4))
 
 
 def tadd(dst, a, dur):
@@ -79,6 +84,13 @@ def edge(xu, cls, cross, rec):
     out += [f"and.b32 o, {rec[2]}, 0x1FFFFFFF;"] + ([f"shl.b32 o, o, {sh};"] if sh else [])
     if cls in (2, 3):
         out += [f"add.u32 s, {RING}, o;"]
+        if IL:                          # both candidates with one 8-byte access
+            if cls == 2:
+                out += ["ld.shared.v2.u32 {y0, y1}, [s];", f"max.u32 y0, y0, {a[0]};",
+                        f"max.u32 y1, y1, {a[1]};", "st.shared.v2.u32 [s], {y0, y1};"]
+            else:
+                out += [f"st.shared.v2.u32 [s], {{{a[0]}, {a[1]}}};"]
+            return out
         for c in range(CPL):
             if cls == 2:
                 out += [f"ld.shared.{TY} y{c}, [s+{CB * c}];", f"max.{TY} y{c}, y{c}, {a[c]};",
@@ -87,11 +99,14 @@ def edge(xu, cls, cross, rec):
                 out += [f"st.shared.{TY} [s+{CB * c}], {a[c]};"]
     else:
         out += ["cvt.u64.u32 g, o;", f"add.u64 g, {COLD}, g;"]
+        if IL and cls == 1:
+            return out + [f"st.global.v2.u32 [g], {{{a[0]}, {a[1]}}};"]
         for c in range(CPL):
+            co = 4 * c if IL else CB * c
             if cls == 1:
-                out += [f"st.global.{TY} [g+{CB * c}], {a[c]};"]
+                out += [f"st.global.{TY} [g+{co}], {a[c]};"]
             else:
-                out += [f"red.relaxed.gpu.global.max.{TY} [g+{CB * c}], {a[c]};"]
+                out += [f"red.relaxed.gpu.global.max.{TY} [g+{co}], {a[c]};"]
     return out
 
 
@@ -103,21 +118,16 @@ def begin(xu):
     return out
 
 
-def kind(rec_succ, k):
-    """k = class*2 + yu: class from bits 27-29, the successor's base code yu from bit 24 (D = 2;
-    bits 25-26 are zero, so the shift leaves class*2); the handler knows cross = (yu != xu)"""
-    return [f"shr.u32 {k}, {rec_succ}, 26;", f"shr.u32 t, {rec_succ}, 24;", "and.b32 t, t, 1;",
-            f"or.b32 {k}, {k}, t;"]
-
-
-def segment(cpl, wide=False):
+def segment(cpl, wide=False, ra=False):
+    """ra: the next step's head is read one step ahead (its kinds feed the jump-table load
+    before the current step's work; 4 register moves per step)"""
     operands(cpl, wide)
     cb = CB * cpl                       # bytes of one ring slot (cpl columns of 32 lanes)
     sh = log2(cb)
     A = ("a0", "a1", "a2", "a3")
     B = ("b0", "b1", "b2", "b3")
-    ta = [f"FA{i}" for i in range(48)]
-    tb = [f"FB{i}" for i in range(24)]
+    ta = [f"FA{i}" for i in range(64)]
+    tb = [f"FB{i}" for i in range(32)]
     P = []
     P += ["{",
           ".reg .pred p, q, q2;",
@@ -125,31 +135,41 @@ def segment(cpl, wide=False):
           f".reg .{TY} r0, r1, w0, w1, y0, y1;",
           ".reg .u64 g, z;",
           "TA: .branchtargets " + ", ".join(ta) + ";",
-          "TB: .branchtargets " + ", ".join(tb) + ";",
-          "FLOOP:",
+          "TB: .branchtargets " + ", ".join(tb) + ";"]
+    if ra:
+        P += [".reg .u32 n0, n1, n2, n3;",
+              f"ld.shared.v4.u32 {{n0, n1, n2, n3}}, [{SP}];"]
+    P += ["FLOOP:",
           f"setp.ge.u32 p, {SP}, {LIM};",
-          "@p bra.uni FDONE;",
-          f"ld.shared.v4.u32 {{h0, h1, h2, h3}}, [{SP}];",
-          f"ld.shared.v4.u32 {{a0, a1, a2, a3}}, [{SP}+16];",
+          "@p bra.uni FDONE;"]
+    if ra:                  # the tile is padded by one step: [sp + 48] is always readable
+        P += ["mov.u32 h0, n0;", "mov.u32 h1, n1;", "mov.u32 h2, n2;", "mov.u32 h3, n3;",
+              f"ld.shared.v4.u32 {{n0, n1, n2, n3}}, [{SP}+48];"]
+    else:
+        P += [f"ld.shared.v4.u32 {{h0, h1, h2, h3}}, [{SP}];"]
+    P += [f"ld.shared.v4.u32 {{a0, a1, a2, a3}}, [{SP}+16];",
           f"ld.shared.v4.u32 {{b0, b1, b2, b3}}, [{SP}+32];",
+          # the slots' jump-table entries, kept by the layout / K4 / swap patches (StepHead.kinds:
+          # yu | class << 1 | xu << 4 per slot byte)
+          "and.b32 k0, h1, 31;",
+          "shr.u32 k1, h1, 8;",
+          "and.b32 k1, k1, 31;",
+          "and.b32 t, h1, 0xE00;",
+          "setp.eq.u32 q2, t, 0xA00;",            # slot 1 empty (class 5): no TB dispatch
           "and.b32 t, h3, 16;",
           "setp.ne.u32 q, t, 0;",
-          f"@!q and.b32 {XU}, h3, 1;"]          # first step: the op's base code (D = 2)
-    P += kind("a1", "k0") + kind("b1", "k1")
-    P += ["setp.ge.u32 q2, k1, 10;",          # step without a second edge: no TB dispatch
-          f"mad.lo.u32 k1, {XU}, 12, k1;",
-          f"mad.lo.u32 k0, {XU}, 12, k0;",
           "@q bra.uni FCONT;",
-          # first step of the op at v + 1: leave special positions to the generic walk
-          f"add.u32 t, {V}, 1;",
-          f"setp.eq.u32 p, t, {NSPEC};",
-          "@p bra.uni FDONE;",
-          f"mov.u32 {V}, t;",
+          # first step of the op at v + 1 (the caller's limit stops the loop at the first step
+          # of the next special position, so every first step here is a uniform op)
+          f"add.u32 {V}, {V}, 1;",
           # far arrivals of v + 11 -> staging ring (zero-filled when the op has no far producer)
           f"add.u32 t, {V}, 11;", "and.b32 t, t, 15;", f"shl.b32 t, t, {sh};", f"add.u32 s, {STAGE}, t;",
           "setp.ge.s32 p, h2, 0;", "max.s32 t, h2, 0;", f"mul.wide.u32 g, t, {cb};",
-          f"add.u64 g, {COLD}, g;", f"selp.u32 sz, {TB_}, 0, p;"]
-    P += [f"cp.async.ca.shared.global [s+{CB * c}], [g+{CB * c}], {TB_}, sz;" for c in range(cpl)]
+          f"add.u64 g, {COLD}, g;", f"selp.u32 sz, {8 if IL else TB_}, 0, p;"]
+    if IL:
+        P += ["cp.async.ca.shared.global [s], [g], 8, sz;"]
+    else:
+        P += [f"cp.async.ca.shared.global [s+{CB * c}], [g+{CB * c}], {TB_}, sz;" for c in range(cpl)]
     P += ["cp.async.commit_group;",
           "cp.async.wait_group 10;",
           # arrivals of v: staged far, forwarded (distance 1), near ring when flagged
@@ -160,29 +180,41 @@ def segment(cpl, wide=False):
     # read ahead the far / near arrivals of v + 1 (final once v starts)
     P += [f"add.u32 t, {V}, 1;", "and.b32 t, t, 15;", f"shl.b32 t, t, {sh};",
           f"add.u32 s, {STAGE}, t;"]
-    P += [f"ld.shared.{TY} {NFAR[c]}, [s+{CB * c}];" for c in range(cpl)]
-    P += [f"add.u32 s, {RING}, t;"]
-    P += [f"ld.shared.{TY} {NNEAR[c]}, [s+{CB * c}];" for c in range(cpl)]
+    if IL:
+        P += [f"ld.shared.v2.u32 {{{NFAR[0]}, {NFAR[1]}}}, [s];", f"add.u32 s, {RING}, t;",
+              f"ld.shared.v2.u32 {{{NNEAR[0]}, {NNEAR[1]}}}, [s];"]
+    else:
+        P += [f"ld.shared.{TY} {NFAR[c]}, [s+{CB * c}];" for c in range(cpl)]
+        P += [f"add.u32 s, {RING}, t;"]
+        P += [f"ld.shared.{TY} {NNEAR[c]}, [s+{CB * c}];" for c in range(cpl)]
     P += [f"mov.{TY} {FWD[c]}, 0;" for c in range(cpl)]
     P += ["brx.idx.uni k0, TA;",
           "FCONT:",
-          "add.u32 k0, k0, 24;",
+          "add.u32 k0, k0, 32;",
           "brx.idx.uni k0, TA;"]
-    for i in range(48):
-        cont, xu, k = i // 24, (i // 12) & 1, i % 12
-        cls, cross = k // 2, int((k & 1) != xu)
+
+    def decode(e):                      # table entry -> (xu, class, cross)
+        yu, cls, xu = e & 1, (e >> 1) & 7, (e >> 4) & 1
+        return xu, cls, int(yu != xu)
+
+    for i in range(64):
+        cont, e = i >> 5, i & 31
+        xu, cls, cross = decode(e)
         P.append(f"FA{i}:")
+        if cls > 5:                     # unused entries (class codes 6, 7)
+            P.append("bra.uni FNEXT;")
+            continue
         if not cont:
             P += begin(xu)
         P += edge(xu, cls, cross, A)
         P.append("@q2 bra.uni FNEXT;")
         P.append("brx.idx.uni k1, TB;")
-    for i in range(24):
-        xu, k = i // 12, i % 12
-        cls, cross = k // 2, int((k & 1) != xu)
+    for i in range(32):
+        xu, cls, cross = decode(i)
         P.append(f"FB{i}:")
-        P += edge(xu, cls, cross, B)
-        if i < 23:
+        if cls <= 5:
+            P += edge(xu, cls, cross, B)
+        if i < 31:
             P.append("bra.uni FNEXT;")
     P += ["FNEXT:", f"add.u32 {SP}, {SP}, 48;", "bra.uni FLOOP;", "FDONE:", "}"]
     return P
@@ -192,8 +224,10 @@ def main():
     with open(OUT, "w") as f:
         f.write("// generated by scripts/gen_fast_walk.py -- do not edit\n")
         f.write("// eval32.cu fast_segment (DESIGN.md §3.4 fast walk): uniform steps in one PTX loop\n")
-        for cpl, wide, name in ((1, False, "1"), (2, False, "2"), (1, True, "1W")):
-            P = segment(cpl, wide)
+        for cpl, wide, ra, name in ((1, False, False, "1"), (2, False, False, "2"),
+                                    (1, True, False, "1W"), (1, False, True, "1_RA"),
+                                    (2, False, True, "2_RA"), (1, True, True, "1W_RA")):
+            P = segment(cpl, wide, ra)
             f.write(f"#define PESTO_FAST_WALK_PTX{name} \\\n" +
                     " \\\n".join('    "' + l + '\\n"' for l in P) + "\n")
             print(OUT, name, len(P), "PTX lines")

@@ -38,9 +38,15 @@ def test_identity_and_move_shapes(O):
     for b in range(P):                                    # different base devices)
         ok, x, o = O.candidate(g, P, b, xs, orders, 0, 2021, 3, mix)
         assert ok and (x == xs[b]).all() and (o == orders[b]).all()
+        W = mix[0] + mix[1] + mix[2]
+        b2 = (128 * (mix[0] + mix[1])) // W
         for j in range(1, 2048):
             ok, x, o = O.candidate(g, P, b, xs, orders, j, 2021, 3, mix)
-            assert ok
+            if not ok:
+                # no masks here: only a WINDOW lane can be invalid (v7: fewer than two eligible
+                # ops from its start, or every window length of that start already used)
+                assert j % 128 >= b2
+                continue
             diff_pos = np.nonzero(o != orders[b])[0]
             if len(diff_pos):
                 seen["swap"] += 1
@@ -139,10 +145,15 @@ def test_step_min_commit_and_sharding(O):
 def test_keys_equal_makespan_of_decoded_candidate(O):
     g, xs, orders = _setup(seed=13, n=30)
     keys = O.candidate_keys(g, 3, 1, xs, orders, 0, 200, 42, 9, MIX)
+    valid = 0
     for j in range(200):
         ok, x, o = O.candidate(g, 3, 1, xs, orders, j, 42, 9, MIX)
-        assert ok
+        if not ok:                                  # an invalid (v7 WINDOW) lane: no key
+            assert int(keys[j]) == 2**64 - 1
+            continue
+        valid += 1
         assert int(keys[j]) == (O.makespan(g, x, o) << 24) | j
+    assert valid > 150
 
 
 def test_coarse_group_moves_spec(O):
@@ -197,7 +208,7 @@ def test_coarse_search_step_commits_best(O):
 
 
 # ---------------------------------------------------------------------------------------------
-# Exact restatement of DESIGN.md §4 S2-S4 (spec v6) in plain Python, written from the text and
+# Exact restatement of DESIGN.md §4 S2-S4 (spec v7) in plain Python, written from the text and
 # compared element by element with the oracle's decode (oracle_candidate).
 # ---------------------------------------------------------------------------------------------
 def _py_draw(seed, step, P, b, j, k):
@@ -256,16 +267,19 @@ def _py_candidate(g, P, b, xs, orders, j, seed, step, mix, edges, preds, succs):
                 return False, x, o
             x[bo[q]] = aq[dr(j, 3 + 2 * i) % len(aq)]
         return True, x, o
-    i, nw = lane - b2, 128 - b2
-    s = c + (ps * nw + i) % ln
-    e = min(s + 1 + dr(j, 3) % 64, c + ln)
+    i, nw = lane - b2, 128 - b2                                # WINDOW (v7)
+    w = ps * nw + i
+    s, visit = c + w % ln, w // ln
     aq = A(s)
     if not aq:
         return False, x, o
     d = aq[dr(j, 4) % len(aq)]
-    for q in range(s, e):
-        if d in allowed(int(bo[q])):
-            x[bo[q]] = d
+    elig = [q for q in range(s, c + ln) if d in allowed(int(bo[q])) and int(bx[bo[q]]) != d]
+    if len(elig) < 2 or visit >= len(elig) - 1:
+        return False, x, o
+    L = 2 + (visit + dr(s, 0)) % (len(elig) - 1)
+    for q in elig[:L]:
+        x[bo[q]] = d
     return True, x, o
 
 
