@@ -307,6 +307,15 @@ pesto_status pesto_search_get(pesto_search *s, int32_t base, int64_t *makespan,
                               uint8_t *x_host, int32_t *order_host);
 int64_t pesto_search_step_count(const pesto_search *s);
 
+/* Checkpoint / resume: every draw of the search is a function of (seed, step, base,
+ * candidate id) (DESIGN.md §4 S1), so a search is fully described by its incumbents
+ * (pesto_search_get), its step counter and its creation parameters (K, mix, seed, rank/world;
+ * S9 coarse moves are re-applied by the caller).  To resume, create a search from the saved
+ * incumbents with the same parameters and set its step counter: the next step draws exactly the
+ * candidates the original would have.  step >= 0; call before the first step of the new
+ * search (synchronises).  Errors: EINVAL. */
+pesto_status pesto_search_set_step(pesto_search *s, int64_t step);
+
 /* Committed adjacent swaps so far: patched in place on the device (in_place)
  * or handled by a host rebuild of that base's layout (rebuilt).  Either pointer may be NULL.
  * Errors: EINVAL if s is NULL. */

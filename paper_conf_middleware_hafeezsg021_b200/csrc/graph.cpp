@@ -890,12 +890,14 @@ extern "C" {
 pesto_status pesto_eval_batch(pesto_graph *g, const int32_t *order, const void *placements,
                               int64_t stride, int64_t n_cand, int64_t *makespans, void *stream) {
     if (!g) return fail(PESTO_EINVAL, "NULL graph");
+    NvtxRange nvtx("pesto_eval_batch (K5 + K1)");
     return eval_batch_ws(g, g->ws, order, placements, stride, n_cand, makespans, stream);
 }
 
 pesto_status pesto_eval_batch_host(pesto_graph *g, const int32_t *order, const void *rows,
                                    int64_t stride, int64_t n_cand, int64_t *mk_host, void *stream) {
     if (!g) return fail(PESTO_EINVAL, "NULL graph");
+    NvtxRange nvtx("pesto_eval_batch_host (H2D + K5 + K1 + D2H)");
     pesto_status s = eval_batch_host_ws(g, g->ws, order, rows, stride, n_cand, mk_host, stream);
     if (s || n_cand == 0) return s;
     DeviceGuard guard(g->device);
@@ -924,6 +926,7 @@ pesto_status pesto_eval_batch_host_async(pesto_workspace *w, const int32_t *orde
                                          int64_t stride, int64_t n_cand, int64_t *mk_host,
                                          void *stream) {
     if (!w) return fail(PESTO_EINVAL, "NULL workspace");
+    NvtxRange nvtx("pesto_eval_batch_host_async");
     return eval_batch_host_ws(w->g, w->ws, order, rows, stride, n_cand, mk_host, stream);
 }
 

@@ -1,5 +1,6 @@
 // host.h -- host-side structures of libpesto (product code).
 #pragma once
+#include <nvtx3/nvToolsExt.h>
 #include <cuda_runtime.h>
 
 #include <cstdint>
@@ -21,6 +22,15 @@ pesto_status cuda_fail(cudaError_t e, const char *what);
 int64_t launch_count_value();
 
 // RAII device buffer
+// NVTX ranges (SURVEY §5 tracing): header-only NVTX 3, a no-op unless a profiler (nsys, ncu
+// --nvtx) injects itself; the C ABI's entry points name their phases
+struct NvtxRange {
+    explicit NvtxRange(const char *name) { nvtxRangePushA(name); }
+    ~NvtxRange() { nvtxRangePop(); }
+    NvtxRange(const NvtxRange &) = delete;
+    NvtxRange &operator=(const NvtxRange &) = delete;
+};
+
 struct DevBuf {
     void *ptr = nullptr;
     size_t bytes = 0;

@@ -734,6 +734,7 @@ pesto_status pesto_search_create(pesto_graph *g, const pesto_search_desc *d, pes
 
 pesto_status pesto_search_eval(pesto_search *s, void *stream) {
     if (!s) return fail(PESTO_EINVAL, "NULL search");
+    NvtxRange nvtx("pesto_search_eval (K1)");
     DeviceGuard guard(s->g->device);
     cudaStream_t st = (cudaStream_t)stream;
     s->last_stream = st;
@@ -766,6 +767,7 @@ pesto_status pesto_search_set_keys(pesto_search *s, const uint64_t *keys_host, v
 
 pesto_status pesto_search_commit(pesto_search *s, void *stream) {
     if (!s) return fail(PESTO_EINVAL, "NULL search");
+    NvtxRange nvtx("pesto_search_commit (K4)");
     pesto_graph *g = s->g;
     if (s->comm_gen != g->comm_gen)
         return fail(PESTO_ESTATE, "the comm model changed after the search was created");
@@ -903,6 +905,7 @@ pesto_status pesto_search_set_coarse_moves(pesto_search *s, const int32_t *coars
 
 pesto_status pesto_search_reduce(pesto_search *s, void *stream) {
     if (!s) return fail(PESTO_EINVAL, "NULL search");
+    NvtxRange nvtx("pesto_search_reduce (allreduce-MIN)");
     if (s->comm) {
         DeviceGuard guard(s->g->device);
         // the step's only cross-GPU exchange: global best (makespan, candidate id) per base
@@ -914,6 +917,7 @@ pesto_status pesto_search_reduce(pesto_search *s, void *stream) {
 }
 
 pesto_status pesto_search_step(pesto_search *s, void *stream) {
+    NvtxRange nvtx("pesto_search_step");
     pesto_status rc = pesto_search_eval(s, stream);
     if (rc) return rc;
     if ((rc = pesto_search_reduce(s, stream))) return rc;
@@ -1067,6 +1071,16 @@ pesto_status pesto_search_get(pesto_search *s, int32_t base, int64_t *mk, uint8_
 }
 
 int64_t pesto_search_step_count(const pesto_search *s) { return s ? s->step : -1; }
+
+pesto_status pesto_search_set_step(pesto_search *s, int64_t step) {
+    if (!s) return fail(PESTO_EINVAL, "NULL search");
+    if (step < 0) return fail(PESTO_EINVAL, "step must be >= 0");
+    DeviceGuard guard(s->g->device);
+    cudaError_t e = s->last_stream ? cudaStreamSynchronize(s->last_stream) : cudaDeviceSynchronize();
+    if (e != cudaSuccess) return cuda_fail(e, "synchronise");
+    s->step = step;
+    return PESTO_OK;
+}
 
 pesto_status pesto_search_swap_stats(const pesto_search *s, int64_t *in_place, int64_t *rebuilt) {
     if (!s) return fail(PESTO_EINVAL, "NULL search");

@@ -87,6 +87,7 @@ SIGNATURES = {
     "pesto_workspace_destroy": (None, [_VP]),
     "pesto_eval_batch_host_async": (_I32, [_VP, _VP, _VP, _I64, _I64, _VP, _VP]),
     "pesto_search_create": (_I32, [_VP, C.POINTER(SearchDesc), C.POINTER(_VP)]),
+    "pesto_search_set_step": (_I32, [_VP, _I64]),
     "pesto_search_step": (_I32, [_VP, _VP]),
     "pesto_search_eval": (_I32, [_VP, _VP]),
     "pesto_search_reduce": (_I32, [_VP, _VP]),
@@ -328,6 +329,7 @@ class Search:
         self.base_order = np.ascontiguousarray(base_order, dtype=np.int32).reshape(-1, graph.n)
         self.P = self.base_x.shape[0]
         self.K = int(k_per_base)
+        self.mix, self.seed, self.rank, self.world = tuple(int(v) for v in mix), int(seed), rank, world
         self._nid = None if nccl_id is None else (C.c_uint8 * 128)(*nccl_id)
         d = SearchDesc(self.P, _ptr(self.base_x), _ptr(self.base_order), self.K,
                        (C.c_int32 * 4)(*mix), seed, rank, world,
@@ -400,6 +402,28 @@ class Search:
     @property
     def step_count(self) -> int:
         return int(_L.pesto_search_step_count(self._h))
+
+    def set_step(self, step: int):
+        _check(_L.pesto_search_set_step(self._h, int(step)))
+
+    def checkpoint(self) -> dict:
+        """Everything a resumed search needs (pesto_search_set_step): incumbents, step, K, mix,
+        seed.  Save with np.savez(path, **ckpt)."""
+        got = [self.get(b) for b in range(self.P)]
+        return {"x": np.stack([g[1] for g in got]), "order": np.stack([g[2] for g in got]),
+                "makespan": np.asarray([g[0] for g in got], np.int64),
+                "step": np.int64(self.step_count), "k_per_base": np.int64(self.K),
+                "mix": np.asarray(self.mix, np.int32), "seed": np.uint64(self.seed)}
+
+    @classmethod
+    def resume(cls, graph: "Graph", ckpt, rank: int = 0, world: int = 1,
+               nccl_id: Optional[bytes] = None) -> "Search":
+        """A search that continues a checkpoint (a dict from checkpoint() or an np.load of it)
+        exactly: same incumbents, parameters and step counter."""
+        S = cls(graph, ckpt["x"], ckpt["order"], int(ckpt["k_per_base"]),
+                tuple(int(v) for v in ckpt["mix"]), int(ckpt["seed"]), rank, world, nccl_id)
+        S.set_step(int(ckpt["step"]))
+        return S
 
     def swap_stats(self) -> tuple:
         """(committed swaps patched in place on the device, swaps that rebuilt a layout)."""

@@ -615,3 +615,35 @@ def _cur(S):
         xs.append(x)
         os_.append(o)
     return np.stack(xs), np.stack(os_)
+
+
+def test_checkpoint_resume_continues_exactly(P, O, tmp_path):
+    """SURVEY §5 checkpoint/resume: a search saved after 3 steps (incumbents, step counter, K,
+    mix, seed) and resumed in a fresh search object takes exactly the steps the uninterrupted
+    search takes (every draw is a function of (seed, step, base, j)), swaps included; both equal
+    the oracle's reference steps."""
+    g = dag.random_dag(401, 900, 1.6, D=2, p_max=4000, max_bytes=300_000, beta0=700,
+                       beta1_fs=30_000)
+    G = P.Graph.from_arrays(g)
+    xs, orders = _bases(g, 2, seed=41)
+    K, mix, seed = 4096, (40, 20, 20, 30), 12
+    A = P.Search(G, xs, orders, K, mix, seed=seed)
+    for _ in range(3):
+        A.step()
+    ck = A.checkpoint()
+    np.savez(tmp_path / "ck.npz", **ck)
+    for _ in range(3):
+        A.step()
+    B = P.Search.resume(G, dict(np.load(tmp_path / "ck.npz")))
+    assert B.step_count == 3
+    for _ in range(3):
+        B.step()
+    rx, ro = xs.copy(), orders.copy()
+    rmk = np.asarray([O.makespan(g, rx[b], ro[b]) for b in range(2)], np.int64)
+    for step in range(6):
+        O.search_step(g, rx, ro, rmk, K, seed, step, mix)
+    for b in range(2):
+        ma, xa, oa = A.get(b)
+        mb, xb, ob = B.get(b)
+        assert ma == mb == rmk[b] and (xa == xb).all() and (oa == ob).all()
+        assert (xa == rx[b]).all() and (oa == ro[b]).all()
