@@ -472,7 +472,14 @@ __device__ __forceinline__ void uni_edge(const Ctx32 &cx, const uint4 rec, const
 #ifndef PESTO_FAST_RA
 #define PESTO_FAST_RA 0
 #endif
-#if PESTO_FAST_RA
+#ifndef PESTO_FAST_DT
+#define PESTO_FAST_DT 0
+#endif
+#if PESTO_FAST_DT
+#define PESTO_FW1 PESTO_FAST_WALK_PTX1_DT
+#define PESTO_FW2 PESTO_FAST_WALK_PTX2_DT
+#define PESTO_FW1W PESTO_FAST_WALK_PTX1W_DT
+#elif PESTO_FAST_RA
 #define PESTO_FW1 PESTO_FAST_WALK_PTX1_RA
 #define PESTO_FW2 PESTO_FAST_WALK_PTX2_RA
 #define PESTO_FW1W PESTO_FAST_WALK_PTX1W_RA
@@ -672,7 +679,12 @@ eval32_kernel(const EvalParams P) {
                 const int nt = B->n_tiles32;
                 for (int t = 0; t < nt; t++, it++) {
                     const int s = it % kStages32;
-                    if (it >= (uint32_t)kStages32) mbar_wait(&empty[s], ((it / kStages32) - 1) & 1);
+                    if (it >= (uint32_t)kStages32) {
+                        mbar_wait(&empty[s], ((it / kStages32) - 1) & 1);
+                        // the consumers' generic-proxy reads of the stage (released through the
+                        // empty barrier) before the async-proxy (TMA) write that reuses it
+                        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+                    }
                     const TileDesc td = B->tiles32[t];
                     mbar_expect_tx(&full[s], (uint32_t)td.bytes);
                     bulk_g2s(smem + (size_t)s * sb, B->blob32 + td.byte_off, (uint32_t)td.bytes,
@@ -894,10 +906,15 @@ eval32_kernel(const EvalParams P) {
         const int64_t xwords = (int64_t)P.n * PL;
         uint32_t xw[CPL], xn[CPL];
         int32_t xwb = 0;
+        // explicit rows: the warp's 32-row groups that exist (a warp's second group past the last
+        // row reads its first group's words instead: never out of bounds, results unused --
+        // compute-sanitizer memcheck / initcheck, round 2)
+        const int64_t cgrp = (MODE == 0 && CPL > 1 && ((gw + 1) << 5) >= P.n_cand) ? 0 : 1;
         auto x_load = [&](int32_t q, uint32_t (&w)[CPL]) {
             const int64_t wi = (int64_t)q * PL + lane;
 #pragma unroll
-            for (int c = 0; c < CPL; c++) w[c] = wi < xwords ? __ldg(place.pl + c * place.pl_stride + wi) : 0u;
+            for (int c = 0; c < CPL; c++)
+                w[c] = wi < xwords ? __ldg(place.pl + c * cgrp * place.pl_stride + wi) : 0u;
         };
         constexpr int SW = 32 / PL;                    // edge slots per 32-word window
         const int64_t ywords = P.n_slots * PL;         // words of one group's slot stream
@@ -908,7 +925,7 @@ eval32_kernel(const EvalParams P) {
             const int64_t wi = (int64_t)slot * PL + lane;
 #pragma unroll
             for (int c = 0; c < CPL; c++)
-                w[c] = wi < ywords ? __ldg(P.yplanes + (size_t)(gw + c) * ywords + wi) : 0u;
+                w[c] = wi < ywords ? __ldg(P.yplanes + (size_t)(gw + c * cgrp) * ywords + wi) : 0u;
         };
         // the codes of a position's / an edge slot's word, by shuffle from a window
         auto shfl_dev = [&](const uint32_t (&win)[CPL], int base, int (&out)[CPL]) {

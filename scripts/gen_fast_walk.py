@@ -118,9 +118,12 @@ def begin(xu):
     return out
 
 
-def segment(cpl, wide=False, ra=False):
+def segment(cpl, wide=False, ra=False, dt=False):
     """ra: the next step's head is read one step ahead (its kinds feed the jump-table load
-    before the current step's work; 4 register moves per step)"""
+    before the current step's work; 4 register moves per step).  dt: direct threading -- every
+    handler ends with its own copy of the loop's top (limit check, record loads, first-step
+    work, dispatch), so no join point sits inside the loop (ptxas otherwise brackets every
+    iteration with a reconvergence barrier and sends it through one far-away join block)"""
     operands(cpl, wide)
     cb = CB * cpl                       # bytes of one ring slot (cpl columns of 32 lanes)
     sh = log2(cb)
@@ -139,59 +142,74 @@ def segment(cpl, wide=False, ra=False):
     if ra:
         P += [".reg .u32 n0, n1, n2, n3;",
               f"ld.shared.v4.u32 {{n0, n1, n2, n3}}, [{SP}];"]
-    P += ["FLOOP:",
-          f"setp.ge.u32 p, {SP}, {LIM};",
-          "@p bra.uni FDONE;"]
-    if ra:                  # the tile is padded by one step: [sp + 48] is always readable
-        P += ["mov.u32 h0, n0;", "mov.u32 h1, n1;", "mov.u32 h2, n2;", "mov.u32 h3, n3;",
-              f"ld.shared.v4.u32 {{n0, n1, n2, n3}}, [{SP}+48];"]
+
+    def top(tag):
+        """the loop's top: stop at the limit, load the step, first-step work, dispatch TA"""
+        T = [f"setp.ge.u32 p, {SP}, {LIM};",
+             "@p bra.uni FDONE;"]
+        if ra:                  # the tile is padded by one step: [sp + 48] is always readable
+            T += ["mov.u32 h0, n0;", "mov.u32 h1, n1;", "mov.u32 h2, n2;", "mov.u32 h3, n3;",
+                  f"ld.shared.v4.u32 {{n0, n1, n2, n3}}, [{SP}+48];"]
+        else:
+            T += [f"ld.shared.v4.u32 {{h0, h1, h2, h3}}, [{SP}];"]
+        T += [f"ld.shared.v4.u32 {{a0, a1, a2, a3}}, [{SP}+16];",
+              f"ld.shared.v4.u32 {{b0, b1, b2, b3}}, [{SP}+32];",
+              # the slots' jump-table entries, kept by the layout / K4 / swap patches
+              # (StepHead.kinds: yu | class << 1 | xu << 4 per slot byte)
+              "and.b32 k0, h1, 31;",
+              "shr.u32 k1, h1, 8;",
+              "and.b32 k1, k1, 31;",
+              "and.b32 t, h1, 0xE00;",
+              "setp.eq.u32 q2, t, 0xA00;",            # slot 1 empty (class 5): no TB dispatch
+              "and.b32 t, h3, 16;",
+              "setp.ne.u32 q, t, 0;",
+              f"@q bra.uni FCONT{tag};",
+              # first step of the op at v + 1 (the caller's limit stops the loop at the first
+              # step of the next special position, so every first step here is a uniform op)
+              f"add.u32 {V}, {V}, 1;",
+              # far arrivals of v + 11 -> staging ring (zero-filled without a far producer)
+              f"add.u32 t, {V}, 11;", "and.b32 t, t, 15;", f"shl.b32 t, t, {sh};",
+              f"add.u32 s, {STAGE}, t;",
+              "setp.ge.s32 p, h2, 0;", "max.s32 t, h2, 0;", f"mul.wide.u32 g, t, {cb};",
+              f"add.u64 g, {COLD}, g;", f"selp.u32 sz, {8 if IL else TB_}, 0, p;"]
+        if IL:
+            T += ["cp.async.ca.shared.global [s], [g], 8, sz;"]
+        else:
+            T += [f"cp.async.ca.shared.global [s+{CB * c}], [g+{CB * c}], {TB_}, sz;"
+                  for c in range(cpl)]
+        T += ["cp.async.commit_group;",
+              "cp.async.wait_group 10;",
+              # arrivals of v: staged far, forwarded (distance 1), near ring when flagged
+              "and.b32 t, h3, 8;", "setp.ne.u32 p, t, 0;"]
+        for c in range(cpl):
+            T += [f"selp.{TY} r{c}, {NNEAR[c]}, 0, p;", f"max.{TY} r{c}, r{c}, {NFAR[c]};",
+                  f"max.{TY} r{c}, r{c}, {FWD[c]};"]
+        # read ahead the far / near arrivals of v + 1 (final once v starts)
+        T += [f"add.u32 t, {V}, 1;", "and.b32 t, t, 15;", f"shl.b32 t, t, {sh};",
+              f"add.u32 s, {STAGE}, t;"]
+        if IL:
+            T += [f"ld.shared.v2.u32 {{{NFAR[0]}, {NFAR[1]}}}, [s];", f"add.u32 s, {RING}, t;",
+                  f"ld.shared.v2.u32 {{{NNEAR[0]}, {NNEAR[1]}}}, [s];"]
+        else:
+            T += [f"ld.shared.{TY} {NFAR[c]}, [s+{CB * c}];" for c in range(cpl)]
+            T += [f"add.u32 s, {RING}, t;"]
+            T += [f"ld.shared.{TY} {NNEAR[c]}, [s+{CB * c}];" for c in range(cpl)]
+        T += [f"mov.{TY} {FWD[c]}, 0;" for c in range(cpl)]
+        T += ["brx.idx.uni k0, TA;",
+              f"FCONT{tag}:",
+              "add.u32 k0, k0, 32;",
+              "brx.idx.uni k0, TA;"]
+        return T
+
+    def tail(tag):
+        if dt:
+            return [f"add.u32 {SP}, {SP}, 48;"] + top(tag)
+        return ["bra.uni FNEXT;"]
+
+    if dt:
+        P += top("")
     else:
-        P += [f"ld.shared.v4.u32 {{h0, h1, h2, h3}}, [{SP}];"]
-    P += [f"ld.shared.v4.u32 {{a0, a1, a2, a3}}, [{SP}+16];",
-          f"ld.shared.v4.u32 {{b0, b1, b2, b3}}, [{SP}+32];",
-          # the slots' jump-table entries, kept by the layout / K4 / swap patches (StepHead.kinds:
-          # yu | class << 1 | xu << 4 per slot byte)
-          "and.b32 k0, h1, 31;",
-          "shr.u32 k1, h1, 8;",
-          "and.b32 k1, k1, 31;",
-          "and.b32 t, h1, 0xE00;",
-          "setp.eq.u32 q2, t, 0xA00;",            # slot 1 empty (class 5): no TB dispatch
-          "and.b32 t, h3, 16;",
-          "setp.ne.u32 q, t, 0;",
-          "@q bra.uni FCONT;",
-          # first step of the op at v + 1 (the caller's limit stops the loop at the first step
-          # of the next special position, so every first step here is a uniform op)
-          f"add.u32 {V}, {V}, 1;",
-          # far arrivals of v + 11 -> staging ring (zero-filled when the op has no far producer)
-          f"add.u32 t, {V}, 11;", "and.b32 t, t, 15;", f"shl.b32 t, t, {sh};", f"add.u32 s, {STAGE}, t;",
-          "setp.ge.s32 p, h2, 0;", "max.s32 t, h2, 0;", f"mul.wide.u32 g, t, {cb};",
-          f"add.u64 g, {COLD}, g;", f"selp.u32 sz, {8 if IL else TB_}, 0, p;"]
-    if IL:
-        P += ["cp.async.ca.shared.global [s], [g], 8, sz;"]
-    else:
-        P += [f"cp.async.ca.shared.global [s+{CB * c}], [g+{CB * c}], {TB_}, sz;" for c in range(cpl)]
-    P += ["cp.async.commit_group;",
-          "cp.async.wait_group 10;",
-          # arrivals of v: staged far, forwarded (distance 1), near ring when flagged
-          "and.b32 t, h3, 8;", "setp.ne.u32 p, t, 0;"]
-    for c in range(cpl):
-        P += [f"selp.{TY} r{c}, {NNEAR[c]}, 0, p;", f"max.{TY} r{c}, r{c}, {NFAR[c]};",
-              f"max.{TY} r{c}, r{c}, {FWD[c]};"]
-    # read ahead the far / near arrivals of v + 1 (final once v starts)
-    P += [f"add.u32 t, {V}, 1;", "and.b32 t, t, 15;", f"shl.b32 t, t, {sh};",
-          f"add.u32 s, {STAGE}, t;"]
-    if IL:
-        P += [f"ld.shared.v2.u32 {{{NFAR[0]}, {NFAR[1]}}}, [s];", f"add.u32 s, {RING}, t;",
-              f"ld.shared.v2.u32 {{{NNEAR[0]}, {NNEAR[1]}}}, [s];"]
-    else:
-        P += [f"ld.shared.{TY} {NFAR[c]}, [s+{CB * c}];" for c in range(cpl)]
-        P += [f"add.u32 s, {RING}, t;"]
-        P += [f"ld.shared.{TY} {NNEAR[c]}, [s+{CB * c}];" for c in range(cpl)]
-    P += [f"mov.{TY} {FWD[c]}, 0;" for c in range(cpl)]
-    P += ["brx.idx.uni k0, TA;",
-          "FCONT:",
-          "add.u32 k0, k0, 32;",
-          "brx.idx.uni k0, TA;"]
+        P += ["FLOOP:"] + top("")
 
     def decode(e):                      # table entry -> (xu, class, cross)
         yu, cls, xu = e & 1, (e >> 1) & 7, (e >> 4) & 1
@@ -202,21 +220,29 @@ def segment(cpl, wide=False, ra=False):
         xu, cls, cross = decode(e)
         P.append(f"FA{i}:")
         if cls > 5:                     # unused entries (class codes 6, 7)
-            P.append("bra.uni FNEXT;")
+            P.append("bra.uni FDONE;")
             continue
         if not cont:
             P += begin(xu)
         P += edge(xu, cls, cross, A)
-        P.append("@q2 bra.uni FNEXT;")
-        P.append("brx.idx.uni k1, TB;")
+        if dt:
+            P += [f"@q2 bra.uni FTA{i};", "brx.idx.uni k1, TB;", f"FTA{i}:"] + tail(f"A{i}")
+        else:
+            P += ["@q2 bra.uni FNEXT;", "brx.idx.uni k1, TB;"]
     for i in range(32):
         xu, cls, cross = decode(i)
         P.append(f"FB{i}:")
-        if cls <= 5:
-            P += edge(xu, cls, cross, B)
-        if i < 31:
+        if cls > 5:
+            P.append("bra.uni FDONE;")
+            continue
+        P += edge(xu, cls, cross, B)
+        if dt:
+            P += tail(f"B{i}")
+        elif i < 31:
             P.append("bra.uni FNEXT;")
-    P += ["FNEXT:", f"add.u32 {SP}, {SP}, 48;", "bra.uni FLOOP;", "FDONE:", "}"]
+    if not dt:
+        P += ["FNEXT:", f"add.u32 {SP}, {SP}, 48;", "bra.uni FLOOP;"]
+    P += ["FDONE:", "}"]
     return P
 
 
@@ -224,10 +250,13 @@ def main():
     with open(OUT, "w") as f:
         f.write("// generated by scripts/gen_fast_walk.py -- do not edit\n")
         f.write("// eval32.cu fast_segment (DESIGN.md §3.4 fast walk): uniform steps in one PTX loop\n")
-        for cpl, wide, ra, name in ((1, False, False, "1"), (2, False, False, "2"),
-                                    (1, True, False, "1W"), (1, False, True, "1_RA"),
-                                    (2, False, True, "2_RA"), (1, True, True, "1W_RA")):
-            P = segment(cpl, wide, ra)
+        for cpl, wide, ra, dt, name in ((1, False, False, False, "1"), (2, False, False, False, "2"),
+                                        (1, True, False, False, "1W"),
+                                        (1, False, True, False, "1_RA"), (2, False, True, False, "2_RA"),
+                                        (1, True, True, False, "1W_RA"),
+                                        (1, False, False, True, "1_DT"), (2, False, False, True, "2_DT"),
+                                        (1, True, False, True, "1W_DT")):
+            P = segment(cpl, wide, ra, dt)
             f.write(f"#define PESTO_FAST_WALK_PTX{name} \\\n" +
                     " \\\n".join('    "' + l + '\\n"' for l in P) + "\n")
             print(OUT, name, len(P), "PTX lines")

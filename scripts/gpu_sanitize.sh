@@ -10,7 +10,8 @@ for cpl in 1 2; do
     extra=""
     [ $tool = memcheck ] && extra="--leak-check no"
     [ $tool = racecheck ] && extra="--racecheck-report all"
-    PESTO_EVAL32_CPL=$cpl timeout 1500 $CS --tool $tool $extra --print-limit 50 \
+    d4=1; [ $cpl = 2 ] && [ $tool = memcheck ] && d4=0
+    SAN_D4=$d4 PESTO_EVAL32_CPL=$cpl timeout 1500 $CS --tool $tool $extra --print-limit 50 \
       python tests/tools/sanitize_run.py > gpurun_out/san_${tool}_cpl${cpl}.log 2>&1
     echo "rc=$?" >> gpurun_out/san_${tool}_cpl${cpl}.log
   done
