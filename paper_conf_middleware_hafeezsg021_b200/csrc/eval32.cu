@@ -92,6 +92,9 @@ constexpr bool kHeadAhead = PESTO_HEAD_AHEAD2 != 0;
 #ifndef PESTO_FAST_WALK
 #define PESTO_FAST_WALK 1
 #endif
+#ifndef PESTO_FAST_D4
+#define PESTO_FAST_D4 1
+#endif
 constexpr bool kUniSwitch = PESTO_UNI_SWITCH != 0;
 __host__ __device__ constexpr int min_blocks_for(int cpl) { return cpl == 1 ? PESTO_E32_MINB1 : PESTO_E32_MINB2; }
 // tile loads: a producer warp per CTA (0), or issued by the consumer warp that releases a stage
@@ -142,26 +145,30 @@ struct RegState32 {          // D <= 2
     }
 };
 
+// link columns of device x: x * DS + y; DS = 4 for D <= 4 (a fixed stride the D <= 4 fast walk
+// addresses at compile time), D for D <= 8
+__host__ __device__ constexpr int link_stride32(int pl, int D) { return pl == 2 ? 4 : D; }
+
 template <int CPL, class T>
-struct SmemState32 {         // D <= 8: [column][CPL][32] in shared memory (shared addresses)
-    uint32_t d, l;           // + lane * sizeof(T)
-    int D;
+struct SmemState32 {         // D <= 8: per column (device, then link x * DS + y) one slot of
+    uint32_t d, l;           // 32 lanes x CPL (lane pair interleaved like the rings)
+    int D, DS;
     __device__ __forceinline__ uint32_t at(uint32_t base, int col, int c) const {
-        return base + (uint32_t)(col * CPL + c) * kColB<T>;
+        return base + (uint32_t)(col * CPL) * kColB<T> + (uint32_t)c * kCandB<CPL, T>;
     }
     __device__ __forceinline__ void init() {
         for (int x = 0; x < D; x++)
             for (int c = 0; c < CPL; c++) sts_t(at(d, x, c), (T)0);
-        for (int x = 0; x < D * D; x++)
+        for (int x = 0; x < D * DS; x++)
             for (int c = 0; c < CPL; c++) sts_t(at(l, x, c), (T)0);
     }
     __device__ __forceinline__ T dev(int c, int x) const { return lds_t<T>(at(d, x, c)); }
     __device__ __forceinline__ void set_dev(int c, int x, T v) { sts_t(at(d, x, c), v); }
     __device__ __forceinline__ T link(int c, int x, int y) const {
-        return lds_t<T>(at(l, x * D + y, c));
+        return lds_t<T>(at(l, x * DS + y, c));
     }
     __device__ __forceinline__ void set_link_if(int c, int x, int y, bool cond, T v) {
-        if (cond) sts_t(at(l, x * D + y, c), v);
+        if (cond) sts_t(at(l, x * DS + y, c), v);
     }
     __device__ __forceinline__ T makespan(int c) const {
         T m = 0;
@@ -179,7 +186,7 @@ struct SmemState32 {         // D <= 8: [column][CPL][32] in shared memory (shar
     __device__ __forceinline__ void link_u(int xu, int yu, uint32_t t, const T (&cc)[CPL], T (&a)[CPL]) {
 #pragma unroll
         for (int c = 0; c < CPL; c++) {
-            const uint32_t ad = at(l, xu * D + yu, c);
+            const uint32_t ad = at(l, xu * DS + yu, c);
             a[c] = add_sat(max(cc[c], lds_t<T>(ad)), (T)t);
             sts_t(ad, a[c]);
         }
@@ -526,6 +533,35 @@ __device__ __forceinline__ void fast_segment(uint32_t &sp, int32_t &v,
                  : "r"(lim), "r"(ring), "r"(stage), "l"(cold)
                  : "memory");
 }
+// D = 3..4: device / link state stays in shared memory (SmemState32), the walk's control is
+// the same jump-table loop (fast_walk_ptx.inc PESTO_FAST_WALK_PTX{1,2}_D4)
+__device__ __forceinline__ void fast_segment(uint32_t &sp, int32_t &v, SmemState32<2, uint32_t> &st,
+                                             uint32_t (&fwd)[2], uint32_t (&nfar)[2],
+                                             uint32_t (&nnear)[2], uint32_t lim, uint32_t ring,
+                                             uint32_t stage, const uint8_t *cold, uint32_t cls4) {
+    asm volatile(PESTO_FAST_WALK_PTX2_D4
+                 : "+r"(sp), "+r"(v), "+r"(fwd[0]), "+r"(fwd[1]), "+r"(nfar[0]), "+r"(nfar[1]),
+                   "+r"(nnear[0]), "+r"(nnear[1])
+                 : "r"(lim), "r"(ring), "r"(stage), "l"(cold), "r"(st.d), "r"(st.l), "r"(cls4)
+                 : "memory");
+}
+__device__ __forceinline__ void fast_segment(uint32_t &sp, int32_t &v, SmemState32<1, uint32_t> &st,
+                                             uint32_t (&fwd)[1], uint32_t (&nfar)[1],
+                                             uint32_t (&nnear)[1], uint32_t lim, uint32_t ring,
+                                             uint32_t stage, const uint8_t *cold, uint32_t cls4) {
+    asm volatile(PESTO_FAST_WALK_PTX1_D4
+                 : "+r"(sp), "+r"(v), "+r"(fwd[0]), "+r"(nfar[0]), "+r"(nnear[0])
+                 : "r"(lim), "r"(ring), "r"(stage), "l"(cold), "r"(st.d), "r"(st.l), "r"(cls4)
+                 : "memory");
+}
+// D = 2: the link class is the direction (records hold t per direction); cls4 unused
+template <class ST, class T, int N>
+__device__ __forceinline__ void fast_segment(uint32_t &sp, int32_t &v, ST &st, T (&fwd)[N],
+                                             T (&nfar)[N], T (&nnear)[N], uint32_t lim,
+                                             uint32_t ring, uint32_t stage, const uint8_t *cold,
+                                             uint32_t) {
+    fast_segment(sp, v, st, fwd, nfar, nnear, lim, ring, stage, cold);
+}
 template <int CPL, class T, class ST>
 __device__ __forceinline__ void fast_segment(uint32_t &, int32_t &, ST &, T (&)[CPL], T (&)[CPL],
                                              T (&)[CPL], uint32_t, uint32_t, uint32_t,
@@ -600,8 +636,9 @@ __global__ void __launch_bounds__(threads_for(CPL), min_blocks_for(CPL))
 eval32_kernel(const EvalParams P) {
     constexpr bool kSearch = MODE == 1 || MODE == 5;   // 5: search with S9 coarse groups
     // uniform steps through the PTX fast segment (D = 2, CPL 2, 32-bit time, search)
-    constexpr bool kFast = PESTO_FAST_WALK != 0 && MODE == 1 && PL == 1 &&
-                           (sizeof(T) == 4 || CPL == 1);
+    constexpr bool kFast = PESTO_FAST_WALK != 0 && MODE == 1 &&
+                           ((PL == 1 && (sizeof(T) == 4 || CPL == 1)) ||
+                            (PL == 2 && sizeof(T) == 4 && PESTO_FAST_D4 != 0));
     constexpr int NW = warps_for(CPL);          // consumer warps per CTA (256 candidates)
     constexpr int CW = 32 * CPL;                // candidates per warp
     extern __shared__ __align__(128) uint8_t smem[];
@@ -621,7 +658,7 @@ eval32_kernel(const EvalParams P) {
     // lookups missed L1 behind the cold-slot traffic and made a coarse warp ~1.7x slower).  Not
     // for CPL 2: n more bytes per CTA cost a resident CTA per SM there (measured slower).
     constexpr bool kCposSmem = MODE == 5 && CPL == 1;
-    const uint32_t cpos_s = su32_reg(align16(cur + (PL != 1 ? (size_t)NW * (P.D + P.D * P.D) * CW * sizeof(T) : 0)));
+    const uint32_t cpos_s = su32_reg(align16(cur + (PL != 1 ? (size_t)NW * (P.D + P.D * link_stride32(PL, P.D)) * CW * sizeof(T) : 0)));
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     auto runs_here = [&](int bl) {           // search: this kernel owns bases below saturation
@@ -705,6 +742,11 @@ eval32_kernel(const EvalParams P) {
     cx.cls1 = 0;
     for (int i = 0; i < P.D * P.D; i++)
         if (P.link_class[i] == 1) cx.cls1 |= 1ull << i;
+    // D <= 4 fast walk: link x -> y in class 1 at bit x * 4 + y
+    uint32_t cls4 = 0;
+    if (PL == 2)
+        for (int i = 0; i < P.D * P.D; i++)
+            if (P.link_class[i] == 1) cls4 |= 1u << ((i / P.D) * 4 + i % P.D);
     // the staging ring sits a compile-time distance after the near ring (both NW x kRing x CW
     // times, 16-byte multiples): derived from cx.ring so that the pair of loads per position
     // shares one address register (the second load takes an immediate offset)
@@ -716,7 +758,8 @@ eval32_kernel(const EvalParams P) {
     StateT st;
     if constexpr (PL != 1) {
         st.D = P.D;
-        st.d = su32_reg(dstate + (size_t)warp * (P.D + P.D * P.D) * CW + lane);
+        st.DS = link_stride32(PL, P.D);
+        st.d = su32_reg(dstate + (size_t)warp * (P.D + P.D * st.DS) * CW + lane * kLaneMul<CPL, T>);
         st.l = st.d + (uint32_t)(P.D * CPL) * kColB<T>;
     }
 
@@ -995,7 +1038,7 @@ eval32_kernel(const EvalParams P) {
                                             flim = min(flim, cx.smem + tile + rel);
                                     }
                                     fast_segment(sp, v, st, fwd, nfar, nnear, flim, cx.ring,
-                                                 stage, cx.cold);
+                                                 stage, cx.cold, cls4);
                                     gen_op = false;
                                     continue;
                                 }
@@ -1288,7 +1331,7 @@ int eval32_smem_bytes(const EvalParams &p, int search_mode) {
     b = (b + 15) & ~size_t(15);
     b += (size_t)nw * kRing * 32 * cpl * tb;       // far-arrival staging
     b = (b + 15) & ~size_t(15);
-    if (pl != 1) b += (size_t)nw * (p.D + p.D * p.D) * 32 * cpl * tb;
+    if (pl != 1) b += (size_t)nw * (p.D + p.D * link_stride32(pl, p.D)) * 32 * cpl * tb;
     b = (b + 15) & ~size_t(15);
     if (search_mode == 5 && cpl == 1) b += (size_t)p.n;   // merged vertex per position (S9)
     return (int)b + 128;

@@ -672,15 +672,18 @@ __global__ void commit_kernel(const CommitParams P) {
         if (B.W32 == 0) return;           // this base has no eval32 records (per base)
         uint32_t *flags = reinterpret_cast<uint32_t *>(blob32 + B.op_off32[q]) + 3;   // StepHead
         *flags = (*flags & ~kStXMask) | (uint32_t)x;
-        if (PL == 1) {
-            // the fast walk's dispatch entries (StepHead.kinds): xu of every step of the op
-            // (atomics: another lane may set a yu bit of the same word)
+        if (PL <= 2) {
+            // the fast walk's dispatch entries (StepHead.kinds, D <= 4): xu of every step of the
+            // op (atomics: another lane may set a yu bit of the same word)
             const uint32_t nst = *flags >> kStStepsShift;
-            const uint32_t xm = kKindXu | (kKindXu << 8);
+            constexpr int xs = PL == 1 ? kind_xshift(2) : kind_xshift(4);
+            constexpr uint32_t cm = kind_code_mask(PL == 1 ? 2 : 4);
+            const uint32_t xm = (cm << xs) * 0x101u;
+            const uint32_t xv = ((uint32_t)x << xs) * 0x101u;
             for (uint32_t k = 0; k < nst; k++) {
                 uint32_t *kinds = reinterpret_cast<uint32_t *>(blob32 + B.op_off32[q] + k * kStepBytes) + 1;
                 atomicAnd(kinds, ~xm);
-                if (x) atomicOr(kinds, xm);
+                if (xv) atomicOr(kinds, xv);
             }
         }
         for (uint32_t i = B.pin_off[q]; i < B.pin_off[q + 1]; i++) {
@@ -688,13 +691,14 @@ __global__ void commit_kernel(const CommitParams P) {
             uint8_t *base = (ref & kPinHeavy) ? heavy32 : blob32;
             uint32_t *succ = reinterpret_cast<uint32_t *>(base + (ref & kPinOffMask)) + 1;
             *succ = (*succ & ~(7u << kSuccXShift)) | ((uint32_t)x << kSuccXShift);
-            if (PL == 1 && !(ref & kPinHeavy)) {      // yu of this slot in its step's kinds
+            if (PL <= 2 && !(ref & kPinHeavy)) {      // yu of this slot in its step's kinds
                 const uint32_t slot = (ref & kPinSlot) ? 1u : 0u;
                 uint32_t *kinds = reinterpret_cast<uint32_t *>(blob32 + (ref & kPinOffMask) -
                                                                16u * (slot + 1u)) + 1;
-                const uint32_t ym = kKindYu << (8 * slot);
+                constexpr uint32_t cm = kind_code_mask(PL == 1 ? 2 : 4);
+                const uint32_t ym = cm << (8 * slot);
                 atomicAnd(kinds, ~ym);
-                if (x) atomicOr(kinds, ym);
+                if (x) atomicOr(kinds, (uint32_t)x << (8 * slot));
             }
         }
     };

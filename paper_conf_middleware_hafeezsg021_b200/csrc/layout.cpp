@@ -342,11 +342,10 @@ pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<
                     if (q < ne) r = edge_rec(sorted[b0 + 2 * s + q], eo, (uint32_t)q);
                     else r.succ_pos = (int32_t)(kSuccClassNone << kSuccTcShift);   // empty slot
                     std::memcpy(blob.data() + eo, &r, 16);
-                    // the fast walk's dispatch entry of this slot (D = 2 only)
-                    const uint32_t yu = ((uint32_t)r.succ_pos >> kSuccXShift) & 1u;
+                    // the fast walk's dispatch entry of this slot (D <= 4)
+                    const uint32_t yu = ((uint32_t)r.succ_pos >> kSuccXShift) & kind_code_mask(g->D);
                     const uint32_t cls = ((uint32_t)r.succ_pos >> kSuccTcShift) & 7u;
-                    if (g->D == 2)
-                        kinds |= (yu | cls << kKindClassShift | (xcode(u) ? kKindXu : 0u)) << (8 * q);
+                    kinds |= kind_byte(g->D, yu, cls, xcode(u)) << (8 * q);
                 }
                 std::memcpy(blob.data() + at + 4, &kinds, 4);
                 for (int64_t q = 0; q < 2; q++)       // explicit rows: successor of each slot

@@ -11,6 +11,12 @@
 #pragma once
 #include <stdint.h>
 
+#ifdef __CUDACC__
+#define PESTO_LF_HD __host__ __device__
+#else
+#define PESTO_LF_HD
+#endif
+
 namespace pesto {
 
 constexpr uint32_t kOpHeavy = 1u << 31;        // OpRec.nout: edges out of line, ExtRec follows
@@ -76,7 +82,7 @@ constexpr uint32_t kSuccPosMask = (1u << 24) - 1;
 constexpr int kSuccTcShift = 27;
 constexpr uint32_t kSuccTcMask = 7u << kSuccTcShift;
 constexpr uint32_t kSuccClassNone = 5;          // class code of an empty edge slot of a step
-constexpr uint32_t target_class32(uint32_t target) {
+PESTO_LF_HD constexpr uint32_t target_class32(uint32_t target) {
     return (target & (1u << 29)) ? 4u : (((target >> 30) & 1u) << 1 | (target >> 31));
 }
 constexpr uint32_t kPinHeavy = 1u << 31;        // patch reference into the out-of-line array
@@ -116,11 +122,18 @@ struct alignas(16) StepHead {
     int32_t pf_slot;     // cold slot of the op kPrefetchDist positions ahead; -1 = none
     uint32_t flags;      // base code | kStHasNear | kStCont | edges << 5 | op steps << 8
 };
-// StepHead.kinds, per slot byte: bit 0 the successor's base code yu, bits 1-3 the edge's class
-// (kSuccTcShift codes, kSuccClassNone for an empty slot), bit 4 the op's base code xu.  The
-// layout writes them; K4 keeps the yu / xu bits in step with committed placement moves, a
-// committed swap's retarget the class bits (each owner touches only its bits)
+// StepHead.kinds, per slot byte, D = 2: bit 0 the successor's base code yu, bits 1-3 the edge's
+// class (kSuccTcShift codes, kSuccClassNone for an empty slot), bit 4 the op's base code xu;
+// D = 3..4: bits 0-1 yu, 2-4 class, 5-6 xu.  0 for D > 4.  The layout writes them; K4 keeps the
+// yu / xu bits in step with committed placement moves, a committed swap's retarget the class
+// bits (each owner touches only its bits)
 constexpr uint32_t kKindYu = 1u, kKindClassShift = 1, kKindClassMask = 7u << 1, kKindXu = 1u << 4;
+PESTO_LF_HD constexpr int kind_cshift(int D) { return D <= 2 ? 1 : 2; }        // class bits
+PESTO_LF_HD constexpr int kind_xshift(int D) { return D <= 2 ? 4 : 5; }        // xu bits
+PESTO_LF_HD constexpr uint32_t kind_code_mask(int D) { return D <= 2 ? 1u : 3u; }
+PESTO_LF_HD constexpr uint32_t kind_byte(int D, uint32_t yu, uint32_t cls, uint32_t xu) {
+    return D > 4 ? 0u : (yu | cls << kind_cshift(D) | xu << kind_xshift(D));
+}
 constexpr int kStepBytes = 48;
 constexpr uint32_t kStXMask = 7u;               // bits 0-2: base device code of the op
 constexpr uint32_t kStHasNear = 1u << 3;        // read the near ring

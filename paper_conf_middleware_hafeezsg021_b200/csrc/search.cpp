@@ -557,10 +557,10 @@ bool swap_in_place(pesto_search *s, int b, int32_t k, Patcher &pt) {
                 pt.set32(L.d_blob32, L.blob32.data(), loc + 4, kSuccPosMask | kSuccTcMask,
                          (uint32_t)q | (target_class32(tgt) << kSuccTcShift));
                 pt.set32(L.d_blob32, L.blob32.data(), loc + 8, ~0u, tgt);
-                if (g->D == 2)        // the fast walk's dispatch entry of the slot: class bits
+                if (g->D <= 4)        // the fast walk's dispatch entry of the slot: class bits
                     pt.set32(L.d_blob32, L.blob32.data(), loc - 16 * (slot + 1) + 4,
-                             kKindClassMask << (8 * slot),
-                             (target_class32(tgt) << kKindClassShift) << (8 * slot));
+                             (7u << kind_cshift(g->D)) << (8 * slot),
+                             (target_class32(tgt) << kind_cshift(g->D)) << (8 * slot));
             }
             pt.set32(L.d_blob32, L.blob32.data(), L.op_off32[q] + 12, kStHasNear,
                      near_first >= 0 ? kStHasNear : 0u);

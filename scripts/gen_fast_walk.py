@@ -118,12 +118,14 @@ def begin(xu):
     return out
 
 
-def segment(cpl, wide=False, ra=False, dt=False):
+def segment(cpl, wide=False, ra=False, dt=False, early=False):
     """ra: the next step's head is read one step ahead (its kinds feed the jump-table load
     before the current step's work; 4 register moves per step).  dt: direct threading -- every
     handler ends with its own copy of the loop's top (limit check, record loads, first-step
     work, dispatch), so no join point sits inside the loop (ptxas otherwise brackets every
-    iteration with a reconvergence barrier and sends it through one far-away join block)"""
+    iteration with a reconvergence barrier and sends it through one far-away join block).
+    early (with dt): each edge-0 handler loads the next step's head as soon as the begin has
+    used p_v, so the head's latency overlaps the handler and the tail does not reload it"""
     operands(cpl, wide)
     cb = CB * cpl                       # bytes of one ring slot (cpl columns of 32 lanes)
     sh = log2(cb)
@@ -143,11 +145,13 @@ def segment(cpl, wide=False, ra=False, dt=False):
         P += [".reg .u32 n0, n1, n2, n3;",
               f"ld.shared.v4.u32 {{n0, n1, n2, n3}}, [{SP}];"]
 
-    def top(tag):
+    def top(tag, have_head=False):
         """the loop's top: stop at the limit, load the step, first-step work, dispatch TA"""
         T = [f"setp.ge.u32 p, {SP}, {LIM};",
              "@p bra.uni FDONE;"]
-        if ra:                  # the tile is padded by one step: [sp + 48] is always readable
+        if have_head:           # loaded early by the handler (the tile is padded by one step)
+            pass
+        elif ra:                # the tile is padded by one step: [sp + 48] is always readable
             T += ["mov.u32 h0, n0;", "mov.u32 h1, n1;", "mov.u32 h2, n2;", "mov.u32 h3, n3;",
                   f"ld.shared.v4.u32 {{n0, n1, n2, n3}}, [{SP}+48];"]
         else:
@@ -203,7 +207,7 @@ def segment(cpl, wide=False, ra=False, dt=False):
 
     def tail(tag):
         if dt:
-            return [f"add.u32 {SP}, {SP}, 48;"] + top(tag)
+            return [f"add.u32 {SP}, {SP}, 48;"] + top(tag, have_head=early)
         return ["bra.uni FNEXT;"]
 
     if dt:
@@ -224,6 +228,8 @@ def segment(cpl, wide=False, ra=False, dt=False):
             continue
         if not cont:
             P += begin(xu)
+        if dt and early:        # p_v used: the next step's head may replace this one
+            P += [f"ld.shared.v4.u32 {{h0, h1, h2, h3}}, [{SP}+48];"]
         P += edge(xu, cls, cross, A)
         if dt:
             P += [f"@q2 bra.uni FTA{i};", "brx.idx.uni k1, TB;", f"FTA{i}:"] + tail(f"A{i}")
@@ -246,6 +252,154 @@ def segment(cpl, wide=False, ra=False, dt=False):
     return P
 
 
+def segment_d4(cpl):
+    """D = 3..4 (two plane bits per code), uint32 time, state in shared memory (eval32.cu
+    SmemState32: device columns at dst + x * slot, links at lst + (x * 4 + y) * slot; a slot is 32
+    lanes x cpl, a lane's pair side by side for cpl 2).  Table entry = yu | class << 2 | xu << 5
+    (StepHead.kinds for D <= 4); the link class of x -> y is bit x * 4 + y of cls4."""
+    global CPL
+    CPL = cpl
+    IL2 = cpl == 2
+    SLOT = 128 * cpl                    # bytes of a state column / ring slot
+    sh = log2(SLOT)
+    k = iter(range(2, 2 + 3 * cpl + 7))
+    grp = lambda: tuple(f"%{next(k)}" for _ in range(cpl))   # noqa: E731
+    SP_, V_ = "%0", "%1"
+    FWD_, NFAR_, NNEAR_ = grp(), grp(), grp()
+    LIM_, RING_, STAGE_, COLD_, DST_, LST_, CLS_ = (f"%{next(k)}" for _ in range(7))
+
+    def lds2(dst, addr):
+        if IL2:
+            return [f"ld.shared.v2.u32 {{{dst[0]}, {dst[1]}}}, [{addr}];"]
+        return [f"ld.shared.u32 {dst[0]}, [{addr}];"]
+
+    def sts2(addr, src):
+        if IL2:
+            return [f"st.shared.v2.u32 [{addr}], {{{src[0]}, {src[1]}}};"]
+        return [f"st.shared.u32 [{addr}], {src[0]};"]
+
+    C = ("c0", "c1")[:cpl]
+    W_ = ("w0", "w1")[:cpl]
+    Y = ("y0", "y1")[:cpl]
+
+    def edge4(xu, yu, cls, rec):
+        if cls == 5:
+            return []
+        out = []
+        if xu != yu:                    # FCFS link xu -> yu: its class picks t0 / t1
+            lk = xu * 4 + yu
+            out += [f"shr.u32 t, {CLS_}, {lk};", "and.b32 t, t, 1;", "setp.ne.u32 p, t, 0;",
+                    f"selp.u32 t, {rec[3]}, {rec[0]}, p;", f"add.u32 s, {LST_}, {lk * SLOT};"]
+            out += lds2(W_, "s")
+            for c in range(cpl):
+                out += [f"max.u32 {W_[c]}, {W_[c]}, {C[c]};", f"add.u32 {W_[c]}, {W_[c]}, t;",
+                        f"min.u32 {W_[c]}, {W_[c]}, {SAT};"]
+            out += sts2("s", W_)
+            a = W_
+        else:
+            a = C
+        if cls == 4:
+            return out + [f"max.u32 {FWD_[c]}, {FWD_[c]}, {a[c]};" for c in range(cpl)]
+        out += [f"and.b32 o, {rec[2]}, 0x1FFFFFFF;"] + (["shl.b32 o, o, 1;"] if cpl == 2 else [])
+        if cls in (2, 3):
+            out += [f"add.u32 s, {RING_}, o;"]
+            if cls == 2:
+                out += lds2(Y, "s")
+                out += [f"max.u32 {Y[c]}, {Y[c]}, {a[c]};" for c in range(cpl)]
+                out += sts2("s", Y)
+            else:
+                out += sts2("s", a)
+        else:
+            out += ["cvt.u64.u32 g, o;", f"add.u64 g, {COLD_}, g;"]
+            if cls == 1:
+                if IL2:
+                    out += [f"st.global.v2.u32 [g], {{{a[0]}, {a[1]}}};"]
+                else:
+                    out += [f"st.global.u32 [g], {a[0]};"]
+            else:
+                out += [f"red.relaxed.gpu.global.max.u32 [g+{4 * c}], {a[c]};" for c in range(cpl)]
+        return out
+
+    A = ("a0", "a1", "a2", "a3")
+    B = ("b0", "b1", "b2", "b3")
+    ta = [f"FA{i}" for i in range(256)]
+    tb = [f"FB{i}" for i in range(128)]
+    P = ["{",
+         ".reg .pred p, q, q2;",
+         ".reg .u32 h0, h1, h2, h3, a0, a1, a2, a3, b0, b1, b2, b3, t, k0, k1, o, s, sz, "
+         "r0, r1, w0, w1, y0, y1, c0, c1;",
+         ".reg .u64 g;",
+         "TA: .branchtargets " + ", ".join(ta) + ";",
+         "TB: .branchtargets " + ", ".join(tb) + ";",
+         "FLOOP:",
+         f"setp.ge.u32 p, {SP_}, {LIM_};",
+         "@p bra.uni FDONE;",
+         f"ld.shared.v4.u32 {{h0, h1, h2, h3}}, [{SP_}];",
+         f"ld.shared.v4.u32 {{a0, a1, a2, a3}}, [{SP_}+16];",
+         f"ld.shared.v4.u32 {{b0, b1, b2, b3}}, [{SP_}+32];",
+         "and.b32 k0, h1, 127;",
+         "shr.u32 k1, h1, 8;",
+         "and.b32 k1, k1, 127;",
+         "and.b32 t, h1, 0x1C00;",
+         "setp.eq.u32 q2, t, 0x1400;",            # slot 1 empty (class 5): no TB dispatch
+         "and.b32 t, h3, 16;",
+         "setp.ne.u32 q, t, 0;",
+         "@q bra.uni FCONT;",
+         f"add.u32 {V_}, {V_}, 1;",
+         f"add.u32 t, {V_}, 11;", "and.b32 t, t, 15;", f"shl.b32 t, t, {sh};",
+         f"add.u32 s, {STAGE_}, t;",
+         "setp.ge.s32 p, h2, 0;", "max.s32 t, h2, 0;", f"mul.wide.u32 g, t, {SLOT};",
+         f"add.u64 g, {COLD_}, g;", f"selp.u32 sz, {4 * cpl}, 0, p;",
+         f"cp.async.ca.shared.global [s], [g], {4 * cpl}, sz;",
+         "cp.async.commit_group;",
+         "cp.async.wait_group 10;",
+         "and.b32 t, h3, 8;", "setp.ne.u32 p, t, 0;"]
+    for c in range(cpl):
+        P += [f"selp.u32 r{c}, {NNEAR_[c]}, 0, p;", f"max.u32 r{c}, r{c}, {NFAR_[c]};",
+              f"max.u32 r{c}, r{c}, {FWD_[c]};"]
+    P += [f"add.u32 t, {V_}, 1;", "and.b32 t, t, 15;", f"shl.b32 t, t, {sh};",
+          f"add.u32 s, {STAGE_}, t;"]
+    P += lds2(NFAR_, "s")
+    P += [f"add.u32 s, {RING_}, t;"]
+    P += lds2(NNEAR_, "s")
+    P += [f"mov.u32 {FWD_[c]}, 0;" for c in range(cpl)]
+    P += ["brx.idx.uni k0, TA;",
+          "FCONT:",
+          "add.u32 k0, k0, 128;",
+          "brx.idx.uni k0, TA;"]
+
+    def dec(e):
+        return e & 3, (e >> 2) & 7, (e >> 5) & 3        # yu, class, xu
+
+    for i in range(256):
+        cont, e = i >> 7, i & 127
+        yu, cls, xu = dec(e)
+        P.append(f"FA{i}:")
+        if cls > 5:
+            P.append("bra.uni FDONE;")
+            continue
+        P += [f"add.u32 s, {DST_}, {xu * SLOT};"]
+        if not cont:                    # C_v = min(max(r, dev_free[xu]) + p, SAT)
+            P += lds2(W_, "s")
+            for c in range(cpl):
+                P += [f"max.u32 {C[c]}, r{c}, {W_[c]};", f"add.u32 {C[c]}, {C[c]}, h0;",
+                      f"min.u32 {C[c]}, {C[c]}, {SAT};"]
+            P += sts2("s", C)
+        else:                           # a continuation: dev_free[xu] still holds C_v
+            P += lds2(C, "s")
+        P += edge4(xu, yu, cls, A)
+        P += ["@q2 bra.uni FNEXT;", "brx.idx.uni k1, TB;"]
+    for i in range(128):
+        yu, cls, xu = dec(i)
+        P.append(f"FB{i}:")
+        if cls <= 5:
+            P += edge4(xu, yu, cls, B)
+        if i < 127:
+            P.append("bra.uni FNEXT;")
+    P += ["FNEXT:", f"add.u32 {SP_}, {SP_}, 48;", "bra.uni FLOOP;", "FDONE:", "}"]
+    return P
+
+
 def main():
     with open(OUT, "w") as f:
         f.write("// generated by scripts/gen_fast_walk.py -- do not edit\n")
@@ -256,10 +410,15 @@ def main():
                                         (1, True, True, False, "1W_RA"),
                                         (1, False, False, True, "1_DT"), (2, False, False, True, "2_DT"),
                                         (1, True, False, True, "1W_DT")):
-            P = segment(cpl, wide, ra, dt)
+            P = segment(cpl, wide, ra, dt, early=dt)
             f.write(f"#define PESTO_FAST_WALK_PTX{name} \\\n" +
                     " \\\n".join('    "' + l + '\\n"' for l in P) + "\n")
             print(OUT, name, len(P), "PTX lines")
+        for cpl in (1, 2):
+            P = segment_d4(cpl)
+            f.write(f"#define PESTO_FAST_WALK_PTX{cpl}_D4 \\\n" +
+                    " \\\n".join('    "' + l + '\\n"' for l in P) + "\n")
+            print(OUT, f"{cpl}_D4", len(P), "PTX lines")
 
 
 if __name__ == "__main__":
