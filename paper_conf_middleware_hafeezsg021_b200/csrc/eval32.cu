@@ -95,6 +95,9 @@ constexpr bool kHeadAhead = PESTO_HEAD_AHEAD2 != 0;
 #ifndef PESTO_FAST_D4
 #define PESTO_FAST_D4 1
 #endif
+#ifndef PESTO_FAST_ROWS
+#define PESTO_FAST_ROWS 1
+#endif
 constexpr bool kUniSwitch = PESTO_UNI_SWITCH != 0;
 __host__ __device__ constexpr int min_blocks_for(int cpl) { return cpl == 1 ? PESTO_E32_MINB1 : PESTO_E32_MINB2; }
 // tile loads: a producer warp per CTA (0), or issued by the consumer warp that releases a stage
@@ -533,6 +536,43 @@ __device__ __forceinline__ void fast_segment(uint32_t &sp, int32_t &v,
                  : "r"(lim), "r"(ring), "r"(stage), "l"(cold)
                  : "memory");
 }
+// explicit rows (mode 0), D = 2: per-lane devices from K5's words, control by class tables
+__device__ __forceinline__ void fast_rows(uint32_t &sp, int32_t &v, uint32_t &ys,
+                                          RegState32<2, uint32_t> &st, uint32_t (&fwd)[2],
+                                          uint32_t (&nfar)[2], uint32_t (&nnear)[2],
+                                          uint32_t (&xr)[2], uint32_t lim, uint32_t ring,
+                                          uint32_t stage, const uint8_t *cold, uint32_t lane,
+                                          const uint32_t *const (&xb)[2],
+                                          const uint32_t *const (&yb)[2]) {
+    asm volatile(PESTO_FAST_ROWS_PTX2
+                 : "+r"(sp), "+r"(v), "+r"(ys), "+r"(st.d0[0]), "+r"(st.d0[1]), "+r"(st.d1[0]),
+                   "+r"(st.d1[1]), "+r"(st.l01[0]), "+r"(st.l01[1]), "+r"(st.l10[0]),
+                   "+r"(st.l10[1]), "+r"(fwd[0]), "+r"(fwd[1]), "+r"(nfar[0]), "+r"(nfar[1]),
+                   "+r"(nnear[0]), "+r"(nnear[1]), "+r"(xr[0]), "+r"(xr[1])
+                 : "r"(lim), "r"(ring), "r"(stage), "l"(cold), "r"(lane), "l"(xb[0]), "l"(xb[1]),
+                   "l"(yb[0]), "l"(yb[1])
+                 : "memory");
+}
+__device__ __forceinline__ void fast_rows(uint32_t &sp, int32_t &v, uint32_t &ys,
+                                          RegState32<1, uint32_t> &st, uint32_t (&fwd)[1],
+                                          uint32_t (&nfar)[1], uint32_t (&nnear)[1],
+                                          uint32_t (&xr)[1], uint32_t lim, uint32_t ring,
+                                          uint32_t stage, const uint8_t *cold, uint32_t lane,
+                                          const uint32_t *const (&xb)[1],
+                                          const uint32_t *const (&yb)[1]) {
+    asm volatile(PESTO_FAST_ROWS_PTX1
+                 : "+r"(sp), "+r"(v), "+r"(ys), "+r"(st.d0[0]), "+r"(st.d1[0]), "+r"(st.l01[0]),
+                   "+r"(st.l10[0]), "+r"(fwd[0]), "+r"(nfar[0]), "+r"(nnear[0]), "+r"(xr[0])
+                 : "r"(lim), "r"(ring), "r"(stage), "l"(cold), "r"(lane), "l"(xb[0]), "l"(yb[0])
+                 : "memory");
+}
+template <int CPL, class T, class ST>
+__device__ __forceinline__ void fast_rows(uint32_t &, int32_t &, uint32_t &, ST &, T (&)[CPL],
+                                          T (&)[CPL], T (&)[CPL], uint32_t (&)[CPL], uint32_t,
+                                          uint32_t, uint32_t, const uint8_t *, uint32_t,
+                                          const uint32_t *const (&)[CPL],
+                                          const uint32_t *const (&)[CPL]) {}
+
 // D = 3..4: device / link state stays in shared memory (SmemState32), the walk's control is
 // the same jump-table loop (fast_walk_ptx.inc PESTO_FAST_WALK_PTX{1,2}_D4)
 __device__ __forceinline__ void fast_segment(uint32_t &sp, int32_t &v, SmemState32<2, uint32_t> &st,
@@ -636,6 +676,8 @@ __global__ void __launch_bounds__(threads_for(CPL), min_blocks_for(CPL))
 eval32_kernel(const EvalParams P) {
     constexpr bool kSearch = MODE == 1 || MODE == 5;   // 5: search with S9 coarse groups
     // uniform steps through the PTX fast segment (D = 2, CPL 2, 32-bit time, search)
+    // explicit rows, D = 2, 32-bit time: every step through the PTX rows segment
+    constexpr bool kFastRows = PESTO_FAST_ROWS != 0 && MODE == 0 && PL == 1 && sizeof(T) == 4;
     constexpr bool kFast = PESTO_FAST_WALK != 0 && MODE == 1 &&
                            ((PL == 1 && (sizeof(T) == 4 || CPL == 1)) ||
                             (PL == 2 && sizeof(T) == 4 && PESTO_FAST_D4 != 0));
@@ -989,7 +1031,7 @@ eval32_kernel(const EvalParams P) {
         };
         // the next op's codes, shuffled one op ahead
         int xnext[CPL];
-        if constexpr (MODE == 0) {
+        if constexpr (MODE == 0 && !kFastRows) {
             if (active) {
                 x_load(0, xw);
                 x_load(SW, xn);
@@ -997,6 +1039,20 @@ eval32_kernel(const EvalParams P) {
                 y_load(SW, yn);
             }
             shfl_dev(xw, 0, xnext);
+        }
+        // rows segment state: the op's device per candidate, the walk's edge-slot counter, and
+        // the words of the warp's 32-row groups (a missing second group reads the first's)
+        uint32_t xr[CPL], yslot = 0;
+        const uint32_t *xbp[CPL], *ybp[CPL];
+#pragma unroll
+        for (int c = 0; c < CPL; c++) {
+            xr[c] = 0;
+            if constexpr (kFastRows) {
+                xbp[c] = place.pl + c * cgrp * place.pl_stride;
+                ybp[c] = P.yplanes + (size_t)(gw + c * cgrp) * ywords;
+            } else {
+                xbp[c] = ybp[c] = nullptr;
+            }
         }
         int32_t v = -1;
         int xu = -1;                 // search: the walked op's device if warp-uniform, else -1
@@ -1022,6 +1078,11 @@ eval32_kernel(const EvalParams P) {
                 }
                 for (;;) {
                     while (sp < lim) {
+                        if constexpr (kFastRows) {
+                            fast_rows(sp, v, yslot, st, fwd, nfar, nnear, xr, lim, cx.ring, stage,
+                                      cx.cold, (uint32_t)lane, xbp, ybp);
+                            continue;
+                        }
                         if constexpr (kFast) {
                             // uniform steps: the PTX segment; a special position's first step
                             // (and its continuation steps) take the C++ step below

@@ -255,8 +255,11 @@ def segment(cpl, wide=False, ra=False, dt=False, early=False):
 def segment_d4(cpl):
     """D = 3..4 (two plane bits per code), uint32 time, state in shared memory (eval32.cu
     SmemState32: device columns at dst + x * slot, links at lst + (x * 4 + y) * slot; a slot is 32
-    lanes x cpl, a lane's pair side by side for cpl 2).  Table entry = yu | class << 2 | xu << 5
-    (StepHead.kinds for D <= 4); the link class of x -> y is bit x * 4 + y of cls4."""
+    lanes x cpl, a lane's pair side by side for cpl 2).  The jump tables dispatch on the edge's
+    (class, crossing) only -- 12 entries; the device and link columns are addressed at run time
+    from the slot's kinds byte (yu | class << 2 | xu << 5; D <= 4), the link class of x -> y is
+    bit x * 4 + y of cls4.  (A table specialised on (xu, yu, class) -- 256 + 128 entries -- ran
+    slower than the C++ walk: the handlers no longer fit the instruction cache.)"""
     global CPL
     CPL = cpl
     IL2 = cpl == 2
@@ -282,14 +285,14 @@ def segment_d4(cpl):
     W_ = ("w0", "w1")[:cpl]
     Y = ("y0", "y1")[:cpl]
 
-    def edge4(xu, yu, cls, rec):
+    def edge4(cls, cross, rec, lk):
+        """lk: register holding x * 4 + y of this edge's link (crossing edges)"""
         if cls == 5:
             return []
         out = []
-        if xu != yu:                    # FCFS link xu -> yu: its class picks t0 / t1
-            lk = xu * 4 + yu
+        if cross:                       # FCFS link xu -> yu: its class picks t0 / t1
             out += [f"shr.u32 t, {CLS_}, {lk};", "and.b32 t, t, 1;", "setp.ne.u32 p, t, 0;",
-                    f"selp.u32 t, {rec[3]}, {rec[0]}, p;", f"add.u32 s, {LST_}, {lk * SLOT};"]
+                    f"selp.u32 t, {rec[3]}, {rec[0]}, p;", f"mad.lo.u32 s, {lk}, {SLOT}, {LST_};"]
             out += lds2(W_, "s")
             for c in range(cpl):
                 out += [f"max.u32 {W_[c]}, {W_[c]}, {C[c]};", f"add.u32 {W_[c]}, {W_[c]}, t;",
@@ -320,14 +323,23 @@ def segment_d4(cpl):
                 out += [f"red.relaxed.gpu.global.max.u32 [g+{4 * c}], {a[c]};" for c in range(cpl)]
         return out
 
+    def kind(byte_shift, k, lk):
+        """k = class * 2 + (yu != xu), lk = xu * 4 + yu, from the slot's kinds byte"""
+        return [f"shr.u32 t, h1, {byte_shift};",
+                "and.b32 u, t, 3;",                       # yu
+                "shr.u32 xx, t, 5;", "and.b32 xx, xx, 3;", # xu
+                f"shl.b32 {lk}, xx, 2;", f"or.b32 {lk}, {lk}, u;",
+                "setp.ne.u32 p, u, xx;", "selp.u32 u, 1, 0, p;",
+                f"shr.u32 {k}, t, 1;", f"and.b32 {k}, {k}, 14;", f"or.b32 {k}, {k}, u;"]
+
     A = ("a0", "a1", "a2", "a3")
     B = ("b0", "b1", "b2", "b3")
-    ta = [f"FA{i}" for i in range(256)]
-    tb = [f"FB{i}" for i in range(128)]
+    ta = [f"FA{i}" for i in range(32)]
+    tb = [f"FB{i}" for i in range(16)]
     P = ["{",
          ".reg .pred p, q, q2;",
-         ".reg .u32 h0, h1, h2, h3, a0, a1, a2, a3, b0, b1, b2, b3, t, k0, k1, o, s, sz, "
-         "r0, r1, w0, w1, y0, y1, c0, c1;",
+         ".reg .u32 h0, h1, h2, h3, a0, a1, a2, a3, b0, b1, b2, b3, t, u, xx, k0, k1, l0, l1, "
+         "o, s, sz, r0, r1, w0, w1, y0, y1, c0, c1;",
          ".reg .u64 g;",
          "TA: .branchtargets " + ", ".join(ta) + ";",
          "TB: .branchtargets " + ", ".join(tb) + ";",
@@ -336,24 +348,23 @@ def segment_d4(cpl):
          "@p bra.uni FDONE;",
          f"ld.shared.v4.u32 {{h0, h1, h2, h3}}, [{SP_}];",
          f"ld.shared.v4.u32 {{a0, a1, a2, a3}}, [{SP_}+16];",
-         f"ld.shared.v4.u32 {{b0, b1, b2, b3}}, [{SP_}+32];",
-         "and.b32 k0, h1, 127;",
-         "shr.u32 k1, h1, 8;",
-         "and.b32 k1, k1, 127;",
-         "and.b32 t, h1, 0x1C00;",
-         "setp.eq.u32 q2, t, 0x1400;",            # slot 1 empty (class 5): no TB dispatch
-         "and.b32 t, h3, 16;",
-         "setp.ne.u32 q, t, 0;",
-         "@q bra.uni FCONT;",
-         f"add.u32 {V_}, {V_}, 1;",
-         f"add.u32 t, {V_}, 11;", "and.b32 t, t, 15;", f"shl.b32 t, t, {sh};",
-         f"add.u32 s, {STAGE_}, t;",
-         "setp.ge.s32 p, h2, 0;", "max.s32 t, h2, 0;", f"mul.wide.u32 g, t, {SLOT};",
-         f"add.u64 g, {COLD_}, g;", f"selp.u32 sz, {4 * cpl}, 0, p;",
-         f"cp.async.ca.shared.global [s], [g], {4 * cpl}, sz;",
-         "cp.async.commit_group;",
-         "cp.async.wait_group 10;",
-         "and.b32 t, h3, 8;", "setp.ne.u32 p, t, 0;"]
+         f"ld.shared.v4.u32 {{b0, b1, b2, b3}}, [{SP_}+32];"]
+    P += kind(0, "k0", "l0") + kind(8, "k1", "l1")
+    P += ["setp.ge.u32 q2, k1, 10;",          # slot 1 empty (class 5): no TB dispatch
+          "and.b32 t, h3, 16;",
+          "setp.ne.u32 q, t, 0;",
+          # the op's device column (xu of slot 0 = the op's base code)
+          "shr.u32 t, l0, 2;", f"mad.lo.u32 xx, t, {SLOT}, {DST_};",
+          "@q bra.uni FCONT;",
+          f"add.u32 {V_}, {V_}, 1;",
+          f"add.u32 t, {V_}, 11;", "and.b32 t, t, 15;", f"shl.b32 t, t, {sh};",
+          f"add.u32 s, {STAGE_}, t;",
+          "setp.ge.s32 p, h2, 0;", "max.s32 t, h2, 0;", f"mul.wide.u32 g, t, {SLOT};",
+          f"add.u64 g, {COLD_}, g;", f"selp.u32 sz, {4 * cpl}, 0, p;",
+          f"cp.async.ca.shared.global [s], [g], {4 * cpl}, sz;",
+          "cp.async.commit_group;",
+          "cp.async.wait_group 10;",
+          "and.b32 t, h3, 8;", "setp.ne.u32 p, t, 0;"]
     for c in range(cpl):
         P += [f"selp.u32 r{c}, {NNEAR_[c]}, 0, p;", f"max.u32 r{c}, r{c}, {NFAR_[c]};",
               f"max.u32 r{c}, r{c}, {FWD_[c]};"]
@@ -363,38 +374,178 @@ def segment_d4(cpl):
     P += [f"add.u32 s, {RING_}, t;"]
     P += lds2(NNEAR_, "s")
     P += [f"mov.u32 {FWD_[c]}, 0;" for c in range(cpl)]
+    # C_v = min(max(r, dev_free[xu]) + p, SAT), dev_free[xu] = C_v
+    P += lds2(W_, "xx")
+    for c in range(cpl):
+        P += [f"max.u32 {C[c]}, r{c}, {W_[c]};", f"add.u32 {C[c]}, {C[c]}, h0;",
+              f"min.u32 {C[c]}, {C[c]}, {SAT};"]
+    P += sts2("xx", C)
     P += ["brx.idx.uni k0, TA;",
-          "FCONT:",
-          "add.u32 k0, k0, 128;",
+          "FCONT:"]                     # a continuation: dev_free[xu] still holds C_v
+    P += lds2(C, "xx")
+    P += ["add.u32 k0, k0, 16;",
           "brx.idx.uni k0, TA;"]
-
-    def dec(e):
-        return e & 3, (e >> 2) & 7, (e >> 5) & 3        # yu, class, xu
-
-    for i in range(256):
-        cont, e = i >> 7, i & 127
-        yu, cls, xu = dec(e)
+    for i in range(32):
+        e = i & 15
+        cls, cross = e >> 1, e & 1
         P.append(f"FA{i}:")
         if cls > 5:
             P.append("bra.uni FDONE;")
             continue
-        P += [f"add.u32 s, {DST_}, {xu * SLOT};"]
-        if not cont:                    # C_v = min(max(r, dev_free[xu]) + p, SAT)
-            P += lds2(W_, "s")
-            for c in range(cpl):
-                P += [f"max.u32 {C[c]}, r{c}, {W_[c]};", f"add.u32 {C[c]}, {C[c]}, h0;",
-                      f"min.u32 {C[c]}, {C[c]}, {SAT};"]
-            P += sts2("s", C)
-        else:                           # a continuation: dev_free[xu] still holds C_v
-            P += lds2(C, "s")
-        P += edge4(xu, yu, cls, A)
+        P += edge4(cls, cross, A, "l0")
         P += ["@q2 bra.uni FNEXT;", "brx.idx.uni k1, TB;"]
-    for i in range(128):
-        yu, cls, xu = dec(i)
+    for i in range(16):
+        cls, cross = i >> 1, i & 1
         P.append(f"FB{i}:")
         if cls <= 5:
-            P += edge4(xu, yu, cls, B)
-        if i < 127:
+            P += edge4(cls, cross, B, "l1")
+        if i < 15:
+            P.append("bra.uni FNEXT;")
+    P += ["FNEXT:", f"add.u32 {SP_}, {SP_}, 48;", "bra.uni FLOOP;", "FDONE:", "}"]
+    return P
+
+
+def segment_rows(cpl):
+    """Explicit rows (eval32 mode 0), D = 2, uint32 time: every lane has its own devices (K5's
+    bit-sliced words: the op's word at xb + 4v, the successors' at yb + 4·slot, bit `lane`), so
+    the device and link choices are per-lane selects, but the control -- first step or not, the
+    edge's class -- is the step's and dispatches through 8-entry jump tables."""
+    global CPL
+    CPL = cpl
+    IL2 = cpl == 2
+    SLOT = 128 * cpl
+    sh = log2(SLOT)
+    k = iter(range(3, 3 + 8 * cpl + 5 + 2 * cpl))
+    grp = lambda: tuple(f"%{next(k)}" for _ in range(cpl))   # noqa: E731
+    SP_, V_, YS_ = "%0", "%1", "%2"
+    D0_, D1_, L01_, L10_, FWD_, NFAR_, NNEAR_, X_ = (grp() for _ in range(8))
+    LIM_, RING_, STAGE_, COLD_, LANE_ = (f"%{next(k)}" for _ in range(5))
+    XB_, YB_ = grp(), grp()
+    C = ("c0", "c1")[:cpl]
+    PX = ("px0", "px1")[:cpl]
+
+    def lds2(dst, addr):
+        if IL2:
+            return [f"ld.shared.v2.u32 {{{dst[0]}, {dst[1]}}}, [{addr}];"]
+        return [f"ld.shared.u32 {dst[0]}, [{addr}];"]
+
+    def sts2(addr, src):
+        if IL2:
+            return [f"st.shared.v2.u32 [{addr}], {{{src[0]}, {src[1]}}};"]
+        return [f"st.shared.u32 [{addr}], {src[0]};"]
+
+    def edge_rows(cls, rec, ywreg):
+        if cls == 5:
+            return []
+        out = []
+        a = ("w0", "w1")[:cpl]
+        for c in range(cpl):
+            out += [f"shr.u32 t, {ywreg[c]}, {LANE_};", "and.b32 t, t, 1;",
+                    f"xor.b32 t, t, {X_[c]};", "setp.ne.u32 pc, t, 0;",             # crossing
+                    f"selp.u32 u, {L10_[c]}, {L01_[c]}, {PX[c]};",
+                    f"selp.u32 tt, {rec[3]}, {rec[0]}, {PX[c]};",
+                    f"max.u32 u, u, {C[c]};", "add.u32 u, u, tt;", f"min.u32 u, u, {SAT};",
+                    f"and.pred pq, pc, {PX[c]};", f"@pq mov.u32 {L10_[c]}, u;",
+                    f"and.pred pq, pc, !{PX[c]};", f"@pq mov.u32 {L01_[c]}, u;",
+                    f"selp.u32 {a[c]}, u, {C[c]}, pc;"]
+        if cls == 4:
+            return out + [f"max.u32 {FWD_[c]}, {FWD_[c]}, {a[c]};" for c in range(cpl)]
+        out += [f"and.b32 o, {rec[2]}, 0x1FFFFFFF;"] + (["shl.b32 o, o, 1;"] if cpl == 2 else [])
+        if cls in (2, 3):
+            out += [f"add.u32 s, {RING_}, o;"]
+            if cls == 2:
+                Y = ("y0", "y1")[:cpl]
+                out += lds2(Y, "s")
+                out += [f"max.u32 {Y[c]}, {Y[c]}, {a[c]};" for c in range(cpl)]
+                out += sts2("s", Y)
+            else:
+                out += sts2("s", a)
+        else:
+            out += ["cvt.u64.u32 g, o;", f"add.u64 g, {COLD_}, g;"]
+            if cls == 1:
+                out += ([f"st.global.v2.u32 [g], {{{a[0]}, {a[1]}}};"] if IL2
+                        else [f"st.global.u32 [g], {a[0]};"])
+            else:
+                out += [f"red.relaxed.gpu.global.max.u32 [g+{4 * c}], {a[c]};" for c in range(cpl)]
+        return out
+
+    A = ("a0", "a1", "a2", "a3")
+    B = ("b0", "b1", "b2", "b3")
+    YA = ("ya0", "ya1")[:cpl]           # slot-0 successor words per candidate group
+    YBw = ("yb0", "yb1")[:cpl]          # slot-1
+    ta = [f"FA{i}" for i in range(16)]
+    tb = [f"FB{i}" for i in range(8)]
+    P = ["{",
+         ".reg .pred p, q, q2, pc, pq, px0, px1;",
+         ".reg .u32 h0, h1, h2, h3, a0, a1, a2, a3, b0, b1, b2, b3, t, u, tt, k0, k1, o, s, sz, "
+         "r0, r1, w0, w1, y0, y1, c0, c1, ya0, ya1, yb0, yb1, xw;",
+         ".reg .u64 g, gy;",
+         "TA: .branchtargets " + ", ".join(ta) + ";",
+         "TB: .branchtargets " + ", ".join(tb) + ";",
+         "FLOOP:",
+         f"setp.ge.u32 p, {SP_}, {LIM_};",
+         "@p bra.uni FDONE;",
+         f"ld.shared.v4.u32 {{h0, h1, h2, h3}}, [{SP_}];",
+         f"ld.shared.v4.u32 {{a0, a1, a2, a3}}, [{SP_}+16];",
+         f"ld.shared.v4.u32 {{b0, b1, b2, b3}}, [{SP_}+32];"]
+    for c in range(cpl):                # both slots' successor words of candidate group c
+        P += [f"mul.wide.u32 gy, {YS_}, 4;", f"add.u64 gy, {YB_[c]}, gy;",
+              f"ld.global.nc.v2.u32 {{{YA[c]}, {YBw[c]}}}, [gy];"]
+    P += [f"add.u32 {YS_}, {YS_}, 2;",
+          "shr.u32 k0, h1, 1;", "and.b32 k0, k0, 7;",
+          "shr.u32 k1, h1, 9;", "and.b32 k1, k1, 7;",
+          "setp.eq.u32 q2, k1, 5;",             # slot 1 empty: no TB dispatch
+          "and.b32 t, h3, 16;",
+          "setp.ne.u32 q, t, 0;",
+          "@q bra.uni FCONT;",
+          f"add.u32 {V_}, {V_}, 1;"]
+    for c in range(cpl):                # the op's device in each lane's row: bit `lane`
+        P += [f"mul.wide.u32 gy, {V_}, 4;", f"add.u64 gy, {XB_[c]}, gy;",
+              "ld.global.nc.u32 xw, [gy];", f"shr.u32 xw, xw, {LANE_};", f"and.b32 {X_[c]}, xw, 1;"]
+    P += [f"add.u32 t, {V_}, 11;", "and.b32 t, t, 15;", f"shl.b32 t, t, {sh};",
+          f"add.u32 s, {STAGE_}, t;",
+          "setp.ge.s32 p, h2, 0;", "max.s32 t, h2, 0;", f"mul.wide.u32 g, t, {SLOT};",
+          f"add.u64 g, {COLD_}, g;", f"selp.u32 sz, {4 * cpl}, 0, p;",
+          f"cp.async.ca.shared.global [s], [g], {4 * cpl}, sz;",
+          "cp.async.commit_group;",
+          "cp.async.wait_group 10;",
+          "and.b32 t, h3, 8;", "setp.ne.u32 p, t, 0;"]
+    for c in range(cpl):
+        P += [f"selp.u32 r{c}, {NNEAR_[c]}, 0, p;", f"max.u32 r{c}, r{c}, {NFAR_[c]};",
+              f"max.u32 r{c}, r{c}, {FWD_[c]};"]
+    P += [f"add.u32 t, {V_}, 1;", "and.b32 t, t, 15;", f"shl.b32 t, t, {sh};",
+          f"add.u32 s, {STAGE_}, t;"]
+    P += lds2(NFAR_, "s")
+    P += [f"add.u32 s, {RING_}, t;"]
+    P += lds2(NNEAR_, "s")
+    P += [f"mov.u32 {FWD_[c]}, 0;" for c in range(cpl)]
+    # C_v = min(max(r, dev_free[x]) + p, SAT) per lane, dev_free[x] = C_v
+    for c in range(cpl):
+        P += [f"setp.ne.u32 {PX[c]}, {X_[c]}, 0;",
+              f"selp.u32 t, {D1_[c]}, {D0_[c]}, {PX[c]};",
+              f"max.u32 {C[c]}, r{c}, t;", f"add.u32 {C[c]}, {C[c]}, h0;",
+              f"min.u32 {C[c]}, {C[c]}, {SAT};",
+              f"@{PX[c]} mov.u32 {D1_[c]}, {C[c]};", f"@!{PX[c]} mov.u32 {D0_[c]}, {C[c]};"]
+    P += ["brx.idx.uni k0, TA;",
+          "FCONT:"]                     # a continuation: dev_free[x] still holds C_v
+    for c in range(cpl):
+        P += [f"setp.ne.u32 {PX[c]}, {X_[c]}, 0;",
+              f"selp.u32 {C[c]}, {D1_[c]}, {D0_[c]}, {PX[c]};"]
+    P += ["add.u32 k0, k0, 8;",
+          "brx.idx.uni k0, TA;"]
+    for i in range(16):
+        cls = i & 7
+        P.append(f"FA{i}:")
+        if cls > 5:
+            P.append("bra.uni FDONE;")
+            continue
+        P += edge_rows(cls, A, YA)
+        P += ["@q2 bra.uni FNEXT;", "brx.idx.uni k1, TB;"]
+    for i in range(8):
+        P.append(f"FB{i}:")
+        if i <= 5:
+            P += edge_rows(i, B, YBw)
+        if i < 7:
             P.append("bra.uni FNEXT;")
     P += ["FNEXT:", f"add.u32 {SP_}, {SP_}, 48;", "bra.uni FLOOP;", "FDONE:", "}"]
     return P
@@ -414,6 +565,11 @@ def main():
             f.write(f"#define PESTO_FAST_WALK_PTX{name} \\\n" +
                     " \\\n".join('    "' + l + '\\n"' for l in P) + "\n")
             print(OUT, name, len(P), "PTX lines")
+        for cpl in (1, 2):
+            P = segment_rows(cpl)
+            f.write(f"#define PESTO_FAST_ROWS_PTX{cpl} \\\n" +
+                    " \\\n".join('    "' + l + '\\n"' for l in P) + "\n")
+            print(OUT, f"{cpl}_ROWS", len(P), "PTX lines")
         for cpl in (1, 2):
             P = segment_d4(cpl)
             f.write(f"#define PESTO_FAST_WALK_PTX{cpl}_D4 \\\n" +
