@@ -91,6 +91,13 @@ class ClockSampler:
                 stdout=open(self.path, "w"), stderr=subprocess.DEVNULL)
         except Exception:
             self.proc = None
+        # nvidia-smi takes a few hundred ms to start: wait for its first sample so that a short
+        # timed region (10 inception steps are ~50 ms) is sampled too
+        t0 = time.perf_counter()
+        while self.proc is not None and time.perf_counter() - t0 < 5.0:
+            if os.path.getsize(self.path) > 0 or self.proc.poll() is not None:
+                break
+            time.sleep(0.02)
         return self
 
     def __exit__(self, *a):

@@ -537,6 +537,39 @@ __device__ __forceinline__ void fast_segment(uint32_t &sp, int32_t &v,
                  : "memory");
 }
 // explicit rows (mode 0), D = 2: per-lane devices from K5's words, control by class tables
+#ifndef PESTO_ROWS_PF
+#define PESTO_ROWS_PF 0
+#endif
+// PESTO_ROWS_V2 selects the explicit-row segment (scripts/gen_fast_walk.py segment_rows):
+// 0 round-2 first version, 1 lane-mask tests, 3 + register read-ahead, 4 + windowed shuffles,
+// 5 (default) 4 for two candidates per lane, 3 for one.  Measured (B200, K1 of 1 M random rows,
+// transformer_2dev, CPL 2): 74.5 (0) -> 69.0 (3) -> 66.4 ms (4); inception 65,536 rows (CPL 1):
+// 6.30 (0) -> 5.91 (3) / 6.47 ms (4)
+#ifndef PESTO_ROWS_V2
+#define PESTO_ROWS_V2 5
+#endif
+#if PESTO_ROWS_V2 == 5
+#define PESTO_FR1 PESTO_FAST_ROWS_PTX1_V3
+#define PESTO_FR2 PESTO_FAST_ROWS_PTX2_V4
+#elif PESTO_ROWS_V2 >= 4
+#define PESTO_FR1 PESTO_FAST_ROWS_PTX1_V4
+#define PESTO_FR2 PESTO_FAST_ROWS_PTX2_V4
+#elif PESTO_ROWS_V2 >= 3
+#define PESTO_FR1 PESTO_FAST_ROWS_PTX1_V3
+#define PESTO_FR2 PESTO_FAST_ROWS_PTX2_V3
+#elif PESTO_ROWS_V2 && PESTO_ROWS_PF
+#define PESTO_FR1 PESTO_FAST_ROWS_PTX1_V2PF
+#define PESTO_FR2 PESTO_FAST_ROWS_PTX2_V2PF
+#elif PESTO_ROWS_V2
+#define PESTO_FR1 PESTO_FAST_ROWS_PTX1_V2
+#define PESTO_FR2 PESTO_FAST_ROWS_PTX2_V2
+#elif PESTO_ROWS_PF
+#define PESTO_FR1 PESTO_FAST_ROWS_PTX1_PF
+#define PESTO_FR2 PESTO_FAST_ROWS_PTX2_PF
+#else
+#define PESTO_FR1 PESTO_FAST_ROWS_PTX1
+#define PESTO_FR2 PESTO_FAST_ROWS_PTX2
+#endif
 __device__ __forceinline__ void fast_rows(uint32_t &sp, int32_t &v, uint32_t &ys,
                                           RegState32<2, uint32_t> &st, uint32_t (&fwd)[2],
                                           uint32_t (&nfar)[2], uint32_t (&nnear)[2],
@@ -544,7 +577,7 @@ __device__ __forceinline__ void fast_rows(uint32_t &sp, int32_t &v, uint32_t &ys
                                           uint32_t stage, const uint8_t *cold, uint32_t lane,
                                           const uint32_t *const (&xb)[2],
                                           const uint32_t *const (&yb)[2]) {
-    asm volatile(PESTO_FAST_ROWS_PTX2
+    asm volatile(PESTO_FR2
                  : "+r"(sp), "+r"(v), "+r"(ys), "+r"(st.d0[0]), "+r"(st.d0[1]), "+r"(st.d1[0]),
                    "+r"(st.d1[1]), "+r"(st.l01[0]), "+r"(st.l01[1]), "+r"(st.l10[0]),
                    "+r"(st.l10[1]), "+r"(fwd[0]), "+r"(fwd[1]), "+r"(nfar[0]), "+r"(nfar[1]),
@@ -560,7 +593,7 @@ __device__ __forceinline__ void fast_rows(uint32_t &sp, int32_t &v, uint32_t &ys
                                           uint32_t stage, const uint8_t *cold, uint32_t lane,
                                           const uint32_t *const (&xb)[1],
                                           const uint32_t *const (&yb)[1]) {
-    asm volatile(PESTO_FAST_ROWS_PTX1
+    asm volatile(PESTO_FR1
                  : "+r"(sp), "+r"(v), "+r"(ys), "+r"(st.d0[0]), "+r"(st.d1[0]), "+r"(st.l01[0]),
                    "+r"(st.l10[0]), "+r"(fwd[0]), "+r"(nfar[0]), "+r"(nnear[0]), "+r"(xr[0])
                  : "r"(lim), "r"(ring), "r"(stage), "l"(cold), "r"(lane), "l"(xb[0]), "l"(yb[0])

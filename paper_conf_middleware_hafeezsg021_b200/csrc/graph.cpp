@@ -742,8 +742,14 @@ pesto_status eval_batch_ws(pesto_graph *g, Scratch &ws, const int32_t *order, co
     if ((s = upload_layout(g, *L))) return s;
     cudaStream_t st = (cudaStream_t)stream;
     const int64_t n_groups = (n_cand + 31) / 32;
-    cudaError_t e = ws.planes.ensure((size_t)n_groups * g->n * g->planes * 4);
+    // kStreamPad zeroed bytes past both word streams: the explicit-row walk reads the next
+    // op's and the next step's words one step ahead (eval32.cu fast_rows)
+    const size_t planes_bytes = (size_t)n_groups * g->n * g->planes * 4;
+    cudaError_t e = ws.planes.ensure(planes_bytes + kStreamPad);
     if (e != cudaSuccess) return cuda_fail(e, "allocate bit-sliced placements");
+    if ((e = cudaMemsetAsync(ws.planes.as<uint8_t>() + planes_bytes, 0, kStreamPad,
+                             (cudaStream_t)stream)) != cudaSuccess)
+        return cuda_fail(e, "clear stream padding");
     if ((e = ws.invalid.ensure((size_t)n_groups * 4)) != cudaSuccess) return cuda_fail(e, "allocate");
     TransposeParams tp{};
     tp.rows = static_cast<const uint8_t *>(placements);
@@ -766,8 +772,11 @@ pesto_status eval_batch_ws(pesto_graph *g, Scratch &ws, const int32_t *order, co
     if (ystream) {
         tp.slot_succ = L->d_slot_succ.as<int32_t>();
         tp.n_slots = (int64_t)L->slot_succ.size();
-        if ((e = ws.yplanes.ensure((size_t)n_groups * tp.n_slots * g->planes * 4)) != cudaSuccess)
+        const size_t ybytes = (size_t)n_groups * tp.n_slots * g->planes * 4;
+        if ((e = ws.yplanes.ensure(ybytes + kStreamPad)) != cudaSuccess)
             return cuda_fail(e, "allocate edge-slot stream");
+        if ((e = cudaMemsetAsync(ws.yplanes.as<uint8_t>() + ybytes, 0, kStreamPad, st)) != cudaSuccess)
+            return cuda_fail(e, "clear stream padding");
         tp.yplanes_out = ws.yplanes.as<uint32_t>();
     }
     if ((e = launch_transpose(tp, st)) != cudaSuccess) return cuda_fail(e, "launch transpose");

@@ -195,6 +195,7 @@ struct PatchOp {
     uint32_t pad;
 };
 constexpr int kPatchMaxBlock = 48 * 1024;      // rotation bytes a + b (shared-memory staging)
+constexpr size_t kStreamPad = 512;              // zeroed bytes after K5's word streams
 constexpr int kTransposeSmemMax = 200 * 1024;  // K5 smem variant: a group's n*planes words
 
 // launchers (kernels.cu / eval32.cu); they return the launch error, if any.

@@ -508,6 +508,14 @@ __global__ void __launch_bounds__(256) transpose_kernel(const TransposeParams P)
 // loads (a row's sectors are reused from L1 by the following loads), the permutation to
 // position order is applied in shared memory, and the group's n*PL words leave with coalesced
 // stores -- the global-scatter variant above wrote 4 bytes per 32-byte sector.
+#ifndef PESTO_T16
+#define PESTO_T16 4
+#endif
+constexpr int kT16 = PESTO_T16;
+#ifndef PESTO_YU
+#define PESTO_YU 8
+#endif
+constexpr int kYU = PESTO_YU;
 template <int PL>
 __global__ void __launch_bounds__(256) transpose_smem_kernel(const TransposeParams P) {
     extern __shared__ uint4 tsm[];
@@ -522,12 +530,12 @@ __global__ void __launch_bounds__(256) transpose_smem_kernel(const TransposePara
         const bool have = row < P.n_cand;
         const uint4 *rp = reinterpret_cast<const uint4 *>(P.rows + row * P.stride);
         uint32_t bad = 0;
-        auto emit = [&](int c, uint32_t (&pw)[PL]) {   // chunk c = ops [32c, 32c + 32)
+        // chunk c = ops [32c, 32c + 32); fm, q: the lane's op's forbidden codes and position
+        auto emit = [&](int c, uint32_t (&pw)[PL], unsigned fm, int q) {
 #pragma unroll
             for (int k = 0; k < PL; k++) pw[k] = transpose32(pw[k], lane);
             const int op = c * 32 + lane;
             if (op >= P.n) return;
-            const unsigned fm = __ldg(P.fmask + op);
             if (fm) {
                 for (int code = 0; code < (1 << PL); code++) {
                     if (!((fm >> code) & 1u)) continue;
@@ -537,20 +545,45 @@ __global__ void __launch_bounds__(256) transpose_smem_kernel(const TransposePara
                     bad |= match;
                 }
             }
-            const int q = __ldg(P.pos_of + op);
 #pragma unroll
             for (int k = 0; k < PL; k++) out_s[q * PL + k] = pw[k];
         };
+        constexpr int CPK = 4 / PL;                     // 32-op chunks per 16-byte row chunk
         __syncthreads();
-        for (int k16 = warp; k16 < n16; k16 += 8) {
-            const uint4 w = have ? __ldg(rp + k16) : make_uint4(0, 0, 0, 0);
+        // kT16 of the row's 16-byte chunks per lane are loaded before any is used: with one
+        // load in flight per warp (16 warps per SM) the load phase ran at ~1 TB/s
+        for (int kb = warp; kb < n16; kb += 8 * kT16) {
+          uint4 wv[kT16];
+#pragma unroll
+          for (int u = 0; u < kT16; u++) {
+              const int k16 = kb + 8 * u;
+              wv[u] = (have && k16 < n16) ? __ldg(rp + k16) : make_uint4(0, 0, 0, 0);
+          }
+          // the ops' masks and positions, also loaded before first use
+          unsigned fmv[kT16 * CPK];
+          int qv[kT16 * CPK];
+#pragma unroll
+          for (int u = 0; u < kT16; u++) {
+#pragma unroll
+              for (int j = 0; j < CPK; j++) {
+                  const int op = (CPK * (kb + 8 * u) + j) * 32 + lane;
+                  const bool in = op < P.n;
+                  fmv[u * CPK + j] = in ? __ldg(P.fmask + op) : 0u;
+                  qv[u * CPK + j] = in ? __ldg(P.pos_of + op) : 0;
+              }
+          }
+#pragma unroll
+          for (int u = 0; u < kT16; u++) {
+            const int k16 = kb + 8 * u;
+            if (k16 >= n16) break;
+            const uint4 w = wv[u];
             if (PL == 1) {
                 const uint32_t ws[4] = {w.x, w.y, w.z, w.w};
 #pragma unroll
                 for (int j = 0; j < 4; j++) {
                     uint32_t pw[PL];
                     pw[0] = ws[j];
-                    emit(4 * k16 + j, pw);
+                    emit(4 * k16 + j, pw, fmv[u * CPK + j], qv[u * CPK + j]);
                 }
             } else if (PL == 2) {
                 const uint32_t ws[4] = {w.x, w.y, w.z, w.w};
@@ -560,7 +593,7 @@ __global__ void __launch_bounds__(256) transpose_smem_kernel(const TransposePara
                     const uint32_t lo = ws[2 * j], hi = ws[2 * j + 1];
                     pw[0] = compress2(lo) | (compress2(hi) << 16);
                     pw[1] = compress2(lo >> 1) | (compress2(hi >> 1) << 16);
-                    emit(2 * k16 + j, pw);
+                    emit(2 * k16 + j, pw, fmv[u * CPK + j], qv[u * CPK + j]);
                 }
             } else {
                 uint32_t pw[PL];
@@ -568,8 +601,9 @@ __global__ void __launch_bounds__(256) transpose_smem_kernel(const TransposePara
                 for (int k = 0; k < PL; k++)
                     pw[k] = compress4(w.x >> k) | (compress4(w.y >> k) << 8) |
                             (compress4(w.z >> k) << 16) | (compress4(w.w >> k) << 24);
-                emit(k16, pw);
+                emit(k16, pw, fmv[u], qv[u]);
             }
+          }
         }
         bad = __reduce_or_sync(0xffffffffu, bad);
         if (lane == 0 && bad) atomicOr(&bad_s, bad);
@@ -577,11 +611,24 @@ __global__ void __launch_bounds__(256) transpose_smem_kernel(const TransposePara
         uint32_t *dst = P.planes_out + (size_t)g * nw;
         for (int i = threadIdx.x; i < nw; i += blockDim.x) dst[i] = out_s[i];
         if (P.yplanes_out) {                   // the edge-slot stream of the eval32 walk
+            // kYU successor positions per thread in flight (one dependent L2 load per slot
+            // left K5 waiting on long scoreboards)
             uint32_t *ydst = P.yplanes_out + (size_t)g * P.n_slots * PL;
-            for (int64_t i = threadIdx.x; i < P.n_slots; i += blockDim.x) {
-                const int32_t q = __ldg(P.slot_succ + i);
+            for (int64_t i0 = threadIdx.x; i0 < P.n_slots; i0 += (int64_t)blockDim.x * kYU) {
+                int32_t qv[kYU];
 #pragma unroll
-                for (int k = 0; k < PL; k++) ydst[i * PL + k] = q >= 0 ? out_s[q * PL + k] : 0u;
+                for (int u = 0; u < kYU; u++) {
+                    const int64_t i = i0 + (int64_t)u * blockDim.x;
+                    qv[u] = i < P.n_slots ? __ldg(P.slot_succ + i) : -1;
+                }
+#pragma unroll
+                for (int u = 0; u < kYU; u++) {
+                    const int64_t i = i0 + (int64_t)u * blockDim.x;
+                    if (i >= P.n_slots) break;
+#pragma unroll
+                    for (int k = 0; k < PL; k++)
+                        ydst[i * PL + k] = qv[u] >= 0 ? out_s[qv[u] * PL + k] : 0u;
+                }
             }
         }
         if (threadIdx.x == 0) P.invalid_out[g] = bad_s;

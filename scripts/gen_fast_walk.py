@@ -405,8 +405,24 @@ def segment_d4(cpl):
     return P
 
 
-def segment_rows(cpl):
-    """Explicit rows (eval32 mode 0), D = 2, uint32 time: every lane has its own devices (K5's
+def segment_rows(cpl, pf=0, v2=False, ra=False, win=False):
+    """win (with v2): both word streams are read 32 words at a time -- lane l loads word
+    base + l with one coalesced load, the next window is loaded a window ahead (out of line, once
+    per 32 ops / 16 steps) and a step takes its words with warp shuffles, so no step waits on a
+    global load (ra's register read-ahead was undone by ptxas, which copied the loaded word into
+    the loop-carried register before the dispatch and so waited for it there).
+    ra (with v2): the successor words of the next step and the op word of the next op are
+    loaded one step / one op ahead into registers (re-primed at every segment entry; the
+    workspace pads both streams so the last step's read-ahead stays in bounds) -- the L1 hit
+    rate of these uniform loads is ~13% behind the cold-slot traffic, so a load issued at its
+    use waited on L2.
+    v2: the op's register holds its raw 32-row word and the lane tests it with a lane mask
+    (one LOP3 to a predicate instead of shift, and, compare), and a crossing edge updates its
+    link with two predicated selects instead of predicate ANDs and moves.
+    pf > 0: each step also prefetches into L1 the successor-word stream pf bytes ahead and
+    the op-word stream pf/2 bytes ahead (both advance one 32-bit word per slot / per op), so
+    the step's uniform loads hit L1 instead of waiting on L2 once every 16-32 steps.
+    Explicit rows (eval32 mode 0), D = 2, uint32 time: every lane has its own devices (K5's
     bit-sliced words: the op's word at xb + 4v, the successors' at yb + 4·slot, bit `lane`), so
     the device and link choices are per-lane selects, but the control -- first step or not, the
     edge's class -- is the step's and dispatches through 8-entry jump tables."""
@@ -440,6 +456,16 @@ def segment_rows(cpl):
         out = []
         a = ("w0", "w1")[:cpl]
         for c in range(cpl):
+            if v2:
+                out += [f"xor.b32 t, {ywreg[c]}, {X_[c]};", "and.b32 t, t, lm;",
+                        "setp.ne.u32 pc, t, 0;",                                      # crossing
+                        f"selp.u32 u, {L10_[c]}, {L01_[c]}, {PX[c]};",
+                        f"selp.u32 tt, {rec[3]}, {rec[0]}, {PX[c]};",
+                        f"max.u32 u, u, {C[c]};", "add.u32 u, u, tt;", f"min.u32 u, u, {SAT};",
+                        f"@pc selp.u32 {L10_[c]}, u, {L10_[c]}, {PX[c]};",
+                        f"@pc selp.u32 {L01_[c]}, {L01_[c]}, u, {PX[c]};",
+                        f"selp.u32 {a[c]}, u, {C[c]}, pc;"]
+                continue
             out += [f"shr.u32 t, {ywreg[c]}, {LANE_};", "and.b32 t, t, 1;",
                     f"xor.b32 t, t, {X_[c]};", "setp.ne.u32 pc, t, 0;",             # crossing
                     f"selp.u32 u, {L10_[c]}, {L01_[c]}, {PX[c]};",
@@ -478,19 +504,56 @@ def segment_rows(cpl):
     P = ["{",
          ".reg .pred p, q, q2, pc, pq, px0, px1;",
          ".reg .u32 h0, h1, h2, h3, a0, a1, a2, a3, b0, b1, b2, b3, t, u, tt, k0, k1, o, s, sz, "
-         "r0, r1, w0, w1, y0, y1, c0, c1, ya0, ya1, yb0, yb1, xw;",
+         "r0, r1, w0, w1, y0, y1, c0, c1, ya0, ya1, yb0, yb1, xw, lm;",
          ".reg .u64 g, gy;",
          "TA: .branchtargets " + ", ".join(ta) + ";",
-         "TB: .branchtargets " + ", ".join(tb) + ";",
-         "FLOOP:",
+         "TB: .branchtargets " + ", ".join(tb) + ";"]
+    YAn = ("yan0", "yan1")[:cpl]
+    YBn = ("ybn0", "ybn1")[:cpl]
+    XN = ("xn0", "xn1")[:cpl]
+    if ra:
+        P += [".reg .u32 yan0, yan1, ybn0, ybn1, xn0, xn1;"]
+        for c in range(cpl):
+            P += [f"mul.wide.u32 gy, {YS_}, 4;", f"add.u64 gy, {YB_[c]}, gy;",
+                  f"ld.global.nc.v2.u32 {{{YAn[c]}, {YBn[c]}}}, [gy];",
+                  f"add.u32 t, {V_}, 1;", "mul.wide.u32 gy, t, 4;", f"add.u64 gy, {XB_[c]}, gy;",
+                  f"ld.global.nc.u32 {XN[c]}, [gy];"]
+    XWC, XWN = ("xwc0", "xwc1")[:cpl], ("xwn0", "xwn1")[:cpl]
+    YWC, YWN = ("ywc0", "ywc1")[:cpl], ("ywn0", "ywn1")[:cpl]
+    if win:
+        P += [".reg .u32 xwc0, xwc1, xwn0, xwn1, ywc0, ywc1, ywn0, ywn1, xwb, ywb, ix;",
+              f"add.u32 xwb, {V_}, 1;", "and.b32 xwb, xwb, -32;",
+              f"and.b32 ywb, {YS_}, -32;"]
+        for c in range(cpl):
+            P += [f"add.u32 t, xwb, {LANE_};", "mul.wide.u32 gy, t, 4;", f"add.u64 gy, {XB_[c]}, gy;",
+                  f"ld.global.nc.u32 {XWC[c]}, [gy];", f"ld.global.nc.u32 {XWN[c]}, [gy+128];",
+                  f"add.u32 t, ywb, {LANE_};", "mul.wide.u32 gy, t, 4;", f"add.u64 gy, {YB_[c]}, gy;",
+                  f"ld.global.nc.u32 {YWC[c]}, [gy];", f"ld.global.nc.u32 {YWN[c]}, [gy+128];"]
+    if v2:
+        P += [f"shl.b32 lm, 1, {LANE_};"]
+    P += ["FLOOP:",
          f"setp.ge.u32 p, {SP_}, {LIM_};",
          "@p bra.uni FDONE;",
          f"ld.shared.v4.u32 {{h0, h1, h2, h3}}, [{SP_}];",
          f"ld.shared.v4.u32 {{a0, a1, a2, a3}}, [{SP_}+16];",
          f"ld.shared.v4.u32 {{b0, b1, b2, b3}}, [{SP_}+32];"]
-    for c in range(cpl):                # both slots' successor words of candidate group c
+    if win:                             # this step's two slots: shuffles from the window
+        P += [f"sub.u32 ix, {YS_}, ywb;", "setp.ge.u32 p, ix, 32;", "@p bra.uni FYW;", "FYR:"]
+        for c in range(cpl):
+            P += [f"shfl.sync.idx.b32 {YA[c]}, {YWC[c]}, ix, 31, -1;"]
+        P += ["add.u32 ix, ix, 1;"]
+        for c in range(cpl):
+            P += [f"shfl.sync.idx.b32 {YBw[c]}, {YWC[c]}, ix, 31, -1;"]
+    for c in range(cpl if not win else 0):   # both slots' successor words of candidate group c
+        if ra:
+            P += [f"mov.u32 {YA[c]}, {YAn[c]};", f"mov.u32 {YBw[c]}, {YBn[c]};",
+                  f"mul.wide.u32 gy, {YS_}, 4;", f"add.u64 gy, {YB_[c]}, gy;",
+                  f"ld.global.nc.v2.u32 {{{YAn[c]}, {YBn[c]}}}, [gy+8];"]
+            continue
         P += [f"mul.wide.u32 gy, {YS_}, 4;", f"add.u64 gy, {YB_[c]}, gy;",
               f"ld.global.nc.v2.u32 {{{YA[c]}, {YBw[c]}}}, [gy];"]
+        if pf:
+            P += [f"prefetch.global.L1 [gy+{pf}];"]
     P += [f"add.u32 {YS_}, {YS_}, 2;",
           "shr.u32 k0, h1, 1;", "and.b32 k0, k0, 7;",
           "shr.u32 k1, h1, 9;", "and.b32 k1, k1, 7;",
@@ -499,9 +562,22 @@ def segment_rows(cpl):
           "setp.ne.u32 q, t, 0;",
           "@q bra.uni FCONT;",
           f"add.u32 {V_}, {V_}, 1;"]
-    for c in range(cpl):                # the op's device in each lane's row: bit `lane`
-        P += [f"mul.wide.u32 gy, {V_}, 4;", f"add.u64 gy, {XB_[c]}, gy;",
-              "ld.global.nc.u32 xw, [gy];", f"shr.u32 xw, xw, {LANE_};", f"and.b32 {X_[c]}, xw, 1;"]
+    if win:
+        P += [f"sub.u32 ix, {V_}, xwb;", "setp.ge.u32 p, ix, 32;", "@p bra.uni FXW;", "FXR:"]
+        for c in range(cpl):
+            P += [f"shfl.sync.idx.b32 {X_[c]}, {XWC[c]}, ix, 31, -1;"]
+    for c in range(cpl if not win else 0):   # the op's device in each lane's row: bit `lane`
+        if ra:
+            P += [f"mov.u32 {X_[c]}, {XN[c]};", f"mul.wide.u32 gy, {V_}, 4;",
+                  f"add.u64 gy, {XB_[c]}, gy;", f"ld.global.nc.u32 {XN[c]}, [gy+4];"]
+            continue
+        P += [f"mul.wide.u32 gy, {V_}, 4;", f"add.u64 gy, {XB_[c]}, gy;"]
+        if v2:
+            P += [f"ld.global.nc.u32 {X_[c]}, [gy];"]
+        else:
+            P += ["ld.global.nc.u32 xw, [gy];", f"shr.u32 xw, xw, {LANE_};", f"and.b32 {X_[c]}, xw, 1;"]
+        if pf:
+            P += [f"prefetch.global.L1 [gy+{pf // 2}];"]
     P += [f"add.u32 t, {V_}, 11;", "and.b32 t, t, 15;", f"shl.b32 t, t, {sh};",
           f"add.u32 s, {STAGE_}, t;",
           "setp.ge.s32 p, h2, 0;", "max.s32 t, h2, 0;", f"mul.wide.u32 g, t, {SLOT};",
@@ -521,16 +597,18 @@ def segment_rows(cpl):
     P += [f"mov.u32 {FWD_[c]}, 0;" for c in range(cpl)]
     # C_v = min(max(r, dev_free[x]) + p, SAT) per lane, dev_free[x] = C_v
     for c in range(cpl):
-        P += [f"setp.ne.u32 {PX[c]}, {X_[c]}, 0;",
-              f"selp.u32 t, {D1_[c]}, {D0_[c]}, {PX[c]};",
+        P += ([f"and.b32 t, {X_[c]}, lm;", f"setp.ne.u32 {PX[c]}, t, 0;"] if v2 else
+              [f"setp.ne.u32 {PX[c]}, {X_[c]}, 0;"])
+        P += [f"selp.u32 t, {D1_[c]}, {D0_[c]}, {PX[c]};",
               f"max.u32 {C[c]}, r{c}, t;", f"add.u32 {C[c]}, {C[c]}, h0;",
               f"min.u32 {C[c]}, {C[c]}, {SAT};",
               f"@{PX[c]} mov.u32 {D1_[c]}, {C[c]};", f"@!{PX[c]} mov.u32 {D0_[c]}, {C[c]};"]
     P += ["brx.idx.uni k0, TA;",
           "FCONT:"]                     # a continuation: dev_free[x] still holds C_v
     for c in range(cpl):
-        P += [f"setp.ne.u32 {PX[c]}, {X_[c]}, 0;",
-              f"selp.u32 {C[c]}, {D1_[c]}, {D0_[c]}, {PX[c]};"]
+        P += ([f"and.b32 t, {X_[c]}, lm;", f"setp.ne.u32 {PX[c]}, t, 0;"] if v2 else
+              [f"setp.ne.u32 {PX[c]}, {X_[c]}, 0;"])
+        P += [f"selp.u32 {C[c]}, {D1_[c]}, {D0_[c]}, {PX[c]};"]
     P += ["add.u32 k0, k0, 8;",
           "brx.idx.uni k0, TA;"]
     for i in range(16):
@@ -547,7 +625,20 @@ def segment_rows(cpl):
             P += edge_rows(i, B, YBw)
         if i < 7:
             P.append("bra.uni FNEXT;")
-    P += ["FNEXT:", f"add.u32 {SP_}, {SP_}, 48;", "bra.uni FLOOP;", "FDONE:", "}"]
+    P += ["FNEXT:", f"add.u32 {SP_}, {SP_}, 48;", "bra.uni FLOOP;"]
+    if win:                             # window switches, out of line
+        P += ["FYW:", "add.u32 ywb, ywb, 32;"]
+        for c in range(cpl):
+            P += [f"mov.u32 {YWC[c]}, {YWN[c]};", f"add.u32 t, ywb, {LANE_};",
+                  "mul.wide.u32 gy, t, 4;", f"add.u64 gy, {YB_[c]}, gy;",
+                  f"ld.global.nc.u32 {YWN[c]}, [gy+128];"]
+        P += [f"sub.u32 ix, {YS_}, ywb;", "bra.uni FYR;", "FXW:", "add.u32 xwb, xwb, 32;"]
+        for c in range(cpl):
+            P += [f"mov.u32 {XWC[c]}, {XWN[c]};", f"add.u32 t, xwb, {LANE_};",
+                  "mul.wide.u32 gy, t, 4;", f"add.u64 gy, {XB_[c]}, gy;",
+                  f"ld.global.nc.u32 {XWN[c]}, [gy+128];"]
+        P += [f"sub.u32 ix, {V_}, xwb;", "bra.uni FXR;"]
+    P += ["FDONE:", "}"]
     return P
 
 
@@ -566,10 +657,18 @@ def main():
                     " \\\n".join('    "' + l + '\\n"' for l in P) + "\n")
             print(OUT, name, len(P), "PTX lines")
         for cpl in (1, 2):
-            P = segment_rows(cpl)
-            f.write(f"#define PESTO_FAST_ROWS_PTX{cpl} \\\n" +
-                    " \\\n".join('    "' + l + '\\n"' for l in P) + "\n")
-            print(OUT, f"{cpl}_ROWS", len(P), "PTX lines")
+            for pf, v2, ra, suf in ((0, False, False, ""), (512, False, False, "_PF"),
+                                    (0, True, False, "_V2"), (512, True, False, "_V2PF"),
+                                    (0, True, True, "_V3")):
+                P = segment_rows(cpl, pf, v2, ra)
+                f.write(f"#define PESTO_FAST_ROWS_PTX{cpl}{suf} \\\n" +
+                        " \\\n".join('    "' + l + '\\n"' for l in P) + "\n")
+                print(OUT, f"{cpl}_ROWS{suf}", len(P), "PTX lines")
+            for suf in ("_V4",):
+                P = segment_rows(cpl, 0, True, False, True)
+                f.write(f"#define PESTO_FAST_ROWS_PTX{cpl}{suf} \\\n" +
+                        " \\\n".join('    "' + l + '\\n"' for l in P) + "\n")
+                print(OUT, f"{cpl}_ROWS{suf}", len(P), "PTX lines")
         for cpl in (1, 2):
             P = segment_d4(cpl)
             f.write(f"#define PESTO_FAST_WALK_PTX{cpl}_D4 \\\n" +
