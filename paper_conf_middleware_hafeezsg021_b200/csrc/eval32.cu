@@ -498,6 +498,15 @@ __device__ __forceinline__ void uni_edge(const Ctx32 &cx, const uint4 rec, const
 #define PESTO_FW2 PESTO_FAST_WALK_PTX2
 #define PESTO_FW1W PESTO_FAST_WALK_PTX1W
 #endif
+// the far-arrival copy of the two-candidates-per-lane fast walk as one 16-byte cp.async.cg per
+// even lane (gen_fast_walk.py segment ce)
+#ifndef PESTO_FAST_CE
+#define PESTO_FAST_CE 1
+#endif
+#if PESTO_FAST_CE
+#undef PESTO_FW2
+#define PESTO_FW2 PESTO_FAST_WALK_PTX2_CE
+#endif
 
 // the uniform steps from sp on (until lim or the first step of the special position nspec),
 // state in registers; returns with sp at the first step it did not take

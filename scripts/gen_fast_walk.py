@@ -118,8 +118,11 @@ def begin(xu):
     return out
 
 
-def segment(cpl, wide=False, ra=False, dt=False, early=False):
-    """ra: the next step's head is read one step ahead (its kinds feed the jump-table load
+def segment(cpl, wide=False, ra=False, dt=False, early=False, ce=False):
+    """ce (two candidates per lane, uint32): the far-arrival copy is one 16-byte cp.async.cg by
+    every even lane (its own and its odd neighbour's pair) instead of an 8-byte cp.async.ca by
+    every lane.
+    ra: the next step's head is read one step ahead (its kinds feed the jump-table load
     before the current step's work; 4 register moves per step).  dt: direct threading -- every
     handler ends with its own copy of the loop's top (limit check, record loads, first-step
     work, dispatch), so no join point sits inside the loop (ptxas otherwise brackets every
@@ -141,6 +144,8 @@ def segment(cpl, wide=False, ra=False, dt=False, early=False):
           ".reg .u64 g, z;",
           "TA: .branchtargets " + ", ".join(ta) + ";",
           "TB: .branchtargets " + ", ".join(tb) + ";"]
+    if ce:
+        P += [".reg .pred pe;", "mov.u32 t, %laneid;", "and.b32 t, t, 1;", "setp.eq.u32 pe, t, 0;"]
     if ra:
         P += [".reg .u32 n0, n1, n2, n3;",
               f"ld.shared.v4.u32 {{n0, n1, n2, n3}}, [{SP}];"]
@@ -175,8 +180,10 @@ def segment(cpl, wide=False, ra=False, dt=False, early=False):
               f"add.u32 t, {V}, 11;", "and.b32 t, t, 15;", f"shl.b32 t, t, {sh};",
               f"add.u32 s, {STAGE}, t;",
               "setp.ge.s32 p, h2, 0;", "max.s32 t, h2, 0;", f"mul.wide.u32 g, t, {cb};",
-              f"add.u64 g, {COLD}, g;", f"selp.u32 sz, {8 if IL else TB_}, 0, p;"]
-        if IL:
+              f"add.u64 g, {COLD}, g;", f"selp.u32 sz, {(16 if ce else 8) if IL else TB_}, 0, p;"]
+        if IL and ce:
+            T += ["@pe cp.async.cg.shared.global [s], [g], 16, sz;"]
+        elif IL:
             T += ["cp.async.ca.shared.global [s], [g], 8, sz;"]
         else:
             T += [f"cp.async.ca.shared.global [s+{CB * c}], [g+{CB * c}], {TB_}, sz;"
@@ -653,6 +660,13 @@ def main():
                                         (1, False, False, True, "1_DT"), (2, False, False, True, "2_DT"),
                                         (1, True, False, True, "1W_DT")):
             P = segment(cpl, wide, ra, dt, early=dt)
+            f.write(f"#define PESTO_FAST_WALK_PTX{name} \\\n" +
+                    " \\\n".join('    "' + l + '\\n"' for l in P) + "\n")
+            print(OUT, name, len(P), "PTX lines")
+            if name != "2":
+                continue
+            name = "2_CE"
+            P = segment(cpl, wide, ra, dt, early=dt, ce=True)
             f.write(f"#define PESTO_FAST_WALK_PTX{name} \\\n" +
                     " \\\n".join('    "' + l + '\\n"' for l in P) + "\n")
             print(OUT, name, len(P), "PTX lines")

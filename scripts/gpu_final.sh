@@ -34,5 +34,15 @@ timeout 900 ncu --set full --clock-control none --import-source on -k regex:eval
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv \
   --log-file gpurun_out/launches_${TAG}_default.csv python bench.py --steps 3 --warmup 3 --no-cpu-baseline \
   > gpurun_out/ncu_launch_${TAG}_default.log 2>&1
+# the explicit-row (e2e) kernels: device times, K1 mode 0 and K5 captures
+for c in transformer_2dev inception_v3_2dev; do
+  timeout 300 python scripts/time_rows.py $c >> gpurun_out/${TAG}_rows.log 2>&1
+done
+timeout 600 ncu --set full --clock-control none --import-source on -k regex:eval32_kernel -s 1 -c 1 \
+  -o gpurun_out/prof_${TAG}_rows python scripts/time_rows.py transformer_2dev > gpurun_out/ncu_${TAG}_rows.log 2>&1
+timeout 600 ncu --set full --clock-control none --import-source on -k regex:transpose -s 1 -c 1 \
+  -o gpurun_out/prof_${TAG}_k5 python scripts/time_rows.py transformer_2dev > gpurun_out/ncu_${TAG}_k5.log 2>&1
+timeout 300 ncu --metrics gpu__time_duration.sum --clock-control none --csv \
+  --log-file gpurun_out/launches_${TAG}_rows.csv python scripts/time_rows.py transformer_2dev > /dev/null 2>&1
 [ -n "$SAN" ] && bash scripts/gpu_sanitize.sh
 echo done

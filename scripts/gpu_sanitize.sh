@@ -6,7 +6,7 @@ mkdir -p gpurun_out
 CS=/usr/local/cuda/bin/compute-sanitizer
 python tests/tools/sanitize_run.py > gpurun_out/san_plain.log 2>&1; echo "rc=$?" >> gpurun_out/san_plain.log
 for cpl in 1 2; do
-  for tool in memcheck racecheck synccheck initcheck; do
+  for tool in ${TOOLS:-memcheck racecheck synccheck initcheck}; do
     extra=""
     [ $tool = memcheck ] && extra="--leak-check no"
     [ $tool = racecheck ] && extra="--racecheck-report all"
