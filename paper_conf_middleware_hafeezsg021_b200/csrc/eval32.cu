@@ -503,7 +503,13 @@ __device__ __forceinline__ void uni_edge(const Ctx32 &cx, const uint4 rec, const
 #ifndef PESTO_FAST_CE
 #define PESTO_FAST_CE 1
 #endif
-#if PESTO_FAST_CE
+#ifndef PESTO_FAST_KS
+#define PESTO_FAST_KS 0
+#endif
+#if PESTO_FAST_CE && PESTO_FAST_KS
+#undef PESTO_FW2
+#define PESTO_FW2 PESTO_FAST_WALK_PTX2_CEKS
+#elif PESTO_FAST_CE
 #undef PESTO_FW2
 #define PESTO_FW2 PESTO_FAST_WALK_PTX2_CE
 #endif

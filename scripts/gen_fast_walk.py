@@ -118,8 +118,10 @@ def begin(xu):
     return out
 
 
-def segment(cpl, wide=False, ra=False, dt=False, early=False, ce=False):
-    """ce (two candidates per lane, uint32): the far-arrival copy is one 16-byte cp.async.cg by
+def segment(cpl, wide=False, ra=False, dt=False, early=False, ce=False, ks=False):
+    """ks: edge 1's table entry is extracted from the head inside the edge-0 handlers, after the
+    slot-1-empty test (77% of steps have no edge 1), instead of at the loop top.
+    ce (two candidates per lane, uint32): the far-arrival copy is one 16-byte cp.async.cg by
     every even lane (its own and its odd neighbour's pair) instead of an 8-byte cp.async.ca by
     every lane.
     ra: the next step's head is read one step ahead (its kinds feed the jump-table load
@@ -165,9 +167,11 @@ def segment(cpl, wide=False, ra=False, dt=False, early=False, ce=False):
               f"ld.shared.v4.u32 {{b0, b1, b2, b3}}, [{SP}+32];",
               # the slots' jump-table entries, kept by the layout / K4 / swap patches
               # (StepHead.kinds: yu | class << 1 | xu << 4 per slot byte)
-              "and.b32 k0, h1, 31;",
-              "shr.u32 k1, h1, 8;",
-              "and.b32 k1, k1, 31;",
+              "and.b32 k0, h1, 31;"]
+        if not ks:
+            T += ["shr.u32 k1, h1, 8;",
+                  "and.b32 k1, k1, 31;"]
+        T += [
               "and.b32 t, h1, 0xE00;",
               "setp.eq.u32 q2, t, 0xA00;",            # slot 1 empty (class 5): no TB dispatch
               "and.b32 t, h3, 16;",
@@ -241,7 +245,10 @@ def segment(cpl, wide=False, ra=False, dt=False, early=False, ce=False):
         if dt:
             P += [f"@q2 bra.uni FTA{i};", "brx.idx.uni k1, TB;", f"FTA{i}:"] + tail(f"A{i}")
         else:
-            P += ["@q2 bra.uni FNEXT;", "brx.idx.uni k1, TB;"]
+            P += ["@q2 bra.uni FNEXT;"]
+            if ks:
+                P += ["shr.u32 k1, h1, 8;", "and.b32 k1, k1, 31;"]
+            P += ["brx.idx.uni k1, TB;"]
     for i in range(32):
         xu, cls, cross = decode(i)
         P.append(f"FB{i}:")
@@ -667,6 +674,11 @@ def main():
                 continue
             name = "2_CE"
             P = segment(cpl, wide, ra, dt, early=dt, ce=True)
+            f.write(f"#define PESTO_FAST_WALK_PTX{name} \\\n" +
+                    " \\\n".join('    "' + l + '\\n"' for l in P) + "\n")
+            print(OUT, name, len(P), "PTX lines")
+            name = "2_CEKS"
+            P = segment(cpl, wide, ra, dt, early=dt, ce=True, ks=True)
             f.write(f"#define PESTO_FAST_WALK_PTX{name} \\\n" +
                     " \\\n".join('    "' + l + '\\n"' for l in P) + "\n")
             print(OUT, name, len(P), "PTX lines")
