@@ -419,8 +419,12 @@ def segment_d4(cpl):
     return P
 
 
-def segment_rows(cpl, pf=0, v2=False, ra=False, win=False):
-    """win (with v2): both word streams are read 32 words at a time -- lane l loads word
+def segment_rows(cpl, pf=0, v2=False, ra=False, win=False, fold=False):
+    """fold (with win): the successor-word window switch rides on the step's dispatch -- the
+    edge-0 table index carries bit 5 = "this step's slots are in the next window" and those 16
+    entries switch the window, redo the step's two shuffles and continue in the normal handler --
+    instead of an if-converted block that ptxas executes (predicated) on every step.
+    win (with v2): both word streams are read 32 words at a time -- lane l loads word
     base + l with one coalesced load, the next window is loaded a window ahead (out of line, once
     per 32 ops / 16 steps) and a step takes its words with warp shuffles, so no step waits on a
     global load (ra's register read-ahead was undone by ptxas, which copied the loaded word into
@@ -514,6 +518,8 @@ def segment_rows(cpl, pf=0, v2=False, ra=False, win=False):
     YA = ("ya0", "ya1")[:cpl]           # slot-0 successor words per candidate group
     YBw = ("yb0", "yb1")[:cpl]          # slot-1
     ta = [f"FA{i}" for i in range(16)]
+    if fold:                            # entries 32-47: window switch, then FA{i}
+        ta += ["FDONE"] * 16 + [f"FS{i}" for i in range(16)]
     tb = [f"FB{i}" for i in range(8)]
     P = ["{",
          ".reg .pred p, q, q2, pc, pq, px0, px1;",
@@ -535,7 +541,7 @@ def segment_rows(cpl, pf=0, v2=False, ra=False, win=False):
     XWC, XWN = ("xwc0", "xwc1")[:cpl], ("xwn0", "xwn1")[:cpl]
     YWC, YWN = ("ywc0", "ywc1")[:cpl], ("ywn0", "ywn1")[:cpl]
     if win:
-        P += [".reg .u32 xwc0, xwc1, xwn0, xwn1, ywc0, ywc1, ywn0, ywn1, xwb, ywb, ix;",
+        P += [".reg .u32 xwc0, xwc1, xwn0, xwn1, ywc0, ywc1, ywn0, ywn1, xwb, ywb, ix, iy, sw;",
               f"add.u32 xwb, {V_}, 1;", "and.b32 xwb, xwb, -32;",
               f"and.b32 ywb, {YS_}, -32;"]
         for c in range(cpl):
@@ -551,7 +557,15 @@ def segment_rows(cpl, pf=0, v2=False, ra=False, win=False):
          f"ld.shared.v4.u32 {{h0, h1, h2, h3}}, [{SP_}];",
          f"ld.shared.v4.u32 {{a0, a1, a2, a3}}, [{SP_}+16];",
          f"ld.shared.v4.u32 {{b0, b1, b2, b3}}, [{SP_}+32];"]
-    if win:                             # this step's two slots: shuffles from the window
+    if fold:                            # shuffles from the current window; a step whose
+        # slots lie in the next one (iy >= 32) redoes them in its FS entry after the switch
+        P += [f"sub.u32 iy, {YS_}, ywb;", "and.b32 sw, iy, 32;"]
+        for c in range(cpl):
+            P += [f"shfl.sync.idx.b32 {YA[c]}, {YWC[c]}, iy, 31, -1;"]
+        P += ["add.u32 t, iy, 1;"]
+        for c in range(cpl):
+            P += [f"shfl.sync.idx.b32 {YBw[c]}, {YWC[c]}, t, 31, -1;"]
+    elif win:                           # this step's two slots: shuffles from the window
         P += [f"sub.u32 ix, {YS_}, ywb;", "setp.ge.u32 p, ix, 32;", "@p bra.uni FYW;", "FYR:"]
         for c in range(cpl):
             P += [f"shfl.sync.idx.b32 {YA[c]}, {YWC[c]}, ix, 31, -1;"]
@@ -569,7 +583,10 @@ def segment_rows(cpl, pf=0, v2=False, ra=False, win=False):
         if pf:
             P += [f"prefetch.global.L1 [gy+{pf}];"]
     P += [f"add.u32 {YS_}, {YS_}, 2;",
-          "shr.u32 k0, h1, 1;", "and.b32 k0, k0, 7;",
+          "shr.u32 k0, h1, 1;", "and.b32 k0, k0, 7;"]
+    if fold:
+        P += ["or.b32 k0, k0, sw;"]
+    P += [
           "shr.u32 k1, h1, 9;", "and.b32 k1, k1, 7;",
           "setp.eq.u32 q2, k1, 5;",             # slot 1 empty: no TB dispatch
           "and.b32 t, h3, 16;",
@@ -640,13 +657,29 @@ def segment_rows(cpl, pf=0, v2=False, ra=False, win=False):
         if i < 7:
             P.append("bra.uni FNEXT;")
     P += ["FNEXT:", f"add.u32 {SP_}, {SP_}, 48;", "bra.uni FLOOP;"]
-    if win:                             # window switches, out of line
+    if fold:                            # the successor-word window switch (entries 32-47)
+        for i in range(16):
+            P += [f"FS{i}:", "add.u32 ywb, ywb, 32;"]
+            for c in range(cpl):
+                P += [f"mov.u32 {YWC[c]}, {YWN[c]};", f"add.u32 t, ywb, {LANE_};",
+                      "mul.wide.u32 gy, t, 4;", f"add.u64 gy, {YB_[c]}, gy;",
+                      f"ld.global.nc.u32 {YWN[c]}, [gy+128];"]
+            P += ["sub.u32 iy, iy, 32;"]
+            for c in range(cpl):
+                P += [f"shfl.sync.idx.b32 {YA[c]}, {YWC[c]}, iy, 31, -1;"]
+            P += ["add.u32 t, iy, 1;"]
+            for c in range(cpl):
+                P += [f"shfl.sync.idx.b32 {YBw[c]}, {YWC[c]}, t, 31, -1;"]
+            P += [f"bra.uni FA{i};"]
+    if win and not fold:                # window switches, out of line
         P += ["FYW:", "add.u32 ywb, ywb, 32;"]
         for c in range(cpl):
             P += [f"mov.u32 {YWC[c]}, {YWN[c]};", f"add.u32 t, ywb, {LANE_};",
                   "mul.wide.u32 gy, t, 4;", f"add.u64 gy, {YB_[c]}, gy;",
                   f"ld.global.nc.u32 {YWN[c]}, [gy+128];"]
-        P += [f"sub.u32 ix, {YS_}, ywb;", "bra.uni FYR;", "FXW:", "add.u32 xwb, xwb, 32;"]
+        P += [f"sub.u32 ix, {YS_}, ywb;", "bra.uni FYR;"]
+    if win:
+        P += ["FXW:", "add.u32 xwb, xwb, 32;"]
         for c in range(cpl):
             P += [f"mov.u32 {XWC[c]}, {XWN[c]};", f"add.u32 t, xwb, {LANE_};",
                   "mul.wide.u32 gy, t, 4;", f"add.u64 gy, {XB_[c]}, gy;",
@@ -690,8 +723,8 @@ def main():
                 f.write(f"#define PESTO_FAST_ROWS_PTX{cpl}{suf} \\\n" +
                         " \\\n".join('    "' + l + '\\n"' for l in P) + "\n")
                 print(OUT, f"{cpl}_ROWS{suf}", len(P), "PTX lines")
-            for suf in ("_V4",):
-                P = segment_rows(cpl, 0, True, False, True)
+            for suf, fold in (("_V4", False), ("_V5", True)):
+                P = segment_rows(cpl, 0, True, False, True, fold)
                 f.write(f"#define PESTO_FAST_ROWS_PTX{cpl}{suf} \\\n" +
                         " \\\n".join('    "' + l + '\\n"' for l in P) + "\n")
                 print(OUT, f"{cpl}_ROWS{suf}", len(P), "PTX lines")
