@@ -44,5 +44,9 @@ timeout 600 ncu --set full --clock-control none --import-source on -k regex:tran
   -o gpurun_out/prof_${TAG}_k5 python scripts/time_rows.py transformer_2dev > gpurun_out/ncu_${TAG}_k5.log 2>&1
 timeout 300 ncu --metrics gpu__time_duration.sum --clock-control none --csv \
   --log-file gpurun_out/launches_${TAG}_rows.csv python scripts/time_rows.py transformer_2dev > /dev/null 2>&1
+# the launcher path the driver's scaling run uses (torchrun, env rendezvous), at one rank
+timeout 600 python -m torch.distributed.run --nnodes=1 --nproc-per-node 1 --master-addr 127.0.0.1 \
+  --master-port 29533 bench.py --gpus 1 --steps 5 --warmup 3 --no-cpu-baseline > gpurun_out/${TAG}_torchrun.log 2>&1
+echo "torchrun rc=$?" >> gpurun_out/${TAG}_torchrun.log
 [ -n "$SAN" ] && bash scripts/gpu_sanitize.sh
 echo done
