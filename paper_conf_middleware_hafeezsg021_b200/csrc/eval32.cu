@@ -99,14 +99,24 @@ constexpr bool kHeadAhead = PESTO_HEAD_AHEAD2 != 0;
 #define PESTO_FAST_ROWS 1
 #endif
 constexpr bool kUniSwitch = PESTO_UNI_SWITCH != 0;
-__host__ __device__ constexpr int min_blocks_for(int cpl) { return cpl == 1 ? PESTO_E32_MINB1 : PESTO_E32_MINB2; }
+// the no-producer instance (np: the consumer that releases a stage last issues its next load)
+// targets five CTAs per SM: 128 threads, no warp slot or registers spent on a mostly sleeping
+// producer
+#ifndef PESTO_E32_MINB_NP
+#define PESTO_E32_MINB_NP 5
+#endif
+__host__ __device__ constexpr int min_blocks_for(int cpl, bool np = false) {
+    return np ? PESTO_E32_MINB_NP : (cpl == 1 ? PESTO_E32_MINB1 : PESTO_E32_MINB2);
+}
 // tile loads: a producer warp per CTA (0), or issued by the consumer warp that releases a stage
 // last (1: no warp slot and no registers spent on a warp that mostly sleeps)
 #ifndef PESTO_E32_NOPROD
 #define PESTO_E32_NOPROD 0
 #endif
 constexpr bool kProducerWarp = PESTO_E32_NOPROD == 0;
-__host__ __device__ constexpr int threads_for(int cpl) { return (warps_for(cpl) + (kProducerWarp ? 1 : 0)) * 32; }
+__host__ __device__ constexpr int threads_for(int cpl, bool np = false) {
+    return (warps_for(cpl) + (kProducerWarp && !np ? 1 : 0)) * 32;
+}
 
 // per-candidate device / link free times
 template <int CPL, class T>
@@ -723,9 +733,10 @@ __device__ __forceinline__ void begin32(const uint4 h, StateT &st, const T (&r)[
     }
 }
 
-template <int MODE, int PL, int CPL, class T>
-__global__ void __launch_bounds__(threads_for(CPL), min_blocks_for(CPL))
+template <int MODE, int PL, int CPL, class T, bool NP = false>
+__global__ void __launch_bounds__(threads_for(CPL, NP), min_blocks_for(CPL, NP))
 eval32_kernel(const EvalParams P) {
+    constexpr bool kProd = kProducerWarp && !NP;       // a producer warp loads the tiles
     constexpr bool kSearch = MODE == 1 || MODE == 5;   // 5: search with S9 coarse groups
     // uniform steps through the PTX fast segment (D = 2, CPL 2, 32-bit time, search)
     // explicit rows, D = 2, 32-bit time: every step through the PTX rows segment
@@ -785,11 +796,11 @@ eval32_kernel(const EvalParams P) {
     if (threadIdx.x == 0) {
         for (int s = 0; s < kStages32; s++) {
             mbar_init(&full[s], 1);
-            if constexpr (kProducerWarp) mbar_init(&empty[s], NW);
+            if constexpr (kProd) mbar_init(&empty[s], NW);
             else empty[s] = 0;
         }
         mbar_fence_init();
-        if constexpr (!kProducerWarp) {
+        if constexpr (!kProd) {
             int64_t task = first_task(blockIdx.x);
             int t = 0;
             for (int s = 0; s < kStages32; s++) {
@@ -800,7 +811,7 @@ eval32_kernel(const EvalParams P) {
     }
     __syncthreads();
 
-    if (kProducerWarp && warp == NW) {
+    if (kProd && warp == NW) {
         if (lane == 0) {
             uint32_t it = 0;
             for (int64_t task = blockIdx.x; task < P.n_tasks; task += gridDim.x) {
@@ -1333,7 +1344,7 @@ eval32_kernel(const EvalParams P) {
                 }
             }
             __syncwarp();
-            if constexpr (kProducerWarp) {
+            if constexpr (kProd) {
                 if (lane == 0) mbar_arrive(&empty[s]);
             } else if (lane == 0) {
                 // the warp that releases stage s last loads the CTA's tile kStages32 iterations
@@ -1388,11 +1399,20 @@ eval32_kernel(const EvalParams P) {
     }
 }
 
+// the no-producer five-CTA instance: search, D = 2, two candidates per lane, 32-bit time
+template <int MODE, int PL, int CPL>
+constexpr bool kHasNp = MODE == 1 && PL == 1 && CPL == 2;
+template <int MODE, int PL, int CPL>
+bool use_np(const EvalParams &p) { return kHasNp<MODE, PL, CPL> && p.np32 && !p.wide32; }
+
 template <int MODE, int PL, int CPL>
 auto kernel_for(const EvalParams &p) {
     // the wide (exact 64-bit) instance serves search bases at or above saturation only
     if constexpr (MODE == 1 || MODE == 5) {
         if (p.wide32) return eval32_kernel<MODE, PL, CPL, uint64_t>;
+    }
+    if constexpr (kHasNp<MODE, PL, CPL>) {
+        if (use_np<MODE, PL, CPL>(p)) return eval32_kernel<MODE, PL, CPL, uint32_t, true>;
     }
     return eval32_kernel<MODE, PL, CPL, uint32_t>;
 }
@@ -1410,7 +1430,7 @@ cudaError_t launch_one32(const EvalParams &p, int grid, cudaStream_t st) {
         (e = cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout,
                                   cudaSharedmemCarveoutMaxShared)) != cudaSuccess)
         return e;
-    kern<<<grid, threads_for(CPL), smem, st>>>(p);
+    kern<<<grid, threads_for(CPL, use_np<MODE, PL, CPL>(p)), smem, st>>>(p);
     return cudaGetLastError();
 }
 
@@ -1421,7 +1441,7 @@ int occupancy_one32(const EvalParams &p) {
     if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) != cudaSuccess)
         return 0;
     int n = 0;
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kern, threads_for(CPL), smem) !=
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kern, threads_for(CPL, use_np<MODE, PL, CPL>(p)), smem) !=
         cudaSuccess)
         return 0;
     return n;

@@ -9,6 +9,7 @@ namespace pesto {
 
 constexpr int kWarps = 8;            // consumer warps per CTA (each = 32 candidates)
 constexpr int kStages = 4;           // TMA tile ring depth
+constexpr int kTileTarget32Search = 6144;   // eval32 search layouts, D = 2 (five CTAs per SM)
 constexpr int kTileTarget = 8192;    // record bytes per tile (a single op may exceed it)
 constexpr int kTileHeader = 16;      // {pos_begin, pos_end, bytes, 0} at the head of each tile
 
@@ -97,6 +98,9 @@ struct EvalParams {
     // eval32 search (mode 1): 1 = the wide instance (exact 64-bit times, same records) for the
     // bases at or above saturation (gate 2)
     int32_t wide32;
+    // eval32 search, two candidates per lane, 32-bit time, launched alone (no wide launch
+    // beside it): 1 = the instance without a producer warp at five CTAs per SM
+    int32_t np32;
     // 1: FCFS link queues; 0: congestion-free links (row f4(ii))
     int32_t link_queue;
     // row f3 feasibility (search mode prologue): memory caps and colocation

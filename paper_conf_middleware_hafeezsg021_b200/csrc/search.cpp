@@ -280,6 +280,15 @@ pesto_status launch_search_eval(pesto_search *s, int b_first, int n_bases, int64
             if ((e = launch_eval32(p32, 1, grid, st)) != cudaSuccess) return cuda_fail(e, "launch wide eval32");
             return PESTO_OK;
         }
+        // launched alone (no wide launch beside it), the two-candidates-per-lane 32-bit walk
+        // runs without a producer warp at five CTAs per SM (PESTO_E32_NP=0
+        // keeps the producer warp): transformer_2dev 35.9 -> 35.0 ms per step.  Beside a wide
+        // launch (nmt4's saturated bases) the producer instance is faster (29.0 vs 31.7 ms).
+        static const bool np_on = [] {
+            const char *e = std::getenv("PESTO_E32_NP");
+            return !(e && std::atoi(e) == 0);
+        }();
+        p32.np32 = (np_on && s->all_below && p32.cpl32 == 2 && g->planes == 1) ? 1 : 0;
         if ((rc = ensure_state32(g, g->ws, p32, 1, p32.n_tasks, &grid))) return rc;
         p32.state32 = g->ws.state32.as<uint32_t>();
         if (s->all_below) {
