@@ -1401,7 +1401,7 @@ eval32_kernel(const EvalParams P) {
 
 // the no-producer five-CTA instance: search, D = 2, two candidates per lane, 32-bit time
 template <int MODE, int PL, int CPL>
-constexpr bool kHasNp = MODE == 1 && PL == 1 && CPL == 2;
+constexpr bool kHasNp = (MODE == 1 || MODE == 0) && PL == 1 && CPL == 2;
 template <int MODE, int PL, int CPL>
 bool use_np(const EvalParams &p) { return kHasNp<MODE, PL, CPL> && p.np32 && !p.wide32; }
 

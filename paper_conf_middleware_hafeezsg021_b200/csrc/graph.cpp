@@ -853,6 +853,15 @@ pesto_status eval_batch_ws(pesto_graph *g, Scratch &ws, const int32_t *order, co
             p32.tasks_per_base = (n_cand + ts - 1) / ts;
             p32.n_tasks = p32.tasks_per_base;
         }
+        // many-wave batches (>= 4 waves at five CTAs per SM) of two candidates per lane run the
+        // no-producer instance at five CTAs per SM (PESTO_E32_NP=0 disables it);
+        // one-wave batches keep room on the SMs for the next batch in flight
+        static const bool np_on = [] {
+            const char *v = std::getenv("PESTO_E32_NP");
+            return !(v && std::atoi(v) == 0);
+        }();
+        p32.np32 = (np_on && p32.cpl32 == 2 && g->planes == 1 &&
+                    p32.n_tasks >= 4 * 5 * (int64_t)g->sms) ? 1 : 0;
         if ((s = ensure_state32(g, ws, p32, 0, p32.n_tasks, &grid))) return s;
         p32.state32 = ws.state32.as<uint32_t>();
         if ((e = launch_eval32(p32, 0, grid, st)) != cudaSuccess) return cuda_fail(e, "launch eval32");

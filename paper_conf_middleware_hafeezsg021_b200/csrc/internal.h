@@ -9,7 +9,7 @@ namespace pesto {
 
 constexpr int kWarps = 8;            // consumer warps per CTA (each = 32 candidates)
 constexpr int kStages = 4;           // TMA tile ring depth
-constexpr int kTileTarget32Search = 6144;   // eval32 search layouts, D = 2 (five CTAs per SM)
+constexpr int kTileTarget32Search = 6144;   // eval32 layouts, D = 2 (five CTAs per SM)
 constexpr int kTileTarget = 8192;    // record bytes per tile (a single op may exceed it)
 constexpr int kTileHeader = 16;      // {pos_begin, pos_end, bytes, 0} at the head of each tile
 

@@ -301,17 +301,17 @@ pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<
         };
         // eval32 tile budget: kTileTarget, or PESTO_TILE32_BYTES (occupancy experiments: a smaller
         // tile lets more CTAs' stages fit in shared memory)
-        // Search layouts of D = 2 graphs use 6 KB tiles, so that five CTAs of the no-producer
-        // instance fit in shared memory (measured neutral for the producer instance:
-        // transformer_2dev 35.93 / 35.95 ms, nmt4 29.02 / 28.92 ms at 8 / 6 KB)
+        // eval32 layouts of D = 2 graphs (search and explicit rows) use 6 KB tiles, so that five
+        // CTAs of the no-producer instance fit in shared memory (measured neutral for the
+        // producer instance: transformer_2dev 35.93 / 35.95 ms, nmt4 29.02 / 28.92 ms at 8 / 6 KB)
         static const size_t env_budget = [] {
             const char *e = std::getenv("PESTO_TILE32_BYTES");
             const long v = e ? std::atol(e) : 0;
             return (size_t)(v >= 1024 && v <= 65536 ? (v & ~15L) : 0);
         }();
         const size_t budget = env_budget ? env_budget
-                                         : (x_op && g->planes == 1 ? (size_t)kTileTarget32Search
-                                                                   : (size_t)kTileTarget);
+                                         : (g->planes == 1 ? (size_t)kTileTarget32Search
+                                                           : (size_t)kTileTarget);
         open();
         for (int32_t k = 0; k < n; k++) {
             const int32_t u = order[k];
