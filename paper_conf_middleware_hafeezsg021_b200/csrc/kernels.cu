@@ -512,11 +512,16 @@ __global__ void __launch_bounds__(256) transpose_kernel(const TransposeParams P)
 #define PESTO_T16 4
 #endif
 constexpr int kT16 = PESTO_T16;
+// successor positions per thread in flight in K5's edge-slot gather: 16 where shared memory
+// allows two CTAs per SM anyway (large graphs: 99 registers fit), 8 where three fit (80 registers)
+// -- transformer_2dev, 1 M rows: 6.89 -> 5.68 ms; inception at 16 would drop to two CTAs per SM
 #ifndef PESTO_YU
 #define PESTO_YU 8
 #endif
-constexpr int kYU = PESTO_YU;
-template <int PL>
+#ifndef PESTO_YU_BIG
+#define PESTO_YU_BIG 16
+#endif
+template <int PL, int kYU = PESTO_YU>
 __global__ void __launch_bounds__(256) transpose_smem_kernel(const TransposeParams P) {
     extern __shared__ uint4 tsm[];
     uint32_t *out_s = reinterpret_cast<uint32_t *>(tsm);
@@ -852,13 +857,17 @@ cudaError_t launch_transpose(const TransposeParams &p, cudaStream_t st) {
         auto set = [&](const void *f) {
             return cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         };
-        cudaError_t e = p.planes == 1 ? set((const void *)transpose_smem_kernel<1>)
+        // two CTAs per SM at most (by shared memory): the deeper gather (more registers)
+        const bool big = 3 * (smem + 1024) > 228 * 1024;
+        cudaError_t e = p.planes == 1 ? (big ? set((const void *)transpose_smem_kernel<1, PESTO_YU_BIG>)
+                                             : set((const void *)transpose_smem_kernel<1>))
                       : p.planes == 2 ? set((const void *)transpose_smem_kernel<2>)
                                       : set((const void *)transpose_smem_kernel<4>);
         if (e != cudaSuccess) return e;
         const int per_sm = std::max(1, (int)(200 * 1024 / std::max<size_t>(smem, 1)));
         const int grid = (int)std::min<int64_t>(p.n_groups, (int64_t)sms * std::min(per_sm, 8));
-        if (p.planes == 1) transpose_smem_kernel<1><<<grid, 256, smem, st>>>(p);
+        if (p.planes == 1 && big) transpose_smem_kernel<1, PESTO_YU_BIG><<<grid, 256, smem, st>>>(p);
+        else if (p.planes == 1) transpose_smem_kernel<1><<<grid, 256, smem, st>>>(p);
         else if (p.planes == 2) transpose_smem_kernel<2><<<grid, 256, smem, st>>>(p);
         else transpose_smem_kernel<4><<<grid, 256, smem, st>>>(p);
         return cudaGetLastError();
