@@ -567,14 +567,18 @@ __device__ __forceinline__ void fast_segment(uint32_t &sp, int32_t &v,
 #endif
 // PESTO_ROWS_V2 selects the explicit-row segment (scripts/gen_fast_walk.py segment_rows):
 // 0 round-2 first version, 1 lane-mask tests, 3 + register read-ahead, 4 + windowed shuffles,
-// 5: 4 for two candidates per lane, 3 for one; 6 (default): the same with the successor-word
-// window switch folded into the step's dispatch (segment_rows fold).  Measured (B200, K1 of 1 M
-// random rows, transformer_2dev, CPL 2): 74.5 (0) -> 69.0 (3) -> 66.4 (4) -> 65.3 ms (fold);
+// 5: 4 for two candidates per lane, 3 for one; 6: the same with the successor-word window
+// switch folded into the step's dispatch (segment_rows fold); 7 (default): both switches folded
+// (foldx).  Measured (B200, K1 of 1 M random rows, transformer_2dev, CPL 2): 74.5 (0) -> 69.0 (3)
+// -> 66.4 (4) -> 65.3 ms (fold); K5 + K1 with the five-CTA instance 65.85 -> 64.99 ms (foldx);
 // inception 65,536 rows (CPL 1): 6.30 (0) -> 5.91 (3) / 6.47 ms (4)
 #ifndef PESTO_ROWS_V2
-#define PESTO_ROWS_V2 6
+#define PESTO_ROWS_V2 7
 #endif
-#if PESTO_ROWS_V2 == 6
+#if PESTO_ROWS_V2 == 7
+#define PESTO_FR1 PESTO_FAST_ROWS_PTX1_V3
+#define PESTO_FR2 PESTO_FAST_ROWS_PTX2_V6
+#elif PESTO_ROWS_V2 == 6
 #define PESTO_FR1 PESTO_FAST_ROWS_PTX1_V3
 #define PESTO_FR2 PESTO_FAST_ROWS_PTX2_V5
 #elif PESTO_ROWS_V2 == 5

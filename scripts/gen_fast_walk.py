@@ -419,8 +419,11 @@ def segment_d4(cpl):
     return P
 
 
-def segment_rows(cpl, pf=0, v2=False, ra=False, win=False, fold=False):
-    """fold (with win): the successor-word window switch rides on the step's dispatch -- the
+def segment_rows(cpl, pf=0, v2=False, ra=False, win=False, fold=False, foldx=False):
+    """foldx (with fold): the op-word window switch rides on the dispatch too -- bit 4 of the
+    edge-0 index = "this op is the last of its 32-op window" (first steps only); entries 16-23
+    switch the op-word window, 48-55 both windows, then continue in the normal handler.
+    fold (with win): the successor-word window switch rides on the step's dispatch -- the
     edge-0 table index carries bit 5 = "this step's slots are in the next window" and those 16
     entries switch the window, redo the step's two shuffles and continue in the normal handler --
     instead of an if-converted block that ptxas executes (predicated) on every step.
@@ -518,7 +521,10 @@ def segment_rows(cpl, pf=0, v2=False, ra=False, win=False, fold=False):
     YA = ("ya0", "ya1")[:cpl]           # slot-0 successor words per candidate group
     YBw = ("yb0", "yb1")[:cpl]          # slot-1
     ta = [f"FA{i}" for i in range(16)]
-    if fold:                            # entries 32-47: window switch, then FA{i}
+    if foldx:                           # 16-23 op-word switch, 32-47 successor-word switch,
+        ta += ([f"FX{i}" for i in range(8)] + ["FDONE"] * 8 +      # 48-55 both
+               [f"FS{i}" for i in range(16)] + [f"FSX{i}" for i in range(8)] + ["FDONE"] * 8)
+    elif fold:                          # entries 32-47: window switch, then FA{i}
         ta += ["FDONE"] * 16 + [f"FS{i}" for i in range(16)]
     tb = [f"FB{i}" for i in range(8)]
     P = ["{",
@@ -593,7 +599,12 @@ def segment_rows(cpl, pf=0, v2=False, ra=False, win=False, fold=False):
           "setp.ne.u32 q, t, 0;",
           "@q bra.uni FCONT;",
           f"add.u32 {V_}, {V_}, 1;"]
-    if win:
+    if foldx:                           # ix < 32: the switch ran at the window's last op
+        P += [f"sub.u32 ix, {V_}, xwb;"]
+        for c in range(cpl):
+            P += [f"shfl.sync.idx.b32 {X_[c]}, {XWC[c]}, ix, 31, -1;"]
+        P += ["add.u32 t, ix, 1;", "shr.u32 t, t, 1;", "and.b32 t, t, 16;", "or.b32 k0, k0, t;"]
+    elif win:
         P += [f"sub.u32 ix, {V_}, xwb;", "setp.ge.u32 p, ix, 32;", "@p bra.uni FXW;", "FXR:"]
         for c in range(cpl):
             P += [f"shfl.sync.idx.b32 {X_[c]}, {XWC[c]}, ix, 31, -1;"]
@@ -657,20 +668,35 @@ def segment_rows(cpl, pf=0, v2=False, ra=False, win=False, fold=False):
         if i < 7:
             P.append("bra.uni FNEXT;")
     P += ["FNEXT:", f"add.u32 {SP_}, {SP_}, 48;", "bra.uni FLOOP;"]
+    def yswitch():
+        out = ["add.u32 ywb, ywb, 32;"]
+        for c in range(cpl):
+            out += [f"mov.u32 {YWC[c]}, {YWN[c]};", f"add.u32 t, ywb, {LANE_};",
+                    "mul.wide.u32 gy, t, 4;", f"add.u64 gy, {YB_[c]}, gy;",
+                    f"ld.global.nc.u32 {YWN[c]}, [gy+128];"]
+        out += ["sub.u32 iy, iy, 32;"]
+        for c in range(cpl):
+            out += [f"shfl.sync.idx.b32 {YA[c]}, {YWC[c]}, iy, 31, -1;"]
+        out += ["add.u32 t, iy, 1;"]
+        for c in range(cpl):
+            out += [f"shfl.sync.idx.b32 {YBw[c]}, {YWC[c]}, t, 31, -1;"]
+        return out
+
+    def xswitch():
+        out = ["add.u32 xwb, xwb, 32;"]
+        for c in range(cpl):
+            out += [f"mov.u32 {XWC[c]}, {XWN[c]};", f"add.u32 t, xwb, {LANE_};",
+                    "mul.wide.u32 gy, t, 4;", f"add.u64 gy, {XB_[c]}, gy;",
+                    f"ld.global.nc.u32 {XWN[c]}, [gy+128];"]
+        return out
+
     if fold:                            # the successor-word window switch (entries 32-47)
         for i in range(16):
-            P += [f"FS{i}:", "add.u32 ywb, ywb, 32;"]
-            for c in range(cpl):
-                P += [f"mov.u32 {YWC[c]}, {YWN[c]};", f"add.u32 t, ywb, {LANE_};",
-                      "mul.wide.u32 gy, t, 4;", f"add.u64 gy, {YB_[c]}, gy;",
-                      f"ld.global.nc.u32 {YWN[c]}, [gy+128];"]
-            P += ["sub.u32 iy, iy, 32;"]
-            for c in range(cpl):
-                P += [f"shfl.sync.idx.b32 {YA[c]}, {YWC[c]}, iy, 31, -1;"]
-            P += ["add.u32 t, iy, 1;"]
-            for c in range(cpl):
-                P += [f"shfl.sync.idx.b32 {YBw[c]}, {YWC[c]}, t, 31, -1;"]
-            P += [f"bra.uni FA{i};"]
+            P += [f"FS{i}:"] + yswitch() + [f"bra.uni FA{i};"]
+    if foldx:                           # the op-word switch (16-23), both (48-55)
+        for i in range(8):
+            P += [f"FX{i}:"] + xswitch() + [f"bra.uni FA{i};"]
+            P += [f"FSX{i}:"] + xswitch() + yswitch() + [f"bra.uni FA{i};"]
     if win and not fold:                # window switches, out of line
         P += ["FYW:", "add.u32 ywb, ywb, 32;"]
         for c in range(cpl):
@@ -678,7 +704,7 @@ def segment_rows(cpl, pf=0, v2=False, ra=False, win=False, fold=False):
                   "mul.wide.u32 gy, t, 4;", f"add.u64 gy, {YB_[c]}, gy;",
                   f"ld.global.nc.u32 {YWN[c]}, [gy+128];"]
         P += [f"sub.u32 ix, {YS_}, ywb;", "bra.uni FYR;"]
-    if win:
+    if win and not foldx:
         P += ["FXW:", "add.u32 xwb, xwb, 32;"]
         for c in range(cpl):
             P += [f"mov.u32 {XWC[c]}, {XWN[c]};", f"add.u32 t, xwb, {LANE_};",
@@ -723,8 +749,9 @@ def main():
                 f.write(f"#define PESTO_FAST_ROWS_PTX{cpl}{suf} \\\n" +
                         " \\\n".join('    "' + l + '\\n"' for l in P) + "\n")
                 print(OUT, f"{cpl}_ROWS{suf}", len(P), "PTX lines")
-            for suf, fold in (("_V4", False), ("_V5", True)):
-                P = segment_rows(cpl, 0, True, False, True, fold)
+            for suf, fold, foldx in (("_V4", False, False), ("_V5", True, False),
+                                     ("_V6", True, True)):
+                P = segment_rows(cpl, 0, True, False, True, fold, foldx)
                 f.write(f"#define PESTO_FAST_ROWS_PTX{cpl}{suf} \\\n" +
                         " \\\n".join('    "' + l + '\\n"' for l in P) + "\n")
                 print(OUT, f"{cpl}_ROWS{suf}", len(P), "PTX lines")
