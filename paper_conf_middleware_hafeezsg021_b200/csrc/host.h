@@ -158,8 +158,9 @@ namespace pesto {
 // graph.cpp helpers used by search.cpp
 pesto_status ensure_comm_tables(pesto_graph *g);
 // x_op (device code per op id, nullable) is embedded in the eval32 records (search bases)
+// tile32: the eval32 tile budget in bytes (0 = automatic: 6 KB at D = 2, else 8 KB)
 pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<Layout> &out,
-                          bool use_cache, const uint8_t *x_op = nullptr);
+                          bool use_cache, const uint8_t *x_op = nullptr, int32_t tile32 = 0);
 pesto_status upload_layout(pesto_graph *g, Layout &L);
 // v4 swap rule (DESIGN.md §4 S3) for the ops a (first) and c (second) of an adjacent pair
 bool pair_blocked(const pesto_graph *g, int32_t a, int32_t c);

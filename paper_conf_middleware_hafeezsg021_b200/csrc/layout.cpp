@@ -97,7 +97,7 @@ void append(std::vector<uint8_t> &buf, const T &v) {
 }  // namespace
 
 pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<Layout> &out,
-                          bool use_cache, const uint8_t *x_op) {
+                          bool use_cache, const uint8_t *x_op, int32_t tile32) {
     pesto_status s = ensure_comm_tables(g);
     if (s) return s;
     const int32_t n = g->n;
@@ -310,8 +310,8 @@ pesto_status build_layout(pesto_graph *g, const int32_t *order, std::shared_ptr<
             return (size_t)(v >= 1024 && v <= 65536 ? (v & ~15L) : 0);
         }();
         const size_t budget = env_budget ? env_budget
-                                         : (g->planes == 1 ? (size_t)kTileTarget32Search
-                                                           : (size_t)kTileTarget);
+                            : tile32 > 0 ? (size_t)tile32
+                            : (g->planes == 1 ? (size_t)kTileTarget32Search : (size_t)kTileTarget);
         open();
         for (int32_t k = 0; k < n; k++) {
             const int32_t u = order[k];

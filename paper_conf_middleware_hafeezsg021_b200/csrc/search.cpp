@@ -61,6 +61,7 @@ struct pesto_search {
     uint64_t seed = 0;
     int32_t rank = 0, world = 1;
     int64_t j_begin = 0, j_end = 0;
+    int32_t tile32 = 0;            // eval32 tile budget of the bases' layouts (0 = automatic)
     int64_t step = 0;
     std::vector<std::vector<int32_t>> order;
     std::vector<std::shared_ptr<Layout>> layouts;
@@ -694,10 +695,19 @@ pesto_status pesto_search_create(pesto_graph *g, const pesto_search_desc *d, pes
     cudaError_t e;
     if ((e = s->d_bits.ensure((size_t)s->P * g->planes * g->words * 4)) != cudaSuccess)
         return cuda_fail(e, "allocate");
+    {
+        // a search whose launches run one candidate per lane (one wave: inception's 64 K) keeps
+        // 8 KB tiles; the 6 KB tiles of D = 2 layouts serve the five-CTA instance of the
+        // two-per-lane launches (inception with 6 KB tiles: 4.10 -> 4.12 ms)
+        EvalParams plan;
+        fill_eval_common(g, plan);
+        plan_eval32(g, plan, s->j_begin, s->j_end, s->P);
+        s->tile32 = plan.cpl32 == 1 ? kTileTarget : 0;
+    }
     for (int b = 0; b < s->P; b++) {
         s->order[b].assign(d->base_order + (size_t)b * n, d->base_order + (size_t)(b + 1) * n);
         pesto_status rc = build_layout(g, s->order[b].data(), s->layouts[b], false,
-                                       d->base_x + (size_t)b * n);
+                                       d->base_x + (size_t)b * n, s->tile32);
         if (rc) return rc;
         if ((rc = upload_layout(g, *s->layouts[b]))) return rc;
         if ((rc = upload_bits(s.get(), b, d->base_x + (size_t)b * n))) return rc;
@@ -846,7 +856,8 @@ pesto_status pesto_search_commit(pesto_search *s, void *stream) {
             std::vector<uint8_t> x_op(g->n);
             pesto_status rc = download_x(s, b, x_op.data());      // K4 already swapped the bits
             if (rc) return rc;
-            if ((rc = build_layout(g, s->order[b].data(), s->layouts[b], false, x_op.data()))) return rc;
+            if ((rc = build_layout(g, s->order[b].data(), s->layouts[b], false, x_op.data(),
+                                   s->tile32))) return rc;
             if ((rc = upload_layout(g, *s->layouts[b]))) return rc;
             changed = true;
         }
