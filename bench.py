@@ -337,7 +337,9 @@ def run_pesto(args, rank, world, local):
     e2e = None
     if not args.no_e2e:
         rows_h = []
-        for r in range(2):                           # two distinct input batches, alternating
+        # two distinct input batches, alternating (one per rank under torchrun: at 8 ranks two
+        # 1 M-row batches each would pin 41 GB of host memory)
+        for r in range(2 if world == 1 else 1):
             rows = dag.random_packed_rows(g, 11 + 2 * rank + r, k_gpu)
             rows_h.append(torch.from_numpy(rows).pin_memory().numpy())
             del rows
@@ -356,13 +358,13 @@ def run_pesto(args, rank, world, local):
                 k = i % nbuf
                 if i >= nbuf:
                     sts[k].synchronize()             # batch i-nbuf is done and its makespans read
-                wss[k].eval_host_async(o, rows_h[i & 1], outs[k], stream=sts[k])
+                wss[k].eval_host_async(o, rows_h[i % len(rows_h)], outs[k], stream=sts[k])
             for st_ in sts:
                 st_.synchronize()
         nw = max(nbuf, args.warmup)
         e2e_run(nw)
         last0 = max(i for i in range(nw) if i % nbuf == 0)   # the batch buffer 0 holds
-        ref0 = G.eval_host(o, rows_h[last0 & 1])     # the synchronous API agrees
+        ref0 = G.eval_host(o, rows_h[last0 % len(rows_h)])   # the synchronous API agrees
         assert (ref0 == outs[0]).all(), "async host-buffer evaluation disagrees"
         if world > 1:
             dist.barrier()
