@@ -512,14 +512,15 @@ __global__ void __launch_bounds__(256) transpose_kernel(const TransposeParams P)
 #define PESTO_T16 4
 #endif
 constexpr int kT16 = PESTO_T16;
-// successor positions per thread in flight in K5's edge-slot gather: 16 where shared memory
-// allows two CTAs per SM anyway (large graphs: 99 registers fit), 8 where three fit (80 registers)
-// -- transformer_2dev, 1 M rows: 6.89 -> 5.68 ms; inception at 16 would drop to two CTAs per SM
+// successor positions per thread in flight in K5's edge-slot gather: 24 where shared memory
+// allows two CTAs per SM anyway (large graphs: 106 registers fit), 8 where three fit (80
+// registers) -- transformer_2dev, 1 M rows: 6.89 (8) -> 5.69 (16) -> 5.50 ms (24); inception at
+// 16 would drop to two CTAs per SM; 8 row chunks per lane in flight instead of 4: 5.93 ms
 #ifndef PESTO_YU
 #define PESTO_YU 8
 #endif
 #ifndef PESTO_YU_BIG
-#define PESTO_YU_BIG 16
+#define PESTO_YU_BIG 24
 #endif
 template <int PL, int kYU = PESTO_YU>
 __global__ void __launch_bounds__(256) transpose_smem_kernel(const TransposeParams P) {
